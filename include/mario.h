@@ -1,0 +1,143 @@
+/* mario.h — C-ABI of libmario.so: a B200-native Mario-scheduled pipeline iteration.
+ *
+ * The library follows the paper's statement of the problem (Listing 1):
+ *   schedule = mario.optimize(mario_conf, model_conf, global_bs);  mario.run(schedule)
+ * as north_star fixes it:  mario_plan(model, stages, microbatches, scheme, mem_budget)
+ * returns per-device instruction lists (IR: Table 3) produced by the four graph
+ * passes (§5.1) and checked by the simulator (§5.2);
+ * mario_run_iter(plan, weights, batch) executes one rank's list and returns loss and grads.
+ *
+ * Conventions
+ *  - Every call returns mario_status (0 = OK, < 0 = error); no C++ exception crosses the
+ *    ABI. mario_last_error() gives a thread-local message valid until the next call.
+ *  - Ownership: plans are owned by the library (opaque, immutable, safe to read from
+ *    several threads) and freed by mario_plan_destroy. Weights, grads, tokens, loss and
+ *    workspace are owned by the caller; the library never frees caller memory.
+ *  - Sizes are in elements unless named *_bytes.
+ */
+#ifndef MARIO_H
+#define MARIO_H
+#include <stddef.h>
+#include <stdint.h>
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  MARIO_OK = 0,
+  MARIO_EINVAL = -1,     /* bad argument, unsupported shape, NULL pointer            */
+  MARIO_EBUDGET = -2,    /* simulated peak memory > mem_budget ("F = 0 if OOM") */
+  MARIO_EDEADLOCK = -3,  /* the instruction graph has a cycle                         */
+  MARIO_ECUDA = -4,      /* CUDA error (sticky: finalize the context)                 */
+  MARIO_ENCCL = -5,      /* NCCL error (sticky)                                       */
+  MARIO_ESTATE = -6      /* wrong call order / plan and context disagree              */
+} mario_status;
+
+typedef enum { MARIO_GPT = 0, MARIO_LLAMA = 1 } mario_family;
+/* Pipeline schemes: "V" 1F1B, "W" Interleave, "X" Chimera. */
+typedef enum { MARIO_1F1B = 0, MARIO_INTERLEAVE = 1, MARIO_CHIMERA = 2 } mario_scheme;
+/* Evaluation configurations: base, ckpt (pass 1 only), ovlp (= passes 1-4). */
+typedef enum { MARIO_LEVEL_BASE = 0, MARIO_LEVEL_CKPT = 1, MARIO_LEVEL_MARIO = 2 } mario_level;
+typedef enum { MARIO_F32 = 0, MARIO_BF16 = 1 } mario_dtype;
+/* Instruction types (Table 3). */
+typedef enum {
+  MARIO_OP_FW = 0, MARIO_OP_CFW = 1, MARIO_OP_RC = 2, MARIO_OP_BW = 3,
+  MARIO_OP_SA = 4, MARIO_OP_RA = 5, MARIO_OP_SG = 6, MARIO_OP_RG = 7
+} mario_op;
+
+/* model_conf (Table 4; details per DESIGN.md readings A1/A2). */
+typedef struct {
+  int32_t family;          /* mario_family                                   */
+  int32_t n_layers, hidden, n_heads, ffn_hidden, vocab, seq_len;
+  int32_t micro_batch;     /* samples per micro-batch (mbs)                  */
+  int32_t tie_embeddings;  /* GPT: LM head tied to wte                       */
+  int32_t dtype;           /* mario_dtype: compute/storage precision         */
+  float norm_eps, rope_base;
+} mario_model;
+
+/* One IR record (micro_id m, part_id p). vstage = virtual stage;
+ * peer = device of the matching SA/RA or SG/RG (-1 otherwise); slot = stage-input
+ * (checkpoint) slot on this device; aslot = activation-set slot (-1 for CFW). */
+typedef struct { int32_t op, micro, part, vstage, peer, slot, aslot; } mario_instr;
+
+/* Optional cost table for the simulator (the paper's profiled estimators).
+ * Arrays are indexed by virtual stage [0, K); NULL arrays fall back to analytic costs
+ * (FLOPs / 1e15 FLOP/s, comm = alpha + bytes / GBps). act/ckpt/work override the
+ * per-virtual-stage dynamic memory model (bytes). */
+typedef struct {
+  const double *fw_ms, *bw_ms, *rc_ms;
+  double p2p_alpha_ms, p2p_GBps;         /* <= 0 GBps: bytes ignored */
+  const double *act_bytes, *ckpt_bytes, *work_bytes;
+  double static_bytes;                   /* < 0: use the analytic static model */
+} mario_costs;
+
+typedef struct {
+  double makespan_ms, bubble_ratio;
+  int32_t n_dev;
+  const double* busy_ms;        /* [n_dev]                          */
+  const uint64_t* peak_bytes;   /* [n_dev] static + peak dynamic    */
+  const int32_t* max_live_act;  /* [n_dev] live activation sets      */
+  const int32_t* max_live_ckpt; /* [n_dev] live stage-input checkpoints */
+} mario_sim;
+
+struct mario_plan;
+
+/* Build a plan: partition (even layers, embedding on virtual stage 0, final norm + head on
+ * the last, reading A8), expand the scheme into per-device lists, apply the passes
+ * for `level`, simulate. chunks = Interleave v (1 otherwise).
+ * Errors: EINVAL (L % (S*v) != 0, h % heads != 0, head_dim not in {16,32,64,80,128},
+ * Interleave with N % S != 0, Chimera with odd S or N % S != 0, NULL out);
+ * EBUDGET if the simulated per-device peak exceeds mem_budget_bytes (0 = no budget). */
+mario_status mario_plan(const mario_model* model, int32_t stages, int32_t microbatches,
+                        int32_t scheme, int32_t chunks, uint64_t mem_budget_bytes, int32_t level,
+                        const mario_costs* costs, struct mario_plan** out);
+/* Borrowed view of device `device`'s ordered list, valid until mario_plan_destroy. */
+mario_status mario_plan_instrs(const struct mario_plan* plan, int32_t device,
+                               const mario_instr** instrs, int32_t* n);
+/* Simulator results (borrowed arrays, valid until destroy). */
+mario_status mario_plan_simulate(const struct mario_plan* plan, mario_sim* out);
+/* Simulated start/finish (ms) of every compute instruction of `device`, in list order of its
+ * compute instructions; arrays of length *n owned by the plan. */
+mario_status mario_plan_timeline(const struct mario_plan* plan, int32_t device,
+                                 const double** start_ms, const double** finish_ms, int32_t* n);
+/* Canonical text serialization (deterministic). If buf is NULL or cap too small, *needed
+ * receives the size including the terminating NUL and MARIO_EINVAL is returned for cap>0. */
+mario_status mario_plan_serialize(const struct mario_plan* plan, char* buf, size_t cap, size_t* needed);
+/* Byte sizes of rank `rank`'s packed fp32 parameters (= grads) and required workspace. */
+mario_status mario_plan_rank_layout(const struct mario_plan* plan, int32_t rank, uint64_t* param_count,
+                                    uint64_t* workspace_bytes);
+/* Packed parameter layout of `rank`: for each tensor j, its global name index (see
+ * mario_param_name), element offset and element count. Arrays owned by the plan. */
+mario_status mario_plan_rank_params(const struct mario_plan* plan, int32_t rank, const int32_t** name_idx,
+                                    const uint64_t** offset, const uint64_t** count, int32_t* n);
+/* Name of the global parameter `idx` (canonical order), e.g. "h3.qkv.w". */
+const char* mario_param_name(const struct mario_plan* plan, int32_t idx);
+int32_t mario_param_count(const struct mario_plan* plan);
+void mario_plan_destroy(struct mario_plan* plan);
+
+/* Executor context. world == 1 with a multi-stage plan runs every rank's list in this
+ * process on one GPU ("loopback": device-to-device copies instead of NCCL). world > 1:
+ * one process per GPU, nccl_unique_id = 128 bytes from mario_nccl_unique_id() on rank 0. */
+mario_status mario_nccl_unique_id(void* out128);
+mario_status mario_init(int32_t rank, int32_t world, int32_t device, const void* nccl_unique_id);
+/* One training iteration of `plan` on this rank (all ranks in loopback).
+ *  weights : device, this rank's packed fp32 parameters (loopback: all ranks concatenated)
+ *  tokens  : HOST int32 [N*mbs][s+1]; x = tokens[:, :s], y = tokens[:, 1:] (reading A4)
+ *  loss    : host, receives the global-batch mean loss (identical on all ranks)
+ *  grads   : device fp32, same layout as weights, OVERWRITTEN (not accumulated) with
+ *            dloss/dtheta; Chimera replicas and tied embeddings are summed (reading A7)
+ *  workspace: device, >= workspace_bytes of mario_plan_rank_layout (loopback: sum)
+ *  stream  : caller's cudaStream_t; the call synchronizes it before returning. */
+mario_status mario_run_iter(const struct mario_plan* plan, const void* weights, const int32_t* tokens,
+                            float* loss, void* grads, void* workspace, void* stream);
+/* Per-instruction measured timeline of the last mario_run_iter on this rank (ms from the
+ * iteration start, CUDA events) when timing was enabled with mario_set_timing(1). */
+mario_status mario_set_timing(int32_t enable);
+mario_status mario_last_timeline(int32_t device, const double** start_ms, const double** finish_ms, int32_t* n);
+mario_status mario_finalize(void);
+const char* mario_last_error(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

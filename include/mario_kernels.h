@@ -1,0 +1,42 @@
+/* mario_kernels.h — kernel-level C-ABI of libmario.so.
+ *
+ * These are the per-layer kernels the executor (mario_run_iter) launches, exported one
+ * call per kernel family so that unit tests and the benchmark's roofline leg can drive
+ * them directly. All pointers are DEVICE pointers owned by the caller; `stream` is a
+ * cudaStream_t (NULL = legacy default stream). Every call is asynchronous and returns a
+ * cudaError_t value (0 = success) for launch/argument errors; no exception crosses the ABI.
+ * Matrices are row-major; ld* are row pitches in ELEMENTS and must be multiples of 8 for
+ * bf16 operands (16-byte TMA pitch), otherwise cudaErrorInvalidValue (1) is returned.
+ */
+#ifndef MARIO_KERNELS_H
+#define MARIO_KERNELS_H
+#include <stddef.h>
+#include <stdint.h>
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+/* K1-K3: D[M,N] = A[M,K] . B[N,K]^T on tcgen05 tensor cores (bf16 in, fp32 accumulate).
+ * The linear layers of SURVEY §8(c) c1 (H = A W^T + b) and their backward passes
+ * (dX = dY W, dW = dY^T X) are the three operand-major combinations:
+ *   a_mn = 0: A stored [M][lda] (K-major);   a_mn = 1: A stored [K][lda] (M-major)
+ *   b_mn = 0: B stored [N][ldb] (K-major);   b_mn = 1: B stored [K][ldb] (N-major)
+ * Epilogue, in order: + bias[N] (fp32, may be NULL); * gelu'(aux[M,N]) if aux != NULL
+ * (GeLU-tanh backward, A1); + residual[M,N] (bf16) if != NULL; then
+ *   out_f32 = 1: D (fp32) = v + beta * D      (wgrad accumulation, beta in {0,1})
+ *   out_f32 = 0: D (bf16) = v, and D2 (bf16, same pitch) = gelu_tanh(v) if D2 != NULL. */
+int mario_k_gemm_bf16(const void* A, int lda, int a_mn, const void* B, int ldb, int b_mn,
+                      int M, int N, int K, void* D, int ldd, int out_f32, float beta,
+                      const float* bias, const void* residual, int ld_res,
+                      void* D2, const void* aux, int ld_aux, void* stream);
+
+/* K4: the same contract in true fp32 on CUDA cores (fp32 mode, reading A6). */
+int mario_k_gemm_f32(const float* A, int lda, int a_mn, const float* B, int ldb, int b_mn,
+                     int M, int N, int K, float* D, int ldd, float beta, const float* bias,
+                     const float* residual, int ld_res, float* D2, const float* aux, int ld_aux,
+                     void* stream);
+
+#ifdef __cplusplus
+}
+#endif
+#endif

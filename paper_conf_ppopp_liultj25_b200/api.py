@@ -1,0 +1,184 @@
+"""Thin Python binding over libmario.so (include/mario.h). Argument marshalling only:
+planning, simulation and every step of the training iteration run inside the library.
+
+    plan = Plan(model, stages=8, microbatches=32, scheme="1f1b", level="mario")
+    ctx  = Context(rank, world, device)            # NCCL / loopback executor
+    loss = ctx.run_iter(plan, weights, tokens, grads, workspace)
+"""
+from __future__ import annotations
+
+import ctypes as C
+from dataclasses import dataclass
+from typing import Dict, List, Optional, Sequence, Tuple
+
+from . import _lib
+
+SCHEMES = {"1f1b": 0, "v": 0, "interleave": 1, "w": 1, "chimera": 2, "x": 2}
+LEVELS = {"base": 0, "ckpt": 1, "mario": 2, "ovlp": 2}
+OPS = ["FW", "CFW", "RC", "BW", "SA", "RA", "SG", "RG"]
+STATUS = {0: "OK", -1: "EINVAL", -2: "EBUDGET", -3: "EDEADLOCK", -4: "ECUDA", -5: "ENCCL", -6: "ESTATE"}
+
+
+class MarioError(RuntimeError):
+    def __init__(self, code, msg):
+        super().__init__(f"{STATUS.get(code, code)}: {msg}")
+        self.code = code
+
+
+class CModel(C.Structure):
+    _fields_ = [("family", C.c_int32), ("n_layers", C.c_int32), ("hidden", C.c_int32), ("n_heads", C.c_int32),
+                ("ffn_hidden", C.c_int32), ("vocab", C.c_int32), ("seq_len", C.c_int32),
+                ("micro_batch", C.c_int32), ("tie_embeddings", C.c_int32), ("dtype", C.c_int32),
+                ("norm_eps", C.c_float), ("rope_base", C.c_float)]
+
+
+class CInstr(C.Structure):
+    _fields_ = [("op", C.c_int32), ("micro", C.c_int32), ("part", C.c_int32), ("vstage", C.c_int32),
+                ("peer", C.c_int32), ("slot", C.c_int32), ("aslot", C.c_int32)]
+
+
+class CCosts(C.Structure):
+    _fields_ = [("fw_ms", C.POINTER(C.c_double)), ("bw_ms", C.POINTER(C.c_double)), ("rc_ms", C.POINTER(C.c_double)),
+                ("p2p_alpha_ms", C.c_double), ("p2p_GBps", C.c_double),
+                ("act_bytes", C.POINTER(C.c_double)), ("ckpt_bytes", C.POINTER(C.c_double)),
+                ("work_bytes", C.POINTER(C.c_double)), ("static_bytes", C.c_double)]
+
+
+class CSim(C.Structure):
+    _fields_ = [("makespan_ms", C.c_double), ("bubble_ratio", C.c_double), ("n_dev", C.c_int32),
+                ("busy_ms", C.POINTER(C.c_double)), ("peak_bytes", C.POINTER(C.c_uint64)),
+                ("max_live_act", C.POINTER(C.c_int32)), ("max_live_ckpt", C.POINTER(C.c_int32))]
+
+
+_P = C.c_void_p
+_lib.register("mario_plan", C.c_int32, [C.POINTER(CModel), C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_uint64,
+                                        C.c_int32, C.POINTER(CCosts), C.POINTER(_P)])
+_lib.register("mario_plan_instrs", C.c_int32, [_P, C.c_int32, C.POINTER(C.POINTER(CInstr)), C.POINTER(C.c_int32)])
+_lib.register("mario_plan_simulate", C.c_int32, [_P, C.POINTER(CSim)])
+_lib.register("mario_plan_timeline", C.c_int32, [_P, C.c_int32, C.POINTER(C.POINTER(C.c_double)),
+                                                 C.POINTER(C.POINTER(C.c_double)), C.POINTER(C.c_int32)])
+_lib.register("mario_plan_serialize", C.c_int32, [_P, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)])
+_lib.register("mario_plan_rank_layout", C.c_int32, [_P, C.c_int32, C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)])
+_lib.register("mario_plan_rank_params", C.c_int32, [_P, C.c_int32, C.POINTER(C.POINTER(C.c_int32)),
+                                                    C.POINTER(C.POINTER(C.c_uint64)),
+                                                    C.POINTER(C.POINTER(C.c_uint64)), C.POINTER(C.c_int32)])
+_lib.register("mario_param_name", C.c_char_p, [_P, C.c_int32])
+_lib.register("mario_param_count", C.c_int32, [_P])
+_lib.register("mario_plan_destroy", None, [_P])
+_lib.register("mario_last_error", C.c_char_p, [])
+_lib.register("mario_nccl_unique_id", C.c_int32, [C.c_void_p])
+_lib.register("mario_init", C.c_int32, [C.c_int32, C.c_int32, C.c_int32, C.c_void_p])
+_lib.register("mario_run_iter", C.c_int32, [_P, C.c_void_p, C.c_void_p, C.POINTER(C.c_float), C.c_void_p,
+                                            C.c_void_p, C.c_void_p])
+_lib.register("mario_set_timing", C.c_int32, [C.c_int32])
+_lib.register("mario_last_timeline", C.c_int32, [C.c_int32, C.POINTER(C.POINTER(C.c_double)),
+                                                 C.POINTER(C.POINTER(C.c_double)), C.POINTER(C.c_int32)])
+_lib.register("mario_finalize", C.c_int32, [])
+
+
+def _check(code):
+    if code != 0:
+        raise MarioError(code, (_lib.lib().mario_last_error() or b"").decode())
+
+
+def cmodel(cfg, dtype: str = "bf16") -> CModel:
+    """synth.ModelCfg (or any object with the same fields) -> mario_model."""
+    return CModel(0 if cfg.family == "gpt" else 1, cfg.n_layers, cfg.hidden, cfg.n_heads, cfg.ffn_hidden,
+                  cfg.vocab, cfg.seq_len, cfg.micro_batch, int(cfg.tie_embeddings),
+                  1 if dtype == "bf16" else 0, cfg.norm_eps, cfg.rope_base)
+
+
+def _darr(xs):
+    if xs is None:
+        return None
+    return (C.c_double * len(xs))(*xs)
+
+
+@dataclass
+class SimReport:
+    makespan_ms: float
+    bubble_ratio: float
+    busy_ms: List[float]
+    peak_bytes: List[int]
+    max_live_act: List[int]
+    max_live_ckpt: List[int]
+
+
+class Plan:
+    """mario_plan(model, stages, microbatches, scheme, mem_budget) (north_star)."""
+
+    def __init__(self, cfg, stages: int, microbatches: int, scheme: str = "1f1b", level: str = "mario",
+                 chunks: int = 1, mem_budget: int = 0, dtype: str = "bf16", costs: Optional[dict] = None):
+        L = _lib.lib()
+        self.cfg, self.dtype = cfg, dtype
+        self.S, self.N, self.scheme, self.level, self.chunks = stages, microbatches, scheme, level, chunks
+        self._m = cmodel(cfg, dtype)
+        cc = None
+        if costs is not None:
+            self._keep = [_darr(costs.get(k)) for k in ("fw_ms", "bw_ms", "rc_ms", "act_bytes", "ckpt_bytes",
+                                                        "work_bytes")]
+            cc = CCosts(self._keep[0], self._keep[1], self._keep[2], costs.get("p2p_alpha_ms", 0.0),
+                        costs.get("p2p_GBps", 0.0), self._keep[3], self._keep[4], self._keep[5],
+                        costs.get("static_bytes", -1.0))
+        h = _P()
+        _check(L.mario_plan(C.byref(self._m), stages, microbatches, SCHEMES[scheme], chunks, mem_budget,
+                            LEVELS[level], C.byref(cc) if cc is not None else None, C.byref(h)))
+        self.handle = h
+
+    def __del__(self):
+        h = getattr(self, "handle", None)
+        if h and _lib._lib is not None:
+            _lib.lib().mario_plan_destroy(h)
+            self.handle = None
+
+    @property
+    def _as_param(self):
+        return self.handle
+
+    def instrs(self, d: int) -> List[Tuple]:
+        p = C.POINTER(CInstr)()
+        n = C.c_int32()
+        _check(_lib.lib().mario_plan_instrs(self.handle, d, C.byref(p), C.byref(n)))
+        return [(OPS[p[i].op], p[i].micro, p[i].part, p[i].vstage, p[i].peer, p[i].slot, p[i].aslot)
+                for i in range(n.value)]
+
+    def lists(self) -> List[List[Tuple[str, int, int]]]:
+        return [[(op, m, p) for (op, m, p, *_r) in self.instrs(d)] for d in range(self.S)]
+
+    def simulate(self) -> SimReport:
+        s = CSim()
+        _check(_lib.lib().mario_plan_simulate(self.handle, C.byref(s)))
+        n = s.n_dev
+        return SimReport(s.makespan_ms, s.bubble_ratio, [s.busy_ms[i] for i in range(n)],
+                         [s.peak_bytes[i] for i in range(n)], [s.max_live_act[i] for i in range(n)],
+                         [s.max_live_ckpt[i] for i in range(n)])
+
+    def timeline(self, d: int):
+        a, b, n = C.POINTER(C.c_double)(), C.POINTER(C.c_double)(), C.c_int32()
+        _check(_lib.lib().mario_plan_timeline(self.handle, d, C.byref(a), C.byref(b), C.byref(n)))
+        return [a[i] for i in range(n.value)], [b[i] for i in range(n.value)]
+
+    def serialize(self) -> str:
+        need = C.c_size_t()
+        _check(_lib.lib().mario_plan_serialize(self.handle, None, 0, C.byref(need)))
+        buf = C.create_string_buffer(need.value)
+        _check(_lib.lib().mario_plan_serialize(self.handle, buf, need.value, C.byref(need)))
+        return buf.value.decode()
+
+    def rank_layout(self, rank: int) -> Tuple[int, int]:
+        """(packed parameter count, workspace bytes); rank=-1: loopback totals."""
+        pc, ws = C.c_uint64(), C.c_uint64()
+        _check(_lib.lib().mario_plan_rank_layout(self.handle, rank, C.byref(pc), C.byref(ws)))
+        return pc.value, ws.value
+
+    def param_names(self) -> List[str]:
+        L = _lib.lib()
+        return [L.mario_param_name(self.handle, i).decode() for i in range(L.mario_param_count(self.handle))]
+
+    def rank_params(self, rank: int) -> List[Tuple[str, int, int]]:
+        """[(name, element offset, element count)] of rank's packed buffer, in order."""
+        idx, off, cnt, n = C.POINTER(C.c_int32)(), C.POINTER(C.c_uint64)(), C.POINTER(C.c_uint64)(), C.c_int32()
+        _check(_lib.lib().mario_plan_rank_params(self.handle, rank, C.byref(idx), C.byref(off), C.byref(cnt),
+                                                 C.byref(n)))
+        names = self.param_names()
+        return [(names[idx[i]], off[i], cnt[i]) for i in range(n.value)]

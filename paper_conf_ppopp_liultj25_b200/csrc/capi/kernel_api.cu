@@ -1,0 +1,35 @@
+// C-ABI kernel-level entry points (include/mario_kernels.h): one call per kernel family,
+// device pointers in, used by the GPU unit tests and the benchmark's per-kernel roofline.
+#include <cuda_runtime.h>
+#include "../kernels/kernels.h"
+#include "../../../include/mario_kernels.h"
+
+using namespace mario;
+
+extern "C" int mario_k_gemm_bf16(const void* A, int lda, int a_mn, const void* B, int ldb, int b_mn,
+                                 int M, int N, int K, void* D, int ldd, int out_f32, float beta,
+                                 const float* bias, const void* residual, int ld_res,
+                                 void* D2, const void* aux, int ld_aux, void* stream) {
+  GemmArgs g;
+  g.A = static_cast<const __nv_bfloat16*>(A); g.lda = lda; g.a_mn = a_mn;
+  g.B = static_cast<const __nv_bfloat16*>(B); g.ldb = ldb; g.b_mn = b_mn;
+  g.M = M; g.N = N; g.K = K;
+  g.ep.out_f32 = out_f32;
+  if (out_f32) g.ep.d_f32 = static_cast<float*>(D); else g.ep.d_bf16 = static_cast<__nv_bfloat16*>(D);
+  g.ep.ldd = ldd; g.ep.beta = beta; g.ep.bias = bias;
+  g.ep.residual = static_cast<const __nv_bfloat16*>(residual); g.ep.ld_res = ld_res;
+  g.ep.d2_bf16 = static_cast<__nv_bfloat16*>(D2);
+  g.ep.aux = static_cast<const __nv_bfloat16*>(aux); g.ep.ld_aux = ld_aux;
+  return static_cast<int>(gemm_bf16(g, static_cast<cudaStream_t>(stream)));
+}
+
+extern "C" int mario_k_gemm_f32(const float* A, int lda, int a_mn, const float* B, int ldb, int b_mn,
+                                int M, int N, int K, float* D, int ldd, float beta, const float* bias,
+                                const float* residual, int ld_res, float* D2, const float* aux, int ld_aux,
+                                void* stream) {
+  GemmF32Args g;
+  g.A = A; g.lda = lda; g.a_mn = a_mn; g.B = B; g.ldb = ldb; g.b_mn = b_mn;
+  g.M = M; g.N = N; g.K = K; g.D = D; g.ldd = ldd; g.beta = beta; g.bias = bias;
+  g.residual = residual; g.ld_res = ld_res; g.D2 = D2; g.aux = aux; g.ld_aux = ld_aux;
+  return static_cast<int>(gemm_f32(g, static_cast<cudaStream_t>(stream)));
+}

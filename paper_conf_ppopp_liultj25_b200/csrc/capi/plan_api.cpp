@@ -1,0 +1,349 @@
+// C-ABI of the planner (include/mario.h): mario_plan and its inspectors.
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <set>
+#include <stdexcept>
+#include <string>
+
+#include "../exec/arena.h"
+#include "../plan/plan_obj.h"
+#include "status.h"
+
+using namespace mario;
+using namespace mario::plan;
+
+namespace {
+
+const char* scheme_name(int s) { return s == MARIO_1F1B ? "1f1b" : s == MARIO_INTERLEAVE ? "interleave" : "chimera"; }
+const char* level_name(int l) { return l == MARIO_LEVEL_BASE ? "base" : l == MARIO_LEVEL_CKPT ? "ckpt" : "mario"; }
+
+// Round-robin walk (the simulator's order, ignoring time): a receive is walked only after its
+// matching send. Used by the loopback executor; returns false on a cycle.
+bool walk_order(const Pipe& pp, const Lists& L, std::vector<std::pair<int, int>>& order) {
+  std::set<std::tuple<int, int, int, int>> posted;
+  std::vector<size_t> ptr(pp.S, 0);
+  size_t total = 0, done = 0;
+  for (auto& l : L) total += l.size();
+  while (done < total) {
+    bool prog = false;
+    for (int d = 0; d < pp.S; ++d) {
+      while (ptr[d] < L[d].size()) {
+        const Instr& x = L[d][ptr[d]];
+        if (is_send(x.op)) posted.insert({d, x.op, x.m, x.p});
+        if (is_recv(x.op)) {
+          int sd, sp;
+          find_inst(pp, d, x.m, x.p, x.op == RA ? FW : BW, false, &sd, &sp);
+          if (!posted.count({sd, x.op == RA ? SA : SG, x.m, sp})) break;
+        }
+        order.push_back({d, static_cast<int>(ptr[d])});
+        ++ptr[d]; ++done; prog = true;
+      }
+    }
+    if (!prog) return false;
+  }
+  return true;
+}
+
+struct SlotPool {
+  std::vector<bool> used;
+  int high = 0;
+  int acquire() {
+    for (size_t i = 0; i < used.size(); ++i) if (!used[i]) { used[i] = true; return static_cast<int>(i); }
+    used.push_back(true);
+    high = static_cast<int>(used.size());
+    return high - 1;
+  }
+  void release(int i) { if (i >= 0) used[i] = false; }
+};
+
+void assign_slots_and_pools(PlanObj& P) {
+  const Pipe& pp = P.pp;
+  const int K = pp.K();
+  P.instrs.assign(pp.S, {});
+  P.pools_mp.assign(pp.S, {});
+  for (int d = 0; d < pp.S; ++d) {
+    SlotPool ck, ac, sa, sg, rg;
+    std::map<std::pair<int, int>, int> ck_of, ac_of, sa_of, sg_of, rg_of;
+    for (const Instr& x : P.lists[d]) {
+      const int k = pp.vstage(d, x.p);
+      const auto key = std::make_pair(x.m, x.p);
+      mario_instr r{x.op, x.m, x.p, k, -1, -1, -1};
+      int sd, sp;
+      switch (x.op) {
+        case RA: ck_of[key] = ck.acquire(); find_inst(pp, d, x.m, x.p, FW, false, &sd, &sp); r.peer = sd; break;
+        case RG: rg_of[key] = rg.acquire(); find_inst(pp, d, x.m, x.p, BW, false, &sd, &sp); r.peer = sd; break;
+        case SA: find_inst(pp, d, x.m, x.p, FW, true, &sd, &sp); r.peer = sd; sa.release(sa_of[key]); break;
+        case SG: find_inst(pp, d, x.m, x.p, BW, true, &sd, &sp); r.peer = sd; sg.release(sg_of[key]); break;
+        case FW: ac_of[key] = ac.acquire(); if (k < K - 1) sa_of[key] = sa.acquire(); break;
+        case CFW: if (k < K - 1) sa_of[key] = sa.acquire(); break;
+        case RC: ac_of[key] = ac.acquire(); break;
+        case BW:
+          if (k > 0) sg_of[key] = sg.acquire();
+          break;
+      }
+      if (ck_of.count(key)) r.slot = ck_of[key];
+      if (ac_of.count(key) && (x.op == FW || x.op == RC || x.op == BW)) r.aslot = ac_of[key];
+      if (x.op == BW) {
+        if (ck_of.count(key)) { ck.release(ck_of[key]); ck_of.erase(key); }
+        ac.release(ac_of[key]); ac_of.erase(key);
+        if (rg_of.count(key)) { rg.release(rg_of[key]); rg_of.erase(key); }
+      }
+      P.instrs[d].push_back(r);
+    }
+    P.pools_mp[d] = {ck.high, ac.high, sa.high, sg.high, rg.high};
+  }
+  // loopback: send slots are held until the receiver copies them out
+  P.pools_lb = P.pools_mp;
+  std::vector<SlotPool> lsa(pp.S), lsg(pp.S);
+  std::map<std::tuple<int, int, int>, int> held_sa, held_sg;  // (sender dev, m, p) -> slot
+  for (auto [d, i] : P.loopback_order) {
+    const Instr& x = P.lists[d][i];
+    const int k = pp.vstage(d, x.p);
+    int sd, sp;
+    if ((x.op == FW || x.op == CFW) && k < K - 1) held_sa[{d, x.m, x.p}] = lsa[d].acquire();
+    if (x.op == BW && k > 0) held_sg[{d, x.m, x.p}] = lsg[d].acquire();
+    if (x.op == RA) {
+      find_inst(pp, d, x.m, x.p, FW, false, &sd, &sp);
+      lsa[sd].release(held_sa[{sd, x.m, sp}]);
+    }
+    if (x.op == RG) {
+      find_inst(pp, d, x.m, x.p, BW, false, &sd, &sp);
+      lsg[sd].release(held_sg[{sd, x.m, sp}]);
+    }
+  }
+  for (int d = 0; d < pp.S; ++d) {
+    P.pools_lb[d].send_act = lsa[d].high;
+    P.pools_lb[d].send_grad = lsg[d].high;
+  }
+}
+
+void build_rank_params(PlanObj& P) {
+  P.params = model_params(P.model);
+  for (auto& ps : P.params) P.param_names.push_back(ps.name);
+  const int K = P.pp.K();
+  P.rank_params.assign(P.pp.S, {});
+  for (int d = 0; d < P.pp.S; ++d) {
+    auto& rp = P.rank_params[d];
+    for (int p = 0; p < P.pp.parts(); ++p) {
+      for (int32_t i : stage_param_indices(P.model, P.pp.vstage(d, p), K)) {
+        rp.idx.push_back(i);
+        rp.part.push_back(p);
+        rp.off.push_back(rp.total);
+        uint64_t n = static_cast<uint64_t>(P.params[i].numel());
+        rp.cnt.push_back(n);
+        rp.total += (n + 63) / 64 * 64;   // 256-byte aligned tensors
+      }
+    }
+  }
+}
+
+void fill_costs(PlanObj& P, const mario_costs* c) {
+  const int K = P.pp.K();
+  SimCosts& s = P.costs;
+  s.fw.resize(K); s.bw.resize(K); s.rc.resize(K); s.act.resize(K); s.ckpt.resize(K); s.work.resize(K);
+  for (int k = 0; k < K; ++k) {
+    const double fl = stage_fwd_flops(P.model, k, K);
+    s.fw[k] = (c && c->fw_ms) ? c->fw_ms[k] : fl / 1e12;   // analytic: 1 PFLOP/s effective
+    s.bw[k] = (c && c->bw_ms) ? c->bw_ms[k] : 2.0 * fl / 1e12;
+    s.rc[k] = (c && c->rc_ms) ? c->rc_ms[k] : s.fw[k];
+    s.act[k] = (c && c->act_bytes) ? c->act_bytes[k] : static_cast<double>(act_set_bytes(P.model, k, K));
+    s.ckpt[k] = (c && c->ckpt_bytes) ? c->ckpt_bytes[k] : (k == 0 ? 0.0 : static_cast<double>(stage_input_bytes(P.model)));
+    s.work[k] = (c && c->work_bytes) ? c->work_bytes[k] : static_cast<double>(cfw_work_bytes(P.model, k, K));
+  }
+  const double msg = static_cast<double>(tokens_per_micro(P.model)) * P.model.hidden * elt_size(P.model);
+  double alpha = 0.01, gbps = 700.0;
+  if (c) { alpha = c->p2p_alpha_ms; gbps = c->p2p_GBps; }
+  s.comm_act = s.comm_grad = alpha + (gbps > 0 ? msg / (gbps * 1e6) : 0.0);
+}
+
+void fill_static(PlanObj& P, const mario_costs* c) {
+  P.costs.static_bytes.assign(P.pp.S, 0.0);
+  for (int d = 0; d < P.pp.S; ++d) {
+    if (c && c->static_bytes >= 0) { P.costs.static_bytes[d] = c->static_bytes; continue; }
+    // caller buffers (fp32 weights + grads) + fixed arena part (everything but slots)
+    PlanObj::Pools none{0, 0, P.pools_mp.empty() ? 1 : P.pools_mp[d].send_act,
+                           P.pools_mp.empty() ? 1 : P.pools_mp[d].send_grad,
+                           P.pools_mp.empty() ? 1 : P.pools_mp[d].recv_grad};
+    Arena a = make_arena(P, d, none);
+    P.costs.static_bytes[d] = static_cast<double>(P.rank_params[d].total) * 8.0 +
+                              static_cast<double>(a.total - a.ckpt_stride - a.act_stride);
+  }
+}
+
+std::string serialize(const PlanObj& P) {
+  std::string s;
+  char buf[512];
+  const mario_model& m = P.model;
+  snprintf(buf, sizeof buf, "mario-plan v1\nmodel family=%s L=%d h=%d heads=%d f=%d V=%d s=%d mbs=%d tie=%d dtype=%s\n",
+           m.family == MARIO_GPT ? "gpt" : "llama", m.n_layers, m.hidden, m.n_heads, m.ffn_hidden, m.vocab,
+           m.seq_len, m.micro_batch, m.tie_embeddings, m.dtype == MARIO_BF16 ? "bf16" : "f32");
+  s += buf;
+  snprintf(buf, sizeof buf, "pipe scheme=%s S=%d N=%d v=%d level=%s\n", scheme_name(P.pp.scheme), P.pp.S, P.pp.N,
+           P.pp.v, level_name(P.level));
+  s += buf;
+  for (int d = 0; d < P.pp.S; ++d) {
+    snprintf(buf, sizeof buf, "dev %d:", d);
+    s += buf;
+    for (const Instr& x : P.lists[d]) {
+      snprintf(buf, sizeof buf, " %s%d.%d", op_name(x.op), x.m, x.p);
+      s += buf;
+    }
+    s += "\n";
+  }
+  return s;
+}
+
+}  // namespace
+
+extern "C" mario_status mario_plan(const mario_model* model, int32_t stages, int32_t microbatches, int32_t scheme,
+                                   int32_t chunks, uint64_t mem_budget_bytes, int32_t level,
+                                   const mario_costs* costs, struct mario_plan** out) {
+  return guard([&]() -> mario_status {
+    if (!model || !out) return set_error(MARIO_EINVAL, "NULL model or out");
+    *out = nullptr;
+    if (const char* e = validate_model(*model)) return set_error(MARIO_EINVAL, e);
+    if (stages < 1 || microbatches < 1) return set_error(MARIO_EINVAL, "stages and microbatches must be >= 1");
+    if (scheme < 0 || scheme > 2) return set_error(MARIO_EINVAL, "unknown scheme");
+    if (level < 0 || level > 2) return set_error(MARIO_EINVAL, "unknown level");
+    if (scheme != MARIO_INTERLEAVE) chunks = 1;
+    if (chunks < 1) return set_error(MARIO_EINVAL, "chunks must be >= 1");
+    Pipe pp{scheme, stages, microbatches, chunks};
+    if (model->n_layers % pp.K()) return set_error(MARIO_EINVAL, "n_layers % (stages*chunks) != 0");
+    if (scheme == MARIO_INTERLEAVE && (microbatches % stages || stages < 2))
+      return set_error(MARIO_EINVAL, "Interleave needs stages >= 2 and microbatches % stages == 0");
+    if (scheme == MARIO_CHIMERA && (stages % 2 || microbatches % stages))
+      return set_error(MARIO_EINVAL, "Chimera needs even stages and microbatches % stages == 0");
+    auto P = std::make_unique<PlanObj>();
+    P->model = *model;
+    P->pp = pp;
+    P->level = level;
+    P->budget = mem_budget_bytes;
+    P->lps = model->n_layers / pp.K();
+    build_rank_params(*P);
+    fill_costs(*P, costs);
+    Lists L = build_base(pp);
+    if (level != MARIO_LEVEL_BASE) {
+      L = pass1_apply_checkpoint(L);
+      if (level == MARIO_LEVEL_MARIO) {
+        L = pass2_overlap_recompute(L);
+        L = pass3_remove_redundancy(L);
+      }
+    }
+    P->lists = L;
+    if (!walk_order(pp, P->lists, P->loopback_order)) return set_error(MARIO_EDEADLOCK, "base lists deadlock");
+    assign_slots_and_pools(*P);
+    fill_static(*P, costs);
+    if (level == MARIO_LEVEL_MARIO) {
+      P->lists = pass4_prepose_forward(pp, P->lists, P->costs, static_cast<double>(mem_budget_bytes));
+      P->loopback_order.clear();
+      if (!walk_order(pp, P->lists, P->loopback_order)) return set_error(MARIO_EDEADLOCK, "plan deadlocks");
+      assign_slots_and_pools(*P);
+      fill_static(*P, costs);
+    }
+    P->sim = simulate(pp, P->lists, P->costs);
+    if (!P->sim.ok) return set_error(MARIO_EDEADLOCK, "simulator found a dependency cycle");
+    P->mem = memory_walk(pp, P->lists, P->costs);
+    for (int d = 0; d < pp.S; ++d) {
+      P->busy.push_back(P->sim.busy[d]);
+      P->peak.push_back(static_cast<uint64_t>(P->mem.peak[d]));
+      P->live_act.push_back(P->mem.max_live_act[d]);
+      P->live_ckpt.push_back(P->mem.max_live_ckpt[d]);
+      P->workspace_mp.push_back(make_arena(*P, d, P->pools_mp[d]).total);
+      P->workspace_lb.push_back(make_arena(*P, d, P->pools_lb[d]).total);
+    }
+    P->serialized = serialize(*P);
+    if (mem_budget_bytes > 0) {
+      uint64_t worst = *std::max_element(P->peak.begin(), P->peak.end());
+      if (worst > mem_budget_bytes) {
+        char b[160];
+        snprintf(b, sizeof b, "simulated peak %llu bytes > budget %llu", (unsigned long long)worst,
+                 (unsigned long long)mem_budget_bytes);
+        return set_error(MARIO_EBUDGET, b);
+      }
+    }
+    *out = P.release();
+    return MARIO_OK;
+  });
+}
+
+extern "C" mario_status mario_plan_instrs(const struct mario_plan* P, int32_t device, const mario_instr** instrs,
+                                          int32_t* n) {
+  if (!P || !instrs || !n || device < 0 || device >= P->pp.S) return set_error(MARIO_EINVAL, "bad argument");
+  *instrs = P->instrs[device].data();
+  *n = static_cast<int32_t>(P->instrs[device].size());
+  return MARIO_OK;
+}
+
+extern "C" mario_status mario_plan_simulate(const struct mario_plan* P, mario_sim* out) {
+  if (!P || !out) return set_error(MARIO_EINVAL, "bad argument");
+  out->makespan_ms = P->sim.makespan;
+  double busy = 0;
+  for (double b : P->busy) busy += b;
+  out->bubble_ratio = P->sim.makespan > 0 ? 1.0 - busy / (P->pp.S * P->sim.makespan) : 0.0;
+  out->n_dev = P->pp.S;
+  out->busy_ms = P->busy.data();
+  out->peak_bytes = P->peak.data();
+  out->max_live_act = P->live_act.data();
+  out->max_live_ckpt = P->live_ckpt.data();
+  return MARIO_OK;
+}
+
+extern "C" mario_status mario_plan_timeline(const struct mario_plan* P, int32_t device, const double** start,
+                                            const double** finish, int32_t* n) {
+  if (!P || device < 0 || device >= P->pp.S || !start || !finish || !n) return set_error(MARIO_EINVAL, "bad argument");
+  *start = P->sim.start[device].data();
+  *finish = P->sim.finish[device].data();
+  *n = static_cast<int32_t>(P->sim.start[device].size());
+  return MARIO_OK;
+}
+
+extern "C" mario_status mario_plan_serialize(const struct mario_plan* P, char* buf, size_t cap, size_t* needed) {
+  if (!P) return set_error(MARIO_EINVAL, "NULL plan");
+  const size_t need = P->serialized.size() + 1;
+  if (needed) *needed = need;
+  if (!buf || cap == 0) return MARIO_OK;
+  if (cap < need) return set_error(MARIO_EINVAL, "buffer too small");
+  memcpy(buf, P->serialized.c_str(), need);
+  return MARIO_OK;
+}
+
+extern "C" mario_status mario_plan_rank_layout(const struct mario_plan* P, int32_t rank, uint64_t* param_count,
+                                               uint64_t* workspace_bytes) {
+  if (!P) return set_error(MARIO_EINVAL, "NULL plan");
+  if (rank == -1) {  // loopback: all ranks concatenated
+    uint64_t pc = 0, ws = 0;
+    for (int d = 0; d < P->pp.S; ++d) { pc += P->rank_params[d].total; ws += align_up(P->workspace_lb[d], 1 << 20); }
+    if (param_count) *param_count = pc;
+    if (workspace_bytes) *workspace_bytes = ws;
+    return MARIO_OK;
+  }
+  if (rank < 0 || rank >= P->pp.S) return set_error(MARIO_EINVAL, "bad rank");
+  if (param_count) *param_count = P->rank_params[rank].total;
+  if (workspace_bytes) *workspace_bytes = P->workspace_mp[rank];
+  return MARIO_OK;
+}
+
+extern "C" mario_status mario_plan_rank_params(const struct mario_plan* P, int32_t rank, const int32_t** name_idx,
+                                               const uint64_t** offset, const uint64_t** count, int32_t* n) {
+  if (!P || rank < 0 || rank >= P->pp.S || !name_idx || !offset || !count || !n)
+    return set_error(MARIO_EINVAL, "bad argument");
+  const auto& rp = P->rank_params[rank];
+  *name_idx = rp.idx.data();
+  *offset = rp.off.data();
+  *count = rp.cnt.data();
+  *n = static_cast<int32_t>(rp.idx.size());
+  return MARIO_OK;
+}
+
+extern "C" const char* mario_param_name(const struct mario_plan* P, int32_t idx) {
+  if (!P || idx < 0 || idx >= static_cast<int32_t>(P->param_names.size())) return nullptr;
+  return P->param_names[idx].c_str();
+}
+
+extern "C" int32_t mario_param_count(const struct mario_plan* P) {
+  return P ? static_cast<int32_t>(P->param_names.size()) : 0;
+}
+
+extern "C" void mario_plan_destroy(struct mario_plan* P) { delete P; }

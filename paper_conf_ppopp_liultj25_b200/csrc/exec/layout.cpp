@@ -1,0 +1,89 @@
+#include "layout.h"
+
+#include <algorithm>
+
+#include "../plan/model.h"
+
+namespace mario {
+
+size_t elt_size(const mario_model& m) { return m.dtype == MARIO_BF16 ? 2 : 4; }
+size_t tokens_per_micro(const mario_model& m) { return static_cast<size_t>(m.micro_batch) * m.seq_len; }
+
+LayerAct layer_act_layout(const mario_model& m) {
+  const size_t T = tokens_per_micro(m), E = elt_size(m), h = m.hidden, f = m.ffn_hidden;
+  const size_t nh = m.n_heads;
+  LayerAct L{};
+  size_t o = 0;
+  auto take = [&](size_t bytes) { size_t r = o; o = align_up(o + bytes); return r; };
+  L.H_in = take(T * h * E);
+  L.st1 = take(T * 2 * 4);          // mean, rstd (fp32)
+  L.A = take(T * h * E);
+  L.QKV = take(T * 3 * h * E);
+  L.O = take(T * h * E);
+  L.LSE = take(nh * T * 4);
+  L.H1 = take(T * h * E);
+  L.st2 = take(T * 2 * 4);
+  L.A2 = take(T * h * E);
+  if (m.family == MARIO_GPT) {
+    L.Z = take(T * f * E);
+    L.G = take(T * f * E);
+  } else {
+    L.Z = take(T * 2 * f * E);     // GU = [gate | up]
+    L.G = take(T * f * E);         // M = silu(gate) * up
+  }
+  L.bytes = o;
+  return L;
+}
+
+HeadAct head_act_layout(const mario_model& m) {
+  const size_t T = tokens_per_micro(m), E = elt_size(m), h = m.hidden, V = m.vocab;
+  HeadAct H{};
+  size_t o = 0;
+  auto take = [&](size_t bytes) { size_t r = o; o = align_up(o + bytes); return r; };
+  H.H_last = take(T * h * E);
+  H.stf = take(T * 2 * 4);
+  H.Hf = take(T * h * E);
+  H.dlogits = take(T * V * E);
+  H.bytes = o;
+  return H;
+}
+
+size_t stage_input_bytes(const mario_model& m) { return align_up(tokens_per_micro(m) * m.hidden * elt_size(m)); }
+
+size_t act_set_bytes(const mario_model& m, int k, int K) {
+  const int lps = m.n_layers / K;
+  size_t b = layer_act_layout(m).bytes * lps;
+  if (k == K - 1) b += head_act_layout(m).bytes;
+  return b;
+}
+
+size_t cfw_work_bytes(const mario_model& m, int k, int K) {
+  // one layer's temporaries + the two running residual buffers (+ head temporaries)
+  size_t b = layer_act_layout(m).bytes + 2 * stage_input_bytes(m);
+  if (k == K - 1) b += head_act_layout(m).bytes;
+  return b;
+}
+
+size_t bw_scratch_bytes(const mario_model& m) {
+  const size_t T = tokens_per_micro(m), E = elt_size(m), h = m.hidden, f = m.ffn_hidden;
+  // dH ping-pong (2 x [T,h]) + dX [T,h] + dQKV [T,3h] + dO [T,h] + dZ [T, 2f] + dP row sums fp32 [heads,T]
+  size_t b = 0;
+  b += align_up(T * h * E) * 3;
+  b += align_up(T * 3 * h * E);
+  b += align_up(T * h * E);
+  b += align_up(T * 2 * f * E);
+  b += align_up(static_cast<size_t>(m.n_heads) * T * 4);
+  return b;
+}
+
+size_t logits_bytes(const mario_model& m) { return align_up(tokens_per_micro(m) * m.vocab * 4); }
+
+size_t weight_copy_bytes(const mario_model& m, const std::vector<int32_t>& idx) {
+  if (m.dtype != MARIO_BF16) return 0;
+  auto ps = model_params(m);
+  size_t b = 0;
+  for (int32_t i : idx) if (ps[i].is_matrix()) b += align_up(ps[i].numel() * 2);
+  return b;
+}
+
+}  // namespace mario

@@ -1,0 +1,327 @@
+// K1-K3: bf16 GEMM on the 5th-gen tensor cores for sm_100a.
+//
+//   D[M,N] = A[M,K] . B[N,K]^T   (fp32 accumulate in TMEM) + fused epilogue
+//
+// A and B are each either K-major (row-major [rows][K]) or MN-major (row-major [K][rows]),
+// which covers the three products of a linear layer without any transpose copies:
+//   forward  Y  = X  W^T : A = X  (K-major), B = W  (K-major)
+//   dgrad    dX = dY W   : A = dY (K-major), B = W  (N-major: stored [out][in] = [K][N])
+//   wgrad    dW = dY^T X : A = dY (M-major), B = X  (N-major), reduction over tokens,
+//                          deterministic (no split-K), beta = 1 read-modify-write into fp32
+//
+// Design (warp-specialised, persistent, one CTA per SM):
+//   warp 0      : TMA producer — cp.async.bulk.tensor tiles (128B swizzle) into a
+//                 kStages-deep smem ring guarded by full/empty mbarriers
+//   warp 1      : TMEM allocator + single-thread tcgen05.mma issuer (M=128, N=BN, K=16)
+//   warps 2..5  : epilogue — tcgen05.ld accumulator rows -> registers -> fused
+//                 bias / GeLU / GeLU' / residual / fp32-accumulate -> global
+//   TMEM holds two BN-column accumulators so the epilogue of tile i overlaps the MMAs
+//   of tile i+1.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+#include <cuda_runtime.h>
+#include <cuda_bf16.h>
+#include <cstdio>
+#include <mutex>
+
+#include "sm100.cuh"
+#include "kernels.h"
+
+namespace mario {
+
+using namespace sm100;
+
+namespace {
+
+constexpr int BM = 128;
+constexpr int BK = 64;            // 64 bf16 = 128 B = one swizzle atom row
+constexpr int kThreads = 192;     // 6 warps
+
+template <int BN>
+struct Cfg {
+  static constexpr int kStages = BN == 256 ? 4 : 6;
+  static constexpr int kABytes = BM * BK * 2;
+  static constexpr int kBBytes = BN * BK * 2;
+  static constexpr int kStageBytes = kABytes + kBBytes;
+  static constexpr int kTmemCols = 2 * BN;     // double-buffered accumulator
+  static constexpr int kSmem = kStages * kStageBytes + 1024 /*align*/ + 256 /*barriers*/;
+};
+
+__device__ __forceinline__ float gelu_tanh_f(float z) {
+  const float c = 0.7978845608028654f;
+  float t = tanhf(c * (z + 0.044715f * z * z * z));
+  return 0.5f * z * (1.f + t);
+}
+__device__ __forceinline__ float gelu_tanh_grad_f(float z) {
+  const float c = 0.7978845608028654f;
+  float t = tanhf(c * (z + 0.044715f * z * z * z));
+  return 0.5f * (1.f + t) + 0.5f * z * (1.f - t * t) * c * (1.f + 3.f * 0.044715f * z * z);
+}
+
+template <int BN, bool A_MN, bool B_MN>
+__global__ void __launch_bounds__(kThreads, 1)
+gemm_bf16_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                    GemmEpilogue ep, int M, int N, int K) {
+  using C = Cfg<BN>;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + C::kStages * C::kStageBytes);
+  uint64_t* empty = full + C::kStages;
+  uint64_t* tfull = empty + C::kStages;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+
+  const int warp = threadIdx.x / 32;
+  const int lane = threadIdx.x % 32;
+  const int num_m = (M + BM - 1) / BM;
+  const int num_n = (N + BN - 1) / BN;
+  const int num_tiles = num_m * num_n;
+  const int nk = (K + BK - 1) / BK;
+
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&tmA);
+    tma_prefetch_desc(&tmB);
+    for (int s = 0; s < C::kStages; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
+    for (int a = 0; a < 2; ++a) { mbar_init(&tfull[a], 1); mbar_init(&tempty[a], 128); }
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc<C::kTmemCols>(tmem_slot);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  if (warp == 0) {
+    // ===================== TMA producer =====================
+    if (elect_one()) {
+      int s = 0; uint32_t ph = 0;
+      for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
+        const int m0 = (tile % num_m) * BM, n0 = (tile / num_m) * BN;
+        for (int kb = 0; kb < nk; ++kb) {
+          mbar_wait(&empty[s], ph ^ 1);
+          uint8_t* sa = smem + s * C::kStageBytes;
+          uint8_t* sb = sa + C::kABytes;
+          mbar_arrive_expect_tx(&full[s], C::kStageBytes);
+          const int k0 = kb * BK;
+          if (A_MN) {
+            for (int j = 0; j < BM / 64; ++j) tma_load_2d(sa + j * 8192, &tmA, &full[s], m0 + 64 * j, k0);
+          } else {
+            tma_load_2d(sa, &tmA, &full[s], k0, m0);
+          }
+          if (B_MN) {
+            for (int j = 0; j < BN / 64; ++j) tma_load_2d(sb + j * 8192, &tmB, &full[s], n0 + 64 * j, k0);
+          } else {
+            tma_load_2d(sb, &tmB, &full[s], k0, n0);
+          }
+          if (++s == C::kStages) { s = 0; ph ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ===================== MMA issuer =====================
+    constexpr uint32_t idesc = umma_idesc_bf16(BM, BN, A_MN ? 1 : 0, B_MN ? 1 : 0);
+    int s = 0; uint32_t ph = 0; int t = 0;
+    for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++t) {
+      const int acc = t & 1;
+      const uint32_t acc_ph = (t >> 1) & 1;
+      mbar_wait(&tempty[acc], acc_ph ^ 1);
+      tc_fence_after();
+      const uint32_t d_tmem = tmem_base + acc * BN;
+      for (int kb = 0; kb < nk; ++kb) {
+        mbar_wait(&full[s], ph);
+        tc_fence_after();
+        if (elect_one()) {
+          const uint32_t sa = smem_u32(smem + s * C::kStageBytes);
+          const uint32_t sb = sa + C::kABytes;
+#pragma unroll
+          for (int kk = 0; kk < BK / 16; ++kk) {
+            // K-major SW128: +32 B per 16-element K step inside the 128 B atom row.
+            // MN-major SW128: +16 rows of 128 B per K step; LBO = 8 KB between 64-wide MN atoms.
+            const uint64_t ad = A_MN ? umma_desc_sw128(sa + kk * 2048, 8192, 1024)
+                                     : umma_desc_sw128(sa + kk * 32, 16, 1024);
+            const uint64_t bd = B_MN ? umma_desc_sw128(sb + kk * 2048, 8192, 1024)
+                                     : umma_desc_sw128(sb + kk * 32, 16, 1024);
+            umma_bf16(d_tmem, ad, bd, idesc, (kb | kk) != 0);
+          }
+          umma_commit(&empty[s]);
+          if (kb == nk - 1) umma_commit(&tfull[acc]);
+        }
+        __syncwarp();
+        if (++s == C::kStages) { s = 0; ph ^= 1; }
+      }
+    }
+  } else {
+    // ===================== epilogue (warps 2..5) =====================
+    const int quarter = warp & 3;               // TMEM lanes [32*quarter, 32*quarter+32)
+    int t = 0;
+    for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++t) {
+      const int acc = t & 1;
+      const uint32_t acc_ph = (t >> 1) & 1;
+      const int m0 = (tile % num_m) * BM, n0 = (tile / num_m) * BN;
+      mbar_wait(&tfull[acc], acc_ph);
+      tc_fence_after();
+      const int row = m0 + quarter * 32 + lane;
+      const bool row_ok = row < M;
+#pragma unroll 1
+      for (int c = 0; c < BN / 32; ++c) {
+        uint32_t r[32];
+        tmem_ld_32x32b_x32(tmem_base + acc * BN + c * 32 + (static_cast<uint32_t>(quarter * 32) << 16), r);
+        tmem_ld_wait();
+        const int col0 = n0 + c * 32;
+        if (!row_ok || col0 >= N) continue;
+        float v[32];
+#pragma unroll
+        for (int j = 0; j < 32; ++j) v[j] = __uint_as_float(r[j]);
+        const bool full_cols = col0 + 32 <= N;
+        if (ep.bias) {
+#pragma unroll
+          for (int j = 0; j < 32; ++j) if (full_cols || col0 + j < N) v[j] += ep.bias[col0 + j];
+        }
+        if (ep.aux) {  // GeLU backward: D = acc * gelu'(Z)
+          const __nv_bfloat16* z = ep.aux + static_cast<size_t>(row) * ep.ld_aux + col0;
+#pragma unroll
+          for (int j = 0; j < 32; ++j) if (full_cols || col0 + j < N) v[j] *= gelu_tanh_grad_f(__bfloat162float(z[j]));
+        }
+        if (ep.residual) {
+          const __nv_bfloat16* rr = ep.residual + static_cast<size_t>(row) * ep.ld_res + col0;
+          if (full_cols) {
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+              uint4 u = *reinterpret_cast<const uint4*>(rr + q * 8);
+              const __nv_bfloat16* h = reinterpret_cast<const __nv_bfloat16*>(&u);
+#pragma unroll
+              for (int j = 0; j < 8; ++j) v[q * 8 + j] += __bfloat162float(h[j]);
+            }
+          } else {
+            for (int j = 0; j < 32; ++j) if (col0 + j < N) v[j] += __bfloat162float(rr[j]);
+          }
+        }
+        if (ep.out_f32) {
+          float* d = ep.d_f32 + static_cast<size_t>(row) * ep.ldd + col0;
+          if (full_cols) {
+#pragma unroll
+            for (int q = 0; q < 8; ++q) {
+              float4 o = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+              if (ep.beta != 0.f) {
+                float4 old = *reinterpret_cast<const float4*>(d + 4 * q);
+                o.x += ep.beta * old.x; o.y += ep.beta * old.y; o.z += ep.beta * old.z; o.w += ep.beta * old.w;
+              }
+              *reinterpret_cast<float4*>(d + 4 * q) = o;
+            }
+          } else {
+            for (int j = 0; j < 32; ++j)
+              if (col0 + j < N) d[j] = v[j] + (ep.beta != 0.f ? ep.beta * d[j] : 0.f);
+          }
+        } else {
+          __nv_bfloat16* d = ep.d_bf16 + static_cast<size_t>(row) * ep.ldd + col0;
+          __nv_bfloat16* d2 = ep.d2_bf16 ? ep.d2_bf16 + static_cast<size_t>(row) * ep.ldd + col0 : nullptr;
+          if (full_cols) {
+#pragma unroll
+            for (int q = 0; q < 4; ++q) {
+              uint4 u, u2;
+              __nv_bfloat16* h = reinterpret_cast<__nv_bfloat16*>(&u);
+              __nv_bfloat16* h2 = reinterpret_cast<__nv_bfloat16*>(&u2);
+#pragma unroll
+              for (int j = 0; j < 8; ++j) {
+                h[j] = __float2bfloat16_rn(v[q * 8 + j]);
+                if (d2) h2[j] = __float2bfloat16_rn(gelu_tanh_f(v[q * 8 + j]));
+              }
+              *reinterpret_cast<uint4*>(d + q * 8) = u;
+              if (d2) *reinterpret_cast<uint4*>(d2 + q * 8) = u2;
+            }
+          } else {
+            for (int j = 0; j < 32; ++j) if (col0 + j < N) {
+              d[j] = __float2bfloat16_rn(v[j]);
+              if (d2) d2[j] = __float2bfloat16_rn(gelu_tanh_f(v[j]));
+            }
+          }
+        }
+      }
+      tc_fence_before();
+      mbar_arrive(&tempty[acc]);
+    }
+  }
+  __syncthreads();
+  if (warp == 1) tmem_dealloc<C::kTmemCols>(tmem_base);
+}
+
+PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    cudaDriverEntryPointQueryResult q;
+    void* p = nullptr;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q) == cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(p);
+  });
+  return fn;
+}
+
+// 2-D bf16 tensor map over a row-major [outer][inner] matrix with row pitch ld (elements).
+bool make_tmap(CUtensorMap* map, const void* base, uint64_t inner, uint64_t outer, uint64_t ld,
+               uint32_t box_inner, uint32_t box_outer) {
+  auto enc = get_encode();
+  if (!enc) return false;
+  cuuint64_t dims[2] = {inner, outer};
+  cuuint64_t strides[1] = {ld * 2};
+  cuuint32_t box[2] = {box_inner, box_outer};
+  cuuint32_t estr[2] = {1, 1};
+  CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, estr,
+                   CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS;
+}
+
+template <int BN, bool A_MN, bool B_MN>
+cudaError_t launch_bn(const GemmArgs& g, cudaStream_t st, int num_sms) {
+  using C = Cfg<BN>;
+  CUtensorMap ta, tb;
+  bool ok = A_MN ? make_tmap(&ta, g.A, g.M, g.K, g.lda, 64, 64) : make_tmap(&ta, g.A, g.K, g.M, g.lda, 64, BM);
+  ok = ok && (B_MN ? make_tmap(&tb, g.B, g.N, g.K, g.ldb, 64, 64) : make_tmap(&tb, g.B, g.K, g.N, g.ldb, 64, BN));
+  if (!ok) return cudaErrorInvalidValue;
+  auto kern = gemm_bf16_tc_kernel<BN, A_MN, B_MN>;
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::kSmem);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  const int tiles = ((g.M + BM - 1) / BM) * ((g.N + BN - 1) / BN);
+  const int grid = tiles < num_sms ? tiles : num_sms;
+  kern<<<grid, kThreads, C::kSmem, st>>>(ta, tb, g.ep, g.M, g.N, g.K);
+  return cudaGetLastError();
+}
+
+template <int BN>
+cudaError_t launch_major(const GemmArgs& g, cudaStream_t st, int num_sms) {
+  if (!g.a_mn && !g.b_mn) return launch_bn<BN, false, false>(g, st, num_sms);
+  if (!g.a_mn && g.b_mn) return launch_bn<BN, false, true>(g, st, num_sms);
+  if (g.a_mn && g.b_mn) return launch_bn<BN, true, true>(g, st, num_sms);
+  return launch_bn<BN, true, false>(g, st, num_sms);
+}
+
+}  // namespace
+
+int device_sm_count() {
+  static int n = 0;
+  if (n == 0) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+    if (n <= 0) n = 148;
+  }
+  return n;
+}
+
+cudaError_t gemm_bf16(const GemmArgs& g, cudaStream_t st) {
+  if (g.M <= 0 || g.N <= 0 || g.K <= 0) return cudaSuccess;
+  if ((g.lda % 8) || (g.ldb % 8)) return cudaErrorInvalidValue;  // TMA: 16-byte row pitch
+  const int sms = device_sm_count();
+  // Prefer BN=256 unless it leaves the machine badly under-filled.
+  const long tiles256 = static_cast<long>((g.M + BM - 1) / BM) * ((g.N + 255) / 256);
+  if (g.N > 128 && tiles256 >= sms / 2) return launch_major<256>(g, st, sms);
+  return launch_major<128>(g, st, sms);
+}
+
+}  // namespace mario

@@ -1,0 +1,48 @@
+// Internal launch interface of the per-layer kernels (K1-K15).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+#include <cuda_bf16.h>
+
+namespace mario {
+
+int device_sm_count();
+
+// ------------------------------------------------------------------ GEMM (K1-K4)
+struct GemmEpilogue {
+  int out_f32 = 0;                        // 1: fp32 output (d_f32), 0: bf16 output (d_bf16)
+  float* d_f32 = nullptr;
+  __nv_bfloat16* d_bf16 = nullptr;
+  __nv_bfloat16* d2_bf16 = nullptr;       // optional second output gelu(D) (GPT fc1)
+  int ldd = 0;
+  float beta = 0.f;                       // fp32 output: D = acc + beta * D
+  const float* bias = nullptr;            // [N], added before activation / residual
+  const __nv_bfloat16* residual = nullptr; int ld_res = 0;   // D += residual
+  const __nv_bfloat16* aux = nullptr; int ld_aux = 0;        // D = acc * gelu'(aux)  (GeLU bwd)
+};
+
+struct GemmArgs {
+  // D[M,N] = A[M,K] . B[N,K]^T ; a_mn / b_mn: operand stored MN-major ([K][rows]).
+  const __nv_bfloat16* A = nullptr; int lda = 0; int a_mn = 0;
+  const __nv_bfloat16* B = nullptr; int ldb = 0; int b_mn = 0;
+  int M = 0, N = 0, K = 0;
+  GemmEpilogue ep;
+};
+
+cudaError_t gemm_bf16(const GemmArgs& g, cudaStream_t st);   // tcgen05 + TMA + TMEM
+
+// fp32 SIMT GEMM (fp32 mode, K4): same contract with float operands.
+struct GemmF32Args {
+  const float* A = nullptr; int lda = 0; int a_mn = 0;
+  const float* B = nullptr; int ldb = 0; int b_mn = 0;
+  int M = 0, N = 0, K = 0;
+  float* D = nullptr; int ldd = 0;
+  float beta = 0.f;
+  const float* bias = nullptr;
+  const float* residual = nullptr; int ld_res = 0;
+  float* D2 = nullptr;                  // gelu(D) second output
+  const float* aux = nullptr; int ld_aux = 0;   // D = acc * gelu'(aux)
+};
+cudaError_t gemm_f32(const GemmF32Args& g, cudaStream_t st);
+
+}  // namespace mario

@@ -1,0 +1,42 @@
+// The opaque mario_plan object (immutable after mario_plan returns).
+#pragma once
+#include <string>
+#include <vector>
+
+#include "model.h"
+#include "plan.h"
+
+struct mario_plan {
+  mario_model model{};
+  mario::plan::Pipe pp;
+  int level = MARIO_LEVEL_MARIO;
+  uint64_t budget = 0;
+  int lps = 1;                       // layers per virtual stage
+  mario::plan::Lists lists;
+  std::vector<std::vector<mario_instr>> instrs;   // per device, exported IR
+  mario::plan::SimCosts costs;
+  mario::plan::SimResult sim;
+  mario::plan::MemResult mem;
+  // exported simulator arrays
+  std::vector<double> busy;
+  std::vector<uint64_t> peak;
+  std::vector<int32_t> live_act, live_ckpt;
+  // parameters
+  std::vector<mario::ParamSpec> params;
+  std::vector<std::string> param_names;
+  struct RankParams {
+    std::vector<int32_t> idx;        // global param index per packed tensor
+    std::vector<uint64_t> off, cnt;  // element offset / count in the packed buffer
+    std::vector<int32_t> part;       // part (virtual stage slot) owning the tensor
+    uint64_t total = 0;
+  };
+  std::vector<RankParams> rank_params;
+  // executor pools per device (slot counts) for multi-process and loopback execution
+  struct Pools { int ckpt = 0, act = 0, send_act = 0, send_grad = 0, recv_grad = 0; };
+  std::vector<Pools> pools_mp, pools_lb;
+  std::vector<uint64_t> workspace_mp, workspace_lb;  // bytes per device
+  // global execution order used by loopback (device, list index), round-robin like the simulator
+  std::vector<std::pair<int, int>> loopback_order;
+  std::string serialized;
+};
+typedef struct mario_plan PlanObj;

@@ -1,0 +1,141 @@
+"""The C++ planner behind the C-ABI (mario_plan) must emit exactly the schedule oracle's
+lists (oracle/schedule.py) and reproduce its simulated makespans; plus ABI checks. CPU only:
+the planner is host code, no GPU is touched."""
+import os
+
+import numpy as np
+import pytest
+
+import synth
+from oracle import schedule as osch
+from paper_conf_ppopp_liultj25_b200 import _lib
+from paper_conf_ppopp_liultj25_b200.api import MarioError, Plan
+
+TINY = synth.TINY_GPT
+OP_SCHEME = {"1f1b": osch.V_1F1B, "interleave": osch.W_INTERLEAVE, "chimera": osch.X_CHIMERA}
+
+
+def unit_costs(K, F=1.0, B=2.0, R=1.0, comm=0.0):
+    return {"fw_ms": [F] * K, "bw_ms": [B] * K, "rc_ms": [R] * K, "p2p_alpha_ms": comm, "p2p_GBps": 0.0,
+            "act_bytes": [1.0] * K, "ckpt_bytes": [0.0] * K, "work_bytes": [0.0] * K, "static_bytes": 0.0}
+
+
+def model_for(L):
+    return synth.with_(TINY, n_layers=L)
+
+
+CASES = [("1f1b", 4, 4, 1), ("1f1b", 2, 4, 1), ("1f1b", 4, 8, 1), ("1f1b", 8, 8, 1), ("1f1b", 3, 5, 1),
+         ("interleave", 4, 4, 2), ("interleave", 4, 8, 2), ("interleave", 2, 4, 2), ("chimera", 4, 4, 1),
+         ("chimera", 4, 8, 1), ("chimera", 2, 4, 1)]
+
+
+@pytest.mark.parametrize("level", ["base", "ckpt", "mario"])
+@pytest.mark.parametrize("scheme,S,N,v", CASES)
+def test_lists_match_oracle(scheme, S, N, v, level):
+    K = S * v
+    pipe = osch.Pipe(OP_SCHEME[scheme], S, N, v)
+    F = 1.0 / v
+    c = osch.UnitCosts(F=F, B=2 * F, R=F)
+    want = osch.transform(pipe, level, c)
+    plan = Plan(model_for(K * 2 if scheme != "chimera" else S * 2), S, N, scheme, level, chunks=v, dtype="f32",
+                costs=unit_costs(K, F, 2 * F, F))
+    assert plan.lists() == want
+    assert plan.simulate().makespan_ms == osch.simulate(pipe, want, c).makespan
+    for d in range(S):
+        a, b = plan.timeline(d)
+        r = osch.simulate(pipe, want, c)
+        comp = [x for x in want[d] if x[0] in osch.COMPUTE]
+        assert a == [r.start[(d,) + x] for x in comp]
+
+
+def test_fig2_through_abi():
+    totals = []
+    for level in ("base", "ckpt", "mario"):
+        p = Plan(model_for(4), 4, 4, "1f1b", level, dtype="f32", costs=unit_costs(4))
+        totals.append(p.simulate().makespan_ms)
+    assert totals == [21.0, 28.0, 22.0]
+
+
+def test_memory_counts_match_oracle():
+    for scheme, S, N, v in [("1f1b", 8, 16, 1), ("interleave", 4, 8, 2), ("chimera", 4, 8, 1)]:
+        pipe = osch.Pipe(OP_SCHEME[scheme], S, N, v)
+        for level in ("base", "mario"):
+            want = osch.memory_walk(pipe, osch.transform(pipe, level, osch.UnitCosts(F=1 / v, B=2 / v, R=1 / v)),
+                                    osch.MemUnits())
+            p = Plan(model_for(S * v * (2 if scheme == "chimera" else 1)), S, N, scheme, level, chunks=v,
+                     dtype="f32", costs=unit_costs(S * v, 1 / v, 2 / v, 1 / v))
+            assert p.simulate().max_live_act == want.max_live_act
+
+
+def test_budget_matches_oracle_and_ebudget():
+    pipe = osch.Pipe(osch.V_1F1B, 4, 4)
+    mem = osch.MemUnits(act=10.0, ckpt=1.0, work=0.0)
+    c = osch.UnitCosts()
+    l3 = osch.pass3_remove_redundancy(osch.pass2_overlap_recompute(osch.pass1_apply_checkpoint(osch.build_base(pipe))))
+    budget = max(osch.memory_walk(pipe, l3, mem).peak)
+    want = osch.pass4_prepose_forward(pipe, l3, c, mem=mem, budget=budget)
+    costs = unit_costs(4)
+    costs.update(act_bytes=[10.0] * 4, ckpt_bytes=[1.0] * 4)
+    p = Plan(model_for(4), 4, 4, "1f1b", "mario", dtype="f32", costs=costs, mem_budget=int(budget))
+    assert p.lists() == want
+    with pytest.raises(MarioError) as e:
+        Plan(model_for(4), 4, 4, "1f1b", "base", dtype="f32", costs=costs, mem_budget=int(budget) - 1)
+    assert e.value.code == -2
+
+
+def test_serialization_deterministic_and_golden():
+    p1 = Plan(model_for(4), 4, 4, "1f1b", "mario", dtype="f32", costs=unit_costs(4))
+    p2 = Plan(model_for(4), 4, 4, "1f1b", "mario", dtype="f32", costs=unit_costs(4))
+    s = p1.serialize()
+    assert s == p2.serialize()
+    gold = open(os.path.join(os.path.dirname(__file__), "golden", "plan_fig2_mario.txt")).read()
+    assert s == gold
+
+
+@pytest.mark.parametrize("bad", [dict(stages=3, N=4, L=4),            # L % S != 0
+                                 dict(stages=4, N=6, L=8, scheme="interleave", v=2),   # N % S
+                                 dict(stages=3, N=6, L=6, scheme="chimera")])          # odd S
+def test_einval(bad):
+    with pytest.raises(MarioError) as e:
+        Plan(model_for(bad["L"]), bad["stages"], bad["N"], bad.get("scheme", "1f1b"), "mario",
+             chunks=bad.get("v", 1), dtype="f32")
+    assert e.value.code == -1
+
+
+def test_param_names_match_synth():
+    for cfg in (TINY, synth.tiny_llama(), synth.with_(TINY, tie_embeddings=False)):
+        p = Plan(cfg, 2, 4, "1f1b", "mario", dtype="f32")
+        assert p.param_names() == [n for n, _ in synth.param_shapes(cfg)]
+
+
+def test_rank_params_cover_model():
+    cfg = TINY
+    shapes = dict(synth.param_shapes(cfg))
+    for scheme, S, v in [("1f1b", 2, 1), ("interleave", 2, 2), ("chimera", 2, 1), ("1f1b", 1, 1)]:
+        p = Plan(cfg, S, 2 * S if scheme != "1f1b" else 4, scheme, "mario", chunks=v, dtype="f32")
+        seen = {}
+        for r in range(S):
+            for name, off, cnt in p.rank_params(r):
+                assert cnt == int(np.prod(shapes[name]))
+                assert off % 64 == 0
+                seen[name] = seen.get(name, 0) + 1
+        assert set(seen) == set(shapes)
+        if scheme == "chimera":
+            assert all(v == 2 for k, v in seen.items() if k != "wte") and seen["wte"] == 4
+        elif S > 1:
+            assert seen["wte"] == 2 and all(v == 1 for k, v in seen.items() if k != "wte")
+
+
+def test_library_exports_every_declared_symbol():
+    """include/*.h declarations are all exported by libmario.so (no compute calls)."""
+    import re
+    root = os.path.dirname(os.path.dirname(__file__))
+    lib = _lib.lib()
+    names = []
+    for h in ("mario.h", "mario_kernels.h"):
+        txt = open(os.path.join(root, "include", h)).read()
+        txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
+        names += re.findall(r"\b(mario_[a-z0-9_]+)\s*\(", txt)
+    assert len(set(names)) > 15
+    for n in set(names):
+        assert hasattr(lib, n), n
