@@ -182,3 +182,92 @@ class Plan:
                                                  C.byref(n)))
         names = self.param_names()
         return [(names[idx[i]], off[i], cnt[i]) for i in range(n.value)]
+
+
+# ------------------------------------------------------------------------- executor
+def pack_params(plan: Plan, params: Dict[str, "object"], rank: int):
+    """Pack a {name: array} model into rank's fp32 buffer (rank=-1: loopback, all ranks
+    concatenated). Pure layout marshalling (offsets come from the library)."""
+    import numpy as np
+    ranks = range(plan.S) if rank == -1 else [rank]
+    bufs = []
+    for r in ranks:
+        total = plan.rank_layout(r)[0]
+        b = np.zeros(total, dtype=np.float32)
+        for name, off, cnt in plan.rank_params(r):
+            b[off:off + cnt] = np.asarray(params[name], dtype=np.float32).reshape(-1)
+        bufs.append(b)
+    return np.concatenate(bufs) if bufs else np.zeros(0, np.float32)
+
+
+def unpack_params(plan: Plan, flat, rank: int) -> Dict[str, "object"]:
+    """Inverse of pack_params for grads: {name: array} (first copy of every tensor)."""
+    import numpy as np
+    shapes = {n: s for n, s in _shapes(plan)}
+    out = {}
+    ranks = range(plan.S) if rank == -1 else [rank]
+    base = 0
+    for r in ranks:
+        for name, off, cnt in plan.rank_params(r):
+            if name not in out:
+                out[name] = np.asarray(flat[base + off: base + off + cnt]).reshape(shapes[name])
+        base += plan.rank_layout(r)[0]
+    return out
+
+
+def _shapes(plan: Plan):
+    import synth
+    return synth.param_shapes(plan.cfg)
+
+
+class Context:
+    """mario_init(rank, world, device, nccl_id). world > 1 uses torch.distributed (already
+    initialised) only to broadcast the 128-byte NCCL unique id."""
+
+    def __init__(self, rank: int = 0, world: int = 1, device: int = 0):
+        L = _lib.lib()
+        uid = C.create_string_buffer(128)
+        if world > 1:
+            import torch
+            import torch.distributed as dist
+            if rank == 0:
+                _check(L.mario_nccl_unique_id(uid))
+            t = torch.tensor(list(uid.raw), dtype=torch.uint8)
+            dist.broadcast(t, src=0)
+            uid = C.create_string_buffer(bytes(t.tolist()), 128)
+        _check(L.mario_init(rank, world, device, uid if world > 1 else None))
+        self.rank, self.world = rank, world
+
+    def run_iter(self, plan: Plan, weights, tokens, grads, workspace, stream=None) -> float:
+        """weights/grads/workspace: device tensors (data_ptr used); tokens: host int32 array."""
+        import numpy as np
+        tok = np.ascontiguousarray(tokens, dtype=np.int32)
+        loss = C.c_float()
+        st = stream.cuda_stream if stream is not None else None
+        _check(_lib.lib().mario_run_iter(plan.handle, C.c_void_p(weights.data_ptr()),
+                                         tok.ctypes.data_as(C.c_void_p), C.byref(loss),
+                                         C.c_void_p(grads.data_ptr()), C.c_void_p(workspace.data_ptr()),
+                                         C.c_void_p(st) if st else None))
+        return float(loss.value)
+
+    def set_timing(self, on: bool):
+        _check(_lib.lib().mario_set_timing(int(on)))
+
+    def last_timeline(self, d: int):
+        a, b, n = C.POINTER(C.c_double)(), C.POINTER(C.c_double)(), C.c_int32()
+        _check(_lib.lib().mario_last_timeline(d, C.byref(a), C.byref(b), C.byref(n)))
+        return [a[i] for i in range(n.value)], [b[i] for i in range(n.value)]
+
+    def close(self):
+        _lib.lib().mario_finalize()
+
+
+def alloc_for(plan: Plan, rank: int, device="cuda"):
+    """Allocate (weights, grads, workspace) device tensors sized from the plan (torch is
+    used only as the device allocator)."""
+    import torch
+    pc, ws = plan.rank_layout(rank)
+    w = torch.zeros(pc, dtype=torch.float32, device=device)
+    g = torch.zeros(pc, dtype=torch.float32, device=device)
+    work = torch.empty(max(ws, 1), dtype=torch.uint8, device=device)
+    return w, g, work

@@ -44,7 +44,7 @@ Arena make_arena(const PlanObj& P, int dev, const PlanObj::Pools& pools) {
   a.sg = take(a.msg_stride * std::max(1, a.n_sg));
   a.rg = take(a.msg_stride * std::max(1, a.n_rg));
   a.tokens = take(static_cast<size_t>(P.pp.N) * m.micro_batch * (m.seq_len + 1) * 4);
-  a.loss = take(static_cast<size_t>(P.pp.N) * P.pp.parts() * 8);
+  a.loss = take(static_cast<size_t>(P.pp.N) * P.pp.parts() * 8 + tokens_per_micro(m) * 4);
   a.red_bytes = static_cast<size_t>(kRedBlocks) * red_width(m) * 4 * 2;
   a.red = take(a.red_bytes);
   a.total = o;

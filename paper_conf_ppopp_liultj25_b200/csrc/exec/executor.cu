@@ -1,0 +1,814 @@
+// Per-rank executor of a Mario plan (Table 3).
+//
+// Each rank walks its instruction list once per iteration and enqueues, asynchronously:
+//   FW / CFW / RC / BW  -> layer kernels on the compute stream (list order = the plan's
+//                          horizontal dependencies, so RC lands exactly where the plan put
+//                          it: before the RG wait, inside the bubble)
+//   RA / RG             -> ncclRecv on the channel's stream into a static slot; the compute
+//                          stream waits on it at the RA/RG position (blocking receive)
+//   SA / SG             -> ncclSend on the channel's stream after everything before it in the
+//                          list (buffered send; a preposed CFW's output stays in its send slot
+//                          until its SA)
+// One NCCL communicator + stream per channel (ordered pair x {activation, gradient}) keeps
+// every channel a FIFO, so any acyclic plan is deadlock-free.
+// Loopback (world == 1, multi-stage plan): every rank's list runs in this process on one GPU
+// in the simulator's round-robin order; RA/RG become device-to-device copies.
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <cmath>
+#include <cstdio>
+#include <cstring>
+#include <algorithm>
+#include <map>
+#include <set>
+#include <memory>
+#include <stdexcept>
+#include <string>
+#include <tuple>
+#include <vector>
+
+#include "../capi/status.h"
+#include "../kernels/kernels.h"
+#include "../kernels/layers.h"
+#include "arena.h"
+
+namespace mario {
+namespace {
+
+using plan::Instr;
+
+#define CU(x)                                                                       \
+  do {                                                                              \
+    cudaError_t e_ = (x);                                                           \
+    if (e_ != cudaSuccess) throw CudaErr(std::string(#x) + ": " + cudaGetErrorString(e_)); \
+  } while (0)
+#define NC(x)                                                                       \
+  do {                                                                              \
+    ncclResult_t r_ = (x);                                                          \
+    if (r_ != ncclSuccess) throw NcclErr(std::string(#x) + ": " + ncclGetErrorString(r_)); \
+  } while (0)
+
+struct CudaErr : std::runtime_error { using std::runtime_error::runtime_error; };
+struct NcclErr : std::runtime_error { using std::runtime_error::runtime_error; };
+
+// ------------------------------------------------------------------ context
+struct Channel {
+  ncclComm_t comm = nullptr;
+  cudaStream_t stream = nullptr;
+};
+
+struct Context {
+  int rank = 0, world = 1, device = 0;
+  bool inited = false;
+  ncclComm_t world_comm = nullptr;
+  std::map<std::tuple<int, int, int>, Channel> channels;   // (src, dst, kind)
+  std::map<std::pair<int, int>, ncclComm_t> pair_comms;      // (lo, hi) 2-rank comms
+  std::set<std::tuple<int, int, int>> created_channels;       // split already done (all ranks)
+  std::set<std::pair<int, int>> created_pairs;
+  cudaStream_t loss_stream = nullptr;
+  bool timing = false;
+  std::vector<std::vector<double>> t_start, t_finish;
+  bool sticky = false;
+};
+Context g;
+
+// ------------------------------------------------------------- per-device state
+template <class T>
+struct Dev {
+  const PlanObj* P = nullptr;
+  int d = 0;
+  Arena a;
+  uint8_t* ws = nullptr;
+  const float* w = nullptr;   // packed fp32 master weights of this rank
+  float* gr = nullptr;        // packed fp32 grads of this rank
+  std::map<std::pair<int, int>, int> tensor;   // (part, global param idx) -> packed index j
+  // host-side slot pools for send / recv-grad buffers
+  std::vector<bool> sa_used, sg_used, rg_used;
+  std::map<std::pair<int, int>, int> sa_of, sg_of, rg_of;
+  std::vector<cudaEvent_t> sa_free, sg_free, rg_free, ck_free;   // event guarding slot reuse
+  std::vector<bool> sa_free_set, sg_free_set, rg_free_set, ck_free_set;
+  std::vector<cudaEvent_t> ev_pool;
+  size_t ev_next = 0;
+  std::vector<std::pair<cudaEvent_t, cudaEvent_t>> timed;   // per compute instr
+
+  const mario_model& M() const { return P->model; }
+  template <class U = uint8_t> U* at(size_t off) const { return reinterpret_cast<U*>(ws + off); }
+  cudaEvent_t event() {
+    if (ev_next == ev_pool.size()) {
+      cudaEvent_t e;
+      CU(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+      ev_pool.push_back(e);
+    }
+    return ev_pool[ev_next++];
+  }
+};
+
+int acquire(std::vector<bool>& used) {
+  for (size_t i = 0; i < used.size(); ++i) if (!used[i]) { used[i] = true; return static_cast<int>(i); }
+  throw std::runtime_error("executor slot pool exhausted (planner/executor mismatch)");
+}
+
+template <class T>
+struct Exec {
+  cudaStream_t st;
+  bool loopback;
+  std::vector<std::unique_ptr<Dev<T>>> devs;   // loopback: all; otherwise one (this rank)
+
+  Dev<T>& dev(int d) { return loopback ? *devs[d] : *devs[0]; }
+
+  // ---- weights --------------------------------------------------------------
+  int tidx(Dev<T>& D, int p, const std::string& name) {
+    const auto& names = D.P->param_names;
+    for (size_t i = 0; i < names.size(); ++i)
+      if (names[i] == name) {
+        auto it = D.tensor.find({p, static_cast<int>(i)});
+        if (it != D.tensor.end()) return it->second;
+      }
+    throw std::runtime_error("parameter " + name + " not held by part " + std::to_string(p));
+  }
+  const T* Wm(Dev<T>& D, int p, const std::string& name) {   // compute-dtype matrix
+    int j = tidx(D, p, name);
+    if (sizeof(T) == 2) return D.template at<T>(D.a.wcopy[j]);
+    return reinterpret_cast<const T*>(D.w + D.P->rank_params[D.d].off[j]);
+  }
+  const float* Wf(Dev<T>& D, int p, const std::string& name) {
+    return D.w + D.P->rank_params[D.d].off[tidx(D, p, name)];
+  }
+  float* G(Dev<T>& D, int p, const std::string& name) {
+    return D.gr + D.P->rank_params[D.d].off[tidx(D, p, name)];
+  }
+
+  // ---- GEMM dispatch --------------------------------------------------------
+  // D[M,N] = A[M,K] . B[N,K]^T  (see kernels.h); bf16 tcgen05 or fp32 SIMT by dtype.
+  void gemm(const T* A, int lda, int a_mn, const T* B, int ldb, int b_mn, int M, int N, int K, void* Dp, int ldd,
+            bool out_f32, float beta, const float* bias = nullptr, const T* resid = nullptr, T* D2 = nullptr,
+            const T* aux = nullptr) {
+    if constexpr (sizeof(T) == 2) {
+      GemmArgs g;
+      g.A = A; g.lda = lda; g.a_mn = a_mn; g.B = B; g.ldb = ldb; g.b_mn = b_mn; g.M = M; g.N = N; g.K = K;
+      g.ep.out_f32 = out_f32;
+      if (out_f32) g.ep.d_f32 = static_cast<float*>(Dp); else g.ep.d_bf16 = static_cast<__nv_bfloat16*>(Dp);
+      g.ep.ldd = ldd; g.ep.beta = beta; g.ep.bias = bias;
+      g.ep.residual = resid; g.ep.ld_res = ldd; g.ep.d2_bf16 = D2; g.ep.aux = aux; g.ep.ld_aux = ldd;
+      CU(gemm_bf16(g, st));
+    } else {
+      GemmF32Args g;
+      g.A = A; g.lda = lda; g.a_mn = a_mn; g.B = B; g.ldb = ldb; g.b_mn = b_mn; g.M = M; g.N = N; g.K = K;
+      g.D = static_cast<float*>(Dp); g.ldd = ldd; g.beta = beta; g.bias = bias; g.residual = resid;
+      g.ld_res = ldd; g.D2 = D2; g.aux = aux; g.ld_aux = ldd;
+      CU(gemm_f32(g, st));
+    }
+  }
+  // Y[T,out] = X W^T (+bias, +resid, D2 = gelu)
+  void lin_fwd(const T* X, const T* W, int Tn, int out, int in, T* Y, const float* bias, const T* resid = nullptr,
+               T* Y2 = nullptr) {
+    gemm(X, in, 0, W, in, 0, Tn, out, in, Y, out, false, 0.f, bias, resid, Y2);
+  }
+  // dX[T,in] = dY W (optionally * gelu'(aux))
+  void lin_dgrad(const T* dY, const T* W, int Tn, int out, int in, T* dX, const T* aux = nullptr) {
+    gemm(dY, out, 0, W, in, 1, Tn, in, out, dX, in, false, 0.f, nullptr, nullptr, nullptr, aux);
+  }
+  // dW[out,in] += dY^T X (fp32)
+  void lin_wgrad(const T* dY, const T* X, int Tn, int out, int in, float* dW) {
+    gemm(dY, out, 1, X, in, 1, out, in, Tn, dW, in, true, 1.f);
+  }
+
+  // ---- forward of one virtual stage -------------------------------------------
+  // mode: 0 = FW (keep activations in act set), 1 = CFW (scratch), 2 = RC (act set, no loss)
+  void stage_forward(Dev<T>& D, const mario_instr& x, int mode, T* out) {
+    const mario_model& m = D.M();
+    const int K = D.P->pp.K(), k = x.vstage, p = x.part, lps = D.P->lps;
+    const int Tn = static_cast<int>(tokens_per_micro(m)), h = m.hidden, f = m.ffn_hidden, nh = m.n_heads;
+    const int dh = h / nh, s = m.seq_len, mbs = m.micro_batch;
+    const bool gpt = m.family == MARIO_GPT;
+    const LayerAct LA = layer_act_layout(m);
+    const HeadAct HA = head_act_layout(m);
+    uint8_t* base;
+    size_t lstride;
+    if (mode == 1) { base = D.template at<uint8_t>(D.a.cfw); lstride = 0; }
+    else { base = D.template at<uint8_t>(D.a.act + static_cast<size_t>(x.aslot) * D.a.act_stride); lstride = LA.bytes; }
+    uint8_t* head_base = (mode == 1) ? base + LA.bytes + 2 * stage_input_bytes(m) : base + LA.bytes * lps;
+    T* run[2] = {reinterpret_cast<T*>(D.template at<uint8_t>(D.a.cfw) + LA.bytes),
+                 reinterpret_cast<T*>(D.template at<uint8_t>(D.a.cfw) + LA.bytes + stage_input_bytes(m))};
+    const int32_t* tok = D.template at<int32_t>(D.a.tokens) + static_cast<size_t>(x.micro) * mbs * (s + 1);
+    // stage input
+    const T* Hin;
+    if (k == 0) {
+      T* H0 = (mode == 1) ? run[0] : reinterpret_cast<T*>(base + LA.H_in);
+      const T* wte = Wm(D, p, gpt ? "wte" : "emb");
+      const T* wpe = gpt ? Wm(D, p, "wpe") : nullptr;
+      embed_fwd<T>(tok, s + 1, mbs, s, wte, wpe, H0, h, st);
+      Hin = H0;
+    } else {
+      Hin = D.template at<T>(D.a.ckpt + static_cast<size_t>(x.slot) * D.a.ckpt_stride);
+    }
+    for (int li = 0; li < lps; ++li) {
+      const int l = k * lps + li;
+      const std::string pre = "h" + std::to_string(l) + ".";
+      uint8_t* L = base + li * lstride;
+      T* A = reinterpret_cast<T*>(L + LA.A);
+      T* QKV = reinterpret_cast<T*>(L + LA.QKV);
+      T* O = reinterpret_cast<T*>(L + LA.O);
+      float* LSE = reinterpret_cast<float*>(L + LA.LSE);
+      T* H1 = reinterpret_cast<T*>(L + LA.H1);
+      T* A2 = reinterpret_cast<T*>(L + LA.A2);
+      T* Z = reinterpret_cast<T*>(L + LA.Z);
+      T* Gt = reinterpret_cast<T*>(L + LA.G);
+      float* st1 = reinterpret_cast<float*>(L + LA.st1);
+      float* st2 = reinterpret_cast<float*>(L + LA.st2);
+      // output of this layer
+      T* Hout;
+      if (li + 1 < lps) Hout = (mode == 1) ? run[(li + 1) & 1] : reinterpret_cast<T*>(base + (li + 1) * lstride + LA.H_in);
+      else if (k == K - 1) Hout = reinterpret_cast<T*>(head_base + HA.H_last);
+      else Hout = out;
+      if (gpt) {
+        layernorm_fwd<T>(Hin, Wf(D, p, pre + "ln1.g"), Wf(D, p, pre + "ln1.b"), A, st1, Tn, h, m.norm_eps, st);
+        lin_fwd(A, Wm(D, p, pre + "qkv.w"), Tn, 3 * h, h, QKV, Wf(D, p, pre + "qkv.b"));
+      } else {
+        rmsnorm_fwd<T>(Hin, Wf(D, p, pre + "n1.g"), A, st1, Tn, h, m.norm_eps, st);
+        lin_fwd(A, Wm(D, p, pre + "qkv.w"), Tn, 3 * h, h, QKV, nullptr);
+        rope<T>(QKV, mbs, s, nh, dh, m.rope_base, 0, st);
+      }
+      attn_fwd<T>(QKV, O, LSE, mbs, s, nh, dh, st);
+      if (gpt) {
+        lin_fwd(O, Wm(D, p, pre + "proj.w"), Tn, h, h, H1, Wf(D, p, pre + "proj.b"), Hin);
+        layernorm_fwd<T>(H1, Wf(D, p, pre + "ln2.g"), Wf(D, p, pre + "ln2.b"), A2, st2, Tn, h, m.norm_eps, st);
+        lin_fwd(A2, Wm(D, p, pre + "fc1.w"), Tn, f, h, Z, Wf(D, p, pre + "fc1.b"), nullptr, Gt);
+        lin_fwd(Gt, Wm(D, p, pre + "fc2.w"), Tn, h, f, Hout, Wf(D, p, pre + "fc2.b"), H1);
+      } else {
+        lin_fwd(O, Wm(D, p, pre + "o.w"), Tn, h, h, H1, nullptr, Hin);
+        rmsnorm_fwd<T>(H1, Wf(D, p, pre + "n2.g"), A2, st2, Tn, h, m.norm_eps, st);
+        lin_fwd(A2, Wm(D, p, pre + "gu.w"), Tn, 2 * f, h, Z, nullptr);
+        swiglu_fwd<T>(Z, Gt, Tn, f, st);
+        lin_fwd(Gt, Wm(D, p, pre + "down.w"), Tn, h, f, Hout, nullptr, H1);
+      }
+      Hin = Hout;
+    }
+    if (k == K - 1) {
+      T* Hl = reinterpret_cast<T*>(head_base + HA.H_last);
+      T* Hf = reinterpret_cast<T*>(head_base + HA.Hf);
+      float* stf = reinterpret_cast<float*>(head_base + HA.stf);
+      T* dlog = reinterpret_cast<T*>(head_base + HA.dlogits);
+      const int V = m.vocab;
+      if (gpt) layernorm_fwd<T>(Hl, Wf(D, p, "lnf.g"), Wf(D, p, "lnf.b"), Hf, stf, Tn, h, m.norm_eps, st);
+      else rmsnorm_fwd<T>(Hl, Wf(D, p, "nf.g"), Hf, stf, Tn, h, m.norm_eps, st);
+      const T* Wh = Wm(D, p, gpt ? (m.tie_embeddings ? "wte" : "head.w") : "out.w");
+      float* logits = D.template at<float>(D.a.logits);
+      gemm(Hf, h, 0, Wh, h, 0, Tn, V, h, logits, V, true, 0.f);
+      float* row_loss = reinterpret_cast<float*>(D.template at<uint8_t>(D.a.loss) +
+                                                 static_cast<size_t>(D.P->pp.N) * D.P->pp.parts() * 8);
+      const float inv_ntok = 1.0f / static_cast<float>(static_cast<double>(D.P->pp.N) * Tn);
+      softmax_ce<T>(logits, tok, s + 1, s, Tn, V, inv_ntok, dlog, row_loss, st);
+      if (mode != 2) loss_reduce(row_loss, Tn, D.template at<double>(D.a.loss) + x.micro, st);
+    }
+  }
+
+  // ---- backward of one virtual stage ------------------------------------------
+  void stage_backward(Dev<T>& D, const mario_instr& x, const T* dout, T* dstage_in) {
+    const mario_model& m = D.M();
+    const int K = D.P->pp.K(), k = x.vstage, p = x.part, lps = D.P->lps;
+    const int Tn = static_cast<int>(tokens_per_micro(m)), h = m.hidden, f = m.ffn_hidden, nh = m.n_heads;
+    const int dh = h / nh, s = m.seq_len, mbs = m.micro_batch;
+    const bool gpt = m.family == MARIO_GPT;
+    const LayerAct LA = layer_act_layout(m);
+    const HeadAct HA = head_act_layout(m);
+    const BwScratch BS = bw_scratch_layout(m);
+    uint8_t* base = D.template at<uint8_t>(D.a.act + static_cast<size_t>(x.aslot) * D.a.act_stride);
+    uint8_t* head_base = base + LA.bytes * lps;
+    uint8_t* sc = D.template at<uint8_t>(D.a.bw);
+    T* dHbuf[3] = {reinterpret_cast<T*>(sc + BS.dH[0]), reinterpret_cast<T*>(sc + BS.dH[1]),
+                   reinterpret_cast<T*>(sc + BS.dH[2])};
+    T* dA = reinterpret_cast<T*>(sc + BS.dA);
+    T* dQKV = reinterpret_cast<T*>(sc + BS.dQKV);
+    T* dO = reinterpret_cast<T*>(sc + BS.dO);
+    T* dZ = reinterpret_cast<T*>(sc + BS.dZ);
+    T* dM = reinterpret_cast<T*>(sc + BS.dM);
+    float* Dsc = reinterpret_cast<float*>(sc + BS.Dsc);
+    float* red = D.template at<float>(D.a.red);
+    const int32_t* tok = D.template at<int32_t>(D.a.tokens) + static_cast<size_t>(x.micro) * mbs * (s + 1);
+    int cur = 0;
+    const T* dH;   // gradient of the current layer's output
+    if (k == K - 1) {
+      const int V = m.vocab;
+      T* Hl = reinterpret_cast<T*>(head_base + HA.H_last);
+      T* Hf = reinterpret_cast<T*>(head_base + HA.Hf);
+      float* stf = reinterpret_cast<float*>(head_base + HA.stf);
+      T* dlog = reinterpret_cast<T*>(head_base + HA.dlogits);
+      const std::string hw = gpt ? (m.tie_embeddings ? "wte" : "head.w") : "out.w";
+      lin_wgrad(dlog, Hf, Tn, V, h, G(D, p, hw));
+      lin_dgrad(dlog, Wm(D, p, hw), Tn, V, h, dA);      // dHf
+      T* dHl = dHbuf[cur];
+      if (gpt) {
+        norm_bwd_dx<T>(dA, Hl, stf, Wf(D, p, "lnf.g"), nullptr, dHl, Tn, h, 0, st);
+        colsum<T>(dA, Hl, stf, Tn, h, h, 1, G(D, p, "lnf.g"), G(D, p, "lnf.b"), red, st);
+      } else {
+        norm_bwd_dx<T>(dA, Hl, stf, Wf(D, p, "nf.g"), nullptr, dHl, Tn, h, 1, st);
+        colsum<T>(dA, Hl, stf, Tn, h, h, 2, G(D, p, "nf.g"), nullptr, red, st);
+      }
+      dH = dHl;
+    } else {
+      dH = dout;
+      cur = 2;   // first written buffer rotates from 0
+    }
+    for (int li = lps - 1; li >= 0; --li) {
+      const int l = k * lps + li;
+      const std::string pre = "h" + std::to_string(l) + ".";
+      uint8_t* L = base + li * LA.bytes;
+      const T* Hin = (li == 0 && k > 0) ? D.template at<T>(D.a.ckpt + static_cast<size_t>(x.slot) * D.a.ckpt_stride)
+                                        : reinterpret_cast<T*>(L + LA.H_in);
+      T* A = reinterpret_cast<T*>(L + LA.A);
+      T* QKV = reinterpret_cast<T*>(L + LA.QKV);
+      T* O = reinterpret_cast<T*>(L + LA.O);
+      float* LSE = reinterpret_cast<float*>(L + LA.LSE);
+      T* H1 = reinterpret_cast<T*>(L + LA.H1);
+      T* A2 = reinterpret_cast<T*>(L + LA.A2);
+      T* Z = reinterpret_cast<T*>(L + LA.Z);
+      T* Gt = reinterpret_cast<T*>(L + LA.G);
+      float* st1 = reinterpret_cast<float*>(L + LA.st1);
+      float* st2 = reinterpret_cast<float*>(L + LA.st2);
+      T* dH1 = dHbuf[(cur + 1) % 3];
+      T* dHin = (li == 0) ? (k == 0 ? dHbuf[(cur + 2) % 3] : dstage_in) : dHbuf[(cur + 2) % 3];
+      if (gpt) {
+        lin_wgrad(dH, Gt, Tn, h, f, G(D, p, pre + "fc2.w"));
+        colsum<T>(dH, nullptr, nullptr, Tn, h, h, 0, G(D, p, pre + "fc2.b"), nullptr, red, st);
+        lin_dgrad(dH, Wm(D, p, pre + "fc2.w"), Tn, h, f, dZ, Z);           // dZ = (dH W2) * gelu'(Z)
+        lin_wgrad(dZ, A2, Tn, f, h, G(D, p, pre + "fc1.w"));
+        colsum<T>(dZ, nullptr, nullptr, Tn, f, f, 0, G(D, p, pre + "fc1.b"), nullptr, red, st);
+        lin_dgrad(dZ, Wm(D, p, pre + "fc1.w"), Tn, f, h, dA);               // dA2
+        norm_bwd_dx<T>(dA, H1, st2, Wf(D, p, pre + "ln2.g"), dH, dH1, Tn, h, 0, st);
+        colsum<T>(dA, H1, st2, Tn, h, h, 1, G(D, p, pre + "ln2.g"), G(D, p, pre + "ln2.b"), red, st);
+        lin_wgrad(dH1, O, Tn, h, h, G(D, p, pre + "proj.w"));
+        colsum<T>(dH1, nullptr, nullptr, Tn, h, h, 0, G(D, p, pre + "proj.b"), nullptr, red, st);
+        lin_dgrad(dH1, Wm(D, p, pre + "proj.w"), Tn, h, h, dO);
+      } else {
+        lin_wgrad(dH, Gt, Tn, h, f, G(D, p, pre + "down.w"));
+        lin_dgrad(dH, Wm(D, p, pre + "down.w"), Tn, h, f, dM);
+        swiglu_bwd<T>(Z, dM, dZ, Tn, f, st);
+        lin_wgrad(dZ, A2, Tn, 2 * f, h, G(D, p, pre + "gu.w"));
+        lin_dgrad(dZ, Wm(D, p, pre + "gu.w"), Tn, 2 * f, h, dA);
+        norm_bwd_dx<T>(dA, H1, st2, Wf(D, p, pre + "n2.g"), dH, dH1, Tn, h, 1, st);
+        colsum<T>(dA, H1, st2, Tn, h, h, 2, G(D, p, pre + "n2.g"), nullptr, red, st);
+        lin_wgrad(dH1, O, Tn, h, h, G(D, p, pre + "o.w"));
+        lin_dgrad(dH1, Wm(D, p, pre + "o.w"), Tn, h, h, dO);
+      }
+      attn_bwd<T>(QKV, O, dO, LSE, dQKV, Dsc, mbs, s, nh, dh, st);
+      if (!gpt) rope<T>(dQKV, mbs, s, nh, dh, m.rope_base, 1, st);
+      lin_wgrad(dQKV, A, Tn, 3 * h, h, G(D, p, pre + "qkv.w"));
+      if (gpt) colsum<T>(dQKV, nullptr, nullptr, Tn, 3 * h, 3 * h, 0, G(D, p, pre + "qkv.b"), nullptr, red, st);
+      lin_dgrad(dQKV, Wm(D, p, pre + "qkv.w"), Tn, 3 * h, h, dA);
+      if (gpt) {
+        norm_bwd_dx<T>(dA, Hin, st1, Wf(D, p, pre + "ln1.g"), dH1, dHin, Tn, h, 0, st);
+        colsum<T>(dA, Hin, st1, Tn, h, h, 1, G(D, p, pre + "ln1.g"), G(D, p, pre + "ln1.b"), red, st);
+      } else {
+        norm_bwd_dx<T>(dA, Hin, st1, Wf(D, p, pre + "n1.g"), dH1, dHin, Tn, h, 1, st);
+        colsum<T>(dA, Hin, st1, Tn, h, h, 2, G(D, p, pre + "n1.g"), nullptr, red, st);
+      }
+      dH = dHin;
+      cur = (cur + 2) % 3;
+    }
+    if (k == 0) {
+      embed_bwd<T>(tok, s + 1, mbs, s, dH, h, G(D, p, gpt ? "wte" : "emb"), gpt ? G(D, p, "wpe") : nullptr,
+                   sc + BS.sort, st);
+    }
+  }
+
+  // ---- one instruction ----------------------------------------------------------
+  T* send_slot(Dev<T>& D, bool grad, int idx) {
+    return D.template at<T>((grad ? D.a.sg : D.a.sa) + static_cast<size_t>(idx) * D.a.msg_stride);
+  }
+
+  void run_instr(int d, const mario_instr& x) {
+    Dev<T>& D = dev(d);
+    const mario_model& m = D.M();
+    const int K = D.P->pp.K();
+    const auto key = std::make_pair(x.micro, x.part);
+    const size_t msg_bytes = tokens_per_micro(m) * m.hidden * sizeof(T);
+    switch (x.op) {
+      case MARIO_OP_FW:
+      case MARIO_OP_CFW:
+      case MARIO_OP_RC: {
+        T* out = nullptr;
+        if (x.op != MARIO_OP_RC && x.vstage < K - 1) {
+          int i = acquire(D.sa_used);
+          D.sa_of[key] = i;
+          if (!loopback && D.sa_free_set[i]) CU(cudaStreamWaitEvent(st, D.sa_free[i], 0));
+          out = send_slot(D, false, i);
+        } else if (x.op == MARIO_OP_RC && x.vstage < K - 1) {
+          out = D.template at<T>(D.a.cfw);   // RC's stage output is not needed: scratch
+        }
+        timed_begin(D);
+        stage_forward(D, x, x.op == MARIO_OP_FW ? 0 : x.op == MARIO_OP_CFW ? 1 : 2, out);
+        timed_end(D);
+        break;
+      }
+      case MARIO_OP_BW: {
+        const T* dout = nullptr;
+        if (x.vstage < K - 1) dout = D.template at<T>(D.a.rg + static_cast<size_t>(D.rg_of[key]) * D.a.msg_stride);
+        T* din = nullptr;
+        if (x.vstage > 0) {
+          int i = acquire(D.sg_used);
+          D.sg_of[key] = i;
+          if (!loopback && D.sg_free_set[i]) CU(cudaStreamWaitEvent(st, D.sg_free[i], 0));
+          din = send_slot(D, true, i);
+        }
+        timed_begin(D);
+        stage_backward(D, x, dout, din);
+        timed_end(D);
+        // release stage-input slot, recv-grad slot (activation slots are list-order, planner-assigned)
+        if (x.slot >= 0) { CU(cudaEventRecord(D.ck_free[x.slot], st)); D.ck_free_set[x.slot] = true; }
+        if (x.vstage < K - 1) {
+          int i = D.rg_of[key];
+          CU(cudaEventRecord(D.rg_free[i], st));
+          D.rg_free_set[i] = true;
+          D.rg_used[i] = false;
+          D.rg_of.erase(key);
+        }
+        break;
+      }
+      case MARIO_OP_SA:
+      case MARIO_OP_SG: {
+        const bool grad = x.op == MARIO_OP_SG;
+        auto& of = grad ? D.sg_of : D.sa_of;
+        const int i = of[key];
+        if (loopback) break;   // the receiver copies out of the held slot
+        Channel& ch = channel(D.d, x.peer, grad ? 1 : 0);
+        cudaEvent_t e = D.event();
+        CU(cudaEventRecord(e, st));
+        CU(cudaStreamWaitEvent(ch.stream, e, 0));
+        NC(ncclSend(send_slot(D, grad, i), msg_bytes, ncclUint8, peer_in_channel(D.d, x.peer), ch.comm, ch.stream));
+        auto& fr = grad ? D.sg_free : D.sa_free;
+        auto& fs = grad ? D.sg_free_set : D.sa_free_set;
+        CU(cudaEventRecord(fr[i], ch.stream));
+        fs[i] = true;
+        (grad ? D.sg_used : D.sa_used)[i] = false;
+        of.erase(key);
+        break;
+      }
+      case MARIO_OP_RA:
+      case MARIO_OP_RG: {
+        const bool grad = x.op == MARIO_OP_RG;
+        T* dst;
+        if (!grad) {
+          dst = D.template at<T>(D.a.ckpt + static_cast<size_t>(x.slot) * D.a.ckpt_stride);
+        } else {
+          int i = acquire(D.rg_used);
+          D.rg_of[key] = i;
+          dst = D.template at<T>(D.a.rg + static_cast<size_t>(i) * D.a.msg_stride);
+        }
+        if (loopback) {
+          Dev<T>& Sd = dev(x.peer);
+          // the sender's part for this micro-batch: find via its held slots
+          int sp = -1;
+          auto& sof = grad ? Sd.sg_of : Sd.sa_of;
+          for (auto& kv : sof) if (kv.first.first == x.micro && sender_part_ok(Sd, kv.first.second, x, grad)) { sp = kv.first.second; break; }
+          if (sp < 0) throw std::runtime_error("loopback: no held send slot for receive");
+          const int i = sof[{x.micro, sp}];
+          CU(cudaMemcpyAsync(dst, send_slot(Sd, grad, i), msg_bytes, cudaMemcpyDeviceToDevice, st));
+          (grad ? Sd.sg_used : Sd.sa_used)[i] = false;
+          sof.erase({x.micro, sp});
+        } else {
+          Channel& ch = channel(x.peer, D.d, grad ? 1 : 0);
+          if (!grad && D.ck_free_set[x.slot]) CU(cudaStreamWaitEvent(ch.stream, D.ck_free[x.slot], 0));
+          if (grad) {
+            int i = D.rg_of[key];
+            if (D.rg_free_set[i]) CU(cudaStreamWaitEvent(ch.stream, D.rg_free[i], 0));
+          }
+          NC(ncclRecv(dst, msg_bytes, ncclUint8, peer_in_channel(D.d, x.peer), ch.comm, ch.stream));
+          cudaEvent_t e = D.event();
+          CU(cudaEventRecord(e, ch.stream));
+          CU(cudaStreamWaitEvent(st, e, 0));   // blocking receive at this list position
+        }
+        break;
+      }
+    }
+  }
+
+  bool sender_part_ok(Dev<T>& Sd, int sp, const mario_instr& x, bool grad) {
+    // the sender's virtual stage must be adjacent to ours in the right direction
+    const int ks = Sd.P->pp.vstage(Sd.d, sp);
+    return grad ? ks == x.vstage + 1 : ks == x.vstage - 1;
+  }
+
+  void timed_begin(Dev<T>& D) {
+    if (!g.timing) return;
+    cudaEvent_t a, b;
+    CU(cudaEventCreate(&a));
+    CU(cudaEventCreate(&b));
+    CU(cudaEventRecord(a, st));
+    D.timed.push_back({a, b});
+  }
+  void timed_end(Dev<T>& D) {
+    if (!g.timing) return;
+    CU(cudaEventRecord(D.timed.back().second, st));
+  }
+
+  Channel& channel(int src, int dst, int kind) {
+    auto it = g.channels.find({src, dst, kind});
+    if (it == g.channels.end()) throw std::runtime_error("missing NCCL channel");
+    return it->second;
+  }
+  static int peer_in_channel(int me, int other) { return me < other ? 1 : 0; }   // 2-rank comm: lo=0, hi=1
+};
+
+// Create per-channel 2-rank communicators for every (src, dst, kind) the plan uses, plus the
+// pair communicators for gradient synchronisation. Collective over all ranks: every rank
+// iterates the same sorted set.
+void ensure_channels(const PlanObj& P) {
+  std::set<std::tuple<int, int, int>> need;
+  std::set<std::pair<int, int>> pairs;
+  for (int d = 0; d < P.pp.S; ++d)
+    for (const mario_instr& x : P.instrs[d]) {
+      if (x.op == MARIO_OP_SA) need.insert({d, x.peer, 0});
+      if (x.op == MARIO_OP_SG) need.insert({d, x.peer, 1});
+    }
+  // replica pairs: any two ranks holding copies of the same parameter
+  std::map<int, std::set<int>> holders;
+  for (int d = 0; d < P.pp.S; ++d)
+    for (int32_t i : P.rank_params[d].idx) holders[i].insert(d);
+  for (auto& kv : holders)
+    for (int a : kv.second)
+      for (int b : kv.second) if (a < b) pairs.insert({a, b});
+  for (auto& c : need) {
+    if (g.created_channels.count(c)) continue;
+    g.created_channels.insert(c);
+    const int lo = std::min(std::get<0>(c), std::get<1>(c)), hi = std::max(std::get<0>(c), std::get<1>(c));
+    const bool member = g.rank == lo || g.rank == hi;
+    ncclComm_t comm = nullptr;
+    NC(ncclCommSplit(g.world_comm, member ? 1 : NCCL_SPLIT_NOCOLOR, g.rank == lo ? 0 : 1, &comm, nullptr));
+    if (member) {
+      Channel ch;
+      ch.comm = comm;
+      CU(cudaStreamCreateWithFlags(&ch.stream, cudaStreamNonBlocking));
+      g.channels[c] = ch;
+    }
+  }
+  for (auto& pr : pairs) {
+    if (g.created_pairs.count(pr)) continue;
+    g.created_pairs.insert(pr);
+    const bool member = g.rank == pr.first || g.rank == pr.second;
+    ncclComm_t comm = nullptr;
+    NC(ncclCommSplit(g.world_comm, member ? 1 : NCCL_SPLIT_NOCOLOR, g.rank == pr.first ? 0 : 1, &comm, nullptr));
+    if (member) g.pair_comms[pr] = comm;
+  }
+}
+
+template <class T>
+mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* tokens, float* loss, void* grads,
+                        void* workspace, cudaStream_t st) {
+  const bool loopback = g.world == 1 && P.pp.S > 1;
+  if (!loopback && P.pp.S != g.world) return set_error(MARIO_ESTATE, "plan stages != world size");
+  Exec<T> E;
+  E.st = st;
+  E.loopback = loopback;
+  const mario_model& m = P.model;
+  const int S = P.pp.S;
+  std::vector<int> my_devs;
+  if (loopback) for (int d = 0; d < S; ++d) my_devs.push_back(d);
+  else my_devs.push_back(g.rank);
+  size_t wofs = 0, wsofs = 0;
+  for (int d : my_devs) {
+    auto D = std::make_unique<Dev<T>>();
+    D->P = &P;
+    D->d = d;
+    const auto& pools = loopback ? P.pools_lb[d] : P.pools_mp[d];
+    D->a = make_arena(P, d, pools);
+    D->ws = static_cast<uint8_t*>(workspace) + wsofs;
+    D->w = static_cast<const float*>(weights) + wofs;
+    D->gr = static_cast<float*>(grads) + wofs;
+    const auto& rp = P.rank_params[d];
+    for (size_t j = 0; j < rp.idx.size(); ++j) D->tensor[{rp.part[j], rp.idx[j]}] = static_cast<int>(j);
+    D->sa_used.assign(std::max(1, pools.send_act), false);
+    D->sg_used.assign(std::max(1, pools.send_grad), false);
+    D->rg_used.assign(std::max(1, pools.recv_grad), false);
+    auto mk = [&](std::vector<cudaEvent_t>& v, std::vector<bool>& set, size_t n) {
+      v.resize(n);
+      set.assign(n, false);
+      for (auto& e : v) CU(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    };
+    mk(D->sa_free, D->sa_free_set, D->sa_used.size());
+    mk(D->sg_free, D->sg_free_set, D->sg_used.size());
+    mk(D->rg_free, D->rg_free_set, D->rg_used.size());
+    mk(D->ck_free, D->ck_free_set, std::max(1, pools.ckpt));
+    if (loopback) {
+      wofs += rp.total;
+      wsofs += align_up(P.workspace_lb[d], 1 << 20);
+    }
+    // iteration prologue: tokens H2D, zero grads and losses, bf16 weight copies
+    const size_t tok_bytes = static_cast<size_t>(P.pp.N) * m.micro_batch * (m.seq_len + 1) * 4;
+    CU(cudaMemcpyAsync(D->ws + D->a.tokens, tokens, tok_bytes, cudaMemcpyHostToDevice, st));
+    CU(cudaMemsetAsync(D->gr, 0, rp.total * 4, st));
+    CU(cudaMemsetAsync(D->ws + D->a.loss, 0, static_cast<size_t>(P.pp.N) * P.pp.parts() * 8, st));
+    if (sizeof(T) == 2)
+      for (size_t j = 0; j < rp.idx.size(); ++j)
+        if (D->a.wcopy[j] != SIZE_MAX)
+          cast_f32_bf16(D->w + rp.off[j], reinterpret_cast<__nv_bfloat16*>(D->ws + D->a.wcopy[j]), rp.cnt[j], st);
+    E.devs.push_back(std::move(D));
+  }
+  if (!loopback && S > 1) ensure_channels(P);
+
+  // walk the plan
+  if (loopback) {
+    for (auto [d, i] : P.loopback_order) E.run_instr(d, P.instrs[d][i]);
+  } else {
+    for (const mario_instr& x : P.instrs[g.rank]) E.run_instr(g.rank, x);
+  }
+
+  // gradient finalization (reading A7): sum every copy of each parameter (tied embeddings,
+  // Chimera replicas) and write the sum back to every copy.
+  std::map<int, std::vector<std::pair<int, int>>> copies;   // global idx -> (dev, packed j)
+  for (int d = 0; d < S; ++d) {
+    const auto& rp = P.rank_params[d];
+    for (size_t j = 0; j < rp.idx.size(); ++j) copies[rp.idx[j]].push_back({d, static_cast<int>(j)});
+  }
+  if (loopback) {
+    for (auto& kv : copies) {
+      if (kv.second.size() < 2) continue;
+      auto ptr = [&](std::pair<int, int> c) { return E.dev(c.first).gr + P.rank_params[c.first].off[c.second]; };
+      const size_t n = P.rank_params[kv.second[0].first].cnt[kv.second[0].second];
+      float* acc = ptr(kv.second[0]);
+      for (size_t c = 1; c < kv.second.size(); ++c) add_f32(acc, ptr(kv.second[c]), n, st);
+      for (size_t c = 1; c < kv.second.size(); ++c) copy_f32(ptr(kv.second[c]), acc, n, st);
+    }
+  } else if (S > 1) {
+    Dev<T>& D = *E.devs[0];
+    // local duplicates first (e.g. Chimera rank 0 holds the tied wte twice)
+    for (auto& kv : copies) {
+      std::vector<int> mine;
+      for (auto& c : kv.second) if (c.first == g.rank) mine.push_back(c.second);
+      for (size_t c = 1; c < mine.size(); ++c)
+        add_f32(D.gr + P.rank_params[g.rank].off[mine[0]], D.gr + P.rank_params[g.rank].off[mine[c]],
+                P.rank_params[g.rank].cnt[mine[0]], st);
+    }
+    // then pairwise all-reduce with every other holder, in global (idx, peer) order
+    NC(ncclGroupStart());
+    for (auto& kv : copies) {
+      std::set<int> ranks;
+      for (auto& c : kv.second) ranks.insert(c.first);
+      if (ranks.size() < 2 || !ranks.count(g.rank)) continue;
+      int j0 = -1;
+      for (auto& c : kv.second) if (c.first == g.rank) { j0 = c.second; break; }
+      float* buf = D.gr + P.rank_params[g.rank].off[j0];
+      const size_t n = P.rank_params[g.rank].cnt[j0];
+      if (ranks.size() == 2) {
+        const int other = *ranks.begin() == g.rank ? *ranks.rbegin() : *ranks.begin();
+        auto pr = std::make_pair(std::min(g.rank, other), std::max(g.rank, other));
+        NC(ncclAllReduce(buf, buf, n, ncclFloat32, ncclSum, g.pair_comms[pr], st));
+      } else {
+        throw std::runtime_error("parameter held by > 2 ranks is not supported in multi-process mode");
+      }
+    }
+    NC(ncclGroupEnd());
+    for (auto& kv : copies) {
+      std::vector<int> mine;
+      for (auto& c : kv.second) if (c.first == g.rank) mine.push_back(c.second);
+      for (size_t c = 1; c < mine.size(); ++c)
+        copy_f32(D.gr + P.rank_params[g.rank].off[mine[c]], D.gr + P.rank_params[g.rank].off[mine[0]],
+                 P.rank_params[g.rank].cnt[mine[0]], st);
+    }
+  }
+
+  // loss (reading A21): per-micro-batch fp64 sums, combined on the host in micro-batch order
+  const int K = P.pp.K();
+  std::vector<double> sums(P.pp.N, 0.0);
+  for (auto& Dp : E.devs) {
+    Dev<T>& D = *Dp;
+    bool has_last = false;
+    for (int p = 0; p < P.pp.parts(); ++p) has_last = has_last || P.pp.vstage(D.d, p) == K - 1;
+    if (!has_last) continue;
+    std::vector<double> h(static_cast<size_t>(P.pp.N));
+    CU(cudaMemcpyAsync(h.data(), D.ws + D.a.loss, P.pp.N * 8, cudaMemcpyDeviceToHost, st));
+    CU(cudaStreamSynchronize(st));
+    for (int i = 0; i < P.pp.N; ++i) sums[i] += h[i];
+  }
+  if (!loopback && S > 1) {
+    // share the last stage(s)' per-micro-batch sums with every rank
+    double* dbuf = reinterpret_cast<double*>(E.devs[0]->ws + E.devs[0]->a.loss);
+    CU(cudaMemcpyAsync(dbuf, sums.data(), P.pp.N * 8, cudaMemcpyHostToDevice, st));
+    NC(ncclAllReduce(dbuf, dbuf, P.pp.N, ncclFloat64, ncclSum, g.world_comm, st));
+    CU(cudaMemcpyAsync(sums.data(), dbuf, P.pp.N * 8, cudaMemcpyDeviceToHost, st));
+  }
+  CU(cudaStreamSynchronize(st));
+  double total = 0.0;
+  for (int i = 0; i < P.pp.N; ++i) total += sums[i];
+  const double ntok = static_cast<double>(P.pp.N) * tokens_per_micro(m);
+  if (loss) *loss = static_cast<float>(total / ntok);
+
+  // timeline export
+  if (g.timing) {
+    g.t_start.assign(S, {});
+    g.t_finish.assign(S, {});
+    cudaEvent_t t0 = nullptr;
+    for (auto& Dp : E.devs) if (!Dp->timed.empty() && !t0) t0 = Dp->timed[0].first;
+    for (auto& Dp : E.devs) {
+      for (auto& pr : Dp->timed) {
+        float a = 0.f, b = 0.f;
+        CU(cudaEventElapsedTime(&a, t0, pr.first));
+        CU(cudaEventElapsedTime(&b, t0, pr.second));
+        g.t_start[Dp->d].push_back(a);
+        g.t_finish[Dp->d].push_back(b);
+      }
+    }
+    for (auto& Dp : E.devs)
+      for (auto& pr : Dp->timed) { cudaEventDestroy(pr.first); cudaEventDestroy(pr.second); }
+  }
+  for (auto& Dp : E.devs) {
+    for (auto v : {&Dp->sa_free, &Dp->sg_free, &Dp->rg_free, &Dp->ck_free, &Dp->ev_pool})
+      for (auto e : *v) cudaEventDestroy(e);
+  }
+  return MARIO_OK;
+}
+
+}  // namespace
+}  // namespace mario
+
+using namespace mario;
+
+extern "C" mario_status mario_nccl_unique_id(void* out128) {
+  if (!out128) return set_error(MARIO_EINVAL, "NULL out");
+  ncclUniqueId id;
+  if (ncclGetUniqueId(&id) != ncclSuccess) return set_error(MARIO_ENCCL, "ncclGetUniqueId failed");
+  static_assert(sizeof(ncclUniqueId) == 128, "nccl id size");
+  memcpy(out128, &id, 128);
+  return MARIO_OK;
+}
+
+extern "C" mario_status mario_init(int32_t rank, int32_t world, int32_t device, const void* nccl_unique_id) {
+  try {
+    if (world < 1 || rank < 0 || rank >= world) return set_error(MARIO_EINVAL, "bad rank/world");
+    if (g.inited) return set_error(MARIO_ESTATE, "already initialised");
+    CU(cudaSetDevice(device));
+    g.rank = rank; g.world = world; g.device = device;
+    if (world > 1) {
+      if (!nccl_unique_id) return set_error(MARIO_EINVAL, "NULL nccl id");
+      ncclUniqueId id;
+      memcpy(&id, nccl_unique_id, 128);
+      NC(ncclCommInitRank(&g.world_comm, world, id, rank));
+    }
+    g.inited = true;
+    g.sticky = false;
+    return MARIO_OK;
+  } catch (const CudaErr& e) {
+    return set_error(MARIO_ECUDA, e.what());
+  } catch (const NcclErr& e) {
+    return set_error(MARIO_ENCCL, e.what());
+  }
+}
+
+extern "C" mario_status mario_run_iter(const struct mario_plan* plan, const void* weights, const int32_t* tokens,
+                                       float* loss, void* grads, void* workspace, void* stream) {
+  if (!g.inited) return set_error(MARIO_ESTATE, "mario_init not called");
+  if (g.sticky) return set_error(MARIO_ECUDA, "context has a sticky error; call mario_finalize");
+  if (!plan || !weights || !tokens || !grads || !workspace) return set_error(MARIO_EINVAL, "NULL argument");
+  try {
+    cudaStream_t st = static_cast<cudaStream_t>(stream);
+    mario_status r = plan->model.dtype == MARIO_BF16
+                         ? run_iter_t<__nv_bfloat16>(*plan, weights, tokens, loss, grads, workspace, st)
+                         : run_iter_t<float>(*plan, weights, tokens, loss, grads, workspace, st);
+    if (r == MARIO_OK) {
+      cudaError_t e = cudaGetLastError();
+      if (e != cudaSuccess) { g.sticky = true; return set_error(MARIO_ECUDA, cudaGetErrorString(e)); }
+    }
+    return r;
+  } catch (const CudaErr& e) {
+    g.sticky = true;
+    return set_error(MARIO_ECUDA, e.what());
+  } catch (const NcclErr& e) {
+    g.sticky = true;
+    return set_error(MARIO_ENCCL, e.what());
+  } catch (const std::exception& e) {
+    return set_error(MARIO_EINVAL, e.what());
+  }
+}
+
+extern "C" mario_status mario_set_timing(int32_t enable) {
+  g.timing = enable != 0;
+  return MARIO_OK;
+}
+
+extern "C" mario_status mario_last_timeline(int32_t device, const double** start_ms, const double** finish_ms,
+                                            int32_t* n) {
+  if (device < 0 || device >= static_cast<int32_t>(g.t_start.size()) || !start_ms || !finish_ms || !n)
+    return set_error(MARIO_EINVAL, "no timeline for device");
+  *start_ms = g.t_start[device].data();
+  *finish_ms = g.t_finish[device].data();
+  *n = static_cast<int32_t>(g.t_start[device].size());
+  return MARIO_OK;
+}
+
+extern "C" mario_status mario_finalize(void) {
+  for (auto& kv : g.channels) {
+    if (kv.second.comm) ncclCommDestroy(kv.second.comm);
+    if (kv.second.stream) cudaStreamDestroy(kv.second.stream);
+  }
+  g.channels.clear();
+  for (auto& kv : g.pair_comms) if (kv.second) ncclCommDestroy(kv.second);
+  g.pair_comms.clear();
+  g.created_channels.clear();
+  g.created_pairs.clear();
+  if (g.world_comm) ncclCommDestroy(g.world_comm);
+  g.world_comm = nullptr;
+  g.inited = false;
+  g.sticky = false;
+  return MARIO_OK;
+}

@@ -64,17 +64,24 @@ size_t cfw_work_bytes(const mario_model& m, int k, int K) {
   return b;
 }
 
-size_t bw_scratch_bytes(const mario_model& m) {
+BwScratch bw_scratch_layout(const mario_model& m) {
   const size_t T = tokens_per_micro(m), E = elt_size(m), h = m.hidden, f = m.ffn_hidden;
-  // dH ping-pong (2 x [T,h]) + dX [T,h] + dQKV [T,3h] + dO [T,h] + dZ [T, 2f] + dP row sums fp32 [heads,T]
-  size_t b = 0;
-  b += align_up(T * h * E) * 3;
-  b += align_up(T * 3 * h * E);
-  b += align_up(T * h * E);
-  b += align_up(T * 2 * f * E);
-  b += align_up(static_cast<size_t>(m.n_heads) * T * 4);
+  BwScratch b{};
+  size_t o = 0;
+  auto take = [&](size_t bytes) { size_t r = o; o = align_up(o + bytes); return r; };
+  for (int i = 0; i < 3; ++i) b.dH[i] = take(T * h * E);
+  b.dA = take(T * h * E);
+  b.dQKV = take(T * 3 * h * E);
+  b.dO = take(T * h * E);
+  b.dZ = take(T * 2 * f * E);
+  b.dM = take(T * f * E);
+  b.Dsc = take(static_cast<size_t>(m.n_heads) * T * 4);
+  b.sort = take(T * 8 * 2);
+  b.bytes = o;
   return b;
 }
+
+size_t bw_scratch_bytes(const mario_model& m) { return bw_scratch_layout(m).bytes; }
 
 size_t logits_bytes(const mario_model& m) { return align_up(tokens_per_micro(m) * m.vocab * 4); }
 

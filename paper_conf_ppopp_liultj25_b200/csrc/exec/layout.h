@@ -32,6 +32,12 @@ size_t tokens_per_micro(const mario_model& m);
 size_t stage_input_bytes(const mario_model& m);                  // [T, h]
 size_t act_set_bytes(const mario_model& m, int k, int K);        // lps layers (+ head)
 size_t cfw_work_bytes(const mario_model& m, int k, int K);       // transient CFW scratch
+// Backward scratch (shared by every BW of the rank): rotating dH buffers and per-layer grads.
+struct BwScratch {
+  size_t dH[3], dA, dQKV, dO, dZ, dM, Dsc, sort;
+  size_t bytes;
+};
+BwScratch bw_scratch_layout(const mario_model& m);
 size_t bw_scratch_bytes(const mario_model& m);
 size_t logits_bytes(const mario_model& m);                      // fp32 [T, V]
 size_t weight_copy_bytes(const mario_model& m, const std::vector<int32_t>& param_idx);

@@ -1,0 +1,567 @@
+// K5-K15 — norms, attention, RoPE, SwiGLU, softmax-CE, embedding, reductions.
+// Formulas: SURVEY §8(c) c1 (readings A1/A2), same definitions as oracle/model.py but an
+// independent implementation (no shared code).
+#include <cfloat>
+#include <cstdint>
+
+#include "layers.h"
+
+namespace mario {
+namespace {
+
+__device__ __forceinline__ float ldf(const float* p) { return *p; }
+__device__ __forceinline__ float ldf(const __nv_bfloat16* p) { return __bfloat162float(*p); }
+__device__ __forceinline__ void stf(float* p, float v) { *p = v; }
+__device__ __forceinline__ void stf(__nv_bfloat16* p, float v) { *p = __float2bfloat16_rn(v); }
+
+__device__ __forceinline__ float warp_sum(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+__device__ __forceinline__ float warp_max(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+
+inline int cdiv(long a, long b) { return static_cast<int>((a + b - 1) / b); }
+
+// ------------------------------------------------------------------ embedding
+template <class T>
+__global__ void embed_fwd_k(const int32_t* tok, int ld_tok, int B, int s, const T* wte, const T* wpe, T* H, int h) {
+  const long n = static_cast<long>(B) * s * h;
+  for (long i = blockIdx.x * static_cast<long>(blockDim.x) + threadIdx.x; i < n; i += static_cast<long>(gridDim.x) * blockDim.x) {
+    const long r = i / h;
+    const int c = static_cast<int>(i % h);
+    const int b = static_cast<int>(r / s), t = static_cast<int>(r % s);
+    const int x = tok[static_cast<long>(b) * ld_tok + t];
+    float v = ldf(wte + static_cast<long>(x) * h + c);
+    if (wpe) v += ldf(wpe + static_cast<long>(t) * h + c);
+    stf(H + i, v);
+  }
+}
+
+// one block bitonic sort of keys (token * T + index) in shared memory
+__global__ void embed_sort_k(const int32_t* tok, int ld_tok, int B, int s, long long* keys_out, int npow2) {
+  extern __shared__ long long sk[];
+  const int T = B * s;
+  for (int i = threadIdx.x; i < npow2; i += blockDim.x) {
+    if (i < T) {
+      const int b = i / s, t = i % s;
+      sk[i] = static_cast<long long>(tok[static_cast<long>(b) * ld_tok + t]) * T + i;
+    } else {
+      sk[i] = LLONG_MAX;
+    }
+  }
+  __syncthreads();
+  for (int k = 2; k <= npow2; k <<= 1) {
+    for (int j = k >> 1; j > 0; j >>= 1) {
+      for (int i = threadIdx.x; i < npow2; i += blockDim.x) {
+        const int ixj = i ^ j;
+        if (ixj > i) {
+          const bool up = (i & k) == 0;
+          const long long a = sk[i], c = sk[ixj];
+          if ((a > c) == up) { sk[i] = c; sk[ixj] = a; }
+        }
+      }
+      __syncthreads();
+    }
+  }
+  for (int i = threadIdx.x; i < T; i += blockDim.x) keys_out[i] = sk[i];
+}
+
+template <class T>
+__global__ void embed_segsum_k(const long long* keys, int Ttok, const T* dH, int h, float* dwte) {
+  const int warp = (blockIdx.x * blockDim.x + threadIdx.x) / 32, lane = threadIdx.x % 32;
+  if (warp >= Ttok) return;
+  const long long v = keys[warp] / Ttok;
+  if (warp > 0 && keys[warp - 1] / Ttok == v) return;   // not a segment start
+  for (int c = lane; c < h; c += 32) {
+    float acc = 0.f;
+    for (int j = warp; j < Ttok && keys[j] / Ttok == v; ++j) acc += ldf(dH + (keys[j] % Ttok) * h + c);
+    dwte[v * h + c] += acc;
+  }
+}
+
+template <class T>
+__global__ void embed_pos_bwd_k(const T* dH, int B, int s, int h, float* dwpe) {
+  const long n = static_cast<long>(s) * h;
+  for (long i = blockIdx.x * static_cast<long>(blockDim.x) + threadIdx.x; i < n; i += static_cast<long>(gridDim.x) * blockDim.x) {
+    const long t = i / h;
+    const int c = static_cast<int>(i % h);
+    float acc = 0.f;
+    for (int b = 0; b < B; ++b) acc += ldf(dH + (static_cast<long>(b) * s + t) * h + c);
+    dwpe[i] += acc;
+  }
+}
+
+// ---------------------------------------------------------------------- norms
+template <class T, bool RMS>
+__global__ void norm_fwd_k(const T* x, const float* g, const float* b, T* y, float* stats, int rows, int n, float eps) {
+  const int row = blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32, lane = threadIdx.x % 32;
+  if (row >= rows) return;
+  const T* xr = x + static_cast<long>(row) * n;
+  float mean = 0.f;
+  if (!RMS) {
+    float s = 0.f;
+    for (int c = lane; c < n; c += 32) s += ldf(xr + c);
+    mean = warp_sum(s) / n;
+  }
+  float v = 0.f;
+  for (int c = lane; c < n; c += 32) { const float d = ldf(xr + c) - mean; v += d * d; }
+  const float rstd = rsqrtf(warp_sum(v) / n + eps);
+  T* yr = y + static_cast<long>(row) * n;
+  for (int c = lane; c < n; c += 32) {
+    float o = (ldf(xr + c) - mean) * rstd * g[c];
+    if (!RMS) o += b[c];
+    stf(yr + c, o);
+  }
+  if (lane == 0) { stats[2 * row] = mean; stats[2 * row + 1] = rstd; }
+}
+
+template <class T>
+__global__ void norm_bwd_dx_k(const T* dy, const T* x, const float* stats, const float* g, const T* dres, T* dx,
+                              int rows, int n, int rms) {
+  const int row = blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32, lane = threadIdx.x % 32;
+  if (row >= rows) return;
+  const long o = static_cast<long>(row) * n;
+  const float mean = stats[2 * row], rstd = stats[2 * row + 1];
+  float sg = 0.f, sgx = 0.f;
+  for (int c = lane; c < n; c += 32) {
+    const float gp = ldf(dy + o + c) * g[c];
+    const float xh = (ldf(x + o + c) - mean) * rstd;
+    sg += gp;
+    sgx += gp * xh;
+  }
+  sg = warp_sum(sg) / n;
+  sgx = warp_sum(sgx) / n;
+  if (rms) sg = 0.f;
+  for (int c = lane; c < n; c += 32) {
+    const float gp = ldf(dy + o + c) * g[c];
+    const float xh = (ldf(x + o + c) - mean) * rstd;
+    float d = (gp - sg - xh * sgx) * rstd;
+    if (dres) d += ldf(dres + o + c);
+    stf(dx + o + c, d);
+  }
+}
+
+template <class T>
+__global__ void colsum_partial_k(const T* a, const T* x, const float* stats, int rows, int n, int lda, int mode,
+                                 float* partial, int nblk) {
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= n) return;
+  const int blk = blockIdx.y;
+  const int r0 = static_cast<int>(static_cast<long>(rows) * blk / nblk);
+  const int r1 = static_cast<int>(static_cast<long>(rows) * (blk + 1) / nblk);
+  float s0 = 0.f, s1 = 0.f;
+  for (int r = r0; r < r1; ++r) {
+    const float dy = ldf(a + static_cast<long>(r) * lda + c);
+    if (mode == 0) { s0 += dy; continue; }
+    const float xh = (ldf(x + static_cast<long>(r) * n + c) - stats[2 * r]) * stats[2 * r + 1];
+    s0 += dy * xh;
+    s1 += dy;
+  }
+  partial[static_cast<long>(blk) * n + c] = s0;
+  if (mode == 1) partial[static_cast<long>(nblk + blk) * n + c] = s1;
+}
+
+__global__ void colsum_final_k(const float* partial, int nblk, int n, int mode, float* out0, float* out1) {
+  const int c = blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= n) return;
+  float s0 = 0.f, s1 = 0.f;
+  for (int b = 0; b < nblk; ++b) {
+    s0 += partial[static_cast<long>(b) * n + c];
+    if (mode == 1) s1 += partial[static_cast<long>(nblk + b) * n + c];
+  }
+  out0[c] += s0;
+  if (mode == 1) out1[c] += s1;
+}
+
+// ------------------------------------------------------------------ attention
+// One warp per (query row, head); keys in chunks of 32 (one per lane); online softmax.
+template <class T>
+__global__ void attn_fwd_k(const T* qkv, T* O, float* lse, int B, int s, int nh, int dh) {
+  __shared__ float qs[8][128];
+  const int w = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const long gw = static_cast<long>(blockIdx.x) * 8 + w;
+  const long Ttok = static_cast<long>(B) * s;
+  if (gw >= Ttok * nh) return;
+  const int head = static_cast<int>(gw % nh);
+  const long r = gw / nh;
+  const int t = static_cast<int>(r % s);
+  const long base = r - t;  // first row of this sample
+  const int h = nh * dh, ld = 3 * h;
+  const float scale = rsqrtf(static_cast<float>(dh));
+  for (int d = lane; d < dh; d += 32) qs[w][d] = ldf(qkv + r * ld + head * dh + d);
+  __syncwarp();
+  float m = -INFINITY, l = 0.f, o[4] = {0.f, 0.f, 0.f, 0.f};
+  for (int c0 = 0; c0 <= t; c0 += 32) {
+    const int u = c0 + lane;
+    float sc = -INFINITY;
+    if (u <= t) {
+      const T* kr = qkv + (base + u) * ld + h + head * dh;
+      float acc = 0.f;
+      for (int d = 0; d < dh; ++d) acc += qs[w][d] * ldf(kr + d);
+      sc = acc * scale;
+    }
+    const float mn = fmaxf(m, warp_max(sc));
+    const float corr = __expf(m - mn);
+    const float p = (u <= t) ? __expf(sc - mn) : 0.f;
+    l = l * corr + warp_sum(p);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) o[i] *= corr;
+    const int nv = min(32, t - c0 + 1);
+    for (int j = 0; j < nv; ++j) {
+      const float pj = __shfl_sync(0xffffffffu, p, j);
+      const T* vr = qkv + (base + c0 + j) * ld + 2 * h + head * dh;
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const int d = lane + 32 * i;
+        if (d < dh) o[i] += pj * ldf(vr + d);
+      }
+    }
+    m = mn;
+  }
+  const float inv = 1.f / l;
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const int d = lane + 32 * i;
+    if (d < dh) stf(O + r * h + head * dh + d, o[i] * inv);
+  }
+  if (lane == 0) lse[static_cast<long>(head) * Ttok + r] = m + logf(l);
+}
+
+template <class T>
+__global__ void attn_bwd_dq_k(const T* qkv, const T* O, const T* dO, const float* lse, T* dqkv, float* Dsc, int B,
+                              int s, int nh, int dh) {
+  __shared__ float qs[8][128], gs[8][128];
+  const int w = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const long gw = static_cast<long>(blockIdx.x) * 8 + w;
+  const long Ttok = static_cast<long>(B) * s;
+  if (gw >= Ttok * nh) return;
+  const int head = static_cast<int>(gw % nh);
+  const long r = gw / nh;
+  const int t = static_cast<int>(r % s);
+  const long base = r - t;
+  const int h = nh * dh, ld = 3 * h;
+  const float scale = rsqrtf(static_cast<float>(dh));
+  float Dp = 0.f;
+  for (int d = lane; d < dh; d += 32) {
+    qs[w][d] = ldf(qkv + r * ld + head * dh + d);
+    const float g = ldf(dO + r * h + head * dh + d);
+    gs[w][d] = g;
+    Dp += g * ldf(O + r * h + head * dh + d);
+  }
+  const float D = warp_sum(Dp);
+  __syncwarp();
+  const float L = lse[static_cast<long>(head) * Ttok + r];
+  float dq[4] = {0.f, 0.f, 0.f, 0.f};
+  for (int c0 = 0; c0 <= t; c0 += 32) {
+    const int u = c0 + lane;
+    float ds = 0.f;
+    if (u <= t) {
+      const T* kr = qkv + (base + u) * ld + h + head * dh;
+      const T* vr = qkv + (base + u) * ld + 2 * h + head * dh;
+      float sc = 0.f, dp = 0.f;
+      for (int d = 0; d < dh; ++d) { sc += qs[w][d] * ldf(kr + d); dp += gs[w][d] * ldf(vr + d); }
+      const float p = __expf(sc * scale - L);
+      ds = p * (dp - D);
+    }
+    const int nv = min(32, t - c0 + 1);
+    for (int j = 0; j < nv; ++j) {
+      const float dsj = __shfl_sync(0xffffffffu, ds, j);
+      const T* kr = qkv + (base + c0 + j) * ld + h + head * dh;
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const int d = lane + 32 * i;
+        if (d < dh) dq[i] += dsj * ldf(kr + d);
+      }
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const int d = lane + 32 * i;
+    if (d < dh) stf(dqkv + r * ld + head * dh + d, dq[i] * scale);
+  }
+  if (lane == 0) Dsc[static_cast<long>(head) * Ttok + r] = D;
+}
+
+template <class T>
+__global__ void attn_bwd_dkdv_k(const T* qkv, const T* dO, const float* lse, const float* Dsc, T* dqkv, int B, int s,
+                                int nh, int dh) {
+  __shared__ float ks[8][128], vs[8][128];
+  const int w = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const long gw = static_cast<long>(blockIdx.x) * 8 + w;
+  const long Ttok = static_cast<long>(B) * s;
+  if (gw >= Ttok * nh) return;
+  const int head = static_cast<int>(gw % nh);
+  const long r = gw / nh;  // key row
+  const int u = static_cast<int>(r % s);
+  const long base = r - u;
+  const int h = nh * dh, ld = 3 * h;
+  const float scale = rsqrtf(static_cast<float>(dh));
+  for (int d = lane; d < dh; d += 32) {
+    ks[w][d] = ldf(qkv + r * ld + h + head * dh + d);
+    vs[w][d] = ldf(qkv + r * ld + 2 * h + head * dh + d);
+  }
+  __syncwarp();
+  float dk[4] = {0.f, 0.f, 0.f, 0.f}, dv[4] = {0.f, 0.f, 0.f, 0.f};
+  for (int c0 = u; c0 < s; c0 += 32) {
+    const int t = c0 + lane;
+    float p = 0.f, ds = 0.f;
+    if (t < s) {
+      const long rt = base + t;
+      const T* qr = qkv + rt * ld + head * dh;
+      const T* gr = dO + rt * h + head * dh;
+      float sc = 0.f, dp = 0.f;
+      for (int d = 0; d < dh; ++d) { sc += ldf(qr + d) * ks[w][d]; dp += ldf(gr + d) * vs[w][d]; }
+      p = __expf(sc * scale - lse[static_cast<long>(head) * Ttok + rt]);
+      ds = p * (dp - Dsc[static_cast<long>(head) * Ttok + rt]);
+    }
+    const int nv = min(32, s - c0);
+    for (int j = 0; j < nv; ++j) {
+      const float pj = __shfl_sync(0xffffffffu, p, j);
+      const float dsj = __shfl_sync(0xffffffffu, ds, j);
+      const long rt = base + c0 + j;
+#pragma unroll
+      for (int i = 0; i < 4; ++i) {
+        const int d = lane + 32 * i;
+        if (d < dh) {
+          dv[i] += pj * ldf(dO + rt * h + head * dh + d);
+          dk[i] += dsj * ldf(qkv + rt * ld + head * dh + d);
+        }
+      }
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < 4; ++i) {
+    const int d = lane + 32 * i;
+    if (d < dh) {
+      stf(dqkv + r * ld + h + head * dh + d, dk[i] * scale);
+      stf(dqkv + r * ld + 2 * h + head * dh + d, dv[i]);
+    }
+  }
+}
+
+// ----------------------------------------------------------------------- RoPE
+template <class T>
+__global__ void rope_k(T* qkv, int B, int s, int nh, int dh, float base, int inverse) {
+  const int half = dh / 2;
+  const long n = static_cast<long>(B) * s * nh * half;
+  const int h = nh * dh;
+  for (long i = blockIdx.x * static_cast<long>(blockDim.x) + threadIdx.x; i < n; i += static_cast<long>(gridDim.x) * blockDim.x) {
+    const int j = static_cast<int>(i % half);
+    const long rh = i / half;
+    const int head = static_cast<int>(rh % nh);
+    const long r = rh / nh;
+    const int t = static_cast<int>(r % s);
+    const double theta = pow(static_cast<double>(base), -2.0 * j / dh);
+    double sn, cs;
+    sincos(t * theta, &sn, &cs);
+    const float c = static_cast<float>(cs), sgn = inverse ? -1.f : 1.f;
+    const float si = sgn * static_cast<float>(sn);
+    for (int part = 0; part < 2; ++part) {  // q, then k
+      T* p = qkv + r * 3 * h + part * h + head * dh;
+      const float x1 = ldf(p + j), x2 = ldf(p + j + half);
+      stf(p + j, x1 * c - x2 * si);
+      stf(p + j + half, x1 * si + x2 * c);
+    }
+  }
+}
+
+// --------------------------------------------------------------------- SwiGLU
+template <class T>
+__global__ void swiglu_fwd_k(const T* GU, T* M, int rows, int f) {
+  const long n = static_cast<long>(rows) * f;
+  for (long i = blockIdx.x * static_cast<long>(blockDim.x) + threadIdx.x; i < n; i += static_cast<long>(gridDim.x) * blockDim.x) {
+    const long r = i / f;
+    const int j = static_cast<int>(i % f);
+    const float g = ldf(GU + r * 2 * f + j), u = ldf(GU + r * 2 * f + f + j);
+    stf(M + i, g / (1.f + __expf(-g)) * u);
+  }
+}
+template <class T>
+__global__ void swiglu_bwd_k(const T* GU, const T* dM, T* dGU, int rows, int f) {
+  const long n = static_cast<long>(rows) * f;
+  for (long i = blockIdx.x * static_cast<long>(blockDim.x) + threadIdx.x; i < n; i += static_cast<long>(gridDim.x) * blockDim.x) {
+    const long r = i / f;
+    const int j = static_cast<int>(i % f);
+    const float g = ldf(GU + r * 2 * f + j), u = ldf(GU + r * 2 * f + f + j), dm = ldf(dM + i);
+    const float sg = 1.f / (1.f + __expf(-g));
+    stf(dGU + r * 2 * f + j, dm * u * sg * (1.f + g * (1.f - sg)));
+    stf(dGU + r * 2 * f + f + j, dm * g * sg);
+  }
+}
+
+// ---------------------------------------------------------------- softmax-CE
+template <class T>
+__global__ void softmax_ce_k(const float* logits, const int32_t* tok, int ld_tok, int s, int V, float inv_ntok,
+                             T* dlogits, float* row_loss) {
+  __shared__ float sm[32], sl[32];
+  const long r = blockIdx.x;
+  const float* z = logits + r * V;
+  float m = -INFINITY, l = 0.f;
+  for (int c = threadIdx.x; c < V; c += blockDim.x) {
+    const float v = z[c];
+    if (v > m) { l = l * __expf(m - v) + 1.f; m = v; } else { l += __expf(v - m); }
+  }
+  // combine (m, l) pairs: warp then block, fixed order
+  for (int o = 16; o > 0; o >>= 1) {
+    const float m2 = __shfl_xor_sync(0xffffffffu, m, o), l2 = __shfl_xor_sync(0xffffffffu, l, o);
+    const float mn = fmaxf(m, m2);
+    l = (mn == -INFINITY) ? 0.f : l * __expf(m - mn) + l2 * __expf(m2 - mn);
+    m = mn;
+  }
+  const int w = threadIdx.x / 32, lane = threadIdx.x % 32, nw = blockDim.x / 32;
+  if (lane == 0) { sm[w] = m; sl[w] = l; }
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    float M = sm[0], Ls = sl[0];
+    for (int i = 1; i < nw; ++i) {
+      const float mn = fmaxf(M, sm[i]);
+      Ls = Ls * __expf(M - mn) + sl[i] * __expf(sm[i] - mn);
+      M = mn;
+    }
+    sm[0] = M; sl[0] = Ls;
+  }
+  __syncthreads();
+  const float lse = sm[0] + logf(sl[0]);
+  const int b = static_cast<int>(r / s), t = static_cast<int>(r % s);
+  const int y = tok[static_cast<long>(b) * ld_tok + t + 1];
+  for (int c = threadIdx.x; c < V; c += blockDim.x) {
+    const float p = __expf(z[c] - lse);
+    stf(dlogits + r * V + c, (p - (c == y ? 1.f : 0.f)) * inv_ntok);
+  }
+  if (threadIdx.x == 0) row_loss[r] = lse - z[y];
+}
+
+__global__ void loss_reduce_k(const float* row_loss, int rows, double* out) {
+  __shared__ double sh[1024];
+  double acc = 0.0;
+  for (int i = threadIdx.x; i < rows; i += blockDim.x) acc += row_loss[i];
+  sh[threadIdx.x] = acc;
+  __syncthreads();
+  for (int o = blockDim.x / 2; o > 0; o >>= 1) {
+    if (threadIdx.x < o) sh[threadIdx.x] += sh[threadIdx.x + o];
+    __syncthreads();
+  }
+  if (threadIdx.x == 0) out[0] = sh[0];
+}
+
+__global__ void cast_k(const float* x, __nv_bfloat16* y, size_t n) {
+  for (size_t i = blockIdx.x * static_cast<size_t>(blockDim.x) + threadIdx.x; i < n; i += static_cast<size_t>(gridDim.x) * blockDim.x)
+    y[i] = __float2bfloat16_rn(x[i]);
+}
+__global__ void add_k(float* a, const float* b, size_t n) {
+  for (size_t i = blockIdx.x * static_cast<size_t>(blockDim.x) + threadIdx.x; i < n; i += static_cast<size_t>(gridDim.x) * blockDim.x)
+    a[i] += b[i];
+}
+__global__ void copy_k(float* a, const float* b, size_t n) {
+  for (size_t i = blockIdx.x * static_cast<size_t>(blockDim.x) + threadIdx.x; i < n; i += static_cast<size_t>(gridDim.x) * blockDim.x)
+    a[i] = b[i];
+}
+
+int grid_for(long n, int threads = 256) { long g = (n + threads - 1) / threads; return static_cast<int>(g < 148 * 16 ? (g < 1 ? 1 : g) : 148 * 16); }
+
+}  // namespace
+
+template <class T>
+void embed_fwd(const int32_t* tok, int ld_tok, int B, int s, const T* wte, const T* wpe, T* H, int h, cudaStream_t st) {
+  embed_fwd_k<T><<<grid_for(static_cast<long>(B) * s * h), 256, 0, st>>>(tok, ld_tok, B, s, wte, wpe, H, h);
+}
+
+template <class T>
+void embed_bwd(const int32_t* tok, int ld_tok, int B, int s, const T* dH, int h, float* dwte, float* dwpe,
+               void* scratch, cudaStream_t st) {
+  const int Ttok = B * s;
+  int np2 = 1;
+  while (np2 < Ttok) np2 <<= 1;
+  long long* keys = static_cast<long long*>(scratch);
+  const size_t smem = static_cast<size_t>(np2) * sizeof(long long);
+  static bool attr = false;
+  if (!attr) { cudaFuncSetAttribute(embed_sort_k, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024); attr = true; }
+  embed_sort_k<<<1, 1024, smem, st>>>(tok, ld_tok, B, s, keys, np2);
+  embed_segsum_k<T><<<cdiv(static_cast<long>(Ttok) * 32, 256), 256, 0, st>>>(keys, Ttok, dH, h, dwte);
+  if (dwpe) embed_pos_bwd_k<T><<<grid_for(static_cast<long>(s) * h), 256, 0, st>>>(dH, B, s, h, dwpe);
+}
+
+template <class T>
+void layernorm_fwd(const T* x, const float* g, const float* b, T* y, float* stats, int rows, int n, float eps, cudaStream_t st) {
+  norm_fwd_k<T, false><<<cdiv(rows, 8), 256, 0, st>>>(x, g, b, y, stats, rows, n, eps);
+}
+template <class T>
+void rmsnorm_fwd(const T* x, const float* g, T* y, float* stats, int rows, int n, float eps, cudaStream_t st) {
+  norm_fwd_k<T, true><<<cdiv(rows, 8), 256, 0, st>>>(x, g, nullptr, y, stats, rows, n, eps);
+}
+template <class T>
+void norm_bwd_dx(const T* dy, const T* x, const float* stats, const float* g, const T* dres, T* dx, int rows, int n,
+                 int rms, cudaStream_t st) {
+  norm_bwd_dx_k<T><<<cdiv(rows, 8), 256, 0, st>>>(dy, x, stats, g, dres, dx, rows, n, rms);
+}
+template <class T>
+void colsum(const T* a, const T* x, const float* stats, int rows, int n, int lda, int mode, float* out0, float* out1,
+            float* partial, cudaStream_t st) {
+  int nblk = rows < 128 ? rows : 128;
+  if (nblk < 1) return;
+  dim3 grid(cdiv(n, 256), nblk);
+  colsum_partial_k<T><<<grid, 256, 0, st>>>(a, x, stats, rows, n, lda, mode == 2 ? 1 : mode, partial, nblk);
+  colsum_final_k<<<cdiv(n, 256), 256, 0, st>>>(partial, nblk, n, mode == 2 ? 0 : mode, out0, out1);
+}
+
+template <class T>
+void attn_fwd(const T* qkv, T* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st) {
+  attn_fwd_k<T><<<cdiv(static_cast<long>(B) * s * nh, 8), 256, 0, st>>>(qkv, O, lse, B, s, nh, dh);
+}
+template <class T>
+void attn_bwd(const T* qkv, const T* O, const T* dO, const float* lse, T* dqkv, float* Dsc, int B, int s, int nh,
+              int dh, cudaStream_t st) {
+  const int grid = cdiv(static_cast<long>(B) * s * nh, 8);
+  attn_bwd_dq_k<T><<<grid, 256, 0, st>>>(qkv, O, dO, lse, dqkv, Dsc, B, s, nh, dh);
+  attn_bwd_dkdv_k<T><<<grid, 256, 0, st>>>(qkv, dO, lse, Dsc, dqkv, B, s, nh, dh);
+}
+
+template <class T>
+void rope(T* qkv, int B, int s, int nh, int dh, float base, int inverse, cudaStream_t st) {
+  rope_k<T><<<grid_for(static_cast<long>(B) * s * nh * (dh / 2)), 256, 0, st>>>(qkv, B, s, nh, dh, base, inverse);
+}
+template <class T>
+void swiglu_fwd(const T* GU, T* M, int rows, int f, cudaStream_t st) {
+  swiglu_fwd_k<T><<<grid_for(static_cast<long>(rows) * f), 256, 0, st>>>(GU, M, rows, f);
+}
+template <class T>
+void swiglu_bwd(const T* GU, const T* dM, T* dGU, int rows, int f, cudaStream_t st) {
+  swiglu_bwd_k<T><<<grid_for(static_cast<long>(rows) * f), 256, 0, st>>>(GU, dM, dGU, rows, f);
+}
+template <class T>
+void softmax_ce(const float* logits, const int32_t* tok, int ld_tok, int s, int rows, int V, float inv_ntok,
+                T* dlogits, float* row_loss, cudaStream_t st) {
+  softmax_ce_k<T><<<rows, 512, 0, st>>>(logits, tok, ld_tok, s, V, inv_ntok, dlogits, row_loss);
+}
+void loss_reduce(const float* row_loss, int rows, double* out, cudaStream_t st) {
+  loss_reduce_k<<<1, 1024, 0, st>>>(row_loss, rows, out);
+}
+void cast_f32_bf16(const float* x, __nv_bfloat16* y, size_t n, cudaStream_t st) {
+  cast_k<<<grid_for(static_cast<long>(n)), 256, 0, st>>>(x, y, n);
+}
+void add_f32(float* a, const float* b, size_t n, cudaStream_t st) { add_k<<<grid_for(static_cast<long>(n)), 256, 0, st>>>(a, b, n); }
+void copy_f32(float* a, const float* b, size_t n, cudaStream_t st) { copy_k<<<grid_for(static_cast<long>(n)), 256, 0, st>>>(a, b, n); }
+
+#define INST(T)                                                                                                     \
+  template void embed_fwd<T>(const int32_t*, int, int, int, const T*, const T*, T*, int, cudaStream_t);              \
+  template void embed_bwd<T>(const int32_t*, int, int, int, const T*, int, float*, float*, void*, cudaStream_t);     \
+  template void layernorm_fwd<T>(const T*, const float*, const float*, T*, float*, int, int, float, cudaStream_t);  \
+  template void rmsnorm_fwd<T>(const T*, const float*, T*, float*, int, int, float, cudaStream_t);                   \
+  template void norm_bwd_dx<T>(const T*, const T*, const float*, const float*, const T*, T*, int, int, int,          \
+                               cudaStream_t);                                                                      \
+  template void colsum<T>(const T*, const T*, const float*, int, int, int, int, float*, float*, float*, cudaStream_t); \
+  template void attn_fwd<T>(const T*, T*, float*, int, int, int, int, cudaStream_t);                                 \
+  template void attn_bwd<T>(const T*, const T*, const T*, const float*, T*, float*, int, int, int, int, cudaStream_t); \
+  template void rope<T>(T*, int, int, int, int, float, int, cudaStream_t);                                           \
+  template void swiglu_fwd<T>(const T*, T*, int, int, cudaStream_t);                                                 \
+  template void swiglu_bwd<T>(const T*, const T*, T*, int, int, cudaStream_t);                                       \
+  template void softmax_ce<T>(const float*, const int32_t*, int, int, int, int, float, T*, float*, cudaStream_t);
+INST(float)
+INST(__nv_bfloat16)
+
+}  // namespace mario

@@ -1,0 +1,55 @@
+// Bandwidth-bound layer kernels, templated on the storage type
+// T in {float, __nv_bfloat16}; all arithmetic in fp32. Every reduction is deterministic
+// (fixed-order, no float atomics) so a Mario plan reproduces its base plan bit for bit.
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+#include <cuda_bf16.h>
+
+namespace mario {
+
+template <class T> void embed_fwd(const int32_t* tok, int ld_tok, int B, int s, const T* wte, const T* wpe,
+                                  T* H, int h, cudaStream_t st);
+// dwte[v] += sum_{tokens x=v} dH  (deterministic: per-micro-batch sort + segmented sum);
+// dwpe[t] += sum_b dH[b,t] (if dwpe). scratch: >= 3*T int64 + 2*T int32 bytes.
+template <class T> void embed_bwd(const int32_t* tok, int ld_tok, int B, int s, const T* dH, int h, float* dwte,
+                                  float* dwpe, void* scratch, cudaStream_t st);
+
+// LayerNorm / RMSNorm over rows of width n. stats = [rows][2] (mean, rstd) fp32.
+template <class T> void layernorm_fwd(const T* x, const float* g, const float* b, T* y, float* stats, int rows,
+                                      int n, float eps, cudaStream_t st);
+template <class T> void rmsnorm_fwd(const T* x, const float* g, T* y, float* stats, int rows, int n, float eps,
+                                    cudaStream_t st);
+// dx = LN'(dy) (+ dres); rms = 1 selects RMSNorm.
+template <class T> void norm_bwd_dx(const T* dy, const T* x, const float* stats, const float* g, const T* dres,
+                                    T* dx, int rows, int n, int rms, cudaStream_t st);
+// Column reductions into fp32 grads (+=): mode 0: out0 += sum_r a[r,c]
+// mode 1 (LN): out0 += sum dy*xhat, out1 += sum dy; mode 2 (RMS): out0 += sum dy*xhat.
+template <class T> void colsum(const T* a, const T* x, const float* stats, int rows, int n, int lda, int mode,
+                               float* out0, float* out1, float* partial, cudaStream_t st);
+
+// Causal attention over QKV [T, 3h] (q | k | v), heads of dh; O [T, h]; lse [nh][T] fp32.
+template <class T> void attn_fwd(const T* qkv, T* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st);
+// dqkv [T, 3h] from dO; Dscratch [nh][T] fp32.
+template <class T> void attn_bwd(const T* qkv, const T* O, const T* dO, const float* lse, T* dqkv, float* Dscratch,
+                                 int B, int s, int nh, int dh, cudaStream_t st);
+
+// RoPE (rotate-half) in place on the q and k parts of QKV; inverse = 1 rotates by -t*theta.
+template <class T> void rope(T* qkv, int B, int s, int nh, int dh, float base, int inverse, cudaStream_t st);
+
+// SwiGLU: M = silu(GU[:, :f]) * GU[:, f:];  backward dGU from dM.
+template <class T> void swiglu_fwd(const T* GU, T* M, int rows, int f, cudaStream_t st);
+template <class T> void swiglu_bwd(const T* GU, const T* dM, T* dGU, int rows, int f, cudaStream_t st);
+
+// Softmax cross-entropy over fp32 logits [rows, V]: row_loss[r] = lse - z_y;
+// dlogits (T) = (softmax - onehot) * inv_ntok. labels = tokens[:, 1:] of the micro-batch.
+template <class T> void softmax_ce(const float* logits, const int32_t* tok, int ld_tok, int s, int rows, int V,
+                                   float inv_ntok, T* dlogits, float* row_loss, cudaStream_t st);
+// out[0] (double) = sum of row_loss[0..rows) in a fixed order.
+void loss_reduce(const float* row_loss, int rows, double* out, cudaStream_t st);
+
+void cast_f32_bf16(const float* x, __nv_bfloat16* y, size_t n, cudaStream_t st);
+void add_f32(float* a, const float* b, size_t n, cudaStream_t st);       // a += b
+void copy_f32(float* a, const float* b, size_t n, cudaStream_t st);
+
+}  // namespace mario
