@@ -1,0 +1,308 @@
+"""Benchmark: one Mario-scheduled training iteration of GPT-3 1.3B (BASELINE.json configs[1]:
+seq 2048, GBS 128 = 32 micro-batches x mbs 4, bf16) on N B200s of one node.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference] [--level mario]
+    torchrun --nproc-per-node N bench.py --gpus N ...   (one pipeline stage per GPU, NCCL p2p)
+
+N GPUs = N pipeline stages (1F1B; at N = 1 the plan is gradient accumulation on one GPU, pass 3
+removes every checkpoint). Work per iteration is fixed (GBS 128) as N grows: "scaling": "strong".
+Rank 0 prints ONE JSON line. `--impl reference` times the CPU oracle (oracle/, numpy fp32) on a
+bounded sample of the same workload (the paper ships no code).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import synth  # noqa: E402
+
+METRIC = "samples/s (GPT-3 1.3B, seq 2048, GBS 128, Mario 1F1B plan, bf16)"
+UNIT = "samples/s"
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--level", default="mario", choices=["base", "ckpt", "mario"])
+    ap.add_argument("--scheme", default="1f1b")
+    ap.add_argument("--micro", type=int, default=32)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-e2e", action="store_true")
+    return ap.parse_args()
+
+
+def measured_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return d, "measured"
+    return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}, "fallback"
+
+
+# ------------------------------------------------------------------ CPU oracle leg
+def cpu_oracle_sample(cfg, layers_list=(1, 2)):
+    """Time the oracle (numpy fp32, all host cores) on ONE sample (mbs=1) of the workload's
+    model truncated to L in layers_list layers + embedding/head, then extrapolate linearly to the
+    full depth: t_sample = t(L=1) + (L_full - 1) * (t(L=2) - t(L=1))."""
+    from oracle import model as om
+    times = {}
+    for L in layers_list:
+        c = synth.with_(cfg, n_layers=L, micro_batch=1)
+        P = synth.make_weights(c, parity=False)
+        toks = synth.make_tokens(c, 1)
+        t0 = time.perf_counter()
+        om.step(c, P, toks, 1, np.float32)
+        times[L] = time.perf_counter() - t0
+    per_layer = max(times[2] - times[1], 1e-9)
+    t_sample = times[1] + (cfg.n_layers - 1) * per_layer
+    return t_sample, times
+
+
+def cores():
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count() or 1
+
+
+def run_reference(args, cfg, gbs):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    n_cores = cores()
+    os.environ.setdefault("OPENBLAS_NUM_THREADS", str(n_cores))
+    ts = []
+    for i in range(args.warmup + args.steps):
+        t, _ = cpu_oracle_sample(cfg)
+        if i >= args.warmup:
+            ts.append(t)
+    t = statistics.median(ts)
+    v = 1.0 / t
+    sample = (f"1 sample (mbs 1) of {cfg.family} L=1 and L=2 (+embedding/head, s={cfg.seq_len}) fwd+bwd "
+              f"fp32 per step, extrapolated to L={cfg.n_layers}")
+    out = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
+           "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3 * gbs,
+           "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
+           "data": "synthetic", "config": config_dict(cfg, args, gbs),
+           "cpu_baseline": {"value": v, "unit": UNIT, "cores": n_cores, "kind": "oracle", "sample": sample},
+           "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+def config_dict(cfg, args, gbs):
+    return {"workload": "cfg2: GPT-3 1.3B, seq 2048, 1F1B+Mario, bf16 (BASELINE.json configs[1])",
+            "model": "gpt3-1.3b", "layers": cfg.n_layers, "hidden": cfg.hidden, "heads": cfg.n_heads,
+            "global_batch": gbs, "seq_len": cfg.seq_len, "micro_batch": cfg.micro_batch,
+            "microbatches": args.micro, "stages": args.gpus, "scheme": args.scheme, "level": args.level,
+            "parallelism": f"pp{args.gpus}",
+            "l2": "no flush: every iteration streams >100 GB of weights/activations through HBM (>> 126 MB L2)"}
+
+
+# ------------------------------------------------------------------- clocks sampler
+class Clocks:
+    def __init__(self, index):
+        self.index, self.rows, self.proc = index, [], None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), "--query-gpu=clocks.sm,clocks.max.sm,clocks_event_reasons.active,"
+                 "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+                 "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap",
+                 "--format=csv,noheader,nounits", "-lms", "200"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL,
+                text=True)
+            threading.Thread(target=self._read, daemon=True).start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.rows.append([x.strip() for x in line.split(",")])
+
+    def stop(self):
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(2)
+            except Exception:
+                self.proc.kill()
+        sm = [float(r[0]) for r in self.rows if r and r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if len(r) > 1 and r[1].replace(".", "").isdigit()]
+        reasons = set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for r in self.rows:
+            for i, n in enumerate(names):
+                if len(r) > 3 + i and r[3 + i].lower() == "active":
+                    reasons.add(n)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+# ----------------------------------------------------------------------- GPU leg
+def init_weights_device(plan, rank, torch, seed=1234):
+    """Random-init weights of the GPT-3 1.3B architecture directly on the device (A20 recipe:
+    matrices N(0,0.02^2), residual-output matrices N(0,(0.02/sqrt(2L))^2), gamma 1, biases 0)."""
+    pc, _ = plan.rank_layout(rank)
+    w = torch.zeros(pc, dtype=torch.float32, device="cuda")
+    g = torch.Generator(device="cuda").manual_seed(seed + rank)
+    L = plan.cfg.n_layers
+    for name, off, cnt in plan.rank_params(rank):
+        leaf = name.split(".", 1)[-1]
+        seg = w[off:off + cnt]
+        if leaf.endswith(".g") or name.endswith(".g"):
+            seg.fill_(1.0)
+        elif leaf.endswith(".b") or name.endswith(".b"):
+            seg.zero_()
+        elif leaf in ("proj.w", "fc2.w", "o.w", "down.w"):
+            seg.normal_(0.0, 0.02 / math.sqrt(2 * L), generator=g)
+        else:
+            seg.normal_(0.0, 0.02, generator=g)
+    return w
+
+
+def main():
+    args = parse()
+    cfg = synth.GPT3_1P3B
+    gbs = args.micro * cfg.micro_batch
+    if args.impl == "reference":
+        run_reference(args, cfg, gbs)
+        return
+
+    import torch
+    import torch.distributed as dist
+    from paper_conf_ppopp_liultj25_b200 import _lib, api
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    assert world == args.gpus, f"--gpus {args.gpus} but WORLD_SIZE {world}"
+    torch.cuda.set_device(local)
+    if world > 1:
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    L = _lib.lib()
+    plan = api.Plan(cfg, world, args.micro, args.scheme, args.level, dtype="bf16")
+    ctx = api.Context(rank, world, local)
+    w = init_weights_device(plan, rank, torch)
+    pc, ws_bytes = plan.rank_layout(rank)
+    grads = torch.zeros(pc, dtype=torch.float32, device="cuda")
+    ws = torch.empty(ws_bytes, dtype=torch.uint8, device="cuda")
+    stream = torch.cuda.current_stream()
+    tok_host = [synth.make_tokens(cfg, args.micro, iteration=i) for i in range(args.warmup + args.steps)]
+    tok_dev = [torch.from_numpy(t).cuda() for t in tok_host]
+    torch.cuda.synchronize()
+
+    def barrier():
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize()
+
+    for i in range(args.warmup):
+        ctx.run_iter(plan, w, tok_dev[i], grads, ws, stream)
+    barrier()
+    clocks = Clocks(local)
+    clocks.start()
+    L.mario_kstats_enable(1)
+    launches0 = L.mario_kernel_launches()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    losses = []
+    barrier()
+    e0.record(stream)
+    for i in range(args.steps):
+        losses.append(ctx.run_iter(plan, w, tok_dev[args.warmup + i], grads, ws, stream))
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ms_total = e0.elapsed_time(e1)
+    launches = L.mario_kernel_launches() - launches0
+    clk = clocks.stop()
+    kst = {}
+    import ctypes as C
+    for kind, name in ((0, "gemm"), (1, "attn_fwd"), (2, "attn_bwd")):
+        ms, fl, by, n = C.c_double(), C.c_double(), C.c_double(), C.c_longlong()
+        L.mario_kstats_read(kind, C.byref(ms), C.byref(fl), C.byref(by), C.byref(n))
+        kst[name] = {"ms": ms.value, "flops": fl.value, "bytes": by.value, "launches": n.value}
+    L.mario_kstats_enable(0)
+    if world > 1:
+        t = torch.tensor([ms_total], device="cuda")
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ms_total = float(t.item())
+    ms_step = ms_total / args.steps
+    value = gbs / (ms_step / 1e3)
+
+    # end-to-end through the public call with pinned host tokens (H2D inside) and host loss (D2H)
+    e2e = None
+    if not args.no_e2e:
+        pinned = [torch.from_numpy(t).pin_memory() for t in tok_host[-args.steps:]]
+        barrier()
+        t0 = time.perf_counter()
+        for i in range(args.steps):
+            ctx.run_iter(plan, w, pinned[i], grads, ws, stream)
+        torch.cuda.synchronize()
+        dt = (time.perf_counter() - t0) / args.steps
+        if world > 1:
+            t = torch.tensor([dt], device="cuda")
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            dt = float(t.item())
+        e2e = {"value": gbs / dt, "unit": UNIT, "h2d_bytes_per_step": int(tok_host[0].nbytes),
+               "d2h_bytes_per_step": 4 + 8 * args.micro}
+
+    sim = plan.simulate()
+    peaks, peak_kind = measured_peaks()
+    g = kst["gemm"]
+    achieved = g["flops"] / (g["ms"] / 1e3) / 1e12 if g["ms"] > 0 else 0.0
+    peak = float(peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops")))
+    model_flops = 3.0 * (cfg.n_layers * (2 * cfg.seq_len * (12 * cfg.hidden ** 2) + 4 * cfg.seq_len ** 2 * cfg.hidden)
+                         + 2 * cfg.seq_len * cfg.hidden * cfg.vocab)
+    tflops_gpu = model_flops * gbs / (ms_step / 1e3) / world / 1e12
+    mem = torch.cuda.max_memory_allocated()
+    out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+           "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "strong",
+           "vs_baseline": None, "dtype": "bf16", "data": "synthetic (uniform tokens, random-init weights)",
+           "config": config_dict(cfg, args, gbs),
+           "model_tflops_per_gpu": tflops_gpu,
+           "loss": losses[-1],
+           "roofline": {"bound": "tensor", "kernel": "gemm_bf16_tc_kernel (tcgen05, all linear layers)",
+                        "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
+                        "peak_source": f"{peak_kind} bf16_tflops_sustained (MEASURED_PEAKS.json)",
+                        "traffic": None, "launches": g["launches"],
+                        "share_of_step": g["ms"] / ms_total if ms_total > 0 else None},
+           "kernels": {k: {"ms_per_step": v["ms"] / args.steps, "tflops": (v["flops"] / (v["ms"] / 1e3) / 1e12)
+                           if v["ms"] > 0 else None, "launches_per_step": v["launches"] / args.steps}
+                       for k, v in kst.items()},
+           "gpu_launches": int(launches),
+           "clocks": clk,
+           "bubble": {"simulated": sim.bubble_ratio, "stages": world},
+           "peak_mem_per_stage": {"simulated_bytes": sim.peak_bytes,
+                                  "measured_torch_max_allocated": int(mem)},
+           "e2e": e2e}
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        n_cores = cores()
+        os.environ.setdefault("OPENBLAS_NUM_THREADS", str(n_cores))
+        t, times = cpu_oracle_sample(cfg)
+        out["cpu_baseline"] = {"value": 1.0 / t, "unit": UNIT, "cores": n_cores, "kind": "oracle",
+                               "sample": f"1 sample (mbs 1), fp32 numpy oracle, L=1 ({times[1]:.2f}s) and L=2 "
+                                         f"({times[2]:.2f}s) + embedding/head at s=2048, extrapolated to 24 layers"}
+    if rank == 0:
+        print(json.dumps(out), flush=True)
+    ctx.close()
+    if world > 1:
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

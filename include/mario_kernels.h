@@ -36,6 +36,27 @@ int mario_k_gemm_f32(const float* A, int lda, int a_mn, const float* B, int ldb,
                      const float* residual, int ld_res, float* D2, const float* aux, int ld_aux,
                      void* stream);
 
+/* K5: causal attention forward (S = QK^T/sqrt(dh), S[t,u] = -inf for u > t,
+ * P = softmax, O = PV) per (sample, head). qkv: [B*s][3*H] with H = n_heads*head_dim, columns
+ * [0,H) = Q, [H,2H) = K, [2H,3H) = V, head j at j*head_dim; O: [B*s][H]; lse: fp32
+ * [n_heads][B*s] row log-sum-exp (natural log). bf16 = 1: bf16 storage on tensor cores
+ * (head_dim in {16,32,64,80,128}), else fp32. */
+int mario_k_attn_fwd(const void* qkv, void* O, float* lse, int B, int s, int n_heads, int head_dim,
+                     int bf16, void* stream);
+/* K6: backward: dqkv [B*s][3*H] (dQ | dK | dV) from dO [B*s][H], with P recomputed from lse;
+ * deterministic (no atomics). scratch: fp32 [n_heads][B*s]. */
+int mario_k_attn_bwd(const void* qkv, const void* O, const void* dO, const float* lse, void* dqkv,
+                     float* scratch, int B, int s, int n_heads, int head_dim, int bf16, void* stream);
+
+/* Instrumentation. mario_kernel_launches: number of kernels this library has launched since it
+ * was loaded (every call above and every mario_run_iter kernel). mario_kstats_enable(1) clears
+ * and starts CUDA-event timing of every GEMM (kind 0), attention forward (1) and backward (2)
+ * launch on its own stream; mario_kstats_read sums durations (ms), algorithmic FLOPs and bytes
+ * and counts launches of one kind (synchronizes on the recorded events). Returns 0 / -1. */
+long long mario_kernel_launches(void);
+int mario_kstats_enable(int on);
+int mario_kstats_read(int kind, double* total_ms, double* flops, double* bytes, long long* launches);
+
 #ifdef __cplusplus
 }
 #endif

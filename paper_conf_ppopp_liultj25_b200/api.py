@@ -127,9 +127,12 @@ class Plan:
 
     def __del__(self):
         h = getattr(self, "handle", None)
-        if h and _lib._lib is not None:
-            _lib.lib().mario_plan_destroy(h)
-            self.handle = None
+        try:
+            if h and _lib is not None and _lib._lib is not None:
+                _lib._lib.mario_plan_destroy(h)
+        except Exception:
+            pass
+        self.handle = None
 
     @property
     def _as_param(self):
@@ -241,11 +244,16 @@ class Context:
     def run_iter(self, plan: Plan, weights, tokens, grads, workspace, stream=None) -> float:
         """weights/grads/workspace: device tensors (data_ptr used); tokens: host int32 array."""
         import numpy as np
-        tok = np.ascontiguousarray(tokens, dtype=np.int32)
+        if hasattr(tokens, "data_ptr"):          # torch tensor (host or device), int32 contiguous
+            assert tokens.dtype.__str__() == "torch.int32" and tokens.is_contiguous()
+            tok_ptr = C.c_void_p(tokens.data_ptr())
+        else:
+            tok = np.ascontiguousarray(tokens, dtype=np.int32)
+            tok_ptr = tok.ctypes.data_as(C.c_void_p)
         loss = C.c_float()
         st = stream.cuda_stream if stream is not None else None
         _check(_lib.lib().mario_run_iter(plan.handle, C.c_void_p(weights.data_ptr()),
-                                         tok.ctypes.data_as(C.c_void_p), C.byref(loss),
+                                         tok_ptr, C.byref(loss),
                                          C.c_void_p(grads.data_ptr()), C.c_void_p(workspace.data_ptr()),
                                          C.c_void_p(st) if st else None))
         return float(loss.value)

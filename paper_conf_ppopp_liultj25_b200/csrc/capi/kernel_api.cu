@@ -2,6 +2,7 @@
 // device pointers in, used by the GPU unit tests and the benchmark's per-kernel roofline.
 #include <cuda_runtime.h>
 #include "../kernels/kernels.h"
+#include "../kernels/layers.h"
 #include "../../../include/mario_kernels.h"
 
 using namespace mario;
@@ -32,4 +33,24 @@ extern "C" int mario_k_gemm_f32(const float* A, int lda, int a_mn, const float* 
   g.M = M; g.N = N; g.K = K; g.D = D; g.ldd = ldd; g.beta = beta; g.bias = bias;
   g.residual = residual; g.ld_res = ld_res; g.D2 = D2; g.aux = aux; g.ld_aux = ld_aux;
   return static_cast<int>(gemm_f32(g, static_cast<cudaStream_t>(stream)));
+}
+
+extern "C" int mario_k_attn_fwd(const void* qkv, void* O, float* lse, int B, int s, int n_heads, int head_dim,
+                                int bf16, void* stream) {
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (bf16) attn_fwd<__nv_bfloat16>(static_cast<const __nv_bfloat16*>(qkv), static_cast<__nv_bfloat16*>(O), lse, B, s,
+                                    n_heads, head_dim, st);
+  else attn_fwd<float>(static_cast<const float*>(qkv), static_cast<float*>(O), lse, B, s, n_heads, head_dim, st);
+  return static_cast<int>(cudaGetLastError());
+}
+
+extern "C" int mario_k_attn_bwd(const void* qkv, const void* O, const void* dO, const float* lse, void* dqkv,
+                                float* scratch, int B, int s, int n_heads, int head_dim, int bf16, void* stream) {
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (bf16) attn_bwd<__nv_bfloat16>(static_cast<const __nv_bfloat16*>(qkv), static_cast<const __nv_bfloat16*>(O),
+                                    static_cast<const __nv_bfloat16*>(dO), lse, static_cast<__nv_bfloat16*>(dqkv),
+                                    scratch, B, s, n_heads, head_dim, st);
+  else attn_bwd<float>(static_cast<const float*>(qkv), static_cast<const float*>(O), static_cast<const float*>(dO), lse,
+                       static_cast<float*>(dqkv), scratch, B, s, n_heads, head_dim, st);
+  return static_cast<int>(cudaGetLastError());
 }

@@ -596,7 +596,7 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
     }
     // iteration prologue: tokens H2D, zero grads and losses, bf16 weight copies
     const size_t tok_bytes = static_cast<size_t>(P.pp.N) * m.micro_batch * (m.seq_len + 1) * 4;
-    CU(cudaMemcpyAsync(D->ws + D->a.tokens, tokens, tok_bytes, cudaMemcpyHostToDevice, st));
+    CU(cudaMemcpyAsync(D->ws + D->a.tokens, tokens, tok_bytes, cudaMemcpyDefault, st));   // host or device tokens
     CU(cudaMemsetAsync(D->gr, 0, rp.total * 4, st));
     CU(cudaMemsetAsync(D->ws + D->a.loss, 0, static_cast<size_t>(P.pp.N) * P.pp.parts() * 8, st));
     if (sizeof(T) == 2)

@@ -3,6 +3,7 @@
 // K-major or MN-major, plus the same fused epilogue. 64x64 tiles, 16x16 threads, 4x4 per thread.
 #include <cuda_runtime.h>
 #include "kernels.h"
+#include "kstats.h"
 
 namespace mario {
 namespace {
@@ -73,7 +74,10 @@ __global__ void __launch_bounds__(256) gemm_f32_kernel(GemmF32Args g) {
 cudaError_t gemm_f32(const GemmF32Args& g, cudaStream_t st) {
   if (g.M <= 0 || g.N <= 0) return cudaSuccess;
   dim3 grid((g.N + T - 1) / T, (g.M + T - 1) / T);
+  const int tok = kstats_begin(K_GEMM, 2.0 * g.M * g.N * g.K, 0.0, st);
   gemm_f32_kernel<<<grid, 256, 0, st>>>(g);
+  kstats_end(tok, st);
+  note_launch();
   return cudaGetLastError();
 }
 

@@ -26,6 +26,7 @@
 
 #include "sm100.cuh"
 #include "kernels.h"
+#include "kstats.h"
 
 namespace mario {
 
@@ -270,6 +271,10 @@ bool make_tmap(CUtensorMap* map, const void* base, uint64_t inner, uint64_t oute
   CUresult r = enc(map, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, estr,
                    CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
                    CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS)
+    fprintf(stderr, "[mario] cuTensorMapEncodeTiled failed (%d): base=%p inner=%llu outer=%llu ld=%llu box=%u,%u\n",
+            static_cast<int>(r), base, (unsigned long long)inner, (unsigned long long)outer, (unsigned long long)ld,
+            box_inner, box_outer);
   return r == CUDA_SUCCESS;
 }
 
@@ -279,17 +284,28 @@ cudaError_t launch_bn(const GemmArgs& g, cudaStream_t st, int num_sms) {
   CUtensorMap ta, tb;
   bool ok = A_MN ? make_tmap(&ta, g.A, g.M, g.K, g.lda, 64, 64) : make_tmap(&ta, g.A, g.K, g.M, g.lda, 64, BM);
   ok = ok && (B_MN ? make_tmap(&tb, g.B, g.N, g.K, g.ldb, 64, 64) : make_tmap(&tb, g.B, g.K, g.N, g.ldb, 64, BN));
-  if (!ok) return cudaErrorInvalidValue;
+  if (!ok) {
+    fprintf(stderr, "[mario] gemm_bf16: tensor map failed M=%d N=%d K=%d lda=%d ldb=%d a_mn=%d b_mn=%d\n", g.M, g.N,
+            g.K, g.lda, g.ldb, g.a_mn, g.b_mn);
+    return cudaErrorInvalidValue;
+  }
   auto kern = gemm_bf16_tc_kernel<BN, A_MN, B_MN>;
   static bool attr_set = false;
   if (!attr_set) {
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C::kSmem);
-    if (e != cudaSuccess) return e;
+    if (e != cudaSuccess) {
+      fprintf(stderr, "[mario] gemm_bf16: cudaFuncSetAttribute(smem=%d) failed: %s\n", C::kSmem, cudaGetErrorString(e));
+      return e;
+    }
     attr_set = true;
   }
   const int tiles = ((g.M + BM - 1) / BM) * ((g.N + BN - 1) / BN);
   const int grid = tiles < num_sms ? tiles : num_sms;
+  const int tok = kstats_begin(K_GEMM, 2.0 * g.M * g.N * g.K,
+                               2.0 * (double(g.M) * g.K + double(g.N) * g.K) + (g.ep.out_f32 ? 4.0 : 2.0) * g.M * g.N, st);
   kern<<<grid, kThreads, C::kSmem, st>>>(ta, tb, g.ep, g.M, g.N, g.K);
+  kstats_end(tok, st);
+  note_launch();
   return cudaGetLastError();
 }
 
@@ -316,7 +332,10 @@ int device_sm_count() {
 
 cudaError_t gemm_bf16(const GemmArgs& g, cudaStream_t st) {
   if (g.M <= 0 || g.N <= 0 || g.K <= 0) return cudaSuccess;
-  if ((g.lda % 8) || (g.ldb % 8)) return cudaErrorInvalidValue;  // TMA: 16-byte row pitch
+  if ((g.lda % 8) || (g.ldb % 8)) {  // TMA: 16-byte row pitch
+    fprintf(stderr, "[mario] gemm_bf16: lda=%d ldb=%d must be multiples of 8\n", g.lda, g.ldb);
+    return cudaErrorInvalidValue;
+  }
   const int sms = device_sm_count();
   // Prefer BN=256 unless it leaves the machine badly under-filled.
   const long tiles256 = static_cast<long>((g.M + BM - 1) / BM) * ((g.N + 255) / 256);

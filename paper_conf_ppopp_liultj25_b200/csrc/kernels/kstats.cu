@@ -1,0 +1,66 @@
+#include "kstats.h"
+
+#include <atomic>
+#include <mutex>
+#include <vector>
+
+#include "../../../include/mario_kernels.h"
+
+namespace mario {
+namespace {
+std::atomic<long long> g_launches{0};
+bool g_on = false;
+struct Rec { int kind; double flops, bytes; cudaEvent_t a, b; };
+std::vector<Rec> g_recs;
+std::mutex g_mu;
+}  // namespace
+
+void note_launch(int n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
+bool kstats_on() { return g_on; }
+
+int kstats_begin(KKind kind, double flops, double bytes, cudaStream_t st) {
+  if (!g_on) return -1;
+  std::lock_guard<std::mutex> lk(g_mu);
+  Rec r{kind, flops, bytes, nullptr, nullptr};
+  cudaEventCreate(&r.a);
+  cudaEventCreate(&r.b);
+  cudaEventRecord(r.a, st);
+  g_recs.push_back(r);
+  return static_cast<int>(g_recs.size()) - 1;
+}
+
+void kstats_end(int token, cudaStream_t st) {
+  if (token < 0) return;
+  std::lock_guard<std::mutex> lk(g_mu);
+  cudaEventRecord(g_recs[token].b, st);
+}
+}  // namespace mario
+
+using namespace mario;
+
+extern "C" long long mario_kernel_launches(void) { return g_launches.load(); }
+
+extern "C" int mario_kstats_enable(int on) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  for (auto& r : g_recs) { cudaEventDestroy(r.a); cudaEventDestroy(r.b); }
+  g_recs.clear();
+  g_on = on != 0;
+  return 0;
+}
+
+extern "C" int mario_kstats_read(int kind, double* total_ms, double* flops, double* bytes, long long* launches) {
+  std::lock_guard<std::mutex> lk(g_mu);
+  double ms = 0, fl = 0, by = 0;
+  long long n = 0;
+  for (auto& r : g_recs) {
+    if (r.kind != kind) continue;
+    float t = 0.f;
+    if (cudaEventSynchronize(r.b) != cudaSuccess || cudaEventElapsedTime(&t, r.a, r.b) != cudaSuccess) return -1;
+    ms += t; fl += r.flops; by += r.bytes; ++n;
+  }
+  if (total_ms) *total_ms = ms;
+  if (flops) *flops = fl;
+  if (bytes) *bytes = by;
+  if (launches) *launches = n;
+  return 0;
+}

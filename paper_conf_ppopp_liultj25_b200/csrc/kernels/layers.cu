@@ -3,8 +3,10 @@
 // independent implementation (no shared code).
 #include <cfloat>
 #include <cstdint>
+#include <type_traits>
 
 #include "layers.h"
+#include "kstats.h"
 
 namespace mario {
 namespace {
@@ -469,6 +471,7 @@ int grid_for(long n, int threads = 256) { long g = (n + threads - 1) / threads; 
 template <class T>
 void embed_fwd(const int32_t* tok, int ld_tok, int B, int s, const T* wte, const T* wpe, T* H, int h, cudaStream_t st) {
   embed_fwd_k<T><<<grid_for(static_cast<long>(B) * s * h), 256, 0, st>>>(tok, ld_tok, B, s, wte, wpe, H, h);
+  note_launch();
 }
 
 template <class T>
@@ -482,22 +485,27 @@ void embed_bwd(const int32_t* tok, int ld_tok, int B, int s, const T* dH, int h,
   static bool attr = false;
   if (!attr) { cudaFuncSetAttribute(embed_sort_k, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024); attr = true; }
   embed_sort_k<<<1, 1024, smem, st>>>(tok, ld_tok, B, s, keys, np2);
+  note_launch();
   embed_segsum_k<T><<<cdiv(static_cast<long>(Ttok) * 32, 256), 256, 0, st>>>(keys, Ttok, dH, h, dwte);
-  if (dwpe) embed_pos_bwd_k<T><<<grid_for(static_cast<long>(s) * h), 256, 0, st>>>(dH, B, s, h, dwpe);
+  note_launch();
+  if (dwpe) { embed_pos_bwd_k<T><<<grid_for(static_cast<long>(s) * h), 256, 0, st>>>(dH, B, s, h, dwpe); note_launch(); }
 }
 
 template <class T>
 void layernorm_fwd(const T* x, const float* g, const float* b, T* y, float* stats, int rows, int n, float eps, cudaStream_t st) {
   norm_fwd_k<T, false><<<cdiv(rows, 8), 256, 0, st>>>(x, g, b, y, stats, rows, n, eps);
+  note_launch();
 }
 template <class T>
 void rmsnorm_fwd(const T* x, const float* g, T* y, float* stats, int rows, int n, float eps, cudaStream_t st) {
   norm_fwd_k<T, true><<<cdiv(rows, 8), 256, 0, st>>>(x, g, nullptr, y, stats, rows, n, eps);
+  note_launch();
 }
 template <class T>
 void norm_bwd_dx(const T* dy, const T* x, const float* stats, const float* g, const T* dres, T* dx, int rows, int n,
                  int rms, cudaStream_t st) {
   norm_bwd_dx_k<T><<<cdiv(rows, 8), 256, 0, st>>>(dy, x, stats, g, dres, dx, rows, n, rms);
+  note_launch();
 }
 template <class T>
 void colsum(const T* a, const T* x, const float* stats, int rows, int n, int lda, int mode, float* out0, float* out1,
@@ -506,46 +514,63 @@ void colsum(const T* a, const T* x, const float* stats, int rows, int n, int lda
   if (nblk < 1) return;
   dim3 grid(cdiv(n, 256), nblk);
   colsum_partial_k<T><<<grid, 256, 0, st>>>(a, x, stats, rows, n, lda, mode == 2 ? 1 : mode, partial, nblk);
+  note_launch();
   colsum_final_k<<<cdiv(n, 256), 256, 0, st>>>(partial, nblk, n, mode == 2 ? 0 : mode, out0, out1);
+  note_launch();
 }
 
 template <class T>
 void attn_fwd(const T* qkv, T* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st) {
+  if constexpr (std::is_same<T, __nv_bfloat16>::value) {
+    if (flash_attn_supported(dh)) { flash_attn_fwd(qkv, O, lse, B, s, nh, dh, st); return; }
+  }
   attn_fwd_k<T><<<cdiv(static_cast<long>(B) * s * nh, 8), 256, 0, st>>>(qkv, O, lse, B, s, nh, dh);
+  note_launch();
 }
 template <class T>
 void attn_bwd(const T* qkv, const T* O, const T* dO, const float* lse, T* dqkv, float* Dsc, int B, int s, int nh,
               int dh, cudaStream_t st) {
+  if constexpr (std::is_same<T, __nv_bfloat16>::value) {
+    if (flash_attn_supported(dh)) { flash_attn_bwd(qkv, O, dO, lse, dqkv, Dsc, B, s, nh, dh, st); return; }
+  }
   const int grid = cdiv(static_cast<long>(B) * s * nh, 8);
   attn_bwd_dq_k<T><<<grid, 256, 0, st>>>(qkv, O, dO, lse, dqkv, Dsc, B, s, nh, dh);
+  note_launch();
   attn_bwd_dkdv_k<T><<<grid, 256, 0, st>>>(qkv, dO, lse, Dsc, dqkv, B, s, nh, dh);
+  note_launch();
 }
 
 template <class T>
 void rope(T* qkv, int B, int s, int nh, int dh, float base, int inverse, cudaStream_t st) {
   rope_k<T><<<grid_for(static_cast<long>(B) * s * nh * (dh / 2)), 256, 0, st>>>(qkv, B, s, nh, dh, base, inverse);
+  note_launch();
 }
 template <class T>
 void swiglu_fwd(const T* GU, T* M, int rows, int f, cudaStream_t st) {
   swiglu_fwd_k<T><<<grid_for(static_cast<long>(rows) * f), 256, 0, st>>>(GU, M, rows, f);
+  note_launch();
 }
 template <class T>
 void swiglu_bwd(const T* GU, const T* dM, T* dGU, int rows, int f, cudaStream_t st) {
   swiglu_bwd_k<T><<<grid_for(static_cast<long>(rows) * f), 256, 0, st>>>(GU, dM, dGU, rows, f);
+  note_launch();
 }
 template <class T>
 void softmax_ce(const float* logits, const int32_t* tok, int ld_tok, int s, int rows, int V, float inv_ntok,
                 T* dlogits, float* row_loss, cudaStream_t st) {
   softmax_ce_k<T><<<rows, 512, 0, st>>>(logits, tok, ld_tok, s, V, inv_ntok, dlogits, row_loss);
+  note_launch();
 }
 void loss_reduce(const float* row_loss, int rows, double* out, cudaStream_t st) {
   loss_reduce_k<<<1, 1024, 0, st>>>(row_loss, rows, out);
+  note_launch();
 }
 void cast_f32_bf16(const float* x, __nv_bfloat16* y, size_t n, cudaStream_t st) {
   cast_k<<<grid_for(static_cast<long>(n)), 256, 0, st>>>(x, y, n);
+  note_launch();
 }
-void add_f32(float* a, const float* b, size_t n, cudaStream_t st) { add_k<<<grid_for(static_cast<long>(n)), 256, 0, st>>>(a, b, n); }
-void copy_f32(float* a, const float* b, size_t n, cudaStream_t st) { copy_k<<<grid_for(static_cast<long>(n)), 256, 0, st>>>(a, b, n); }
+void add_f32(float* a, const float* b, size_t n, cudaStream_t st) { add_k<<<grid_for(static_cast<long>(n)), 256, 0, st>>>(a, b, n); note_launch(); }
+void copy_f32(float* a, const float* b, size_t n, cudaStream_t st) { copy_k<<<grid_for(static_cast<long>(n)), 256, 0, st>>>(a, b, n); note_launch(); }
 
 #define INST(T)                                                                                                     \
   template void embed_fwd<T>(const int32_t*, int, int, int, const T*, const T*, T*, int, cudaStream_t);              \

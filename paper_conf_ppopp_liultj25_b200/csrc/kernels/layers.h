@@ -48,6 +48,12 @@ template <class T> void softmax_ce(const float* logits, const int32_t* tok, int 
 // out[0] (double) = sum of row_loss[0..rows) in a fixed order.
 void loss_reduce(const float* row_loss, int rows, double* out, cudaStream_t st);
 
+// Tensor-core flash attention (bf16, mma.sync), used by attn_fwd/attn_bwd<bf16>.
+bool flash_attn_supported(int dh);
+void flash_attn_fwd(const __nv_bfloat16* qkv, __nv_bfloat16* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st);
+void flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* O, const __nv_bfloat16* dO, const float* lse,
+                    __nv_bfloat16* dqkv, float* Dd, int B, int s, int nh, int dh, cudaStream_t st);
+
 void cast_f32_bf16(const float* x, __nv_bfloat16* y, size_t n, cudaStream_t st);
 void add_f32(float* a, const float* b, size_t n, cudaStream_t st);       // a += b
 void copy_f32(float* a, const float* b, size_t n, cudaStream_t st);
