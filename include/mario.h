@@ -80,6 +80,15 @@ typedef struct {
   const int32_t* max_live_ckpt; /* [n_dev] live stage-input checkpoints */
 } mario_sim;
 
+/* One communication operation of a rank's NCCL program, in issue order (see
+ * mario_plan_comm_ops). kind: 0 = split a 2-rank channel communicator (a = src, b = dst,
+ * c = 0 activation / 1 gradient; collective over ALL ranks), 1 = split a replica-pair
+ * communicator (a < b), 2 = send on channel (a -> b, c) the message of (micro, part = sender
+ * part), issued right after list instruction list_index, 3 = receive on channel (a -> b, c) at
+ * list instruction list_index (part = receiver part), 4 = all-reduce of parameter a (count
+ * floats) on pair (b, c), 5 = all-reduce of count fp64 loss partials on the world. */
+typedef struct { int32_t kind, a, b, c, micro, part, list_index; int64_t count; } mario_commop;
+
 struct mario_plan;
 
 /* Build a plan: partition (even layers, embedding on virtual stage 0, final norm + head on
@@ -100,6 +109,11 @@ mario_status mario_plan_simulate(const struct mario_plan* plan, mario_sim* out);
  * compute instructions; arrays of length *n owned by the plan. */
 mario_status mario_plan_timeline(const struct mario_plan* plan, int32_t device,
                                  const double** start_ms, const double** finish_ms, int32_t* n);
+/* The ordered communication program of `rank` under world = stages (multi-process mode).
+ * Sends on each channel are issued in the receiver's receive order (sends are buffered, so
+ * this adds no dependency) — required because pass 4 may move an SA ahead of an earlier
+ * micro-batch's SA while NCCL channels are FIFO. Array owned by the plan. */
+mario_status mario_plan_comm_ops(const struct mario_plan* plan, int32_t rank, const mario_commop** ops, int32_t* n);
 /* Canonical text serialization (deterministic). If buf is NULL or cap too small, *needed
  * receives the size including the terminating NUL and MARIO_EINVAL is returned for cap>0. */
 mario_status mario_plan_serialize(const struct mario_plan* plan, char* buf, size_t cap, size_t* needed);

@@ -44,6 +44,11 @@ class CCosts(C.Structure):
                 ("work_bytes", C.POINTER(C.c_double)), ("static_bytes", C.c_double)]
 
 
+class CCommOp(C.Structure):
+    _fields_ = [("kind", C.c_int32), ("a", C.c_int32), ("b", C.c_int32), ("c", C.c_int32), ("micro", C.c_int32),
+                ("part", C.c_int32), ("list_index", C.c_int32), ("count", C.c_int64)]
+
+
 class CSim(C.Structure):
     _fields_ = [("makespan_ms", C.c_double), ("bubble_ratio", C.c_double), ("n_dev", C.c_int32),
                 ("busy_ms", C.POINTER(C.c_double)), ("peak_bytes", C.POINTER(C.c_uint64)),
@@ -57,6 +62,7 @@ _lib.register("mario_plan_instrs", C.c_int32, [_P, C.c_int32, C.POINTER(C.POINTE
 _lib.register("mario_plan_simulate", C.c_int32, [_P, C.POINTER(CSim)])
 _lib.register("mario_plan_timeline", C.c_int32, [_P, C.c_int32, C.POINTER(C.POINTER(C.c_double)),
                                                  C.POINTER(C.POINTER(C.c_double)), C.POINTER(C.c_int32)])
+_lib.register("mario_plan_comm_ops", C.c_int32, [_P, C.c_int32, C.POINTER(C.POINTER(CCommOp)), C.POINTER(C.c_int32)])
 _lib.register("mario_plan_serialize", C.c_int32, [_P, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)])
 _lib.register("mario_plan_rank_layout", C.c_int32, [_P, C.c_int32, C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)])
 _lib.register("mario_plan_rank_params", C.c_int32, [_P, C.c_int32, C.POINTER(C.POINTER(C.c_int32)),
@@ -160,6 +166,13 @@ class Plan:
         a, b, n = C.POINTER(C.c_double)(), C.POINTER(C.c_double)(), C.c_int32()
         _check(_lib.lib().mario_plan_timeline(self.handle, d, C.byref(a), C.byref(b), C.byref(n)))
         return [a[i] for i in range(n.value)], [b[i] for i in range(n.value)]
+
+    def comm_ops(self, rank: int):
+        """Rank's NCCL program: [(kind, a, b, c, micro, part, list_index, count)] (mario_commop)."""
+        p, n = C.POINTER(CCommOp)(), C.c_int32()
+        _check(_lib.lib().mario_plan_comm_ops(self.handle, rank, C.byref(p), C.byref(n)))
+        return [(p[i].kind, p[i].a, p[i].b, p[i].c, p[i].micro, p[i].part, p[i].list_index, p[i].count)
+                for i in range(n.value)]
 
     def serialize(self) -> str:
         need = C.c_size_t()

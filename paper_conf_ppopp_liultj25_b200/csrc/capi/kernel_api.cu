@@ -5,7 +5,14 @@
 #include "../kernels/layers.h"
 #include "../../../include/mario_kernels.h"
 
+namespace mario { extern int g_gemm_variant; }
 using namespace mario;
+
+extern "C" int mario_k_gemm_set_variant(int variant) {
+  if (variant < -1 || variant > 1) return 1;
+  g_gemm_variant = variant;
+  return 0;
+}
 
 extern "C" int mario_k_gemm_bf16(const void* A, int lda, int a_mn, const void* B, int ldb, int b_mn,
                                  int M, int N, int K, void* D, int ldd, int out_f32, float beta,

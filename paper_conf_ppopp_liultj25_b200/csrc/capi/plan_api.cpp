@@ -172,6 +172,70 @@ void fill_static(PlanObj& P, const mario_costs* c) {
   }
 }
 
+// Per-rank NCCL program (include/mario.h mario_commop). Channels and pairs are enumerated in
+// one global sorted order so every rank issues the same sequence of collective splits.
+void build_comm_program(PlanObj& P) {
+  const Pipe& pp = P.pp;
+  const int S = pp.S;
+  const size_t msg = tokens_per_micro(P.model) * P.model.hidden * elt_size(P.model);
+  std::set<std::tuple<int, int, int>> chans;
+  for (int d = 0; d < S; ++d)
+    for (const mario_instr& x : P.instrs[d]) {
+      if (x.op == MARIO_OP_SA) chans.insert({d, x.peer, 0});
+      if (x.op == MARIO_OP_SG) chans.insert({d, x.peer, 1});
+    }
+  std::map<int, std::vector<std::pair<int, int>>> holders;   // param idx -> (rank, packed j)
+  for (int d = 0; d < S; ++d)
+    for (size_t j = 0; j < P.rank_params[d].idx.size(); ++j) holders[P.rank_params[d].idx[j]].push_back({d, (int)j});
+  std::set<std::pair<int, int>> pairs;
+  for (auto& kv : holders)
+    for (auto& a : kv.second)
+      for (auto& b : kv.second) if (a.first < b.first) pairs.insert({a.first, b.first});
+  P.comm_ops.assign(S, {});
+  for (int r = 0; r < S; ++r) {
+    auto& ops = P.comm_ops[r];
+    for (auto& c : chans) ops.push_back({0, std::get<0>(c), std::get<1>(c), std::get<2>(c), -1, -1, -1, 0});
+    for (auto& pr : pairs) ops.push_back({1, pr.first, pr.second, 0, -1, -1, -1, 0});
+    // expected message order per outgoing channel = the receiver's receive order
+    std::map<std::tuple<int, int>, std::vector<std::pair<int, int>>> expect;   // (peer, kind) -> (m, sender vstage)
+    for (int q = 0; q < S; ++q)
+      for (const mario_instr& x : P.instrs[q])
+        if ((x.op == MARIO_OP_RA || x.op == MARIO_OP_RG) && x.peer == r)
+          expect[{q, x.op == MARIO_OP_RG ? 1 : 0}].push_back({x.micro, x.op == MARIO_OP_RA ? x.vstage - 1 : x.vstage + 1});
+    std::map<std::tuple<int, int>, size_t> next;
+    std::map<std::tuple<int, int>, std::set<std::pair<int, int>>> ready;
+    const auto& L = P.instrs[r];
+    for (size_t i = 0; i < L.size(); ++i) {
+      const mario_instr& x = L[i];
+      if (x.op == MARIO_OP_RA || x.op == MARIO_OP_RG)
+        ops.push_back({3, x.peer, r, x.op == MARIO_OP_RG ? 1 : 0, x.micro, x.part, (int)i, (int64_t)msg});
+      if (x.op == MARIO_OP_SA || x.op == MARIO_OP_SG) {
+        const auto key = std::make_tuple(x.peer, x.op == MARIO_OP_SG ? 1 : 0);
+        ready[key].insert({x.micro, x.vstage});
+        auto& ex = expect[key];
+        size_t& nx = next[key];
+        while (nx < ex.size() && ready[key].count(ex[nx])) {
+          const int m = ex[nx].first, ks = ex[nx].second;
+          int sp = -1;
+          for (int p = 0; p < pp.parts(); ++p) if (pp.vstage(r, p) == ks) sp = p;
+          ops.push_back({2, r, x.peer, std::get<1>(key), m, sp, (int)i, (int64_t)msg});
+          ++nx;
+        }
+      }
+    }
+    for (auto& kv : holders) {
+      std::set<int> ranks;
+      for (auto& c : kv.second) ranks.insert(c.first);
+      if (ranks.size() == 2 && ranks.count(r)) {
+        int j0 = -1;
+        for (auto& c : kv.second) if (c.first == r) { j0 = c.second; break; }
+        ops.push_back({4, kv.first, *ranks.begin(), *ranks.rbegin(), -1, -1, -1, (int64_t)P.rank_params[r].cnt[j0]});
+      }
+    }
+    ops.push_back({5, -1, -1, -1, -1, -1, -1, (int64_t)pp.N});
+  }
+}
+
 std::string serialize(const PlanObj& P) {
   std::string s;
   char buf[512];
@@ -254,6 +318,7 @@ extern "C" mario_status mario_plan(const mario_model* model, int32_t stages, int
       P->workspace_lb.push_back(make_arena(*P, d, P->pools_lb[d]).total);
     }
     P->serialized = serialize(*P);
+    build_comm_program(*P);
     if (mem_budget_bytes > 0) {
       uint64_t worst = *std::max_element(P->peak.begin(), P->peak.end());
       if (worst > mem_budget_bytes) {
@@ -296,6 +361,14 @@ extern "C" mario_status mario_plan_timeline(const struct mario_plan* P, int32_t 
   *start = P->sim.start[device].data();
   *finish = P->sim.finish[device].data();
   *n = static_cast<int32_t>(P->sim.start[device].size());
+  return MARIO_OK;
+}
+
+extern "C" mario_status mario_plan_comm_ops(const struct mario_plan* P, int32_t rank, const mario_commop** ops,
+                                            int32_t* n) {
+  if (!P || rank < 0 || rank >= P->pp.S || !ops || !n) return set_error(MARIO_EINVAL, "bad argument");
+  *ops = P->comm_ops[rank].data();
+  *n = static_cast<int32_t>(P->comm_ops[rank].size());
   return MARIO_OK;
 }
 

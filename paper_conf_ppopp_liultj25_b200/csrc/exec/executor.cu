@@ -427,24 +427,10 @@ struct Exec {
         break;
       }
       case MARIO_OP_SA:
-      case MARIO_OP_SG: {
-        const bool grad = x.op == MARIO_OP_SG;
-        auto& of = grad ? D.sg_of : D.sa_of;
-        const int i = of[key];
-        if (loopback) break;   // the receiver copies out of the held slot
-        Channel& ch = channel(D.d, x.peer, grad ? 1 : 0);
-        cudaEvent_t e = D.event();
-        CU(cudaEventRecord(e, st));
-        CU(cudaStreamWaitEvent(ch.stream, e, 0));
-        NC(ncclSend(send_slot(D, grad, i), msg_bytes, ncclUint8, peer_in_channel(D.d, x.peer), ch.comm, ch.stream));
-        auto& fr = grad ? D.sg_free : D.sa_free;
-        auto& fs = grad ? D.sg_free_set : D.sa_free_set;
-        CU(cudaEventRecord(fr[i], ch.stream));
-        fs[i] = true;
-        (grad ? D.sg_used : D.sa_used)[i] = false;
-        of.erase(key);
+      case MARIO_OP_SG:
+        // loopback: the receiver copies out of the held slot; NCCL: the send is issued by
+        // issue_send() from the rank's comm program, in the receiver's order
         break;
-      }
       case MARIO_OP_RA:
       case MARIO_OP_RG: {
         const bool grad = x.op == MARIO_OP_RG;
@@ -484,6 +470,27 @@ struct Exec {
     }
   }
 
+  void issue_send(Dev<T>& D, const mario_commop& op) {
+    const bool grad = op.c == 1;
+    auto& of = grad ? D.sg_of : D.sa_of;
+    const auto key = std::make_pair(op.micro, op.part);
+    auto it = of.find(key);
+    if (it == of.end()) throw std::runtime_error("send: message not produced");
+    const int i = it->second;
+    Channel& ch = channel(D.d, op.b, op.c);
+    cudaEvent_t e = D.event();
+    CU(cudaEventRecord(e, st));
+    CU(cudaStreamWaitEvent(ch.stream, e, 0));
+    NC(ncclSend(send_slot(D, grad, i), static_cast<size_t>(op.count), ncclUint8, peer_in_channel(D.d, op.b), ch.comm,
+                ch.stream));
+    auto& fr = grad ? D.sg_free : D.sa_free;
+    auto& fs = grad ? D.sg_free_set : D.sa_free_set;
+    CU(cudaEventRecord(fr[i], ch.stream));
+    fs[i] = true;
+    (grad ? D.sg_used : D.sa_used)[i] = false;
+    of.erase(it);
+  }
+
   bool sender_part_ok(Dev<T>& Sd, int sp, const mario_instr& x, bool grad) {
     // the sender's virtual stage must be adjacent to ours in the right direction
     const int ks = Sd.P->pp.vstage(Sd.d, sp);
@@ -515,41 +522,30 @@ struct Exec {
 // pair communicators for gradient synchronisation. Collective over all ranks: every rank
 // iterates the same sorted set.
 void ensure_channels(const PlanObj& P) {
-  std::set<std::tuple<int, int, int>> need;
-  std::set<std::pair<int, int>> pairs;
-  for (int d = 0; d < P.pp.S; ++d)
-    for (const mario_instr& x : P.instrs[d]) {
-      if (x.op == MARIO_OP_SA) need.insert({d, x.peer, 0});
-      if (x.op == MARIO_OP_SG) need.insert({d, x.peer, 1});
+  for (const mario_commop& op : P.comm_ops[g.rank]) {
+    if (op.kind == 0) {
+      const auto c = std::make_tuple(op.a, op.b, op.c);
+      if (g.created_channels.count(c)) continue;
+      g.created_channels.insert(c);
+      const int lo = std::min(op.a, op.b), hi = std::max(op.a, op.b);
+      const bool member = g.rank == lo || g.rank == hi;
+      ncclComm_t comm = nullptr;
+      NC(ncclCommSplit(g.world_comm, member ? 1 : NCCL_SPLIT_NOCOLOR, g.rank == lo ? 0 : 1, &comm, nullptr));
+      if (member) {
+        Channel ch;
+        ch.comm = comm;
+        CU(cudaStreamCreateWithFlags(&ch.stream, cudaStreamNonBlocking));
+        g.channels[c] = ch;
+      }
+    } else if (op.kind == 1) {
+      const auto pr = std::make_pair(op.a, op.b);
+      if (g.created_pairs.count(pr)) continue;
+      g.created_pairs.insert(pr);
+      const bool member = g.rank == op.a || g.rank == op.b;
+      ncclComm_t comm = nullptr;
+      NC(ncclCommSplit(g.world_comm, member ? 1 : NCCL_SPLIT_NOCOLOR, g.rank == op.a ? 0 : 1, &comm, nullptr));
+      if (member) g.pair_comms[pr] = comm;
     }
-  // replica pairs: any two ranks holding copies of the same parameter
-  std::map<int, std::set<int>> holders;
-  for (int d = 0; d < P.pp.S; ++d)
-    for (int32_t i : P.rank_params[d].idx) holders[i].insert(d);
-  for (auto& kv : holders)
-    for (int a : kv.second)
-      for (int b : kv.second) if (a < b) pairs.insert({a, b});
-  for (auto& c : need) {
-    if (g.created_channels.count(c)) continue;
-    g.created_channels.insert(c);
-    const int lo = std::min(std::get<0>(c), std::get<1>(c)), hi = std::max(std::get<0>(c), std::get<1>(c));
-    const bool member = g.rank == lo || g.rank == hi;
-    ncclComm_t comm = nullptr;
-    NC(ncclCommSplit(g.world_comm, member ? 1 : NCCL_SPLIT_NOCOLOR, g.rank == lo ? 0 : 1, &comm, nullptr));
-    if (member) {
-      Channel ch;
-      ch.comm = comm;
-      CU(cudaStreamCreateWithFlags(&ch.stream, cudaStreamNonBlocking));
-      g.channels[c] = ch;
-    }
-  }
-  for (auto& pr : pairs) {
-    if (g.created_pairs.count(pr)) continue;
-    g.created_pairs.insert(pr);
-    const bool member = g.rank == pr.first || g.rank == pr.second;
-    ncclComm_t comm = nullptr;
-    NC(ncclCommSplit(g.world_comm, member ? 1 : NCCL_SPLIT_NOCOLOR, g.rank == pr.first ? 0 : 1, &comm, nullptr));
-    if (member) g.pair_comms[pr] = comm;
   }
 }
 
@@ -611,7 +607,20 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
   if (loopback) {
     for (auto [d, i] : P.loopback_order) E.run_instr(d, P.instrs[d][i]);
   } else {
-    for (const mario_instr& x : P.instrs[g.rank]) E.run_instr(g.rank, x);
+    const auto& L = P.instrs[g.rank];
+    std::vector<std::vector<const mario_commop*>> sends_after(L.size());
+    for (const mario_commop& op : P.comm_ops[g.rank])
+      if (op.kind == 2) sends_after[op.list_index].push_back(&op);
+    for (size_t i = 0; i < L.size(); ++i) {
+      E.run_instr(g.rank, L[i]);
+      for (const mario_commop* op : sends_after[i]) E.issue_send(*E.devs[0], *op);
+    }
+    // the iteration ends when every channel stream has drained (its last sends complete)
+    for (auto& kv : g.channels) {
+      cudaEvent_t e = E.devs[0]->event();
+      CU(cudaEventRecord(e, kv.second.stream));
+      CU(cudaStreamWaitEvent(st, e, 0));
+    }
   }
 
   // gradient finalization (reading A7): sum every copy of each parameter (tied embeddings,
@@ -640,23 +649,14 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
         add_f32(D.gr + P.rank_params[g.rank].off[mine[0]], D.gr + P.rank_params[g.rank].off[mine[c]],
                 P.rank_params[g.rank].cnt[mine[0]], st);
     }
-    // then pairwise all-reduce with every other holder, in global (idx, peer) order
+    // then pairwise all-reduce with the other holder, in the comm program's (global) order
     NC(ncclGroupStart());
-    for (auto& kv : copies) {
-      std::set<int> ranks;
-      for (auto& c : kv.second) ranks.insert(c.first);
-      if (ranks.size() < 2 || !ranks.count(g.rank)) continue;
+    for (const mario_commop& op : P.comm_ops[g.rank]) {
+      if (op.kind != 4) continue;
       int j0 = -1;
-      for (auto& c : kv.second) if (c.first == g.rank) { j0 = c.second; break; }
+      for (auto& c : copies[op.a]) if (c.first == g.rank) { j0 = c.second; break; }
       float* buf = D.gr + P.rank_params[g.rank].off[j0];
-      const size_t n = P.rank_params[g.rank].cnt[j0];
-      if (ranks.size() == 2) {
-        const int other = *ranks.begin() == g.rank ? *ranks.rbegin() : *ranks.begin();
-        auto pr = std::make_pair(std::min(g.rank, other), std::max(g.rank, other));
-        NC(ncclAllReduce(buf, buf, n, ncclFloat32, ncclSum, g.pair_comms[pr], st));
-      } else {
-        throw std::runtime_error("parameter held by > 2 ranks is not supported in multi-process mode");
-      }
+      NC(ncclAllReduce(buf, buf, static_cast<size_t>(op.count), ncclFloat32, ncclSum, g.pair_comms[{op.b, op.c}], st));
     }
     NC(ncclGroupEnd());
     for (auto& kv : copies) {

@@ -48,15 +48,89 @@ struct Cfg {
   static constexpr int kSmem = kStages * kStageBytes + 1024 /*align*/ + 256 /*barriers*/;
 };
 
+// bf16 outputs: the SFU tanh (rel. err ~2^-11) is far below bf16 resolution (2^-8)
 __device__ __forceinline__ float gelu_tanh_f(float z) {
   const float c = 0.7978845608028654f;
-  float t = tanhf(c * (z + 0.044715f * z * z * z));
+  float t = tanh_approx(c * (z + 0.044715f * z * z * z));
   return 0.5f * z * (1.f + t);
 }
 __device__ __forceinline__ float gelu_tanh_grad_f(float z) {
   const float c = 0.7978845608028654f;
-  float t = tanhf(c * (z + 0.044715f * z * z * z));
+  float t = tanh_approx(c * (z + 0.044715f * z * z * z));
   return 0.5f * (1.f + t) + 0.5f * z * (1.f - t * t) * c * (1.f + 3.f * 0.044715f * z * z);
+}
+
+// Fused epilogue for 32 consecutive accumulator columns of one output row (fp32 in r[]).
+__device__ __forceinline__ void epilogue_chunk(const GemmEpilogue& ep, const uint32_t (&r)[32], int row, int col0,
+                                               bool row_ok, int N) {
+  if (!row_ok || col0 >= N) return;
+  float v[32];
+#pragma unroll
+  for (int j = 0; j < 32; ++j) v[j] = __uint_as_float(r[j]);
+  const bool full_cols = col0 + 32 <= N;
+  if (ep.bias) {
+#pragma unroll
+    for (int j = 0; j < 32; ++j) if (full_cols || col0 + j < N) v[j] += ep.bias[col0 + j];
+  }
+  if (ep.aux) {  // GeLU backward: D = acc * gelu'(Z)
+    const __nv_bfloat16* z = ep.aux + static_cast<size_t>(row) * ep.ld_aux + col0;
+#pragma unroll
+    for (int j = 0; j < 32; ++j) if (full_cols || col0 + j < N) v[j] *= gelu_tanh_grad_f(__bfloat162float(z[j]));
+  }
+  if (ep.residual) {
+    const __nv_bfloat16* rr = ep.residual + static_cast<size_t>(row) * ep.ld_res + col0;
+    if (full_cols) {
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        uint4 u = *reinterpret_cast<const uint4*>(rr + q * 8);
+        const __nv_bfloat16* h = reinterpret_cast<const __nv_bfloat16*>(&u);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) v[q * 8 + j] += __bfloat162float(h[j]);
+      }
+    } else {
+      for (int j = 0; j < 32; ++j) if (col0 + j < N) v[j] += __bfloat162float(rr[j]);
+    }
+  }
+  if (ep.out_f32) {
+    float* d = ep.d_f32 + static_cast<size_t>(row) * ep.ldd + col0;
+    if (full_cols) {
+#pragma unroll
+      for (int q = 0; q < 8; ++q) {
+        float4 o = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
+        if (ep.beta != 0.f) {
+          float4 old = *reinterpret_cast<const float4*>(d + 4 * q);
+          o.x += ep.beta * old.x; o.y += ep.beta * old.y; o.z += ep.beta * old.z; o.w += ep.beta * old.w;
+        }
+        *reinterpret_cast<float4*>(d + 4 * q) = o;
+      }
+    } else {
+      for (int j = 0; j < 32; ++j)
+        if (col0 + j < N) d[j] = v[j] + (ep.beta != 0.f ? ep.beta * d[j] : 0.f);
+    }
+  } else {
+    __nv_bfloat16* d = ep.d_bf16 + static_cast<size_t>(row) * ep.ldd + col0;
+    __nv_bfloat16* d2 = ep.d2_bf16 ? ep.d2_bf16 + static_cast<size_t>(row) * ep.ldd + col0 : nullptr;
+    if (full_cols) {
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        uint4 u, u2;
+        __nv_bfloat16* h = reinterpret_cast<__nv_bfloat16*>(&u);
+        __nv_bfloat16* h2 = reinterpret_cast<__nv_bfloat16*>(&u2);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          h[j] = __float2bfloat16_rn(v[q * 8 + j]);
+          if (d2) h2[j] = __float2bfloat16_rn(gelu_tanh_f(v[q * 8 + j]));
+        }
+        *reinterpret_cast<uint4*>(d + q * 8) = u;
+        if (d2) *reinterpret_cast<uint4*>(d2 + q * 8) = u2;
+      }
+    } else {
+      for (int j = 0; j < 32; ++j) if (col0 + j < N) {
+        d[j] = __float2bfloat16_rn(v[j]);
+        if (d2) d2[j] = __float2bfloat16_rn(gelu_tanh_f(v[j]));
+      }
+    }
+  }
 }
 
 template <int BN, bool A_MN, bool B_MN>
@@ -168,75 +242,7 @@ gemm_bf16_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
         uint32_t r[32];
         tmem_ld_32x32b_x32(tmem_base + acc * BN + c * 32 + (static_cast<uint32_t>(quarter * 32) << 16), r);
         tmem_ld_wait();
-        const int col0 = n0 + c * 32;
-        if (!row_ok || col0 >= N) continue;
-        float v[32];
-#pragma unroll
-        for (int j = 0; j < 32; ++j) v[j] = __uint_as_float(r[j]);
-        const bool full_cols = col0 + 32 <= N;
-        if (ep.bias) {
-#pragma unroll
-          for (int j = 0; j < 32; ++j) if (full_cols || col0 + j < N) v[j] += ep.bias[col0 + j];
-        }
-        if (ep.aux) {  // GeLU backward: D = acc * gelu'(Z)
-          const __nv_bfloat16* z = ep.aux + static_cast<size_t>(row) * ep.ld_aux + col0;
-#pragma unroll
-          for (int j = 0; j < 32; ++j) if (full_cols || col0 + j < N) v[j] *= gelu_tanh_grad_f(__bfloat162float(z[j]));
-        }
-        if (ep.residual) {
-          const __nv_bfloat16* rr = ep.residual + static_cast<size_t>(row) * ep.ld_res + col0;
-          if (full_cols) {
-#pragma unroll
-            for (int q = 0; q < 4; ++q) {
-              uint4 u = *reinterpret_cast<const uint4*>(rr + q * 8);
-              const __nv_bfloat16* h = reinterpret_cast<const __nv_bfloat16*>(&u);
-#pragma unroll
-              for (int j = 0; j < 8; ++j) v[q * 8 + j] += __bfloat162float(h[j]);
-            }
-          } else {
-            for (int j = 0; j < 32; ++j) if (col0 + j < N) v[j] += __bfloat162float(rr[j]);
-          }
-        }
-        if (ep.out_f32) {
-          float* d = ep.d_f32 + static_cast<size_t>(row) * ep.ldd + col0;
-          if (full_cols) {
-#pragma unroll
-            for (int q = 0; q < 8; ++q) {
-              float4 o = make_float4(v[4 * q], v[4 * q + 1], v[4 * q + 2], v[4 * q + 3]);
-              if (ep.beta != 0.f) {
-                float4 old = *reinterpret_cast<const float4*>(d + 4 * q);
-                o.x += ep.beta * old.x; o.y += ep.beta * old.y; o.z += ep.beta * old.z; o.w += ep.beta * old.w;
-              }
-              *reinterpret_cast<float4*>(d + 4 * q) = o;
-            }
-          } else {
-            for (int j = 0; j < 32; ++j)
-              if (col0 + j < N) d[j] = v[j] + (ep.beta != 0.f ? ep.beta * d[j] : 0.f);
-          }
-        } else {
-          __nv_bfloat16* d = ep.d_bf16 + static_cast<size_t>(row) * ep.ldd + col0;
-          __nv_bfloat16* d2 = ep.d2_bf16 ? ep.d2_bf16 + static_cast<size_t>(row) * ep.ldd + col0 : nullptr;
-          if (full_cols) {
-#pragma unroll
-            for (int q = 0; q < 4; ++q) {
-              uint4 u, u2;
-              __nv_bfloat16* h = reinterpret_cast<__nv_bfloat16*>(&u);
-              __nv_bfloat16* h2 = reinterpret_cast<__nv_bfloat16*>(&u2);
-#pragma unroll
-              for (int j = 0; j < 8; ++j) {
-                h[j] = __float2bfloat16_rn(v[q * 8 + j]);
-                if (d2) h2[j] = __float2bfloat16_rn(gelu_tanh_f(v[q * 8 + j]));
-              }
-              *reinterpret_cast<uint4*>(d + q * 8) = u;
-              if (d2) *reinterpret_cast<uint4*>(d2 + q * 8) = u2;
-            }
-          } else {
-            for (int j = 0; j < 32; ++j) if (col0 + j < N) {
-              d[j] = __float2bfloat16_rn(v[j]);
-              if (d2) d2[j] = __float2bfloat16_rn(gelu_tanh_f(v[j]));
-            }
-          }
-        }
+        epilogue_chunk(ep, r, row, n0 + c * 32, row_ok, N);
       }
       tc_fence_before();
       mbar_arrive(&tempty[acc]);
@@ -244,6 +250,133 @@ gemm_bf16_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
   }
   __syncthreads();
   if (warp == 1) tmem_dealloc<C::kTmemCols>(tmem_base);
+}
+
+
+// ------------------------------------------------------------------------------------------
+// CTA-pair variant (cta_group::2): a cluster of 2 CTAs computes a 256x256 tile with
+// tcgen05.mma M=256 N=256 issued by the leader CTA. Each CTA TMA-loads its 128-row half of A
+// and its 128-row half of B (operand bytes per FLOP 1.5x lower than the 128x256 single-CTA
+// tile) and owns 128 accumulator rows x 256 columns in its TMEM (double-buffered, 512 cols).
+// 10 warps: producer, MMA (leader only), 8 epilogue warps (2 per TMEM lane quarter).
+constexpr int kThreads2 = 320;
+constexpr int kStages2 = 6;
+constexpr int kHalfBytes = 128 * BK * 2;            // 16 KB: one CTA's half of A (or B) per stage
+constexpr int kStage2Bytes = 2 * kHalfBytes;        // A half + B half
+constexpr int kSmem2 = kStages2 * kStage2Bytes + 1024 + 256;
+
+template <bool A_MN, bool B_MN>
+__global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads2, 1)
+gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+                     GemmEpilogue ep, int M, int N, int K) {
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* full = reinterpret_cast<uint64_t*>(smem + kStages2 * kStage2Bytes);
+  uint64_t* empty = full + kStages2;
+  uint64_t* tfull = empty + kStages2;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
+
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const uint32_t rank = cluster_ctarank();
+  const bool leader = rank == 0;
+  const int pair = blockIdx.x / 2, npairs = gridDim.x / 2;
+  const int num_m = (M + 255) / 256, num_n = (N + 255) / 256;
+  const int num_tiles = num_m * num_n;
+  const int nk = (K + BK - 1) / BK;
+
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&tmA);
+    tma_prefetch_desc(&tmB);
+    for (int s = 0; s < kStages2; ++s) { mbar_init(&full[s], 2); mbar_init(&empty[s], 1); }
+    for (int a = 0; a < 2; ++a) { mbar_init(&tfull[a], 1); mbar_init(&tempty[a], 16); }
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc_2sm<512>(tmem_slot);
+  tc_fence_before();
+  cluster_sync();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  if (warp == 0) {
+    if (elect_one()) {
+      int s = 0; uint32_t ph = 0;
+      for (int tile = pair; tile < num_tiles; tile += npairs) {
+        const int m0 = (tile % num_m) * 256 + 128 * rank, n0 = (tile / num_m) * 256 + 128 * rank;
+        for (int kb = 0; kb < nk; ++kb) {
+          mbar_wait(&empty[s], ph ^ 1);
+          uint8_t* sa = smem + s * kStage2Bytes;
+          uint8_t* sb = sa + kHalfBytes;
+          const uint32_t lbar = mapa(&full[s], 0);
+          if (leader) mbar_arrive_expect_tx(&full[s], 2 * kStage2Bytes);
+          else mbar_arrive_cluster(lbar);
+          const int k0 = kb * BK;
+          if (A_MN) { tma_load_2d_2sm(sa, &tmA, lbar, m0, k0); tma_load_2d_2sm(sa + 8192, &tmA, lbar, m0 + 64, k0); }
+          else tma_load_2d_2sm(sa, &tmA, lbar, k0, m0);
+          if (B_MN) { tma_load_2d_2sm(sb, &tmB, lbar, n0, k0); tma_load_2d_2sm(sb + 8192, &tmB, lbar, n0 + 64, k0); }
+          else tma_load_2d_2sm(sb, &tmB, lbar, k0, n0);
+          if (++s == kStages2) { s = 0; ph ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (leader) {
+      constexpr uint32_t idesc = umma_idesc_bf16(256, 256, A_MN ? 1 : 0, B_MN ? 1 : 0);
+      int s = 0; uint32_t ph = 0; int t = 0;
+      for (int tile = pair; tile < num_tiles; tile += npairs, ++t) {
+        const int acc = t & 1;
+        const uint32_t acc_ph = (t >> 1) & 1;
+        mbar_wait(&tempty[acc], acc_ph ^ 1);
+        tc_fence_after();
+        const uint32_t d_tmem = tmem_base + acc * 256;
+        for (int kb = 0; kb < nk; ++kb) {
+          mbar_wait(&full[s], ph);
+          tc_fence_after();
+          if (elect_one()) {
+            const uint32_t sa = smem_u32(smem + s * kStage2Bytes);
+            const uint32_t sb = sa + kHalfBytes;
+#pragma unroll
+            for (int kk = 0; kk < BK / 16; ++kk) {
+              const uint64_t ad = A_MN ? umma_desc_sw128(sa + kk * 2048, 8192, 1024) : umma_desc_sw128(sa + kk * 32, 16, 1024);
+              const uint64_t bd = B_MN ? umma_desc_sw128(sb + kk * 2048, 8192, 1024) : umma_desc_sw128(sb + kk * 32, 16, 1024);
+              umma_bf16_2sm(d_tmem, ad, bd, idesc, (kb | kk) != 0);
+            }
+            umma_commit_2sm(&empty[s], 0x3);
+            if (kb == nk - 1) umma_commit_2sm(&tfull[acc], 0x3);
+          }
+          __syncwarp();
+          if (++s == kStages2) { s = 0; ph ^= 1; }
+        }
+      }
+    }
+  } else {
+    const int quarter = warp & 3, half = (warp - 2) >> 2;   // column half of the 256-wide tile
+    const uint32_t tempty_leader0 = mapa(&tempty[0], 0), tempty_leader1 = mapa(&tempty[1], 0);
+    int t = 0;
+    for (int tile = pair; tile < num_tiles; tile += npairs, ++t) {
+      const int acc = t & 1;
+      const uint32_t acc_ph = (t >> 1) & 1;
+      const int m0 = (tile % num_m) * 256 + 128 * rank, n0 = (tile / num_m) * 256;
+      mbar_wait(&tfull[acc], acc_ph);
+      tc_fence_after();
+      const int row = m0 + quarter * 32 + lane;
+      const bool row_ok = row < M;
+#pragma unroll 1
+      for (int c = 0; c < 4; ++c) {
+        uint32_t r[32];
+        const int col = half * 128 + c * 32;
+        tmem_ld_32x32b_x32(tmem_base + acc * 256 + col + (static_cast<uint32_t>(quarter * 32) << 16), r);
+        tmem_ld_wait();
+        epilogue_chunk(ep, r, row, n0 + col, row_ok, N);
+      }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive_cluster(acc ? tempty_leader1 : tempty_leader0);
+    }
+  }
+  tc_fence_before();
+  cluster_sync();
+  if (warp == 1) tmem_dealloc_2sm<512>(tmem_base);
 }
 
 PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
@@ -309,6 +442,33 @@ cudaError_t launch_bn(const GemmArgs& g, cudaStream_t st, int num_sms) {
   return cudaGetLastError();
 }
 
+
+template <bool A_MN, bool B_MN>
+cudaError_t launch_pair(const GemmArgs& g, cudaStream_t st, int num_sms) {
+  CUtensorMap ta, tb;
+  bool ok = A_MN ? make_tmap(&ta, g.A, g.M, g.K, g.lda, 64, 64) : make_tmap(&ta, g.A, g.K, g.M, g.lda, 64, 128);
+  ok = ok && (B_MN ? make_tmap(&tb, g.B, g.N, g.K, g.ldb, 64, 64) : make_tmap(&tb, g.B, g.K, g.N, g.ldb, 64, 128));
+  if (!ok) {
+    fprintf(stderr, "[mario] gemm_bf16 (pair): tensor map failed M=%d N=%d K=%d\n", g.M, g.N, g.K);
+    return cudaErrorInvalidValue;
+  }
+  auto kern = gemm_bf16_tc2_kernel<A_MN, B_MN>;
+  static bool attr_set = false;
+  if (!attr_set) {
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem2);
+    if (e != cudaSuccess) return e;
+    attr_set = true;
+  }
+  const int tiles = ((g.M + 255) / 256) * ((g.N + 255) / 256);
+  const int pairs = tiles < num_sms / 2 ? tiles : num_sms / 2;
+  const int tok = kstats_begin(K_GEMM, 2.0 * g.M * g.N * g.K,
+                               2.0 * (double(g.M) * g.K + double(g.N) * g.K) + (g.ep.out_f32 ? 4.0 : 2.0) * g.M * g.N, st);
+  kern<<<2 * pairs, kThreads2, kSmem2, st>>>(ta, tb, g.ep, g.M, g.N, g.K);
+  kstats_end(tok, st);
+  note_launch();
+  return cudaGetLastError();
+}
+
 template <int BN>
 cudaError_t launch_major(const GemmArgs& g, cudaStream_t st, int num_sms) {
   if (!g.a_mn && !g.b_mn) return launch_bn<BN, false, false>(g, st, num_sms);
@@ -330,14 +490,25 @@ int device_sm_count() {
   return n;
 }
 
-cudaError_t gemm_bf16(const GemmArgs& g, cudaStream_t st) {
+int g_gemm_variant = -1;   // mario_k_gemm_set_variant: -1 auto, 0 single-CTA only, 1 prefer CTA pair
+
+cudaError_t gemm_bf16(const GemmArgs& g0, cudaStream_t st) {
+  GemmArgs g = g0;
+  if (g.use_pair == -1) g.use_pair = g_gemm_variant;
   if (g.M <= 0 || g.N <= 0 || g.K <= 0) return cudaSuccess;
   if ((g.lda % 8) || (g.ldb % 8)) {  // TMA: 16-byte row pitch
     fprintf(stderr, "[mario] gemm_bf16: lda=%d ldb=%d must be multiples of 8\n", g.lda, g.ldb);
     return cudaErrorInvalidValue;
   }
   const int sms = device_sm_count();
-  // Prefer BN=256 unless it leaves the machine badly under-filled.
+  // Prefer the CTA-pair 256x256 tile when it fills the machine, else 128x256 / 128x128.
+  const long tiles_pair = static_cast<long>((g.M + 255) / 256) * ((g.N + 255) / 256);
+  if (g.use_pair != 0 && g.M >= 256 && g.N >= 256 && (tiles_pair >= sms / 2 || g.use_pair > 0)) {
+    if (!g.a_mn && !g.b_mn) return launch_pair<false, false>(g, st, sms);
+    if (!g.a_mn && g.b_mn) return launch_pair<false, true>(g, st, sms);
+    if (g.a_mn && g.b_mn) return launch_pair<true, true>(g, st, sms);
+    return launch_pair<true, false>(g, st, sms);
+  }
   const long tiles256 = static_cast<long>((g.M + BM - 1) / BM) * ((g.N + 255) / 256);
   if (g.N > 128 && tiles256 >= sms / 2) return launch_major<256>(g, st, sms);
   return launch_major<128>(g, st, sms);

@@ -27,6 +27,7 @@ struct GemmArgs {
   const __nv_bfloat16* B = nullptr; int ldb = 0; int b_mn = 0;
   int M = 0, N = 0, K = 0;
   GemmEpilogue ep;
+  int use_pair = -1;   // -1: auto, 0: never use the CTA-pair kernel, 1: always (if M, N >= 256)
 };
 
 cudaError_t gemm_bf16(const GemmArgs& g, cudaStream_t st);   // tcgen05 + TMA + TMEM

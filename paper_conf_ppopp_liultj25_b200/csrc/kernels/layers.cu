@@ -122,6 +122,91 @@ __global__ void norm_fwd_k(const T* x, const float* g, const float* b, T* y, flo
   if (lane == 0) { stats[2 * row] = mean; stats[2 * row + 1] = rstd; }
 }
 
+template <bool RMS>
+__global__ void norm_fwd_v8_k(const __nv_bfloat16* x, const float* g, const float* b, __nv_bfloat16* y, float* stats,
+                              int rows, int n, float eps) {
+  const int row = blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32, lane = threadIdx.x % 32;
+  if (row >= rows) return;
+  const __nv_bfloat16* xr = x + static_cast<long>(row) * n;
+  float mean = 0.f;
+  if (!RMS) {
+    float s = 0.f;
+    for (int c = lane * 8; c < n; c += 256) {
+      const uint4 u = *reinterpret_cast<const uint4*>(xr + c);
+      const __nv_bfloat16* hv = reinterpret_cast<const __nv_bfloat16*>(&u);
+#pragma unroll
+      for (int j = 0; j < 8; ++j) s += __bfloat162float(hv[j]);
+    }
+    mean = warp_sum(s) / n;
+  }
+  float v = 0.f;
+  for (int c = lane * 8; c < n; c += 256) {
+    const uint4 u = *reinterpret_cast<const uint4*>(xr + c);
+    const __nv_bfloat16* hv = reinterpret_cast<const __nv_bfloat16*>(&u);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) { const float d = __bfloat162float(hv[j]) - mean; v += d * d; }
+  }
+  const float rstd = rsqrtf(warp_sum(v) / n + eps);
+  __nv_bfloat16* yr = y + static_cast<long>(row) * n;
+  for (int c = lane * 8; c < n; c += 256) {
+    const uint4 u = *reinterpret_cast<const uint4*>(xr + c);
+    const __nv_bfloat16* hv = reinterpret_cast<const __nv_bfloat16*>(&u);
+    uint4 o;
+    __nv_bfloat16* ho = reinterpret_cast<__nv_bfloat16*>(&o);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      float t = (__bfloat162float(hv[j]) - mean) * rstd * g[c + j];
+      if (!RMS) t += b[c + j];
+      ho[j] = __float2bfloat16_rn(t);
+    }
+    *reinterpret_cast<uint4*>(yr + c) = o;
+  }
+  if (lane == 0) { stats[2 * row] = mean; stats[2 * row + 1] = rstd; }
+}
+
+__global__ void norm_bwd_dx_v8_k(const __nv_bfloat16* dy, const __nv_bfloat16* x, const float* stats, const float* g,
+                                 const __nv_bfloat16* dres, __nv_bfloat16* dx, int rows, int n, int rms) {
+  const int row = blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32, lane = threadIdx.x % 32;
+  if (row >= rows) return;
+  const long o = static_cast<long>(row) * n;
+  const float mean = stats[2 * row], rstd = stats[2 * row + 1];
+  float sg = 0.f, sgx = 0.f;
+  for (int c = lane * 8; c < n; c += 256) {
+    const uint4 ud = *reinterpret_cast<const uint4*>(dy + o + c);
+    const uint4 ux = *reinterpret_cast<const uint4*>(x + o + c);
+    const __nv_bfloat16* hd = reinterpret_cast<const __nv_bfloat16*>(&ud);
+    const __nv_bfloat16* hx = reinterpret_cast<const __nv_bfloat16*>(&ux);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const float gp = __bfloat162float(hd[j]) * g[c + j];
+      sg += gp;
+      sgx += gp * (__bfloat162float(hx[j]) - mean) * rstd;
+    }
+  }
+  sg = rms ? 0.f : warp_sum(sg) / n;
+  sgx = warp_sum(sgx) / n;
+  for (int c = lane * 8; c < n; c += 256) {
+    const uint4 ud = *reinterpret_cast<const uint4*>(dy + o + c);
+    const uint4 ux = *reinterpret_cast<const uint4*>(x + o + c);
+    const __nv_bfloat16* hd = reinterpret_cast<const __nv_bfloat16*>(&ud);
+    const __nv_bfloat16* hx = reinterpret_cast<const __nv_bfloat16*>(&ux);
+    uint4 ur = make_uint4(0, 0, 0, 0);
+    if (dres) ur = *reinterpret_cast<const uint4*>(dres + o + c);
+    const __nv_bfloat16* hr = reinterpret_cast<const __nv_bfloat16*>(&ur);
+    uint4 uo;
+    __nv_bfloat16* ho = reinterpret_cast<__nv_bfloat16*>(&uo);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const float gp = __bfloat162float(hd[j]) * g[c + j];
+      const float xh = (__bfloat162float(hx[j]) - mean) * rstd;
+      float d = (gp - sg - xh * sgx) * rstd;
+      if (dres) d += __bfloat162float(hr[j]);
+      ho[j] = __float2bfloat16_rn(d);
+    }
+    *reinterpret_cast<uint4*>(dx + o + c) = uo;
+  }
+}
+
 template <class T>
 __global__ void norm_bwd_dx_k(const T* dy, const T* x, const float* stats, const float* g, const T* dres, T* dx,
                               int rows, int n, int rms) {
@@ -166,6 +251,40 @@ __global__ void colsum_partial_k(const T* a, const T* x, const float* stats, int
   }
   partial[static_cast<long>(blk) * n + c] = s0;
   if (mode == 1) partial[static_cast<long>(nblk + blk) * n + c] = s1;
+}
+
+// bf16, n % 8 == 0: each thread owns 8 consecutive columns (16-byte loads).
+__global__ void colsum_partial_v8_k(const __nv_bfloat16* a, const __nv_bfloat16* x, const float* stats, int rows,
+                                    int n, int lda, int mode, float* partial, int nblk) {
+  const int c8 = (blockIdx.x * blockDim.x + threadIdx.x) * 8;
+  if (c8 >= n) return;
+  const int blk = blockIdx.y;
+  const int r0 = static_cast<int>(static_cast<long>(rows) * blk / nblk);
+  const int r1 = static_cast<int>(static_cast<long>(rows) * (blk + 1) / nblk);
+  float s0[8] = {0, 0, 0, 0, 0, 0, 0, 0}, s1[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  for (int r = r0; r < r1; ++r) {
+    const uint4 ua = *reinterpret_cast<const uint4*>(a + static_cast<long>(r) * lda + c8);
+    const __nv_bfloat16* ha = reinterpret_cast<const __nv_bfloat16*>(&ua);
+    if (mode == 0) {
+#pragma unroll
+      for (int j = 0; j < 8; ++j) s0[j] += __bfloat162float(ha[j]);
+      continue;
+    }
+    const uint4 ux = *reinterpret_cast<const uint4*>(x + static_cast<long>(r) * n + c8);
+    const __nv_bfloat16* hx = reinterpret_cast<const __nv_bfloat16*>(&ux);
+    const float mu = stats[2 * r], rs = stats[2 * r + 1];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const float dy = __bfloat162float(ha[j]);
+      s0[j] += dy * ((__bfloat162float(hx[j]) - mu) * rs);
+      s1[j] += dy;
+    }
+  }
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    partial[static_cast<long>(blk) * n + c8 + j] = s0[j];
+    if (mode == 1) partial[static_cast<long>(nblk + blk) * n + c8 + j] = s1[j];
+  }
 }
 
 __global__ void colsum_final_k(const float* partial, int nblk, int n, int mode, float* out0, float* out1) {
@@ -493,17 +612,26 @@ void embed_bwd(const int32_t* tok, int ld_tok, int B, int s, const T* dH, int h,
 
 template <class T>
 void layernorm_fwd(const T* x, const float* g, const float* b, T* y, float* stats, int rows, int n, float eps, cudaStream_t st) {
+  if constexpr (std::is_same<T, __nv_bfloat16>::value) {
+    if (n % 8 == 0) { norm_fwd_v8_k<false><<<cdiv(rows, 8), 256, 0, st>>>(x, g, b, y, stats, rows, n, eps); note_launch(); return; }
+  }
   norm_fwd_k<T, false><<<cdiv(rows, 8), 256, 0, st>>>(x, g, b, y, stats, rows, n, eps);
   note_launch();
 }
 template <class T>
 void rmsnorm_fwd(const T* x, const float* g, T* y, float* stats, int rows, int n, float eps, cudaStream_t st) {
+  if constexpr (std::is_same<T, __nv_bfloat16>::value) {
+    if (n % 8 == 0) { norm_fwd_v8_k<true><<<cdiv(rows, 8), 256, 0, st>>>(x, g, nullptr, y, stats, rows, n, eps); note_launch(); return; }
+  }
   norm_fwd_k<T, true><<<cdiv(rows, 8), 256, 0, st>>>(x, g, nullptr, y, stats, rows, n, eps);
   note_launch();
 }
 template <class T>
 void norm_bwd_dx(const T* dy, const T* x, const float* stats, const float* g, const T* dres, T* dx, int rows, int n,
                  int rms, cudaStream_t st) {
+  if constexpr (std::is_same<T, __nv_bfloat16>::value) {
+    if (n % 8 == 0) { norm_bwd_dx_v8_k<<<cdiv(rows, 8), 256, 0, st>>>(dy, x, stats, g, dres, dx, rows, n, rms); note_launch(); return; }
+  }
   norm_bwd_dx_k<T><<<cdiv(rows, 8), 256, 0, st>>>(dy, x, stats, g, dres, dx, rows, n, rms);
   note_launch();
 }
@@ -512,6 +640,16 @@ void colsum(const T* a, const T* x, const float* stats, int rows, int n, int lda
             float* partial, cudaStream_t st) {
   int nblk = rows < 128 ? rows : 128;
   if (nblk < 1) return;
+  if constexpr (std::is_same<T, __nv_bfloat16>::value) {
+    if (n % 8 == 0 && lda % 8 == 0) {
+      dim3 grid(cdiv(n / 8, 128), nblk);
+      colsum_partial_v8_k<<<grid, 128, 0, st>>>(a, x, stats, rows, n, lda, mode == 2 ? 1 : mode, partial, nblk);
+      note_launch();
+      colsum_final_k<<<cdiv(n, 256), 256, 0, st>>>(partial, nblk, n, mode == 2 ? 0 : mode, out0, out1);
+      note_launch();
+      return;
+    }
+  }
   dim3 grid(cdiv(n, 256), nblk);
   colsum_partial_k<T><<<grid, 256, 0, st>>>(a, x, stats, rows, n, lda, mode == 2 ? 1 : mode, partial, nblk);
   note_launch();

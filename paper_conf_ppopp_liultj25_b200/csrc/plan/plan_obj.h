@@ -38,5 +38,6 @@ struct mario_plan {
   // global execution order used by loopback (device, list index), round-robin like the simulator
   std::vector<std::pair<int, int>> loopback_order;
   std::string serialized;
+  std::vector<std::vector<mario_commop>> comm_ops;   // per rank, issue order
 };
 typedef struct mario_plan PlanObj;

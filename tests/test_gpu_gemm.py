@@ -53,18 +53,26 @@ def _run(a_mn, b_mn, M, N, K, out_f32, bias=False, resid=False, gelu2=False, aux
         assert (D2.float() - gref).abs().max().item() <= 2e-2 * gref.abs().max().item() + 1e-2
 
 
+@pytest.fixture(params=[0, 1], ids=["single_cta", "cta_pair"])
+def variant(request):
+    L = _lib.lib()
+    assert L.mario_k_gemm_set_variant(request.param) == 0
+    yield request.param
+    L.mario_k_gemm_set_variant(-1)
+
+
 @pytest.mark.parametrize("a_mn,b_mn", [(0, 0), (0, 1), (1, 1), (1, 0)])
-@pytest.mark.parametrize("M,N,K", SHAPES)
-def test_gemm_bf16_majors(a_mn, b_mn, M, N, K):
+@pytest.mark.parametrize("M,N,K", SHAPES + [(768, 1280, 320), (520, 264, 200)])
+def test_gemm_bf16_majors(a_mn, b_mn, M, N, K, variant):
     _run(a_mn, b_mn, M, N, K, out_f32=False)
 
 
-@pytest.mark.parametrize("M,N,K", SHAPES[:4])
-def test_gemm_bf16_wgrad_accumulate(M, N, K):
+@pytest.mark.parametrize("M,N,K", SHAPES[:4] + [(768, 1280, 320)])
+def test_gemm_bf16_wgrad_accumulate(M, N, K, variant):
     _run(1, 1, M, N, K, out_f32=True, beta=1.0)
 
 
-def test_gemm_bf16_epilogues():
+def test_gemm_bf16_epilogues(variant):
     _run(0, 0, 384, 640, 256, out_f32=False, bias=True, resid=True)
     _run(0, 0, 384, 640, 256, out_f32=False, bias=True, gelu2=True)
     _run(0, 1, 384, 640, 256, out_f32=False, aux=True)

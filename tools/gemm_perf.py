@@ -8,7 +8,10 @@ L = _lib.lib()
 shapes = [("qkv", 8192, 6144, 2048), ("proj", 8192, 2048, 2048), ("fc1", 8192, 8192, 2048),
           ("fc2", 8192, 2048, 8192), ("head", 8192, 50304, 2048), ("sq8k", 8192, 8192, 8192)]
 res = []
-for name, M, N, K in shapes:
+VARIANTS = [int(v) for v in (sys.argv[1].split(",") if len(sys.argv) > 1 else ["0", "1"])]
+for variant in VARIANTS:
+  L.mario_k_gemm_set_variant(variant)
+  for name, M, N, K in shapes:
     for mode in ("fwd", "dgrad", "wgrad"):
         if mode == "fwd":
             A = torch.randn(M, K, device="cuda").bfloat16(); B = torch.randn(N, K, device="cuda").bfloat16()
@@ -43,6 +46,6 @@ for name, M, N, K in shapes:
         e1.record(); torch.cuda.synchronize()
         ms_ref = e0.elapsed_time(e1) / it
         tf = 2.0 * M * N * K / ms / 1e9
-        res.append(dict(name=name, mode=mode, M=m, N=n, K=k, ms=round(ms, 4), tflops=round(tf, 1),
+        res.append(dict(variant=variant, name=name, mode=mode, M=m, N=n, K=k, ms=round(ms, 4), tflops=round(tf, 1),
                         cublas_tflops=round(2.0 * M * N * K / ms_ref / 1e9, 1)))
         print(json.dumps(res[-1]), flush=True)
