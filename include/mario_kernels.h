@@ -48,6 +48,9 @@ int mario_k_gemm_f32(const float* A, int lda, int a_mn, const float* B, int ldb,
  * (head_dim in {16,32,64,80,128}), else fp32. */
 int mario_k_attn_fwd(const void* qkv, void* O, float* lse, int B, int s, int n_heads, int head_dim,
                      int bf16, void* stream);
+/* Kernel selection for K5/K6 (bf16): -1 = auto (tcgen05 backward for head_dim 64/128, mma.sync
+ * otherwise), 0 = mma.sync only. Process-global; returns 0, or 1 for an invalid value. */
+int mario_k_attn_set_variant(int variant);
 /* K6: backward: dqkv [B*s][3*H] (dQ | dK | dV) from dO [B*s][H], with P recomputed from lse;
  * deterministic (no atomics). scratch: fp32 [n_heads][B*s]. */
 int mario_k_attn_bwd(const void* qkv, const void* O, const void* dO, const float* lse, void* dqkv,

@@ -23,6 +23,7 @@ _SIGS = {
     "mario_k_attn_bwd": (i32, [vp, vp, vp, vp, vp, vp, i32, i32, i32, i32, i32, vp]),
     "mario_kernel_launches": (C.c_longlong, []),
     "mario_k_gemm_set_variant": (i32, [i32]),
+    "mario_k_attn_set_variant": (i32, [i32]),
     "mario_kstats_enable": (i32, [i32]),
     "mario_kstats_read": (i32, [i32, C.POINTER(C.c_double), C.POINTER(C.c_double), C.POINTER(C.c_double),
                                 C.POINTER(C.c_longlong)]),

@@ -11,6 +11,11 @@
 #include "kstats.h"
 
 namespace mario {
+
+int g_attn_variant = -1;   // mario_k_attn_set_variant: -1 auto (tcgen05 where supported), 0 mma.sync only
+bool flash_attn_bwd_tc(const __nv_bfloat16* qkv, const __nv_bfloat16* dO, const float* lse, const float* Dd,
+                       __nv_bfloat16* dqkv, int B, int s, int nh, int dh, cudaStream_t st);   // attn_tc.cu
+
 namespace {
 
 using bf16 = __nv_bfloat16;
@@ -429,6 +434,13 @@ void launch_bwd(const bf16* qkv, const bf16* O, const bf16* dO, const float* lse
                 int nh, cudaStream_t st) {
   const long Ttok = static_cast<long>(B) * s;
   fa_bwd_dot_k<<<static_cast<int>((Ttok * nh * 32 + 255) / 256), 256, 0, st>>>(O, dO, Dd, Ttok, nh, D);
+  if (g_attn_variant != 0) {   // tcgen05 backward (attn_tc.cu) when supported
+    const double fl = 8.0 * B * nh * D * (static_cast<double>(s) * (s + 1) / 2);
+    const int tok = kstats_begin(K_ATTN_BWD, fl, 0.0, st);
+    const bool ok = flash_attn_bwd_tc(qkv, dO, lse, Dd, dqkv, B, s, nh, D, st);
+    kstats_end(tok, st);
+    if (ok) { note_launch(); return; }
+  }
   constexpr size_t smem_kv = (2 * BR + 2 * BCB) * (D + 8) * sizeof(bf16) + 2 * BCB * sizeof(float);
   constexpr size_t smem_q = (2 * BR + 2 * BCB) * (D + 8) * sizeof(bf16);
   static bool set = false;

@@ -1,0 +1,495 @@
+// K6 on tcgen05: causal flash-attention backward for bf16, head_dim 64 / 128.
+// Same math as attn_mma.cu / SURVEY §8(c) c1:  P = exp(S - lse), dS = P (dP - D),
+//   dV = P^T dO,  dK = dS^T Q / sqrt(dh),  dQ = dS K / sqrt(dh),   D = rowsum(dO * O).
+//
+// dK/dV kernel: one CTA per 128 keys (= 128 TMEM lanes) of one (sample, head); loop over
+// 64-query tiles q >= first key:
+//   warp 0      TMA: K, V once; Q_i / dO_i into a 2-stage ring (128B swizzle)
+//   warp 1      single-thread tcgen05.mma:  S^T = K Q_i^T, dP^T = V dO_i^T  (M128 N64, into a
+//               double-buffered TMEM pair), then dV += P^T dO_i, dK += dS^T Q_i (M128 N=dh,
+//               accumulated in TMEM across the whole loop). The Q_i / dO_i tiles are read as
+//               K-major B for the first products and as MN-major B for the second.
+//   warps 2..5  one key row per thread: tcgen05.ld S^T, dP^T rows -> P^T, dS^T (bf16) into
+//               swizzled smem for the next MMAs; epilogue tcgen05.ld dK, dV -> global.
+// dQ kernel: the mirror image (128 queries per CTA, loop over 64-key tiles, dQ += dS K).
+// No atomics: deterministic.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+#include <cuda_runtime.h>
+#include <cuda_bf16.h>
+#include <cstdio>
+#include <cstdlib>
+
+#include "kstats.h"
+#include "layers.h"
+#include "sm100.cuh"
+
+namespace mario {
+
+bool make_tmap_bf16_2d(CUtensorMap* map, const void* base, uint64_t inner, uint64_t outer, uint64_t ld,
+                       uint32_t box_inner, uint32_t box_outer);   // gemm_tc.cu
+
+namespace {
+using namespace sm100;
+using bf16 = __nv_bfloat16;
+constexpr float LOG2E = 1.4426950408889634f;
+constexpr int kRows = 128;   // rows per CTA (TMEM lanes)
+constexpr int kCols = 64;    // inner tile
+constexpr int kThreads = 192;
+
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
+__device__ __forceinline__ void named_bar(int id, int n) { asm volatile("bar.sync %0, %1;" :: "r"(id), "r"(n) : "memory"); }
+
+// write 64 bf16 values (one 128-byte row) of a K-major SW128 tile with 128-byte rows
+__device__ __forceinline__ void st_row_sw128(uint8_t* tile, int row, const float (&v)[64]) {
+  uint8_t* rp = tile + row * 128;
+#pragma unroll
+  for (int j = 0; j < 8; ++j) {
+    uint4 u;
+    __nv_bfloat162* h = reinterpret_cast<__nv_bfloat162*>(&u);
+#pragma unroll
+    for (int e = 0; e < 4; ++e) h[e] = __floats2bfloat162_rn(v[8 * j + 2 * e], v[8 * j + 2 * e + 1]);
+    *reinterpret_cast<uint4*>(rp + ((j ^ (row & 7)) << 4)) = u;
+  }
+}
+
+template <int DH>
+struct Smem {
+  static constexpr int kBig = kRows * DH * 2;        // 128-row tile (K,V or Q,dO)
+  static constexpr int kSmall = kCols * DH * 2;      // 64-row tile
+  static constexpr int kP = kRows * kCols * 2;       // 128 x 64 bf16
+};
+
+// ------------------------------------------------------------------------ dK / dV
+template <int DH>
+__global__ void __launch_bounds__(kThreads, 1)
+fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_qkv64,
+               const __grid_constant__ CUtensorMap tm_do64, const float* lse, const float* Dd, bf16* dqkv, int B,
+               int s, int nh) {
+  using SM = Smem<DH>;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sK = smem;
+  uint8_t* sV = sK + SM::kBig;
+  uint8_t* sQ[2] = {sV + SM::kBig, sV + SM::kBig + 2 * SM::kSmall};
+  uint8_t* sG[2] = {sQ[0] + SM::kSmall, sQ[1] + SM::kSmall};
+  uint8_t* sP = sV + SM::kBig + 4 * SM::kSmall;
+  uint8_t* sS = sP + SM::kP;    // dS^T
+  float* sL = reinterpret_cast<float*>(sS + SM::kP);       // [2][64] lse * log2e
+  float* sDv = sL + 2 * kCols;                             // [2][64] D
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sDv + 2 * kCols);
+  uint64_t* kv_full = bar;          // 1
+  uint64_t* q_full = bar + 1;       // 2
+  uint64_t* q_empty = bar + 3;      // 2
+  uint64_t* s_full = bar + 5;       // 2
+  uint64_t* s_free = bar + 7;       // 2
+  uint64_t* p_full = bar + 9;       // 1
+  uint64_t* p_free = bar + 10;      // 1
+  uint64_t* acc_done = bar + 11;    // 1
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 12);
+
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int kt = blockIdx.x, b = blockIdx.y / nh, head = blockIdx.y % nh;
+  const int h = nh * DH;
+  const long Ttok = static_cast<long>(B) * s;
+  const int i0 = (kt * kRows) / kCols;
+  const int nq = (s + kCols - 1) / kCols;
+  const int ntiles = nq - i0;
+  const float sl2 = rsqrtf(static_cast<float>(DH)) * LOG2E;
+
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&tm_qkv128);
+    tma_prefetch_desc(&tm_qkv64);
+    tma_prefetch_desc(&tm_do64);
+    mbar_init(kv_full, 1);
+    for (int i = 0; i < 2; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); mbar_init(&s_full[i], 1); mbar_init(&s_free[i], 4); }
+    mbar_init(p_full, 4);
+    mbar_init(p_free, 1);
+    mbar_init(acc_done, 1);
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc<512>(tmem_slot);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tm = *tmem_slot;
+  const uint32_t tm_dV = tm, tm_dK = tm + DH, tm_S = tm + 2 * DH, tm_dP = tm + 2 * DH + 2 * kCols;
+
+  if (ntiles <= 0) {  // keys entirely beyond the sample: nothing to do (dK = dV = 0 not needed: rows >= s)
+    __syncthreads();
+    if (warp == 1) tmem_dealloc<512>(tm);
+    return;
+  }
+
+  if (warp == 0) {
+    if (elect_one()) {
+      const int row0 = b * s;
+      mbar_arrive_expect_tx(kv_full, 2 * SM::kBig);
+#pragma unroll
+      for (int a = 0; a < DH / 64; ++a) {
+        tma_load_2d(sK + a * (kRows * 128), &tm_qkv128, kv_full, h + head * DH + a * 64, row0 + kt * kRows);
+        tma_load_2d(sV + a * (kRows * 128), &tm_qkv128, kv_full, 2 * h + head * DH + a * 64, row0 + kt * kRows);
+      }
+      for (int idx = 0; idx < ntiles; ++idx) {
+        const int st = idx & 1;
+        mbar_wait(&q_empty[st], ((idx >> 1) & 1) ^ 1);
+        mbar_arrive_expect_tx(&q_full[st], 2 * SM::kSmall);
+        const int qr = row0 + (i0 + idx) * kCols;
+#pragma unroll
+        for (int a = 0; a < DH / 64; ++a) {
+          tma_load_2d(sQ[st] + a * (kCols * 128), &tm_qkv64, &q_full[st], head * DH + a * 64, qr);
+          tma_load_2d(sG[st] + a * (kCols * 128), &tm_do64, &q_full[st], head * DH + a * 64, qr);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    constexpr uint32_t id_s = umma_idesc_bf16(128, kCols, 0, 0);   // S^T, dP^T: K-major A and B
+    constexpr uint32_t id_a = umma_idesc_bf16(128, DH, 0, 1);      // dV, dK: B = Q/dO read MN-major
+    mbar_wait(kv_full, 0);
+    tc_fence_after();
+    auto issue_s = [&](int idx) {
+      const int st = idx & 1, buf = idx & 1;
+      mbar_wait(&q_full[st], (idx >> 1) & 1);
+      mbar_wait(&s_free[buf], ((idx >> 1) & 1) ^ 1);
+      tc_fence_after();
+      if (elect_one()) {
+        const uint32_t k = smem_u32(sK), v = smem_u32(sV), q = smem_u32(sQ[st]), g = smem_u32(sG[st]);
+#pragma unroll
+        for (int kk = 0; kk < DH / 16; ++kk) {
+          const uint32_t ao = (kk >> 2) * (kRows * 128) + (kk & 3) * 32, bo = (kk >> 2) * (kCols * 128) + (kk & 3) * 32;
+          umma_bf16(tm_S + buf * kCols, umma_desc_sw128(k + ao, 16, 1024), umma_desc_sw128(q + bo, 16, 1024), id_s, kk > 0);
+          umma_bf16(tm_dP + buf * kCols, umma_desc_sw128(v + ao, 16, 1024), umma_desc_sw128(g + bo, 16, 1024), id_s, kk > 0);
+        }
+        umma_commit(&s_full[buf]);
+      }
+      __syncwarp();
+    };
+    auto issue_acc = [&](int idx) {
+      const int st = idx & 1;
+      mbar_wait(p_full, idx & 1);
+      tc_fence_after();
+      if (elect_one()) {
+        const uint32_t p = smem_u32(sP), ds = smem_u32(sS), q = smem_u32(sQ[st]), g = smem_u32(sG[st]);
+#pragma unroll
+        for (int kk = 0; kk < kCols / 16; ++kk) {
+          const uint64_t pa = umma_desc_sw128(p + kk * 32, 16, 1024), sa = umma_desc_sw128(ds + kk * 32, 16, 1024);
+          umma_bf16(tm_dV, pa, umma_desc_sw128(g + kk * 2048, kCols * 128, 1024), id_a, (idx | kk) != 0);
+          umma_bf16(tm_dK, sa, umma_desc_sw128(q + kk * 2048, kCols * 128, 1024), id_a, (idx | kk) != 0);
+        }
+        umma_commit(p_free);
+        umma_commit(&q_empty[st]);
+        if (idx == ntiles - 1) umma_commit(acc_done);
+      }
+      __syncwarp();
+    };
+    issue_s(0);
+    for (int idx = 1; idx < ntiles; ++idx) {
+      issue_s(idx);
+      issue_acc(idx - 1);
+    }
+    issue_acc(ntiles - 1);
+  } else {
+    const int quarter = warp & 3;
+    const int row = quarter * 32 + lane;             // key row within the tile
+    const int key = kt * kRows + row;
+    const uint32_t lane_off = static_cast<uint32_t>(quarter * 32) << 16;
+    const int tid = threadIdx.x - 64;                // 0..127
+    for (int idx = 0; idx < ntiles; ++idx) {
+      const int buf = idx & 1, i = i0 + idx;
+      // lse / D of this query tile into smem (threads 0..63: lse, 64..127: D)
+      {
+        const int c = tid & 63, qq = i * kCols + c;
+        const long r = static_cast<long>(b) * s + (qq < s ? qq : 0);
+        if (tid < 64) sL[buf * kCols + c] = lse[static_cast<long>(head) * Ttok + r] * LOG2E;
+        else sDv[buf * kCols + c] = Dd[static_cast<long>(head) * Ttok + r];
+      }
+      named_bar(1, 128);
+      mbar_wait(&s_full[buf], (idx >> 1) & 1);
+      tc_fence_after();
+      uint32_t sr[64], dr[64];
+      tmem_ld_32x32b_x32(tm_S + buf * kCols + lane_off, *reinterpret_cast<uint32_t(*)[32]>(sr));
+      tmem_ld_32x32b_x32(tm_S + buf * kCols + 32 + lane_off, *reinterpret_cast<uint32_t(*)[32]>(sr + 32));
+      tmem_ld_32x32b_x32(tm_dP + buf * kCols + lane_off, *reinterpret_cast<uint32_t(*)[32]>(dr));
+      tmem_ld_32x32b_x32(tm_dP + buf * kCols + 32 + lane_off, *reinterpret_cast<uint32_t(*)[32]>(dr + 32));
+      tmem_ld_wait();
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&s_free[buf]);
+      float p[64], ds[64];
+#pragma unroll
+      for (int c = 0; c < 64; ++c) {
+        const int qq = i * kCols + c;
+        float pv = exp2f(__uint_as_float(sr[c]) * sl2 - sL[buf * kCols + c]);
+        if (qq < key || qq >= s) pv = 0.f;
+        p[c] = pv;
+        ds[c] = pv * (__uint_as_float(dr[c]) - sDv[buf * kCols + c]);
+      }
+      mbar_wait(p_free, (idx & 1) ^ 1);   // previous tile's dV/dK MMAs have consumed sP/sS
+      st_row_sw128(sP, row, p);
+      st_row_sw128(sS, row, ds);
+      fence_proxy_async();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(p_full);
+    }
+    // epilogue: dV, dK rows of this thread's key
+    mbar_wait(acc_done, 0);
+    tc_fence_after();
+    // tcgen05.ld is warp-collective (.sync.aligned): every lane loads, only valid keys store
+    const float scale = rsqrtf(static_cast<float>(DH));
+    const long krow_idx = static_cast<long>(b) * s + (key < s ? key : 0);
+    bf16* krow = dqkv + krow_idx * (3 * h) + h + head * DH;
+    bf16* vrow = krow + h;
+#pragma unroll 1
+    for (int c = 0; c < DH; c += 32) {
+      uint32_t rv[32], rk[32];
+      tmem_ld_32x32b_x32(tm_dV + c + lane_off, rv);
+      tmem_ld_32x32b_x32(tm_dK + c + lane_off, rk);
+      tmem_ld_wait();
+      if (key < s) {
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+          uint4 uv, uk;
+          __nv_bfloat162* hv = reinterpret_cast<__nv_bfloat162*>(&uv);
+          __nv_bfloat162* hk = reinterpret_cast<__nv_bfloat162*>(&uk);
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            hv[e] = __floats2bfloat162_rn(__uint_as_float(rv[8 * q + 2 * e]), __uint_as_float(rv[8 * q + 2 * e + 1]));
+            hk[e] = __floats2bfloat162_rn(__uint_as_float(rk[8 * q + 2 * e]) * scale,
+                                          __uint_as_float(rk[8 * q + 2 * e + 1]) * scale);
+          }
+          *reinterpret_cast<uint4*>(vrow + c + 8 * q) = uv;
+          *reinterpret_cast<uint4*>(krow + c + 8 * q) = uk;
+        }
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) tmem_dealloc<512>(tm);
+}
+
+// ------------------------------------------------------------------------------ dQ
+template <int DH>
+__global__ void __launch_bounds__(kThreads, 1)
+fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_qkv64,
+             const __grid_constant__ CUtensorMap tm_do128, const float* lse, const float* Dd, bf16* dqkv, int B, int s,
+             int nh) {
+  using SM = Smem<DH>;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sQ = smem;
+  uint8_t* sG = sQ + SM::kBig;
+  uint8_t* sK[2] = {sG + SM::kBig, sG + SM::kBig + 2 * SM::kSmall};
+  uint8_t* sV[2] = {sK[0] + SM::kSmall, sK[1] + SM::kSmall};
+  uint8_t* sS = sG + SM::kBig + 4 * SM::kSmall;   // dS [128 q][64 keys]
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sS + SM::kP);
+  uint64_t* q_fullb = bar;          // Q, dO loaded
+  uint64_t* k_full = bar + 1;       // 2
+  uint64_t* k_empty = bar + 3;      // 2
+  uint64_t* s_full = bar + 5;       // 2
+  uint64_t* s_free = bar + 7;       // 2
+  uint64_t* p_full = bar + 9;
+  uint64_t* p_free = bar + 10;
+  uint64_t* acc_done = bar + 11;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 12);
+
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int qt = blockIdx.x, b = blockIdx.y / nh, head = blockIdx.y % nh;
+  const int h = nh * DH;
+  const long Ttok = static_cast<long>(B) * s;
+  const int last_q = min(qt * kRows + kRows - 1, s - 1);
+  const int ntiles = last_q / kCols + 1;   // key tiles 0 .. last_q/64
+  const float sl2 = rsqrtf(static_cast<float>(DH)) * LOG2E;
+
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&tm_qkv128);
+    tma_prefetch_desc(&tm_qkv64);
+    tma_prefetch_desc(&tm_do128);
+    mbar_init(q_fullb, 1);
+    for (int i = 0; i < 2; ++i) { mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1); mbar_init(&s_full[i], 1); mbar_init(&s_free[i], 4); }
+    mbar_init(p_full, 4);
+    mbar_init(p_free, 1);
+    mbar_init(acc_done, 1);
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc<512>(tmem_slot);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tm = *tmem_slot;
+  const uint32_t tm_dQ = tm, tm_S = tm + DH, tm_dP = tm + DH + 2 * kCols;
+
+  if (warp == 0) {
+    if (elect_one()) {
+      const int row0 = b * s;
+      mbar_arrive_expect_tx(q_fullb, 2 * SM::kBig);
+#pragma unroll
+      for (int a = 0; a < DH / 64; ++a) {
+        tma_load_2d(sQ + a * (kRows * 128), &tm_qkv128, q_fullb, head * DH + a * 64, row0 + qt * kRows);
+        tma_load_2d(sG + a * (kRows * 128), &tm_do128, q_fullb, head * DH + a * 64, row0 + qt * kRows);
+      }
+      for (int idx = 0; idx < ntiles; ++idx) {
+        const int st = idx & 1;
+        mbar_wait(&k_empty[st], ((idx >> 1) & 1) ^ 1);
+        mbar_arrive_expect_tx(&k_full[st], 2 * SM::kSmall);
+        const int kr = row0 + idx * kCols;
+#pragma unroll
+        for (int a = 0; a < DH / 64; ++a) {
+          tma_load_2d(sK[st] + a * (kCols * 128), &tm_qkv64, &k_full[st], h + head * DH + a * 64, kr);
+          tma_load_2d(sV[st] + a * (kCols * 128), &tm_qkv64, &k_full[st], 2 * h + head * DH + a * 64, kr);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    constexpr uint32_t id_s = umma_idesc_bf16(128, kCols, 0, 0);
+    constexpr uint32_t id_a = umma_idesc_bf16(128, DH, 0, 1);   // dQ += dS K: B = K_j read MN-major
+    mbar_wait(q_fullb, 0);
+    tc_fence_after();
+    auto issue_s = [&](int idx) {
+      const int st = idx & 1, buf = idx & 1;
+      mbar_wait(&k_full[st], (idx >> 1) & 1);
+      mbar_wait(&s_free[buf], ((idx >> 1) & 1) ^ 1);
+      tc_fence_after();
+      if (elect_one()) {
+        const uint32_t q = smem_u32(sQ), g = smem_u32(sG), k = smem_u32(sK[st]), v = smem_u32(sV[st]);
+#pragma unroll
+        for (int kk = 0; kk < DH / 16; ++kk) {
+          const uint32_t ao = (kk >> 2) * (kRows * 128) + (kk & 3) * 32, bo = (kk >> 2) * (kCols * 128) + (kk & 3) * 32;
+          umma_bf16(tm_S + buf * kCols, umma_desc_sw128(q + ao, 16, 1024), umma_desc_sw128(k + bo, 16, 1024), id_s, kk > 0);
+          umma_bf16(tm_dP + buf * kCols, umma_desc_sw128(g + ao, 16, 1024), umma_desc_sw128(v + bo, 16, 1024), id_s, kk > 0);
+        }
+        umma_commit(&s_full[buf]);
+      }
+      __syncwarp();
+    };
+    auto issue_acc = [&](int idx) {
+      const int st = idx & 1;
+      mbar_wait(p_full, idx & 1);
+      tc_fence_after();
+      if (elect_one()) {
+        const uint32_t ds = smem_u32(sS), k = smem_u32(sK[st]);
+#pragma unroll
+        for (int kk = 0; kk < kCols / 16; ++kk)
+          umma_bf16(tm_dQ, umma_desc_sw128(ds + kk * 32, 16, 1024), umma_desc_sw128(k + kk * 2048, kCols * 128, 1024),
+                    id_a, (idx | kk) != 0);
+        umma_commit(p_free);
+        umma_commit(&k_empty[st]);
+        if (idx == ntiles - 1) umma_commit(acc_done);
+      }
+      __syncwarp();
+    };
+    issue_s(0);
+    for (int idx = 1; idx < ntiles; ++idx) {
+      issue_s(idx);
+      issue_acc(idx - 1);
+    }
+    issue_acc(ntiles - 1);
+  } else {
+    const int quarter = warp & 3;
+    const int row = quarter * 32 + lane;
+    const int q = qt * kRows + row;
+    const uint32_t lane_off = static_cast<uint32_t>(quarter * 32) << 16;
+    const long gr = static_cast<long>(b) * s + (q < s ? q : 0);
+    const float L = lse[static_cast<long>(head) * Ttok + gr] * LOG2E;
+    const float Dr = Dd[static_cast<long>(head) * Ttok + gr];
+    for (int idx = 0; idx < ntiles; ++idx) {
+      const int buf = idx & 1;
+      mbar_wait(&s_full[buf], (idx >> 1) & 1);
+      tc_fence_after();
+      uint32_t sr[64], dr[64];
+      tmem_ld_32x32b_x32(tm_S + buf * kCols + lane_off, *reinterpret_cast<uint32_t(*)[32]>(sr));
+      tmem_ld_32x32b_x32(tm_S + buf * kCols + 32 + lane_off, *reinterpret_cast<uint32_t(*)[32]>(sr + 32));
+      tmem_ld_32x32b_x32(tm_dP + buf * kCols + lane_off, *reinterpret_cast<uint32_t(*)[32]>(dr));
+      tmem_ld_32x32b_x32(tm_dP + buf * kCols + 32 + lane_off, *reinterpret_cast<uint32_t(*)[32]>(dr + 32));
+      tmem_ld_wait();
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&s_free[buf]);
+      float ds[64];
+#pragma unroll
+      for (int c = 0; c < 64; ++c) {
+        const int key = idx * kCols + c;
+        float pv = exp2f(__uint_as_float(sr[c]) * sl2 - L);
+        if (key > q) pv = 0.f;
+        ds[c] = pv * (__uint_as_float(dr[c]) - Dr);
+      }
+      mbar_wait(p_free, (idx & 1) ^ 1);
+      st_row_sw128(sS, row, ds);
+      fence_proxy_async();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(p_full);
+    }
+    mbar_wait(acc_done, 0);
+    tc_fence_after();
+    const float scale = rsqrtf(static_cast<float>(DH));
+    bf16* qrow = dqkv + gr * (3 * h) + head * DH;
+#pragma unroll 1
+    for (int c = 0; c < DH; c += 32) {
+      uint32_t rq[32];
+      tmem_ld_32x32b_x32(tm_dQ + c + lane_off, rq);
+      tmem_ld_wait();
+      if (q < s) {
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          uint4 u;
+          __nv_bfloat162* hq = reinterpret_cast<__nv_bfloat162*>(&u);
+#pragma unroll
+          for (int f = 0; f < 4; ++f)
+            hq[f] = __floats2bfloat162_rn(__uint_as_float(rq[8 * e + 2 * f]) * scale, __uint_as_float(rq[8 * e + 2 * f + 1]) * scale);
+          *reinterpret_cast<uint4*>(qrow + c + 8 * e) = u;
+        }
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) tmem_dealloc<512>(tm);
+}
+
+// >= 116 KB so that one CTA owns the SM (each allocates all 512 TMEM columns)
+constexpr int at_least_one_sm(int b) { return b < 116 * 1024 ? 116 * 1024 : b; }
+template <int DH>
+constexpr int smem_dkdv() { return at_least_one_sm(2 * Smem<DH>::kBig + 4 * Smem<DH>::kSmall + 2 * Smem<DH>::kP + 4 * kCols * 4 + 128 + 1024); }
+template <int DH>
+constexpr int smem_dq() { return at_least_one_sm(2 * Smem<DH>::kBig + 4 * Smem<DH>::kSmall + Smem<DH>::kP + 128 + 1024); }
+
+template <int DH>
+bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, bf16* dqkv, int B, int s, int nh,
+            cudaStream_t st) {
+  const int h = nh * DH;
+  const long T = static_cast<long>(B) * s;
+  CUtensorMap m128, m64, d64, d128;
+  if (!make_tmap_bf16_2d(&m128, qkv, 3 * h, T, 3 * h, 64, 128) || !make_tmap_bf16_2d(&m64, qkv, 3 * h, T, 3 * h, 64, 64) ||
+      !make_tmap_bf16_2d(&d64, dO, h, T, h, 64, 64) || !make_tmap_bf16_2d(&d128, dO, h, T, h, 64, 128))
+    return false;
+  static bool set = false;
+  if (!set) {
+    cudaFuncSetAttribute(fa_bwd_dkdv_tc<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_dkdv<DH>());
+    cudaFuncSetAttribute(fa_bwd_dq_tc<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_dq<DH>());
+    set = true;
+  }
+  dim3 grid((s + kRows - 1) / kRows, B * nh);
+  const char* only = getenv("MARIO_ATTN_TC_ONLY");   // debugging aid: "dkdv" or "dq"
+  if (!only || only[1] == 'k')
+    fa_bwd_dkdv_tc<DH><<<grid, kThreads, smem_dkdv<DH>(), st>>>(m128, m64, d64, lse, Dd, dqkv, B, s, nh);
+  if (!only || only[1] == 'q')
+    fa_bwd_dq_tc<DH><<<grid, kThreads, smem_dq<DH>(), st>>>(m128, m64, d128, lse, Dd, dqkv, B, s, nh);
+  note_launch(2);
+  return true;
+}
+
+}  // namespace
+
+bool flash_attn_bwd_tc_supported(int dh, int B, int s, int nh) {
+  return (dh == 64 || dh == 128) && ((nh * dh) % 64 == 0);
+}
+
+// Returns false if the configuration is unsupported (caller falls back to the mma.sync kernels).
+bool flash_attn_bwd_tc(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, bf16* dqkv, int B, int s,
+                       int nh, int dh, cudaStream_t st) {
+  if (dh == 128) return launch<128>(qkv, dO, lse, Dd, dqkv, B, s, nh, st);
+  if (dh == 64) return launch<64>(qkv, dO, lse, Dd, dqkv, B, s, nh, st);
+  return false;
+}
+
+}  // namespace mario

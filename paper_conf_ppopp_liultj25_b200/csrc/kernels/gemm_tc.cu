@@ -479,6 +479,11 @@ cudaError_t launch_major(const GemmArgs& g, cudaStream_t st, int num_sms) {
 
 }  // namespace
 
+bool make_tmap_bf16_2d(CUtensorMap* map, const void* base, uint64_t inner, uint64_t outer, uint64_t ld,
+                       uint32_t box_inner, uint32_t box_outer) {
+  return make_tmap(map, base, inner, outer, ld, box_inner, box_outer);
+}
+
 int device_sm_count() {
   static int n = 0;
   if (n == 0) {

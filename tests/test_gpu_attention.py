@@ -23,10 +23,18 @@ def _ref(qkv, B, s, nh, dh, dO):
     return o.permute(0, 2, 1, 3).reshape(B * s, h), lse.permute(1, 0, 2).reshape(nh, B * s), dqkv
 
 
+@pytest.fixture(params=[-1, 0], ids=["auto_tcgen05", "mma_sync"])
+def attn_variant(request):
+    L = _lib.lib()
+    assert L.mario_k_attn_set_variant(request.param) == 0
+    yield request.param
+    L.mario_k_attn_set_variant(-1)
+
+
 @pytest.mark.parametrize("B,s,nh,dh", [(2, 200, 3, 128), (1, 1024, 2, 80), (2, 130, 4, 64), (3, 64, 2, 16),
-                                       (1, 2048, 2, 128)])
+                                       (1, 2048, 2, 128), (2, 300, 2, 64), (1, 128, 1, 128)])
 @pytest.mark.parametrize("bf16", [1, 0])
-def test_attention_vs_sdpa(B, s, nh, dh, bf16):
+def test_attention_vs_sdpa(B, s, nh, dh, bf16, attn_variant):
     if not bf16 and s > 1024:
         pytest.skip("fp32 SIMT path checked at smaller s")
     g = torch.Generator(device="cuda").manual_seed(s * nh + dh)

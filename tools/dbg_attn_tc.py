@@ -1,0 +1,18 @@
+import sys, torch
+sys.path.insert(0, ".")
+from paper_conf_ppopp_liultj25_b200 import _lib, api  # noqa
+L = _lib.lib()
+B, s, nh, dh = map(int, sys.argv[1:5])
+h = nh * dh
+qkv = torch.randn(B * s, 3 * h, device="cuda").bfloat16()
+O = torch.empty(B * s, h, device="cuda", dtype=torch.bfloat16)
+lse = torch.empty(nh, B * s, device="cuda")
+dO = torch.randn(B * s, h, device="cuda").bfloat16()
+dq = torch.empty(B * s, 3 * h, device="cuda", dtype=torch.bfloat16)
+scr = torch.empty(nh, B * s, device="cuda")
+L.mario_k_attn_set_variant(-1)
+assert L.mario_k_attn_fwd(qkv.data_ptr(), O.data_ptr(), lse.data_ptr(), B, s, nh, dh, 1, None) == 0
+torch.cuda.synchronize()
+assert L.mario_k_attn_bwd(qkv.data_ptr(), O.data_ptr(), dO.data_ptr(), lse.data_ptr(), dq.data_ptr(), scr.data_ptr(), B, s, nh, dh, 1, None) == 0
+torch.cuda.synchronize()
+print("ok", B, s, nh, dh, flush=True)
