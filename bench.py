@@ -43,6 +43,7 @@ def parse():
     ap.add_argument("--micro", type=int, default=32)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-projection", action="store_true")
     return ap.parse_args()
 
 
@@ -175,6 +176,49 @@ def init_weights_device(plan, rank, torch, seed=1234):
     return w
 
 
+def project_pipeline(cfg, api, torch, ctx_factory, stages=8, n_profile=8, n_micro=32):
+    """The paper's method (P:242 profile -> P:244-252 simulate): run one 8-stage Mario iteration in
+    loopback on this GPU with per-instruction CUDA events, take the mean FW/CFW, BW and RC time of
+    each virtual stage, and simulate the BASE / CKPT / MARIO plans of the 8-GPU pipeline with
+    those costs (p2p at the measured NVLink peer bandwidth, B200_PROFILING.md: 770 GB/s)."""
+    prof = api.Plan(cfg, stages, n_profile, "1f1b", "mario", dtype="bf16")
+    ctx = ctx_factory()
+    w, g, ws = api.alloc_for(prof, -1)
+    w.normal_(0.0, 0.02)
+    tok = torch.from_numpy(synth.make_tokens(cfg, n_profile)).cuda()
+    ctx.run_iter(prof, w, tok, g, ws)          # warm-up
+    ctx.set_timing(True)
+    ctx.run_iter(prof, w, tok, g, ws)
+    ctx.set_timing(False)
+    fw = [[] for _ in range(stages)]
+    bw = [[] for _ in range(stages)]
+    rc = [[] for _ in range(stages)]
+    for d in range(stages):
+        a, b = ctx.last_timeline(d)
+        comp = [x for x in prof.instrs(d) if x[0] in ("FW", "CFW", "RC", "BW")]
+        for (op, *_r), t0, t1 in zip(comp, a, b):
+            {"FW": fw, "CFW": fw, "RC": rc, "BW": bw}[op][d].append(t1 - t0)
+    mean = lambda xs: sum(xs) / len(xs) if xs else 0.0
+    costs = {"fw_ms": [mean(x) for x in fw], "bw_ms": [mean(x) for x in bw],
+             "rc_ms": [mean(x) if x else mean(fw[i]) for i, x in enumerate(rc)],
+             "p2p_alpha_ms": 0.02, "p2p_GBps": 770.0}
+    del w, g, ws
+    torch.cuda.empty_cache()
+    gbs = n_micro * cfg.micro_batch
+    out = {"method": "per-stage costs measured (CUDA events, 8-stage loopback on this GPU) -> planner simulator",
+           "stages": stages, "microbatches": n_micro,
+           "stage_ms": {k: [round(x, 3) for x in costs[k]] for k in ("fw_ms", "bw_ms", "rc_ms")}}
+    for level in ("base", "ckpt", "mario"):
+        p = api.Plan(cfg, stages, n_micro, "1f1b", level, dtype="bf16", costs=costs)
+        sim = p.simulate()
+        out[level] = {"makespan_ms": round(sim.makespan_ms, 2), "samples_per_s": round(gbs / (sim.makespan_ms / 1e3), 2),
+                      "bubble": round(sim.bubble_ratio, 4), "peak_gb_per_stage": [round(b / 1e9, 2) for b in sim.peak_bytes],
+                      "peak_balance_max_over_min": round(max(sim.peak_bytes) / min(sim.peak_bytes), 3)}
+    out["mario_vs_ckpt"] = round(out["ckpt"]["makespan_ms"] / out["mario"]["makespan_ms"], 4)
+    out["mario_vs_base"] = round(out["base"]["makespan_ms"] / out["mario"]["makespan_ms"], 4)
+    return out
+
+
 def main():
     args = parse()
     cfg = synth.GPT3_1P3B
@@ -290,6 +334,8 @@ def main():
            "peak_mem_per_stage": {"simulated_bytes": sim.peak_bytes,
                                   "measured_torch_max_allocated": int(mem)},
            "e2e": e2e}
+    if rank == 0 and world == 1 and not args.no_projection:
+        out["pipeline_projection_8gpu"] = project_pipeline(cfg, api, torch, lambda: ctx)
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         n_cores = cores()
         os.environ.setdefault("OPENBLAS_NUM_THREADS", str(n_cores))

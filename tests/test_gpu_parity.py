@@ -37,14 +37,25 @@ def rounded(params):
     return {k: (synth.round_to_bf16(v) if v.ndim == 2 else v) for k, v in params.items()}
 
 
-def check(loss, grads, l_o, g_o, tol):
+def check(loss, grads, l_o, g_o, tol, norm="inf", inf_guard=None):
+    """Reading A19: per-tensor relative error. norm="inf": ||g-o||_inf/||o||_inf <= tol (small
+    cases); norm="l2": ||g-o||_2/||o||_2 <= tol plus ||.||_inf-relative <= inf_guard (full-width
+    bf16 cases, where bf16 activation storage alone moves the fp32 definition by ~2% in the
+    worst element at h = 4096; tools/bf16_storage_error.py, A19)."""
     assert abs(loss - l_o) <= tol * abs(l_o), (loss, l_o)
-    worst = (None, 0.0)
+    worst_inf, worst_l2 = (None, 0.0), (None, 0.0)
     for k, v in g_o.items():
-        err = float(np.abs(grads[k] - v).max() / max(np.abs(v).max(), 1e-30))
-        if err > worst[1]:
-            worst = (k, err)
-    assert worst[1] <= tol, worst
+        d = grads[k].astype(np.float64) - v
+        e_inf = float(np.abs(d).max() / max(np.abs(v).max(), 1e-30))
+        e_l2 = float(np.linalg.norm(d) / max(np.linalg.norm(v), 1e-30))
+        worst_inf = max(worst_inf, (k, e_inf), key=lambda t: t[1])
+        worst_l2 = max(worst_l2, (k, e_l2), key=lambda t: t[1])
+    if norm == "inf":
+        assert worst_inf[1] <= tol, worst_inf
+    else:
+        assert worst_l2[1] <= tol, worst_l2
+        assert worst_inf[1] <= inf_guard, worst_inf
+    return worst_inf, worst_l2
 
 
 TINY_L = synth.tiny_llama()
@@ -106,3 +117,29 @@ def test_deterministic_repeat():
     a = run_plan(cfg, 2, 4, "1f1b", "mario", "bf16", params, toks)[2]
     b = run_plan(cfg, 2, 4, "1f1b", "mario", "bf16", params, toks)[2]
     assert np.array_equal(a, b)
+
+
+# ---------------------------------------------------------------------------------------------
+# Full-width parity: the BASELINE.json model widths (h, heads, f, V, s) truncated to 2 layers so
+# the fp32 CPU oracle finishes in seconds; run through the same bf16 kernels and launch shapes
+# bench.py times (tcgen05 GEMMs incl. CTA-pair tiles, tcgen05 attention backward).
+# (name, cfg, scheme, S, N, v, l2 tol, inf guard). LLaMA2-7B width: bf16 *storage* alone moves the
+# fp32 definition by 2.37% (l2) / 2.29% (inf) on h1.qkv.w at s = 2048 (tools/bf16_storage_error.py
+# lin,norm,attn 2048), so its bound is set at ~1.7x that floor (A19).
+FULL = [
+    ("gpt3-1.3b", synth.with_(synth.GPT3_1P3B, n_layers=2, micro_batch=1), "1f1b", 2, 2, 1, 2e-2, 5e-2),
+    ("llama2-7b-s2048", synth.with_(synth.LLAMA2_7B, n_layers=2, micro_batch=1, seq_len=2048), "1f1b", 2, 2, 1,
+     4e-2, 6e-2),
+    ("gpt3-2.7b-chimera", synth.with_(synth.GPT3_2P7B, n_layers=2, micro_batch=1), "chimera", 2, 2, 1, 2e-2, 5e-2),
+]
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("name,cfg,scheme,S,N,v,tol,guard", FULL, ids=[f[0] for f in FULL])
+def test_full_width_parity_bf16(name, cfg, scheme, S, N, v, tol, guard):
+    params = synth.make_weights(cfg)
+    toks = synth.make_tokens(cfg, N)
+    loss, grads, _ = run_plan(cfg, S, N, scheme, "mario", "bf16", params, toks, chunks=v)
+    l_o, g_o = om.step(cfg, rounded(params), toks, N, np.float32)
+    wi, wl = check(loss, grads, l_o, g_o, tol, norm="l2", inf_guard=guard)
+    print(f"[full-width {name}] loss {loss:.6f} vs {l_o:.6f}; worst inf-rel {wi}; worst l2-rel {wl}")
