@@ -15,6 +15,8 @@ namespace mario {
 int g_attn_variant = -1;   // mario_k_attn_set_variant: -1 auto (tcgen05 where supported), 0 mma.sync only
 bool flash_attn_bwd_tc(const __nv_bfloat16* qkv, const __nv_bfloat16* dO, const float* lse, const float* Dd,
                        __nv_bfloat16* dqkv, int B, int s, int nh, int dh, cudaStream_t st);   // attn_tc.cu
+bool flash_attn_fwd_tc(const __nv_bfloat16* qkv, __nv_bfloat16* O, float* lse, int B, int s, int nh, int dh,
+                       cudaStream_t st);   // attn_tc.cu
 
 namespace {
 
@@ -425,6 +427,10 @@ void launch_fwd(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, cuda
   // causal algorithmic FLOPs: QK^T and PV over the lower triangle
   const double fl = 4.0 * B * nh * D * (static_cast<double>(s) * (s + 1) / 2);
   const int tok = kstats_begin(K_ATTN_FWD, fl, 0.0, st);
+  if (g_attn_variant != 0 && flash_attn_fwd_tc(qkv, O, lse, B, s, nh, D, st)) {
+    kstats_end(tok, st);
+    return;
+  }
   fa_fwd_k<D><<<grid, 128, smem, st>>>(qkv, O, lse, B, s, nh);
   kstats_end(tok, st);
   note_launch();

@@ -478,10 +478,243 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
   return true;
 }
 
+
+// ------------------------------------------------------------------------------ forward
+// One CTA per 128 queries (TMEM lanes); loop over 64-key tiles j <= last query:
+//   MMA thread: S_j = Q K_j^T (M128 N64) into a double-buffered TMEM pair, PV_j = P_j V_j
+//   (M128 N=dh, fresh accumulator per tile, double-buffered) once P_j is in smem.
+//   4 softmax warps (one query row per thread): online max/sum, P_j (bf16, swizzled smem),
+//   and O (fp32 registers) += PV_{j-1} one tile late so the PV MMA latency is hidden:
+//   O <- O * exp(m_{j-2} - m_{j-1}) + PV_{j-1}.
+template <int DH>
+__global__ void __launch_bounds__(kThreads, 1)
+fa_fwd_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_qkv64, bf16* O,
+          float* lse, int B, int s, int nh) {
+  using SM = Smem<DH>;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sQ = smem;
+  uint8_t* sK[2] = {sQ + SM::kBig, sQ + SM::kBig + 2 * SM::kSmall};
+  uint8_t* sV[2] = {sK[0] + SM::kSmall, sK[1] + SM::kSmall};
+  uint8_t* sP[2] = {sQ + SM::kBig + 4 * SM::kSmall, sQ + SM::kBig + 4 * SM::kSmall + SM::kP};
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sP[1] + SM::kP);
+  uint64_t* q_fullb = bar;          // 1
+  uint64_t* k_full = bar + 1;       // 2
+  uint64_t* k_empty = bar + 3;      // 2
+  uint64_t* s_full = bar + 5;       // 2
+  uint64_t* s_free = bar + 7;       // 2
+  uint64_t* p_full = bar + 9;       // 2
+  uint64_t* o_full = bar + 11;      // 2  (PV_j done: also frees P_j smem)
+  uint64_t* o_free = bar + 13;      // 2  (softmax read PV_j out of TMEM)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 15);
+
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int qt = blockIdx.x, b = blockIdx.y / nh, head = blockIdx.y % nh;
+  const int h = nh * DH;
+  const long Ttok = static_cast<long>(B) * s;
+  const int last_q = min(qt * kRows + kRows - 1, s - 1);
+  const int ntiles = last_q / kCols + 1;
+  const float sl2 = rsqrtf(static_cast<float>(DH)) * LOG2E;
+
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&tm_qkv128);
+    tma_prefetch_desc(&tm_qkv64);
+    mbar_init(q_fullb, 1);
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1); mbar_init(&s_full[i], 1); mbar_init(&s_free[i], 4);
+      mbar_init(&p_full[i], 4); mbar_init(&o_full[i], 1); mbar_init(&o_free[i], 4);
+    }
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc<512>(tmem_slot);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tm = *tmem_slot;
+  const uint32_t tm_S = tm, tm_O = tm + 2 * kCols;   // S[2] x 64 cols, PV[2] x DH cols
+
+  if (warp == 0) {
+    if (elect_one()) {
+      const int row0 = b * s;
+      mbar_arrive_expect_tx(q_fullb, SM::kBig);
+#pragma unroll
+      for (int a = 0; a < DH / 64; ++a)
+        tma_load_2d(sQ + a * (kRows * 128), &tm_qkv128, q_fullb, head * DH + a * 64, row0 + qt * kRows);
+      for (int j = 0; j < ntiles; ++j) {
+        const int st = j & 1;
+        mbar_wait(&k_empty[st], ((j >> 1) & 1) ^ 1);
+        mbar_arrive_expect_tx(&k_full[st], 2 * SM::kSmall);
+#pragma unroll
+        for (int a = 0; a < DH / 64; ++a) {
+          tma_load_2d(sK[st] + a * (kCols * 128), &tm_qkv64, &k_full[st], h + head * DH + a * 64, row0 + j * kCols);
+          tma_load_2d(sV[st] + a * (kCols * 128), &tm_qkv64, &k_full[st], 2 * h + head * DH + a * 64, row0 + j * kCols);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    constexpr uint32_t id_s = umma_idesc_bf16(128, kCols, 0, 0);
+    constexpr uint32_t id_o = umma_idesc_bf16(128, DH, 0, 1);   // PV: B = V_j read MN-major
+    mbar_wait(q_fullb, 0);
+    tc_fence_after();
+    auto issue_s = [&](int j) {
+      const int st = j & 1;
+      mbar_wait(&k_full[st], (j >> 1) & 1);
+      mbar_wait(&s_free[st], ((j >> 1) & 1) ^ 1);
+      tc_fence_after();
+      if (elect_one()) {
+        const uint32_t q = smem_u32(sQ), k = smem_u32(sK[st]);
+#pragma unroll
+        for (int kk = 0; kk < DH / 16; ++kk) {
+          const uint32_t ao = (kk >> 2) * (kRows * 128) + (kk & 3) * 32, bo = (kk >> 2) * (kCols * 128) + (kk & 3) * 32;
+          umma_bf16(tm_S + st * kCols, umma_desc_sw128(q + ao, 16, 1024), umma_desc_sw128(k + bo, 16, 1024), id_s, kk > 0);
+        }
+        umma_commit(&s_full[st]);
+      }
+      __syncwarp();
+    };
+    auto issue_pv = [&](int j) {
+      const int st = j & 1;
+      mbar_wait(&p_full[st], (j >> 1) & 1);
+      mbar_wait(&o_free[st], ((j >> 1) & 1) ^ 1);
+      tc_fence_after();
+      if (elect_one()) {
+        const uint32_t p = smem_u32(sP[st]), v = smem_u32(sV[st]);
+#pragma unroll
+        for (int kk = 0; kk < kCols / 16; ++kk)
+          umma_bf16(tm_O + st * DH, umma_desc_sw128(p + kk * 32, 16, 1024),
+                    umma_desc_sw128(v + kk * 2048, kCols * 128, 1024), id_o, kk > 0);
+        umma_commit(&o_full[st]);
+        umma_commit(&k_empty[st]);
+      }
+      __syncwarp();
+    };
+    issue_s(0);
+    for (int j = 1; j < ntiles; ++j) {
+      issue_s(j);
+      issue_pv(j - 1);
+    }
+    issue_pv(ntiles - 1);
+  } else {
+    const int quarter = warp & 3;
+    const int row = quarter * 32 + lane;
+    const int q = qt * kRows + row;
+    const uint32_t lane_off = static_cast<uint32_t>(quarter * 32) << 16;
+    float o[DH];
+#pragma unroll
+    for (int d = 0; d < DH; ++d) o[d] = 0.f;
+    float m_run = -INFINITY, l_run = 0.f;
+    float m_prev_tile = -INFINITY;   // max used for P of the tile whose PV is pending
+    // fold PV_j (computed relative to m_j) into O (relative to m_{j-1}): O = O*exp(m_{j-1} - m_j) + PV_j
+    auto fold = [&](int j, float m_j, float m_before) {
+      const int st = j & 1;
+      mbar_wait(&o_full[st], (j >> 1) & 1);
+      tc_fence_after();
+      const float c = exp2f(m_before - m_j);
+#pragma unroll
+      for (int c0 = 0; c0 < DH; c0 += 32) {
+        uint32_t r[32];
+        tmem_ld_32x32b_x32(tm_O + st * DH + c0 + lane_off, r);
+        tmem_ld_wait();
+#pragma unroll
+        for (int e = 0; e < 32; ++e) o[c0 + e] = o[c0 + e] * c + __uint_as_float(r[e]);
+      }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&o_free[st]);
+    };
+    float m_pending = -INFINITY, m_folded = -INFINITY;
+    for (int j = 0; j < ntiles; ++j) {
+      const int st = j & 1;
+      mbar_wait(&s_full[st], (j >> 1) & 1);
+      tc_fence_after();
+      uint32_t sr[64];
+      tmem_ld_32x32b_x32(tm_S + st * kCols + lane_off, *reinterpret_cast<uint32_t(*)[32]>(sr));
+      tmem_ld_32x32b_x32(tm_S + st * kCols + 32 + lane_off, *reinterpret_cast<uint32_t(*)[32]>(sr + 32));
+      tmem_ld_wait();
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&s_free[st]);
+      float mx = m_run;
+#pragma unroll
+      for (int c = 0; c < 64; ++c) {
+        const int key = j * kCols + c;
+        float x = __uint_as_float(sr[c]) * sl2;
+        if (key > q) x = -INFINITY;
+        sr[c] = __float_as_uint(x);
+        mx = fmaxf(mx, x);
+      }
+      const float m_new = mx;   // finite: key 0 <= q for every row
+      float p[64], ls = 0.f;
+#pragma unroll
+      for (int c = 0; c < 64; ++c) {
+        p[c] = exp2f(__uint_as_float(sr[c]) - m_new);
+        ls += p[c];
+      }
+      l_run = l_run * exp2f(m_run - m_new) + ls;
+      m_run = m_new;
+      // P_j into smem (buffer st is free once PV_{j-2} completed, which fold(j-2) waited on)
+      st_row_sw128(sP[st], row, p);
+      fence_proxy_async();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&p_full[st]);
+      if (j > 0) {
+        fold(j - 1, m_pending, m_folded);
+        m_folded = m_pending;
+      }
+      m_pending = m_new;
+    }
+    fold(ntiles - 1, m_pending, m_folded);
+    // O is relative to m_run (= m_pending of the last tile)
+    const float inv = 1.f / l_run;
+    if (q < s) {
+      bf16* orow = O + (static_cast<long>(b) * s + q) * h + head * DH;
+#pragma unroll
+      for (int d = 0; d < DH; d += 8) {
+        uint4 u;
+        __nv_bfloat162* hh = reinterpret_cast<__nv_bfloat162*>(&u);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) hh[e] = __floats2bfloat162_rn(o[d + 2 * e] * inv, o[d + 2 * e + 1] * inv);
+        *reinterpret_cast<uint4*>(orow + d) = u;
+      }
+      lse[static_cast<long>(head) * Ttok + static_cast<long>(b) * s + q] = (m_run + log2f(l_run)) / LOG2E;
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) tmem_dealloc<512>(tm);
+}
+
+template <int DH>
+constexpr int smem_fwd() { return at_least_one_sm(Smem<DH>::kBig + 4 * Smem<DH>::kSmall + 2 * Smem<DH>::kP + 128 + 1024); }
+
+template <int DH>
+bool launch_fwd_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, cudaStream_t st) {
+  const int h = nh * DH;
+  const long T = static_cast<long>(B) * s;
+  CUtensorMap m128, m64;
+  if (!make_tmap_bf16_2d(&m128, qkv, 3 * h, T, 3 * h, 64, 128) || !make_tmap_bf16_2d(&m64, qkv, 3 * h, T, 3 * h, 64, 64))
+    return false;
+  static bool set = false;
+  if (!set) {
+    cudaFuncSetAttribute(fa_fwd_tc<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_fwd<DH>());
+    set = true;
+  }
+  dim3 grid((s + kRows - 1) / kRows, B * nh);
+  fa_fwd_tc<DH><<<grid, kThreads, smem_fwd<DH>(), st>>>(m128, m64, O, lse, B, s, nh);
+  note_launch();
+  return true;
+}
+
 }  // namespace
 
 bool flash_attn_bwd_tc_supported(int dh, int B, int s, int nh) {
   return (dh == 64 || dh == 128) && ((nh * dh) % 64 == 0);
+}
+
+bool flash_attn_fwd_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st) {
+  if (dh == 128) return launch_fwd_tc<128>(qkv, O, lse, B, s, nh, st);
+  if (dh == 64) return launch_fwd_tc<64>(qkv, O, lse, B, s, nh, st);
+  return false;
 }
 
 // Returns false if the configuration is unsupported (caller falls back to the mma.sync kernels).
