@@ -183,14 +183,18 @@ struct Exec {
     const int dh = h / nh, s = m.seq_len, mbs = m.micro_batch;
     const bool gpt = m.family == MARIO_GPT;
     const LayerAct LA = layer_act_layout(m);
+    const LayerTrans LT = layer_trans_layout(m);
     const HeadAct HA = head_act_layout(m);
+    // cfw scratch: [one layer's stored tensors][transients A, A2, G][run0][run1][head]
+    uint8_t* cfw = D.template at<uint8_t>(D.a.cfw);
+    uint8_t* trans = cfw + LA.bytes;
     uint8_t* base;
     size_t lstride;
-    if (mode == 1) { base = D.template at<uint8_t>(D.a.cfw); lstride = 0; }
+    if (mode == 1) { base = cfw; lstride = 0; }
     else { base = D.template at<uint8_t>(D.a.act + static_cast<size_t>(x.aslot) * D.a.act_stride); lstride = LA.bytes; }
-    uint8_t* head_base = (mode == 1) ? base + LA.bytes + 2 * stage_input_bytes(m) : base + LA.bytes * lps;
-    T* run[2] = {reinterpret_cast<T*>(D.template at<uint8_t>(D.a.cfw) + LA.bytes),
-                 reinterpret_cast<T*>(D.template at<uint8_t>(D.a.cfw) + LA.bytes + stage_input_bytes(m))};
+    uint8_t* run_base = trans + LT.bytes;
+    uint8_t* head_base = (mode == 1) ? run_base + 2 * stage_input_bytes(m) : base + LA.bytes * lps;
+    T* run[2] = {reinterpret_cast<T*>(run_base), reinterpret_cast<T*>(run_base + stage_input_bytes(m))};
     const int32_t* tok = D.template at<int32_t>(D.a.tokens) + static_cast<size_t>(x.micro) * mbs * (s + 1);
     // stage input
     const T* Hin;
@@ -207,14 +211,14 @@ struct Exec {
       const int l = k * lps + li;
       const std::string pre = "h" + std::to_string(l) + ".";
       uint8_t* L = base + li * lstride;
-      T* A = reinterpret_cast<T*>(L + LA.A);
+      T* A = reinterpret_cast<T*>(trans + LT.A);
       T* QKV = reinterpret_cast<T*>(L + LA.QKV);
       T* O = reinterpret_cast<T*>(L + LA.O);
       float* LSE = reinterpret_cast<float*>(L + LA.LSE);
       T* H1 = reinterpret_cast<T*>(L + LA.H1);
-      T* A2 = reinterpret_cast<T*>(L + LA.A2);
+      T* A2 = reinterpret_cast<T*>(trans + LT.A2);
       T* Z = reinterpret_cast<T*>(L + LA.Z);
-      T* Gt = reinterpret_cast<T*>(L + LA.G);
+      T* Gt = reinterpret_cast<T*>(trans + LT.G);
       float* st1 = reinterpret_cast<float*>(L + LA.st1);
       float* st2 = reinterpret_cast<float*>(L + LA.st2);
       // output of this layer
@@ -317,22 +321,25 @@ struct Exec {
       uint8_t* L = base + li * LA.bytes;
       const T* Hin = (li == 0 && k > 0) ? D.template at<T>(D.a.ckpt + static_cast<size_t>(x.slot) * D.a.ckpt_stride)
                                         : reinterpret_cast<T*>(L + LA.H_in);
-      T* A = reinterpret_cast<T*>(L + LA.A);
+      // recomputed transients: A / A2 (norm outputs) share Arec, G / M share the dM buffer
+      T* A = reinterpret_cast<T*>(sc + BS.Arec);
+      T* A2 = A;
+      T* Gt = dM;
       T* QKV = reinterpret_cast<T*>(L + LA.QKV);
       T* O = reinterpret_cast<T*>(L + LA.O);
       float* LSE = reinterpret_cast<float*>(L + LA.LSE);
       T* H1 = reinterpret_cast<T*>(L + LA.H1);
-      T* A2 = reinterpret_cast<T*>(L + LA.A2);
       T* Z = reinterpret_cast<T*>(L + LA.Z);
-      T* Gt = reinterpret_cast<T*>(L + LA.G);
       float* st1 = reinterpret_cast<float*>(L + LA.st1);
       float* st2 = reinterpret_cast<float*>(L + LA.st2);
       T* dH1 = dHbuf[(cur + 1) % 3];
       T* dHin = (li == 0) ? (k == 0 ? dHbuf[(cur + 2) % 3] : dstage_in) : dHbuf[(cur + 2) % 3];
       if (gpt) {
+        gelu_fwd<T>(Z, Gt, static_cast<size_t>(Tn) * f, st);                 // recompute G = gelu(Z)
         lin_wgrad(dH, Gt, Tn, h, f, G(D, p, pre + "fc2.w"));
         colsum<T>(dH, nullptr, nullptr, Tn, h, h, 0, G(D, p, pre + "fc2.b"), nullptr, red, st);
         lin_dgrad(dH, Wm(D, p, pre + "fc2.w"), Tn, h, f, dZ, Z);           // dZ = (dH W2) * gelu'(Z)
+        layernorm_fwd<T>(H1, Wf(D, p, pre + "ln2.g"), Wf(D, p, pre + "ln2.b"), A2, st2, Tn, h, m.norm_eps, st);
         lin_wgrad(dZ, A2, Tn, f, h, G(D, p, pre + "fc1.w"));
         colsum<T>(dZ, nullptr, nullptr, Tn, f, f, 0, G(D, p, pre + "fc1.b"), nullptr, red, st);
         lin_dgrad(dZ, Wm(D, p, pre + "fc1.w"), Tn, f, h, dA);               // dA2
@@ -342,9 +349,11 @@ struct Exec {
         colsum<T>(dH1, nullptr, nullptr, Tn, h, h, 0, G(D, p, pre + "proj.b"), nullptr, red, st);
         lin_dgrad(dH1, Wm(D, p, pre + "proj.w"), Tn, h, h, dO);
       } else {
+        swiglu_fwd<T>(Z, Gt, Tn, f, st);                                      // recompute M (into dM)
         lin_wgrad(dH, Gt, Tn, h, f, G(D, p, pre + "down.w"));
-        lin_dgrad(dH, Wm(D, p, pre + "down.w"), Tn, h, f, dM);
+        lin_dgrad(dH, Wm(D, p, pre + "down.w"), Tn, h, f, dM);              // overwrites M (consumed)
         swiglu_bwd<T>(Z, dM, dZ, Tn, f, st);
+        rmsnorm_fwd<T>(H1, Wf(D, p, pre + "n2.g"), A2, st2, Tn, h, m.norm_eps, st);
         lin_wgrad(dZ, A2, Tn, 2 * f, h, G(D, p, pre + "gu.w"));
         lin_dgrad(dZ, Wm(D, p, pre + "gu.w"), Tn, 2 * f, h, dA);
         norm_bwd_dx<T>(dA, H1, st2, Wf(D, p, pre + "n2.g"), dH, dH1, Tn, h, 1, st);
@@ -354,6 +363,8 @@ struct Exec {
       }
       attn_bwd<T>(QKV, O, dO, LSE, dQKV, Dsc, mbs, s, nh, dh, st);
       if (!gpt) rope<T>(dQKV, mbs, s, nh, dh, m.rope_base, 1, st);
+      if (gpt) layernorm_fwd<T>(Hin, Wf(D, p, pre + "ln1.g"), Wf(D, p, pre + "ln1.b"), A, st1, Tn, h, m.norm_eps, st);
+      else rmsnorm_fwd<T>(Hin, Wf(D, p, pre + "n1.g"), A, st1, Tn, h, m.norm_eps, st);
       lin_wgrad(dQKV, A, Tn, 3 * h, h, G(D, p, pre + "qkv.w"));
       if (gpt) colsum<T>(dQKV, nullptr, nullptr, Tn, 3 * h, 3 * h, 0, G(D, p, pre + "qkv.b"), nullptr, red, st);
       lin_dgrad(dQKV, Wm(D, p, pre + "qkv.w"), Tn, 3 * h, h, dA);

@@ -17,20 +17,24 @@ LayerAct layer_act_layout(const mario_model& m) {
   auto take = [&](size_t bytes) { size_t r = o; o = align_up(o + bytes); return r; };
   L.H_in = take(T * h * E);
   L.st1 = take(T * 2 * 4);          // mean, rstd (fp32)
-  L.A = take(T * h * E);
   L.QKV = take(T * 3 * h * E);
   L.O = take(T * h * E);
   L.LSE = take(nh * T * 4);
   L.H1 = take(T * h * E);
   L.st2 = take(T * 2 * 4);
+  L.Z = take(T * (m.family == MARIO_GPT ? f : 2 * f) * E);   // GPT: Z; LLaMA: GU = [gate | up]
+  L.bytes = o;
+  return L;
+}
+
+LayerTrans layer_trans_layout(const mario_model& m) {
+  const size_t T = tokens_per_micro(m), E = elt_size(m), h = m.hidden, f = m.ffn_hidden;
+  LayerTrans L{};
+  size_t o = 0;
+  auto take = [&](size_t bytes) { size_t r = o; o = align_up(o + bytes); return r; };
+  L.A = take(T * h * E);
   L.A2 = take(T * h * E);
-  if (m.family == MARIO_GPT) {
-    L.Z = take(T * f * E);
-    L.G = take(T * f * E);
-  } else {
-    L.Z = take(T * 2 * f * E);     // GU = [gate | up]
-    L.G = take(T * f * E);         // M = silu(gate) * up
-  }
+  L.G = take(T * f * E);
   L.bytes = o;
   return L;
 }
@@ -58,8 +62,8 @@ size_t act_set_bytes(const mario_model& m, int k, int K) {
 }
 
 size_t cfw_work_bytes(const mario_model& m, int k, int K) {
-  // one layer's temporaries + the two running residual buffers (+ head temporaries)
-  size_t b = layer_act_layout(m).bytes + 2 * stage_input_bytes(m);
+  // one layer's stored + transient tensors + the two running residual buffers (+ head)
+  size_t b = layer_act_layout(m).bytes + layer_trans_layout(m).bytes + 2 * stage_input_bytes(m);
   if (k == K - 1) b += head_act_layout(m).bytes;
   return b;
 }
@@ -77,6 +81,7 @@ BwScratch bw_scratch_layout(const mario_model& m) {
   b.dM = take(T * f * E);
   b.Dsc = take(static_cast<size_t>(m.n_heads) * T * 4);
   b.sort = take(T * 8 * 2);
+  b.Arec = take(T * h * E);
   b.bytes = o;
   return b;
 }

@@ -53,6 +53,21 @@ __device__ __forceinline__ void st_row_sw128(uint8_t* tile, int row, const float
   }
 }
 
+// write 32 bf16 values = chunks [c0, c0+4) of one 128-byte row of a K-major SW128 tile
+__device__ __forceinline__ void st_half_row_sw128(uint8_t* tile, int row, int c0, const float (&v)[32]) {
+  uint8_t* rp = tile + row * 128;
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    uint4 u;
+    __nv_bfloat162* h = reinterpret_cast<__nv_bfloat162*>(&u);
+#pragma unroll
+    for (int e = 0; e < 4; ++e) h[e] = __floats2bfloat162_rn(v[8 * j + 2 * e], v[8 * j + 2 * e + 1]);
+    *reinterpret_cast<uint4*>(rp + (((c0 + j) ^ (row & 7)) << 4)) = u;
+  }
+}
+
+constexpr int kThreadsB = 320;   // backward: TMA, MMA, 8 softmax warps (2 per TMEM lane quarter)
+
 template <int DH>
 struct Smem {
   static constexpr int kBig = kRows * DH * 2;        // 128-row tile (K,V or Q,dO)
@@ -62,7 +77,7 @@ struct Smem {
 
 // ------------------------------------------------------------------------ dK / dV
 template <int DH>
-__global__ void __launch_bounds__(kThreads, 1)
+__global__ void __launch_bounds__(kThreadsB, 1)
 fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_qkv64,
                const __grid_constant__ CUtensorMap tm_do64, const float* lse, const float* Dd, bf16* dqkv, int B,
                int s, int nh) {
@@ -102,8 +117,8 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
     tma_prefetch_desc(&tm_qkv64);
     tma_prefetch_desc(&tm_do64);
     mbar_init(kv_full, 1);
-    for (int i = 0; i < 2; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); mbar_init(&s_full[i], 1); mbar_init(&s_free[i], 4); }
-    mbar_init(p_full, 4);
+    for (int i = 0; i < 2; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); mbar_init(&s_full[i], 1); mbar_init(&s_free[i], 8); }
+    mbar_init(p_full, 8);
     mbar_init(p_free, 1);
     mbar_init(acc_done, 1);
     fence_barrier_init();
@@ -189,48 +204,48 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
     }
     issue_acc(ntiles - 1);
   } else {
-    const int quarter = warp & 3;
+    const int quarter = warp & 3, half = (warp - 2) >> 2;   // column half [32*half, 32*half+32)
     const int row = quarter * 32 + lane;             // key row within the tile
     const int key = kt * kRows + row;
     const uint32_t lane_off = static_cast<uint32_t>(quarter * 32) << 16;
-    const int tid = threadIdx.x - 64;                // 0..127
+    const int tid = threadIdx.x - 64;                // 0..255
     for (int idx = 0; idx < ntiles; ++idx) {
       const int buf = idx & 1, i = i0 + idx;
       // lse / D of this query tile into smem (threads 0..63: lse, 64..127: D)
-      {
+      if (tid < 128) {
         const int c = tid & 63, qq = i * kCols + c;
         const long r = static_cast<long>(b) * s + (qq < s ? qq : 0);
         if (tid < 64) sL[buf * kCols + c] = lse[static_cast<long>(head) * Ttok + r] * LOG2E;
         else sDv[buf * kCols + c] = Dd[static_cast<long>(head) * Ttok + r];
       }
-      named_bar(1, 128);
+      named_bar(1, 256);
       mbar_wait(&s_full[buf], (idx >> 1) & 1);
       tc_fence_after();
-      uint32_t sr[64], dr[64];
-      tmem_ld_32x32b_x32(tm_S + buf * kCols + lane_off, *reinterpret_cast<uint32_t(*)[32]>(sr));
-      tmem_ld_32x32b_x32(tm_S + buf * kCols + 32 + lane_off, *reinterpret_cast<uint32_t(*)[32]>(sr + 32));
-      tmem_ld_32x32b_x32(tm_dP + buf * kCols + lane_off, *reinterpret_cast<uint32_t(*)[32]>(dr));
-      tmem_ld_32x32b_x32(tm_dP + buf * kCols + 32 + lane_off, *reinterpret_cast<uint32_t(*)[32]>(dr + 32));
+      uint32_t sr[32], dr[32];
+      tmem_ld_32x32b_x32(tm_S + buf * kCols + half * 32 + lane_off, sr);
+      tmem_ld_32x32b_x32(tm_dP + buf * kCols + half * 32 + lane_off, dr);
       tmem_ld_wait();
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&s_free[buf]);
-      float p[64], ds[64];
+      float p[32], ds[32];
 #pragma unroll
-      for (int c = 0; c < 64; ++c) {
-        const int qq = i * kCols + c;
-        float pv = exp2f(__uint_as_float(sr[c]) * sl2 - sL[buf * kCols + c]);
+      for (int c = 0; c < 32; ++c) {
+        const int cc = half * 32 + c;
+        const int qq = i * kCols + cc;
+        float pv = exp2f(__uint_as_float(sr[c]) * sl2 - sL[buf * kCols + cc]);
         if (qq < key || qq >= s) pv = 0.f;
         p[c] = pv;
-        ds[c] = pv * (__uint_as_float(dr[c]) - sDv[buf * kCols + c]);
+        ds[c] = pv * (__uint_as_float(dr[c]) - sDv[buf * kCols + cc]);
       }
       mbar_wait(p_free, (idx & 1) ^ 1);   // previous tile's dV/dK MMAs have consumed sP/sS
-      st_row_sw128(sP, row, p);
-      st_row_sw128(sS, row, ds);
+      st_half_row_sw128(sP, row, 4 * half, p);
+      st_half_row_sw128(sS, row, 4 * half, ds);
       fence_proxy_async();
       __syncwarp();
       if (lane == 0) mbar_arrive(p_full);
     }
+    if (half == 1) goto done_dkdv;   // the epilogue uses one warp per lane quarter
     // epilogue: dV, dK rows of this thread's key
     mbar_wait(acc_done, 0);
     tc_fence_after();
@@ -263,6 +278,7 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
       }
     }
   }
+done_dkdv:
   tc_fence_before();
   __syncthreads();
   if (warp == 1) tmem_dealloc<512>(tm);
@@ -270,7 +286,7 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
 
 // ------------------------------------------------------------------------------ dQ
 template <int DH>
-__global__ void __launch_bounds__(kThreads, 1)
+__global__ void __launch_bounds__(kThreadsB, 1)
 fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_qkv64,
              const __grid_constant__ CUtensorMap tm_do128, const float* lse, const float* Dd, bf16* dqkv, int B, int s,
              int nh) {
@@ -306,8 +322,8 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
     tma_prefetch_desc(&tm_qkv64);
     tma_prefetch_desc(&tm_do128);
     mbar_init(q_fullb, 1);
-    for (int i = 0; i < 2; ++i) { mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1); mbar_init(&s_full[i], 1); mbar_init(&s_free[i], 4); }
-    mbar_init(p_full, 4);
+    for (int i = 0; i < 2; ++i) { mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1); mbar_init(&s_full[i], 1); mbar_init(&s_free[i], 8); }
+    mbar_init(p_full, 8);
     mbar_init(p_free, 1);
     mbar_init(acc_done, 1);
     fence_barrier_init();
@@ -385,7 +401,7 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
     }
     issue_acc(ntiles - 1);
   } else {
-    const int quarter = warp & 3;
+    const int quarter = warp & 3, half = (warp - 2) >> 2;
     const int row = quarter * 32 + lane;
     const int q = qt * kRows + row;
     const uint32_t lane_off = static_cast<uint32_t>(quarter * 32) << 16;
@@ -396,29 +412,28 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
       const int buf = idx & 1;
       mbar_wait(&s_full[buf], (idx >> 1) & 1);
       tc_fence_after();
-      uint32_t sr[64], dr[64];
-      tmem_ld_32x32b_x32(tm_S + buf * kCols + lane_off, *reinterpret_cast<uint32_t(*)[32]>(sr));
-      tmem_ld_32x32b_x32(tm_S + buf * kCols + 32 + lane_off, *reinterpret_cast<uint32_t(*)[32]>(sr + 32));
-      tmem_ld_32x32b_x32(tm_dP + buf * kCols + lane_off, *reinterpret_cast<uint32_t(*)[32]>(dr));
-      tmem_ld_32x32b_x32(tm_dP + buf * kCols + 32 + lane_off, *reinterpret_cast<uint32_t(*)[32]>(dr + 32));
+      uint32_t sr[32], dr[32];
+      tmem_ld_32x32b_x32(tm_S + buf * kCols + half * 32 + lane_off, sr);
+      tmem_ld_32x32b_x32(tm_dP + buf * kCols + half * 32 + lane_off, dr);
       tmem_ld_wait();
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&s_free[buf]);
-      float ds[64];
+      float ds[32];
 #pragma unroll
-      for (int c = 0; c < 64; ++c) {
-        const int key = idx * kCols + c;
+      for (int c = 0; c < 32; ++c) {
+        const int key = idx * kCols + half * 32 + c;
         float pv = exp2f(__uint_as_float(sr[c]) * sl2 - L);
         if (key > q) pv = 0.f;
         ds[c] = pv * (__uint_as_float(dr[c]) - Dr);
       }
       mbar_wait(p_free, (idx & 1) ^ 1);
-      st_row_sw128(sS, row, ds);
+      st_half_row_sw128(sS, row, 4 * half, ds);
       fence_proxy_async();
       __syncwarp();
       if (lane == 0) mbar_arrive(p_full);
     }
+    if (half == 1) goto done_dq;
     mbar_wait(acc_done, 0);
     tc_fence_after();
     const float scale = rsqrtf(static_cast<float>(DH));
@@ -441,6 +456,7 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
       }
     }
   }
+done_dq:
   tc_fence_before();
   __syncthreads();
   if (warp == 1) tmem_dealloc<512>(tm);
@@ -471,9 +487,9 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
   dim3 grid((s + kRows - 1) / kRows, B * nh);
   const char* only = getenv("MARIO_ATTN_TC_ONLY");   // debugging aid: "dkdv" or "dq"
   if (!only || only[1] == 'k')
-    fa_bwd_dkdv_tc<DH><<<grid, kThreads, smem_dkdv<DH>(), st>>>(m128, m64, d64, lse, Dd, dqkv, B, s, nh);
+    fa_bwd_dkdv_tc<DH><<<grid, kThreadsB, smem_dkdv<DH>(), st>>>(m128, m64, d64, lse, Dd, dqkv, B, s, nh);
   if (!only || only[1] == 'q')
-    fa_bwd_dq_tc<DH><<<grid, kThreads, smem_dq<DH>(), st>>>(m128, m64, d128, lse, Dd, dqkv, B, s, nh);
+    fa_bwd_dq_tc<DH><<<grid, kThreadsB, smem_dq<DH>(), st>>>(m128, m64, d128, lse, Dd, dqkv, B, s, nh);
   note_launch(2);
   return true;
 }
@@ -487,7 +503,7 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
 //   and O (fp32 registers) += PV_{j-1} one tile late so the PV MMA latency is hidden:
 //   O <- O * exp(m_{j-2} - m_{j-1}) + PV_{j-1}.
 template <int DH>
-__global__ void __launch_bounds__(kThreads, 1)
+__global__ void __launch_bounds__(kThreadsB, 1)
 fa_fwd_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_qkv64, bf16* O,
           float* lse, int B, int s, int nh) {
   using SM = Smem<DH>;
@@ -497,7 +513,8 @@ fa_fwd_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__
   uint8_t* sK[2] = {sQ + SM::kBig, sQ + SM::kBig + 2 * SM::kSmall};
   uint8_t* sV[2] = {sK[0] + SM::kSmall, sK[1] + SM::kSmall};
   uint8_t* sP[2] = {sQ + SM::kBig + 4 * SM::kSmall, sQ + SM::kBig + 4 * SM::kSmall + SM::kP};
-  uint64_t* bar = reinterpret_cast<uint64_t*>(sP[1] + SM::kP);
+  float* xch = reinterpret_cast<float*>(sP[1] + SM::kP);   // [2 halves][128 rows] max / sum exchange
+  uint64_t* bar = reinterpret_cast<uint64_t*>(xch + 2 * kRows);
   uint64_t* q_fullb = bar;          // 1
   uint64_t* k_full = bar + 1;       // 2
   uint64_t* k_empty = bar + 3;      // 2
@@ -521,8 +538,8 @@ fa_fwd_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__
     tma_prefetch_desc(&tm_qkv64);
     mbar_init(q_fullb, 1);
     for (int i = 0; i < 2; ++i) {
-      mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1); mbar_init(&s_full[i], 1); mbar_init(&s_free[i], 4);
-      mbar_init(&p_full[i], 4); mbar_init(&o_full[i], 1); mbar_init(&o_free[i], 4);
+      mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1); mbar_init(&s_full[i], 1); mbar_init(&s_free[i], 8);
+      mbar_init(&p_full[i], 8); mbar_init(&o_full[i], 1); mbar_init(&o_free[i], 8);
     }
     fence_barrier_init();
   }
@@ -595,25 +612,27 @@ fa_fwd_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__
     }
     issue_pv(ntiles - 1);
   } else {
-    const int quarter = warp & 3;
+    // 8 softmax warps: warps w and w+4 share TMEM lane quarter (w & 3); `half` selects the 32 S
+    // columns of each key tile and the DH/2 O columns this warp owns. The row max is exchanged
+    // through smem each tile (64-thread named barrier per quarter); row sums stay partial.
+    const int quarter = warp & 3, half = (warp - 2) >> 2;
     const int row = quarter * 32 + lane;
     const int q = qt * kRows + row;
     const uint32_t lane_off = static_cast<uint32_t>(quarter * 32) << 16;
-    float o[DH];
+    constexpr int HD = DH / 2;
+    float o[HD];
 #pragma unroll
-    for (int d = 0; d < DH; ++d) o[d] = 0.f;
+    for (int d = 0; d < HD; ++d) o[d] = 0.f;
     float m_run = -INFINITY, l_run = 0.f;
-    float m_prev_tile = -INFINITY;   // max used for P of the tile whose PV is pending
-    // fold PV_j (computed relative to m_j) into O (relative to m_{j-1}): O = O*exp(m_{j-1} - m_j) + PV_j
     auto fold = [&](int j, float m_j, float m_before) {
       const int st = j & 1;
       mbar_wait(&o_full[st], (j >> 1) & 1);
       tc_fence_after();
       const float c = exp2f(m_before - m_j);
 #pragma unroll
-      for (int c0 = 0; c0 < DH; c0 += 32) {
+      for (int c0 = 0; c0 < HD; c0 += 32) {
         uint32_t r[32];
-        tmem_ld_32x32b_x32(tm_O + st * DH + c0 + lane_off, r);
+        tmem_ld_32x32b_x32(tm_O + st * DH + half * HD + c0 + lane_off, r);
         tmem_ld_wait();
 #pragma unroll
         for (int e = 0; e < 32; ++e) o[c0 + e] = o[c0 + e] * c + __uint_as_float(r[e]);
@@ -627,33 +646,34 @@ fa_fwd_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__
       const int st = j & 1;
       mbar_wait(&s_full[st], (j >> 1) & 1);
       tc_fence_after();
-      uint32_t sr[64];
-      tmem_ld_32x32b_x32(tm_S + st * kCols + lane_off, *reinterpret_cast<uint32_t(*)[32]>(sr));
-      tmem_ld_32x32b_x32(tm_S + st * kCols + 32 + lane_off, *reinterpret_cast<uint32_t(*)[32]>(sr + 32));
+      uint32_t sr[32];
+      tmem_ld_32x32b_x32(tm_S + st * kCols + half * 32 + lane_off, sr);
       tmem_ld_wait();
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&s_free[st]);
       float mx = m_run;
 #pragma unroll
-      for (int c = 0; c < 64; ++c) {
-        const int key = j * kCols + c;
+      for (int c = 0; c < 32; ++c) {
+        const int key = j * kCols + half * 32 + c;
         float x = __uint_as_float(sr[c]) * sl2;
         if (key > q) x = -INFINITY;
         sr[c] = __float_as_uint(x);
         mx = fmaxf(mx, x);
       }
-      const float m_new = mx;   // finite: key 0 <= q for every row
-      float p[64], ls = 0.f;
+      xch[half * kRows + row] = mx;
+      named_bar(2 + quarter, 64);
+      const float m_new = fmaxf(mx, xch[(half ^ 1) * kRows + row]);   // finite: key 0 <= q
+      named_bar(2 + quarter, 64);                                     // xch reusable next tile
+      float p[32], ls = 0.f;
 #pragma unroll
-      for (int c = 0; c < 64; ++c) {
+      for (int c = 0; c < 32; ++c) {
         p[c] = exp2f(__uint_as_float(sr[c]) - m_new);
         ls += p[c];
       }
       l_run = l_run * exp2f(m_run - m_new) + ls;
       m_run = m_new;
-      // P_j into smem (buffer st is free once PV_{j-2} completed, which fold(j-2) waited on)
-      st_row_sw128(sP[st], row, p);
+      st_half_row_sw128(sP[st], row, 4 * half, p);
       fence_proxy_async();
       __syncwarp();
       if (lane == 0) mbar_arrive(&p_full[st]);
@@ -664,19 +684,22 @@ fa_fwd_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__
       m_pending = m_new;
     }
     fold(ntiles - 1, m_pending, m_folded);
-    // O is relative to m_run (= m_pending of the last tile)
-    const float inv = 1.f / l_run;
+    // total row sum = both halves' partial sums (same running max)
+    xch[half * kRows + row] = l_run;
+    named_bar(2 + quarter, 64);
+    const float l_tot = l_run + xch[(half ^ 1) * kRows + row];
+    const float inv = 1.f / l_tot;
     if (q < s) {
-      bf16* orow = O + (static_cast<long>(b) * s + q) * h + head * DH;
+      bf16* orow = O + (static_cast<long>(b) * s + q) * h + head * DH + half * HD;
 #pragma unroll
-      for (int d = 0; d < DH; d += 8) {
+      for (int d = 0; d < HD; d += 8) {
         uint4 u;
         __nv_bfloat162* hh = reinterpret_cast<__nv_bfloat162*>(&u);
 #pragma unroll
         for (int e = 0; e < 4; ++e) hh[e] = __floats2bfloat162_rn(o[d + 2 * e] * inv, o[d + 2 * e + 1] * inv);
         *reinterpret_cast<uint4*>(orow + d) = u;
       }
-      lse[static_cast<long>(head) * Ttok + static_cast<long>(b) * s + q] = (m_run + log2f(l_run)) / LOG2E;
+      if (half == 0) lse[static_cast<long>(head) * Ttok + static_cast<long>(b) * s + q] = (m_run + log2f(l_tot)) / LOG2E;
     }
   }
   tc_fence_before();
@@ -685,7 +708,7 @@ fa_fwd_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__
 }
 
 template <int DH>
-constexpr int smem_fwd() { return at_least_one_sm(Smem<DH>::kBig + 4 * Smem<DH>::kSmall + 2 * Smem<DH>::kP + 128 + 1024); }
+constexpr int smem_fwd() { return at_least_one_sm(Smem<DH>::kBig + 4 * Smem<DH>::kSmall + 2 * Smem<DH>::kP + 2 * kRows * 4 + 128 + 1024); }
 
 template <int DH>
 bool launch_fwd_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, cudaStream_t st) {
@@ -700,7 +723,7 @@ bool launch_fwd_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, c
     set = true;
   }
   dim3 grid((s + kRows - 1) / kRows, B * nh);
-  fa_fwd_tc<DH><<<grid, kThreads, smem_fwd<DH>(), st>>>(m128, m64, O, lse, B, s, nh);
+  fa_fwd_tc<DH><<<grid, kThreadsB, smem_fwd<DH>(), st>>>(m128, m64, O, lse, B, s, nh);
   note_launch();
   return true;
 }

@@ -122,6 +122,115 @@ __global__ void norm_fwd_k(const T* x, const float* g, const float* b, T* y, flo
   if (lane == 0) { stats[2 * row] = mean; stats[2 * row + 1] = rstd; }
 }
 
+// Row cached in registers: NV uint4 (8 bf16) per lane covers n <= 256 * NV.
+template <bool RMS, int NV>
+__global__ void norm_fwd_reg_k(const __nv_bfloat16* x, const float* g, const float* b, __nv_bfloat16* y, float* stats,
+                               int rows, int n, float eps) {
+  const int row = blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32, lane = threadIdx.x % 32;
+  if (row >= rows) return;
+  const __nv_bfloat16* xr = x + static_cast<long>(row) * n;
+  uint4 v[NV];
+#pragma unroll
+  for (int i = 0; i < NV; ++i) {
+    const int c = (i * 32 + lane) * 8;
+    v[i] = c < n ? *reinterpret_cast<const uint4*>(xr + c) : make_uint4(0, 0, 0, 0);
+  }
+  float mean = 0.f;
+  if (!RMS) {
+    float s = 0.f;
+#pragma unroll
+    for (int i = 0; i < NV; ++i) {
+      const __nv_bfloat16* hv = reinterpret_cast<const __nv_bfloat16*>(&v[i]);
+#pragma unroll
+      for (int j = 0; j < 8; ++j) s += __bfloat162float(hv[j]);
+    }
+    mean = warp_sum(s) / n;
+  }
+  float q = 0.f;
+#pragma unroll
+  for (int i = 0; i < NV; ++i) {
+    const int c = (i * 32 + lane) * 8;
+    if (c >= n) continue;
+    const __nv_bfloat16* hv = reinterpret_cast<const __nv_bfloat16*>(&v[i]);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) { const float d = __bfloat162float(hv[j]) - mean; q += d * d; }
+  }
+  const float rstd = rsqrtf(warp_sum(q) / n + eps);
+  __nv_bfloat16* yr = y + static_cast<long>(row) * n;
+#pragma unroll
+  for (int i = 0; i < NV; ++i) {
+    const int c = (i * 32 + lane) * 8;
+    if (c >= n) continue;
+    const __nv_bfloat16* hv = reinterpret_cast<const __nv_bfloat16*>(&v[i]);
+    const float4 g0 = *reinterpret_cast<const float4*>(g + c), g1 = *reinterpret_cast<const float4*>(g + c + 4);
+    const float gg[8] = {g0.x, g0.y, g0.z, g0.w, g1.x, g1.y, g1.z, g1.w};
+    float bb[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+    if (!RMS) {
+      const float4 b0 = *reinterpret_cast<const float4*>(b + c), b1 = *reinterpret_cast<const float4*>(b + c + 4);
+      bb[0] = b0.x; bb[1] = b0.y; bb[2] = b0.z; bb[3] = b0.w; bb[4] = b1.x; bb[5] = b1.y; bb[6] = b1.z; bb[7] = b1.w;
+    }
+    uint4 o;
+    __nv_bfloat16* ho = reinterpret_cast<__nv_bfloat16*>(&o);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) ho[j] = __float2bfloat16_rn((__bfloat162float(hv[j]) - mean) * rstd * gg[j] + bb[j]);
+    *reinterpret_cast<uint4*>(yr + c) = o;
+  }
+  if (lane == 0) { stats[2 * row] = mean; stats[2 * row + 1] = rstd; }
+}
+
+template <int NV>
+__global__ void norm_bwd_dx_reg_k(const __nv_bfloat16* dy, const __nv_bfloat16* x, const float* stats, const float* g,
+                                  const __nv_bfloat16* dres, __nv_bfloat16* dx, int rows, int n, int rms) {
+  const int row = blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32, lane = threadIdx.x % 32;
+  if (row >= rows) return;
+  const long o = static_cast<long>(row) * n;
+  const float mean = stats[2 * row], rstd = stats[2 * row + 1];
+  uint4 vd[NV], vx[NV];
+#pragma unroll
+  for (int i = 0; i < NV; ++i) {
+    const int c = (i * 32 + lane) * 8;
+    vd[i] = c < n ? *reinterpret_cast<const uint4*>(dy + o + c) : make_uint4(0, 0, 0, 0);
+    vx[i] = c < n ? *reinterpret_cast<const uint4*>(x + o + c) : make_uint4(0, 0, 0, 0);
+  }
+  float sg = 0.f, sgx = 0.f;
+#pragma unroll
+  for (int i = 0; i < NV; ++i) {
+    const int c = (i * 32 + lane) * 8;
+    if (c >= n) continue;
+    const __nv_bfloat16* hd = reinterpret_cast<const __nv_bfloat16*>(&vd[i]);
+    const __nv_bfloat16* hx = reinterpret_cast<const __nv_bfloat16*>(&vx[i]);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const float gp = __bfloat162float(hd[j]) * g[c + j];
+      sg += gp;
+      sgx += gp * (__bfloat162float(hx[j]) - mean) * rstd;
+    }
+  }
+  sg = rms ? 0.f : warp_sum(sg) / n;
+  sgx = warp_sum(sgx) / n;
+#pragma unroll
+  for (int i = 0; i < NV; ++i) {
+    const int c = (i * 32 + lane) * 8;
+    if (c >= n) continue;
+    const __nv_bfloat16* hd = reinterpret_cast<const __nv_bfloat16*>(&vd[i]);
+    const __nv_bfloat16* hx = reinterpret_cast<const __nv_bfloat16*>(&vx[i]);
+    uint4 ur = make_uint4(0, 0, 0, 0);
+    if (dres) ur = *reinterpret_cast<const uint4*>(dres + o + c);
+    const __nv_bfloat16* hr = reinterpret_cast<const __nv_bfloat16*>(&ur);
+    uint4 uo;
+    __nv_bfloat16* ho = reinterpret_cast<__nv_bfloat16*>(&uo);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const float gp = __bfloat162float(hd[j]) * g[c + j];
+      const float xh = (__bfloat162float(hx[j]) - mean) * rstd;
+      float d = (gp - sg - xh * sgx) * rstd;
+      if (dres) d += __bfloat162float(hr[j]);
+      ho[j] = __float2bfloat16_rn(d);
+    }
+    *reinterpret_cast<uint4*>(dx + o + c) = uo;
+  }
+}
+
 template <bool RMS>
 __global__ void norm_fwd_v8_k(const __nv_bfloat16* x, const float* g, const float* b, __nv_bfloat16* y, float* stats,
                               int rows, int n, float eps) {
@@ -284,6 +393,50 @@ __global__ void colsum_partial_v8_k(const __nv_bfloat16* a, const __nv_bfloat16*
   for (int j = 0; j < 8; ++j) {
     partial[static_cast<long>(blk) * n + c8 + j] = s0[j];
     if (mode == 1) partial[static_cast<long>(nblk + blk) * n + c8 + j] = s1[j];
+  }
+}
+
+__global__ void __launch_bounds__(256) colsum_partial_v2_k(const __nv_bfloat16* a, const __nv_bfloat16* x,
+                                                           const float* stats, int rows, int n, int lda, int mode,
+                                                           float* partial, int nblk) {
+  __shared__ float red[2][8][256 + 8];
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int c8 = blockIdx.x * 256 + lane * 8;
+  const int blk = blockIdx.y;
+  const int r0 = static_cast<int>(static_cast<long>(rows) * blk / nblk);
+  const int r1 = static_cast<int>(static_cast<long>(rows) * (blk + 1) / nblk);
+  float s0[8] = {0, 0, 0, 0, 0, 0, 0, 0}, s1[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+  if (c8 < n) {
+    for (int r = r0 + warp; r < r1; r += 8) {
+      const uint4 ua = *reinterpret_cast<const uint4*>(a + static_cast<long>(r) * lda + c8);
+      const __nv_bfloat16* ha = reinterpret_cast<const __nv_bfloat16*>(&ua);
+      if (mode == 0) {
+#pragma unroll
+        for (int j = 0; j < 8; ++j) s0[j] += __bfloat162float(ha[j]);
+        continue;
+      }
+      const uint4 ux = *reinterpret_cast<const uint4*>(x + static_cast<long>(r) * n + c8);
+      const __nv_bfloat16* hx = reinterpret_cast<const __nv_bfloat16*>(&ux);
+      const float mu = stats[2 * r], rs = stats[2 * r + 1];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        const float dy = __bfloat162float(ha[j]);
+        s0[j] += dy * ((__bfloat162float(hx[j]) - mu) * rs);
+        s1[j] += dy;
+      }
+    }
+  }
+#pragma unroll
+  for (int j = 0; j < 8; ++j) { red[0][warp][lane * 8 + j] = s0[j]; red[1][warp][lane * 8 + j] = s1[j]; }
+  __syncthreads();
+  const int c = threadIdx.x;                // one column of the 256 per thread
+  const int col = blockIdx.x * 256 + c;
+  if (col < n) {
+    float t0 = 0.f, t1 = 0.f;
+#pragma unroll
+    for (int w = 0; w < 8; ++w) { t0 += red[0][w][c]; t1 += red[1][w][c]; }
+    partial[static_cast<long>(blk) * n + col] = t0;
+    if (mode == 1) partial[static_cast<long>(nblk + blk) * n + col] = t1;
   }
 }
 
@@ -515,6 +668,18 @@ __global__ void swiglu_bwd_k(const T* GU, const T* dM, T* dGU, int rows, int f) 
   }
 }
 
+template <class T>
+__global__ void gelu_fwd_k(const T* Z, T* G, size_t n) {
+  const float c = 0.7978845608028654f;
+  for (size_t i = blockIdx.x * static_cast<size_t>(blockDim.x) + threadIdx.x; i < n; i += static_cast<size_t>(gridDim.x) * blockDim.x) {
+    const float z = ldf(Z + i);
+    float t;
+    if constexpr (std::is_same<T, __nv_bfloat16>::value) asm("tanh.approx.f32 %0, %1;" : "=f"(t) : "f"(c * (z + 0.044715f * z * z * z)));
+    else t = tanhf(c * (z + 0.044715f * z * z * z));
+    stf(G + i, 0.5f * z * (1.f + t));
+  }
+}
+
 // ---------------------------------------------------------------- softmax-CE
 template <class T>
 __global__ void softmax_ce_k(const float* logits, const int32_t* tok, int ld_tok, int s, int V, float inv_ntok,
@@ -613,7 +778,15 @@ void embed_bwd(const int32_t* tok, int ld_tok, int B, int s, const T* dH, int h,
 template <class T>
 void layernorm_fwd(const T* x, const float* g, const float* b, T* y, float* stats, int rows, int n, float eps, cudaStream_t st) {
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
-    if (n % 8 == 0) { norm_fwd_v8_k<false><<<cdiv(rows, 8), 256, 0, st>>>(x, g, b, y, stats, rows, n, eps); note_launch(); return; }
+    if (n % 8 == 0) {
+      if (n <= 1024) norm_fwd_reg_k<false, 4><<<cdiv(rows, 8), 256, 0, st>>>(x, g, b, y, stats, rows, n, eps);
+      else if (n <= 2048) norm_fwd_reg_k<false, 8><<<cdiv(rows, 8), 256, 0, st>>>(x, g, b, y, stats, rows, n, eps);
+      else if (n <= 4096) norm_fwd_reg_k<false, 16><<<cdiv(rows, 8), 256, 0, st>>>(x, g, b, y, stats, rows, n, eps);
+      else if (n <= 5120) norm_fwd_reg_k<false, 20><<<cdiv(rows, 8), 256, 0, st>>>(x, g, b, y, stats, rows, n, eps);
+      else norm_fwd_v8_k<false><<<cdiv(rows, 8), 256, 0, st>>>(x, g, b, y, stats, rows, n, eps);
+      note_launch();
+      return;
+    }
   }
   norm_fwd_k<T, false><<<cdiv(rows, 8), 256, 0, st>>>(x, g, b, y, stats, rows, n, eps);
   note_launch();
@@ -621,7 +794,15 @@ void layernorm_fwd(const T* x, const float* g, const float* b, T* y, float* stat
 template <class T>
 void rmsnorm_fwd(const T* x, const float* g, T* y, float* stats, int rows, int n, float eps, cudaStream_t st) {
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
-    if (n % 8 == 0) { norm_fwd_v8_k<true><<<cdiv(rows, 8), 256, 0, st>>>(x, g, nullptr, y, stats, rows, n, eps); note_launch(); return; }
+    if (n % 8 == 0) {
+      if (n <= 1024) norm_fwd_reg_k<true, 4><<<cdiv(rows, 8), 256, 0, st>>>(x, g, nullptr, y, stats, rows, n, eps);
+      else if (n <= 2048) norm_fwd_reg_k<true, 8><<<cdiv(rows, 8), 256, 0, st>>>(x, g, nullptr, y, stats, rows, n, eps);
+      else if (n <= 4096) norm_fwd_reg_k<true, 16><<<cdiv(rows, 8), 256, 0, st>>>(x, g, nullptr, y, stats, rows, n, eps);
+      else if (n <= 5120) norm_fwd_reg_k<true, 20><<<cdiv(rows, 8), 256, 0, st>>>(x, g, nullptr, y, stats, rows, n, eps);
+      else norm_fwd_v8_k<true><<<cdiv(rows, 8), 256, 0, st>>>(x, g, nullptr, y, stats, rows, n, eps);
+      note_launch();
+      return;
+    }
   }
   norm_fwd_k<T, true><<<cdiv(rows, 8), 256, 0, st>>>(x, g, nullptr, y, stats, rows, n, eps);
   note_launch();
@@ -630,7 +811,13 @@ template <class T>
 void norm_bwd_dx(const T* dy, const T* x, const float* stats, const float* g, const T* dres, T* dx, int rows, int n,
                  int rms, cudaStream_t st) {
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
-    if (n % 8 == 0) { norm_bwd_dx_v8_k<<<cdiv(rows, 8), 256, 0, st>>>(dy, x, stats, g, dres, dx, rows, n, rms); note_launch(); return; }
+    if (n % 8 == 0) {
+      if (n <= 1024) norm_bwd_dx_reg_k<4><<<cdiv(rows, 8), 256, 0, st>>>(dy, x, stats, g, dres, dx, rows, n, rms);
+      else if (n <= 2048) norm_bwd_dx_reg_k<8><<<cdiv(rows, 8), 256, 0, st>>>(dy, x, stats, g, dres, dx, rows, n, rms);
+      else norm_bwd_dx_v8_k<<<cdiv(rows, 8), 256, 0, st>>>(dy, x, stats, g, dres, dx, rows, n, rms);
+      note_launch();
+      return;
+    }
   }
   norm_bwd_dx_k<T><<<cdiv(rows, 8), 256, 0, st>>>(dy, x, stats, g, dres, dx, rows, n, rms);
   note_launch();
@@ -642,8 +829,13 @@ void colsum(const T* a, const T* x, const float* stats, int rows, int n, int lda
   if (nblk < 1) return;
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
     if (n % 8 == 0 && lda % 8 == 0) {
-      dim3 grid(cdiv(n / 8, 128), nblk);
-      colsum_partial_v8_k<<<grid, 128, 0, st>>>(a, x, stats, rows, n, lda, mode == 2 ? 1 : mode, partial, nblk);
+      const int cb = cdiv(n, 256);
+      int rb = (2 * 148 + cb - 1) / cb;
+      rb = rb < 1 ? 1 : (rb > 128 ? 128 : rb);
+      rb = rb > rows ? rows : rb;
+      nblk = rb;
+      dim3 grid(cb, nblk);
+      colsum_partial_v2_k<<<grid, 256, 0, st>>>(a, x, stats, rows, n, lda, mode == 2 ? 1 : mode, partial, nblk);
       note_launch();
       colsum_final_k<<<cdiv(n, 256), 256, 0, st>>>(partial, nblk, n, mode == 2 ? 0 : mode, out0, out1);
       note_launch();
@@ -699,6 +891,11 @@ void softmax_ce(const float* logits, const int32_t* tok, int ld_tok, int s, int 
   softmax_ce_k<T><<<rows, 512, 0, st>>>(logits, tok, ld_tok, s, V, inv_ntok, dlogits, row_loss);
   note_launch();
 }
+template <class T>
+void gelu_fwd(const T* Z, T* G, size_t n, cudaStream_t st) {
+  gelu_fwd_k<T><<<grid_for(static_cast<long>(n)), 256, 0, st>>>(Z, G, n);
+  note_launch();
+}
 void loss_reduce(const float* row_loss, int rows, double* out, cudaStream_t st) {
   loss_reduce_k<<<1, 1024, 0, st>>>(row_loss, rows, out);
   note_launch();
@@ -723,7 +920,8 @@ void copy_f32(float* a, const float* b, size_t n, cudaStream_t st) { copy_k<<<gr
   template void rope<T>(T*, int, int, int, int, float, int, cudaStream_t);                                           \
   template void swiglu_fwd<T>(const T*, T*, int, int, cudaStream_t);                                                 \
   template void swiglu_bwd<T>(const T*, const T*, T*, int, int, cudaStream_t);                                       \
-  template void softmax_ce<T>(const float*, const int32_t*, int, int, int, int, float, T*, float*, cudaStream_t);
+  template void softmax_ce<T>(const float*, const int32_t*, int, int, int, int, float, T*, float*, cudaStream_t); \
+  template void gelu_fwd<T>(const T*, T*, size_t, cudaStream_t);
 INST(float)
 INST(__nv_bfloat16)
 

@@ -41,6 +41,9 @@ template <class T> void rope(T* qkv, int B, int s, int nh, int dh, float base, i
 template <class T> void swiglu_fwd(const T* GU, T* M, int rows, int f, cudaStream_t st);
 template <class T> void swiglu_bwd(const T* GU, const T* dM, T* dGU, int rows, int f, cudaStream_t st);
 
+// G = gelu_tanh(Z) elementwise (backward recompute of the MLP activation, GPT).
+template <class T> void gelu_fwd(const T* Z, T* G, size_t n, cudaStream_t st);
+
 // Softmax cross-entropy over fp32 logits [rows, V]: row_loss[r] = lse - z_y;
 // dlogits (T) = (softmax - onehot) * inv_ntok. labels = tokens[:, 1:] of the micro-batch.
 template <class T> void softmax_ce(const float* logits, const int32_t* tok, int ld_tok, int s, int rows, int V,

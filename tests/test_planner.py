@@ -139,3 +139,23 @@ def test_library_exports_every_declared_symbol():
     assert len(set(names)) > 15
     for n in set(names):
         assert hasattr(lib, n), n
+
+
+def test_cfg5_memory_cap_base_infeasible_mario_fits():
+    """BASELINE.json configs[4]: LLaMA2-13B, s = 16384, 8 stages, 40 GB per GPU (the paper's
+    A100-40G): plain 1F1B exceeds the cap on device 0 (Table 1: D x M_theta), full-checkpoint
+    1F1B and Mario fit (M_theta per device), and Mario's simulated makespan beats ckpt."""
+    cfg = synth.LLAMA2_13B
+    cap = 40 * 10 ** 9
+    with pytest.raises(MarioError) as e:
+        Plan(cfg, 8, 16, "1f1b", "base", dtype="bf16", mem_budget=cap)
+    assert e.value.code == -2
+    ck = Plan(cfg, 8, 16, "1f1b", "ckpt", dtype="bf16", mem_budget=cap).simulate()
+    ma = Plan(cfg, 8, 16, "1f1b", "mario", dtype="bf16", mem_budget=cap).simulate()
+    assert max(ma.peak_bytes) <= cap and max(ck.peak_bytes) <= cap
+    assert ma.makespan_ms < ck.makespan_ms
+    assert ma.max_live_act == [1] * 8
+    base = Plan(cfg, 8, 16, "1f1b", "base", dtype="bf16").simulate()
+    assert base.max_live_act == [8, 7, 6, 5, 4, 3, 2, 1]            # Table 1, P:92
+    assert max(base.peak_bytes) / min(base.peak_bytes) > 2.0          # imbalanced
+    assert max(ma.peak_bytes) / min(ma.peak_bytes) < 1.25            # balanced (SURVEY d3 bar)
