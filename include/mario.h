@@ -129,6 +129,30 @@ const char* mario_param_name(const struct mario_plan* plan, int32_t idx);
 int32_t mario_param_count(const struct mario_plan* plan);
 void mario_plan_destroy(struct mario_plan* plan);
 
+/* Schedule tuner (§5.3, Eq. 1): grid search
+ *   max F(b, E(a, b, pp, mbs), dmem, dp)  over  a in {no ckpt (BASE), Mario (passes 1-4)},
+ *   b in {1F1B, Interleave (v = 2), Chimera}, pp in [min(4, D), D] with dp * pp = D,
+ *   mbs in {1, 2, 4, 8, ...} with global_batch = dp * mbs * N,
+ * where F = global_batch / simulated makespan, times dp_efficiency if dp > 1, and F = 0 when the
+ * simulated per-device peak exceeds mem_budget_bytes. Per-layer costs per micro-batch
+ * size (the profiled estimators E) may be supplied; NULL arrays = analytic (FLOPs at
+ * 1 PFLOP/s, linear in mbs). Writes up to cap results (every evaluated configuration) and the
+ * index of the best one (-1 if none is feasible). The "Auto" scheme of P:167 is the best row. */
+typedef struct {
+  int32_t n_mbs;              /* number of micro-batch sizes in mbs[] (0 = {1,2,4,8})        */
+  const int32_t* mbs;
+  const double *layer_fw_ms, *layer_bw_ms, *head_fw_ms, *head_bw_ms;   /* [n_mbs] or NULL */
+  double p2p_alpha_ms, p2p_GBps, dp_efficiency;
+} mario_tune_costs;
+typedef struct {
+  int32_t scheme, pp, chunks, dp, micro_batch, microbatches, level, feasible;
+  double makespan_ms, samples_per_s, bubble_ratio;
+  uint64_t peak_bytes;
+} mario_tune_result;
+mario_status mario_tune(const mario_model* model, int32_t devices, int32_t global_batch, uint64_t mem_budget_bytes,
+                        const mario_tune_costs* costs, mario_tune_result* results, int32_t cap, int32_t* n,
+                        int32_t* best);
+
 /* Executor context. world == 1 with a multi-stage plan runs every rank's list in this
  * process on one GPU ("loopback": device-to-device copies instead of NCCL). world > 1:
  * one process per GPU, nccl_unique_id = 128 bytes from mario_nccl_unique_id() on rank 0. */

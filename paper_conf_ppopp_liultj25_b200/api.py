@@ -55,6 +55,20 @@ class CSim(C.Structure):
                 ("max_live_act", C.POINTER(C.c_int32)), ("max_live_ckpt", C.POINTER(C.c_int32))]
 
 
+class CTuneCosts(C.Structure):
+    _fields_ = [("n_mbs", C.c_int32), ("mbs", C.POINTER(C.c_int32)), ("layer_fw_ms", C.POINTER(C.c_double)),
+                ("layer_bw_ms", C.POINTER(C.c_double)), ("head_fw_ms", C.POINTER(C.c_double)),
+                ("head_bw_ms", C.POINTER(C.c_double)), ("p2p_alpha_ms", C.c_double), ("p2p_GBps", C.c_double),
+                ("dp_efficiency", C.c_double)]
+
+
+class CTuneResult(C.Structure):
+    _fields_ = [("scheme", C.c_int32), ("pp", C.c_int32), ("chunks", C.c_int32), ("dp", C.c_int32),
+                ("micro_batch", C.c_int32), ("microbatches", C.c_int32), ("level", C.c_int32),
+                ("feasible", C.c_int32), ("makespan_ms", C.c_double), ("samples_per_s", C.c_double),
+                ("bubble_ratio", C.c_double), ("peak_bytes", C.c_uint64)]
+
+
 _P = C.c_void_p
 _lib.register("mario_plan", C.c_int32, [C.POINTER(CModel), C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_uint64,
                                         C.c_int32, C.POINTER(CCosts), C.POINTER(_P)])
@@ -72,6 +86,8 @@ _lib.register("mario_param_name", C.c_char_p, [_P, C.c_int32])
 _lib.register("mario_param_count", C.c_int32, [_P])
 _lib.register("mario_plan_destroy", None, [_P])
 _lib.register("mario_last_error", C.c_char_p, [])
+_lib.register("mario_tune", C.c_int32, [C.POINTER(CModel), C.c_int32, C.c_int32, C.c_uint64, C.POINTER(CTuneCosts),
+                                        C.POINTER(CTuneResult), C.c_int32, C.POINTER(C.c_int32), C.POINTER(C.c_int32)])
 _lib.register("mario_nccl_unique_id", C.c_int32, [C.c_void_p])
 _lib.register("mario_init", C.c_int32, [C.c_int32, C.c_int32, C.c_int32, C.c_void_p])
 _lib.register("mario_run_iter", C.c_int32, [_P, C.c_void_p, C.c_void_p, C.POINTER(C.c_float), C.c_void_p,
@@ -292,3 +308,34 @@ def alloc_for(plan: Plan, rank: int, device="cuda"):
     g = torch.zeros(pc, dtype=torch.float32, device=device)
     work = torch.empty(max(ws, 1), dtype=torch.uint8, device=device)
     return w, g, work
+
+
+SCHEME_NAMES = {0: "1f1b", 1: "interleave", 2: "chimera"}
+LEVEL_NAMES = {0: "base", 1: "ckpt", 2: "mario"}
+
+
+def tune(cfg, devices: int, global_batch: int, mem_budget: int = 0, costs: Optional[dict] = None,
+         dtype: str = "bf16"):
+    """mario_tune (Eq. 1): returns (all evaluated configurations as dicts, index of the best)."""
+    m = cmodel(cfg, dtype)
+    cc = None
+    keep = []
+    if costs is not None:
+        mbs = costs.get("mbs", [])
+        keep = [(C.c_int32 * len(mbs))(*mbs)] + [_darr(costs.get(k)) for k in ("layer_fw_ms", "layer_bw_ms",
+                                                                               "head_fw_ms", "head_bw_ms")]
+        cc = CTuneCosts(len(mbs), keep[0], keep[1], keep[2], keep[3], keep[4], costs.get("p2p_alpha_ms", 0.01),
+                        costs.get("p2p_GBps", 700.0), costs.get("dp_efficiency", 0.95))
+    cap = 1024
+    res = (CTuneResult * cap)()
+    n, best = C.c_int32(), C.c_int32()
+    _check(_lib.lib().mario_tune(C.byref(m), devices, global_batch, mem_budget, C.byref(cc) if cc else None, res,
+                                 cap, C.byref(n), C.byref(best)))
+    rows = []
+    for i in range(n.value):
+        r = res[i]
+        rows.append({"scheme": SCHEME_NAMES[r.scheme], "pp": r.pp, "chunks": r.chunks, "dp": r.dp,
+                     "micro_batch": r.micro_batch, "microbatches": r.microbatches, "level": LEVEL_NAMES[r.level],
+                     "feasible": bool(r.feasible), "makespan_ms": r.makespan_ms, "samples_per_s": r.samples_per_s,
+                     "bubble_ratio": r.bubble_ratio, "peak_bytes": r.peak_bytes})
+    return rows, best.value

@@ -5,6 +5,7 @@
 
 #include <algorithm>
 #include <cmath>
+#include <limits>
 #include <map>
 #include <set>
 #include <stdexcept>
@@ -226,13 +227,14 @@ Lists pass3_remove_redundancy(const Lists& in) {
 // block the device until the data arrives; sends are buffered and posted when everything
 // before them in the list has completed.
 SimResult simulate(const Pipe& pp, const Lists& L, const SimCosts& c) {
-  const int S = pp.S;
+  const int S = pp.S, P = pp.parts();
   SimResult r;
   r.busy.assign(S, 0.0);
   r.start.assign(S, {});
   r.finish.assign(S, {});
-  // post time of sends, keyed by (device, op, m, p)
-  std::map<std::tuple<int, int, int, int>, double> post;
+  // post time of sends, flat index ((device * N + micro) * parts + part) * 2 + (SG ? 1 : 0); NaN = not posted
+  std::vector<double> post(static_cast<size_t>(S) * pp.N * P * 2, std::numeric_limits<double>::quiet_NaN());
+  auto key = [&](int d, int m, int p, bool grad) { return ((static_cast<size_t>(d) * pp.N + m) * P + p) * 2 + (grad ? 1 : 0); };
   std::vector<size_t> ptr(S, 0);
   std::vector<double> dev_t(S, 0.0);
   size_t total = 0, done = 0;
@@ -247,13 +249,13 @@ SimResult simulate(const Pipe& pp, const Lists& L, const SimCosts& c) {
         const Instr& x = l[ptr[d]];
         const int k = pp.vstage(d, x.p);
         if (is_send(x.op)) {
-          post[{d, x.op, x.m, x.p}] = dev_t[d];
+          post[key(d, x.m, x.p, x.op == SG)] = dev_t[d];
         } else if (is_recv(x.op)) {
           int sd, sp;
           if (!find_inst(pp, d, x.m, x.p, x.op == RA ? FW : BW, false, &sd, &sp)) return r;  // malformed
-          auto it = post.find({sd, x.op == RA ? SA : SG, x.m, sp});
-          if (it == post.end()) break;
-          dev_t[d] = std::max(dev_t[d], it->second + (x.op == RA ? c.comm_act : c.comm_grad));
+          const double t = post[key(sd, x.m, sp, x.op == RG)];
+          if (std::isnan(t)) break;
+          dev_t[d] = std::max(dev_t[d], t + (x.op == RA ? c.comm_act : c.comm_grad));
         } else {
           double dur = (x.op == FW || x.op == CFW) ? c.fw[k] : x.op == RC ? c.rc[k] : c.bw[k];
           r.start[d].push_back(dev_t[d]);
