@@ -172,6 +172,12 @@ mario_status mario_run_iter(const struct mario_plan* plan, const void* weights, 
  * iteration start, CUDA events) when timing was enabled with mario_set_timing(1). */
 mario_status mario_set_timing(int32_t enable);
 mario_status mario_last_timeline(int32_t device, const double** start_ms, const double** finish_ms, int32_t* n);
+/* OS (Table 3): AdamW (reading A27: decoupled weight decay, bias correction; step >= 1)
+ * applied in place to n packed fp32 parameters with fp32 moments m, v (device pointers, caller
+ * owned, zero-initialised before step 1); grads as returned by mario_run_iter. Asynchronous on
+ * `stream`. EINVAL on NULL pointers or step < 1. */
+mario_status mario_adamw_step(void* params, const void* grads, void* m, void* v, uint64_t n, float lr, float beta1,
+                              float beta2, float eps, float weight_decay, int32_t step, void* stream);
 mario_status mario_finalize(void);
 const char* mario_last_error(void);
 

@@ -96,6 +96,8 @@ _lib.register("mario_set_timing", C.c_int32, [C.c_int32])
 _lib.register("mario_last_timeline", C.c_int32, [C.c_int32, C.POINTER(C.POINTER(C.c_double)),
                                                  C.POINTER(C.POINTER(C.c_double)), C.POINTER(C.c_int32)])
 _lib.register("mario_finalize", C.c_int32, [])
+_lib.register("mario_adamw_step", C.c_int32, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint64, C.c_float,
+                                              C.c_float, C.c_float, C.c_float, C.c_float, C.c_int32, C.c_void_p])
 
 
 def _check(code):
@@ -339,3 +341,32 @@ def tune(cfg, devices: int, global_batch: int, mem_budget: int = 0, costs: Optio
                      "feasible": bool(r.feasible), "makespan_ms": r.makespan_ms, "samples_per_s": r.samples_per_s,
                      "bubble_ratio": r.bubble_ratio, "peak_bytes": r.peak_bytes})
     return rows, best.value
+
+
+def adamw_step(params, grads, m, v, step: int, lr: float, beta1=0.9, beta2=0.95, eps=1e-8, weight_decay=0.1,
+               stream=None):
+    """mario_adamw_step on packed device buffers (torch tensors)."""
+    st = stream.cuda_stream if stream is not None else None
+    _check(_lib.lib().mario_adamw_step(C.c_void_p(params.data_ptr()), C.c_void_p(grads.data_ptr()),
+                                       C.c_void_p(m.data_ptr()), C.c_void_p(v.data_ptr()), params.numel(), lr, beta1,
+                                       beta2, eps, weight_decay, step, C.c_void_p(st) if st else None))
+
+
+def chrome_trace(plan: Plan, measured: Optional[List[Tuple[List[float], List[float]]]] = None) -> dict:
+    """Chrome-trace (chrome://tracing / Perfetto) of a plan's simulated timeline (pid 0) and,
+    optionally, a measured one from Context.last_timeline per device (pid 1): the visualization of
+    PAPER.md P:256 (Fig. 5), one row per device, one box per FW/CFW/RC/BW instruction."""
+    events = []
+    for pid, label, src in ((0, "simulated", None), (1, "measured", measured)):
+        if pid == 1 and measured is None:
+            continue
+        events.append({"name": "process_name", "ph": "M", "pid": pid, "args": {"name": label}})
+        for d in range(plan.S):
+            comp = [x for x in plan.instrs(d) if x[0] in ("FW", "CFW", "RC", "BW")]
+            starts, fins = plan.timeline(d) if src is None else src[d]
+            events.append({"name": "thread_name", "ph": "M", "pid": pid, "tid": d, "args": {"name": f"device {d}"}})
+            for (op, m, p, k, *_r), t0, t1 in zip(comp, starts, fins):
+                events.append({"name": f"{op}{m}" + (f".{p}" if plan.scheme != "1f1b" else ""), "cat": op, "ph": "X",
+                               "pid": pid, "tid": d, "ts": t0 * 1e3, "dur": (t1 - t0) * 1e3,
+                               "args": {"micro": m, "part": p, "vstage": k}})
+    return {"traceEvents": events, "displayTimeUnit": "ms"}

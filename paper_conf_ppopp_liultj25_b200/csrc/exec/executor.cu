@@ -792,6 +792,23 @@ extern "C" mario_status mario_run_iter(const struct mario_plan* plan, const void
   }
 }
 
+namespace mario {
+void adamw_step(float* p, const float* g, float* m, float* v, size_t n, float lr, float b1, float b2, float eps,
+                float wd, int step, cudaStream_t st);
+}
+
+extern "C" mario_status mario_adamw_step(void* params, const void* grads, void* m, void* v, uint64_t n, float lr,
+                                         float beta1, float beta2, float eps, float weight_decay, int32_t step,
+                                         void* stream) {
+  if (!params || !grads || !m || !v || step < 1) return set_error(MARIO_EINVAL, "bad argument");
+  mario::adamw_step(static_cast<float*>(params), static_cast<const float*>(grads), static_cast<float*>(m),
+                    static_cast<float*>(v), static_cast<size_t>(n), lr, beta1, beta2, eps, weight_decay, step,
+                    static_cast<cudaStream_t>(stream));
+  const cudaError_t e = cudaGetLastError();
+  if (e != cudaSuccess) return set_error(MARIO_ECUDA, cudaGetErrorString(e));
+  return MARIO_OK;
+}
+
 extern "C" mario_status mario_set_timing(int32_t enable) {
   g.timing = enable != 0;
   return MARIO_OK;

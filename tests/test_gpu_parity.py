@@ -143,3 +143,45 @@ def test_full_width_parity_bf16(name, cfg, scheme, S, N, v, tol, guard):
     l_o, g_o = om.step(cfg, rounded(params), toks, N, np.float32)
     wi, wl = check(loss, grads, l_o, g_o, tol, norm="l2", inf_guard=guard)
     print(f"[full-width {name}] loss {loss:.6f} vs {l_o:.6f}; worst inf-rel {wi}; worst l2-rel {wl}")
+
+
+def test_training_loop_adamw_matches_oracle():
+    """Five iterations of run_iter + mario_adamw_step (fp32 mode, Mario plan, S = 2 loopback)
+    follow the oracle's loss trajectory (oracle.model.step + oracle.optim.adamw_step), and the
+    loss decreases."""
+    from oracle import optim
+    cfg = synth.TINY_GPT
+    params = synth.make_weights(cfg)
+    plan = api.Plan(cfg, 2, 4, "1f1b", "mario", dtype="f32")
+    w, g, ws = api.alloc_for(plan, -1)
+    w.copy_(torch.from_numpy(api.pack_params(plan, params, -1)))
+    m_, v_ = torch.zeros_like(w), torch.zeros_like(w)
+    P = {k: v.astype(np.float64) for k, v in params.items()}
+    M = {k: np.zeros_like(v) for k, v in P.items()}
+    V = {k: np.zeros_like(v) for k, v in P.items()}
+    gpu_losses, ora_losses = [], []
+    toks = synth.make_tokens(cfg, 4)      # one fixed batch: uniform tokens are only learnable by memorizing
+    for it in range(1, 6):
+        gpu_losses.append(ctx().run_iter(plan, w, toks, g, ws))
+        api.adamw_step(w, g, m_, v_, it, lr=3e-3)
+        l_o, G_o = om.step(cfg, P, toks, 4, np.float64)
+        ora_losses.append(l_o)
+        optim.adamw_step(P, G_o, M, V, it, lr=3e-3)
+    torch.cuda.synchronize()
+    assert np.allclose(gpu_losses, ora_losses, rtol=2e-4), (gpu_losses, ora_losses)
+    assert ora_losses[-1] < ora_losses[0]
+    # every copy of a parameter (the two tied wte copies) stays bitwise identical, and no weight
+    # moved further from the oracle than Adam's per-step bound lr * steps (its normalized update
+    # makes near-zero gradients of either sign move a weight by up to lr per step)
+    flat = w.cpu().numpy()
+    copies = {}
+    base = 0
+    for r in range(plan.S):
+        for name, off, cnt in plan.rank_params(r):
+            copies.setdefault(name, []).append(flat[base + off: base + off + cnt])
+        base += plan.rank_layout(r)[0]
+    assert len(copies["wte"]) == 2 and np.array_equal(copies["wte"][0], copies["wte"][1])
+    for k in P:
+        d = np.abs(copies[k][0].reshape(P[k].shape) - P[k])
+        assert d.max() <= 5 * 3e-3 + 1e-6, k
+        assert np.median(d) < 1e-4, k

@@ -248,3 +248,29 @@ def test_initial_loss_near_lnV():
     P = synth.make_weights(cfg, parity=False)
     loss, _ = om.step(cfg, P, synth.make_tokens(cfg, 2), 2, np.float32)
     assert abs(loss - math.log(cfg.vocab)) < 0.05
+
+
+def test_adamw_oracle_closed_forms():
+    """Pins for oracle/optim.py: step 1 with g != 0 moves every weight by lr*(sign(g) + wd*p)
+    up to eps (bias-corrected m/sqrt(v) = g/|g|); zero grads only decay; a constant gradient
+    keeps the normalized update at 1."""
+    from oracle import optim
+    rng = np.random.default_rng(0)
+    p = {"w": rng.standard_normal(50)}
+    g = {"w": rng.standard_normal(50)}
+    m = {"w": np.zeros(50)}
+    v = {"w": np.zeros(50)}
+    p0 = p["w"].copy()
+    optim.adamw_step(p, g, m, v, 1, lr=1e-2, eps=0.0, weight_decay=0.1)
+    assert np.allclose(p["w"], p0 - 1e-2 * (np.sign(g["w"]) + 0.1 * p0), atol=1e-15)
+    q = {"w": p0.copy()}
+    z = {"w": np.zeros(50)}
+    optim.adamw_step(q, z, {"w": np.zeros(50)}, {"w": np.zeros(50)}, 1, lr=1e-2, eps=1e-8, weight_decay=0.1)
+    assert np.allclose(q["w"], p0 * (1 - 1e-3), atol=1e-15)
+    c = {"w": np.full(50, 0.3)}
+    r = {"w": np.zeros(50)}
+    mm, vv = {"w": np.zeros(50)}, {"w": np.zeros(50)}
+    for t in range(1, 6):
+        before = r["w"].copy()
+        optim.adamw_step(r, c, mm, vv, t, lr=1.0, eps=0.0, weight_decay=0.0)
+        assert np.allclose(before - r["w"], 1.0, atol=1e-12)

@@ -9,6 +9,7 @@ import pytest
 import synth
 from oracle import schedule as osch
 from paper_conf_ppopp_liultj25_b200 import _lib
+from paper_conf_ppopp_liultj25_b200 import api
 from paper_conf_ppopp_liultj25_b200.api import MarioError, Plan
 
 TINY = synth.TINY_GPT
@@ -159,3 +160,14 @@ def test_cfg5_memory_cap_base_infeasible_mario_fits():
     assert base.max_live_act == [8, 7, 6, 5, 4, 3, 2, 1]            # Table 1
     assert max(base.peak_bytes) / min(base.peak_bytes) > 2.0          # imbalanced
     assert max(ma.peak_bytes) / min(ma.peak_bytes) < 1.25            # balanced (SURVEY d3 bar)
+
+
+def test_chrome_trace_of_fig2():
+    """P:256 visualization: one box per compute instruction, simulated start/finish."""
+    import json
+    p = Plan(model_for(4), 4, 4, "1f1b", "mario", dtype="f32", costs=unit_costs(4))
+    tr = api.chrome_trace(p)
+    boxes = [e for e in tr["traceEvents"] if e.get("ph") == "X"]
+    assert len(boxes) == sum(1 for d in range(4) for x in p.instrs(d) if x[0] in ("FW", "CFW", "RC", "BW"))
+    assert max(e["ts"] + e["dur"] for e in boxes) == 22.0 * 1e3   # Fig. 2 step 4: 22t
+    json.dumps(tr)
