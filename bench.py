@@ -44,6 +44,7 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-projection", action="store_true")
+    ap.add_argument("--graphs", type=int, default=1, help="also time CUDA-graph replay (N = 1)")
     return ap.parse_args()
 
 
@@ -305,6 +306,25 @@ def main():
         e2e = {"value": gbs / dt, "unit": UNIT, "h2d_bytes_per_step": int(tok_host[0].nbytes),
                "d2h_bytes_per_step": 4 + 8 * args.micro}
 
+    # CUDA-graph replay of the same iteration (mario_set_graphs), timed separately: the headline
+    # region above runs eager so that the per-kernel roofline is measured live inside it
+    graph_replay = None
+    if world == 1 and args.graphs:
+        ctx.set_graphs(True)
+        for i in range(2):
+            ctx.run_iter(plan, w, tok_dev[i], grads, ws, stream)   # capture on the 2nd call
+        torch.cuda.synchronize()
+        g0 = L.mario_kernel_launches()
+        e0.record(stream)
+        for i in range(args.steps):
+            ctx.run_iter(plan, w, tok_dev[args.warmup + i], grads, ws, stream)
+        e1.record(stream)
+        torch.cuda.synchronize()
+        gms = e0.elapsed_time(e1) / args.steps
+        graph_replay = {"value": gbs / (gms / 1e3), "ms_per_step": gms,
+                        "gpu_launches": int(L.mario_kernel_launches() - g0)}
+        ctx.set_graphs(False)
+
     sim = plan.simulate()
     peaks, peak_kind = measured_peaks()
     g = kst["gemm"]
@@ -333,7 +353,7 @@ def main():
            "bubble": {"simulated": sim.bubble_ratio, "stages": world},
            "peak_mem_per_stage": {"simulated_bytes": sim.peak_bytes,
                                   "measured_torch_max_allocated": int(mem)},
-           "e2e": e2e}
+           "e2e": e2e, "graph_replay": graph_replay}
     if rank == 0 and world == 1 and not args.no_projection:
         out["pipeline_projection_8gpu"] = project_pipeline(cfg, api, torch, lambda: ctx)
     if rank == 0 and world == 1 and not args.no_cpu_baseline:

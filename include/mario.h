@@ -168,6 +168,11 @@ mario_status mario_init(int32_t rank, int32_t world, int32_t device, const void*
  *  stream  : caller's cudaStream_t; the call synchronizes it before returning. */
 mario_status mario_run_iter(const struct mario_plan* plan, const void* weights, const int32_t* tokens,
                             float* loss, void* grads, void* workspace, void* stream);
+/* Replay single-process iterations (world = 1: S = 1 or loopback) from a CUDA graph captured on
+ * the second call with the same (plan, weights, grads, workspace) pointers; the graph is reused
+ * while those pointers are unchanged (weights may change in place, e.g. by mario_adamw_step).
+ * Disabled automatically while timing or kernel statistics are enabled. 0 disables and frees. */
+mario_status mario_set_graphs(int32_t enable);
 /* Per-instruction measured timeline of the last mario_run_iter on this rank (ms from the
  * iteration start, CUDA events) when timing was enabled with mario_set_timing(1). */
 mario_status mario_set_timing(int32_t enable);

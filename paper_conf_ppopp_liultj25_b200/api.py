@@ -93,6 +93,7 @@ _lib.register("mario_init", C.c_int32, [C.c_int32, C.c_int32, C.c_int32, C.c_voi
 _lib.register("mario_run_iter", C.c_int32, [_P, C.c_void_p, C.c_void_p, C.POINTER(C.c_float), C.c_void_p,
                                             C.c_void_p, C.c_void_p])
 _lib.register("mario_set_timing", C.c_int32, [C.c_int32])
+_lib.register("mario_set_graphs", C.c_int32, [C.c_int32])
 _lib.register("mario_last_timeline", C.c_int32, [C.c_int32, C.POINTER(C.POINTER(C.c_double)),
                                                  C.POINTER(C.POINTER(C.c_double)), C.POINTER(C.c_int32)])
 _lib.register("mario_finalize", C.c_int32, [])
@@ -288,6 +289,9 @@ class Context:
                                          C.c_void_p(grads.data_ptr()), C.c_void_p(workspace.data_ptr()),
                                          C.c_void_p(st) if st else None))
         return float(loss.value)
+
+    def set_graphs(self, on: bool):
+        _check(_lib.lib().mario_set_graphs(int(on)))
 
     def set_timing(self, on: bool):
         _check(_lib.lib().mario_set_timing(int(on)))

@@ -185,3 +185,28 @@ def test_training_loop_adamw_matches_oracle():
         d = np.abs(copies[k][0].reshape(P[k].shape) - P[k])
         assert d.max() <= 5 * 3e-3 + 1e-6, k
         assert np.median(d) < 1e-4, k
+
+
+@pytest.mark.parametrize("S", [1, 2])
+def test_cuda_graph_replay_bitwise(S):
+    """mario_set_graphs: the 2nd call captures, later calls replay; every call must equal the eager
+    result bit for bit, with different tokens per call (tokens are copied outside the graph)."""
+    cfg = synth.tiny_llama()
+    params = synth.make_weights(cfg)
+    plan = api.Plan(cfg, S, 4, "1f1b", "mario", dtype="bf16")
+    rank = -1 if S > 1 else 0
+    w, g, ws = api.alloc_for(plan, rank)
+    w.copy_(torch.from_numpy(api.pack_params(plan, params, rank)))
+    toks = [synth.make_tokens(cfg, 4, iteration=i) for i in range(4)]
+    eager = []
+    for t in toks:
+        l = ctx().run_iter(plan, w, t, g, ws)
+        eager.append((l, g.cpu().numpy().copy()))
+    ctx().set_graphs(True)
+    try:
+        for i, t in enumerate(toks):
+            l = ctx().run_iter(plan, w, t, g, ws)
+            assert l == eager[i][0]
+            assert np.array_equal(g.cpu().numpy(), eager[i][1]), i
+    finally:
+        ctx().set_graphs(False)
