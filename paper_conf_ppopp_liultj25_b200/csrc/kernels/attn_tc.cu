@@ -66,7 +66,8 @@ __device__ __forceinline__ void st_half_row_sw128(uint8_t* tile, int row, int c0
   }
 }
 
-constexpr int kThreadsB = 320;   // backward: TMA, MMA, 8 softmax warps (2 per TMEM lane quarter)
+constexpr int kThreadsB = 320;
+constexpr int kRing = 4;   // depth of the streamed-operand TMA ring (K/V or Q/dO tiles)   // backward: TMA, MMA, 8 softmax warps (2 per TMEM lane quarter)
 
 template <int DH>
 struct Smem {
@@ -86,22 +87,23 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sK = smem;
   uint8_t* sV = sK + SM::kBig;
-  uint8_t* sQ[2] = {sV + SM::kBig, sV + SM::kBig + 2 * SM::kSmall};
-  uint8_t* sG[2] = {sQ[0] + SM::kSmall, sQ[1] + SM::kSmall};
-  uint8_t* sP = sV + SM::kBig + 4 * SM::kSmall;
+  uint8_t* sQ[kRing];
+  uint8_t* sG[kRing];
+  for (int r = 0; r < kRing; ++r) { sQ[r] = sV + SM::kBig + 2 * r * SM::kSmall; sG[r] = sQ[r] + SM::kSmall; }
+  uint8_t* sP = sV + SM::kBig + 2 * kRing * SM::kSmall;
   uint8_t* sS = sP + SM::kP;    // dS^T
   float* sL = reinterpret_cast<float*>(sS + SM::kP);       // [2][64] lse * log2e
   float* sDv = sL + 2 * kCols;                             // [2][64] D
   uint64_t* bar = reinterpret_cast<uint64_t*>(sDv + 2 * kCols);
-  uint64_t* kv_full = bar;          // 1
-  uint64_t* q_full = bar + 1;       // 2
-  uint64_t* q_empty = bar + 3;      // 2
-  uint64_t* s_full = bar + 5;       // 2
-  uint64_t* s_free = bar + 7;       // 2
-  uint64_t* p_full = bar + 9;       // 1
-  uint64_t* p_free = bar + 10;      // 1
-  uint64_t* acc_done = bar + 11;    // 1
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 12);
+  uint64_t* kv_full = bar;                 // 1
+  uint64_t* q_full = bar + 1;              // kRing
+  uint64_t* q_empty = q_full + kRing;      // kRing
+  uint64_t* s_full = q_empty + kRing;      // 2
+  uint64_t* s_free = s_full + 2;           // 2
+  uint64_t* p_full = s_free + 2;           // 1
+  uint64_t* p_free = p_full + 1;           // 1
+  uint64_t* acc_done = p_free + 1;         // 1
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_done + 1);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const int kt = blockIdx.x, b = blockIdx.y / nh, head = blockIdx.y % nh;
@@ -117,7 +119,8 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
     tma_prefetch_desc(&tm_qkv64);
     tma_prefetch_desc(&tm_do64);
     mbar_init(kv_full, 1);
-    for (int i = 0; i < 2; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); mbar_init(&s_full[i], 1); mbar_init(&s_free[i], 8); }
+    for (int i = 0; i < kRing; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); }
+    for (int i = 0; i < 2; ++i) { mbar_init(&s_full[i], 1); mbar_init(&s_free[i], 8); }
     mbar_init(p_full, 8);
     mbar_init(p_free, 1);
     mbar_init(acc_done, 1);
@@ -146,8 +149,8 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
         tma_load_2d(sV + a * (kRows * 128), &tm_qkv128, kv_full, 2 * h + head * DH + a * 64, row0 + kt * kRows);
       }
       for (int idx = 0; idx < ntiles; ++idx) {
-        const int st = idx & 1;
-        mbar_wait(&q_empty[st], ((idx >> 1) & 1) ^ 1);
+        const int st = idx % kRing;
+        mbar_wait(&q_empty[st], ((idx / kRing) & 1) ^ 1);
         mbar_arrive_expect_tx(&q_full[st], 2 * SM::kSmall);
         const int qr = row0 + (i0 + idx) * kCols;
 #pragma unroll
@@ -163,8 +166,8 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
     mbar_wait(kv_full, 0);
     tc_fence_after();
     auto issue_s = [&](int idx) {
-      const int st = idx & 1, buf = idx & 1;
-      mbar_wait(&q_full[st], (idx >> 1) & 1);
+      const int st = idx % kRing, buf = idx & 1;
+      mbar_wait(&q_full[st], (idx / kRing) & 1);
       mbar_wait(&s_free[buf], ((idx >> 1) & 1) ^ 1);
       tc_fence_after();
       if (elect_one()) {
@@ -180,7 +183,7 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
       __syncwarp();
     };
     auto issue_acc = [&](int idx) {
-      const int st = idx & 1;
+      const int st = idx % kRing;
       mbar_wait(p_full, idx & 1);
       tc_fence_after();
       if (elect_one()) {
@@ -295,19 +298,20 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sQ = smem;
   uint8_t* sG = sQ + SM::kBig;
-  uint8_t* sK[2] = {sG + SM::kBig, sG + SM::kBig + 2 * SM::kSmall};
-  uint8_t* sV[2] = {sK[0] + SM::kSmall, sK[1] + SM::kSmall};
-  uint8_t* sS = sG + SM::kBig + 4 * SM::kSmall;   // dS [128 q][64 keys]
+  uint8_t* sK[kRing];
+  uint8_t* sV[kRing];
+  for (int r = 0; r < kRing; ++r) { sK[r] = sG + SM::kBig + 2 * r * SM::kSmall; sV[r] = sK[r] + SM::kSmall; }
+  uint8_t* sS = sG + SM::kBig + 2 * kRing * SM::kSmall;   // dS [128 q][64 keys]
   uint64_t* bar = reinterpret_cast<uint64_t*>(sS + SM::kP);
-  uint64_t* q_fullb = bar;          // Q, dO loaded
-  uint64_t* k_full = bar + 1;       // 2
-  uint64_t* k_empty = bar + 3;      // 2
-  uint64_t* s_full = bar + 5;       // 2
-  uint64_t* s_free = bar + 7;       // 2
-  uint64_t* p_full = bar + 9;
-  uint64_t* p_free = bar + 10;
-  uint64_t* acc_done = bar + 11;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 12);
+  uint64_t* q_fullb = bar;                // Q, dO loaded
+  uint64_t* k_full = bar + 1;             // kRing
+  uint64_t* k_empty = k_full + kRing;     // kRing
+  uint64_t* s_full = k_empty + kRing;     // 2
+  uint64_t* s_free = s_full + 2;          // 2
+  uint64_t* p_full = s_free + 2;
+  uint64_t* p_free = p_full + 1;
+  uint64_t* acc_done = p_free + 1;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_done + 1);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const int qt = blockIdx.x, b = blockIdx.y / nh, head = blockIdx.y % nh;
@@ -322,7 +326,8 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
     tma_prefetch_desc(&tm_qkv64);
     tma_prefetch_desc(&tm_do128);
     mbar_init(q_fullb, 1);
-    for (int i = 0; i < 2; ++i) { mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1); mbar_init(&s_full[i], 1); mbar_init(&s_free[i], 8); }
+    for (int i = 0; i < kRing; ++i) { mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1); }
+    for (int i = 0; i < 2; ++i) { mbar_init(&s_full[i], 1); mbar_init(&s_free[i], 8); }
     mbar_init(p_full, 8);
     mbar_init(p_free, 1);
     mbar_init(acc_done, 1);
@@ -345,8 +350,8 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
         tma_load_2d(sG + a * (kRows * 128), &tm_do128, q_fullb, head * DH + a * 64, row0 + qt * kRows);
       }
       for (int idx = 0; idx < ntiles; ++idx) {
-        const int st = idx & 1;
-        mbar_wait(&k_empty[st], ((idx >> 1) & 1) ^ 1);
+        const int st = idx % kRing;
+        mbar_wait(&k_empty[st], ((idx / kRing) & 1) ^ 1);
         mbar_arrive_expect_tx(&k_full[st], 2 * SM::kSmall);
         const int kr = row0 + idx * kCols;
 #pragma unroll
@@ -362,8 +367,8 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
     mbar_wait(q_fullb, 0);
     tc_fence_after();
     auto issue_s = [&](int idx) {
-      const int st = idx & 1, buf = idx & 1;
-      mbar_wait(&k_full[st], (idx >> 1) & 1);
+      const int st = idx % kRing, buf = idx & 1;
+      mbar_wait(&k_full[st], (idx / kRing) & 1);
       mbar_wait(&s_free[buf], ((idx >> 1) & 1) ^ 1);
       tc_fence_after();
       if (elect_one()) {
@@ -379,7 +384,7 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
       __syncwarp();
     };
     auto issue_acc = [&](int idx) {
-      const int st = idx & 1;
+      const int st = idx % kRing;
       mbar_wait(p_full, idx & 1);
       tc_fence_after();
       if (elect_one()) {
@@ -465,9 +470,9 @@ done_dq:
 // >= 116 KB so that one CTA owns the SM (each allocates all 512 TMEM columns)
 constexpr int at_least_one_sm(int b) { return b < 116 * 1024 ? 116 * 1024 : b; }
 template <int DH>
-constexpr int smem_dkdv() { return at_least_one_sm(2 * Smem<DH>::kBig + 4 * Smem<DH>::kSmall + 2 * Smem<DH>::kP + 4 * kCols * 4 + 128 + 1024); }
+constexpr int smem_dkdv() { return at_least_one_sm(2 * Smem<DH>::kBig + 2 * kRing * Smem<DH>::kSmall + 2 * Smem<DH>::kP + 4 * kCols * 4 + 256 + 1024); }
 template <int DH>
-constexpr int smem_dq() { return at_least_one_sm(2 * Smem<DH>::kBig + 4 * Smem<DH>::kSmall + Smem<DH>::kP + 128 + 1024); }
+constexpr int smem_dq() { return at_least_one_sm(2 * Smem<DH>::kBig + 2 * kRing * Smem<DH>::kSmall + Smem<DH>::kP + 256 + 1024); }
 
 template <int DH>
 bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, bf16* dqkv, int B, int s, int nh,
@@ -510,20 +515,21 @@ fa_fwd_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sQ = smem;
-  uint8_t* sK[2] = {sQ + SM::kBig, sQ + SM::kBig + 2 * SM::kSmall};
-  uint8_t* sV[2] = {sK[0] + SM::kSmall, sK[1] + SM::kSmall};
-  uint8_t* sP[2] = {sQ + SM::kBig + 4 * SM::kSmall, sQ + SM::kBig + 4 * SM::kSmall + SM::kP};
+  uint8_t* sK[kRing];
+  uint8_t* sV[kRing];
+  for (int r = 0; r < kRing; ++r) { sK[r] = sQ + SM::kBig + 2 * r * SM::kSmall; sV[r] = sK[r] + SM::kSmall; }
+  uint8_t* sP[2] = {sQ + SM::kBig + 2 * kRing * SM::kSmall, sQ + SM::kBig + 2 * kRing * SM::kSmall + SM::kP};
   float* xch = reinterpret_cast<float*>(sP[1] + SM::kP);   // [2 halves][128 rows] max / sum exchange
   uint64_t* bar = reinterpret_cast<uint64_t*>(xch + 2 * kRows);
-  uint64_t* q_fullb = bar;          // 1
-  uint64_t* k_full = bar + 1;       // 2
-  uint64_t* k_empty = bar + 3;      // 2
-  uint64_t* s_full = bar + 5;       // 2
-  uint64_t* s_free = bar + 7;       // 2
-  uint64_t* p_full = bar + 9;       // 2
-  uint64_t* o_full = bar + 11;      // 2  (PV_j done: also frees P_j smem)
-  uint64_t* o_free = bar + 13;      // 2  (softmax read PV_j out of TMEM)
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bar + 15);
+  uint64_t* q_fullb = bar;                // 1
+  uint64_t* k_full = bar + 1;             // kRing
+  uint64_t* k_empty = k_full + kRing;     // kRing
+  uint64_t* s_full = k_empty + kRing;     // 2
+  uint64_t* s_free = s_full + 2;          // 2
+  uint64_t* p_full = s_free + 2;          // 2
+  uint64_t* o_full = p_full + 2;          // 2  (PV_j done: also frees P_j smem)
+  uint64_t* o_free = o_full + 2;          // 2  (softmax read PV_j out of TMEM)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(o_free + 2);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const int qt = blockIdx.x, b = blockIdx.y / nh, head = blockIdx.y % nh;
@@ -537,8 +543,9 @@ fa_fwd_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__
     tma_prefetch_desc(&tm_qkv128);
     tma_prefetch_desc(&tm_qkv64);
     mbar_init(q_fullb, 1);
+    for (int i = 0; i < kRing; ++i) { mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1); }
     for (int i = 0; i < 2; ++i) {
-      mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1); mbar_init(&s_full[i], 1); mbar_init(&s_free[i], 8);
+      mbar_init(&s_full[i], 1); mbar_init(&s_free[i], 8);
       mbar_init(&p_full[i], 8); mbar_init(&o_full[i], 1); mbar_init(&o_free[i], 8);
     }
     fence_barrier_init();
@@ -558,8 +565,8 @@ fa_fwd_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__
       for (int a = 0; a < DH / 64; ++a)
         tma_load_2d(sQ + a * (kRows * 128), &tm_qkv128, q_fullb, head * DH + a * 64, row0 + qt * kRows);
       for (int j = 0; j < ntiles; ++j) {
-        const int st = j & 1;
-        mbar_wait(&k_empty[st], ((j >> 1) & 1) ^ 1);
+        const int st = j % kRing;
+        mbar_wait(&k_empty[st], ((j / kRing) & 1) ^ 1);
         mbar_arrive_expect_tx(&k_full[st], 2 * SM::kSmall);
 #pragma unroll
         for (int a = 0; a < DH / 64; ++a) {
@@ -574,33 +581,33 @@ fa_fwd_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__
     mbar_wait(q_fullb, 0);
     tc_fence_after();
     auto issue_s = [&](int j) {
-      const int st = j & 1;
-      mbar_wait(&k_full[st], (j >> 1) & 1);
-      mbar_wait(&s_free[st], ((j >> 1) & 1) ^ 1);
+      const int st = j % kRing, b2 = j & 1;
+      mbar_wait(&k_full[st], (j / kRing) & 1);
+      mbar_wait(&s_free[b2], ((j >> 1) & 1) ^ 1);
       tc_fence_after();
       if (elect_one()) {
         const uint32_t q = smem_u32(sQ), k = smem_u32(sK[st]);
 #pragma unroll
         for (int kk = 0; kk < DH / 16; ++kk) {
           const uint32_t ao = (kk >> 2) * (kRows * 128) + (kk & 3) * 32, bo = (kk >> 2) * (kCols * 128) + (kk & 3) * 32;
-          umma_bf16(tm_S + st * kCols, umma_desc_sw128(q + ao, 16, 1024), umma_desc_sw128(k + bo, 16, 1024), id_s, kk > 0);
+          umma_bf16(tm_S + b2 * kCols, umma_desc_sw128(q + ao, 16, 1024), umma_desc_sw128(k + bo, 16, 1024), id_s, kk > 0);
         }
-        umma_commit(&s_full[st]);
+        umma_commit(&s_full[b2]);
       }
       __syncwarp();
     };
     auto issue_pv = [&](int j) {
-      const int st = j & 1;
-      mbar_wait(&p_full[st], (j >> 1) & 1);
-      mbar_wait(&o_free[st], ((j >> 1) & 1) ^ 1);
+      const int st = j % kRing, b2 = j & 1;
+      mbar_wait(&p_full[b2], (j >> 1) & 1);
+      mbar_wait(&o_free[b2], ((j >> 1) & 1) ^ 1);
       tc_fence_after();
       if (elect_one()) {
-        const uint32_t p = smem_u32(sP[st]), v = smem_u32(sV[st]);
+        const uint32_t p = smem_u32(sP[b2]), v = smem_u32(sV[st]);
 #pragma unroll
         for (int kk = 0; kk < kCols / 16; ++kk)
-          umma_bf16(tm_O + st * DH, umma_desc_sw128(p + kk * 32, 16, 1024),
+          umma_bf16(tm_O + b2 * DH, umma_desc_sw128(p + kk * 32, 16, 1024),
                     umma_desc_sw128(v + kk * 2048, kCols * 128, 1024), id_o, kk > 0);
-        umma_commit(&o_full[st]);
+        umma_commit(&o_full[b2]);
         umma_commit(&k_empty[st]);
       }
       __syncwarp();
@@ -708,7 +715,7 @@ fa_fwd_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__
 }
 
 template <int DH>
-constexpr int smem_fwd() { return at_least_one_sm(Smem<DH>::kBig + 4 * Smem<DH>::kSmall + 2 * Smem<DH>::kP + 2 * kRows * 4 + 128 + 1024); }
+constexpr int smem_fwd() { return at_least_one_sm(Smem<DH>::kBig + 2 * kRing * Smem<DH>::kSmall + 2 * Smem<DH>::kP + 2 * kRows * 4 + 256 + 1024); }
 
 template <int DH>
 bool launch_fwd_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, cudaStream_t st) {
