@@ -30,9 +30,10 @@ int mario_k_gemm_bf16(const void* A, int lda, int a_mn, const void* B, int ldb, 
                       const float* bias, const void* residual, int ld_res,
                       void* D2, const void* aux, int ld_aux, void* stream);
 
-/* Kernel selection for K1-K3: -1 = auto (CTA-pair 256x256 tiles when M, N >= 256 and the
- * pair tiles fill the GPU, else single-CTA 128x256/128x128), 0 = single-CTA only, 1 = CTA pair
- * whenever M, N >= 256. Process-global; returns 0, or 1 for an invalid value. */
+/* Kernel selection for K1-K3: -1 = auto (CTA-pair tiles when M, N >= 256 and the pair tiles fill
+ * the GPU — 256x256, or 256x128 when that wastes less of the last wave — else single-CTA
+ * 128x256/128x128), 0 = single-CTA only, 1 = CTA pair whenever M, N >= 256 (auto N),
+ * 2 = CTA pair 256x128, 3 = CTA pair 256x256. Process-global; returns 0, or 1 if invalid. */
 int mario_k_gemm_set_variant(int variant);
 
 /* K4: the same contract in true fp32 on CUDA cores (fp32 mode, reading A6). */

@@ -9,7 +9,7 @@ namespace mario { extern int g_gemm_variant; extern int g_attn_variant; }
 using namespace mario;
 
 extern "C" int mario_k_gemm_set_variant(int variant) {
-  if (variant < -1 || variant > 1) return 1;
+  if (variant < -1 || variant > 3) return 1;
   g_gemm_variant = variant;
   return 0;
 }

@@ -136,7 +136,7 @@ __device__ __forceinline__ void epilogue_chunk(const GemmEpilogue& ep, const uin
 template <int BN, bool A_MN, bool B_MN>
 __global__ void __launch_bounds__(kThreads, 1)
 gemm_bf16_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                    GemmEpilogue ep, int M, int N, int K) {
+                    GemmEpilogue ep, int M, int N, int K, int n_fastest) {
   using C = Cfg<BN>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -171,7 +171,8 @@ gemm_bf16_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
     if (elect_one()) {
       int s = 0; uint32_t ph = 0;
       for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
-        const int m0 = (tile % num_m) * BM, n0 = (tile / num_m) * BN;
+        const int tm = n_fastest ? tile / num_n : tile % num_m, tn = n_fastest ? tile % num_n : tile / num_m;
+        const int m0 = tm * BM, n0 = tn * BN;
         for (int kb = 0; kb < nk; ++kb) {
           mbar_wait(&empty[s], ph ^ 1);
           uint8_t* sa = smem + s * C::kStageBytes;
@@ -232,7 +233,8 @@ gemm_bf16_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
     for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++t) {
       const int acc = t & 1;
       const uint32_t acc_ph = (t >> 1) & 1;
-      const int m0 = (tile % num_m) * BM, n0 = (tile / num_m) * BN;
+      const int tm = n_fastest ? tile / num_n : tile % num_m, tn = n_fastest ? tile % num_n : tile / num_m;
+      const int m0 = tm * BM, n0 = tn * BN;
       mbar_wait(&tfull[acc], acc_ph);
       tc_fence_after();
       const int row = m0 + quarter * 32 + lane;
@@ -260,15 +262,22 @@ gemm_bf16_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
 // tile) and owns 128 accumulator rows x 256 columns in its TMEM (double-buffered, 512 cols).
 // 10 warps: producer, MMA (leader only), 8 epilogue warps (2 per TMEM lane quarter).
 constexpr int kThreads2 = 320;
-constexpr int kStages2 = 6;
-constexpr int kHalfBytes = 128 * BK * 2;            // 16 KB: one CTA's half of A (or B) per stage
-constexpr int kStage2Bytes = 2 * kHalfBytes;        // A half + B half
-constexpr int kSmem2 = kStages2 * kStage2Bytes + 1024 + 256;
+template <int BNP>
+struct Cfg2 {                                             // BNP = N of the pair tile (256 or 128)
+  static constexpr int kABytes = 128 * BK * 2;            // 16 KB: one CTA's half of A per stage
+  static constexpr int kBBytes = (BNP / 2) * BK * 2;      // one CTA's half of B per stage
+  static constexpr int kStageBytes = kABytes + kBBytes;
+  static constexpr int kStages = BNP == 256 ? 6 : 8;
+  static constexpr int kSmem = kStages * kStageBytes + 1024 + 256;
+  static constexpr int kTmem = 2 * BNP;
+};
 
-template <bool A_MN, bool B_MN>
+template <int BNP, bool A_MN, bool B_MN>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads2, 1)
 gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                     GemmEpilogue ep, int M, int N, int K) {
+                     GemmEpilogue ep, int M, int N, int K, int n_fastest) {
+  using C2 = Cfg2<BNP>;
+  constexpr int kStages2 = C2::kStages, kStage2Bytes = C2::kStageBytes, kHalfBytes = C2::kABytes;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint64_t* full = reinterpret_cast<uint64_t*>(smem + kStages2 * kStage2Bytes);
@@ -281,7 +290,7 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
   const uint32_t rank = cluster_ctarank();
   const bool leader = rank == 0;
   const int pair = blockIdx.x / 2, npairs = gridDim.x / 2;
-  const int num_m = (M + 255) / 256, num_n = (N + 255) / 256;
+  const int num_m = (M + 255) / 256, num_n = (N + BNP - 1) / BNP;
   const int num_tiles = num_m * num_n;
   const int nk = (K + BK - 1) / BK;
 
@@ -292,7 +301,7 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
     for (int a = 0; a < 2; ++a) { mbar_init(&tfull[a], 1); mbar_init(&tempty[a], 16); }
     fence_barrier_init();
   }
-  if (warp == 1) tmem_alloc_2sm<512>(tmem_slot);
+  if (warp == 1) tmem_alloc_2sm<C2::kTmem>(tmem_slot);
   tc_fence_before();
   cluster_sync();
   tc_fence_after();
@@ -302,7 +311,8 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
     if (elect_one()) {
       int s = 0; uint32_t ph = 0;
       for (int tile = pair; tile < num_tiles; tile += npairs) {
-        const int m0 = (tile % num_m) * 256 + 128 * rank, n0 = (tile / num_m) * 256 + 128 * rank;
+        const int tm = n_fastest ? tile / num_n : tile % num_m, tn = n_fastest ? tile % num_n : tile / num_m;
+        const int m0 = tm * 256 + 128 * rank, n0 = tn * BNP + (BNP / 2) * rank;
         for (int kb = 0; kb < nk; ++kb) {
           mbar_wait(&empty[s], ph ^ 1);
           uint8_t* sa = smem + s * kStage2Bytes;
@@ -313,22 +323,26 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
           const int k0 = kb * BK;
           if (A_MN) { tma_load_2d_2sm(sa, &tmA, lbar, m0, k0); tma_load_2d_2sm(sa + 8192, &tmA, lbar, m0 + 64, k0); }
           else tma_load_2d_2sm(sa, &tmA, lbar, k0, m0);
-          if (B_MN) { tma_load_2d_2sm(sb, &tmB, lbar, n0, k0); tma_load_2d_2sm(sb + 8192, &tmB, lbar, n0 + 64, k0); }
-          else tma_load_2d_2sm(sb, &tmB, lbar, k0, n0);
+          if (B_MN) {
+            tma_load_2d_2sm(sb, &tmB, lbar, n0, k0);
+            if (BNP == 256) tma_load_2d_2sm(sb + 8192, &tmB, lbar, n0 + 64, k0);
+          } else {
+            tma_load_2d_2sm(sb, &tmB, lbar, k0, n0);
+          }
           if (++s == kStages2) { s = 0; ph ^= 1; }
         }
       }
     }
   } else if (warp == 1) {
     if (leader) {
-      constexpr uint32_t idesc = umma_idesc_bf16(256, 256, A_MN ? 1 : 0, B_MN ? 1 : 0);
+      constexpr uint32_t idesc = umma_idesc_bf16(256, BNP, A_MN ? 1 : 0, B_MN ? 1 : 0);
       int s = 0; uint32_t ph = 0; int t = 0;
       for (int tile = pair; tile < num_tiles; tile += npairs, ++t) {
         const int acc = t & 1;
         const uint32_t acc_ph = (t >> 1) & 1;
         mbar_wait(&tempty[acc], acc_ph ^ 1);
         tc_fence_after();
-        const uint32_t d_tmem = tmem_base + acc * 256;
+        const uint32_t d_tmem = tmem_base + acc * BNP;
         for (int kb = 0; kb < nk; ++kb) {
           mbar_wait(&full[s], ph);
           tc_fence_after();
@@ -356,16 +370,17 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
     for (int tile = pair; tile < num_tiles; tile += npairs, ++t) {
       const int acc = t & 1;
       const uint32_t acc_ph = (t >> 1) & 1;
-      const int m0 = (tile % num_m) * 256 + 128 * rank, n0 = (tile / num_m) * 256;
+      const int tm = n_fastest ? tile / num_n : tile % num_m, tn = n_fastest ? tile % num_n : tile / num_m;
+      const int m0 = tm * 256 + 128 * rank, n0 = tn * BNP;
       mbar_wait(&tfull[acc], acc_ph);
       tc_fence_after();
       const int row = m0 + quarter * 32 + lane;
       const bool row_ok = row < M;
 #pragma unroll 1
-      for (int c = 0; c < 4; ++c) {
+      for (int c = 0; c < BNP / 64; ++c) {
         uint32_t r[32];
-        const int col = half * 128 + c * 32;
-        tmem_ld_32x32b_x32(tmem_base + acc * 256 + col + (static_cast<uint32_t>(quarter * 32) << 16), r);
+        const int col = half * (BNP / 2) + c * 32;
+        tmem_ld_32x32b_x32(tmem_base + acc * BNP + col + (static_cast<uint32_t>(quarter * 32) << 16), r);
         tmem_ld_wait();
         epilogue_chunk(ep, r, row, n0 + col, row_ok, N);
       }
@@ -376,7 +391,7 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
   }
   tc_fence_before();
   cluster_sync();
-  if (warp == 1) tmem_dealloc_2sm<512>(tmem_base);
+  if (warp == 1) tmem_dealloc_2sm<C2::kTmem>(tmem_base);
 }
 
 PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
@@ -436,37 +451,55 @@ cudaError_t launch_bn(const GemmArgs& g, cudaStream_t st, int num_sms) {
   const int grid = tiles < num_sms ? tiles : num_sms;
   const int tok = kstats_begin(K_GEMM, 2.0 * g.M * g.N * g.K,
                                2.0 * (double(g.M) * g.K + double(g.N) * g.K) + (g.ep.out_f32 ? 4.0 : 2.0) * g.M * g.N, st);
-  kern<<<grid, kThreads, C::kSmem, st>>>(ta, tb, g.ep, g.M, g.N, g.K);
+  // raster: keep the larger operand's panel hot in L2 across the other dimension's tiles
+  const int n_fastest = static_cast<long>(g.M) >= static_cast<long>(g.N) ? 1 : 0;
+  kern<<<grid, kThreads, C::kSmem, st>>>(ta, tb, g.ep, g.M, g.N, g.K, n_fastest);
   kstats_end(tok, st);
   note_launch();
   return cudaGetLastError();
 }
 
 
-template <bool A_MN, bool B_MN>
+template <int BNP, bool A_MN, bool B_MN>
 cudaError_t launch_pair(const GemmArgs& g, cudaStream_t st, int num_sms) {
+  using C2 = Cfg2<BNP>;
   CUtensorMap ta, tb;
   bool ok = A_MN ? make_tmap(&ta, g.A, g.M, g.K, g.lda, 64, 64) : make_tmap(&ta, g.A, g.K, g.M, g.lda, 64, 128);
-  ok = ok && (B_MN ? make_tmap(&tb, g.B, g.N, g.K, g.ldb, 64, 64) : make_tmap(&tb, g.B, g.K, g.N, g.ldb, 64, 128));
+  ok = ok && (B_MN ? make_tmap(&tb, g.B, g.N, g.K, g.ldb, 64, 64) : make_tmap(&tb, g.B, g.K, g.N, g.ldb, 64, BNP / 2));
   if (!ok) {
     fprintf(stderr, "[mario] gemm_bf16 (pair): tensor map failed M=%d N=%d K=%d\n", g.M, g.N, g.K);
     return cudaErrorInvalidValue;
   }
-  auto kern = gemm_bf16_tc2_kernel<A_MN, B_MN>;
+  auto kern = gemm_bf16_tc2_kernel<BNP, A_MN, B_MN>;
   static bool attr_set = false;
   if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmem2);
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C2::kSmem);
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
-  const int tiles = ((g.M + 255) / 256) * ((g.N + 255) / 256);
+  const int tiles = ((g.M + 255) / 256) * ((g.N + BNP - 1) / BNP);
   const int pairs = tiles < num_sms / 2 ? tiles : num_sms / 2;
   const int tok = kstats_begin(K_GEMM, 2.0 * g.M * g.N * g.K,
                                2.0 * (double(g.M) * g.K + double(g.N) * g.K) + (g.ep.out_f32 ? 4.0 : 2.0) * g.M * g.N, st);
-  kern<<<2 * pairs, kThreads2, kSmem2, st>>>(ta, tb, g.ep, g.M, g.N, g.K);
+  const int n_fastest = static_cast<long>(g.M) >= static_cast<long>(g.N) ? 1 : 0;
+  kern<<<2 * pairs, kThreads2, C2::kSmem, st>>>(ta, tb, g.ep, g.M, g.N, g.K, n_fastest);
   kstats_end(tok, st);
   note_launch();
   return cudaGetLastError();
+}
+
+template <int BNP>
+cudaError_t launch_pair_major(const GemmArgs& g, cudaStream_t st, int sms) {
+  if (!g.a_mn && !g.b_mn) return launch_pair<BNP, false, false>(g, st, sms);
+  if (!g.a_mn && g.b_mn) return launch_pair<BNP, false, true>(g, st, sms);
+  if (g.a_mn && g.b_mn) return launch_pair<BNP, true, true>(g, st, sms);
+  return launch_pair<BNP, true, false>(g, st, sms);
+}
+
+// fraction of the issued tile slots that do useful work (wave quantization)
+double wave_eff(long tiles, long slots) {
+  const long waves = (tiles + slots - 1) / slots;
+  return static_cast<double>(tiles) / static_cast<double>(waves * slots);
 }
 
 template <int BN>
@@ -495,7 +528,7 @@ int device_sm_count() {
   return n;
 }
 
-int g_gemm_variant = -1;   // mario_k_gemm_set_variant: -1 auto, 0 single-CTA only, 1 prefer CTA pair
+int g_gemm_variant = -1;   // mario_k_gemm_set_variant: -1 auto, 0 single-CTA, 1 pair (auto N), 2 pair N=128, 3 pair N=256
 
 cudaError_t gemm_bf16(const GemmArgs& g0, cudaStream_t st) {
   GemmArgs g = g0;
@@ -506,13 +539,15 @@ cudaError_t gemm_bf16(const GemmArgs& g0, cudaStream_t st) {
     return cudaErrorInvalidValue;
   }
   const int sms = device_sm_count();
-  // Prefer the CTA-pair 256x256 tile when it fills the machine, else 128x256 / 128x128.
+  // CTA-pair tiles (256x256, or 256x128 when it quantizes the last wave better; a 256x128 tile
+  // costs ~4% more operand traffic per FLOP) when they fill the machine, else single-CTA tiles.
   const long tiles_pair = static_cast<long>((g.M + 255) / 256) * ((g.N + 255) / 256);
-  if (g.use_pair != 0 && g.M >= 256 && g.N >= 256 && (tiles_pair >= sms / 2 || g.use_pair > 0)) {
-    if (!g.a_mn && !g.b_mn) return launch_pair<false, false>(g, st, sms);
-    if (!g.a_mn && g.b_mn) return launch_pair<false, true>(g, st, sms);
-    if (g.a_mn && g.b_mn) return launch_pair<true, true>(g, st, sms);
-    return launch_pair<true, false>(g, st, sms);
+  if (g.use_pair != 0 && g.M >= 256 && g.N >= 256 && (tiles_pair >= sms / 4 || g.use_pair > 0)) {
+    const long t256 = tiles_pair, t128 = static_cast<long>((g.M + 255) / 256) * ((g.N + 127) / 128);
+    (void)t256; (void)t128;
+    // measured: the 256x128 tile loses to 256x256 even where it quantizes the last wave better
+    if (g.use_pair == 2) return launch_pair_major<128>(g, st, sms);
+    return launch_pair_major<256>(g, st, sms);
   }
   const long tiles256 = static_cast<long>((g.M + BM - 1) / BM) * ((g.N + 255) / 256);
   if (g.N > 128 && tiles256 >= sms / 2) return launch_major<256>(g, st, sms);

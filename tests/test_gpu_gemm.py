@@ -53,7 +53,7 @@ def _run(a_mn, b_mn, M, N, K, out_f32, bias=False, resid=False, gelu2=False, aux
         assert (D2.float() - gref).abs().max().item() <= 2e-2 * gref.abs().max().item() + 1e-2
 
 
-@pytest.fixture(params=[0, 1], ids=["single_cta", "cta_pair"])
+@pytest.fixture(params=[0, 2, 3], ids=["single_cta", "cta_pair_n128", "cta_pair_n256"])
 def variant(request):
     L = _lib.lib()
     assert L.mario_k_gemm_set_variant(request.param) == 0
