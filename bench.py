@@ -277,7 +277,8 @@ def main():
     clk = clocks.stop()
     kst = {}
     import ctypes as C
-    for kind, name in ((0, "gemm"), (1, "attn_fwd"), (2, "attn_bwd")):
+    for kind, name in ((0, "gemm"), (1, "attn_fwd"), (2, "attn_bwd"), (4, "norm"), (5, "colsum"), (6, "softmax_ce"),
+                       (7, "elementwise"), (8, "embedding")):
         ms, fl, by, n = C.c_double(), C.c_double(), C.c_double(), C.c_longlong()
         L.mario_kstats_read(kind, C.byref(ms), C.byref(fl), C.byref(by), C.byref(n))
         kst[name] = {"ms": ms.value, "flops": fl.value, "bytes": by.value, "launches": n.value}

@@ -57,6 +57,17 @@ int mario_k_attn_set_variant(int variant);
 int mario_k_attn_bwd(const void* qkv, const void* O, const void* dO, const float* lse, void* dqkv,
                      float* scratch, int B, int s, int n_heads, int head_dim, int bf16, void* stream);
 
+/* K7/K8: LayerNorm (rms = 0: y = (x - mean)/sqrt(var + eps) * g + b) or RMSNorm (rms = 1:
+ * y = x / sqrt(mean(x^2) + eps) * g) over rows of width n; stats =
+ * fp32 [rows][2] (mean, rstd; mean = 0 for RMS). x, y: [rows][n] bf16 (bf16 = 1) or fp32. */
+int mario_k_norm_fwd(const void* x, const float* g, const float* b, void* y, float* stats, int rows, int n,
+                     float eps, int rms, int bf16, void* stream);
+/* Backward: dx = norm'(dy) (+ dres if non-NULL); if dg != NULL also dg (+ db for LN) += column sums
+ * (deterministic two-pass; partial: fp32 scratch >= 2 * 128 * n). */
+int mario_k_norm_bwd(const void* dy, const void* x, const float* stats, const float* g, const void* dres,
+                     void* dx, float* dg, float* db, float* partial, int rows, int n, int rms, int bf16,
+                     void* stream);
+
 /* Instrumentation. mario_kernel_launches: number of kernels this library has launched since it
  * was loaded (every call above and every mario_run_iter kernel). mario_kstats_enable(1) clears
  * and starts CUDA-event timing of every GEMM (kind 0), attention forward (1) and backward (2)

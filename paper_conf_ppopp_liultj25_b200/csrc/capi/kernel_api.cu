@@ -67,3 +67,35 @@ extern "C" int mario_k_attn_bwd(const void* qkv, const void* O, const void* dO, 
                        static_cast<float*>(dqkv), scratch, B, s, n_heads, head_dim, st);
   return static_cast<int>(cudaGetLastError());
 }
+
+extern "C" int mario_k_norm_fwd(const void* x, const float* g, const float* b, void* y, float* stats, int rows, int n,
+                                float eps, int rms, int bf16, void* stream) {
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (bf16) {
+    if (rms) rmsnorm_fwd<__nv_bfloat16>(static_cast<const __nv_bfloat16*>(x), g, static_cast<__nv_bfloat16*>(y), stats, rows, n, eps, st);
+    else layernorm_fwd<__nv_bfloat16>(static_cast<const __nv_bfloat16*>(x), g, b, static_cast<__nv_bfloat16*>(y), stats, rows, n, eps, st);
+  } else {
+    if (rms) rmsnorm_fwd<float>(static_cast<const float*>(x), g, static_cast<float*>(y), stats, rows, n, eps, st);
+    else layernorm_fwd<float>(static_cast<const float*>(x), g, b, static_cast<float*>(y), stats, rows, n, eps, st);
+  }
+  return static_cast<int>(cudaGetLastError());
+}
+
+extern "C" int mario_k_norm_bwd(const void* dy, const void* x, const float* stats, const float* g, const void* dres,
+                                void* dx, float* dg, float* db, float* partial, int rows, int n, int rms, int bf16,
+                                void* stream) {
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (bf16) {
+    auto* X = static_cast<const __nv_bfloat16*>(x);
+    auto* DY = static_cast<const __nv_bfloat16*>(dy);
+    norm_bwd_dx<__nv_bfloat16>(DY, X, stats, g, static_cast<const __nv_bfloat16*>(dres), static_cast<__nv_bfloat16*>(dx),
+                               rows, n, rms, st);
+    if (dg) colsum<__nv_bfloat16>(DY, X, stats, rows, n, n, rms ? 2 : 1, dg, db, partial, st);
+  } else {
+    auto* X = static_cast<const float*>(x);
+    auto* DY = static_cast<const float*>(dy);
+    norm_bwd_dx<float>(DY, X, stats, g, static_cast<const float*>(dres), static_cast<float*>(dx), rows, n, rms, st);
+    if (dg) colsum<float>(DY, X, stats, rows, n, n, rms ? 2 : 1, dg, db, partial, st);
+  }
+  return static_cast<int>(cudaGetLastError());
+}

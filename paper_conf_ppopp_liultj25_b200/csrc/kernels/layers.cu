@@ -754,6 +754,7 @@ int grid_for(long n, int threads = 256) { long g = (n + threads - 1) / threads; 
 
 template <class T>
 void embed_fwd(const int32_t* tok, int ld_tok, int B, int s, const T* wte, const T* wpe, T* H, int h, cudaStream_t st) {
+  KScope ks_(K_EMBED, st);
   embed_fwd_k<T><<<grid_for(static_cast<long>(B) * s * h), 256, 0, st>>>(tok, ld_tok, B, s, wte, wpe, H, h);
   note_launch();
 }
@@ -761,6 +762,7 @@ void embed_fwd(const int32_t* tok, int ld_tok, int B, int s, const T* wte, const
 template <class T>
 void embed_bwd(const int32_t* tok, int ld_tok, int B, int s, const T* dH, int h, float* dwte, float* dwpe,
                void* scratch, cudaStream_t st) {
+  KScope ks_(K_EMBED, st);
   const int Ttok = B * s;
   int np2 = 1;
   while (np2 < Ttok) np2 <<= 1;
@@ -777,6 +779,7 @@ void embed_bwd(const int32_t* tok, int ld_tok, int B, int s, const T* dH, int h,
 
 template <class T>
 void layernorm_fwd(const T* x, const float* g, const float* b, T* y, float* stats, int rows, int n, float eps, cudaStream_t st) {
+  KScope ks_(K_NORM, st);
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
     if (n % 8 == 0) {
       if (n <= 1024) norm_fwd_reg_k<false, 4><<<cdiv(rows, 8), 256, 0, st>>>(x, g, b, y, stats, rows, n, eps);
@@ -793,6 +796,7 @@ void layernorm_fwd(const T* x, const float* g, const float* b, T* y, float* stat
 }
 template <class T>
 void rmsnorm_fwd(const T* x, const float* g, T* y, float* stats, int rows, int n, float eps, cudaStream_t st) {
+  KScope ks_(K_NORM, st);
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
     if (n % 8 == 0) {
       if (n <= 1024) norm_fwd_reg_k<true, 4><<<cdiv(rows, 8), 256, 0, st>>>(x, g, nullptr, y, stats, rows, n, eps);
@@ -810,6 +814,7 @@ void rmsnorm_fwd(const T* x, const float* g, T* y, float* stats, int rows, int n
 template <class T>
 void norm_bwd_dx(const T* dy, const T* x, const float* stats, const float* g, const T* dres, T* dx, int rows, int n,
                  int rms, cudaStream_t st) {
+  KScope ks_(K_NORM, st);
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
     if (n % 8 == 0) {
       if (n <= 1024) norm_bwd_dx_reg_k<4><<<cdiv(rows, 8), 256, 0, st>>>(dy, x, stats, g, dres, dx, rows, n, rms);
@@ -825,6 +830,7 @@ void norm_bwd_dx(const T* dy, const T* x, const float* stats, const float* g, co
 template <class T>
 void colsum(const T* a, const T* x, const float* stats, int rows, int n, int lda, int mode, float* out0, float* out1,
             float* partial, cudaStream_t st) {
+  KScope ks_(K_COLSUM, st);
   int nblk = rows < 128 ? rows : 128;
   if (nblk < 1) return;
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
@@ -872,35 +878,42 @@ void attn_bwd(const T* qkv, const T* O, const T* dO, const float* lse, T* dqkv, 
 
 template <class T>
 void rope(T* qkv, int B, int s, int nh, int dh, float base, int inverse, cudaStream_t st) {
+  KScope ks_(K_ELEMWISE, st);
   rope_k<T><<<grid_for(static_cast<long>(B) * s * nh * (dh / 2)), 256, 0, st>>>(qkv, B, s, nh, dh, base, inverse);
   note_launch();
 }
 template <class T>
 void swiglu_fwd(const T* GU, T* M, int rows, int f, cudaStream_t st) {
+  KScope ks_(K_ELEMWISE, st);
   swiglu_fwd_k<T><<<grid_for(static_cast<long>(rows) * f), 256, 0, st>>>(GU, M, rows, f);
   note_launch();
 }
 template <class T>
 void swiglu_bwd(const T* GU, const T* dM, T* dGU, int rows, int f, cudaStream_t st) {
+  KScope ks_(K_ELEMWISE, st);
   swiglu_bwd_k<T><<<grid_for(static_cast<long>(rows) * f), 256, 0, st>>>(GU, dM, dGU, rows, f);
   note_launch();
 }
 template <class T>
 void softmax_ce(const float* logits, const int32_t* tok, int ld_tok, int s, int rows, int V, float inv_ntok,
                 T* dlogits, float* row_loss, cudaStream_t st) {
+  KScope ks_(K_CE, st);
   softmax_ce_k<T><<<rows, 512, 0, st>>>(logits, tok, ld_tok, s, V, inv_ntok, dlogits, row_loss);
   note_launch();
 }
 template <class T>
 void gelu_fwd(const T* Z, T* G, size_t n, cudaStream_t st) {
+  KScope ks_(K_ELEMWISE, st);
   gelu_fwd_k<T><<<grid_for(static_cast<long>(n)), 256, 0, st>>>(Z, G, n);
   note_launch();
 }
 void loss_reduce(const float* row_loss, int rows, double* out, cudaStream_t st) {
+  KScope ks_(K_CE, st);
   loss_reduce_k<<<1, 1024, 0, st>>>(row_loss, rows, out);
   note_launch();
 }
 void cast_f32_bf16(const float* x, __nv_bfloat16* y, size_t n, cudaStream_t st) {
+  KScope ks_(K_ELEMWISE, st);
   cast_k<<<grid_for(static_cast<long>(n)), 256, 0, st>>>(x, y, n);
   note_launch();
 }
