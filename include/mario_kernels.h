@@ -62,11 +62,17 @@ int mario_k_attn_bwd(const void* qkv, const void* O, const void* dO, const float
  * fp32 [rows][2] (mean, rstd; mean = 0 for RMS). x, y: [rows][n] bf16 (bf16 = 1) or fp32. */
 int mario_k_norm_fwd(const void* x, const float* g, const float* b, void* y, float* stats, int rows, int n,
                      float eps, int rms, int bf16, void* stream);
-/* Backward: dx = norm'(dy) (+ dres if non-NULL); if dg != NULL also dg (+ db for LN) += column sums
- * (deterministic two-pass; partial: fp32 scratch >= 2 * 128 * n). */
+/* Backward (A1/A2 derivative): dx = norm'(dy) (+ dres if non-NULL). If dg != NULL, also, fused:
+ * dg += sum_rows dy * xhat, db += sum_rows dy (LN; ignored for RMS) and, if dsum != NULL,
+ * dsum += sum_rows dx (column sums of the written dx: the bias gradient of the producing linear).
+ * partial: fp32 device scratch of partial_floats (>= 3 * n * 148 * 4 uses the fused kernel; the
+ * column sums are deterministic: fixed-order two-pass). Returns a cudaError_t value. */
 int mario_k_norm_bwd(const void* dy, const void* x, const float* stats, const float* g, const void* dres,
-                     void* dx, float* dg, float* db, float* partial, int rows, int n, int rms, int bf16,
-                     void* stream);
+                     void* dx, float* dg, float* db, float* dsum, float* partial, long long partial_floats,
+                     int rows, int n, int rms, int bf16, void* stream);
+/* 1: block-per-row-tile backward with fused column sums (default); 0: warp-per-row backward +
+ * separate column-sum passes. (The forward always uses the warp-per-row kernels.) */
+int mario_k_norm_set_variant(int v);
 
 /* Instrumentation. mario_kernel_launches: number of kernels this library has launched since it
  * was loaded (every call above and every mario_run_iter kernel). mario_kstats_enable(1) clears

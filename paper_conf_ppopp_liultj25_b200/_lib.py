@@ -22,7 +22,8 @@ _SIGS = {
     "mario_k_attn_fwd": (i32, [vp, vp, vp, i32, i32, i32, i32, i32, vp]),
     "mario_k_attn_bwd": (i32, [vp, vp, vp, vp, vp, vp, i32, i32, i32, i32, i32, vp]),
     "mario_k_norm_fwd": (i32, [vp, vp, vp, vp, vp, i32, i32, f32, i32, i32, vp]),
-    "mario_k_norm_bwd": (i32, [vp, vp, vp, vp, vp, vp, vp, vp, vp, i32, i32, i32, i32, vp]),
+    "mario_k_norm_bwd": (i32, [vp, vp, vp, vp, vp, vp, vp, vp, vp, vp, C.c_longlong, i32, i32, i32, i32, vp]),
+    "mario_k_norm_set_variant": (i32, [i32]),
     "mario_kernel_launches": (C.c_longlong, []),
     "mario_k_gemm_set_variant": (i32, [i32]),
     "mario_k_attn_set_variant": (i32, [i32]),

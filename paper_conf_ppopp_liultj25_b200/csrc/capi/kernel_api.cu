@@ -82,20 +82,30 @@ extern "C" int mario_k_norm_fwd(const void* x, const float* g, const float* b, v
 }
 
 extern "C" int mario_k_norm_bwd(const void* dy, const void* x, const float* stats, const float* g, const void* dres,
-                                void* dx, float* dg, float* db, float* partial, int rows, int n, int rms, int bf16,
-                                void* stream) {
+                                void* dx, float* dg, float* db, float* dsum, float* partial, long long partial_floats,
+                                int rows, int n, int rms, int bf16, void* stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (dg && !partial) return static_cast<int>(cudaErrorInvalidValue);
+  const size_t pf = partial_floats > 0 ? static_cast<size_t>(partial_floats) : 0;
   if (bf16) {
     auto* X = static_cast<const __nv_bfloat16*>(x);
     auto* DY = static_cast<const __nv_bfloat16*>(dy);
-    norm_bwd_dx<__nv_bfloat16>(DY, X, stats, g, static_cast<const __nv_bfloat16*>(dres), static_cast<__nv_bfloat16*>(dx),
-                               rows, n, rms, st);
-    if (dg) colsum<__nv_bfloat16>(DY, X, stats, rows, n, n, rms ? 2 : 1, dg, db, partial, st);
+    if (dg) norm_bwd<__nv_bfloat16>(DY, X, stats, g, static_cast<const __nv_bfloat16*>(dres),
+                                    static_cast<__nv_bfloat16*>(dx), rows, n, rms, dg, db, dsum, partial, pf, st);
+    else norm_bwd_dx<__nv_bfloat16>(DY, X, stats, g, static_cast<const __nv_bfloat16*>(dres),
+                                    static_cast<__nv_bfloat16*>(dx), rows, n, rms, st);
   } else {
     auto* X = static_cast<const float*>(x);
     auto* DY = static_cast<const float*>(dy);
-    norm_bwd_dx<float>(DY, X, stats, g, static_cast<const float*>(dres), static_cast<float*>(dx), rows, n, rms, st);
-    if (dg) colsum<float>(DY, X, stats, rows, n, n, rms ? 2 : 1, dg, db, partial, st);
+    if (dg) norm_bwd<float>(DY, X, stats, g, static_cast<const float*>(dres), static_cast<float*>(dx), rows, n, rms, dg,
+                            db, dsum, partial, pf, st);
+    else norm_bwd_dx<float>(DY, X, stats, g, static_cast<const float*>(dres), static_cast<float*>(dx), rows, n, rms, st);
   }
   return static_cast<int>(cudaGetLastError());
+}
+
+extern "C" int mario_k_norm_set_variant(int v) {
+  if (v < 0 || v > 1) return static_cast<int>(cudaErrorInvalidValue);
+  g_norm_tile = v;
+  return 0;
 }

@@ -299,6 +299,7 @@ struct Exec {
     T* dM = reinterpret_cast<T*>(sc + BS.dM);
     float* Dsc = reinterpret_cast<float*>(sc + BS.Dsc);
     float* red = D.template at<float>(D.a.red);
+    const size_t red_floats = D.a.red_bytes / sizeof(float);
     const int32_t* tok = D.template at<int32_t>(D.a.tokens) + static_cast<size_t>(x.micro) * mbs * (s + 1);
     int cur = 0;
     const T* dH;   // gradient of the current layer's output
@@ -313,11 +314,12 @@ struct Exec {
       lin_dgrad(dlog, Wm(D, p, hw), Tn, V, h, dA);      // dHf
       T* dHl = dHbuf[cur];
       if (gpt) {
-        norm_bwd_dx<T>(dA, Hl, stf, Wf(D, p, "lnf.g"), nullptr, dHl, Tn, h, 0, st);
-        colsum<T>(dA, Hl, stf, Tn, h, h, 1, G(D, p, "lnf.g"), G(D, p, "lnf.b"), red, st);
+        // + the fc2 bias gradient of this stage's last layer (column sums of dHl)
+        norm_bwd<T>(dA, Hl, stf, Wf(D, p, "lnf.g"), nullptr, dHl, Tn, h, 0, G(D, p, "lnf.g"), G(D, p, "lnf.b"),
+                    G(D, p, "h" + std::to_string(k * lps + lps - 1) + ".fc2.b"), red, red_floats, st);
       } else {
-        norm_bwd_dx<T>(dA, Hl, stf, Wf(D, p, "nf.g"), nullptr, dHl, Tn, h, 1, st);
-        colsum<T>(dA, Hl, stf, Tn, h, h, 2, G(D, p, "nf.g"), nullptr, red, st);
+        norm_bwd<T>(dA, Hl, stf, Wf(D, p, "nf.g"), nullptr, dHl, Tn, h, 1, G(D, p, "nf.g"), nullptr, nullptr, red,
+                    red_floats, st);
       }
       dH = dHl;
     } else {
@@ -346,16 +348,16 @@ struct Exec {
       if (gpt) {
         gelu_fwd<T>(Z, Gt, static_cast<size_t>(Tn) * f, st);                 // recompute G = gelu(Z)
         lin_wgrad(dH, Gt, Tn, h, f, G(D, p, pre + "fc2.w"));
-        colsum<T>(dH, nullptr, nullptr, Tn, h, h, 0, G(D, p, pre + "fc2.b"), nullptr, red, st);
+        // fc2.b: fused into the norm backward that wrote dH (this stage), else a column sum here
+        if (li == lps - 1 && k != K - 1) colsum<T>(dH, nullptr, nullptr, Tn, h, h, 0, G(D, p, pre + "fc2.b"), nullptr, red, st);
         lin_dgrad(dH, Wm(D, p, pre + "fc2.w"), Tn, h, f, dZ, Z);           // dZ = (dH W2) * gelu'(Z)
         layernorm_fwd<T>(H1, Wf(D, p, pre + "ln2.g"), Wf(D, p, pre + "ln2.b"), A2, st2, Tn, h, m.norm_eps, st);
         lin_wgrad(dZ, A2, Tn, f, h, G(D, p, pre + "fc1.w"));
         colsum<T>(dZ, nullptr, nullptr, Tn, f, f, 0, G(D, p, pre + "fc1.b"), nullptr, red, st);
         lin_dgrad(dZ, Wm(D, p, pre + "fc1.w"), Tn, f, h, dA);               // dA2
-        norm_bwd_dx<T>(dA, H1, st2, Wf(D, p, pre + "ln2.g"), dH, dH1, Tn, h, 0, st);
-        colsum<T>(dA, H1, st2, Tn, h, h, 1, G(D, p, pre + "ln2.g"), G(D, p, pre + "ln2.b"), red, st);
+        norm_bwd<T>(dA, H1, st2, Wf(D, p, pre + "ln2.g"), dH, dH1, Tn, h, 0, G(D, p, pre + "ln2.g"),
+                    G(D, p, pre + "ln2.b"), G(D, p, pre + "proj.b"), red, red_floats, st);
         lin_wgrad(dH1, O, Tn, h, h, G(D, p, pre + "proj.w"));
-        colsum<T>(dH1, nullptr, nullptr, Tn, h, h, 0, G(D, p, pre + "proj.b"), nullptr, red, st);
         lin_dgrad(dH1, Wm(D, p, pre + "proj.w"), Tn, h, h, dO);
       } else {
         swiglu_fwd<T>(Z, Gt, Tn, f, st);                                      // recompute M (into dM)
@@ -365,8 +367,8 @@ struct Exec {
         rmsnorm_fwd<T>(H1, Wf(D, p, pre + "n2.g"), A2, st2, Tn, h, m.norm_eps, st);
         lin_wgrad(dZ, A2, Tn, 2 * f, h, G(D, p, pre + "gu.w"));
         lin_dgrad(dZ, Wm(D, p, pre + "gu.w"), Tn, 2 * f, h, dA);
-        norm_bwd_dx<T>(dA, H1, st2, Wf(D, p, pre + "n2.g"), dH, dH1, Tn, h, 1, st);
-        colsum<T>(dA, H1, st2, Tn, h, h, 2, G(D, p, pre + "n2.g"), nullptr, red, st);
+        norm_bwd<T>(dA, H1, st2, Wf(D, p, pre + "n2.g"), dH, dH1, Tn, h, 1, G(D, p, pre + "n2.g"), nullptr, nullptr,
+                    red, red_floats, st);
         lin_wgrad(dH1, O, Tn, h, h, G(D, p, pre + "o.w"));
         lin_dgrad(dH1, Wm(D, p, pre + "o.w"), Tn, h, h, dO);
       }
@@ -378,11 +380,13 @@ struct Exec {
       if (gpt) colsum<T>(dQKV, nullptr, nullptr, Tn, 3 * h, 3 * h, 0, G(D, p, pre + "qkv.b"), nullptr, red, st);
       lin_dgrad(dQKV, Wm(D, p, pre + "qkv.w"), Tn, 3 * h, h, dA);
       if (gpt) {
-        norm_bwd_dx<T>(dA, Hin, st1, Wf(D, p, pre + "ln1.g"), dH1, dHin, Tn, h, 0, st);
-        colsum<T>(dA, Hin, st1, Tn, h, h, 1, G(D, p, pre + "ln1.g"), G(D, p, pre + "ln1.b"), red, st);
+        // + the previous layer's fc2 bias gradient (column sums of dHin) when it is on this stage
+        norm_bwd<T>(dA, Hin, st1, Wf(D, p, pre + "ln1.g"), dH1, dHin, Tn, h, 0, G(D, p, pre + "ln1.g"),
+                    G(D, p, pre + "ln1.b"), li > 0 ? G(D, p, "h" + std::to_string(l - 1) + ".fc2.b") : nullptr, red,
+                    red_floats, st);
       } else {
-        norm_bwd_dx<T>(dA, Hin, st1, Wf(D, p, pre + "n1.g"), dH1, dHin, Tn, h, 1, st);
-        colsum<T>(dA, Hin, st1, Tn, h, h, 2, G(D, p, pre + "n1.g"), nullptr, red, st);
+        norm_bwd<T>(dA, Hin, st1, Wf(D, p, pre + "n1.g"), dH1, dHin, Tn, h, 1, G(D, p, pre + "n1.g"), nullptr, nullptr,
+                    red, red_floats, st);
       }
       dH = dHin;
       cur = (cur + 2) % 3;

@@ -28,6 +28,11 @@ __device__ __forceinline__ float warp_max(float v) {
 }
 
 inline int cdiv(long a, long b) { return static_cast<int>((a + b - 1) / b); }
+}  // namespace
+
+int g_norm_tile = 1;   // 0: the warp-per-row kernels (kept for A/B measurement)
+
+namespace {
 
 // ------------------------------------------------------------------ embedding
 template <class T>
@@ -452,6 +457,209 @@ __global__ void colsum_final_k(const float* partial, int nblk, int n, int mode, 
   if (mode == 1) out1[c] += s1;
 }
 
+// Block-per-row-tile norm backward (bf16, n = 8 * VPT * nthreads, nthreads % 32 == 0). Thread t owns
+// the 16-byte chunks t, t + nthreads, ... of every row (coalesced), R rows are in flight per
+// iteration, row sums are reduced warp -> shared memory -> block, and each thread keeps its
+// columns' gradient sums in registers across the CTA's contiguous row range. One wave of CTAs.
+// (A forward of the same shape measured no faster than the warp-per-row kernels: not used.)
+__device__ __forceinline__ void load_g8(const float* g, int c, float (&o)[8]) {
+  const float4 a = *reinterpret_cast<const float4*>(g + c), b = *reinterpret_cast<const float4*>(g + c + 4);
+  o[0] = a.x; o[1] = a.y; o[2] = a.z; o[3] = a.w; o[4] = b.x; o[5] = b.y; o[6] = b.z; o[7] = b.w;
+}
+
+// dx = norm'(dy) (+ dres), and, fused, the column partial sums of this CTA's contiguous row range:
+// partial[0][blk] = sum dy * xhat (d gamma), partial[1][blk] = sum dy (d beta, LN only),
+// partial[2][blk] = sum dx (the stored, rounded output: the bias gradient of the linear layer that
+// produced the residual, when sum_out).
+template <int VPT, int R>
+__global__ void __launch_bounds__(VPT == 1 ? 512 : 384) norm_bwd_tile_k(const __nv_bfloat16* dy, const __nv_bfloat16* x,
+                                                       const float* stats, const float* g,
+                                                       const __nv_bfloat16* dres, __nv_bfloat16* dx, int rows, int n,
+                                                       int rms, float* partial, int nblk, int sum_out) {
+  __shared__ float red[2][2][R][32];
+  const int nt = blockDim.x, t = threadIdx.x, w = t / 32, lane = t % 32, nw = nt / 32;
+  const int blk = blockIdx.x;
+  const int rb = static_cast<int>(static_cast<long>(rows) * blk / nblk);
+  const int re = static_cast<int>(static_cast<long>(rows) * (blk + 1) / nblk);
+  float gg[VPT][8], ag[VPT][8], ab[VPT][8], ao[VPT][8];
+#pragma unroll
+  for (int v = 0; v < VPT; ++v) {
+    load_g8(g, (t + v * nt) * 8, gg[v]);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) { ag[v][j] = 0.f; ab[v][j] = 0.f; ao[v][j] = 0.f; }
+  }
+  int it = 0;
+  for (int r0 = rb; r0 < re; r0 += R, ++it) {
+    uint4 ud[R][VPT], ux[R][VPT];
+    float mean[R], rstd[R];
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      const bool ok = r0 + r < re;
+      mean[r] = ok ? stats[2 * (r0 + r)] : 0.f;
+      rstd[r] = ok ? stats[2 * (r0 + r) + 1] : 0.f;
+#pragma unroll
+      for (int v = 0; v < VPT; ++v) {
+        const long o = static_cast<long>(r0 + r) * n + (t + v * nt) * 8;
+        ud[r][v] = ok ? *reinterpret_cast<const uint4*>(dy + o) : make_uint4(0, 0, 0, 0);
+        ux[r][v] = ok ? *reinterpret_cast<const uint4*>(x + o) : make_uint4(0, 0, 0, 0);
+      }
+    }
+    const int pb = it & 1;
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      float sg = 0.f, sgx = 0.f;
+#pragma unroll
+      for (int v = 0; v < VPT; ++v) {
+        const __nv_bfloat16* hd = reinterpret_cast<const __nv_bfloat16*>(&ud[r][v]);
+        const __nv_bfloat16* hx = reinterpret_cast<const __nv_bfloat16*>(&ux[r][v]);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          const float d = __bfloat162float(hd[j]);
+          const float xh = (__bfloat162float(hx[j]) - mean[r]) * rstd[r];
+          const float gp = d * gg[v][j];
+          sg += gp;
+          sgx += gp * xh;
+          ag[v][j] += d * xh;
+          ab[v][j] += d;
+        }
+      }
+      sg = warp_sum(sg);
+      sgx = warp_sum(sgx);
+      if (lane == 0) { red[pb][0][r][w] = sg; red[pb][1][r][w] = sgx; }
+    }
+    __syncthreads();
+#pragma unroll
+    for (int r = 0; r < R; ++r) {
+      if (r0 + r >= re) break;
+      float sg = 0.f, sgx = 0.f;
+      for (int i = 0; i < nw; ++i) { sg += red[pb][0][r][i]; sgx += red[pb][1][r][i]; }
+      sg = rms ? 0.f : sg / n;
+      sgx /= n;
+#pragma unroll
+      for (int v = 0; v < VPT; ++v) {
+        const long o = static_cast<long>(r0 + r) * n + (t + v * nt) * 8;
+        uint4 ur = make_uint4(0, 0, 0, 0);
+        if (dres) ur = *reinterpret_cast<const uint4*>(dres + o);
+        const __nv_bfloat16* hd = reinterpret_cast<const __nv_bfloat16*>(&ud[r][v]);
+        const __nv_bfloat16* hx = reinterpret_cast<const __nv_bfloat16*>(&ux[r][v]);
+        const __nv_bfloat16* hr = reinterpret_cast<const __nv_bfloat16*>(&ur);
+        uint4 uo;
+        __nv_bfloat16* ho = reinterpret_cast<__nv_bfloat16*>(&uo);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) {
+          const float xh = (__bfloat162float(hx[j]) - mean[r]) * rstd[r];
+          float d = (__bfloat162float(hd[j]) * gg[v][j] - sg - xh * sgx) * rstd[r];
+          if (dres) d += __bfloat162float(hr[j]);
+          ho[j] = __float2bfloat16_rn(d);
+          ao[v][j] += __bfloat162float(ho[j]);
+        }
+        *reinterpret_cast<uint4*>(dx + o) = uo;
+      }
+    }
+  }
+  if (!partial) return;
+#pragma unroll
+  for (int v = 0; v < VPT; ++v) {
+    const int c = (t + v * nt) * 8;
+    float* p0 = partial + static_cast<long>(blk) * n + c;
+    float* p1 = partial + static_cast<long>(nblk + blk) * n + c;
+    float* p2 = partial + static_cast<long>(2 * nblk + blk) * n + c;
+    *reinterpret_cast<float4*>(p0) = make_float4(ag[v][0], ag[v][1], ag[v][2], ag[v][3]);
+    *reinterpret_cast<float4*>(p0 + 4) = make_float4(ag[v][4], ag[v][5], ag[v][6], ag[v][7]);
+    if (!rms) {
+      *reinterpret_cast<float4*>(p1) = make_float4(ab[v][0], ab[v][1], ab[v][2], ab[v][3]);
+      *reinterpret_cast<float4*>(p1 + 4) = make_float4(ab[v][4], ab[v][5], ab[v][6], ab[v][7]);
+    }
+    if (sum_out) {
+      *reinterpret_cast<float4*>(p2) = make_float4(ao[v][0], ao[v][1], ao[v][2], ao[v][3]);
+      *reinterpret_cast<float4*>(p2 + 4) = make_float4(ao[v][4], ao[v][5], ao[v][6], ao[v][7]);
+    }
+  }
+}
+
+// out_k[c] += sum_b partial[k][b][c] for the non-null outputs. Block = 32 columns x 8 warps: warp w
+// sums blocks w, w + 8, ... (coalesced 128-byte rows), then the 8 warp sums are added in fixed
+// order (deterministic).
+__global__ void __launch_bounds__(256) colsum_final3_k(const float* partial, int nblk, int n, float* out0, float* out1,
+                                                       float* out2) {
+  __shared__ float red[3][8][33];
+  const int w = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int c = blockIdx.x * 32 + lane;
+  float s0 = 0.f, s1 = 0.f, s2 = 0.f;
+  if (c < n) {
+    for (int b = w; b < nblk; b += 8) {
+      s0 += partial[static_cast<long>(b) * n + c];
+      if (out1) s1 += partial[static_cast<long>(nblk + b) * n + c];
+      if (out2) s2 += partial[static_cast<long>(2 * nblk + b) * n + c];
+    }
+  }
+  red[0][w][lane] = s0; red[1][w][lane] = s1; red[2][w][lane] = s2;
+  __syncthreads();
+  if (w < 3 && c < n) {
+    float t = 0.f;
+#pragma unroll
+    for (int i = 0; i < 8; ++i) t += red[w][i][lane];
+    float* o = w == 0 ? out0 : (w == 1 ? out1 : out2);
+    if (o) o[c] += t;
+  }
+}
+
+// VPT (16-byte chunks per thread) for the tile kernels, 0 when the width does not tile
+inline int tile_vpt(int n) {
+  if (n % 8) return 0;
+  const int ch = n / 8;
+  for (int v = 1; v <= 4; v *= 2)
+    if (ch % v == 0 && (ch / v) % 32 == 0 && ch / v <= (v == 1 ? 512 : 384)) return v;
+  return 0;
+}
+
+int device_sms() {
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    if (sms <= 0) sms = 148;
+  }
+  return sms;
+}
+
+template <class K>
+int resident_grid(K kernel, int threads) {
+  int occ = 1;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, threads, 0);
+  return device_sms() * (occ < 1 ? 1 : occ);
+}
+
+// returns false when the shape does not tile (caller falls back to the row kernels)
+bool norm_bwd_tile(const __nv_bfloat16* dy, const __nv_bfloat16* x, const float* stats, const float* g,
+                   const __nv_bfloat16* dres, __nv_bfloat16* dx, int rows, int n, int rms, float* dg, float* db,
+                   float* dsum, float* partial, size_t partial_floats, cudaStream_t st) {
+  const int vpt = tile_vpt(n);
+  if (!vpt || vpt > 2) return false;
+  const int nt = n / 8 / vpt;
+  const int R = vpt == 1 ? 4 : 2;
+  int nblk = vpt == 1 ? resident_grid(norm_bwd_tile_k<1, 4>, nt) : resident_grid(norm_bwd_tile_k<2, 2>, nt);
+  if (dg) {
+    const long cap = static_cast<long>(partial_floats / (3 * static_cast<size_t>(n)));
+    if (cap < 1) return false;
+    nblk = nblk < cap ? nblk : static_cast<int>(cap);
+  }
+  const int need = cdiv(rows, R);
+  nblk = nblk < need ? nblk : need;
+  if (nblk < 1) return true;
+  float* part = dg ? partial : nullptr;
+  const int so = dsum ? 1 : 0;
+  if (vpt == 1) norm_bwd_tile_k<1, 4><<<nblk, nt, 0, st>>>(dy, x, stats, g, dres, dx, rows, n, rms, part, nblk, so);
+  else norm_bwd_tile_k<2, 2><<<nblk, nt, 0, st>>>(dy, x, stats, g, dres, dx, rows, n, rms, part, nblk, so);
+  note_launch();
+  if (dg) {
+    colsum_final3_k<<<cdiv(n, 32), 256, 0, st>>>(partial, nblk, n, dg, rms ? nullptr : db, dsum);
+    note_launch();
+  }
+  return true;
+}
+
 // ------------------------------------------------------------------ attention
 // One warp per (query row, head); keys in chunks of 32 (one per lane); online softmax.
 template <class T>
@@ -680,6 +888,75 @@ __global__ void gelu_fwd_k(const T* Z, T* G, size_t n) {
   }
 }
 
+// bf16, 16-byte vectors (8 elements per thread-iteration); widths % 8 == 0
+__device__ __forceinline__ float tanh_fast(float x) {
+  float t;
+  asm("tanh.approx.f32 %0, %1;" : "=f"(t) : "f"(x));
+  return t;
+}
+__global__ void gelu_fwd_v8_k(const uint4* Z, uint4* G, size_t n8) {
+  const float c = 0.7978845608028654f;
+  for (size_t i = blockIdx.x * static_cast<size_t>(blockDim.x) + threadIdx.x; i < n8; i += static_cast<size_t>(gridDim.x) * blockDim.x) {
+    const uint4 u = Z[i];
+    const __nv_bfloat16* hz = reinterpret_cast<const __nv_bfloat16*>(&u);
+    uint4 o;
+    __nv_bfloat16* ho = reinterpret_cast<__nv_bfloat16*>(&o);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const float z = __bfloat162float(hz[j]);
+      ho[j] = __float2bfloat16_rn(0.5f * z * (1.f + tanh_fast(c * (z + 0.044715f * z * z * z))));
+    }
+    G[i] = o;
+  }
+}
+// GU row = [gate (f) | up (f)]; M = silu(gate) * up
+__global__ void swiglu_fwd_v8_k(const __nv_bfloat16* GU, __nv_bfloat16* M, int rows, int f) {
+  const int f8 = f / 8;
+  const long n8 = static_cast<long>(rows) * f8;
+  for (long i = blockIdx.x * static_cast<long>(blockDim.x) + threadIdx.x; i < n8; i += static_cast<long>(gridDim.x) * blockDim.x) {
+    const long r = i / f8;
+    const int j8 = static_cast<int>(i - r * f8) * 8;
+    const uint4 ug = *reinterpret_cast<const uint4*>(GU + r * 2 * f + j8);
+    const uint4 uu = *reinterpret_cast<const uint4*>(GU + r * 2 * f + f + j8);
+    const __nv_bfloat16* hg = reinterpret_cast<const __nv_bfloat16*>(&ug);
+    const __nv_bfloat16* hu = reinterpret_cast<const __nv_bfloat16*>(&uu);
+    uint4 o;
+    __nv_bfloat16* ho = reinterpret_cast<__nv_bfloat16*>(&o);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const float g = __bfloat162float(hg[j]);
+      ho[j] = __float2bfloat16_rn(g / (1.f + __expf(-g)) * __bfloat162float(hu[j]));
+    }
+    *reinterpret_cast<uint4*>(M + i * 8) = o;
+  }
+}
+__global__ void swiglu_bwd_v8_k(const __nv_bfloat16* GU, const __nv_bfloat16* dM, __nv_bfloat16* dGU, int rows, int f) {
+  const int f8 = f / 8;
+  const long n8 = static_cast<long>(rows) * f8;
+  for (long i = blockIdx.x * static_cast<long>(blockDim.x) + threadIdx.x; i < n8; i += static_cast<long>(gridDim.x) * blockDim.x) {
+    const long r = i / f8;
+    const int j8 = static_cast<int>(i - r * f8) * 8;
+    const uint4 ug = *reinterpret_cast<const uint4*>(GU + r * 2 * f + j8);
+    const uint4 uu = *reinterpret_cast<const uint4*>(GU + r * 2 * f + f + j8);
+    const uint4 ud = *reinterpret_cast<const uint4*>(dM + i * 8);
+    const __nv_bfloat16* hg = reinterpret_cast<const __nv_bfloat16*>(&ug);
+    const __nv_bfloat16* hu = reinterpret_cast<const __nv_bfloat16*>(&uu);
+    const __nv_bfloat16* hd = reinterpret_cast<const __nv_bfloat16*>(&ud);
+    uint4 og, ou;
+    __nv_bfloat16* hog = reinterpret_cast<__nv_bfloat16*>(&og);
+    __nv_bfloat16* hou = reinterpret_cast<__nv_bfloat16*>(&ou);
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      const float g = __bfloat162float(hg[j]), u = __bfloat162float(hu[j]), dm = __bfloat162float(hd[j]);
+      const float sg = 1.f / (1.f + __expf(-g));
+      hog[j] = __float2bfloat16_rn(dm * u * sg * (1.f + g * (1.f - sg)));
+      hou[j] = __float2bfloat16_rn(dm * g * sg);
+    }
+    *reinterpret_cast<uint4*>(dGU + r * 2 * f + j8) = og;
+    *reinterpret_cast<uint4*>(dGU + r * 2 * f + f + j8) = ou;
+  }
+}
+
 // ---------------------------------------------------------------- softmax-CE
 template <class T>
 __global__ void softmax_ce_k(const float* logits, const int32_t* tok, int ld_tok, int s, int V, float inv_ntok,
@@ -816,6 +1093,8 @@ void norm_bwd_dx(const T* dy, const T* x, const float* stats, const float* g, co
                  int rms, cudaStream_t st) {
   KScope ks_(K_NORM, st);
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
+    if (g_norm_tile && norm_bwd_tile(dy, x, stats, g, dres, dx, rows, n, rms, nullptr, nullptr, nullptr, nullptr, 0, st))
+      return;
     if (n % 8 == 0) {
       if (n <= 1024) norm_bwd_dx_reg_k<4><<<cdiv(rows, 8), 256, 0, st>>>(dy, x, stats, g, dres, dx, rows, n, rms);
       else if (n <= 2048) norm_bwd_dx_reg_k<8><<<cdiv(rows, 8), 256, 0, st>>>(dy, x, stats, g, dres, dx, rows, n, rms);
@@ -856,6 +1135,20 @@ void colsum(const T* a, const T* x, const float* stats, int rows, int n, int lda
 }
 
 template <class T>
+void norm_bwd(const T* dy, const T* x, const float* stats, const float* g, const T* dres, T* dx, int rows, int n,
+              int rms, float* dg, float* db, float* dsum, float* partial, size_t partial_floats, cudaStream_t st) {
+  if constexpr (std::is_same<T, __nv_bfloat16>::value) {
+    if (g_norm_tile) {
+      KScope ks_(K_NORM, st);
+      if (norm_bwd_tile(dy, x, stats, g, dres, dx, rows, n, rms, dg, db, dsum, partial, partial_floats, st)) return;
+    }
+  }
+  norm_bwd_dx<T>(dy, x, stats, g, dres, dx, rows, n, rms, st);
+  colsum<T>(dy, x, stats, rows, n, n, rms ? 2 : 1, dg, db, partial, st);
+  if (dsum) colsum<T>(dx, nullptr, nullptr, rows, n, n, 0, dsum, nullptr, partial, st);
+}
+
+template <class T>
 void attn_fwd(const T* qkv, T* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st) {
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
     if (flash_attn_supported(dh)) { flash_attn_fwd(qkv, O, lse, B, s, nh, dh, st); return; }
@@ -885,12 +1178,26 @@ void rope(T* qkv, int B, int s, int nh, int dh, float base, int inverse, cudaStr
 template <class T>
 void swiglu_fwd(const T* GU, T* M, int rows, int f, cudaStream_t st) {
   KScope ks_(K_ELEMWISE, st);
+  if constexpr (std::is_same<T, __nv_bfloat16>::value) {
+    if (f % 8 == 0) {
+      swiglu_fwd_v8_k<<<grid_for(static_cast<long>(rows) * f / 8), 256, 0, st>>>(GU, M, rows, f);
+      note_launch();
+      return;
+    }
+  }
   swiglu_fwd_k<T><<<grid_for(static_cast<long>(rows) * f), 256, 0, st>>>(GU, M, rows, f);
   note_launch();
 }
 template <class T>
 void swiglu_bwd(const T* GU, const T* dM, T* dGU, int rows, int f, cudaStream_t st) {
   KScope ks_(K_ELEMWISE, st);
+  if constexpr (std::is_same<T, __nv_bfloat16>::value) {
+    if (f % 8 == 0) {
+      swiglu_bwd_v8_k<<<grid_for(static_cast<long>(rows) * f / 8), 256, 0, st>>>(GU, dM, dGU, rows, f);
+      note_launch();
+      return;
+    }
+  }
   swiglu_bwd_k<T><<<grid_for(static_cast<long>(rows) * f), 256, 0, st>>>(GU, dM, dGU, rows, f);
   note_launch();
 }
@@ -904,6 +1211,14 @@ void softmax_ce(const float* logits, const int32_t* tok, int ld_tok, int s, int 
 template <class T>
 void gelu_fwd(const T* Z, T* G, size_t n, cudaStream_t st) {
   KScope ks_(K_ELEMWISE, st);
+  if constexpr (std::is_same<T, __nv_bfloat16>::value) {
+    if (n % 8 == 0 && reinterpret_cast<uintptr_t>(Z) % 16 == 0 && reinterpret_cast<uintptr_t>(G) % 16 == 0) {
+      gelu_fwd_v8_k<<<grid_for(static_cast<long>(n / 8)), 256, 0, st>>>(reinterpret_cast<const uint4*>(Z),
+                                                                        reinterpret_cast<uint4*>(G), n / 8);
+      note_launch();
+      return;
+    }
+  }
   gelu_fwd_k<T><<<grid_for(static_cast<long>(n)), 256, 0, st>>>(Z, G, n);
   note_launch();
 }
@@ -928,6 +1243,8 @@ void copy_f32(float* a, const float* b, size_t n, cudaStream_t st) { copy_k<<<gr
   template void norm_bwd_dx<T>(const T*, const T*, const float*, const float*, const T*, T*, int, int, int,          \
                                cudaStream_t);                                                                      \
   template void colsum<T>(const T*, const T*, const float*, int, int, int, int, float*, float*, float*, cudaStream_t); \
+  template void norm_bwd<T>(const T*, const T*, const float*, const float*, const T*, T*, int, int, int, float*,      \
+                            float*, float*, float*, size_t, cudaStream_t);                                           \
   template void attn_fwd<T>(const T*, T*, float*, int, int, int, int, cudaStream_t);                                 \
   template void attn_bwd<T>(const T*, const T*, const T*, const float*, T*, float*, int, int, int, int, cudaStream_t); \
   template void rope<T>(T*, int, int, int, int, float, int, cudaStream_t);                                           \

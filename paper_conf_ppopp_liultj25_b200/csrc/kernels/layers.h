@@ -23,6 +23,13 @@ template <class T> void rmsnorm_fwd(const T* x, const float* g, T* y, float* sta
 // dx = LN'(dy) (+ dres); rms = 1 selects RMSNorm.
 template <class T> void norm_bwd_dx(const T* dy, const T* x, const float* stats, const float* g, const T* dres,
                                     T* dx, int rows, int n, int rms, cudaStream_t st);
+// Fused norm backward: dx as norm_bwd_dx, plus dg (+ db for LN) += the norm's column sums and, if
+// dsum != NULL, dsum += column sums of the written dx (the bias gradient of the producing linear).
+// partial: fp32 scratch of partial_floats (>= 3 * n * blocks used; falls back to separate passes).
+template <class T> void norm_bwd(const T* dy, const T* x, const float* stats, const float* g, const T* dres, T* dx,
+                                 int rows, int n, int rms, float* dg, float* db, float* dsum, float* partial,
+                                 size_t partial_floats, cudaStream_t st);
+extern int g_norm_tile;
 // Column reductions into fp32 grads (+=): mode 0: out0 += sum_r a[r,c]
 // mode 1 (LN): out0 += sum dy*xhat, out1 += sum dy; mode 2 (RMS): out0 += sum dy*xhat.
 template <class T> void colsum(const T* a, const T* x, const float* stats, int rows, int n, int lda, int mode,
