@@ -37,7 +37,11 @@ typedef enum { MARIO_GPT = 0, MARIO_LLAMA = 1 } mario_family;
 /* Pipeline schemes: "V" 1F1B, "W" Interleave, "X" Chimera. */
 typedef enum { MARIO_1F1B = 0, MARIO_INTERLEAVE = 1, MARIO_CHIMERA = 2 } mario_scheme;
 /* Evaluation configurations: base, ckpt (pass 1 only), ovlp (= passes 1-4). */
-typedef enum { MARIO_LEVEL_BASE = 0, MARIO_LEVEL_CKPT = 1, MARIO_LEVEL_MARIO = 2 } mario_level;
+/* MARIO_LEVEL_BUDGET (extension, DESIGN reading A28): passes 1-4 on devices
+ * 0 .. S-k-1 while the tail devices S-k .. S-1 keep their full activations in base order; k is the
+ * feasible choice (every device's simulated peak <= mem_budget) with the smallest simulated
+ * makespan, ties to the smaller k. Needs mem_budget_bytes > 0. */
+typedef enum { MARIO_LEVEL_BASE = 0, MARIO_LEVEL_CKPT = 1, MARIO_LEVEL_MARIO = 2, MARIO_LEVEL_BUDGET = 3 } mario_level;
 typedef enum { MARIO_F32 = 0, MARIO_BF16 = 1 } mario_dtype;
 /* Instruction types (Table 3). */
 typedef enum {
@@ -127,6 +131,8 @@ mario_status mario_plan_rank_params(const struct mario_plan* plan, int32_t rank,
 /* Name of the global parameter `idx` (canonical order), e.g. "h3.qkv.w". */
 const char* mario_param_name(const struct mario_plan* plan, int32_t idx);
 int32_t mario_param_count(const struct mario_plan* plan);
+/* k of MARIO_LEVEL_BUDGET (0 for the other levels); -1 on NULL. */
+int32_t mario_plan_unckpt_tail(const struct mario_plan* plan);
 void mario_plan_destroy(struct mario_plan* plan);
 
 /* Schedule tuner (§5.3, Eq. 1): grid search

@@ -33,6 +33,7 @@ SEND = (SA, SG)
 
 V_1F1B, W_INTERLEAVE, X_CHIMERA = "1f1b", "interleave", "chimera"
 BASE, CKPT, MARIO = "base", "ckpt", "mario"
+MARIO_BUDGET = "mario_budget"   # extension (reading A28)
 
 Instr = Tuple[str, int, int]  # (op, micro, part)
 
@@ -245,11 +246,15 @@ def build_base(pipe: Pipe) -> List[List[Instr]]:
 
 
 # ------------------------------------------------------------------------------ passes
-def pass1_apply_checkpoint(lists):
+def pass1_apply_checkpoint(lists, keep=()):
     """every FW_i -> CFW_i; RC_i inserted right before BW_i (after RG_i: the naive
-    placement of Fig. 2 step 1, reading A14)."""
+    placement of Fig. 2 step 1, reading A14). Devices in `keep` stay un-checkpointed in their
+    base order (the budget-driven extension, reading A28; empty for the paper's passes)."""
     out = []
-    for L in lists:
+    for d, L in enumerate(lists):
+        if d in keep:
+            out.append(list(L))
+            continue
         N = []
         for (op, m, p) in L:
             if op == FW:
@@ -362,18 +367,47 @@ def pass4_prepose_forward(pipe, lists, costs, mem=None, budget=None, max_rounds=
     return lists
 
 
-def transform(pipe: Pipe, level: str, costs=None, mem=None, budget=None):
-    """BASE: base lists. CKPT: pass 1 only (naive full-checkpoint, A14). MARIO: passes 1-4."""
+def transform(pipe: Pipe, level: str, costs=None, mem=None, budget=None, keep=()):
+    """BASE: base lists. CKPT: pass 1 only (naive full-checkpoint, A14). MARIO: passes 1-4.
+    MARIO_BUDGET: passes 1-4 with the tail devices chosen by pass5_budget left un-checkpointed.
+    `keep`: devices passes 1-4 leave in their base order (used by pass5_budget)."""
+    if level == MARIO_BUDGET:
+        return pass5_budget(pipe, costs or UnitCosts(), mem, budget)[0]
     lists = build_base(pipe)
     if level == BASE:
         return lists
-    lists = pass1_apply_checkpoint(lists)
+    lists = pass1_apply_checkpoint(lists, keep)
     if level == CKPT:
         return lists
     lists = pass2_overlap_recompute(lists)
     lists = pass3_remove_redundancy(lists)
     costs = costs or UnitCosts()
     return pass4_prepose_forward(pipe, lists, costs, mem, budget)
+
+
+def pass5_budget(pipe: Pipe, costs, mem, budget):
+    """Budget-driven partial checkpointing (reading A28): Pass 3 un-checkpoints
+    a stage only when CFW_i and BW_i are adjacent; with memory to spare (mem_budget)
+    the tail devices d >= S - k can keep their full activations in their 1F1B order (device d then
+    holds its base in-flight count of activation sets, Table 1) while devices < S - k go through
+    passes 1-4. For k = 0 .. S: lists_k = transform(MARIO, keep = tail k); feasible iff the peak
+    of every device is within the budget; pick the smallest makespan, ties to the smaller k.
+    Returns (lists, k)."""
+    assert mem is not None and budget is not None, "MARIO_BUDGET needs mem and budget"
+    best = None
+    for k in range(pipe.S + 1):
+        keep = set(range(pipe.S - k, pipe.S))
+        L = transform(pipe, MARIO, costs, mem, budget, keep=keep)
+        if max(memory_walk(pipe, L, mem).peak) > budget:
+            continue
+        r = simulate(pipe, L, costs)
+        if r is None:
+            continue
+        if best is None or r.makespan < best[0] - 1e-9:
+            best = (r.makespan, L, k)
+    if best is None:   # nothing fits: the paper's passes (the caller reports EBUDGET)
+        return transform(pipe, MARIO, costs, mem, budget), 0
+    return best[1], best[2]
 
 
 # ---------------------------------------------------------------------------- simulator

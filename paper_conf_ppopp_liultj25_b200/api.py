@@ -8,13 +8,13 @@ planning, simulation and every step of the training iteration run inside the lib
 from __future__ import annotations
 
 import ctypes as C
-from dataclasses import dataclass
+from dataclasses import replace, dataclass
 from typing import Dict, List, Optional, Sequence, Tuple
 
 from . import _lib
 
 SCHEMES = {"1f1b": 0, "v": 0, "interleave": 1, "w": 1, "chimera": 2, "x": 2}
-LEVELS = {"base": 0, "ckpt": 1, "mario": 2, "ovlp": 2}
+LEVELS = {"base": 0, "ckpt": 1, "mario": 2, "ovlp": 2, "mario_budget": 3}
 OPS = ["FW", "CFW", "RC", "BW", "SA", "RA", "SG", "RG"]
 STATUS = {0: "OK", -1: "EINVAL", -2: "EBUDGET", -3: "EDEADLOCK", -4: "ECUDA", -5: "ENCCL", -6: "ESTATE"}
 
@@ -85,6 +85,7 @@ _lib.register("mario_plan_rank_params", C.c_int32, [_P, C.c_int32, C.POINTER(C.P
 _lib.register("mario_param_name", C.c_char_p, [_P, C.c_int32])
 _lib.register("mario_param_count", C.c_int32, [_P])
 _lib.register("mario_plan_destroy", None, [_P])
+_lib.register("mario_plan_unckpt_tail", C.c_int32, [_P])
 _lib.register("mario_last_error", C.c_char_p, [])
 _lib.register("mario_tune", C.c_int32, [C.POINTER(CModel), C.c_int32, C.c_int32, C.c_uint64, C.POINTER(CTuneCosts),
                                         C.POINTER(CTuneResult), C.c_int32, C.POINTER(C.c_int32), C.POINTER(C.c_int32)])
@@ -169,6 +170,11 @@ class Plan:
         _check(_lib.lib().mario_plan_instrs(self.handle, d, C.byref(p), C.byref(n)))
         return [(OPS[p[i].op], p[i].micro, p[i].part, p[i].vstage, p[i].peer, p[i].slot, p[i].aslot)
                 for i in range(n.value)]
+
+    @property
+    def unckpt_tail(self) -> int:
+        """MARIO_LEVEL_BUDGET: how many tail devices keep full activations (reading A28)."""
+        return int(_lib.lib().mario_plan_unckpt_tail(self.handle))
 
     def lists(self) -> List[List[Tuple[str, int, int]]]:
         return [[(op, m, p) for (op, m, p, *_r) in self.instrs(d)] for d in range(self.S)]
@@ -317,7 +323,7 @@ def alloc_for(plan: Plan, rank: int, device="cuda"):
 
 
 SCHEME_NAMES = {0: "1f1b", 1: "interleave", 2: "chimera"}
-LEVEL_NAMES = {0: "base", 1: "ckpt", 2: "mario"}
+LEVEL_NAMES = {0: "base", 1: "ckpt", 2: "mario", 3: "mario_budget"}
 
 
 def tune(cfg, devices: int, global_batch: int, mem_budget: int = 0, costs: Optional[dict] = None,
@@ -345,6 +351,36 @@ def tune(cfg, devices: int, global_batch: int, mem_budget: int = 0, costs: Optio
                      "feasible": bool(r.feasible), "makespan_ms": r.makespan_ms, "samples_per_s": r.samples_per_s,
                      "bubble_ratio": r.bubble_ratio, "peak_bytes": r.peak_bytes})
     return rows, best.value
+
+
+def max_seq_len(cfg, stages: int, microbatches: int, level: str, mem_budget: int, scheme: str = "1f1b",
+                chunks: int = 1, start: int = 1024, step: int = 64, limit: int = 1 << 20) -> int:
+    """Sequence-length scaling (§6.5): the largest s = start + i*step
+    whose plan's simulated per-device peak (static + activations) fits mem_budget, or 0 when
+    `start` does not fit. Planner only: nothing is executed. Peaks grow with s, so the search is a
+    doubling phase then a bisection over multiples of `step`."""
+    def fits(s_len):
+        try:
+            Plan(replace(cfg, seq_len=s_len), stages, microbatches, scheme, level, chunks=chunks,
+                 mem_budget=mem_budget)
+            return True
+        except MarioError as e:
+            if e.code != -2:
+                raise
+            return False
+    if not fits(start):
+        return 0
+    lo, hi = 0, 1   # in steps beyond start: lo fits, hi unknown
+    while start + hi * step <= limit and fits(start + hi * step):
+        lo, hi = hi, hi * 2
+    hi = min(hi, (limit - start) // step + 1)
+    while hi - lo > 1:
+        mid = (lo + hi) // 2
+        if fits(start + mid * step):
+            lo = mid
+        else:
+            hi = mid
+    return start + lo * step
 
 
 def adamw_step(params, grads, m, v, step: int, lr: float, beta1=0.9, beta2=0.95, eps=1e-8, weight_decay=0.1,

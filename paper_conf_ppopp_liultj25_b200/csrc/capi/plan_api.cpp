@@ -17,7 +17,9 @@ using namespace mario::plan;
 namespace {
 
 const char* scheme_name(int s) { return s == MARIO_1F1B ? "1f1b" : s == MARIO_INTERLEAVE ? "interleave" : "chimera"; }
-const char* level_name(int l) { return l == MARIO_LEVEL_BASE ? "base" : l == MARIO_LEVEL_CKPT ? "ckpt" : "mario"; }
+const char* level_name(int l) {
+  return l == MARIO_LEVEL_BASE ? "base" : l == MARIO_LEVEL_CKPT ? "ckpt" : l == MARIO_LEVEL_MARIO ? "mario" : "mario_budget";
+}
 
 // Round-robin walk (the simulator's order, ignoring time): a receive is walked only after its
 // matching send. Used by the loopback executor; returns false on a cycle.
@@ -247,6 +249,10 @@ std::string serialize(const PlanObj& P) {
   snprintf(buf, sizeof buf, "pipe scheme=%s S=%d N=%d v=%d level=%s\n", scheme_name(P.pp.scheme), P.pp.S, P.pp.N,
            P.pp.v, level_name(P.level));
   s += buf;
+  if (P.level == MARIO_LEVEL_BUDGET) {
+    snprintf(buf, sizeof buf, "unckpt_tail=%d\n", P.unckpt_tail);
+    s += buf;
+  }
   for (int d = 0; d < P.pp.S; ++d) {
     snprintf(buf, sizeof buf, "dev %d:", d);
     s += buf;
@@ -270,7 +276,9 @@ extern "C" mario_status mario_plan(const mario_model* model, int32_t stages, int
     if (const char* e = validate_model(*model)) return set_error(MARIO_EINVAL, e);
     if (stages < 1 || microbatches < 1) return set_error(MARIO_EINVAL, "stages and microbatches must be >= 1");
     if (scheme < 0 || scheme > 2) return set_error(MARIO_EINVAL, "unknown scheme");
-    if (level < 0 || level > 2) return set_error(MARIO_EINVAL, "unknown level");
+    if (level < 0 || level > 3) return set_error(MARIO_EINVAL, "unknown level");
+    if (level == MARIO_LEVEL_BUDGET && mem_budget_bytes == 0)
+      return set_error(MARIO_EINVAL, "MARIO_LEVEL_BUDGET needs mem_budget_bytes > 0");
     if (scheme != MARIO_INTERLEAVE) chunks = 1;
     if (chunks < 1) return set_error(MARIO_EINVAL, "chunks must be >= 1");
     Pipe pp{scheme, stages, microbatches, chunks};
@@ -279,32 +287,58 @@ extern "C" mario_status mario_plan(const mario_model* model, int32_t stages, int
       return set_error(MARIO_EINVAL, "Interleave needs stages >= 2 and microbatches % stages == 0");
     if (scheme == MARIO_CHIMERA && (stages % 2 || microbatches % stages))
       return set_error(MARIO_EINVAL, "Chimera needs even stages and microbatches % stages == 0");
-    auto P = std::make_unique<PlanObj>();
-    P->model = *model;
-    P->pp = pp;
-    P->level = level;
-    P->budget = mem_budget_bytes;
-    P->lps = model->n_layers / pp.K();
-    build_rank_params(*P);
-    fill_costs(*P, costs);
-    Lists L = build_base(pp);
-    if (level != MARIO_LEVEL_BASE) {
-      L = pass1_apply_checkpoint(L);
-      if (level == MARIO_LEVEL_MARIO) {
-        L = pass2_overlap_recompute(L);
-        L = pass3_remove_redundancy(L);
+    // one candidate plan: `lvl` in {BASE, CKPT, MARIO}; `keep_tail` devices un-checkpointed (A28)
+    auto build = [&](int lvl, int keep_tail, std::unique_ptr<PlanObj>& P) -> mario_status {
+      P = std::make_unique<PlanObj>();
+      P->model = *model;
+      P->pp = pp;
+      P->level = level;
+      P->budget = mem_budget_bytes;
+      P->unckpt_tail = keep_tail;
+      P->lps = model->n_layers / pp.K();
+      build_rank_params(*P);
+      fill_costs(*P, costs);
+      std::vector<bool> keep(pp.S, false);
+      for (int d = pp.S - keep_tail; d < pp.S; ++d) keep[d] = true;
+      Lists L = build_base(pp);
+      if (lvl != MARIO_LEVEL_BASE) {
+        L = pass1_apply_checkpoint(L, keep);
+        if (lvl == MARIO_LEVEL_MARIO) {
+          L = pass2_overlap_recompute(L);
+          L = pass3_remove_redundancy(L);
+        }
       }
-    }
-    P->lists = L;
-    if (!walk_order(pp, P->lists, P->loopback_order)) return set_error(MARIO_EDEADLOCK, "base lists deadlock");
-    assign_slots_and_pools(*P);
-    fill_static(*P, costs);
-    if (level == MARIO_LEVEL_MARIO) {
-      P->lists = pass4_prepose_forward(pp, P->lists, P->costs, static_cast<double>(mem_budget_bytes));
-      P->loopback_order.clear();
-      if (!walk_order(pp, P->lists, P->loopback_order)) return set_error(MARIO_EDEADLOCK, "plan deadlocks");
+      P->lists = L;
+      if (!walk_order(pp, P->lists, P->loopback_order)) return set_error(MARIO_EDEADLOCK, "base lists deadlock");
       assign_slots_and_pools(*P);
       fill_static(*P, costs);
+      if (lvl == MARIO_LEVEL_MARIO) {
+        P->lists = pass4_prepose_forward(pp, P->lists, P->costs, static_cast<double>(mem_budget_bytes));
+        P->loopback_order.clear();
+        if (!walk_order(pp, P->lists, P->loopback_order)) return set_error(MARIO_EDEADLOCK, "plan deadlocks");
+        assign_slots_and_pools(*P);
+        fill_static(*P, costs);
+      }
+      return MARIO_OK;
+    };
+    std::unique_ptr<PlanObj> P;
+    if (level != MARIO_LEVEL_BUDGET) {
+      if (mario_status st = build(level, 0, P)) return st;
+    } else {
+      // k = 0 .. S: feasible (max peak <= budget) with the smallest makespan, ties to smaller k
+      int best_k = -1;
+      double best_t = 0;
+      for (int k = 0; k <= pp.S; ++k) {
+        std::unique_ptr<PlanObj> C;
+        if (build(MARIO_LEVEL_MARIO, k, C) != MARIO_OK) continue;
+        const SimResult r = simulate(pp, C->lists, C->costs);
+        if (!r.ok) continue;
+        const MemResult mr = memory_walk(pp, C->lists, C->costs);
+        const double worst = *std::max_element(mr.peak.begin(), mr.peak.end());
+        if (worst > static_cast<double>(mem_budget_bytes)) continue;
+        if (best_k < 0 || r.makespan < best_t - 1e-9) { best_k = k; best_t = r.makespan; }
+      }
+      if (mario_status st = build(MARIO_LEVEL_MARIO, best_k < 0 ? 0 : best_k, P)) return st;
     }
     P->sim = simulate(pp, P->lists, P->costs);
     if (!P->sim.ok) return set_error(MARIO_EDEADLOCK, "simulator found a dependency cycle");
@@ -332,6 +366,8 @@ extern "C" mario_status mario_plan(const mario_model* model, int32_t stages, int
     return MARIO_OK;
   });
 }
+
+extern "C" int32_t mario_plan_unckpt_tail(const struct mario_plan* P) { return P ? P->unckpt_tail : -1; }
 
 extern "C" mario_status mario_plan_instrs(const struct mario_plan* P, int32_t device, const mario_instr** instrs,
                                           int32_t* n) {

@@ -56,10 +56,14 @@ extern "C" mario_status mario_tune(const mario_model* model, int32_t devices, in
           }
           mario_costs mc{fw.data(), bw.data(), rc.data(), costs ? costs->p2p_alpha_ms : 0.01,
                          costs ? costs->p2p_GBps : 700.0, nullptr, nullptr, nullptr, -1.0};
-          for (int level : {MARIO_LEVEL_BASE, MARIO_LEVEL_MARIO}) {
+          // the budget-driven level (A28) joins the grid when there is a budget to drive it
+          std::vector<int> levels{MARIO_LEVEL_BASE, MARIO_LEVEL_MARIO};
+          if (mem_budget_bytes > 0) levels.push_back(MARIO_LEVEL_BUDGET);
+          for (int level : levels) {
             PlanObj* P = nullptr;
             mario_tune_result r{sch, pp, v, dp, mbs, N, level, 0, 0.0, 0.0, 0.0, 0};
-            if (mario_plan(&m, pp, N, sch, v, 0, level, &mc, &P) == MARIO_OK) {
+            const uint64_t plan_budget = level == MARIO_LEVEL_BUDGET ? mem_budget_bytes : 0;
+            if (mario_plan(&m, pp, N, sch, v, plan_budget, level, &mc, &P) == MARIO_OK) {
               mario_sim sim;
               mario_plan_simulate(P, &sim);
               r.makespan_ms = sim.makespan_ms;

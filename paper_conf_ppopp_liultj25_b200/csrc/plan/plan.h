@@ -52,7 +52,8 @@ struct Pipe {
 bool find_inst(const Pipe& pp, int d, int m, int p, int t, bool nxt, int* d_o, int* p_o);
 
 Lists build_base(const Pipe& pp);
-Lists pass1_apply_checkpoint(const Lists& in);
+// keep: devices left un-checkpointed in their base order (budget extension, reading A28)
+Lists pass1_apply_checkpoint(const Lists& in, const std::vector<bool>& keep = {});
 Lists pass2_overlap_recompute(const Lists& in);
 Lists pass3_remove_redundancy(const Lists& in);
 

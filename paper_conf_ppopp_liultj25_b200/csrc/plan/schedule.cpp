@@ -172,9 +172,11 @@ Lists build_base(const Pipe& pp) {
 }
 
 // Pass 1: FW -> CFW; RC inserted right before BW (after RG), reading A14.
-Lists pass1_apply_checkpoint(const Lists& in) {
+Lists pass1_apply_checkpoint(const Lists& in, const std::vector<bool>& keep) {
   Lists out;
-  for (const List& L : in) {
+  for (size_t d = 0; d < in.size(); ++d) {
+    const List& L = in[d];
+    if (d < keep.size() && keep[d]) { out.push_back(L); continue; }
     List N;
     for (const Instr& x : L) {
       if (x.op == FW) N.push_back({CFW, x.m, x.p});

@@ -22,8 +22,8 @@ def ctx():
     return _CTX["c"]
 
 
-def run_plan(cfg, S, N, scheme, level, dtype, params, toks, chunks=1):
-    plan = api.Plan(cfg, S, N, scheme, level, chunks=chunks, dtype=dtype)
+def run_plan(cfg, S, N, scheme, level, dtype, params, toks, chunks=1, mem_budget=0, costs=None):
+    plan = api.Plan(cfg, S, N, scheme, level, chunks=chunks, dtype=dtype, mem_budget=mem_budget, costs=costs)
     rank = -1 if S > 1 else 0
     w, g, ws = api.alloc_for(plan, rank)
     w.copy_(torch.from_numpy(api.pack_params(plan, params, rank)))
@@ -98,6 +98,21 @@ def test_mario_bitwise_equals_base(dtype):
     toks = synth.make_tokens(cfg, 8)
     outs = [run_plan(cfg, 4, 8, "1f1b", lvl, dtype, params, toks)[2] for lvl in ("base", "ckpt", "mario")]
     assert np.array_equal(outs[0], outs[1]) and np.array_equal(outs[0], outs[2])
+
+
+@pytest.mark.parametrize("dtype", ["f32", "bf16"])
+def test_budget_level_bitwise_equals_base(dtype):
+    """Budget-driven partial checkpointing (f2, A28) mixes FW devices (base order) with CFW/RC
+    devices: still bitwise equal. Unit costs, one unit per activation set, budget 2 -> k = 2 of 4."""
+    cfg = synth.TINY_GPT
+    params = synth.make_weights(cfg)
+    toks = synth.make_tokens(cfg, 8)
+    unit = {"fw_ms": [1.0] * 4, "bw_ms": [2.0] * 4, "rc_ms": [1.0] * 4, "act_bytes": [1.0] * 4,
+            "ckpt_bytes": [0.0] * 4, "work_bytes": [0.0] * 4, "static_bytes": 0.0}
+    assert api.Plan(cfg, 4, 8, "1f1b", "mario_budget", dtype=dtype, mem_budget=2, costs=unit).unckpt_tail == 2
+    a = run_plan(cfg, 4, 8, "1f1b", "base", dtype, params, toks)[2]
+    b = run_plan(cfg, 4, 8, "1f1b", "mario_budget", dtype, params, toks, mem_budget=2, costs=unit)[2]
+    assert np.array_equal(a, b)
 
 
 def test_ragged_multi_tile_bf16():

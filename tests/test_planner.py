@@ -49,6 +49,34 @@ def test_lists_match_oracle(scheme, S, N, v, level):
         assert a == [r.start[(d,) + x] for x in comp]
 
 
+@pytest.mark.parametrize("budget", [1, 2, 3, 5, 100])
+@pytest.mark.parametrize("scheme,S,N,v", CASES)
+def test_budget_level_matches_oracle(scheme, S, N, v, budget):
+    """MARIO_LEVEL_BUDGET (f2, reading A28): same lists and tail k as oracle pass5_budget."""
+    K = S * v
+    pipe = osch.Pipe(OP_SCHEME[scheme], S, N, v)
+    F = 1.0 / v
+    c = osch.UnitCosts(F=F, B=2 * F, R=F)
+    want, k = osch.pass5_budget(pipe, c, osch.MemUnits(), budget)
+    try:
+        plan = Plan(model_for(K * 2 if scheme != "chimera" else S * 2), S, N, scheme, "mario_budget", chunks=v,
+                    dtype="f32", costs=unit_costs(K, F, 2 * F, F), mem_budget=budget)
+    except MarioError as e:   # nothing fits: EBUDGET, and the oracle's lists exceed the budget too
+        assert e.code == -2
+        assert max(osch.memory_walk(pipe, want, osch.MemUnits()).peak) > budget
+        return
+    assert plan.lists() == want
+    assert plan.unckpt_tail == k
+    assert plan.simulate().makespan_ms == osch.simulate(pipe, want, c).makespan
+    assert "unckpt_tail=%d" % k in plan.serialize()
+
+
+def test_budget_level_needs_a_budget():
+    with pytest.raises(MarioError) as e:
+        Plan(model_for(4), 4, 4, "1f1b", "mario_budget", dtype="f32", costs=unit_costs(4))
+    assert e.value.code == -1
+
+
 def test_fig2_through_abi():
     totals = []
     for level in ("base", "ckpt", "mario"):
@@ -171,3 +199,20 @@ def test_chrome_trace_of_fig2():
     assert len(boxes) == sum(1 for d in range(4) for x in p.instrs(d) if x[0] in ("FW", "CFW", "RC", "BW"))
     assert max(e["ts"] + e["dur"] for e in boxes) == 22.0 * 1e3   # Fig. 2 step 4: 22t
     json.dumps(tr)
+
+
+def test_max_seq_len_boundary_and_order():
+    """§6.5 analogue: PP 8, mbs 1, N = 2 x stages, 40 GB cap (the paper's
+    A100-40G). The returned s fits and s + 64 does not; freeing activation memory (Mario) admits a
+    longer sequence than base 1F1B and no shorter one than naive full checkpointing."""
+    cfg = synth.with_(synth.GPT3_1P3B, micro_batch=1)
+    cap = 40 * 10 ** 9
+    got = {lvl: api.max_seq_len(cfg, 8, 16, lvl, cap) for lvl in ("base", "ckpt", "mario", "mario_budget")}
+    for lvl, s in got.items():
+        assert s >= 1024 and (s - 1024) % 64 == 0
+        Plan(synth.with_(cfg, seq_len=s), 8, 16, "1f1b", lvl, mem_budget=cap)
+        with pytest.raises(MarioError):
+            Plan(synth.with_(cfg, seq_len=s + 64), 8, 16, "1f1b", lvl, mem_budget=cap)
+    assert got["mario"] > 1.3 * got["base"]
+    assert got["mario"] >= got["ckpt"] and got["mario_budget"] >= got["mario"]
+    assert api.max_seq_len(cfg, 8, 16, "base", 10 ** 6) == 0

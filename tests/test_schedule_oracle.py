@@ -5,11 +5,11 @@ import os
 
 import pytest
 
-from oracle.schedule import (BASE, CKPT, MARIO, BW, CFW, FW, RA, RC, RG, SA, SG, V_1F1B,
+from oracle.schedule import (BASE, CKPT, MARIO, MARIO_BUDGET, BW, CFW, FW, RA, RC, RG, SA, SG, V_1F1B,
                              W_INTERLEAVE, X_CHIMERA, MemUnits, Pipe, UnitCosts, build_base,
                              check_structure, find_inst, memory_walk, pass1_apply_checkpoint,
                              pass2_overlap_recompute, pass3_remove_redundancy,
-                             pass4_prepose_forward, simulate, transform)
+                             pass4_prepose_forward, pass5_budget, simulate, transform)
 
 GOLD = os.path.join(os.path.dirname(__file__), "golden")
 
@@ -152,3 +152,61 @@ def test_budget_blocks_prepose():
     l4 = pass4_prepose_forward(pipe, l3, c, mem=mem, budget=peak3)
     assert max(memory_walk(pipe, l4, mem).peak) <= peak3
     assert simulate(pipe, l4, c).makespan >= 22
+
+
+# ------------------------------------------------ budget-driven partial checkpointing (f2, A28)
+def _tail_makespan(S, N, k):
+    """[derived] 1F1B, F = 1, B = 2, RC = 1: Mario's closed form (S-2)(F+B) + N(F+B+R) for k <= 1;
+    each further un-checkpointed tail device takes one RC off the critical path (3 units, SURVEY d4:
+    146 -> 143 -> ... -> 128 at S = 8, N = 32), never below base (N+S-1)(F+B); k = S is base."""
+    mario_t, base_t = (S - 2) * 3 + N * 4, (N + S - 1) * 3
+    if k <= 1:
+        return mario_t
+    return base_t if k == S else max(base_t, mario_t - 3 * (k - 1))
+
+
+@pytest.mark.parametrize("S,N", [(4, 8), (4, 16), (6, 12), (8, 16)])
+def test_budget_tail_1f1b_closed_form(S, N):
+    """A tail device d keeps its base in-flight count S - d (Table 1), so a budget of b activation
+    sets admits tails k <= b; the level picks the fastest, ties to the smaller k."""
+    pipe, c, mem = Pipe(V_1F1B, S, N), UnitCosts(), MemUnits()
+    for b in range(1, S + 1):
+        L, k = pass5_budget(pipe, c, mem, b)
+        check_structure(pipe, L)
+        ks = [0] + list(range(2, min(b, S) + 1))
+        want_t = min(_tail_makespan(S, N, j) for j in ks)
+        want_k = min(j for j in ks if _tail_makespan(S, N, j) == want_t)
+        assert (k, simulate(pipe, L, c).makespan) == (want_k, want_t)
+        peaks = memory_walk(pipe, L, mem).peak
+        assert peaks == [float(S - d) if d >= S - k else 1.0 for d in range(S)]
+        if k == S:
+            assert L == build_base(pipe)
+
+
+def test_budget_tail_survey_sequence():
+    """SURVEY d4 [derived]: S = 8, N = 32, budgets of 2 .. 7 activation sets."""
+    pipe, c, mem = Pipe(V_1F1B, 8, 32), UnitCosts(), MemUnits()
+    got = [simulate(pipe, pass5_budget(pipe, c, mem, b)[0], c).makespan for b in (2, 4, 7)]
+    assert got == [143, 137, 128]
+
+
+def test_budget_tail_picks_fastest_not_largest():
+    """Chimera S = 4, N = 8: un-checkpointing only the last device lengthens the schedule
+    (44 > 42), so with room for it the rule still keeps k = 0 (smallest makespan, ties to k)."""
+    pipe, c, mem = Pipe(X_CHIMERA, 4, 8), UnitCosts(), MemUnits()
+    L0 = transform(pipe, MARIO, c)
+    L, k = pass5_budget(pipe, c, mem, 3)
+    assert k == 0 and L == L0
+    L, k = pass5_budget(pipe, c, mem, 4)
+    assert k in (3, 4) and simulate(pipe, L, c).makespan == 38
+
+
+def test_budget_level_keeps_invariants_all_schemes():
+    c, mem = UnitCosts(F=0.5, B=1.0, R=0.5), MemUnits()
+    for pipe in (Pipe(V_1F1B, 4, 8), Pipe(W_INTERLEAVE, 4, 8, 2), Pipe(X_CHIMERA, 4, 8)):
+        for b in (1, 2, 4, 6, 12):
+            L = transform(pipe, MARIO_BUDGET, c, mem, b)
+            check_structure(pipe, L)
+            assert simulate(pipe, L, c) is not None
+            # never slower than the paper's passes when those fit
+            assert simulate(pipe, L, c).makespan <= simulate(pipe, transform(pipe, MARIO, c, mem, b), c).makespan

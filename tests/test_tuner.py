@@ -29,7 +29,7 @@ def test_oom_configs_score_zero_and_cfg5_picks_mario():
         assert (r["samples_per_s"] == 0.0) == (not r["feasible"])
         if r["level"] == "base":
             assert not r["feasible"]
-    assert best >= 0 and rows[best]["level"] == "mario" and rows[best]["feasible"]
+    assert best >= 0 and rows[best]["level"] in ("mario", "mario_budget") and rows[best]["feasible"]
 
 
 def test_lmbs_freed_memory_buys_a_larger_microbatch():
@@ -51,7 +51,7 @@ def test_lmbs_freed_memory_buys_a_larger_microbatch():
     win = rows[best]
     # the best feasible base configuration uses a smaller micro-batch than the winner
     feas_base = [r for r in rows if r["level"] == "base" and r["feasible"]]
-    assert win["level"] == "mario"
+    assert win["level"] in ("mario", "mario_budget")
     assert not feas_base or max(r["micro_batch"] for r in feas_base) < win["micro_batch"] or \
         max(r["samples_per_s"] for r in feas_base) < win["samples_per_s"]
     assert win["peak_bytes"] <= budget
@@ -60,3 +60,24 @@ def test_lmbs_freed_memory_buys_a_larger_microbatch():
 def test_tune_rejects_bad_arguments():
     with pytest.raises(api.MarioError):
         api.tune(synth.TINY_GPT, 0, 8)
+
+
+def test_budget_level_in_grid_never_worse_than_mario():
+    """With a budget, MARIO_LEVEL_BUDGET (reading A28) joins the grid; per grid point it is never
+    slower than plain Mario (k = 0 is one of its candidates) and always within the budget."""
+    budget = 20 * 10 ** 9
+    rows, best = api.tune(synth.GPT3_1P3B, 8, 128, mem_budget=budget)
+    key = lambda r: (r["scheme"], r["pp"], r["chunks"], r["dp"], r["micro_batch"])
+    mario = {key(r): r for r in rows if r["level"] == "mario"}
+    n = 0
+    for r in rows:
+        if r["level"] != "mario_budget" or not r["feasible"]:
+            continue
+        n += 1
+        assert r["peak_bytes"] <= budget
+        m = mario[key(r)]
+        if m["feasible"]:
+            assert r["makespan_ms"] <= m["makespan_ms"] + 1e-9
+    assert n > 0
+    _, b0 = api.tune(synth.GPT3_1P3B, 8, 128)
+    assert all(r["level"] != "mario_budget" for r in api.tune(synth.GPT3_1P3B, 8, 128)[0])
