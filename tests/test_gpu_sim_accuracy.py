@@ -1,0 +1,44 @@
+"""Simulator accuracy on one GPU (§6.6): the planner's simulated
+peak memory and its makespan from profiled per-instruction costs against the measured iteration.
+Full study: tools/sim_accuracy.py (profiles/r01_sim_accuracy.json)."""
+import pytest
+import torch
+
+import synth
+from paper_conf_ppopp_liultj25_b200 import api
+
+pytestmark = pytest.mark.gpu
+
+
+def test_single_device_memory_and_time_match_simulation():
+    torch.cuda.set_device(0)
+    cfg = synth.with_(synth.GPT3_1P3B, n_layers=4, micro_batch=2)
+    ctx = api.Context(0, 1, 0)
+    plan = api.Plan(cfg, 1, 4, "1f1b", "mario", dtype="bf16")
+    torch.cuda.synchronize()
+    torch.cuda.empty_cache()
+    free0 = torch.cuda.mem_get_info()[0]
+    w, g, ws = api.alloc_for(plan, 0)
+    w.normal_(0.0, 0.02)
+    tok = torch.from_numpy(synth.make_tokens(cfg, 4)).cuda()
+    ctx.run_iter(plan, w, tok, g, ws)
+    torch.cuda.synchronize()
+    used = free0 - torch.cuda.mem_get_info()[0]
+    sim_peak = plan.simulate().peak_bytes[0]
+    assert abs(sim_peak - used) / used < 0.03, (sim_peak, used)
+    e0, e1 = torch.cuda.Event(True), torch.cuda.Event(True)
+    e0.record()
+    ctx.run_iter(plan, w, tok, g, ws)
+    e1.record()
+    torch.cuda.synchronize()
+    t_meas = e0.elapsed_time(e1)
+    ctx.set_timing(True)
+    ctx.run_iter(plan, w, tok, g, ws)
+    ctx.set_timing(False)
+    a, b = ctx.last_timeline(0)
+    comp = [x for x in plan.instrs(0) if x[0] in ("FW", "CFW", "RC", "BW")]
+    fw = [t1 - t0 for (op, *_r), t0, t1 in zip(comp, a, b) if op in ("FW", "CFW")]
+    bw = [t1 - t0 for (op, *_r), t0, t1 in zip(comp, a, b) if op == "BW"]
+    costs = {"fw_ms": [sum(fw) / len(fw)], "bw_ms": [sum(bw) / len(bw)], "rc_ms": [sum(fw) / len(fw)]}
+    t_sim = api.Plan(cfg, 1, 4, "1f1b", "mario", dtype="bf16", costs=costs).simulate().makespan_ms
+    assert abs(t_sim - t_meas) / t_meas < 0.10, (t_sim, t_meas)
