@@ -39,6 +39,8 @@ def parse():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--level", default="mario", choices=["base", "ckpt", "mario"])
+    ap.add_argument("--dp", type=int, default=1,
+                    help="PP x DP: gpus = stages * dp; the global batch stays --micro micro-batches (strong)")
     ap.add_argument("--scheme", default="1f1b")
     ap.add_argument("--micro", type=int, default=32)
     ap.add_argument("--no-cpu-baseline", action="store_true")
@@ -110,8 +112,8 @@ def config_dict(cfg, args, gbs):
     return {"workload": "cfg2: GPT-3 1.3B, seq 2048, 1F1B+Mario, bf16 (BASELINE.json configs[1])",
             "model": "gpt3-1.3b", "layers": cfg.n_layers, "hidden": cfg.hidden, "heads": cfg.n_heads,
             "global_batch": gbs, "seq_len": cfg.seq_len, "micro_batch": cfg.micro_batch,
-            "microbatches": args.micro, "stages": args.gpus, "scheme": args.scheme, "level": args.level,
-            "parallelism": f"pp{args.gpus}",
+            "microbatches": args.micro, "stages": args.gpus // args.dp, "scheme": args.scheme, "level": args.level,
+            "parallelism": f"pp{args.gpus // args.dp}" + (f"xdp{args.dp}" if args.dp > 1 else ""),
             "l2": "no flush: every iteration streams >100 GB of weights/activations through HBM (>> 126 MB L2)"}
 
 
@@ -241,14 +243,17 @@ def main():
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
         dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     L = _lib.lib()
-    plan = api.Plan(cfg, world, args.micro, args.scheme, args.level, dtype="bf16")
-    ctx = api.Context(rank, world, local)
-    w = init_weights_device(plan, rank, torch)
-    pc, ws_bytes = plan.rank_layout(rank)
+    assert world % args.dp == 0 and args.micro % args.dp == 0, "--dp must divide --gpus and --micro"
+    S, rep, n_rep = world // args.dp, rank // (world // args.dp), args.micro // args.dp
+    stage = rank % S
+    plan = api.Plan(cfg, S, n_rep, args.scheme, args.level, dtype="bf16")
+    ctx = api.Context(rank, world, local, dp=args.dp)
+    w = init_weights_device(plan, stage, torch)          # replicas of a stage hold identical weights
+    pc, ws_bytes = plan.rank_layout(stage)
     grads = torch.zeros(pc, dtype=torch.float32, device="cuda")
     ws = torch.empty(ws_bytes, dtype=torch.uint8, device="cuda")
     stream = torch.cuda.current_stream()
-    tok_host = [synth.make_tokens(cfg, args.micro, iteration=i) for i in range(args.warmup + args.steps)]
+    tok_host = [synth.make_tokens(cfg, n_rep, iteration=i * args.dp + rep) for i in range(args.warmup + args.steps)]
     tok_dev = [torch.from_numpy(t).cuda() for t in tok_host]
     torch.cuda.synchronize()
 
@@ -305,7 +310,7 @@ def main():
             dist.all_reduce(t, op=dist.ReduceOp.MAX)
             dt = float(t.item())
         e2e = {"value": gbs / dt, "unit": UNIT, "h2d_bytes_per_step": int(tok_host[0].nbytes),
-               "d2h_bytes_per_step": 4 + 8 * args.micro}
+               "d2h_bytes_per_step": 4 + 8 * n_rep}
 
     # CUDA-graph replay of the same iteration (mario_set_graphs), timed separately: the headline
     # region above runs eager so that the per-kernel roofline is measured live inside it

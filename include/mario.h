@@ -90,7 +90,10 @@ typedef struct {
  * communicator (a < b), 2 = send on channel (a -> b, c) the message of (micro, part = sender
  * part), issued right after list instruction list_index, 3 = receive on channel (a -> b, c) at
  * list instruction list_index (part = receiver part), 4 = all-reduce of parameter a (count
- * floats) on pair (b, c), 5 = all-reduce of count fp64 loss partials on the world. */
+ * floats) on pair (b, c), 5 = all-reduce of count fp64 loss partials on the world,
+ * 6 = split the data-parallel communicator of stage a (b = replica, c = dp; collective over ALL
+ * ranks), 7 = average the rank's whole fp32 gradient buffer (count floats) over that
+ * communicator (the AR phase of Table 3; reading A29). Kinds 6/7 appear only for dp > 1. */
 typedef struct { int32_t kind, a, b, c, micro, part, list_index; int64_t count; } mario_commop;
 
 struct mario_plan;
@@ -118,6 +121,12 @@ mario_status mario_plan_timeline(const struct mario_plan* plan, int32_t device,
  * this adds no dependency) — required because pass 4 may move an SA ahead of an earlier
  * micro-batch's SA while NCCL channels are FIFO. Array owned by the plan. */
 mario_status mario_plan_comm_ops(const struct mario_plan* plan, int32_t rank, const mario_commop** ops, int32_t* n);
+/* PP x DP (reading A29): the program of world rank `rank` when world =
+ * stages * dp and rank = replica * stages + stage. Same as mario_plan_comm_ops(rank % stages) with
+ * every rank field offset into the replica's range, preceded by a kind-6 split and with a kind-7
+ * gradient average before the loss all-reduce. EINVAL unless 0 <= rank < stages * dp. */
+mario_status mario_plan_comm_ops_dp(const struct mario_plan* plan, int32_t dp, int32_t rank, const mario_commop** ops,
+                                    int32_t* n);
 /* Canonical text serialization (deterministic). If buf is NULL or cap too small, *needed
  * receives the size including the terminating NUL and MARIO_EINVAL is returned for cap>0. */
 mario_status mario_plan_serialize(const struct mario_plan* plan, char* buf, size_t cap, size_t* needed);
@@ -164,6 +173,11 @@ mario_status mario_tune(const mario_model* model, int32_t devices, int32_t globa
  * one process per GPU, nccl_unique_id = 128 bytes from mario_nccl_unique_id() on rank 0. */
 mario_status mario_nccl_unique_id(void* out128);
 mario_status mario_init(int32_t rank, int32_t world, int32_t device, const void* nccl_unique_id);
+/* PP x DP: world = stages * dp processes, rank = replica * stages + stage; every replica runs the
+ * same plan on its own micro-batches, gradients are averaged over the replicas of each stage
+ * (ncclAvg) after the pipeline flush and the loss is the mean over all replicas' tokens.
+ * mario_init(...) == mario_init_dp(..., dp = 1, ...). EINVAL if world % dp != 0. */
+mario_status mario_init_dp(int32_t rank, int32_t world, int32_t device, int32_t dp, const void* nccl_unique_id);
 /* One training iteration of `plan` on this rank (all ranks in loopback).
  *  weights : device, this rank's packed fp32 parameters (loopback: all ranks concatenated)
  *  tokens  : HOST int32 [N*mbs][s+1]; x = tokens[:, :s], y = tokens[:, 1:] (reading A4)

@@ -76,6 +76,8 @@ _lib.register("mario_plan_instrs", C.c_int32, [_P, C.c_int32, C.POINTER(C.POINTE
 _lib.register("mario_plan_simulate", C.c_int32, [_P, C.POINTER(CSim)])
 _lib.register("mario_plan_timeline", C.c_int32, [_P, C.c_int32, C.POINTER(C.POINTER(C.c_double)),
                                                  C.POINTER(C.POINTER(C.c_double)), C.POINTER(C.c_int32)])
+_lib.register("mario_plan_comm_ops_dp", C.c_int32, [_P, C.c_int32, C.c_int32, C.POINTER(C.POINTER(CCommOp)),
+                                                    C.POINTER(C.c_int32)])
 _lib.register("mario_plan_comm_ops", C.c_int32, [_P, C.c_int32, C.POINTER(C.POINTER(CCommOp)), C.POINTER(C.c_int32)])
 _lib.register("mario_plan_serialize", C.c_int32, [_P, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)])
 _lib.register("mario_plan_rank_layout", C.c_int32, [_P, C.c_int32, C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)])
@@ -91,6 +93,7 @@ _lib.register("mario_tune", C.c_int32, [C.POINTER(CModel), C.c_int32, C.c_int32,
                                         C.POINTER(CTuneResult), C.c_int32, C.POINTER(C.c_int32), C.POINTER(C.c_int32)])
 _lib.register("mario_nccl_unique_id", C.c_int32, [C.c_void_p])
 _lib.register("mario_init", C.c_int32, [C.c_int32, C.c_int32, C.c_int32, C.c_void_p])
+_lib.register("mario_init_dp", C.c_int32, [C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_void_p])
 _lib.register("mario_run_iter", C.c_int32, [_P, C.c_void_p, C.c_void_p, C.POINTER(C.c_float), C.c_void_p,
                                             C.c_void_p, C.c_void_p])
 _lib.register("mario_set_timing", C.c_int32, [C.c_int32])
@@ -199,6 +202,13 @@ class Plan:
         return [(p[i].kind, p[i].a, p[i].b, p[i].c, p[i].micro, p[i].part, p[i].list_index, p[i].count)
                 for i in range(n.value)]
 
+    def comm_ops_dp(self, rank: int, dp: int):
+        """World rank's program under PP x DP (world = S * dp; mario_plan_comm_ops_dp)."""
+        p, n = C.POINTER(CCommOp)(), C.c_int32()
+        _check(_lib.lib().mario_plan_comm_ops_dp(self.handle, dp, rank, C.byref(p), C.byref(n)))
+        return [(p[i].kind, p[i].a, p[i].b, p[i].c, p[i].micro, p[i].part, p[i].list_index, p[i].count)
+                for i in range(n.value)]
+
     def serialize(self) -> str:
         need = C.c_size_t()
         _check(_lib.lib().mario_plan_serialize(self.handle, None, 0, C.byref(need)))
@@ -262,10 +272,11 @@ def _shapes(plan: Plan):
 
 
 class Context:
-    """mario_init(rank, world, device, nccl_id). world > 1 uses torch.distributed (already
-    initialised) only to broadcast the 128-byte NCCL unique id."""
+    """mario_init_dp(rank, world, device, dp, nccl_id). world > 1 uses torch.distributed (already
+    initialised) only to broadcast the 128-byte NCCL unique id. dp > 1: PP x DP, world = S * dp,
+    rank = replica * S + stage (reading A29)."""
 
-    def __init__(self, rank: int = 0, world: int = 1, device: int = 0):
+    def __init__(self, rank: int = 0, world: int = 1, device: int = 0, dp: int = 1):
         L = _lib.lib()
         uid = C.create_string_buffer(128)
         if world > 1:
@@ -276,8 +287,8 @@ class Context:
             t = torch.tensor(list(uid.raw), dtype=torch.uint8)
             dist.broadcast(t, src=0)
             uid = C.create_string_buffer(bytes(t.tolist()), 128)
-        _check(L.mario_init(rank, world, device, uid if world > 1 else None))
-        self.rank, self.world = rank, world
+        _check(L.mario_init_dp(rank, world, device, dp, uid if world > 1 else None))
+        self.rank, self.world, self.dp = rank, world, dp
 
     def run_iter(self, plan: Plan, weights, tokens, grads, workspace, stream=None) -> float:
         """weights/grads/workspace: device tensors (data_ptr used); tokens: host int32 array."""

@@ -238,6 +238,38 @@ void build_comm_program(PlanObj& P) {
   }
 }
 
+}  // namespace
+
+// PP x DP (reading A29): world = S * dp, world rank = replica * S + stage. The stage
+// program of `rank % S` with every rank field moved into the replica's rank range; splits stay
+// collective over all ranks (one call per split op, each replica gets its own communicator);
+// kind 6 splits the data-parallel communicator of the stage (a = stage, b = replica, c = dp),
+// kind 7 averages the rank's gradient buffer (count floats) over it, after the pair all-reduces
+// and before the loss all-reduce.
+const std::vector<mario_commop>& comm_program_dp(const PlanObj& P, int dp, int rank) {
+  const int S = P.pp.S;
+  auto key = std::make_pair(dp, rank);
+  auto it = P.comm_ops_dp.find(key);
+  if (it != P.comm_ops_dp.end()) return it->second;
+  const int st = rank % S, rep = rank / S, off = rep * S;
+  std::vector<mario_commop> out;
+  if (dp > 1) out.push_back({6, st, rep, dp, -1, -1, -1, 0});
+  for (mario_commop op : P.comm_ops[st]) {
+    switch (op.kind) {
+      case 0: case 2: case 3: op.a += off; op.b += off; break;
+      case 1: op.a += off; op.b += off; break;
+      case 4: op.b += off; op.c += off; break;
+      default: break;
+    }
+    if (op.kind == 5 && dp > 1)
+      out.push_back({7, st, rep, dp, -1, -1, -1, static_cast<int64_t>(P.rank_params[st].total)});
+    out.push_back(op);
+  }
+  return P.comm_ops_dp[key] = out;
+}
+
+namespace {
+
 std::string serialize(const PlanObj& P) {
   std::string s;
   char buf[512];
@@ -397,6 +429,15 @@ extern "C" mario_status mario_plan_timeline(const struct mario_plan* P, int32_t 
   *start = P->sim.start[device].data();
   *finish = P->sim.finish[device].data();
   *n = static_cast<int32_t>(P->sim.start[device].size());
+  return MARIO_OK;
+}
+
+extern "C" mario_status mario_plan_comm_ops_dp(const struct mario_plan* P, int32_t dp, int32_t rank,
+                                              const mario_commop** ops, int32_t* n) {
+  if (!P || !ops || !n || dp < 1 || rank < 0 || rank >= P->pp.S * dp) return set_error(MARIO_EINVAL, "bad argument");
+  const auto& v = comm_program_dp(*P, dp, rank);
+  *ops = v.data();
+  *n = static_cast<int32_t>(v.size());
   return MARIO_OK;
 }
 

@@ -63,8 +63,10 @@ struct Channel {
 
 struct Context {
   int rank = 0, world = 1, device = 0;
+  int dp = 1;                         // data-parallel replicas: world = stages * dp (reading A29)
   bool inited = false;
   ncclComm_t world_comm = nullptr;
+  ncclComm_t dp_comm = nullptr;       // this stage's replicas (kind 6 split)
   std::map<std::tuple<int, int, int>, Channel> channels;   // (src, dst, kind)
   std::map<std::pair<int, int>, ncclComm_t> pair_comms;      // (lo, hi) 2-rank comms
   std::set<std::tuple<int, int, int>> created_channels;       // split already done (all ranks)
@@ -544,16 +546,20 @@ struct Exec {
 // Create per-channel 2-rank communicators for every (src, dst, kind) the plan uses, plus the
 // pair communicators for gradient synchronisation. Collective over all ranks: every rank
 // iterates the same sorted set.
+// With PP x DP every split op is issued by all ranks of all replicas; each replica's members pass
+// their replica as the colour, so one call creates one communicator per replica. Channels and
+// pairs are stored in stage space (the replica offset removed).
 void ensure_channels(const PlanObj& P) {
-  for (const mario_commop& op : P.comm_ops[g.rank]) {
+  const int S = P.pp.S, off = (g.rank / S) * S, color = 1 + g.rank / S;
+  for (const mario_commop& op : comm_program_dp(P, g.dp, g.rank)) {
     if (op.kind == 0) {
-      const auto c = std::make_tuple(op.a, op.b, op.c);
+      const auto c = std::make_tuple(op.a - off, op.b - off, op.c);
       if (g.created_channels.count(c)) continue;
       g.created_channels.insert(c);
       const int lo = std::min(op.a, op.b), hi = std::max(op.a, op.b);
       const bool member = g.rank == lo || g.rank == hi;
       ncclComm_t comm = nullptr;
-      NC(ncclCommSplit(g.world_comm, member ? 1 : NCCL_SPLIT_NOCOLOR, g.rank == lo ? 0 : 1, &comm, nullptr));
+      NC(ncclCommSplit(g.world_comm, member ? color : NCCL_SPLIT_NOCOLOR, g.rank == lo ? 0 : 1, &comm, nullptr));
       if (member) {
         Channel ch;
         ch.comm = comm;
@@ -561,13 +567,15 @@ void ensure_channels(const PlanObj& P) {
         g.channels[c] = ch;
       }
     } else if (op.kind == 1) {
-      const auto pr = std::make_pair(op.a, op.b);
+      const auto pr = std::make_pair(op.a - off, op.b - off);
       if (g.created_pairs.count(pr)) continue;
       g.created_pairs.insert(pr);
       const bool member = g.rank == op.a || g.rank == op.b;
       ncclComm_t comm = nullptr;
-      NC(ncclCommSplit(g.world_comm, member ? 1 : NCCL_SPLIT_NOCOLOR, g.rank == op.a ? 0 : 1, &comm, nullptr));
+      NC(ncclCommSplit(g.world_comm, member ? color : NCCL_SPLIT_NOCOLOR, g.rank == op.a ? 0 : 1, &comm, nullptr));
       if (member) g.pair_comms[pr] = comm;
+    } else if (op.kind == 6 && !g.dp_comm) {
+      NC(ncclCommSplit(g.world_comm, op.a, op.b, &g.dp_comm, nullptr));   // colour = stage, key = replica
     }
   }
 }
@@ -576,7 +584,9 @@ template <class T>
 mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* tokens, float* loss, void* grads,
                         void* workspace, cudaStream_t st) {
   const bool loopback = g.world == 1 && P.pp.S > 1;
-  if (!loopback && P.pp.S != g.world) return set_error(MARIO_ESTATE, "plan stages != world size");
+  if (!loopback && P.pp.S * g.dp != g.world) return set_error(MARIO_ESTATE, "plan stages * dp != world size");
+  const int me = g.rank % P.pp.S, off = g.rank - me;   // stage and the replica's rank offset
+  const auto& prog = comm_program_dp(P, g.dp, g.rank);
   Exec<T> E;
   E.st = st;
   E.loopback = loopback;
@@ -584,7 +594,7 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
   const int S = P.pp.S;
   std::vector<int> my_devs;
   if (loopback) for (int d = 0; d < S; ++d) my_devs.push_back(d);
-  else my_devs.push_back(g.rank);
+  else my_devs.push_back(me);
   size_t wofs = 0, wsofs = 0;
   for (int d : my_devs) {
     auto D = std::make_unique<Dev<T>>();
@@ -618,7 +628,7 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
     CU(cudaMemcpyAsync(D->ws + D->a.tokens, tokens, tok_bytes, cudaMemcpyDefault, st));   // host or device tokens
     E.devs.push_back(std::move(D));
   }
-  if (!loopback && S > 1) ensure_channels(P);
+  if (!loopback && g.world > 1) ensure_channels(P);
 
   // Single-process iterations are a fixed launch sequence over fixed buffers: the second call
   // with the same (plan, weights, grads, workspace) is captured into a CUDA graph, later calls
@@ -663,13 +673,13 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
   if (loopback) {
     for (auto [d, i] : P.loopback_order) E.run_instr(d, P.instrs[d][i]);
   } else {
-    const auto& L = P.instrs[g.rank];
-    std::vector<std::vector<const mario_commop*>> sends_after(L.size());
-    for (const mario_commop& op : P.comm_ops[g.rank])
-      if (op.kind == 2) sends_after[op.list_index].push_back(&op);
+    const auto& L = P.instrs[me];
+    std::vector<std::vector<mario_commop>> sends_after(L.size());
+    for (mario_commop op : prog)
+      if (op.kind == 2) { op.a -= off; op.b -= off; sends_after[op.list_index].push_back(op); }   // stage space
     for (size_t i = 0; i < L.size(); ++i) {
-      E.run_instr(g.rank, L[i]);
-      for (const mario_commop* op : sends_after[i]) E.issue_send(*E.devs[0], *op);
+      E.run_instr(me, L[i]);
+      for (const mario_commop& op : sends_after[i]) E.issue_send(*E.devs[0], op);
     }
     // the iteration ends when every channel stream has drained (its last sends complete)
     for (auto& kv : g.channels) {
@@ -695,33 +705,37 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
       for (size_t c = 1; c < kv.second.size(); ++c) add_f32(acc, ptr(kv.second[c]), n, E.st);
       for (size_t c = 1; c < kv.second.size(); ++c) copy_f32(ptr(kv.second[c]), acc, n, E.st);
     }
-  } else if (S > 1) {
+  } else if (S > 1 || g.dp > 1) {
     Dev<T>& D = *E.devs[0];
     // local duplicates first (e.g. Chimera rank 0 holds the tied wte twice)
     for (auto& kv : copies) {
       std::vector<int> mine;
-      for (auto& c : kv.second) if (c.first == g.rank) mine.push_back(c.second);
+      for (auto& c : kv.second) if (c.first == me) mine.push_back(c.second);
       for (size_t c = 1; c < mine.size(); ++c)
-        add_f32(D.gr + P.rank_params[g.rank].off[mine[0]], D.gr + P.rank_params[g.rank].off[mine[c]],
-                P.rank_params[g.rank].cnt[mine[0]], st);
+        add_f32(D.gr + P.rank_params[me].off[mine[0]], D.gr + P.rank_params[me].off[mine[c]],
+                P.rank_params[me].cnt[mine[0]], st);
     }
     // then pairwise all-reduce with the other holder, in the comm program's (global) order
     NC(ncclGroupStart());
-    for (const mario_commop& op : P.comm_ops[g.rank]) {
+    for (const mario_commop& op : prog) {
       if (op.kind != 4) continue;
       int j0 = -1;
-      for (auto& c : copies[op.a]) if (c.first == g.rank) { j0 = c.second; break; }
-      float* buf = D.gr + P.rank_params[g.rank].off[j0];
-      NC(ncclAllReduce(buf, buf, static_cast<size_t>(op.count), ncclFloat32, ncclSum, g.pair_comms[{op.b, op.c}], st));
+      for (auto& c : copies[op.a]) if (c.first == me) { j0 = c.second; break; }
+      float* buf = D.gr + P.rank_params[me].off[j0];
+      NC(ncclAllReduce(buf, buf, static_cast<size_t>(op.count), ncclFloat32, ncclSum,
+                       g.pair_comms[{op.b - off, op.c - off}], st));
     }
     NC(ncclGroupEnd());
     for (auto& kv : copies) {
       std::vector<int> mine;
-      for (auto& c : kv.second) if (c.first == g.rank) mine.push_back(c.second);
+      for (auto& c : kv.second) if (c.first == me) mine.push_back(c.second);
       for (size_t c = 1; c < mine.size(); ++c)
-        copy_f32(D.gr + P.rank_params[g.rank].off[mine[c]], D.gr + P.rank_params[g.rank].off[mine[0]],
-                 P.rank_params[g.rank].cnt[mine[0]], st);
+        copy_f32(D.gr + P.rank_params[me].off[mine[c]], D.gr + P.rank_params[me].off[mine[0]],
+                 P.rank_params[me].cnt[mine[0]], st);
     }
+    // AR (Table 3; reading A29): average the whole gradient buffer over the stage's replicas
+    for (const mario_commop& op : prog)
+      if (op.kind == 7) NC(ncclAllReduce(D.gr, D.gr, static_cast<size_t>(op.count), ncclFloat32, ncclAvg, g.dp_comm, st));
   }
 
   }   // !replayed
@@ -755,8 +769,8 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
     CU(cudaStreamSynchronize(st));
     for (int i = 0; i < P.pp.N; ++i) sums[i] += h[i];
   }
-  if (!loopback && S > 1) {
-    // share the last stage(s)' per-micro-batch sums with every rank
+  if (!loopback && g.world > 1) {
+    // share the last stage(s)' per-micro-batch sums with every rank (summed over replicas too)
     double* dbuf = reinterpret_cast<double*>(E.devs[0]->ws + E.devs[0]->a.loss);
     CU(cudaMemcpyAsync(dbuf, sums.data(), P.pp.N * 8, cudaMemcpyHostToDevice, st));
     NC(ncclAllReduce(dbuf, dbuf, P.pp.N, ncclFloat64, ncclSum, g.world_comm, st));
@@ -765,7 +779,7 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
   CU(cudaStreamSynchronize(st));
   double total = 0.0;
   for (int i = 0; i < P.pp.N; ++i) total += sums[i];
-  const double ntok = static_cast<double>(P.pp.N) * tokens_per_micro(m);
+  const double ntok = static_cast<double>(P.pp.N) * tokens_per_micro(m) * (loopback ? 1 : g.dp);
   if (loss) *loss = static_cast<float>(total / ntok);
 
   // timeline export
@@ -807,12 +821,14 @@ extern "C" mario_status mario_nccl_unique_id(void* out128) {
   return MARIO_OK;
 }
 
-extern "C" mario_status mario_init(int32_t rank, int32_t world, int32_t device, const void* nccl_unique_id) {
+extern "C" mario_status mario_init_dp(int32_t rank, int32_t world, int32_t device, int32_t dp,
+                                      const void* nccl_unique_id) {
   try {
     if (world < 1 || rank < 0 || rank >= world) return set_error(MARIO_EINVAL, "bad rank/world");
+    if (dp < 1 || world % dp) return set_error(MARIO_EINVAL, "world % dp != 0");
     if (g.inited) return set_error(MARIO_ESTATE, "already initialised");
     CU(cudaSetDevice(device));
-    g.rank = rank; g.world = world; g.device = device;
+    g.rank = rank; g.world = world; g.device = device; g.dp = dp;
     if (world > 1) {
       if (!nccl_unique_id) return set_error(MARIO_EINVAL, "NULL nccl id");
       ncclUniqueId id;
@@ -827,6 +843,10 @@ extern "C" mario_status mario_init(int32_t rank, int32_t world, int32_t device, 
   } catch (const NcclErr& e) {
     return set_error(MARIO_ENCCL, e.what());
   }
+}
+
+extern "C" mario_status mario_init(int32_t rank, int32_t world, int32_t device, const void* nccl_unique_id) {
+  return mario_init_dp(rank, world, device, 1, nccl_unique_id);
 }
 
 extern "C" mario_status mario_run_iter(const struct mario_plan* plan, const void* weights, const int32_t* tokens,
@@ -910,8 +930,11 @@ extern "C" mario_status mario_finalize(void) {
   for (auto& kv : g.graph_cache) cudaGraphExecDestroy(kv.second);
   g.graph_cache.clear();
   g.graph_seen.clear();
+  if (g.dp_comm) ncclCommDestroy(g.dp_comm);
+  g.dp_comm = nullptr;
   if (g.world_comm) ncclCommDestroy(g.world_comm);
   g.world_comm = nullptr;
+  g.dp = 1;
   g.inited = false;
   g.sticky = false;
   return MARIO_OK;

@@ -1,6 +1,7 @@
 // The opaque mario_plan object (immutable after mario_plan returns).
 #pragma once
 #include <string>
+#include <map>
 #include <vector>
 
 #include "model.h"
@@ -40,5 +41,8 @@ struct mario_plan {
   std::vector<std::pair<int, int>> loopback_order;
   std::string serialized;
   std::vector<std::vector<mario_commop>> comm_ops;   // per rank, issue order
+  // world-rank programs for PP x DP (key: (dp, world rank)), built on first use
+  mutable std::map<std::pair<int, int>, std::vector<mario_commop>> comm_ops_dp;
 };
 typedef struct mario_plan PlanObj;
+const std::vector<mario_commop>& comm_program_dp(const PlanObj& P, int dp, int rank);   // plan_api.cpp
