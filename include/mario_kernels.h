@@ -75,12 +75,15 @@ int mario_k_norm_bwd(const void* dy, const void* x, const float* stats, const fl
 int mario_k_norm_set_variant(int v);
 
 /* Instrumentation. mario_kernel_launches: number of kernels this library has launched since it
- * was loaded (every call above and every mario_run_iter kernel). mario_kstats_enable(1) clears
- * and starts CUDA-event timing of every GEMM (kind 0), attention forward (1) and backward (2)
- * launch on its own stream; mario_kstats_read sums durations (ms), algorithmic FLOPs and bytes
- * and counts launches of one kind (synchronizes on the recorded events). Returns 0 / -1. */
+ * was loaded (every call above and every mario_run_iter kernel). mario_kstats_enable(mask) clears
+ * the records and starts CUDA-event timing, on the launching stream, of every launch of the kinds
+ * whose bit is set (bit k = kind k: 0 GEMM, 1 attention forward, 2 attention backward, 4 norms,
+ * 5 column sums, 6 softmax-CE, 7 elementwise, 8 embedding; -1 = all; 0 = off). Each timed launch
+ * costs two event records, so time only what you need inside a measured region.
+ * mario_kstats_read sums durations (ms), algorithmic FLOPs and bytes and counts launches of one
+ * kind (synchronizes on the recorded events). Returns 0 / -1. */
 long long mario_kernel_launches(void);
-int mario_kstats_enable(int on);
+int mario_kstats_enable(int mask);
 int mario_kstats_read(int kind, double* total_ms, double* flops, double* bytes, long long* launches);
 
 #ifdef __cplusplus

@@ -322,6 +322,19 @@ class Context:
         _lib.lib().mario_finalize()
 
 
+_DEFAULT_CTX = []
+
+
+def default_context(device: int = 0) -> "Context":
+    """The process's single-GPU context (rank 0 of world 1), created on first use. The library
+    holds one executor context per process, so every single-process caller shares this one."""
+    if not _DEFAULT_CTX:
+        import torch
+        torch.cuda.set_device(device)
+        _DEFAULT_CTX.append(Context(0, 1, device))
+    return _DEFAULT_CTX[0]
+
+
 def alloc_for(plan: Plan, rank: int, device="cuda"):
     """Allocate (weights, grads, workspace) device tensors sized from the plan (torch is
     used only as the device allocator)."""

@@ -10,6 +10,7 @@ namespace mario {
 namespace {
 std::atomic<long long> g_launches{0};
 bool g_on = false;
+unsigned g_mask = 0;   // bit k: time kind k
 struct Rec { int kind; double flops, bytes; cudaEvent_t a, b; };
 std::vector<Rec> g_recs;
 std::mutex g_mu;
@@ -19,7 +20,7 @@ void note_launch(int n) { g_launches.fetch_add(n, std::memory_order_relaxed); }
 bool kstats_on() { return g_on; }
 
 int kstats_begin(KKind kind, double flops, double bytes, cudaStream_t st) {
-  if (!g_on) return -1;
+  if (!g_on || !((g_mask >> kind) & 1u)) return -1;
   std::lock_guard<std::mutex> lk(g_mu);
   Rec r{kind, flops, bytes, nullptr, nullptr};
   cudaEventCreate(&r.a);
@@ -40,11 +41,12 @@ using namespace mario;
 
 extern "C" long long mario_kernel_launches(void) { return g_launches.load(); }
 
-extern "C" int mario_kstats_enable(int on) {
+extern "C" int mario_kstats_enable(int mask) {
   std::lock_guard<std::mutex> lk(g_mu);
   for (auto& r : g_recs) { cudaEventDestroy(r.a); cudaEventDestroy(r.b); }
   g_recs.clear();
-  g_on = on != 0;
+  g_mask = static_cast<unsigned>(mask);
+  g_on = mask != 0;
   return 0;
 }
 

@@ -12,14 +12,8 @@ from paper_conf_ppopp_liultj25_b200 import api
 
 pytestmark = pytest.mark.gpu
 
-_CTX = {}
-
-
 def ctx():
-    if "c" not in _CTX:
-        torch.cuda.set_device(0)
-        _CTX["c"] = api.Context(0, 1, 0)
-    return _CTX["c"]
+    return api.default_context()
 
 
 def run_plan(cfg, S, N, scheme, level, dtype, params, toks, chunks=1, mem_budget=0, costs=None):

@@ -13,7 +13,7 @@ pytestmark = pytest.mark.gpu
 def test_single_device_memory_and_time_match_simulation():
     torch.cuda.set_device(0)
     cfg = synth.with_(synth.GPT3_1P3B, n_layers=4, micro_batch=2)
-    ctx = api.Context(0, 1, 0)
+    ctx = api.default_context()
     plan = api.Plan(cfg, 1, 4, "1f1b", "mario", dtype="bf16")
     torch.cuda.synchronize()
     torch.cuda.empty_cache()
