@@ -49,8 +49,10 @@ int mario_k_gemm_f32(const float* A, int lda, int a_mn, const float* B, int ldb,
  * (head_dim in {16,32,64,80,128}), else fp32. */
 int mario_k_attn_fwd(const void* qkv, void* O, float* lse, int B, int s, int n_heads, int head_dim,
                      int bf16, void* stream);
-/* Kernel selection for K5/K6 (bf16): -1 = auto (tcgen05 backward for head_dim 64/128, mma.sync
- * otherwise), 0 = mma.sync only. Process-global; returns 0, or 1 for an invalid value. */
+/* Kernel selection for K5/K6 (bf16): -1 = auto (tcgen05 for head_dim 64/128: the two-Q-tile
+ * forward when it fills the GPU, else the one-Q-tile forward; mma.sync otherwise), 0 = mma.sync
+ * only, 2 / 3 = tcgen05 with the one- / two-Q-tile forward forced. Process-global; returns 0, or 1
+ * for an invalid value. */
 int mario_k_attn_set_variant(int variant);
 /* K6: backward: dqkv [B*s][3*H] (dQ | dK | dV) from dO [B*s][H], with P recomputed from lse;
  * deterministic (no atomics). scratch: fp32 [n_heads][B*s]. */

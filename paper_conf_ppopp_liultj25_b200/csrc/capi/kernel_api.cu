@@ -32,7 +32,7 @@ extern "C" int mario_k_gemm_bf16(const void* A, int lda, int a_mn, const void* B
 }
 
 extern "C" int mario_k_attn_set_variant(int variant) {
-  if (variant < -1 || variant > 1) return 1;
+  if (variant < -1 || variant > 3) return 1;
   g_attn_variant = variant;
   return 0;
 }

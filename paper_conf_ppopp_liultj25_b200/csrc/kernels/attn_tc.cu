@@ -26,6 +26,7 @@
 
 namespace mario {
 
+extern int g_attn_variant;   // attn_mma.cu
 bool make_tmap_bf16_2d(CUtensorMap* map, const void* base, uint64_t inner, uint64_t outer, uint64_t ld,
                        uint32_t box_inner, uint32_t box_outer);   // gemm_tc.cu
 
@@ -36,6 +37,22 @@ constexpr float LOG2E = 1.4426950408889634f;
 constexpr int kRows = 128;   // rows per CTA (TMEM lanes)
 constexpr int kCols = 64;    // inner tile
 constexpr int kThreads = 192;
+
+// 2^x on the SFU: one MUFU.EX2 (flush-to-zero; P underflowing to 0 instead of a subnormal is
+// harmless) instead of exp2f's range fix-up (FSETP/FSEL/FMUL around the MUFU)
+__device__ __forceinline__ float ex2(float x) {
+  float y;
+  asm("ex2.approx.ftz.f32 %0, %1;" : "=f"(y) : "f"(x));
+  return y;
+}
+__device__ __forceinline__ void st_shared_f32(const void* p, float v) {
+  asm volatile("st.shared.f32 [%0], %1;" :: "r"(static_cast<uint32_t>(__cvta_generic_to_shared(p))), "f"(v) : "memory");
+}
+__device__ __forceinline__ float ld_shared_f32(const void* p) {
+  float v;
+  asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(static_cast<uint32_t>(__cvta_generic_to_shared(p))) : "memory");
+  return v;
+}
 
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void named_bar(int id, int n) { asm volatile("bar.sync %0, %1;" :: "r"(id), "r"(n) : "memory"); }
@@ -232,14 +249,26 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
       __syncwarp();
       if (lane == 0) mbar_arrive(&s_free[buf]);
       float p[32], ds[32];
+      // only tiles crossing the diagonal (queries < this block's last key) or the sequence end mask
+      const bool edge = i * kCols < kt * kRows + kRows || i * kCols + kCols > s;
+      if (edge) {
 #pragma unroll
-      for (int c = 0; c < 32; ++c) {
-        const int cc = half * 32 + c;
-        const int qq = i * kCols + cc;
-        float pv = exp2f(__uint_as_float(sr[c]) * sl2 - sL[buf * kCols + cc]);
-        if (qq < key || qq >= s) pv = 0.f;
-        p[c] = pv;
-        ds[c] = pv * (__uint_as_float(dr[c]) - sDv[buf * kCols + cc]);
+        for (int c = 0; c < 32; ++c) {
+          const int cc = half * 32 + c;
+          const int qq = i * kCols + cc;
+          float pv = ex2(__uint_as_float(sr[c]) * sl2 - sL[buf * kCols + cc]);
+          if (qq < key || qq >= s) pv = 0.f;
+          p[c] = pv;
+          ds[c] = pv * (__uint_as_float(dr[c]) - sDv[buf * kCols + cc]);
+        }
+      } else {
+#pragma unroll
+        for (int c = 0; c < 32; ++c) {
+          const int cc = half * 32 + c;
+          const float pv = ex2(__uint_as_float(sr[c]) * sl2 - sL[buf * kCols + cc]);
+          p[c] = pv;
+          ds[c] = pv * (__uint_as_float(dr[c]) - sDv[buf * kCols + cc]);
+        }
       }
       mbar_wait(p_free, (idx & 1) ^ 1);   // previous tile's dV/dK MMAs have consumed sP/sS
       st_half_row_sw128(sP, row, 4 * half, p);
@@ -425,12 +454,20 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
       __syncwarp();
       if (lane == 0) mbar_arrive(&s_free[buf]);
       float ds[32];
+      if (idx * kCols + kCols - 1 > qt * kRows) {   // tile crosses the diagonal: causal mask
 #pragma unroll
-      for (int c = 0; c < 32; ++c) {
-        const int key = idx * kCols + half * 32 + c;
-        float pv = exp2f(__uint_as_float(sr[c]) * sl2 - L);
-        if (key > q) pv = 0.f;
-        ds[c] = pv * (__uint_as_float(dr[c]) - Dr);
+        for (int c = 0; c < 32; ++c) {
+          const int key = idx * kCols + half * 32 + c;
+          float pv = ex2(__uint_as_float(sr[c]) * sl2 - L);
+          if (key > q) pv = 0.f;
+          ds[c] = pv * (__uint_as_float(dr[c]) - Dr);
+        }
+      } else {
+#pragma unroll
+        for (int c = 0; c < 32; ++c) {
+          const float pv = ex2(__uint_as_float(sr[c]) * sl2 - L);
+          ds[c] = pv * (__uint_as_float(dr[c]) - Dr);
+        }
       }
       mbar_wait(p_free, (idx & 1) ^ 1);
       st_half_row_sw128(sS, row, 4 * half, ds);
@@ -635,7 +672,7 @@ fa_fwd_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__
       const int st = j & 1;
       mbar_wait(&o_full[st], (j >> 1) & 1);
       tc_fence_after();
-      const float c = exp2f(m_before - m_j);
+      const float c = ex2(m_before - m_j);
 #pragma unroll
       for (int c0 = 0; c0 < HD; c0 += 32) {
         uint32_t r[32];
@@ -659,26 +696,32 @@ fa_fwd_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__
       tc_fence_before();
       __syncwarp();
       if (lane == 0) mbar_arrive(&s_free[st]);
-      float mx = m_run;
+      // max over the raw scores (sl2 > 0), masked to -inf only on tiles crossing the diagonal;
+      // then p = 2^(s * sl2 - m) as one FFMA + one MUFU per element
+      float mr = -INFINITY;
+      if (j * kCols + kCols - 1 > qt * kRows) {
 #pragma unroll
-      for (int c = 0; c < 32; ++c) {
-        const int key = j * kCols + half * 32 + c;
-        float x = __uint_as_float(sr[c]) * sl2;
-        if (key > q) x = -INFINITY;
-        sr[c] = __float_as_uint(x);
-        mx = fmaxf(mx, x);
+        for (int c = 0; c < 32; ++c) {
+          const int key = j * kCols + half * 32 + c;
+          if (key > q) sr[c] = __float_as_uint(-INFINITY);
+          mr = fmaxf(mr, __uint_as_float(sr[c]));
+        }
+      } else {
+#pragma unroll
+        for (int c = 0; c < 32; ++c) mr = fmaxf(mr, __uint_as_float(sr[c]));
       }
-      xch[half * kRows + row] = mx;
+      const float mx = fmaxf(m_run, mr * sl2);
+      st_shared_f32(&xch[half * kRows + row], mx);
       named_bar(2 + quarter, 64);
-      const float m_new = fmaxf(mx, xch[(half ^ 1) * kRows + row]);   // finite: key 0 <= q
-      named_bar(2 + quarter, 64);                                     // xch reusable next tile
+      const float m_new = fmaxf(mx, ld_shared_f32(&xch[(half ^ 1) * kRows + row]));   // finite: key 0 <= q
+      named_bar(2 + quarter, 64);                                                      // xch reusable next tile
       float p[32], ls = 0.f;
 #pragma unroll
       for (int c = 0; c < 32; ++c) {
-        p[c] = exp2f(__uint_as_float(sr[c]) - m_new);
+        p[c] = ex2(fmaf(__uint_as_float(sr[c]), sl2, -m_new));
         ls += p[c];
       }
-      l_run = l_run * exp2f(m_run - m_new) + ls;
+      l_run = l_run * ex2(m_run - m_new) + ls;
       m_run = m_new;
       st_half_row_sw128(sP[st], row, 4 * half, p);
       fence_proxy_async();
@@ -692,9 +735,9 @@ fa_fwd_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__
     }
     fold(ntiles - 1, m_pending, m_folded);
     // total row sum = both halves' partial sums (same running max)
-    xch[half * kRows + row] = l_run;
+    st_shared_f32(&xch[half * kRows + row], l_run);
     named_bar(2 + quarter, 64);
-    const float l_tot = l_run + xch[(half ^ 1) * kRows + row];
+    const float l_tot = l_run + ld_shared_f32(&xch[(half ^ 1) * kRows + row]);
     const float inv = 1.f / l_tot;
     if (q < s) {
       bf16* orow = O + (static_cast<long>(b) * s + q) * h + head * DH + half * HD;
@@ -712,6 +755,283 @@ fa_fwd_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__
   tc_fence_before();
   __syncthreads();
   if (warp == 1) tmem_dealloc<512>(tm);
+}
+
+// ------------------------------------------------------------- forward, two Q tiles
+// fa_fwd2_tc: one CTA = 256 queries (Q tiles t = 0, 1 of 128 rows) of one (sample, head); keys in
+// tiles of 128. Warpgroup 0: warp 0 TMA, warp 1 MMA (one elected thread), warps 2-3 idle; it
+// gives registers away (setmaxnreg 56) to warpgroups 1 and 2 (224), the softmax of Q tile 0 and 1
+// (one thread per query row, the whole 128-key S row in registers: no cross-thread max exchange). TMEM: S_0, S_1 (128 columns each), O_0, O_1 (DH each). The MMA
+// warp interleaves the two tiles (S_0(j+1), S_1(j+1), PV_0(j), PV_1(j)) so one tile's softmax
+// overlaps the other's MMAs. O accumulates in TMEM; the running max is only raised (and O, l
+// rescaled in TMEM) when a row's max grows by more than 2^8 (warp-uniform decision), so most tiles
+// need no correction. K/V tiles stream through a 3-slot TMA ring in the MMA's consumption order
+// K0, K1, V0, K2, V1, ..., V_{n-1}. Causal: Q tile 0 of query block qb sees key tiles 0..2qb,
+// tile 1 sees 0..2qb+1; only the last (diagonal) tile of each is masked.
+constexpr int kF2Q = 128;        // rows per Q tile
+constexpr int kF2N = 128;        // keys per tile
+constexpr int kF2Threads = 384;
+constexpr int kF2Stages = 3;
+
+template <int DH>
+struct SmemF2 {
+  static constexpr int kTile = kF2Q * DH * 2;       // a Q, K or V tile (bf16)
+  static constexpr int kP = kF2Q * kF2N * 2;        // P tile (bf16)
+  static constexpr int kBytes = 2 * kTile + kF2Stages * kTile + 2 * kP + 256 + 1024;
+};
+
+// which tile the i-th ring item is (load order == MMA consumption order)
+__device__ __forceinline__ void f2_item(int i, int n, bool& is_v, int& j) {
+  if (i == 0) { is_v = false; j = 0; return; }
+  if (i == 2 * n - 1) { is_v = true; j = n - 1; return; }
+  const int t = (i + 1) >> 1;       // i = 2t - 1 -> K_t, i = 2t -> V_{t-1}
+  if (i & 1) { is_v = false; j = t; } else { is_v = true; j = t - 1; }
+}
+
+template <int DH>
+__global__ void __launch_bounds__(kF2Threads, 1)
+fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, int B, int s, int nh) {
+  using SM = SmemF2<DH>;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sQ = smem;                                   // [2][kTile]
+  uint8_t* sRing = sQ + 2 * SM::kTile;                  // [kF2Stages][kTile]
+  uint8_t* sP = sRing + kF2Stages * SM::kTile;          // [2][kP]
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sP + 2 * SM::kP);
+  uint64_t* q_full = bar;                          // 1
+  uint64_t* full = bar + 1;                        // kF2Stages
+  uint64_t* empty = full + kF2Stages;              // kF2Stages
+  uint64_t* s_full = empty + kF2Stages;            // 2
+  uint64_t* s_free = s_full + 2;                   // 2
+  uint64_t* p_full = s_free + 2;                   // 2
+  uint64_t* o_done = p_full + 2;                   // 2
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(o_done + 2);
+
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int BH = B * nh, nqb = (s + 2 * kF2Q - 1) / (2 * kF2Q);
+  const int qb = nqb - 1 - static_cast<int>(blockIdx.x) / BH;   // heaviest query blocks first
+  const int bh = static_cast<int>(blockIdx.x) % BH, b = bh / nh, head = bh % nh;
+  const int h = nh * DH;
+  const long Ttok = static_cast<long>(B) * s;
+  const int q0 = qb * 2 * kF2Q;
+  const int n0 = 2 * qb + 1, n1 = 2 * qb + 2;      // key tiles seen by Q tile 0 / 1
+  const float sl2 = rsqrtf(static_cast<float>(DH)) * LOG2E;
+
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&tm_qkv128);
+    mbar_init(q_full, 1);
+    for (int i = 0; i < kF2Stages; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
+    for (int t = 0; t < 2; ++t) {
+      mbar_init(&s_full[t], 1); mbar_init(&s_free[t], 4); mbar_init(&p_full[t], 4); mbar_init(&o_done[t], 1);
+    }
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc<512>(tmem_slot);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tm = *tmem_slot;
+  const uint32_t tm_S0 = tm, tm_O0 = tm + 2 * kF2N;
+
+  if (warp < 4) {
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");
+  if (warp == 0) {
+    if (elect_one()) {
+      const int row0 = b * s;
+      mbar_arrive_expect_tx(q_full, 2 * SM::kTile);
+#pragma unroll
+      for (int t = 0; t < 2; ++t)
+#pragma unroll
+        for (int a = 0; a < DH / 64; ++a)
+          tma_load_2d(sQ + t * SM::kTile + a * (kF2Q * 128), &tm_qkv128, q_full, head * DH + a * 64,
+                      row0 + q0 + t * kF2Q);
+      for (int i = 0; i < 2 * n1; ++i) {
+        bool is_v;
+        int j;
+        f2_item(i, n1, is_v, j);
+        const int st = i % kF2Stages;
+        mbar_wait(&empty[st], ((i / kF2Stages) & 1) ^ 1);
+        mbar_arrive_expect_tx(&full[st], SM::kTile);
+        uint8_t* dst = sRing + st * SM::kTile;
+#pragma unroll
+        for (int a = 0; a < DH / 64; ++a)
+          tma_load_2d(dst + a * (kF2N * 128), &tm_qkv128, &full[st], (is_v ? 2 * h : h) + head * DH + a * 64,
+                      row0 + j * kF2N);
+      }
+    }
+  } else if (warp == 1) {
+    constexpr uint32_t id_s = umma_idesc_bf16(kF2Q, kF2N, 0, 0);
+    constexpr uint32_t id_o = umma_idesc_bf16(kF2Q, DH, 0, 1);   // B = V read MN-major
+    mbar_wait(q_full, 0);
+    tc_fence_after();
+    int item = 0;
+    auto issue_s = [&](int j) {
+      const int st = item % kF2Stages;
+      mbar_wait(&full[st], (item / kF2Stages) & 1);
+      for (int t = 0; t < 2; ++t) {
+        if (t == 0 && j >= n0) continue;
+        mbar_wait(&s_free[t], (j & 1) ^ 1);
+        tc_fence_after();
+        if (elect_one()) {
+          const uint32_t q = smem_u32(sQ + t * SM::kTile), k = smem_u32(sRing + st * SM::kTile);
+#pragma unroll
+          for (int kk = 0; kk < DH / 16; ++kk) {
+            const uint32_t ao = (kk >> 2) * (kF2Q * 128) + (kk & 3) * 32, bo = (kk >> 2) * (kF2N * 128) + (kk & 3) * 32;
+            umma_bf16(tm_S0 + t * kF2N, umma_desc_sw128(q + ao, 16, 1024), umma_desc_sw128(k + bo, 16, 1024), id_s,
+                      kk > 0);
+          }
+          umma_commit(&s_full[t]);
+        }
+        __syncwarp();
+      }
+      if (elect_one()) umma_commit(&empty[st]);
+      __syncwarp();
+      ++item;
+    };
+    auto issue_pv = [&](int j) {
+      const int st = item % kF2Stages;
+      mbar_wait(&full[st], (item / kF2Stages) & 1);
+      for (int t = 0; t < 2; ++t) {
+        if (t == 0 && j >= n0) continue;
+        mbar_wait(&p_full[t], j & 1);
+        tc_fence_after();
+        if (elect_one()) {
+          const uint32_t p = smem_u32(sP + t * SM::kP), v = smem_u32(sRing + st * SM::kTile);
+#pragma unroll
+          for (int kk = 0; kk < kF2N / 16; ++kk) {
+            const uint32_t ao = (kk >> 2) * (kF2Q * 128) + (kk & 3) * 32;
+            umma_bf16(tm_O0 + t * DH, umma_desc_sw128(p + ao, 16, 1024),
+                      umma_desc_sw128(v + kk * 2048, kF2N * 128, 1024), id_o, (j | kk) != 0);
+          }
+          umma_commit(&o_done[t]);
+        }
+        __syncwarp();
+      }
+      if (elect_one()) umma_commit(&empty[st]);
+      __syncwarp();
+      ++item;
+    };
+    issue_s(0);
+    for (int j = 0; j < n1; ++j) {
+      if (j + 1 < n1) issue_s(j + 1);
+      issue_pv(j);
+    }
+  }
+  } else {
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 224;");
+    const int t = (warp - 4) >> 2, quarter = warp & 3;
+    const int row = quarter * 32 + lane;
+    const int q = q0 + t * kF2Q + row;
+    const int nt = t == 0 ? n0 : n1;
+    const uint32_t lane_off = static_cast<uint32_t>(quarter * 32) << 16;
+    const uint32_t tS = tm_S0 + t * kF2N + lane_off, tO = tm_O0 + t * DH + lane_off;
+    uint8_t* myP = sP + t * SM::kP;
+    float m_used = -INFINITY, l = 0.f;
+    for (int j = 0; j < nt; ++j) {
+      mbar_wait(&s_full[t], j & 1);
+      tc_fence_after();
+      uint32_t xr[kF2N];
+#pragma unroll
+      for (int c0 = 0; c0 < kF2N; c0 += 32) tmem_ld_32x32b_x32(tS + c0, *reinterpret_cast<uint32_t(*)[32]>(&xr[c0]));
+      tmem_ld_wait();
+      float* x = reinterpret_cast<float*>(xr);
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&s_free[t]);   // S_t may be overwritten by the next tile's MMA
+      if (j == nt - 1) {                         // diagonal tile: causal mask
+#pragma unroll
+        for (int c = 0; c < kF2N; ++c)
+          if (j * kF2N + c > q) x[c] = -INFINITY;
+      }
+      float mr = x[0];
+#pragma unroll
+      for (int c = 1; c < kF2N; ++c) mr = fmaxf(mr, x[c]);
+      const float m_cand = mr * sl2;
+      bool waited = false;
+      if (j == 0) {
+        m_used = m_cand;                          // finite: key 0 <= q
+      } else if (__any_sync(0xffffffffu, m_cand > m_used + 8.f)) {
+        // raise the running max: O_t (after PV_t(j-1)) and l rescaled by 2^(m_old - m_new)
+        mbar_wait(&o_done[t], (j - 1) & 1);
+        tc_fence_after();
+        waited = true;
+        const float m_new = fmaxf(m_used, m_cand);
+        const float f = ex2(m_used - m_new);
+        l *= f;
+        m_used = m_new;
+#pragma unroll 1
+        for (int c0 = 0; c0 < DH; c0 += 32) {
+          uint32_t r[32];
+          tmem_ld_32x32b_x32(tO + c0, r);
+          tmem_ld_wait();
+#pragma unroll
+          for (int e = 0; e < 32; ++e) r[e] = __float_as_uint(__uint_as_float(r[e]) * f);
+          tmem_st_32x32b_x32(tO + c0, r);
+        }
+        tmem_st_wait();
+      }
+      float ls = 0.f;
+#pragma unroll
+      for (int c = 0; c < kF2N; ++c) {
+        x[c] = ex2(fmaf(x[c], sl2, -m_used));
+        ls += x[c];
+      }
+      l += ls;
+      if (j > 0 && !waited) {                     // P_t smem is free once PV_t(j-1) completed
+        mbar_wait(&o_done[t], (j - 1) & 1);
+      }
+#pragma unroll
+      for (int c0 = 0; c0 < kF2N; c0 += 32)
+        st_half_row_sw128(myP + (c0 / 64) * (kF2Q * 128), row, (c0 % 64) / 8, *reinterpret_cast<float(*)[32]>(&x[c0]));
+      fence_proxy_async();
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&p_full[t]);
+    }
+    mbar_wait(&o_done[t], (nt - 1) & 1);
+    tc_fence_after();
+    const float inv = 1.f / l;
+    bf16* orow = O + (static_cast<long>(b) * s + (q < s ? q : 0)) * h + head * DH;
+#pragma unroll 1
+    for (int c0 = 0; c0 < DH; c0 += 32) {
+      uint32_t r[32];
+      tmem_ld_32x32b_x32(tO + c0, r);
+      tmem_ld_wait();
+      if (q < s) {
+#pragma unroll
+        for (int d = 0; d < 32; d += 8) {
+          uint4 u;
+          __nv_bfloat162* hh = reinterpret_cast<__nv_bfloat162*>(&u);
+#pragma unroll
+          for (int e = 0; e < 4; ++e)
+            hh[e] = __floats2bfloat162_rn(__uint_as_float(r[d + 2 * e]) * inv, __uint_as_float(r[d + 2 * e + 1]) * inv);
+          *reinterpret_cast<uint4*>(orow + c0 + d) = u;
+        }
+      }
+    }
+    if (q < s) lse[static_cast<long>(head) * Ttok + static_cast<long>(b) * s + q] = (m_used + log2f(l)) / LOG2E;
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) tmem_dealloc<512>(tm);
+}
+
+template <int DH>
+bool launch_fwd2_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, cudaStream_t st) {
+  const int h = nh * DH;
+  const long T = static_cast<long>(B) * s;
+  CUtensorMap m128;
+  if (!make_tmap_bf16_2d(&m128, qkv, 3 * h, T, 3 * h, 64, 128)) return false;
+  constexpr int smem = SmemF2<DH>::kBytes < 116 * 1024 ? 116 * 1024 : SmemF2<DH>::kBytes;
+  static bool set = false;
+  if (!set) {
+    cudaFuncSetAttribute(fa_fwd2_tc<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    set = true;
+  }
+  const int nqb = (s + 2 * kF2Q - 1) / (2 * kF2Q);
+  fa_fwd2_tc<DH><<<nqb * B * nh, kF2Threads, smem, st>>>(m128, O, lse, B, s, nh);
+  note_launch();
+  return true;
 }
 
 template <int DH>
@@ -742,8 +1062,22 @@ bool flash_attn_bwd_tc_supported(int dh, int B, int s, int nh) {
 }
 
 bool flash_attn_fwd_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st) {
-  if (dh == 128) return launch_fwd_tc<128>(qkv, O, lse, B, s, nh, st);
-  if (dh == 64) return launch_fwd_tc<64>(qkv, O, lse, B, s, nh, st);
+  // g_attn_variant: -1 auto (two-Q-tile kernel unless it would launch fewer CTAs than SMs: the
+  // one-Q-tile kernel has twice as many), 2 force the one-Q-tile kernel, 3 force the two-Q-tile one
+  int sms = 148;
+  {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  }
+  const long ctas2 = static_cast<long>((s + 2 * kF2Q - 1) / (2 * kF2Q)) * B * nh;
+  if (g_attn_variant == 2 || (g_attn_variant != 3 && ctas2 < sms)) {
+    if (dh == 128) return launch_fwd_tc<128>(qkv, O, lse, B, s, nh, st);
+    if (dh == 64) return launch_fwd_tc<64>(qkv, O, lse, B, s, nh, st);
+    return false;
+  }
+  if (dh == 128) return launch_fwd2_tc<128>(qkv, O, lse, B, s, nh, st);
+  if (dh == 64) return launch_fwd2_tc<64>(qkv, O, lse, B, s, nh, st);
   return false;
 }
 

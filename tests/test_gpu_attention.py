@@ -23,7 +23,7 @@ def _ref(qkv, B, s, nh, dh, dO):
     return o.permute(0, 2, 1, 3).reshape(B * s, h), lse.permute(1, 0, 2).reshape(nh, B * s), dqkv
 
 
-@pytest.fixture(params=[-1, 0], ids=["auto_tcgen05", "mma_sync"])
+@pytest.fixture(params=[-1, 2, 3, 0], ids=["auto_tcgen05", "tcgen05_1q", "tcgen05_2q", "mma_sync"])
 def attn_variant(request):
     L = _lib.lib()
     assert L.mario_k_attn_set_variant(request.param) == 0
