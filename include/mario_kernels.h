@@ -83,7 +83,10 @@ int mario_k_norm_set_variant(int v);
  * 5 column sums, 6 softmax-CE, 7 elementwise, 8 embedding; -1 = all; 0 = off). Each timed launch
  * costs two event records, so time only what you need inside a measured region.
  * mario_kstats_read sums durations (ms), algorithmic FLOPs and bytes and counts launches of one
- * kind (synchronizes on the recorded events). Returns 0 / -1. */
+ * kind (synchronizes on the recorded events). Launches captured into a CUDA graph (mario_set_graphs)
+ * re-record their events on every replay: when such records exist only they are read, i.e. the
+ * latest replay. Each mario_kstats_enable invalidates captured iterations (the next call
+ * re-captures). Returns 0 / -1. */
 long long mario_kernel_launches(void);
 int mario_kstats_enable(int mask);
 int mario_kstats_read(int kind, double* total_ms, double* flops, double* bytes, long long* launches);

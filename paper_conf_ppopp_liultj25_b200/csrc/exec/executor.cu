@@ -77,9 +77,12 @@ struct Context {
   // CUDA-graph replay of whole iterations (single-process: S = 1 or loopback)
   bool graphs = false;
   cudaStream_t cap_stream = nullptr;
-  std::map<std::tuple<const void*, const void*, const void*, const void*>, cudaGraphExec_t> graph_cache;
-  std::map<std::tuple<const void*, const void*, const void*, const void*>, long long> graph_kernels;
-  std::set<std::tuple<const void*, const void*, const void*, const void*>> graph_seen;
+  // key: (plan, weights, grads, workspace, kstats generation) — event-timed launches captured in a
+  // graph re-record their events on every replay, so a new timing set needs a new capture
+  using GKey = std::tuple<const void*, const void*, const void*, const void*, long long>;
+  std::map<GKey, cudaGraphExec_t> graph_cache;
+  std::map<GKey, long long> graph_kernels;
+  std::set<GKey> graph_seen;
   bool sticky = false;
 };
 Context g;
@@ -633,9 +636,9 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
   // Single-process iterations are a fixed launch sequence over fixed buffers: the second call
   // with the same (plan, weights, grads, workspace) is captured into a CUDA graph, later calls
   // replay it (no per-kernel launch cost). Disabled while timing/kstats instrumentation is on.
-  const bool graphable = g.graphs && g.world == 1 && !g.timing && !kstats_on();
+  const bool graphable = g.graphs && g.world == 1 && !g.timing;
   const auto gkey = std::make_tuple(static_cast<const void*>(&P), weights, static_cast<const void*>(grads),
-                                    static_cast<const void*>(workspace));
+                                    static_cast<const void*>(workspace), kstats_generation());
   bool replayed = false, capturing = false;
   if (graphable) {
     if (!g.cap_stream) CU(cudaStreamCreateWithFlags(&g.cap_stream, cudaStreamNonBlocking));

@@ -84,7 +84,8 @@ __device__ __forceinline__ void st_half_row_sw128(uint8_t* tile, int row, int c0
 }
 
 constexpr int kThreadsB = 320;
-constexpr int kRing = 4;   // depth of the streamed-operand TMA ring (K/V or Q/dO tiles)   // backward: TMA, MMA, 8 softmax warps (2 per TMEM lane quarter)
+constexpr int kRing = 4;     // depth of the streamed-operand TMA ring (K/V or Q/dO tiles)
+constexpr int kRingKV = 3;   // dK/dV kernel: 3 Q/dO stages leave room for double-buffered P^T / dS^T
 
 template <int DH>
 struct Smem {
@@ -104,22 +105,27 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sK = smem;
   uint8_t* sV = sK + SM::kBig;
-  uint8_t* sQ[kRing];
-  uint8_t* sG[kRing];
-  for (int r = 0; r < kRing; ++r) { sQ[r] = sV + SM::kBig + 2 * r * SM::kSmall; sG[r] = sQ[r] + SM::kSmall; }
-  uint8_t* sP = sV + SM::kBig + 2 * kRing * SM::kSmall;
-  uint8_t* sS = sP + SM::kP;    // dS^T
-  float* sL = reinterpret_cast<float*>(sS + SM::kP);       // [2][64] lse * log2e
+  uint8_t* sQ[kRingKV];
+  uint8_t* sG[kRingKV];
+  for (int r = 0; r < kRingKV; ++r) { sQ[r] = sV + SM::kBig + 2 * r * SM::kSmall; sG[r] = sQ[r] + SM::kSmall; }
+  // P^T and dS^T double-buffered: tile idx + 1 is written while the dV/dK MMAs read tile idx
+  uint8_t* sP[2];
+  uint8_t* sS[2];
+  for (int i = 0; i < 2; ++i) {
+    sP[i] = sV + SM::kBig + 2 * kRingKV * SM::kSmall + 2 * i * SM::kP;
+    sS[i] = sP[i] + SM::kP;
+  }
+  float* sL = reinterpret_cast<float*>(sS[1] + SM::kP);    // [2][64] lse * log2e
   float* sDv = sL + 2 * kCols;                             // [2][64] D
   uint64_t* bar = reinterpret_cast<uint64_t*>(sDv + 2 * kCols);
   uint64_t* kv_full = bar;                 // 1
-  uint64_t* q_full = bar + 1;              // kRing
-  uint64_t* q_empty = q_full + kRing;      // kRing
-  uint64_t* s_full = q_empty + kRing;      // 2
+  uint64_t* q_full = bar + 1;              // kRingKV
+  uint64_t* q_empty = q_full + kRingKV;    // kRingKV
+  uint64_t* s_full = q_empty + kRingKV;    // 2
   uint64_t* s_free = s_full + 2;           // 2
-  uint64_t* p_full = s_free + 2;           // 1
-  uint64_t* p_free = p_full + 1;           // 1
-  uint64_t* acc_done = p_free + 1;         // 1
+  uint64_t* p_full = s_free + 2;           // 2
+  uint64_t* p_free = p_full + 2;           // 2
+  uint64_t* acc_done = p_free + 2;         // 1
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_done + 1);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
@@ -136,10 +142,10 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
     tma_prefetch_desc(&tm_qkv64);
     tma_prefetch_desc(&tm_do64);
     mbar_init(kv_full, 1);
-    for (int i = 0; i < kRing; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); }
-    for (int i = 0; i < 2; ++i) { mbar_init(&s_full[i], 1); mbar_init(&s_free[i], 8); }
-    mbar_init(p_full, 8);
-    mbar_init(p_free, 1);
+    for (int i = 0; i < kRingKV; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); }
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&s_full[i], 1); mbar_init(&s_free[i], 8); mbar_init(&p_full[i], 8); mbar_init(&p_free[i], 1);
+    }
     mbar_init(acc_done, 1);
     fence_barrier_init();
   }
@@ -166,8 +172,8 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
         tma_load_2d(sV + a * (kRows * 128), &tm_qkv128, kv_full, 2 * h + head * DH + a * 64, row0 + kt * kRows);
       }
       for (int idx = 0; idx < ntiles; ++idx) {
-        const int st = idx % kRing;
-        mbar_wait(&q_empty[st], ((idx / kRing) & 1) ^ 1);
+        const int st = idx % kRingKV;
+        mbar_wait(&q_empty[st], ((idx / kRingKV) & 1) ^ 1);
         mbar_arrive_expect_tx(&q_full[st], 2 * SM::kSmall);
         const int qr = row0 + (i0 + idx) * kCols;
 #pragma unroll
@@ -183,8 +189,8 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
     mbar_wait(kv_full, 0);
     tc_fence_after();
     auto issue_s = [&](int idx) {
-      const int st = idx % kRing, buf = idx & 1;
-      mbar_wait(&q_full[st], (idx / kRing) & 1);
+      const int st = idx % kRingKV, buf = idx & 1;
+      mbar_wait(&q_full[st], (idx / kRingKV) & 1);
       mbar_wait(&s_free[buf], ((idx >> 1) & 1) ^ 1);
       tc_fence_after();
       if (elect_one()) {
@@ -200,18 +206,18 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
       __syncwarp();
     };
     auto issue_acc = [&](int idx) {
-      const int st = idx % kRing;
-      mbar_wait(p_full, idx & 1);
+      const int st = idx % kRingKV, pb = idx & 1;
+      mbar_wait(&p_full[pb], (idx >> 1) & 1);
       tc_fence_after();
       if (elect_one()) {
-        const uint32_t p = smem_u32(sP), ds = smem_u32(sS), q = smem_u32(sQ[st]), g = smem_u32(sG[st]);
+        const uint32_t p = smem_u32(sP[pb]), ds = smem_u32(sS[pb]), q = smem_u32(sQ[st]), g = smem_u32(sG[st]);
 #pragma unroll
         for (int kk = 0; kk < kCols / 16; ++kk) {
           const uint64_t pa = umma_desc_sw128(p + kk * 32, 16, 1024), sa = umma_desc_sw128(ds + kk * 32, 16, 1024);
           umma_bf16(tm_dV, pa, umma_desc_sw128(g + kk * 2048, kCols * 128, 1024), id_a, (idx | kk) != 0);
           umma_bf16(tm_dK, sa, umma_desc_sw128(q + kk * 2048, kCols * 128, 1024), id_a, (idx | kk) != 0);
         }
-        umma_commit(p_free);
+        umma_commit(&p_free[pb]);
         umma_commit(&q_empty[st]);
         if (idx == ntiles - 1) umma_commit(acc_done);
       }
@@ -270,12 +276,12 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
           ds[c] = pv * (__uint_as_float(dr[c]) - sDv[buf * kCols + cc]);
         }
       }
-      mbar_wait(p_free, (idx & 1) ^ 1);   // previous tile's dV/dK MMAs have consumed sP/sS
-      st_half_row_sw128(sP, row, 4 * half, p);
-      st_half_row_sw128(sS, row, 4 * half, ds);
+      mbar_wait(&p_free[buf], ((idx >> 1) & 1) ^ 1);   // the dV/dK MMAs of tile idx-2 consumed this buffer
+      st_half_row_sw128(sP[buf], row, 4 * half, p);
+      st_half_row_sw128(sS[buf], row, 4 * half, ds);
       fence_proxy_async();
       __syncwarp();
-      if (lane == 0) mbar_arrive(p_full);
+      if (lane == 0) mbar_arrive(&p_full[buf]);
     }
     if (half == 1) goto done_dkdv;   // the epilogue uses one warp per lane quarter
     // epilogue: dV, dK rows of this thread's key
@@ -330,16 +336,17 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
   uint8_t* sK[kRing];
   uint8_t* sV[kRing];
   for (int r = 0; r < kRing; ++r) { sK[r] = sG + SM::kBig + 2 * r * SM::kSmall; sV[r] = sK[r] + SM::kSmall; }
-  uint8_t* sS = sG + SM::kBig + 2 * kRing * SM::kSmall;   // dS [128 q][64 keys]
-  uint64_t* bar = reinterpret_cast<uint64_t*>(sS + SM::kP);
+  uint8_t* sS[2] = {sG + SM::kBig + 2 * kRing * SM::kSmall,               // dS [128 q][64 keys],
+                    sG + SM::kBig + 2 * kRing * SM::kSmall + SM::kP};     // double-buffered
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sS[1] + SM::kP);
   uint64_t* q_fullb = bar;                // Q, dO loaded
   uint64_t* k_full = bar + 1;             // kRing
   uint64_t* k_empty = k_full + kRing;     // kRing
   uint64_t* s_full = k_empty + kRing;     // 2
   uint64_t* s_free = s_full + 2;          // 2
-  uint64_t* p_full = s_free + 2;
-  uint64_t* p_free = p_full + 1;
-  uint64_t* acc_done = p_free + 1;
+  uint64_t* p_full = s_free + 2;          // 2
+  uint64_t* p_free = p_full + 2;          // 2
+  uint64_t* acc_done = p_free + 2;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_done + 1);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
@@ -357,8 +364,7 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
     mbar_init(q_fullb, 1);
     for (int i = 0; i < kRing; ++i) { mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1); }
     for (int i = 0; i < 2; ++i) { mbar_init(&s_full[i], 1); mbar_init(&s_free[i], 8); }
-    mbar_init(p_full, 8);
-    mbar_init(p_free, 1);
+    for (int i = 0; i < 2; ++i) { mbar_init(&p_full[i], 8); mbar_init(&p_free[i], 1); }
     mbar_init(acc_done, 1);
     fence_barrier_init();
   }
@@ -413,16 +419,16 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
       __syncwarp();
     };
     auto issue_acc = [&](int idx) {
-      const int st = idx % kRing;
-      mbar_wait(p_full, idx & 1);
+      const int st = idx % kRing, pb = idx & 1;
+      mbar_wait(&p_full[pb], (idx >> 1) & 1);
       tc_fence_after();
       if (elect_one()) {
-        const uint32_t ds = smem_u32(sS), k = smem_u32(sK[st]);
+        const uint32_t ds = smem_u32(sS[pb]), k = smem_u32(sK[st]);
 #pragma unroll
         for (int kk = 0; kk < kCols / 16; ++kk)
           umma_bf16(tm_dQ, umma_desc_sw128(ds + kk * 32, 16, 1024), umma_desc_sw128(k + kk * 2048, kCols * 128, 1024),
                     id_a, (idx | kk) != 0);
-        umma_commit(p_free);
+        umma_commit(&p_free[pb]);
         umma_commit(&k_empty[st]);
         if (idx == ntiles - 1) umma_commit(acc_done);
       }
@@ -469,11 +475,11 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
           ds[c] = pv * (__uint_as_float(dr[c]) - Dr);
         }
       }
-      mbar_wait(p_free, (idx & 1) ^ 1);
-      st_half_row_sw128(sS, row, 4 * half, ds);
+      mbar_wait(&p_free[buf], ((idx >> 1) & 1) ^ 1);
+      st_half_row_sw128(sS[buf], row, 4 * half, ds);
       fence_proxy_async();
       __syncwarp();
-      if (lane == 0) mbar_arrive(p_full);
+      if (lane == 0) mbar_arrive(&p_full[buf]);
     }
     if (half == 1) goto done_dq;
     mbar_wait(acc_done, 0);
@@ -507,9 +513,9 @@ done_dq:
 // >= 116 KB so that one CTA owns the SM (each allocates all 512 TMEM columns)
 constexpr int at_least_one_sm(int b) { return b < 116 * 1024 ? 116 * 1024 : b; }
 template <int DH>
-constexpr int smem_dkdv() { return at_least_one_sm(2 * Smem<DH>::kBig + 2 * kRing * Smem<DH>::kSmall + 2 * Smem<DH>::kP + 4 * kCols * 4 + 256 + 1024); }
+constexpr int smem_dkdv() { return at_least_one_sm(2 * Smem<DH>::kBig + 2 * kRingKV * Smem<DH>::kSmall + 4 * Smem<DH>::kP + 4 * kCols * 4 + 256 + 1024); }
 template <int DH>
-constexpr int smem_dq() { return at_least_one_sm(2 * Smem<DH>::kBig + 2 * kRing * Smem<DH>::kSmall + Smem<DH>::kP + 256 + 1024); }
+constexpr int smem_dq() { return at_least_one_sm(2 * Smem<DH>::kBig + 2 * kRing * Smem<DH>::kSmall + 2 * Smem<DH>::kP + 256 + 1024); }
 
 template <int DH>
 bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, bf16* dqkv, int B, int s, int nh,

@@ -9,6 +9,7 @@ enum KKind { K_GEMM = 0, K_ATTN_FWD = 1, K_ATTN_BWD = 2, K_OTHER = 3, K_NORM = 4
 
 void note_launch(int n = 1);
 bool kstats_on();
+long long kstats_generation();   // bumped by every mario_kstats_enable (invalidates captured graphs)
 // returns a token to pass to kstats_end (or -1 when disabled)
 int kstats_begin(KKind kind, double flops, double bytes, cudaStream_t st);
 void kstats_end(int token, cudaStream_t st);
