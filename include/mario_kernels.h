@@ -72,9 +72,20 @@ int mario_k_norm_fwd(const void* x, const float* g, const float* b, void* y, flo
 int mario_k_norm_bwd(const void* dy, const void* x, const float* stats, const float* g, const void* dres,
                      void* dx, float* dg, float* db, float* dsum, float* partial, long long partial_floats,
                      int rows, int n, int rms, int bf16, void* stream);
-/* 1: block-per-row-tile backward with fused column sums (default); 0: warp-per-row backward +
- * separate column-sum passes. (The forward always uses the warp-per-row kernels.) */
+/* Kernel variant for both directions (bf16): 2 (default): row-pipelined persistent kernels — each CTA
+ * streams its contiguous row range through a ring of shared-memory stages filled by cp.async.bulk,
+ * column sums reduced per CTA and finished by a fixed-order pass; 1: block-per-row-tile backward
+ * with fused column sums + warp-per-row forward; 0: warp-per-row kernels + separate column-sum
+ * passes. Widths the selected variant does not tile fall back to the next one. */
 int mario_k_norm_set_variant(int v);
+
+/* K13: softmax cross-entropy of one micro-batch (readings A4/A21): logits fp32
+ * [rows][V] (rows = B * s, device), tokens int32 [B][ld_tok] (device; labels y = tokens[b][t + 1]).
+ * row_loss[r] = logsumexp(logits[r]) - logits[r][y] (fp32, device); dlogits [rows][V] =
+ * (softmax(logits[r]) - onehot(y)) * inv_ntok, bf16 (bf16 = 1) or fp32. bf16 with V % 4 == 0 and
+ * V <= 51200 uses the register-resident one-read kernel. Returns a cudaError_t value. */
+int mario_k_softmax_ce(const float* logits, const int* tokens, int ld_tok, int s, int rows, int V, float inv_ntok,
+                       void* dlogits, float* row_loss, int bf16, void* stream);
 
 /* Instrumentation. mario_kernel_launches: number of kernels this library has launched since it
  * was loaded (every call above and every mario_run_iter kernel). mario_kstats_enable(mask) clears

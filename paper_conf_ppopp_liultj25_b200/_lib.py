@@ -24,6 +24,7 @@ _SIGS = {
     "mario_k_norm_fwd": (i32, [vp, vp, vp, vp, vp, i32, i32, f32, i32, i32, vp]),
     "mario_k_norm_bwd": (i32, [vp, vp, vp, vp, vp, vp, vp, vp, vp, vp, C.c_longlong, i32, i32, i32, i32, vp]),
     "mario_k_norm_set_variant": (i32, [i32]),
+    "mario_k_softmax_ce": (i32, [vp, vp, i32, i32, i32, i32, f32, vp, vp, i32, vp]),
     "mario_kernel_launches": (C.c_longlong, []),
     "mario_k_gemm_set_variant": (i32, [i32]),
     "mario_k_attn_set_variant": (i32, [i32]),

@@ -105,7 +105,18 @@ extern "C" int mario_k_norm_bwd(const void* dy, const void* x, const float* stat
 }
 
 extern "C" int mario_k_norm_set_variant(int v) {
-  if (v < 0 || v > 1) return static_cast<int>(cudaErrorInvalidValue);
+  if (v < 0 || v > 2) return static_cast<int>(cudaErrorInvalidValue);
   g_norm_tile = v;
   return 0;
+}
+
+extern "C" int mario_k_softmax_ce(const float* logits, const int* tokens, int ld_tok, int s, int rows, int V,
+                                  float inv_ntok, void* dlogits, float* row_loss, int bf16, void* stream) {
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  if (!logits || !tokens || !dlogits || !row_loss || s <= 0 || V <= 0 || ld_tok < s + 1)
+    return static_cast<int>(cudaErrorInvalidValue);
+  if (bf16) softmax_ce<__nv_bfloat16>(logits, tokens, ld_tok, s, rows, V, inv_ntok,
+                                      static_cast<__nv_bfloat16*>(dlogits), row_loss, st);
+  else softmax_ce<float>(logits, tokens, ld_tok, s, rows, V, inv_ntok, static_cast<float*>(dlogits), row_loss, st);
+  return static_cast<int>(cudaGetLastError());
 }

@@ -203,6 +203,33 @@ __global__ void fa_bwd_dot_k(const bf16* O, const bf16* dO, float* Dd, long Ttok
   if (lane == 0) Dd[static_cast<long>(head) * Ttok + r] = acc;
 }
 
+// D = rowsum(dO * O) with 16-byte loads: G = dh / 8 lanes per (token, head) (G a power of two)
+template <int G>
+__global__ void fa_bwd_dot_v8_k(const bf16* O, const bf16* dO, float* Dd, long Ttok, int nh) {
+  const long gi = static_cast<long>(blockIdx.x) * blockDim.x + threadIdx.x;
+  const long pair = gi / G;                 // (token, head), head fastest
+  const int sub = static_cast<int>(gi % G);
+  const bool ok = pair < Ttok * nh;
+  const int head = static_cast<int>(pair % nh);
+  const long r = pair / nh;
+  const int dh = G * 8, h = nh * dh;
+  float acc = 0.f;
+  if (ok) {
+    const long off = r * h + head * dh + sub * 8;
+    const uint4 a = *reinterpret_cast<const uint4*>(O + off), b = *reinterpret_cast<const uint4*>(dO + off);
+    const __nv_bfloat162* ha = reinterpret_cast<const __nv_bfloat162*>(&a);
+    const __nv_bfloat162* hb = reinterpret_cast<const __nv_bfloat162*>(&b);
+#pragma unroll
+    for (int i = 0; i < 4; ++i) {
+      const float2 x = __bfloat1622float2(ha[i]), y = __bfloat1622float2(hb[i]);
+      acc += x.x * y.x + x.y * y.y;
+    }
+  }
+#pragma unroll
+  for (int o = G / 2; o > 0; o >>= 1) acc += __shfl_xor_sync(0xffffffffu, acc, o);
+  if (ok && sub == 0) Dd[static_cast<long>(head) * Ttok + r] = acc;
+}
+
 // ---------------------------------------------------- backward: dK, dV per key tile
 template <int D>
 __global__ void __launch_bounds__(128) fa_bwd_dkdv_k(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd,
@@ -439,7 +466,15 @@ template <int D>
 void launch_bwd(const bf16* qkv, const bf16* O, const bf16* dO, const float* lse, bf16* dqkv, float* Dd, int B, int s,
                 int nh, cudaStream_t st) {
   const long Ttok = static_cast<long>(B) * s;
-  fa_bwd_dot_k<<<static_cast<int>((Ttok * nh * 32 + 255) / 256), 256, 0, st>>>(O, dO, Dd, Ttok, nh, D);
+  {
+    const long thr = Ttok * nh * (D / 8);
+    const int grid = static_cast<int>((thr + 255) / 256);
+    if (D == 128) fa_bwd_dot_v8_k<16><<<grid, 256, 0, st>>>(O, dO, Dd, Ttok, nh);
+    else if (D == 64) fa_bwd_dot_v8_k<8><<<grid, 256, 0, st>>>(O, dO, Dd, Ttok, nh);
+    else if (D == 32) fa_bwd_dot_v8_k<4><<<grid, 256, 0, st>>>(O, dO, Dd, Ttok, nh);
+    else if (D == 16) fa_bwd_dot_v8_k<2><<<grid, 256, 0, st>>>(O, dO, Dd, Ttok, nh);
+    else fa_bwd_dot_k<<<static_cast<int>((Ttok * nh * 32 + 255) / 256), 256, 0, st>>>(O, dO, Dd, Ttok, nh, D);
+  }
   if (g_attn_variant != 0) {   // tcgen05 backward (attn_tc.cu) when supported
     const double fl = 8.0 * B * nh * D * (static_cast<double>(s) * (s + 1) / 2);
     const int tok = kstats_begin(K_ATTN_BWD, fl, 0.0, st);

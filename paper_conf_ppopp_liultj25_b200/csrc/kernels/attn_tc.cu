@@ -129,7 +129,8 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_done + 1);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-  const int kt = blockIdx.x, b = blockIdx.y / nh, head = blockIdx.y % nh;
+  // heaviest first: key tile 0 sees every query tile; blockIdx.x runs over (sample, head)
+  const int kt = blockIdx.y, b = blockIdx.x / nh, head = blockIdx.x % nh;
   const int h = nh * DH;
   const long Ttok = static_cast<long>(B) * s;
   const int i0 = (kt * kRows) / kCols;
@@ -350,7 +351,8 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_done + 1);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-  const int qt = blockIdx.x, b = blockIdx.y / nh, head = blockIdx.y % nh;
+  // heaviest first: the last query tile sees every key tile
+  const int qt = gridDim.y - 1 - blockIdx.y, b = blockIdx.x / nh, head = blockIdx.x % nh;
   const int h = nh * DH;
   const long Ttok = static_cast<long>(B) * s;
   const int last_q = min(qt * kRows + kRows - 1, s - 1);
@@ -532,7 +534,7 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
     cudaFuncSetAttribute(fa_bwd_dq_tc<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_dq<DH>());
     set = true;
   }
-  dim3 grid((s + kRows - 1) / kRows, B * nh);
+  dim3 grid(B * nh, (s + kRows - 1) / kRows);
   const char* only = getenv("MARIO_ATTN_TC_ONLY");   // debugging aid: "dkdv" or "dq"
   if (!only || only[1] == 'k')
     fa_bwd_dkdv_tc<DH><<<grid, kThreadsB, smem_dkdv<DH>(), st>>>(m128, m64, d64, lse, Dd, dqkv, B, s, nh);

@@ -30,7 +30,7 @@ __device__ __forceinline__ float warp_max(float v) {
 inline int cdiv(long a, long b) { return static_cast<int>((a + b - 1) / b); }
 }  // namespace
 
-int g_norm_tile = 1;   // 0: the warp-per-row kernels (kept for A/B measurement)
+int g_norm_tile = 2;   // 2: row-pipelined (rowpipe.cu); 1: block-per-row-tile; 0: warp-per-row (A/B)
 
 namespace {
 
@@ -1058,6 +1058,7 @@ template <class T>
 void layernorm_fwd(const T* x, const float* g, const float* b, T* y, float* stats, int rows, int n, float eps, cudaStream_t st) {
   KScope ks_(K_NORM, st);
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
+    if (g_norm_tile == 2 && norm_fwd_pipe(x, g, b, y, stats, rows, n, eps, 0, st)) return;
     if (n % 8 == 0) {
       if (n <= 1024) norm_fwd_reg_k<false, 4><<<cdiv(rows, 8), 256, 0, st>>>(x, g, b, y, stats, rows, n, eps);
       else if (n <= 2048) norm_fwd_reg_k<false, 8><<<cdiv(rows, 8), 256, 0, st>>>(x, g, b, y, stats, rows, n, eps);
@@ -1075,6 +1076,7 @@ template <class T>
 void rmsnorm_fwd(const T* x, const float* g, T* y, float* stats, int rows, int n, float eps, cudaStream_t st) {
   KScope ks_(K_NORM, st);
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
+    if (g_norm_tile == 2 && norm_fwd_pipe(x, g, nullptr, y, stats, rows, n, eps, 1, st)) return;
     if (n % 8 == 0) {
       if (n <= 1024) norm_fwd_reg_k<true, 4><<<cdiv(rows, 8), 256, 0, st>>>(x, g, nullptr, y, stats, rows, n, eps);
       else if (n <= 2048) norm_fwd_reg_k<true, 8><<<cdiv(rows, 8), 256, 0, st>>>(x, g, nullptr, y, stats, rows, n, eps);
@@ -1093,6 +1095,8 @@ void norm_bwd_dx(const T* dy, const T* x, const float* stats, const float* g, co
                  int rms, cudaStream_t st) {
   KScope ks_(K_NORM, st);
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
+    if (g_norm_tile == 2 && norm_bwd_pipe(dy, x, stats, g, dres, dx, rows, n, rms, nullptr, nullptr, nullptr, nullptr, 0, st))
+      return;
     if (g_norm_tile && norm_bwd_tile(dy, x, stats, g, dres, dx, rows, n, rms, nullptr, nullptr, nullptr, nullptr, 0, st))
       return;
     if (n % 8 == 0) {
@@ -1140,6 +1144,9 @@ void norm_bwd(const T* dy, const T* x, const float* stats, const float* g, const
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
     if (g_norm_tile) {
       KScope ks_(K_NORM, st);
+      if (g_norm_tile == 2 &&
+          norm_bwd_pipe(dy, x, stats, g, dres, dx, rows, n, rms, dg, db, dsum, partial, partial_floats, st))
+        return;
       if (norm_bwd_tile(dy, x, stats, g, dres, dx, rows, n, rms, dg, db, dsum, partial, partial_floats, st)) return;
     }
   }
@@ -1205,6 +1212,9 @@ template <class T>
 void softmax_ce(const float* logits, const int32_t* tok, int ld_tok, int s, int rows, int V, float inv_ntok,
                 T* dlogits, float* row_loss, cudaStream_t st) {
   KScope ks_(K_CE, st);
+  if constexpr (std::is_same<T, __nv_bfloat16>::value) {
+    if (softmax_ce_fast(logits, tok, ld_tok, s, rows, V, inv_ntok, dlogits, row_loss, st)) return;
+  }
   softmax_ce_k<T><<<rows, 512, 0, st>>>(logits, tok, ld_tok, s, V, inv_ntok, dlogits, row_loss);
   note_launch();
 }

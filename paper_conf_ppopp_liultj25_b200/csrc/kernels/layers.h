@@ -30,6 +30,15 @@ template <class T> void norm_bwd(const T* dy, const T* x, const float* stats, co
                                  int rows, int n, int rms, float* dg, float* db, float* dsum, float* partial,
                                  size_t partial_floats, cudaStream_t st);
 extern int g_norm_tile;
+// Row-pipelined bf16 kernels (rowpipe.cu); false = shape not supported (caller falls back).
+bool norm_pipe_supported(int n);
+bool norm_fwd_pipe(const __nv_bfloat16* x, const float* g, const float* b, __nv_bfloat16* y, float* stats, int rows,
+                   int n, float eps, int rms, cudaStream_t st);
+bool norm_bwd_pipe(const __nv_bfloat16* dy, const __nv_bfloat16* x, const float* stats, const float* g,
+                   const __nv_bfloat16* dres, __nv_bfloat16* dx, int rows, int n, int rms, float* dg, float* db,
+                   float* dsum, float* partial, size_t partial_floats, cudaStream_t st);
+bool softmax_ce_fast(const float* logits, const int32_t* tok, int ld_tok, int s, int rows, int V, float inv_ntok,
+                     __nv_bfloat16* dlogits, float* row_loss, cudaStream_t st);
 // Column reductions into fp32 grads (+=): mode 0: out0 += sum_r a[r,c]
 // mode 1 (LN): out0 += sum dy*xhat, out1 += sum dy; mode 2 (RMS): out0 += sum dy*xhat.
 template <class T> void colsum(const T* a, const T* x, const float* stats, int rows, int n, int lda, int mode,

@@ -1,0 +1,495 @@
+// Row-pipelined bandwidth kernels (SURVEY §2.2 K7/K8 norms, K13 softmax-CE, K14 column sums), bf16.
+//
+// Norms: a persistent grid (occupancy x SMs CTAs); CTA b owns the contiguous row range
+// [rows*b/nblk, rows*(b+1)/nblk). Its rows stream through a ring of S shared-memory stages filled by
+// 1-D bulk copies (cp.async.bulk, one mbarrier per stage), so S rows per CTA are in flight while
+// the current one is reduced: the DRAM queue never drains between rows (the warp-per-row kernels
+// load, reduce, store and only then start the next row: 1.5 TB/s measured). Thread t owns the
+// 16-byte chunk t of a row (block = n/8 threads rounded up to a warp): row sums go warp -> shared
+// memory -> every thread in a fixed order (deterministic), one __syncthreads per row, after which
+// thread 0 refills the stage just consumed.
+// Formulas: SURVEY §8(c) c1 (LN/RMS forward, readings A1/A2; backward dx = (g - mean g - xhat
+// mean(g xhat)) / sigma, dgamma = sum dy xhat, dbeta = sum dy).
+#include <cstdint>
+#include <cuda_bf16.h>
+#include <cuda_runtime.h>
+
+#include "kstats.h"
+#include "layers.h"
+#include "sm100.cuh"
+
+namespace mario {
+int device_sms();
+
+namespace {
+using bf16 = __nv_bfloat16;
+using namespace sm100;
+
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ uint4 lds128(const void* p) {
+  uint4 v;
+  asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];"
+               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(smem_u32(p)) : "memory");
+  return v;
+}
+__device__ __forceinline__ float wsum(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+__device__ __forceinline__ float wmax(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o));
+  return v;
+}
+__device__ __forceinline__ void unpack8(const uint4& u, float (&f)[8]) {
+  const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&u);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) { const float2 p = __bfloat1622float2(h[i]); f[2 * i] = p.x; f[2 * i + 1] = p.y; }
+}
+__device__ __forceinline__ uint4 pack8(const float (&f)[8]) {
+  uint4 u;
+  __nv_bfloat162* h = reinterpret_cast<__nv_bfloat162*>(&u);
+#pragma unroll
+  for (int i = 0; i < 4; ++i) h[i] = __floats2bfloat162_rn(f[2 * i], f[2 * i + 1]);
+  return u;
+}
+__device__ __forceinline__ void load8(const float* p, float (&f)[8]) {
+  const float4 a = *reinterpret_cast<const float4*>(p), b = *reinterpret_cast<const float4*>(p + 4);
+  f[0] = a.x; f[1] = a.y; f[2] = a.z; f[3] = a.w; f[4] = b.x; f[5] = b.y; f[6] = b.z; f[7] = b.w;
+}
+
+// shared-memory carve-up: S stages of `stage_bytes` (16-byte multiples), S mbarriers, reductions
+struct PipeSmem {
+  uint8_t* stage0;
+  uint64_t* bar;
+  float* red;   // [2 parity][3][32 warps]
+};
+__device__ __forceinline__ PipeSmem carve(uint8_t* raw, int S, int stage_bytes) {
+  PipeSmem p;
+  p.stage0 = raw;
+  p.bar = reinterpret_cast<uint64_t*>(raw + static_cast<size_t>(S) * stage_bytes);
+  p.red = reinterpret_cast<float*>(p.bar + S);
+  return p;
+}
+inline size_t pipe_smem_bytes(int S, int stage_bytes) {
+  return static_cast<size_t>(S) * stage_bytes + S * sizeof(uint64_t) + 2 * 3 * 32 * sizeof(float);
+}
+
+// ------------------------------------------------------------------------- forward
+// y = (x - mean) * rstd * g (+ b); stats[r] = (mean, rstd). LN: per-thread (count, mean, M2) of its
+// 8 values combined by Chan's rule (warp, then the warps in fixed order), so one barrier per row.
+template <bool RMS>
+__global__ void __launch_bounds__(1024) norm_fwd_pipe_k(const bf16* __restrict__ x, const float* __restrict__ g,
+                                                        const float* __restrict__ b, bf16* __restrict__ y,
+                                                        float* __restrict__ stats, int rows, int n, float eps, int S,
+                                                        int nblk) {
+  extern __shared__ __align__(128) uint8_t smem_raw[];
+  const int stage_bytes = n * 2;
+  PipeSmem sm = carve(smem_raw, S, stage_bytes);
+  const int t = threadIdx.x, w = t / 32, lane = t % 32, nw = blockDim.x / 32;
+  const bool act = t * 8 < n;
+  const int rb = static_cast<int>(static_cast<long>(rows) * blockIdx.x / nblk);
+  const int re = static_cast<int>(static_cast<long>(rows) * (blockIdx.x + 1) / nblk);
+  if (t == 0) {
+    for (int i = 0; i < S; ++i) mbar_init(&sm.bar[i], 1);
+    fence_barrier_init();
+  }
+  __syncthreads();
+  if (t == 0) {
+    for (int i = 0; i < S && rb + i < re; ++i) {
+      mbar_arrive_expect_tx(&sm.bar[i], stage_bytes);
+      bulk_g2s(sm.stage0 + static_cast<size_t>(i) * stage_bytes, x + static_cast<long>(rb + i) * n, stage_bytes,
+               &sm.bar[i]);
+    }
+  }
+  float gg[8], bb[8];
+  if (act) {
+    load8(g + t * 8, gg);
+    if (!RMS) load8(b + t * 8, bb);
+  }
+  const float inv_n = 1.f / n;
+  for (int r = rb, it = 0; r < re; ++r, ++it) {
+    const int st = it % S, par = it & 1;
+    uint8_t* buf = sm.stage0 + static_cast<size_t>(st) * stage_bytes;
+    mbar_wait(&sm.bar[st], (it / S) & 1);
+    float v[8];
+    if (act) unpack8(lds128(buf + t * 16), v);
+    else {
+#pragma unroll
+      for (int j = 0; j < 8; ++j) v[j] = 0.f;
+    }
+    float* red = sm.red + par * 96;
+    if (RMS) {
+      float q = 0.f;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) q += v[j] * v[j];
+      q = wsum(q);
+      if (lane == 0) red[w] = q;
+    } else {
+      // thread-local mean and M2 over its 8 values (or none), then Chan's pairwise combination
+      float c = act ? 8.f : 0.f, s = 0.f;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) s += v[j];
+      float mu = act ? s * 0.125f : 0.f, m2 = 0.f;
+#pragma unroll
+      for (int j = 0; j < 8; ++j) { const float d = v[j] - mu; m2 += act ? d * d : 0.f; }
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const float c2 = __shfl_xor_sync(0xffffffffu, c, o), mu2 = __shfl_xor_sync(0xffffffffu, mu, o),
+                    q2 = __shfl_xor_sync(0xffffffffu, m2, o);
+        const float cn = c + c2;
+        // both xor partners combine the same pair in the same roles (lower lane = "a"), so they
+        // hold bitwise-identical results
+        const bool lo = (lane & o) == 0;
+        const float ma = lo ? mu : mu2, mb = lo ? mu2 : mu, ca = lo ? c : c2, cb = lo ? c2 : c;
+        const float qa = lo ? m2 : q2, qb = lo ? q2 : m2;
+        const float dd = mb - ma, fb = cn > 0.f ? cb / cn : 0.f;
+        mu = ma + dd * fb;
+        m2 = qa + qb + dd * dd * ca * fb;
+        c = cn;
+      }
+      if (lane == 0) { red[w] = c; red[32 + w] = mu; red[64 + w] = m2; }
+    }
+    __syncthreads();
+    // every thread has its chunk in registers: refill this stage with row r + S
+    if (t == 0 && r + S < re) {
+      mbar_arrive_expect_tx(&sm.bar[st], stage_bytes);
+      bulk_g2s(buf, x + static_cast<long>(r + S) * n, stage_bytes, &sm.bar[st]);
+    }
+    float mean = 0.f, rstd;
+    if (RMS) {
+      float q = 0.f;
+      for (int i = 0; i < nw; ++i) q += red[i];
+      rstd = rsqrtf(q * inv_n + eps);
+    } else {
+      float c = red[0], mu = red[32], m2 = red[64];
+      for (int i = 1; i < nw; ++i) {
+        const float cb = red[i], mb = red[32 + i], qb = red[64 + i];
+        const float cn = c + cb;
+        if (cn > 0.f) {
+          const float dd = mb - mu, fb = cb / cn;
+          mu += dd * fb;
+          m2 += qb + dd * dd * c * fb;
+          c = cn;
+        }
+      }
+      mean = mu;
+      rstd = rsqrtf(m2 * inv_n + eps);
+    }
+    if (act) {
+      float o[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) o[j] = (v[j] - mean) * rstd * gg[j] + (RMS ? 0.f : bb[j]);
+      *reinterpret_cast<uint4*>(y + static_cast<long>(r) * n + t * 8) = pack8(o);
+    }
+    if (t == 0) *reinterpret_cast<float2*>(stats + 2 * static_cast<long>(r)) = make_float2(mean, rstd);
+  }
+}
+
+// ------------------------------------------------------------------------ backward
+// dx = (dy g - mean(dy g) - xhat mean(dy g xhat)) rstd (+ dres); the CTA's column partial sums
+// partial[0][blk] = sum dy xhat, [1] = sum dy (LN), [2] = sum of the written dx (when sum_out).
+// Stage = [dy row | x row | dres row]. Stats of the CTA's range are staged in shared memory.
+__global__ void __launch_bounds__(640) norm_bwd_pipe_k(const bf16* __restrict__ dy, const bf16* __restrict__ x,
+                                                        const float* __restrict__ stats, const float* __restrict__ g,
+                                                        const bf16* __restrict__ dres, bf16* __restrict__ dx, int rows,
+                                                        int n, int rms, float* __restrict__ partial, int nblk,
+                                                        int sum_out, int S, int max_range) {
+  extern __shared__ __align__(128) uint8_t smem_raw[];
+  const int nin = dres ? 3 : 2;
+  const int row_bytes = n * 2, stage_bytes = nin * row_bytes;
+  PipeSmem sm = carve(smem_raw, S, stage_bytes);
+  float2* sstat = reinterpret_cast<float2*>(sm.red + 2 * 96);
+  const int t = threadIdx.x, w = t / 32, lane = t % 32, nw = blockDim.x / 32;
+  const bool act = t * 8 < n;
+  const int rb = static_cast<int>(static_cast<long>(rows) * blockIdx.x / nblk);
+  const int re = static_cast<int>(static_cast<long>(rows) * (blockIdx.x + 1) / nblk);
+  auto issue = [&](int i, int r) {
+    uint8_t* buf = sm.stage0 + static_cast<size_t>(i) * stage_bytes;
+    mbar_arrive_expect_tx(&sm.bar[i], stage_bytes);
+    bulk_g2s(buf, dy + static_cast<long>(r) * n, row_bytes, &sm.bar[i]);
+    bulk_g2s(buf + row_bytes, x + static_cast<long>(r) * n, row_bytes, &sm.bar[i]);
+    if (dres) bulk_g2s(buf + 2 * row_bytes, dres + static_cast<long>(r) * n, row_bytes, &sm.bar[i]);
+  };
+  if (t == 0) {
+    for (int i = 0; i < S; ++i) mbar_init(&sm.bar[i], 1);
+    fence_barrier_init();
+  }
+  __syncthreads();
+  if (t == 0)
+    for (int i = 0; i < S && rb + i < re; ++i) issue(i, rb + i);
+  for (int i = t; i < re - rb && i < max_range; i += blockDim.x)
+    sstat[i] = *reinterpret_cast<const float2*>(stats + 2 * static_cast<long>(rb + i));
+  float gg[8], ag[8], ab[8], ao[8];
+#pragma unroll
+  for (int j = 0; j < 8; ++j) { gg[j] = 0.f; ag[j] = 0.f; ab[j] = 0.f; ao[j] = 0.f; }
+  if (act) load8(g + t * 8, gg);
+  __syncthreads();
+  const float inv_n = 1.f / n;
+  for (int r = rb, it = 0; r < re; ++r, ++it) {
+    const int st = it % S, par = it & 1;
+    uint8_t* buf = sm.stage0 + static_cast<size_t>(st) * stage_bytes;
+    const float2 ms = sstat[it];
+    mbar_wait(&sm.bar[st], (it / S) & 1);
+    float d[8], xh[8], rr[8];
+#pragma unroll
+    for (int j = 0; j < 8; ++j) { d[j] = 0.f; xh[j] = 0.f; rr[j] = 0.f; }
+    if (act) {
+      unpack8(lds128(buf + t * 16), d);
+      unpack8(lds128(buf + row_bytes + t * 16), xh);
+      if (dres) unpack8(lds128(buf + 2 * row_bytes + t * 16), rr);
+    }
+    float sg = 0.f, sgx = 0.f;
+#pragma unroll
+    for (int j = 0; j < 8; ++j) {
+      xh[j] = (xh[j] - ms.x) * ms.y;
+      const float gp = d[j] * gg[j];
+      sg += gp;
+      sgx += gp * xh[j];
+      ag[j] += d[j] * xh[j];
+      ab[j] += d[j];
+    }
+    sg = wsum(sg);
+    sgx = wsum(sgx);
+    float* red = sm.red + par * 96;
+    if (lane == 0) { red[w] = sg; red[32 + w] = sgx; }
+    __syncthreads();
+    if (t == 0 && r + S < re) issue(st, r + S);
+    float tg = 0.f, tgx = 0.f;
+    for (int i = 0; i < nw; ++i) { tg += red[i]; tgx += red[32 + i]; }
+    tg = rms ? 0.f : tg * inv_n;
+    tgx *= inv_n;
+    if (act) {
+      float o[8];
+#pragma unroll
+      for (int j = 0; j < 8; ++j) o[j] = (d[j] * gg[j] - tg - xh[j] * tgx) * ms.y + rr[j];
+      const uint4 u = pack8(o);
+      *reinterpret_cast<uint4*>(dx + static_cast<long>(r) * n + t * 8) = u;
+      float q[8];
+      unpack8(u, q);
+#pragma unroll
+      for (int j = 0; j < 8; ++j) ao[j] += q[j];
+    }
+  }
+  if (!partial || !act) return;
+  const int c = t * 8;
+  float* p0 = partial + static_cast<long>(blockIdx.x) * n + c;
+  *reinterpret_cast<float4*>(p0) = make_float4(ag[0], ag[1], ag[2], ag[3]);
+  *reinterpret_cast<float4*>(p0 + 4) = make_float4(ag[4], ag[5], ag[6], ag[7]);
+  if (!rms) {
+    float* p1 = partial + static_cast<long>(nblk + blockIdx.x) * n + c;
+    *reinterpret_cast<float4*>(p1) = make_float4(ab[0], ab[1], ab[2], ab[3]);
+    *reinterpret_cast<float4*>(p1 + 4) = make_float4(ab[4], ab[5], ab[6], ab[7]);
+  }
+  if (sum_out) {
+    float* p2 = partial + static_cast<long>(2 * nblk + blockIdx.x) * n + c;
+    *reinterpret_cast<float4*>(p2) = make_float4(ao[0], ao[1], ao[2], ao[3]);
+    *reinterpret_cast<float4*>(p2 + 4) = make_float4(ao[4], ao[5], ao[6], ao[7]);
+  }
+}
+
+// out_k[c] += sum_b partial[k][b][c] (k = 0..2, null outputs skipped). Block = 32 columns x 32 warps:
+// warp w sums partial rows w, w + 32, ... (4 loads in flight per array), then the warp sums are
+// added in fixed order (deterministic).
+__global__ void __launch_bounds__(1024) colsum_final_wide_k(const float* __restrict__ partial, int nblk, int n,
+                                                            float* out0, float* out1, float* out2) {
+  __shared__ float red[3][32][33];
+  const int w = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int c = blockIdx.x * 32 + lane;
+  float s[3] = {0.f, 0.f, 0.f};
+  if (c < n) {
+    const float* p[3] = {partial, out1 ? partial + static_cast<long>(nblk) * n : nullptr,
+                         out2 ? partial + static_cast<long>(2 * nblk) * n : nullptr};
+#pragma unroll
+    for (int k = 0; k < 3; ++k) {
+      if (!p[k]) continue;
+      float a0 = 0.f, a1 = 0.f, a2 = 0.f, a3 = 0.f;
+      int bb = w;
+      for (; bb + 96 < nblk; bb += 128) {
+        a0 += p[k][static_cast<long>(bb) * n + c];
+        a1 += p[k][static_cast<long>(bb + 32) * n + c];
+        a2 += p[k][static_cast<long>(bb + 64) * n + c];
+        a3 += p[k][static_cast<long>(bb + 96) * n + c];
+      }
+      for (; bb < nblk; bb += 32) a0 += p[k][static_cast<long>(bb) * n + c];
+      s[k] = (a0 + a1) + (a2 + a3);
+    }
+  }
+#pragma unroll
+  for (int k = 0; k < 3; ++k) red[k][w][lane] = s[k];
+  __syncthreads();
+  if (w < 3 && c < n) {
+    float* o = w == 0 ? out0 : (w == 1 ? out1 : out2);
+    if (o) {
+      float tt = 0.f;
+      for (int i = 0; i < 32; ++i) tt += red[w][i][lane];
+      o[c] += tt;
+    }
+  }
+}
+
+// ---------------------------------------------------------------- softmax-CE
+// One CTA (512 threads) per row; the whole fp32 row is held in registers (thread t: float4 chunks
+// t, t + 512, ...), so the logits are read from HBM exactly once: block max, then p = 2^((z-M)log2e)
+// kept in place, block sum, dlogits = (p / sum - [c == y]) / Ntok written as bf16, row_loss =
+// log(sum) + M - z_y.
+template <int NV>
+__global__ void __launch_bounds__(512, 1) softmax_ce_reg_k(const float* __restrict__ logits,
+                                                           const int32_t* __restrict__ tok, int ld_tok, int s, int V,
+                                                           float inv_ntok, bf16* __restrict__ dlogits,
+                                                           float* __restrict__ row_loss) {
+  __shared__ float red[2][16];
+  constexpr float LOG2E = 1.4426950408889634f;
+  const long r = blockIdx.x;
+  const int t = threadIdx.x, w = t / 32, lane = t % 32;
+  const int nv4 = V / 4;
+  const float4* z = reinterpret_cast<const float4*>(logits + r * V);
+  const int bi = static_cast<int>(r / s), ti = static_cast<int>(r % s);
+  const int y = tok[static_cast<long>(bi) * ld_tok + ti + 1];
+  float zy = 0.f;
+  if (t == 0) zy = logits[r * V + y];
+  float4 v[NV];
+  float m = -INFINITY;
+#pragma unroll
+  for (int i = 0; i < NV; ++i) {
+    const int c = t + i * 512;
+    v[i] = c < nv4 ? z[c] : make_float4(-INFINITY, -INFINITY, -INFINITY, -INFINITY);
+    m = fmaxf(m, fmaxf(fmaxf(v[i].x, v[i].y), fmaxf(v[i].z, v[i].w)));
+  }
+  m = wmax(m);
+  if (lane == 0) red[0][w] = m;
+  __syncthreads();
+  float M = red[0][0];
+#pragma unroll
+  for (int i = 1; i < 16; ++i) M = fmaxf(M, red[0][i]);
+  const float ml = M * LOG2E;
+  float l = 0.f;
+#pragma unroll
+  for (int i = 0; i < NV; ++i) {
+    v[i].x = exp2f(fmaf(v[i].x, LOG2E, -ml));
+    v[i].y = exp2f(fmaf(v[i].y, LOG2E, -ml));
+    v[i].z = exp2f(fmaf(v[i].z, LOG2E, -ml));
+    v[i].w = exp2f(fmaf(v[i].w, LOG2E, -ml));
+    l += (v[i].x + v[i].y) + (v[i].z + v[i].w);
+  }
+  l = wsum(l);
+  if (lane == 0) red[1][w] = l;
+  __syncthreads();
+  float L = 0.f;
+#pragma unroll
+  for (int i = 0; i < 16; ++i) L += red[1][i];
+  const float sc = inv_ntok / L;
+  uint2* out = reinterpret_cast<uint2*>(dlogits + r * V);
+#pragma unroll
+  for (int i = 0; i < NV; ++i) {
+    const int c = t + i * 512;
+    if (c < nv4) {
+      const int c0 = 4 * c;
+      const float a = v[i].x * sc - (c0 == y ? inv_ntok : 0.f);
+      const float b = v[i].y * sc - (c0 + 1 == y ? inv_ntok : 0.f);
+      const float cc = v[i].z * sc - (c0 + 2 == y ? inv_ntok : 0.f);
+      const float d = v[i].w * sc - (c0 + 3 == y ? inv_ntok : 0.f);
+      uint2 u;
+      *reinterpret_cast<__nv_bfloat162*>(&u.x) = __floats2bfloat162_rn(a, b);
+      *reinterpret_cast<__nv_bfloat162*>(&u.y) = __floats2bfloat162_rn(cc, d);
+      out[c] = u;
+    }
+  }
+  if (t == 0) row_loss[r] = (M + logf(L)) - zy;
+}
+
+template <class K>
+int occ_grid(K kernel, int threads, size_t smem) {
+  int occ = 1;
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&occ, kernel, threads, smem);
+  return device_sms() * (occ < 1 ? 1 : occ);
+}
+inline int threads_for(int n) { return ((n / 8 + 31) / 32) * 32; }
+inline int cdivl(long a, long b) { return static_cast<int>((a + b - 1) / b); }
+}  // namespace
+
+bool norm_pipe_supported(int n) { return n % 8 == 0 && n >= 8 && n <= 8192; }
+
+bool norm_fwd_pipe(const bf16* x, const float* g, const float* b, bf16* y, float* stats, int rows, int n, float eps,
+                   int rms, cudaStream_t st) {
+  if (!norm_pipe_supported(n)) return false;
+  if (rows <= 0) return true;
+  const int nt = threads_for(n), sb = n * 2;
+  int S = 24576 / sb;
+  S = S < 2 ? 2 : (S > 8 ? 8 : S);
+  const size_t smem = pipe_smem_bytes(S, sb);
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(norm_fwd_pipe_k<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+    cudaFuncSetAttribute(norm_fwd_pipe_k<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+    attr = true;
+  }
+  int nblk = rms ? occ_grid(norm_fwd_pipe_k<true>, nt, smem) : occ_grid(norm_fwd_pipe_k<false>, nt, smem);
+  nblk = nblk < rows ? nblk : rows;
+  if (rms) norm_fwd_pipe_k<true><<<nblk, nt, smem, st>>>(x, g, b, y, stats, rows, n, eps, S, nblk);
+  else norm_fwd_pipe_k<false><<<nblk, nt, smem, st>>>(x, g, b, y, stats, rows, n, eps, S, nblk);
+  note_launch();
+  return true;
+}
+
+bool norm_bwd_pipe(const bf16* dy, const bf16* x, const float* stats, const float* g, const bf16* dres, bf16* dx,
+                   int rows, int n, int rms, float* dg, float* db, float* dsum, float* partial, size_t partial_floats,
+                   cudaStream_t st) {
+  if (!norm_pipe_supported(n) || threads_for(n) > 640) return false;
+  if (rows <= 0) return true;
+  const int nt = threads_for(n), nin = dres ? 3 : 2, sb = nin * n * 2;
+  int S = 49152 / sb;
+  S = S < 2 ? 2 : (S > 6 ? 6 : S);
+  static bool attr = false;
+  if (!attr) {
+    cudaFuncSetAttribute(norm_bwd_pipe_k, cudaFuncAttributeMaxDynamicSharedMemorySize, 220 * 1024);
+    attr = true;
+  }
+  // the stats of a CTA's range are staged in shared memory: size for the smallest grid we may use
+  const size_t base = pipe_smem_bytes(S, sb);
+  int nblk = occ_grid(norm_bwd_pipe_k, nt, base + 8 * static_cast<size_t>(cdivl(rows, device_sms())));
+  if (dg) {
+    const long cap = static_cast<long>(partial_floats / (3 * static_cast<size_t>(n)));
+    if (cap < 1) return false;
+    nblk = nblk < cap ? nblk : static_cast<int>(cap);
+  }
+  nblk = nblk < rows ? nblk : rows;
+  const int max_range = cdivl(rows, nblk) + 1;
+  const size_t smem = base + 8 * static_cast<size_t>(max_range);
+  if (smem > 220 * 1024) return false;
+  norm_bwd_pipe_k<<<nblk, nt, smem, st>>>(dy, x, stats, g, dres, dx, rows, n, rms, dg ? partial : nullptr, nblk,
+                                          dsum ? 1 : 0, S, max_range);
+  note_launch();
+  if (dg) {
+    colsum_final_wide_k<<<cdivl(n, 32), 1024, 0, st>>>(partial, nblk, n, dg, rms ? nullptr : db, dsum);
+    note_launch();
+  }
+  return true;
+}
+
+bool softmax_ce_fast(const float* logits, const int32_t* tok, int ld_tok, int s, int rows, int V, float inv_ntok,
+                     bf16* dlogits, float* row_loss, cudaStream_t st) {
+  if (V % 4 || V < 4) return false;
+  const int need = cdivl(V / 4, 512);
+  if (rows <= 0) return true;
+#define CE_CASE(NV)                                                                                            \
+  if (need <= NV) {                                                                                            \
+    softmax_ce_reg_k<NV><<<rows, 512, 0, st>>>(logits, tok, ld_tok, s, V, inv_ntok, dlogits, row_loss);        \
+    note_launch();                                                                                             \
+    return true;                                                                                               \
+  }
+  CE_CASE(1)
+  CE_CASE(2)
+  CE_CASE(4)
+  CE_CASE(8)
+  CE_CASE(16)
+  CE_CASE(25)
+#undef CE_CASE
+  return false;
+}
+
+}  // namespace mario
