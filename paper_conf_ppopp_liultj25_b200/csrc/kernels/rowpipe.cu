@@ -71,161 +71,163 @@ __device__ __forceinline__ void load8(const float* p, float (&f)[8]) {
   f[0] = a.x; f[1] = a.y; f[2] = a.z; f[3] = a.w; f[4] = b.x; f[5] = b.y; f[6] = b.z; f[7] = b.w;
 }
 
-// shared-memory carve-up: S stages of `stage_bytes` (16-byte multiples), S mbarriers, reductions
-struct PipeSmem {
-  uint8_t* stage0;
-  uint64_t* bar;
-  float* red;   // [2 parity][3][32 warps]
-};
-__device__ __forceinline__ PipeSmem carve(uint8_t* raw, int S, int stage_bytes) {
-  PipeSmem p;
-  p.stage0 = raw;
-  p.bar = reinterpret_cast<uint64_t*>(raw + static_cast<size_t>(S) * stage_bytes);
-  p.red = reinterpret_cast<float*>(p.bar + S);
-  return p;
-}
+// shared memory: S slots of `stage_bytes` (16-byte multiples), S mbarriers, the reduction buffers
+constexpr int kPipeR = 2;   // rows per iteration of the norm kernels
 inline size_t pipe_smem_bytes(int S, int stage_bytes) {
-  return static_cast<size_t>(S) * stage_bytes + S * sizeof(uint64_t) + 2 * 3 * 32 * sizeof(float);
+  return static_cast<size_t>(S) * stage_bytes + S * sizeof(uint64_t) + 2 * 32 * kPipeR * 2 * sizeof(float);
 }
 
 // ------------------------------------------------------------------------- forward
-// y = (x - mean) * rstd * g (+ b); stats[r] = (mean, rstd). LN: per-thread (count, mean, M2) of its
-// 8 values combined by Chan's rule (warp, then the warps in fixed order), so one barrier per row.
-template <bool RMS>
+// y = (x - mean) * rstd * g (+ b); stats[r] = (mean, rstd). R rows per iteration (their reductions
+// interleave), one __syncthreads per iteration. LN sums are shifted by the row's first element K
+// (one broadcast shared load): mean = K + S1/n, var = S2/n - (S1/n)^2 with S1 = sum(x - K),
+// S2 = sum((x - K)^2), so the cancellation is relative to |mean - K| ~ one standard deviation, not
+// |mean|. Warp sums -> shared memory [par][warp][R][2] -> every thread adds the warps in order.
+template <bool RMS, int R>
 __global__ void __launch_bounds__(1024) norm_fwd_pipe_k(const bf16* __restrict__ x, const float* __restrict__ g,
                                                         const float* __restrict__ b, bf16* __restrict__ y,
                                                         float* __restrict__ stats, int rows, int n, float eps, int S,
                                                         int nblk) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
-  const int stage_bytes = n * 2;
-  PipeSmem sm = carve(smem_raw, S, stage_bytes);
+  const int sb = n * 2;
+  uint8_t* stage0 = smem_raw;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(smem_raw + static_cast<size_t>(S) * sb);
+  float* red = reinterpret_cast<float*>(bar + S);     // [2][32][R][2]
   const int t = threadIdx.x, w = t / 32, lane = t % 32, nw = blockDim.x / 32;
   const bool act = t * 8 < n;
   const int rb = static_cast<int>(static_cast<long>(rows) * blockIdx.x / nblk);
   const int re = static_cast<int>(static_cast<long>(rows) * (blockIdx.x + 1) / nblk);
   if (t == 0) {
-    for (int i = 0; i < S; ++i) mbar_init(&sm.bar[i], 1);
+    for (int i = 0; i < S; ++i) mbar_init(&bar[i], 1);
     fence_barrier_init();
   }
   __syncthreads();
   if (t == 0) {
     for (int i = 0; i < S && rb + i < re; ++i) {
-      mbar_arrive_expect_tx(&sm.bar[i], stage_bytes);
-      bulk_g2s(sm.stage0 + static_cast<size_t>(i) * stage_bytes, x + static_cast<long>(rb + i) * n, stage_bytes,
-               &sm.bar[i]);
+      mbar_arrive_expect_tx(&bar[i], sb);
+      bulk_g2s(stage0 + static_cast<size_t>(i) * sb, x + static_cast<long>(rb + i) * n, sb, &bar[i]);
     }
   }
   float gg[8], bb[8];
+#pragma unroll
+  for (int j = 0; j < 8; ++j) { gg[j] = 0.f; bb[j] = 0.f; }
   if (act) {
     load8(g + t * 8, gg);
     if (!RMS) load8(b + t * 8, bb);
   }
   const float inv_n = 1.f / n;
-  for (int r = rb, it = 0; r < re; ++r, ++it) {
-    const int st = it % S, par = it & 1;
-    uint8_t* buf = sm.stage0 + static_cast<size_t>(st) * stage_bytes;
-    mbar_wait(&sm.bar[st], (it / S) & 1);
-    float v[8];
-    if (act) unpack8(lds128(buf + t * 16), v);
-    else {
+  for (int r0 = rb, it = 0; r0 < re; r0 += R, ++it) {
+    float v[R][8], K[R], s1[R], s2[R];
+    const int par = it & 1;
 #pragma unroll
-      for (int j = 0; j < 8; ++j) v[j] = 0.f;
-    }
-    float* red = sm.red + par * 96;
-    if (RMS) {
-      float q = 0.f;
+    for (int q = 0; q < R; ++q) {
+      const int u = it * R + q, sl = u % S;
+      s1[q] = 0.f; s2[q] = 0.f; K[q] = 0.f;
 #pragma unroll
-      for (int j = 0; j < 8; ++j) q += v[j] * v[j];
-      q = wsum(q);
-      if (lane == 0) red[w] = q;
-    } else {
-      // thread-local mean and M2 over its 8 values (or none), then Chan's pairwise combination
-      float c = act ? 8.f : 0.f, s = 0.f;
-#pragma unroll
-      for (int j = 0; j < 8; ++j) s += v[j];
-      float mu = act ? s * 0.125f : 0.f, m2 = 0.f;
-#pragma unroll
-      for (int j = 0; j < 8; ++j) { const float d = v[j] - mu; m2 += act ? d * d : 0.f; }
-#pragma unroll
-      for (int o = 1; o < 32; o <<= 1) {
-        const float c2 = __shfl_xor_sync(0xffffffffu, c, o), mu2 = __shfl_xor_sync(0xffffffffu, mu, o),
-                    q2 = __shfl_xor_sync(0xffffffffu, m2, o);
-        const float cn = c + c2;
-        // both xor partners combine the same pair in the same roles (lower lane = "a"), so they
-        // hold bitwise-identical results
-        const bool lo = (lane & o) == 0;
-        const float ma = lo ? mu : mu2, mb = lo ? mu2 : mu, ca = lo ? c : c2, cb = lo ? c2 : c;
-        const float qa = lo ? m2 : q2, qb = lo ? q2 : m2;
-        const float dd = mb - ma, fb = cn > 0.f ? cb / cn : 0.f;
-        mu = ma + dd * fb;
-        m2 = qa + qb + dd * dd * ca * fb;
-        c = cn;
+      for (int j = 0; j < 8; ++j) v[q][j] = 0.f;
+      if (r0 + q < re) {
+        const uint8_t* buf = stage0 + static_cast<size_t>(sl) * sb;
+        mbar_wait(&bar[sl], (u / S) & 1);
+        if (act) unpack8(lds128(buf + t * 16), v[q]);
+        if (!RMS) K[q] = __bfloat162float(*reinterpret_cast<const bf16*>(buf));
       }
-      if (lane == 0) { red[w] = c; red[32 + w] = mu; red[64 + w] = m2; }
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        const float d = act ? v[q][j] - K[q] : 0.f;
+        s1[q] += d;
+        s2[q] = fmaf(d, d, s2[q]);
+      }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+#pragma unroll
+      for (int q = 0; q < R; ++q) {
+        if (!RMS) s1[q] += __shfl_xor_sync(0xffffffffu, s1[q], o);
+        s2[q] += __shfl_xor_sync(0xffffffffu, s2[q], o);
+      }
+    }
+    float* rp = red + par * (32 * R * 2);
+    if (lane == 0) {
+#pragma unroll
+      for (int q = 0; q < R; ++q) { rp[(w * R + q) * 2] = s1[q]; rp[(w * R + q) * 2 + 1] = s2[q]; }
     }
     __syncthreads();
-    // every thread has its chunk in registers: refill this stage with row r + S
-    if (t == 0 && r + S < re) {
-      mbar_arrive_expect_tx(&sm.bar[st], stage_bytes);
-      bulk_g2s(buf, x + static_cast<long>(r + S) * n, stage_bytes, &sm.bar[st]);
-    }
-    float mean = 0.f, rstd;
-    if (RMS) {
-      float q = 0.f;
-      for (int i = 0; i < nw; ++i) q += red[i];
-      rstd = rsqrtf(q * inv_n + eps);
-    } else {
-      float c = red[0], mu = red[32], m2 = red[64];
-      for (int i = 1; i < nw; ++i) {
-        const float cb = red[i], mb = red[32 + i], qb = red[64 + i];
-        const float cn = c + cb;
-        if (cn > 0.f) {
-          const float dd = mb - mu, fb = cb / cn;
-          mu += dd * fb;
-          m2 += qb + dd * dd * c * fb;
-          c = cn;
+    // every thread holds its chunks in registers: refill the slots just consumed
+    if (t == 0) {
+#pragma unroll
+      for (int q = 0; q < R; ++q) {
+        const int u = it * R + q, rn = rb + u + S;
+        if (rn < re) {
+          const int sl = u % S;
+          mbar_arrive_expect_tx(&bar[sl], sb);
+          bulk_g2s(stage0 + static_cast<size_t>(sl) * sb, x + static_cast<long>(rn) * n, sb, &bar[sl]);
         }
       }
-      mean = mu;
-      rstd = rsqrtf(m2 * inv_n + eps);
     }
-    if (act) {
-      float o[8];
+    float S1[R], S2[R];
 #pragma unroll
-      for (int j = 0; j < 8; ++j) o[j] = (v[j] - mean) * rstd * gg[j] + (RMS ? 0.f : bb[j]);
-      *reinterpret_cast<uint4*>(y + static_cast<long>(r) * n + t * 8) = pack8(o);
+    for (int q = 0; q < R; ++q) { S1[q] = 0.f; S2[q] = 0.f; }
+    for (int i = 0; i < nw; ++i) {
+#pragma unroll
+      for (int q = 0; q < R; ++q) { S1[q] += rp[(i * R + q) * 2]; S2[q] += rp[(i * R + q) * 2 + 1]; }
     }
-    if (t == 0) *reinterpret_cast<float2*>(stats + 2 * static_cast<long>(r)) = make_float2(mean, rstd);
+#pragma unroll
+    for (int q = 0; q < R; ++q) {
+      const int r = r0 + q;
+      if (r >= re) break;
+      float mean = 0.f, var;
+      if (RMS) {
+        var = S2[q] * inv_n;
+      } else {
+        const float m1 = S1[q] * inv_n;
+        mean = K[q] + m1;
+        var = fmaxf(S2[q] * inv_n - m1 * m1, 0.f);
+      }
+      const float rstd = rsqrtf(var + eps);
+      if (act) {
+        float o[8];
+#pragma unroll
+        for (int j = 0; j < 8; ++j) o[j] = (v[q][j] - mean) * rstd * gg[j] + bb[j];
+        *reinterpret_cast<uint4*>(y + static_cast<long>(r) * n + t * 8) = pack8(o);
+      }
+      if (t == 0) *reinterpret_cast<float2*>(stats + 2 * static_cast<long>(r)) = make_float2(mean, rstd);
+    }
   }
 }
 
 // ------------------------------------------------------------------------ backward
 // dx = (dy g - mean(dy g) - xhat mean(dy g xhat)) rstd (+ dres); the CTA's column partial sums
 // partial[0][blk] = sum dy xhat, [1] = sum dy (LN), [2] = sum of the written dx (when sum_out).
-// Stage = [dy row | x row | dres row]. Stats of the CTA's range are staged in shared memory.
+// Slot = [dy row | x row | dres row]; R rows per iteration. Phase 1 reads dy, x from shared
+// memory (row sums), phase 2 (after the barrier) re-reads dy, x, dres and writes dx, so nothing
+// but the column accumulators stays in registers; a slot is refilled at the NEXT iteration's
+// barrier, when every thread is past its phase 2. Stats of the CTA's range are staged in smem.
+template <int R>
 __global__ void __launch_bounds__(640) norm_bwd_pipe_k(const bf16* __restrict__ dy, const bf16* __restrict__ x,
-                                                        const float* __restrict__ stats, const float* __restrict__ g,
-                                                        const bf16* __restrict__ dres, bf16* __restrict__ dx, int rows,
-                                                        int n, int rms, float* __restrict__ partial, int nblk,
-                                                        int sum_out, int S, int max_range) {
+                                                       const float* __restrict__ stats, const float* __restrict__ g,
+                                                       const bf16* __restrict__ dres, bf16* __restrict__ dx, int rows,
+                                                       int n, int rms, float* __restrict__ partial, int nblk,
+                                                       int sum_out, int S, int max_range) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
   const int nin = dres ? 3 : 2;
-  const int row_bytes = n * 2, stage_bytes = nin * row_bytes;
-  PipeSmem sm = carve(smem_raw, S, stage_bytes);
-  float2* sstat = reinterpret_cast<float2*>(sm.red + 2 * 96);
+  const int row_bytes = n * 2, sb = nin * row_bytes;
+  uint8_t* stage0 = smem_raw;
+  uint64_t* bar = reinterpret_cast<uint64_t*>(smem_raw + static_cast<size_t>(S) * sb);
+  float* red = reinterpret_cast<float*>(bar + S);            // [2][32][R][2]
+  float2* sstat = reinterpret_cast<float2*>(red + 2 * 32 * R * 2);
   const int t = threadIdx.x, w = t / 32, lane = t % 32, nw = blockDim.x / 32;
   const bool act = t * 8 < n;
   const int rb = static_cast<int>(static_cast<long>(rows) * blockIdx.x / nblk);
   const int re = static_cast<int>(static_cast<long>(rows) * (blockIdx.x + 1) / nblk);
-  auto issue = [&](int i, int r) {
-    uint8_t* buf = sm.stage0 + static_cast<size_t>(i) * stage_bytes;
-    mbar_arrive_expect_tx(&sm.bar[i], stage_bytes);
-    bulk_g2s(buf, dy + static_cast<long>(r) * n, row_bytes, &sm.bar[i]);
-    bulk_g2s(buf + row_bytes, x + static_cast<long>(r) * n, row_bytes, &sm.bar[i]);
-    if (dres) bulk_g2s(buf + 2 * row_bytes, dres + static_cast<long>(r) * n, row_bytes, &sm.bar[i]);
+  auto issue = [&](int sl, int r) {
+    uint8_t* buf = stage0 + static_cast<size_t>(sl) * sb;
+    mbar_arrive_expect_tx(&bar[sl], sb);
+    bulk_g2s(buf, dy + static_cast<long>(r) * n, row_bytes, &bar[sl]);
+    bulk_g2s(buf + row_bytes, x + static_cast<long>(r) * n, row_bytes, &bar[sl]);
+    if (dres) bulk_g2s(buf + 2 * row_bytes, dres + static_cast<long>(r) * n, row_bytes, &bar[sl]);
   };
   if (t == 0) {
-    for (int i = 0; i < S; ++i) mbar_init(&sm.bar[i], 1);
+    for (int i = 0; i < S; ++i) mbar_init(&bar[i], 1);
     fence_barrier_init();
   }
   __syncthreads();
@@ -239,49 +241,87 @@ __global__ void __launch_bounds__(640) norm_bwd_pipe_k(const bf16* __restrict__ 
   if (act) load8(g + t * 8, gg);
   __syncthreads();
   const float inv_n = 1.f / n;
-  for (int r = rb, it = 0; r < re; ++r, ++it) {
-    const int st = it % S, par = it & 1;
-    uint8_t* buf = sm.stage0 + static_cast<size_t>(st) * stage_bytes;
-    const float2 ms = sstat[it];
-    mbar_wait(&sm.bar[st], (it / S) & 1);
-    float d[8], xh[8], rr[8];
+  for (int r0 = rb, it = 0; r0 < re; r0 += R, ++it) {
+    const int par = it & 1;
+    float sg[R], sgx[R];
 #pragma unroll
-    for (int j = 0; j < 8; ++j) { d[j] = 0.f; xh[j] = 0.f; rr[j] = 0.f; }
-    if (act) {
+    for (int q = 0; q < R; ++q) {
+      const int u = it * R + q, sl = u % S;
+      sg[q] = 0.f; sgx[q] = 0.f;
+      if (r0 + q >= re) continue;
+      const uint8_t* buf = stage0 + static_cast<size_t>(sl) * sb;
+      const float2 ms = sstat[u];
+      mbar_wait(&bar[sl], (u / S) & 1);
+      if (!act) continue;
+      float d[8], xh[8];
+      unpack8(lds128(buf + t * 16), d);
+      unpack8(lds128(buf + row_bytes + t * 16), xh);
+#pragma unroll
+      for (int j = 0; j < 8; ++j) {
+        xh[j] = (xh[j] - ms.x) * ms.y;
+        const float gp = d[j] * gg[j];
+        sg[q] += gp;
+        sgx[q] = fmaf(gp, xh[j], sgx[q]);
+        ag[j] = fmaf(d[j], xh[j], ag[j]);
+        ab[j] += d[j];
+      }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) {
+#pragma unroll
+      for (int q = 0; q < R; ++q) {
+        sg[q] += __shfl_xor_sync(0xffffffffu, sg[q], o);
+        sgx[q] += __shfl_xor_sync(0xffffffffu, sgx[q], o);
+      }
+    }
+    float* rp = red + par * (32 * R * 2);
+    if (lane == 0) {
+#pragma unroll
+      for (int q = 0; q < R; ++q) { rp[(w * R + q) * 2] = sg[q]; rp[(w * R + q) * 2 + 1] = sgx[q]; }
+    }
+    __syncthreads();
+    // every thread is past phase 2 of the previous iteration: refill its slots
+    if (t == 0 && it > 0) {
+#pragma unroll
+      for (int q = 0; q < R; ++q) {
+        const int u = (it - 1) * R + q, rn = rb + u + S;
+        if (rn < re) issue(u % S, rn);
+      }
+    }
+    float tg[R], tgx[R];
+#pragma unroll
+    for (int q = 0; q < R; ++q) { tg[q] = 0.f; tgx[q] = 0.f; }
+    for (int i = 0; i < nw; ++i) {
+#pragma unroll
+      for (int q = 0; q < R; ++q) { tg[q] += rp[(i * R + q) * 2]; tgx[q] += rp[(i * R + q) * 2 + 1]; }
+    }
+    if (!act) continue;
+#pragma unroll
+    for (int q = 0; q < R; ++q) {
+      const int r = r0 + q;
+      if (r >= re) break;
+      const int u = it * R + q;
+      const uint8_t* buf = stage0 + static_cast<size_t>(u % S) * sb;
+      const float2 ms = sstat[u];
+      const float mg = rms ? 0.f : tg[q] * inv_n, mgx = tgx[q] * inv_n;
+      float d[8], xh[8], rr[8];
       unpack8(lds128(buf + t * 16), d);
       unpack8(lds128(buf + row_bytes + t * 16), xh);
       if (dres) unpack8(lds128(buf + 2 * row_bytes + t * 16), rr);
-    }
-    float sg = 0.f, sgx = 0.f;
-#pragma unroll
-    for (int j = 0; j < 8; ++j) {
-      xh[j] = (xh[j] - ms.x) * ms.y;
-      const float gp = d[j] * gg[j];
-      sg += gp;
-      sgx += gp * xh[j];
-      ag[j] += d[j] * xh[j];
-      ab[j] += d[j];
-    }
-    sg = wsum(sg);
-    sgx = wsum(sgx);
-    float* red = sm.red + par * 96;
-    if (lane == 0) { red[w] = sg; red[32 + w] = sgx; }
-    __syncthreads();
-    if (t == 0 && r + S < re) issue(st, r + S);
-    float tg = 0.f, tgx = 0.f;
-    for (int i = 0; i < nw; ++i) { tg += red[i]; tgx += red[32 + i]; }
-    tg = rms ? 0.f : tg * inv_n;
-    tgx *= inv_n;
-    if (act) {
       float o[8];
 #pragma unroll
-      for (int j = 0; j < 8; ++j) o[j] = (d[j] * gg[j] - tg - xh[j] * tgx) * ms.y + rr[j];
-      const uint4 u = pack8(o);
-      *reinterpret_cast<uint4*>(dx + static_cast<long>(r) * n + t * 8) = u;
-      float q[8];
-      unpack8(u, q);
+      for (int j = 0; j < 8; ++j) {
+        const float xhat = (xh[j] - ms.x) * ms.y;
+        o[j] = (d[j] * gg[j] - mg - xhat * mgx) * ms.y + (dres ? rr[j] : 0.f);
+      }
+      const uint4 pk = pack8(o);
+      *reinterpret_cast<uint4*>(dx + static_cast<long>(r) * n + t * 8) = pk;
+      if (sum_out) {
+        float qv[8];
+        unpack8(pk, qv);
 #pragma unroll
-      for (int j = 0; j < 8; ++j) ao[j] += q[j];
+        for (int j = 0; j < 8; ++j) ao[j] += qv[j];
+      }
     }
   }
   if (!partial || !act) return;
@@ -429,18 +469,19 @@ bool norm_fwd_pipe(const bf16* x, const float* g, const float* b, bf16* y, float
   if (rows <= 0) return true;
   const int nt = threads_for(n), sb = n * 2;
   int S = 24576 / sb;
-  S = S < 2 ? 2 : (S > 8 ? 8 : S);
+  S = S < 2 * kPipeR ? 2 * kPipeR : (S > 8 ? 8 : S);
+  S -= S % kPipeR;
   const size_t smem = pipe_smem_bytes(S, sb);
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(norm_fwd_pipe_k<false>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
-    cudaFuncSetAttribute(norm_fwd_pipe_k<true>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+    cudaFuncSetAttribute(norm_fwd_pipe_k<false, kPipeR>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
+    cudaFuncSetAttribute(norm_fwd_pipe_k<true, kPipeR>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
     attr = true;
   }
-  int nblk = rms ? occ_grid(norm_fwd_pipe_k<true>, nt, smem) : occ_grid(norm_fwd_pipe_k<false>, nt, smem);
+  int nblk = rms ? occ_grid(norm_fwd_pipe_k<true, kPipeR>, nt, smem) : occ_grid(norm_fwd_pipe_k<false, kPipeR>, nt, smem);
   nblk = nblk < rows ? nblk : rows;
-  if (rms) norm_fwd_pipe_k<true><<<nblk, nt, smem, st>>>(x, g, b, y, stats, rows, n, eps, S, nblk);
-  else norm_fwd_pipe_k<false><<<nblk, nt, smem, st>>>(x, g, b, y, stats, rows, n, eps, S, nblk);
+  if (rms) norm_fwd_pipe_k<true, kPipeR><<<nblk, nt, smem, st>>>(x, g, b, y, stats, rows, n, eps, S, nblk);
+  else norm_fwd_pipe_k<false, kPipeR><<<nblk, nt, smem, st>>>(x, g, b, y, stats, rows, n, eps, S, nblk);
   note_launch();
   return true;
 }
@@ -452,15 +493,16 @@ bool norm_bwd_pipe(const bf16* dy, const bf16* x, const float* stats, const floa
   if (rows <= 0) return true;
   const int nt = threads_for(n), nin = dres ? 3 : 2, sb = nin * n * 2;
   int S = 49152 / sb;
-  S = S < 2 ? 2 : (S > 6 ? 6 : S);
+  S = S < 2 * kPipeR ? 2 * kPipeR : (S > 6 ? 6 : S);
+  S -= S % kPipeR;
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(norm_bwd_pipe_k, cudaFuncAttributeMaxDynamicSharedMemorySize, 220 * 1024);
+    cudaFuncSetAttribute(norm_bwd_pipe_k<kPipeR>, cudaFuncAttributeMaxDynamicSharedMemorySize, 220 * 1024);
     attr = true;
   }
   // the stats of a CTA's range are staged in shared memory: size for the smallest grid we may use
   const size_t base = pipe_smem_bytes(S, sb);
-  int nblk = occ_grid(norm_bwd_pipe_k, nt, base + 8 * static_cast<size_t>(cdivl(rows, device_sms())));
+  int nblk = occ_grid(norm_bwd_pipe_k<kPipeR>, nt, base + 8 * static_cast<size_t>(cdivl(rows, device_sms())));
   if (dg) {
     const long cap = static_cast<long>(partial_floats / (3 * static_cast<size_t>(n)));
     if (cap < 1) return false;
@@ -470,7 +512,7 @@ bool norm_bwd_pipe(const bf16* dy, const bf16* x, const float* stats, const floa
   const int max_range = cdivl(rows, nblk) + 1;
   const size_t smem = base + 8 * static_cast<size_t>(max_range);
   if (smem > 220 * 1024) return false;
-  norm_bwd_pipe_k<<<nblk, nt, smem, st>>>(dy, x, stats, g, dres, dx, rows, n, rms, dg ? partial : nullptr, nblk,
+  norm_bwd_pipe_k<kPipeR><<<nblk, nt, smem, st>>>(dy, x, stats, g, dres, dx, rows, n, rms, dg ? partial : nullptr, nblk,
                                           dsum ? 1 : 0, S, max_range);
   note_launch();
   if (dg) {
