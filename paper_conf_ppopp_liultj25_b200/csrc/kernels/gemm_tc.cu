@@ -45,7 +45,7 @@ struct Cfg {
   static constexpr int kBBytes = BN * BK * 2;
   static constexpr int kStageBytes = kABytes + kBBytes;
   static constexpr int kTmemCols = 2 * BN;     // double-buffered accumulator
-  static constexpr int kSmem = kStages * kStageBytes + 1024 /*align*/ + 256 /*barriers*/;
+  static constexpr int kSmem = kStages * kStageBytes + 1024 /*align*/ + 256 /*barriers*/ + 4 * 4096 /*epilogue*/;
 };
 
 // bf16 outputs: the SFU tanh (rel. err ~2^-11) is far below bf16 resolution (2^-8)
@@ -129,6 +129,140 @@ __device__ __forceinline__ void epilogue_chunk(const GemmEpilogue& ep, const uin
         d[j] = __float2bfloat16_rn(v[j]);
         if (d2) d2[j] = __float2bfloat16_rn(gelu_tanh_f(v[j]));
       }
+    }
+  }
+}
+
+// Warp-cooperative epilogue for one 32x32 block: lane i holds row rbase + i, columns
+// [col0, col0 + 32) (fp32 in r[]). Global traffic is coalesced through a per-warp 4 KB shared
+// staging buffer `sw`: bf16 inputs (residual, GeLU aux) are loaded 4 lanes per 64-byte row segment
+// and transposed to rows, bf16 outputs are written row-wise to `sw` and stored 4 lanes per row
+// segment, fp32 outputs (wgrad D += v) 8 lanes per 128-byte row segment. Swizzled 16-byte chunks
+// keep every shared access conflict-free. Same arithmetic, in the same order, as epilogue_chunk
+// (which handles ragged column blocks and unaligned pitches).
+__device__ __forceinline__ bool epilogue_vec_ok(const GemmEpilogue& ep) {
+  auto al = [](const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; };
+  return (ep.ldd % 8) == 0 && (ep.out_f32 ? al(ep.d_f32) : al(ep.d_bf16)) && (!ep.d2_bf16 || al(ep.d2_bf16)) &&
+         (!ep.residual || ((ep.ld_res % 8) == 0 && al(ep.residual))) &&
+         (!ep.aux || ((ep.ld_aux % 8) == 0 && al(ep.aux))) && (!ep.bias || al(ep.bias));
+}
+__device__ __forceinline__ void sts128(uint8_t* p, const uint4& v) {
+  asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" :: "r"(smem_u32(p)), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
+               : "memory");
+}
+__device__ __forceinline__ uint4 lds128u(const uint8_t* p) {
+  uint4 v;
+  asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w)
+               : "r"(smem_u32(p)) : "memory");
+  return v;
+}
+// [32 rows][64 B] bf16 block: chunk j of row r lives at r*64 + 16*(j ^ ((r >> 1) & 3))
+__device__ __forceinline__ uint8_t* sw64(uint8_t* sw, int r, int j) { return sw + r * 64 + 16 * (j ^ ((r >> 1) & 3)); }
+// [32 rows][128 B] fp32 block: chunk j of row r at r*128 + 16*(j ^ (r & 7))
+__device__ __forceinline__ uint8_t* sw128(uint8_t* sw, int r, int j) { return sw + r * 128 + 16 * (j ^ (r & 7)); }
+
+// coalesced load of a bf16 [32 rows][32 cols] block (rows >= M read as 0) into sw, then each lane
+// reads back its own row's 32 values
+__device__ __forceinline__ void load_block_bf16(const __nv_bfloat16* base, int ld, int rbase, int col0, int M, int lane,
+                                                uint8_t* sw, float (&out)[32]) {
+#pragma unroll
+  for (int it = 0; it < 4; ++it) {
+    const int rr = it * 8 + lane / 4, ch = lane % 4;
+    uint4 u = make_uint4(0, 0, 0, 0);
+    if (rbase + rr < M) u = *reinterpret_cast<const uint4*>(base + static_cast<size_t>(rbase + rr) * ld + col0 + ch * 8);
+    sts128(sw64(sw, rr, ch), u);
+  }
+  __syncwarp();
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    const uint4 u = lds128u(sw64(sw, lane, j));
+    const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&u);
+#pragma unroll
+    for (int e = 0; e < 4; ++e) {
+      const float2 f = __bfloat1622float2(h[e]);
+      out[8 * j + 2 * e] = f.x;
+      out[8 * j + 2 * e + 1] = f.y;
+    }
+  }
+  __syncwarp();
+}
+// each lane's row of 32 values -> bf16 -> coalesced store of the block (rows >= M skipped)
+__device__ __forceinline__ void store_block_bf16(__nv_bfloat16* base, int ld, int rbase, int col0, int M, int lane,
+                                                 uint8_t* sw, const float (&v)[32]) {
+#pragma unroll
+  for (int j = 0; j < 4; ++j) {
+    uint4 u;
+    __nv_bfloat162* h = reinterpret_cast<__nv_bfloat162*>(&u);
+#pragma unroll
+    for (int e = 0; e < 4; ++e) h[e] = __floats2bfloat162_rn(v[8 * j + 2 * e], v[8 * j + 2 * e + 1]);
+    sts128(sw64(sw, lane, j), u);
+  }
+  __syncwarp();
+#pragma unroll
+  for (int it = 0; it < 4; ++it) {
+    const int rr = it * 8 + lane / 4, ch = lane % 4;
+    const uint4 u = lds128u(sw64(sw, rr, ch));
+    if (rbase + rr < M) *reinterpret_cast<uint4*>(base + static_cast<size_t>(rbase + rr) * ld + col0 + ch * 8) = u;
+  }
+  __syncwarp();
+}
+
+__device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool vec_ok, const uint32_t (&r)[32],
+                                                    int rbase, int lane, int col0, int M, int N, uint8_t* sw) {
+  if (col0 >= N) return;
+  if (!vec_ok || col0 + 32 > N) {   // warp-uniform: ragged column block or unaligned pitches
+    epilogue_chunk(ep, r, rbase + lane, col0, rbase + lane < M, N);
+    return;
+  }
+  float v[32];
+#pragma unroll
+  for (int j = 0; j < 32; ++j) v[j] = __uint_as_float(r[j]);
+  if (ep.bias) {
+#pragma unroll
+    for (int q = 0; q < 8; ++q) {
+      const float4 b = *reinterpret_cast<const float4*>(ep.bias + col0 + 4 * q);
+      v[4 * q] += b.x; v[4 * q + 1] += b.y; v[4 * q + 2] += b.z; v[4 * q + 3] += b.w;
+    }
+  }
+  if (ep.aux) {   // GeLU backward: D = acc * gelu'(Z)
+    float z[32];
+    load_block_bf16(ep.aux, ep.ld_aux, rbase, col0, M, lane, sw, z);
+#pragma unroll
+    for (int j = 0; j < 32; ++j) v[j] *= gelu_tanh_grad_f(z[j]);
+  }
+  if (ep.residual) {
+    float rr[32];
+    load_block_bf16(ep.residual, ep.ld_res, rbase, col0, M, lane, sw, rr);
+#pragma unroll
+    for (int j = 0; j < 32; ++j) v[j] += rr[j];
+  }
+  if (ep.out_f32) {
+#pragma unroll
+    for (int j = 0; j < 8; ++j)
+      sts128(sw128(sw, lane, j), make_uint4(__float_as_uint(v[4 * j]), __float_as_uint(v[4 * j + 1]),
+                                            __float_as_uint(v[4 * j + 2]), __float_as_uint(v[4 * j + 3])));
+    __syncwarp();
+#pragma unroll
+    for (int it = 0; it < 8; ++it) {
+      const int rr = it * 4 + lane / 8, ch = lane % 8;
+      const uint4 u = lds128u(sw128(sw, rr, ch));
+      if (rbase + rr < M) {
+        float* d = ep.d_f32 + static_cast<size_t>(rbase + rr) * ep.ldd + col0 + ch * 4;
+        float4 o = make_float4(__uint_as_float(u.x), __uint_as_float(u.y), __uint_as_float(u.z), __uint_as_float(u.w));
+        if (ep.beta != 0.f) {
+          const float4 old = *reinterpret_cast<const float4*>(d);
+          o.x += ep.beta * old.x; o.y += ep.beta * old.y; o.z += ep.beta * old.z; o.w += ep.beta * old.w;
+        }
+        *reinterpret_cast<float4*>(d) = o;
+      }
+    }
+    __syncwarp();
+  } else {
+    store_block_bf16(ep.d_bf16, ep.ldd, rbase, col0, M, lane, sw, v);
+    if (ep.d2_bf16) {
+#pragma unroll
+      for (int j = 0; j < 32; ++j) v[j] = gelu_tanh_f(v[j]);
+      store_block_bf16(ep.d2_bf16, ep.ldd, rbase, col0, M, lane, sw, v);
     }
   }
 }
@@ -229,6 +363,8 @@ gemm_bf16_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
   } else {
     // ===================== epilogue (warps 2..5) =====================
     const int quarter = warp & 3;               // TMEM lanes [32*quarter, 32*quarter+32)
+    uint8_t* sw = smem + C::kStages * C::kStageBytes + 256 + (warp - 2) * 4096;
+    const bool vec_ok = epilogue_vec_ok(ep);
     int t = 0;
     for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++t) {
       const int acc = t & 1;
@@ -237,14 +373,13 @@ gemm_bf16_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
       const int m0 = tm * BM, n0 = tn * BN;
       mbar_wait(&tfull[acc], acc_ph);
       tc_fence_after();
-      const int row = m0 + quarter * 32 + lane;
-      const bool row_ok = row < M;
+      const int rbase = m0 + quarter * 32;
 #pragma unroll 1
       for (int c = 0; c < BN / 32; ++c) {
         uint32_t r[32];
         tmem_ld_32x32b_x32(tmem_base + acc * BN + c * 32 + (static_cast<uint32_t>(quarter * 32) << 16), r);
         tmem_ld_wait();
-        epilogue_chunk(ep, r, row, n0 + c * 32, row_ok, N);
+        epilogue_chunk_warp(ep, vec_ok, r, rbase, lane, n0 + c * 32, M, N, sw);
       }
       tc_fence_before();
       mbar_arrive(&tempty[acc]);
@@ -268,7 +403,7 @@ struct Cfg2 {                                             // BNP = N of the pair
   static constexpr int kBBytes = (BNP / 2) * BK * 2;      // one CTA's half of B per stage
   static constexpr int kStageBytes = kABytes + kBBytes;
   static constexpr int kStages = BNP == 256 ? 6 : 8;
-  static constexpr int kSmem = kStages * kStageBytes + 1024 + 256;
+  static constexpr int kSmem = kStages * kStageBytes + 1024 + 256 + 8 * 4096 /*epilogue staging*/;
   static constexpr int kTmem = 2 * BNP;
 };
 
@@ -366,6 +501,8 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
   } else {
     const int quarter = warp & 3, half = (warp - 2) >> 2;   // column half of the 256-wide tile
     const uint32_t tempty_leader0 = mapa(&tempty[0], 0), tempty_leader1 = mapa(&tempty[1], 0);
+    uint8_t* sw = smem + kStages2 * kStage2Bytes + 256 + (warp - 2) * 4096;
+    const bool vec_ok = epilogue_vec_ok(ep);
     int t = 0;
     for (int tile = pair; tile < num_tiles; tile += npairs, ++t) {
       const int acc = t & 1;
@@ -374,15 +511,14 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
       const int m0 = tm * 256 + 128 * rank, n0 = tn * BNP;
       mbar_wait(&tfull[acc], acc_ph);
       tc_fence_after();
-      const int row = m0 + quarter * 32 + lane;
-      const bool row_ok = row < M;
+      const int rbase = m0 + quarter * 32;
 #pragma unroll 1
       for (int c = 0; c < BNP / 64; ++c) {
         uint32_t r[32];
         const int col = half * (BNP / 2) + c * 32;
         tmem_ld_32x32b_x32(tmem_base + acc * BNP + col + (static_cast<uint32_t>(quarter * 32) << 16), r);
         tmem_ld_wait();
-        epilogue_chunk(ep, r, row, n0 + col, row_ok, N);
+        epilogue_chunk_warp(ep, vec_ok, r, rbase, lane, n0 + col, M, N, sw);
       }
       tc_fence_before();
       __syncwarp();
