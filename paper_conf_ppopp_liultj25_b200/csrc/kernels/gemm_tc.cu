@@ -237,6 +237,17 @@ __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool
     for (int j = 0; j < 32; ++j) v[j] += rr[j];
   }
   if (ep.out_f32) {
+    // issue the coalesced reads of the old D first so their latency overlaps the transposition
+    float4 old[8];
+    if (ep.beta != 0.f) {
+#pragma unroll
+      for (int it = 0; it < 8; ++it) {
+        const int rr = it * 4 + lane / 8, ch = lane % 8;
+        old[it] = rbase + rr < M ? *reinterpret_cast<const float4*>(ep.d_f32 + static_cast<size_t>(rbase + rr) * ep.ldd +
+                                                                    col0 + ch * 4)
+                                 : make_float4(0.f, 0.f, 0.f, 0.f);
+      }
+    }
 #pragma unroll
     for (int j = 0; j < 8; ++j)
       sts128(sw128(sw, lane, j), make_uint4(__float_as_uint(v[4 * j]), __float_as_uint(v[4 * j + 1]),
@@ -250,8 +261,7 @@ __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool
         float* d = ep.d_f32 + static_cast<size_t>(rbase + rr) * ep.ldd + col0 + ch * 4;
         float4 o = make_float4(__uint_as_float(u.x), __uint_as_float(u.y), __uint_as_float(u.z), __uint_as_float(u.w));
         if (ep.beta != 0.f) {
-          const float4 old = *reinterpret_cast<const float4*>(d);
-          o.x += ep.beta * old.x; o.y += ep.beta * old.y; o.z += ep.beta * old.z; o.w += ep.beta * old.w;
+          o.x += ep.beta * old[it].x; o.y += ep.beta * old[it].y; o.z += ep.beta * old[it].z; o.w += ep.beta * old[it].w;
         }
         *reinterpret_cast<float4*>(d) = o;
       }
