@@ -27,6 +27,7 @@ _SIGS = {
     "mario_k_softmax_ce": (i32, [vp, vp, i32, i32, i32, i32, f32, vp, vp, i32, vp]),
     "mario_kernel_launches": (C.c_longlong, []),
     "mario_k_gemm_set_variant": (i32, [i32]),
+    "mario_k_gemm_set_streamk": (i32, [i32]),
     "mario_k_attn_set_variant": (i32, [i32]),
     "mario_kstats_enable": (i32, [i32]),
     "mario_kstats_read": (i32, [i32, C.POINTER(C.c_double), C.POINTER(C.c_double), C.POINTER(C.c_double),

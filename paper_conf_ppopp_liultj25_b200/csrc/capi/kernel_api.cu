@@ -5,7 +5,7 @@
 #include "../kernels/layers.h"
 #include "../../../include/mario_kernels.h"
 
-namespace mario { extern int g_gemm_variant; extern int g_attn_variant; }
+namespace mario { extern int g_gemm_variant; extern int g_attn_variant; extern int g_gemm_streamk; }
 using namespace mario;
 
 extern "C" int mario_k_gemm_set_variant(int variant) {
@@ -29,6 +29,12 @@ extern "C" int mario_k_gemm_bf16(const void* A, int lda, int a_mn, const void* B
   g.ep.d2_bf16 = static_cast<__nv_bfloat16*>(D2);
   g.ep.aux = static_cast<const __nv_bfloat16*>(aux); g.ep.ld_aux = ld_aux;
   return static_cast<int>(gemm_bf16(g, static_cast<cudaStream_t>(stream)));
+}
+
+extern "C" int mario_k_gemm_set_streamk(int on) {
+  if (on != 0 && on != 1) return 1;
+  g_gemm_streamk = on;
+  return 0;
 }
 
 extern "C" int mario_k_attn_set_variant(int variant) {

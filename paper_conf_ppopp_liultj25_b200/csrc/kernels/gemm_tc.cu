@@ -22,6 +22,7 @@
 #include <cuda_runtime.h>
 #include <cuda_bf16.h>
 #include <cstdio>
+#include <map>
 #include <mutex>
 
 #include "sm100.cuh"
@@ -31,6 +32,8 @@
 namespace mario {
 
 using namespace sm100;
+
+int g_gemm_streamk = 1;   // mario_k_gemm_set_streamk
 
 namespace {
 
@@ -417,10 +420,53 @@ struct Cfg2 {                                             // BNP = N of the pair
   static constexpr int kTmem = 2 * BNP;
 };
 
+// Stream-K decomposition of the pair kernel (BNP = 256): the num_tiles * nk k-block iterations are
+// cut into npairs equal contiguous ranges; pair p runs the (tile, [kb0, kb1)) units of its range in
+// order. A tile split between pairs is finished by the unit holding k-block 0 (the LAST unit of
+// the earlier pair); every later part is the FIRST unit of a later pair q, which stores its raw
+// fp32 accumulators to ws[q] and raises flags[q] (per CTA of the pair). The finisher waits for
+// its contributors (already done: they ran first), adds them in pair order (deterministic) and
+// runs the normal epilogue. Waits only point to higher pair indices, so with in-order CTA dispatch
+// no cycle can form even when not every pair is resident.
+struct StreamK {
+  int on = 0;
+  float* ws = nullptr;     // [npairs][2 CTAs][128 rows][256 cols] fp32
+  int* flags = nullptr;    // [npairs][2], zero between launches
+};
+struct SkUnit { int tile, kb0, kb1; };
+struct SkIter {
+  long long it, it1;   // stream-K: global k-block iteration range
+  int tile, stride;    // tile-per-pair mode
+  __device__ bool next(bool sk, int nk, int num_tiles, SkUnit& u) {
+    if (sk) {
+      if (it >= it1) return false;
+      u.tile = static_cast<int>(it / nk);
+      u.kb0 = static_cast<int>(it % nk);
+      const long long rem = it1 - it;
+      u.kb1 = rem < nk - u.kb0 ? u.kb0 + static_cast<int>(rem) : nk;
+      it += u.kb1 - u.kb0;
+      return true;
+    }
+    if (tile >= num_tiles) return false;
+    u.tile = tile; u.kb0 = 0; u.kb1 = nk;
+    tile += stride;
+    return true;
+  }
+};
+__device__ __forceinline__ long long sk_bound(int q, long long I, int P) { return static_cast<long long>(q) * I / P; }
+__device__ __forceinline__ int ld_acquire(const int* p) {
+  int v;
+  asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void st_release(int* p, int v) {
+  asm volatile("st.release.gpu.global.b32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
+}
+
 template <int BNP, bool A_MN, bool B_MN>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads2, 1)
 gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-                     GemmEpilogue ep, int M, int N, int K, int n_fastest) {
+                     GemmEpilogue ep, int M, int N, int K, int n_fastest, StreamK sk) {
   using C2 = Cfg2<BNP>;
   constexpr int kStages2 = C2::kStages, kStage2Bytes = C2::kStageBytes, kHalfBytes = C2::kABytes;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -438,6 +484,8 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
   const int num_m = (M + 255) / 256, num_n = (N + BNP - 1) / BNP;
   const int num_tiles = num_m * num_n;
   const int nk = (K + BK - 1) / BK;
+  const bool skon = sk.on != 0;
+  const long long I = static_cast<long long>(num_tiles) * nk;
 
   if (warp == 0 && lane == 0) {
     tma_prefetch_desc(&tmA);
@@ -455,10 +503,13 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
   if (warp == 0) {
     if (elect_one()) {
       int s = 0; uint32_t ph = 0;
-      for (int tile = pair; tile < num_tiles; tile += npairs) {
+      SkIter itr{sk_bound(pair, I, npairs), sk_bound(pair + 1, I, npairs), pair, npairs};
+      SkUnit u;
+      while (itr.next(skon, nk, num_tiles, u)) {
+        const int tile = u.tile;
         const int tm = n_fastest ? tile / num_n : tile % num_m, tn = n_fastest ? tile % num_n : tile / num_m;
         const int m0 = tm * 256 + 128 * rank, n0 = tn * BNP + (BNP / 2) * rank;
-        for (int kb = 0; kb < nk; ++kb) {
+        for (int kb = u.kb0; kb < u.kb1; ++kb) {
           mbar_wait(&empty[s], ph ^ 1);
           uint8_t* sa = smem + s * kStage2Bytes;
           uint8_t* sb = sa + kHalfBytes;
@@ -482,13 +533,15 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
     if (leader) {
       constexpr uint32_t idesc = umma_idesc_bf16(256, BNP, A_MN ? 1 : 0, B_MN ? 1 : 0);
       int s = 0; uint32_t ph = 0; int t = 0;
-      for (int tile = pair; tile < num_tiles; tile += npairs, ++t) {
+      SkIter itr{sk_bound(pair, I, npairs), sk_bound(pair + 1, I, npairs), pair, npairs};
+      SkUnit u;
+      for (; itr.next(skon, nk, num_tiles, u); ++t) {
         const int acc = t & 1;
         const uint32_t acc_ph = (t >> 1) & 1;
         mbar_wait(&tempty[acc], acc_ph ^ 1);
         tc_fence_after();
         const uint32_t d_tmem = tmem_base + acc * BNP;
-        for (int kb = 0; kb < nk; ++kb) {
+        for (int kb = u.kb0; kb < u.kb1; ++kb) {
           mbar_wait(&full[s], ph);
           tc_fence_after();
           if (elect_one()) {
@@ -498,10 +551,10 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
             for (int kk = 0; kk < BK / 16; ++kk) {
               const uint64_t ad = A_MN ? umma_desc_sw128(sa + kk * 2048, 8192, 1024) : umma_desc_sw128(sa + kk * 32, 16, 1024);
               const uint64_t bd = B_MN ? umma_desc_sw128(sb + kk * 2048, 8192, 1024) : umma_desc_sw128(sb + kk * 32, 16, 1024);
-              umma_bf16_2sm(d_tmem, ad, bd, idesc, (kb | kk) != 0);
+              umma_bf16_2sm(d_tmem, ad, bd, idesc, (kb != u.kb0) || kk != 0);
             }
             umma_commit_2sm(&empty[s], 0x3);
-            if (kb == nk - 1) umma_commit_2sm(&tfull[acc], 0x3);
+            if (kb == u.kb1 - 1) umma_commit_2sm(&tfull[acc], 0x3);
           }
           __syncwarp();
           if (++s == kStages2) { s = 0; ph ^= 1; }
@@ -514,7 +567,11 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
     uint8_t* sw = smem + kStages2 * kStage2Bytes + 256 + (warp - 2) * 4096;
     const bool vec_ok = epilogue_vec_ok(ep);
     int t = 0;
-    for (int tile = pair; tile < num_tiles; tile += npairs, ++t) {
+    SkIter itr{sk_bound(pair, I, npairs), sk_bound(pair + 1, I, npairs), pair, npairs};
+    SkUnit u;
+    const int etid = threadIdx.x - 64;   // 0..255 over the epilogue warps
+    for (; itr.next(skon, nk, num_tiles, u); ++t) {
+      const int tile = u.tile;
       const int acc = t & 1;
       const uint32_t acc_ph = (t >> 1) & 1;
       const int tm = n_fastest ? tile / num_n : tile % num_m, tn = n_fastest ? tile % num_n : tile / num_m;
@@ -522,13 +579,61 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
       mbar_wait(&tfull[acc], acc_ph);
       tc_fence_after();
       const int rbase = m0 + quarter * 32;
+      const int lrow = quarter * 32 + lane;                     // accumulator row within this CTA
+      if (skon && u.kb0 != 0) {
+        // later k-part of a split tile (this pair's first unit): raw partial to ws[pair]
+        float* wp = sk.ws + ((static_cast<size_t>(pair) * 2 + rank) * 128 + lrow) * 256;
 #pragma unroll 1
-      for (int c = 0; c < BNP / 64; ++c) {
-        uint32_t r[32];
-        const int col = half * (BNP / 2) + c * 32;
-        tmem_ld_32x32b_x32(tmem_base + acc * BNP + col + (static_cast<uint32_t>(quarter * 32) << 16), r);
-        tmem_ld_wait();
-        epilogue_chunk_warp(ep, vec_ok, r, rbase, lane, n0 + col, M, N, sw);
+        for (int c = 0; c < BNP / 64; ++c) {
+          uint32_t r[32];
+          const int col = half * (BNP / 2) + c * 32;
+          tmem_ld_32x32b_x32(tmem_base + acc * BNP + col + (static_cast<uint32_t>(quarter * 32) << 16), r);
+          tmem_ld_wait();
+#pragma unroll
+          for (int q = 0; q < 8; ++q)
+            *reinterpret_cast<uint4*>(wp + col + 4 * q) = make_uint4(r[4 * q], r[4 * q + 1], r[4 * q + 2], r[4 * q + 3]);
+        }
+        __threadfence();
+        asm volatile("bar.sync 1, 256;" ::: "memory");
+        if (etid == 0) st_release(&sk.flags[pair * 2 + rank], 1);
+      } else {
+        // contributors of a tile whose k-block 0 this unit holds: pairs q > pair starting inside the tile
+        int q1 = pair + 1;
+        if (skon && u.kb1 < nk) {
+          const long long tend = static_cast<long long>(tile + 1) * nk;
+          while (q1 < npairs && sk_bound(q1, I, npairs) < tend) ++q1;
+          if (etid == 0)
+            for (int q = pair + 1; q < q1; ++q)
+              if (sk_bound(q + 1, I, npairs) > sk_bound(q, I, npairs))   // empty ranges contribute nothing
+                while (ld_acquire(&sk.flags[q * 2 + rank]) == 0) __nanosleep(64);
+          asm volatile("bar.sync 1, 256;" ::: "memory");
+        }
+#pragma unroll 1
+        for (int c = 0; c < BNP / 64; ++c) {
+          uint32_t r[32];
+          const int col = half * (BNP / 2) + c * 32;
+          tmem_ld_32x32b_x32(tmem_base + acc * BNP + col + (static_cast<uint32_t>(quarter * 32) << 16), r);
+          tmem_ld_wait();
+          for (int q = pair + 1; q < q1; ++q) {
+            if (sk_bound(q + 1, I, npairs) == sk_bound(q, I, npairs)) continue;
+            const float* wp = sk.ws + ((static_cast<size_t>(q) * 2 + rank) * 128 + lrow) * 256 + col;
+#pragma unroll
+            for (int e = 0; e < 8; ++e) {
+              const float4 pv = *reinterpret_cast<const float4*>(wp + 4 * e);
+              r[4 * e] = __float_as_uint(__uint_as_float(r[4 * e]) + pv.x);
+              r[4 * e + 1] = __float_as_uint(__uint_as_float(r[4 * e + 1]) + pv.y);
+              r[4 * e + 2] = __float_as_uint(__uint_as_float(r[4 * e + 2]) + pv.z);
+              r[4 * e + 3] = __float_as_uint(__uint_as_float(r[4 * e + 3]) + pv.w);
+            }
+          }
+          epilogue_chunk_warp(ep, vec_ok, r, rbase, lane, n0 + col, M, N, sw);
+        }
+        if (q1 > pair + 1) {
+          asm volatile("bar.sync 1, 256;" ::: "memory");
+          if (etid == 0)
+            for (int q = pair + 1; q < q1; ++q)
+              if (sk_bound(q + 1, I, npairs) > sk_bound(q, I, npairs)) sk.flags[q * 2 + rank] = 0;
+        }
       }
       tc_fence_before();
       __syncwarp();
@@ -606,6 +711,39 @@ cudaError_t launch_bn(const GemmArgs& g, cudaStream_t st, int num_sms) {
 }
 
 
+// stream-K when whole tiles would leave more than 5% of the last wave's pair slots idle
+bool use_streamk(long tiles, long pairs, int nk) {
+  if (!g_gemm_streamk || pairs < 2 || nk < 2) return false;
+  const long waves = (tiles + pairs - 1) / pairs;
+  return static_cast<double>(tiles) / static_cast<double>(waves * pairs) < 0.95;
+}
+
+// per-device partial-tile workspace [pairs][2][128][256] fp32 + zeroed flags, allocated on first
+// use outside stream capture (a captured launch without it runs tile-per-pair instead)
+bool streamk_workspace(int pairs, cudaStream_t st, float** ws, int** flags) {
+  static std::mutex mu;
+  static std::map<int, std::pair<float*, int*>> bufs;
+  int dev = 0;
+  cudaGetDevice(&dev);
+  std::lock_guard<std::mutex> lk(mu);
+  auto it = bufs.find(dev);
+  if (it == bufs.end()) {
+    cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+    if (cudaStreamIsCapturing(st, &cs) != cudaSuccess || cs != cudaStreamCaptureStatusNone) return false;
+    float* w = nullptr;
+    int* f = nullptr;
+    const size_t wb = static_cast<size_t>(pairs) * 2 * 128 * 256 * sizeof(float);
+    if (cudaMalloc(&w, wb) != cudaSuccess) return false;
+    if (cudaMalloc(&f, static_cast<size_t>(pairs) * 2 * sizeof(int)) != cudaSuccess) { cudaFree(w); return false; }
+    if (cudaMemset(f, 0, static_cast<size_t>(pairs) * 2 * sizeof(int)) != cudaSuccess) return false;
+    cudaDeviceSynchronize();
+    it = bufs.emplace(dev, std::make_pair(w, f)).first;
+  }
+  *ws = it->second.first;
+  *flags = it->second.second;
+  return true;
+}
+
 template <int BNP, bool A_MN, bool B_MN>
 cudaError_t launch_pair(const GemmArgs& g, cudaStream_t st, int num_sms) {
   using C2 = Cfg2<BNP>;
@@ -624,11 +762,20 @@ cudaError_t launch_pair(const GemmArgs& g, cudaStream_t st, int num_sms) {
     attr_set = true;
   }
   const int tiles = ((g.M + 255) / 256) * ((g.N + BNP - 1) / BNP);
-  const int pairs = tiles < num_sms / 2 ? tiles : num_sms / 2;
+  int pairs = tiles < num_sms / 2 ? tiles : num_sms / 2;
+  StreamK sk;
+  if (BNP == 256 && use_streamk(tiles, num_sms / 2, (g.K + BK - 1) / BK)) {
+    float* ws = nullptr;
+    int* flags = nullptr;
+    if (streamk_workspace(num_sms / 2, st, &ws, &flags)) {
+      sk.on = 1; sk.ws = ws; sk.flags = flags;
+      pairs = num_sms / 2;
+    }
+  }
   const int tok = kstats_begin(K_GEMM, 2.0 * g.M * g.N * g.K,
                                2.0 * (double(g.M) * g.K + double(g.N) * g.K) + (g.ep.out_f32 ? 4.0 : 2.0) * g.M * g.N, st);
   const int n_fastest = static_cast<long>(g.M) >= static_cast<long>(g.N) ? 1 : 0;
-  kern<<<2 * pairs, kThreads2, C2::kSmem, st>>>(ta, tb, g.ep, g.M, g.N, g.K, n_fastest);
+  kern<<<2 * pairs, kThreads2, C2::kSmem, st>>>(ta, tb, g.ep, g.M, g.N, g.K, n_fastest, sk);
   kstats_end(tok, st);
   note_launch();
   return cudaGetLastError();
