@@ -434,26 +434,31 @@ struct StreamK {
   int* flags = nullptr;    // [npairs][2], zero between launches
 };
 struct SkUnit { int tile, kb0, kb1; };
+// Hybrid order: whole tiles [0, dp_tiles) round-robin over the pairs first (full waves, operand
+// panels shared in L2 by the concurrently running band of tiles), then the remaining tiles'
+// k-blocks split evenly (stream-K), so only the last partial wave is divided.
 struct SkIter {
-  long long it, it1;   // stream-K: global k-block iteration range
-  int tile, stride;    // tile-per-pair mode
-  __device__ bool next(bool sk, int nk, int num_tiles, SkUnit& u) {
-    if (sk) {
-      if (it >= it1) return false;
-      u.tile = static_cast<int>(it / nk);
-      u.kb0 = static_cast<int>(it % nk);
-      const long long rem = it1 - it;
-      u.kb1 = rem < nk - u.kb0 ? u.kb0 + static_cast<int>(rem) : nk;
-      it += u.kb1 - u.kb0;
+  int tile, stride, dp_tiles;   // data-parallel phase
+  long long it, it1;            // stream-K phase: global k-block iteration range of this pair
+  __device__ bool next(int nk, SkUnit& u) {
+    if (tile < dp_tiles) {
+      u.tile = tile; u.kb0 = 0; u.kb1 = nk;
+      tile += stride;
       return true;
     }
-    if (tile >= num_tiles) return false;
-    u.tile = tile; u.kb0 = 0; u.kb1 = nk;
-    tile += stride;
+    if (it >= it1) return false;
+    u.tile = static_cast<int>(it / nk);
+    u.kb0 = static_cast<int>(it % nk);
+    const long long rem = it1 - it;
+    u.kb1 = rem < nk - u.kb0 ? u.kb0 + static_cast<int>(rem) : nk;
+    it += u.kb1 - u.kb0;
     return true;
   }
 };
-__device__ __forceinline__ long long sk_bound(int q, long long I, int P) { return static_cast<long long>(q) * I / P; }
+// first stream-K iteration of pair q
+__device__ __forceinline__ long long sk_bound(int q, long long I0, long long Isk, int P) {
+  return I0 + static_cast<long long>(q) * Isk / P;
+}
 __device__ __forceinline__ int ld_acquire(const int* p) {
   int v;
   asm volatile("ld.acquire.gpu.global.b32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
@@ -485,7 +490,8 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
   const int num_tiles = num_m * num_n;
   const int nk = (K + BK - 1) / BK;
   const bool skon = sk.on != 0;
-  const long long I = static_cast<long long>(num_tiles) * nk;
+  const int dp_tiles = skon ? (num_tiles / npairs) * npairs : num_tiles;
+  const long long I0 = static_cast<long long>(dp_tiles) * nk, Isk = static_cast<long long>(num_tiles - dp_tiles) * nk;
 
   if (warp == 0 && lane == 0) {
     tma_prefetch_desc(&tmA);
@@ -503,9 +509,9 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
   if (warp == 0) {
     if (elect_one()) {
       int s = 0; uint32_t ph = 0;
-      SkIter itr{sk_bound(pair, I, npairs), sk_bound(pair + 1, I, npairs), pair, npairs};
+      SkIter itr{pair, npairs, dp_tiles, sk_bound(pair, I0, Isk, npairs), sk_bound(pair + 1, I0, Isk, npairs)};
       SkUnit u;
-      while (itr.next(skon, nk, num_tiles, u)) {
+      while (itr.next(nk, u)) {
         const int tile = u.tile;
         const int tm = n_fastest ? tile / num_n : tile % num_m, tn = n_fastest ? tile % num_n : tile / num_m;
         const int m0 = tm * 256 + 128 * rank, n0 = tn * BNP + (BNP / 2) * rank;
@@ -533,9 +539,9 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
     if (leader) {
       constexpr uint32_t idesc = umma_idesc_bf16(256, BNP, A_MN ? 1 : 0, B_MN ? 1 : 0);
       int s = 0; uint32_t ph = 0; int t = 0;
-      SkIter itr{sk_bound(pair, I, npairs), sk_bound(pair + 1, I, npairs), pair, npairs};
+      SkIter itr{pair, npairs, dp_tiles, sk_bound(pair, I0, Isk, npairs), sk_bound(pair + 1, I0, Isk, npairs)};
       SkUnit u;
-      for (; itr.next(skon, nk, num_tiles, u); ++t) {
+      for (; itr.next(nk, u); ++t) {
         const int acc = t & 1;
         const uint32_t acc_ph = (t >> 1) & 1;
         mbar_wait(&tempty[acc], acc_ph ^ 1);
@@ -567,10 +573,10 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
     uint8_t* sw = smem + kStages2 * kStage2Bytes + 256 + (warp - 2) * 4096;
     const bool vec_ok = epilogue_vec_ok(ep);
     int t = 0;
-    SkIter itr{sk_bound(pair, I, npairs), sk_bound(pair + 1, I, npairs), pair, npairs};
+    SkIter itr{pair, npairs, dp_tiles, sk_bound(pair, I0, Isk, npairs), sk_bound(pair + 1, I0, Isk, npairs)};
     SkUnit u;
     const int etid = threadIdx.x - 64;   // 0..255 over the epilogue warps
-    for (; itr.next(skon, nk, num_tiles, u); ++t) {
+    for (; itr.next(nk, u); ++t) {
       const int tile = u.tile;
       const int acc = t & 1;
       const uint32_t acc_ph = (t >> 1) & 1;
@@ -601,10 +607,10 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
         int q1 = pair + 1;
         if (skon && u.kb1 < nk) {
           const long long tend = static_cast<long long>(tile + 1) * nk;
-          while (q1 < npairs && sk_bound(q1, I, npairs) < tend) ++q1;
+          while (q1 < npairs && sk_bound(q1, I0, Isk, npairs) < tend) ++q1;
           if (etid == 0)
             for (int q = pair + 1; q < q1; ++q)
-              if (sk_bound(q + 1, I, npairs) > sk_bound(q, I, npairs))   // empty ranges contribute nothing
+              if (sk_bound(q + 1, I0, Isk, npairs) > sk_bound(q, I0, Isk, npairs))   // empty ranges contribute nothing
                 while (ld_acquire(&sk.flags[q * 2 + rank]) == 0) __nanosleep(64);
           asm volatile("bar.sync 1, 256;" ::: "memory");
         }
@@ -615,7 +621,7 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
           tmem_ld_32x32b_x32(tmem_base + acc * BNP + col + (static_cast<uint32_t>(quarter * 32) << 16), r);
           tmem_ld_wait();
           for (int q = pair + 1; q < q1; ++q) {
-            if (sk_bound(q + 1, I, npairs) == sk_bound(q, I, npairs)) continue;
+            if (sk_bound(q + 1, I0, Isk, npairs) == sk_bound(q, I0, Isk, npairs)) continue;
             const float* wp = sk.ws + ((static_cast<size_t>(q) * 2 + rank) * 128 + lrow) * 256 + col;
 #pragma unroll
             for (int e = 0; e < 8; ++e) {
@@ -632,7 +638,7 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
           asm volatile("bar.sync 1, 256;" ::: "memory");
           if (etid == 0)
             for (int q = pair + 1; q < q1; ++q)
-              if (sk_bound(q + 1, I, npairs) > sk_bound(q, I, npairs)) sk.flags[q * 2 + rank] = 0;
+              if (sk_bound(q + 1, I0, Isk, npairs) > sk_bound(q, I0, Isk, npairs)) sk.flags[q * 2 + rank] = 0;
         }
       }
       tc_fence_before();
