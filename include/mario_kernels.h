@@ -35,11 +35,13 @@ int mario_k_gemm_bf16(const void* A, int lda, int a_mn, const void* B, int ldb, 
  * 128x256/128x128), 0 = single-CTA only, 1 = CTA pair whenever M, N >= 256 (auto N),
  * 2 = CTA pair 256x128, 3 = CTA pair 256x256. Process-global; returns 0, or 1 if invalid. */
 int mario_k_gemm_set_variant(int variant);
-/* Stream-K for the 256x256 CTA-pair kernel (1 = on, default): when whole tiles would leave > 5% of
+/* Stream-K for the 256x256 CTA-pair kernel (0 = off, default; 1 = on): when whole tiles would leave > 5% of
  * the last wave idle, every pair runs an equal contiguous share of the (tile, k-block) iterations;
  * a tile split between pairs is finished by the part holding k-block 0, which adds the other
  * parts' fp32 partials (library-owned per-device workspace, ~19 MB) in pair order — deterministic.
- * GEMMs using it must not run concurrently on two streams of one device. Returns 0, or 1. */
+ * GEMMs using it must not run concurrently on two streams of one device. Measured on B200 at the cfg-2
+ * layer shapes: no faster than whole tiles (the chip is power-capped, so idle SMs in the last wave
+ * raise the clock of the busy ones; K = 2048 parts cost more in fix-up than they save). Returns 0, or 1. */
 int mario_k_gemm_set_streamk(int on);
 
 /* K4: the same contract in true fp32 on CUDA cores (fp32 mode, reading A6). */

@@ -33,7 +33,7 @@ namespace mario {
 
 using namespace sm100;
 
-int g_gemm_streamk = 1;   // mario_k_gemm_set_streamk
+int g_gemm_streamk = 0;   // mario_k_gemm_set_streamk (off: measured no gain under the power cap)
 
 namespace {
 

@@ -122,11 +122,13 @@ def test_gemm_streamk(sk, a_mn, b_mn, out_f32):
             _run(a_mn, b_mn, 2184, 1280, 2112, out_f32=False, aux=True)
             _run(a_mn, b_mn, 2184, 1280, 2112, out_f32=False, bias=True, gelu2=True)
     finally:
-        L.mario_k_gemm_set_streamk(1)
+        L.mario_k_gemm_set_streamk(0)
 
 
-def test_gemm_streamk_deterministic():
+@pytest.mark.parametrize("sk", [1, 0], ids=["streamk", "tiles"])
+def test_gemm_streamk_deterministic(sk):
     L = _lib.lib()
+    assert L.mario_k_gemm_set_streamk(sk) == 0
     g = torch.Generator(device="cuda").manual_seed(3)
     M, N, K = 8192, 2048, 8192
     A = torch.randn(M, K, device="cuda", generator=g).bfloat16()
@@ -138,6 +140,7 @@ def test_gemm_streamk_deterministic():
                                    None, N, None, None, N, None) == 0
         outs.append(D)
     torch.cuda.synchronize()
+    L.mario_k_gemm_set_streamk(0)
     assert torch.equal(outs[0], outs[1]) and torch.equal(outs[0], outs[2])
     ref = A.float() @ B.float().t()
     assert (outs[0].float() - ref).abs().max().item() <= 1e-2 * ref.abs().max().item()
