@@ -157,7 +157,7 @@ struct Exec {
   // D[M,N] = A[M,K] . B[N,K]^T  (see kernels.h); bf16 tcgen05 or fp32 SIMT by dtype.
   void gemm(const T* A, int lda, int a_mn, const T* B, int ldb, int b_mn, int M, int N, int K, void* Dp, int ldd,
             bool out_f32, float beta, const float* bias = nullptr, const T* resid = nullptr, T* D2 = nullptr,
-            const T* aux = nullptr) {
+            const T* aux = nullptr, bool d2_from_aux = false) {
     if constexpr (sizeof(T) == 2) {
       GemmArgs g;
       g.A = A; g.lda = lda; g.a_mn = a_mn; g.B = B; g.ldb = ldb; g.b_mn = b_mn; g.M = M; g.N = N; g.K = K;
@@ -165,12 +165,13 @@ struct Exec {
       if (out_f32) g.ep.d_f32 = static_cast<float*>(Dp); else g.ep.d_bf16 = static_cast<__nv_bfloat16*>(Dp);
       g.ep.ldd = ldd; g.ep.beta = beta; g.ep.bias = bias;
       g.ep.residual = resid; g.ep.ld_res = ldd; g.ep.d2_bf16 = D2; g.ep.aux = aux; g.ep.ld_aux = ldd;
+      g.ep.d2_from_aux = d2_from_aux ? 1 : 0;
       CU(gemm_bf16(g, st));
     } else {
       GemmF32Args g;
       g.A = A; g.lda = lda; g.a_mn = a_mn; g.B = B; g.ldb = ldb; g.b_mn = b_mn; g.M = M; g.N = N; g.K = K;
       g.D = static_cast<float*>(Dp); g.ldd = ldd; g.beta = beta; g.bias = bias; g.residual = resid;
-      g.ld_res = ldd; g.D2 = D2; g.aux = aux; g.ld_aux = ldd;
+      g.ld_res = ldd; g.D2 = D2; g.aux = aux; g.ld_aux = ldd; g.d2_from_aux = d2_from_aux ? 1 : 0;
       CU(gemm_f32(g, st));
     }
   }
@@ -179,9 +180,9 @@ struct Exec {
                T* Y2 = nullptr) {
     gemm(X, in, 0, W, in, 0, Tn, out, in, Y, out, false, 0.f, bias, resid, Y2);
   }
-  // dX[T,in] = dY W (optionally * gelu'(aux))
-  void lin_dgrad(const T* dY, const T* W, int Tn, int out, int in, T* dX, const T* aux = nullptr) {
-    gemm(dY, out, 0, W, in, 1, Tn, in, out, dX, in, false, 0.f, nullptr, nullptr, nullptr, aux);
+  // dX[T,in] = dY W (optionally * gelu'(aux); G = gelu(aux) as a second output when G != NULL)
+  void lin_dgrad(const T* dY, const T* W, int Tn, int out, int in, T* dX, const T* aux = nullptr, T* G = nullptr) {
+    gemm(dY, out, 0, W, in, 1, Tn, in, out, dX, in, false, 0.f, nullptr, nullptr, G, aux, G != nullptr);
   }
   // dW[out,in] += dY^T X (fp32)
   void lin_wgrad(const T* dY, const T* X, int Tn, int out, int in, float* dW) {
@@ -351,11 +352,11 @@ struct Exec {
       T* dH1 = dHbuf[(cur + 1) % 3];
       T* dHin = (li == 0) ? (k == 0 ? dHbuf[(cur + 2) % 3] : dstage_in) : dHbuf[(cur + 2) % 3];
       if (gpt) {
-        gelu_fwd<T>(Z, Gt, static_cast<size_t>(Tn) * f, st);                 // recompute G = gelu(Z)
+        // dZ = (dH W2) * gelu'(Z); the epilogue also recomputes G = gelu(Z) for the fc2 wgrad
+        lin_dgrad(dH, Wm(D, p, pre + "fc2.w"), Tn, h, f, dZ, Z, Gt);
         lin_wgrad(dH, Gt, Tn, h, f, G(D, p, pre + "fc2.w"));
         // fc2.b: fused into the norm backward that wrote dH (this stage), else a column sum here
         if (li == lps - 1 && k != K - 1) colsum<T>(dH, nullptr, nullptr, Tn, h, h, 0, G(D, p, pre + "fc2.b"), nullptr, red, st);
-        lin_dgrad(dH, Wm(D, p, pre + "fc2.w"), Tn, h, f, dZ, Z);           // dZ = (dH W2) * gelu'(Z)
         layernorm_fwd<T>(H1, Wf(D, p, pre + "ln2.g"), Wf(D, p, pre + "ln2.b"), A2, st2, Tn, h, m.norm_eps, st);
         lin_wgrad(dZ, A2, Tn, f, h, G(D, p, pre + "fc1.w"));
         colsum<T>(dZ, nullptr, nullptr, Tn, f, f, 0, G(D, p, pre + "fc1.b"), nullptr, red, st);

@@ -64,7 +64,7 @@ __global__ void __launch_bounds__(256) gemm_f32_kernel(GemmF32Args g) {
       float* d = g.D + (size_t)m * g.ldd + n;
       if (g.beta != 0.f) v += g.beta * *d;
       *d = v;
-      if (g.D2) g.D2[(size_t)m * g.ldd + n] = gelu_f(v);
+      if (g.D2) g.D2[(size_t)m * g.ldd + n] = (g.aux && g.d2_from_aux) ? gelu_f(g.aux[(size_t)m * g.ld_aux + n]) : gelu_f(v);
     }
   }
 }

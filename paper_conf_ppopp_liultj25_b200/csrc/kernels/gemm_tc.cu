@@ -75,10 +75,17 @@ __device__ __forceinline__ void epilogue_chunk(const GemmEpilogue& ep, const uin
 #pragma unroll
     for (int j = 0; j < 32; ++j) if (full_cols || col0 + j < N) v[j] += ep.bias[col0 + j];
   }
-  if (ep.aux) {  // GeLU backward: D = acc * gelu'(Z)
+  float g2[32];
+  const bool g_aux = ep.aux && ep.d2_from_aux;
+  if (ep.aux) {  // GeLU backward: D = acc * gelu'(Z) (and D2 = gelu(Z) when d2_from_aux)
     const __nv_bfloat16* z = ep.aux + static_cast<size_t>(row) * ep.ld_aux + col0;
 #pragma unroll
-    for (int j = 0; j < 32; ++j) if (full_cols || col0 + j < N) v[j] *= gelu_tanh_grad_f(__bfloat162float(z[j]));
+    for (int j = 0; j < 32; ++j)
+      if (full_cols || col0 + j < N) {
+        const float zz = __bfloat162float(z[j]);
+        v[j] *= gelu_tanh_grad_f(zz);
+        if (g_aux) g2[j] = gelu_tanh_f(zz);
+      }
   }
   if (ep.residual) {
     const __nv_bfloat16* rr = ep.residual + static_cast<size_t>(row) * ep.ld_res + col0;
@@ -122,7 +129,7 @@ __device__ __forceinline__ void epilogue_chunk(const GemmEpilogue& ep, const uin
 #pragma unroll
         for (int j = 0; j < 8; ++j) {
           h[j] = __float2bfloat16_rn(v[q * 8 + j]);
-          if (d2) h2[j] = __float2bfloat16_rn(gelu_tanh_f(v[q * 8 + j]));
+          if (d2) h2[j] = __float2bfloat16_rn(g_aux ? g2[q * 8 + j] : gelu_tanh_f(v[q * 8 + j]));
         }
         *reinterpret_cast<uint4*>(d + q * 8) = u;
         if (d2) *reinterpret_cast<uint4*>(d2 + q * 8) = u2;
@@ -130,7 +137,7 @@ __device__ __forceinline__ void epilogue_chunk(const GemmEpilogue& ep, const uin
     } else {
       for (int j = 0; j < 32; ++j) if (col0 + j < N) {
         d[j] = __float2bfloat16_rn(v[j]);
-        if (d2) d2[j] = __float2bfloat16_rn(gelu_tanh_f(v[j]));
+        if (d2) d2[j] = __float2bfloat16_rn(g_aux ? g2[j] : gelu_tanh_f(v[j]));
       }
     }
   }
@@ -227,8 +234,8 @@ __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool
       v[4 * q] += b.x; v[4 * q + 1] += b.y; v[4 * q + 2] += b.z; v[4 * q + 3] += b.w;
     }
   }
+  float z[32];
   if (ep.aux) {   // GeLU backward: D = acc * gelu'(Z)
-    float z[32];
     load_block_bf16(ep.aux, ep.ld_aux, rbase, col0, M, lane, sw, z);
 #pragma unroll
     for (int j = 0; j < 32; ++j) v[j] *= gelu_tanh_grad_f(z[j]);
@@ -273,8 +280,9 @@ __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool
   } else {
     store_block_bf16(ep.d_bf16, ep.ldd, rbase, col0, M, lane, sw, v);
     if (ep.d2_bf16) {
+      const bool g_aux = ep.aux && ep.d2_from_aux;
 #pragma unroll
-      for (int j = 0; j < 32; ++j) v[j] = gelu_tanh_f(v[j]);
+      for (int j = 0; j < 32; ++j) v[j] = gelu_tanh_f(g_aux ? z[j] : v[j]);
       store_block_bf16(ep.d2_bf16, ep.ldd, rbase, col0, M, lane, sw, v);
     }
   }

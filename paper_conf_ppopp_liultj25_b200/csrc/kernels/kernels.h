@@ -19,6 +19,7 @@ struct GemmEpilogue {
   const float* bias = nullptr;            // [N], added before activation / residual
   const __nv_bfloat16* residual = nullptr; int ld_res = 0;   // D += residual
   const __nv_bfloat16* aux = nullptr; int ld_aux = 0;        // D = acc * gelu'(aux)  (GeLU bwd)
+  int d2_from_aux = 0;                    // with aux: D2 = gelu(aux) (recomputed MLP activation)
 };
 
 struct GemmArgs {
@@ -43,6 +44,7 @@ struct GemmF32Args {
   const float* residual = nullptr; int ld_res = 0;
   float* D2 = nullptr;                  // gelu(D) second output
   const float* aux = nullptr; int ld_aux = 0;   // D = acc * gelu'(aux)
+  int d2_from_aux = 0;                  // with aux: D2 = gelu(aux)
 };
 cudaError_t gemm_f32(const GemmF32Args& g, cudaStream_t st);
 
