@@ -54,6 +54,18 @@ __device__ __forceinline__ float ld_shared_f32(const void* p) {
   return v;
 }
 
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+               :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void tma_store_2d(const void* tmap, const void* src, int c0, int c1) {
+  asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];"
+               :: "l"(reinterpret_cast<uint64_t>(tmap)), "r"(smem_u32(src)), "r"(c0), "r"(c1) : "memory");
+}
+__device__ __forceinline__ void bulk_commit_wait_read() {
+  asm volatile("cp.async.bulk.commit_group;" ::: "memory");
+  asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
+}
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void named_bar(int id, int n) { asm volatile("bar.sync %0, %1;" :: "r"(id), "r"(n) : "memory"); }
 
@@ -98,26 +110,24 @@ struct Smem {
 template <int DH>
 __global__ void __launch_bounds__(kThreadsB, 1)
 fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_qkv64,
-               const __grid_constant__ CUtensorMap tm_do64, const float* lse, const float* Dd, bf16* dqkv, int B,
-               int s, int nh) {
+               const __grid_constant__ CUtensorMap tm_do64, const __grid_constant__ CUtensorMap tm_dqkv,
+               const float* lse, const float* Dd, bf16* dqkv, int B, int s, int nh, int dbg) {
+  const bool bulk_ld = (s % kCols) == 0;
   using SM = Smem<DH>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sK = smem;
   uint8_t* sV = sK + SM::kBig;
-  uint8_t* sQ[kRingKV];
-  uint8_t* sG[kRingKV];
-  for (int r = 0; r < kRingKV; ++r) { sQ[r] = sV + SM::kBig + 2 * r * SM::kSmall; sG[r] = sQ[r] + SM::kSmall; }
+  // ring slot / buffer addresses as arithmetic (a runtime-indexed pointer array would live in local memory)
+  auto sQ = [&](int r) { return sV + SM::kBig + 2 * r * SM::kSmall; };
+  auto sG = [&](int r) { return sV + SM::kBig + 2 * r * SM::kSmall + SM::kSmall; };
   // P^T and dS^T double-buffered: tile idx + 1 is written while the dV/dK MMAs read tile idx
-  uint8_t* sP[2];
-  uint8_t* sS[2];
-  for (int i = 0; i < 2; ++i) {
-    sP[i] = sV + SM::kBig + 2 * kRingKV * SM::kSmall + 2 * i * SM::kP;
-    sS[i] = sP[i] + SM::kP;
-  }
-  float* sL = reinterpret_cast<float*>(sS[1] + SM::kP);    // [2][64] lse * log2e
-  float* sDv = sL + 2 * kCols;                             // [2][64] D
-  uint64_t* bar = reinterpret_cast<uint64_t*>(sDv + 2 * kCols);
+  auto sP = [&](int i) { return sV + SM::kBig + 2 * kRingKV * SM::kSmall + 2 * i * SM::kP; };
+  auto sS = [&](int i) { return sV + SM::kBig + 2 * kRingKV * SM::kSmall + 2 * i * SM::kP + SM::kP; };
+  // per ring slot: lse (natural log) and D of the slot's 64 queries, [kRingKV][2][64] fp32; TMA
+  // bulk-copied with the Q/dO tile when s % 64 == 0, else staged by the softmax warps
+  float* sLD = reinterpret_cast<float*>(sS(1) + SM::kP);
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sLD + kRingKV * 2 * kCols);
   uint64_t* kv_full = bar;                 // 1
   uint64_t* q_full = bar + 1;              // kRingKV
   uint64_t* q_empty = q_full + kRingKV;    // kRingKV
@@ -129,13 +139,15 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_done + 1);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-  // heaviest first: key tile 0 sees every query tile; blockIdx.x runs over (sample, head)
-  const int kt = blockIdx.y, b = blockIdx.x / nh, head = blockIdx.x % nh;
+  // heaviest first over all (sample, head) (key tile 0 sees every query tile); dbg bit 3: (sample, head)-major
+  const int nt = (s + kRows - 1) / kRows, BH = B * nh;
+  const int j = (dbg & 8) ? blockIdx.x % nt : blockIdx.x / BH, bh = (dbg & 8) ? blockIdx.x / nt : blockIdx.x % BH;
+  const int kt = j, b = bh / nh, head = bh % nh;
   const int h = nh * DH;
   const long Ttok = static_cast<long>(B) * s;
   const int i0 = (kt * kRows) / kCols;
   const int nq = (s + kCols - 1) / kCols;
-  const int ntiles = nq - i0;
+  const int ntiles = (dbg & 32) ? min(nq - i0, 1) : nq - i0;
   const float sl2 = rsqrtf(static_cast<float>(DH)) * LOG2E;
 
   if (warp == 0 && lane == 0) {
@@ -166,21 +178,29 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
   if (warp == 0) {
     if (elect_one()) {
       const int row0 = b * s;
-      mbar_arrive_expect_tx(kv_full, 2 * SM::kBig);
+      if (dbg & 128) mbar_arrive(kv_full);
+      else mbar_arrive_expect_tx(kv_full, 2 * SM::kBig);
 #pragma unroll
       for (int a = 0; a < DH / 64; ++a) {
+        if (dbg & 128) break;
         tma_load_2d(sK + a * (kRows * 128), &tm_qkv128, kv_full, h + head * DH + a * 64, row0 + kt * kRows);
         tma_load_2d(sV + a * (kRows * 128), &tm_qkv128, kv_full, 2 * h + head * DH + a * 64, row0 + kt * kRows);
       }
       for (int idx = 0; idx < ntiles; ++idx) {
         const int st = idx % kRingKV;
         mbar_wait(&q_empty[st], ((idx / kRingKV) & 1) ^ 1);
-        mbar_arrive_expect_tx(&q_full[st], 2 * SM::kSmall);
+        if (dbg & 16) { mbar_arrive(&q_full[st]); continue; }
+        mbar_arrive_expect_tx(&q_full[st], 2 * SM::kSmall + (bulk_ld ? 2 * kCols * 4 : 0));
         const int qr = row0 + (i0 + idx) * kCols;
 #pragma unroll
         for (int a = 0; a < DH / 64; ++a) {
-          tma_load_2d(sQ[st] + a * (kCols * 128), &tm_qkv64, &q_full[st], head * DH + a * 64, qr);
-          tma_load_2d(sG[st] + a * (kCols * 128), &tm_do64, &q_full[st], head * DH + a * 64, qr);
+          tma_load_2d(sQ(st) + a * (kCols * 128), &tm_qkv64, &q_full[st], head * DH + a * 64, qr);
+          tma_load_2d(sG(st) + a * (kCols * 128), &tm_do64, &q_full[st], head * DH + a * 64, qr);
+        }
+        if (bulk_ld) {
+          const long o = static_cast<long>(head) * Ttok + qr;
+          bulk_g2s(sLD + st * 2 * kCols, lse + o, kCols * 4, &q_full[st]);
+          bulk_g2s(sLD + st * 2 * kCols + kCols, Dd + o, kCols * 4, &q_full[st]);
         }
       }
     }
@@ -195,9 +215,10 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
       mbar_wait(&s_free[buf], ((idx >> 1) & 1) ^ 1);
       tc_fence_after();
       if (elect_one()) {
-        const uint32_t k = smem_u32(sK), v = smem_u32(sV), q = smem_u32(sQ[st]), g = smem_u32(sG[st]);
+        const uint32_t k = smem_u32(sK), v = smem_u32(sV), q = smem_u32(sQ(st)), g = smem_u32(sG(st));
 #pragma unroll
         for (int kk = 0; kk < DH / 16; ++kk) {
+          if (dbg & 2) break;
           const uint32_t ao = (kk >> 2) * (kRows * 128) + (kk & 3) * 32, bo = (kk >> 2) * (kCols * 128) + (kk & 3) * 32;
           umma_bf16(tm_S + buf * kCols, umma_desc_sw128(k + ao, 16, 1024), umma_desc_sw128(q + bo, 16, 1024), id_s, kk > 0);
           umma_bf16(tm_dP + buf * kCols, umma_desc_sw128(v + ao, 16, 1024), umma_desc_sw128(g + bo, 16, 1024), id_s, kk > 0);
@@ -211,9 +232,10 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
       mbar_wait(&p_full[pb], (idx >> 1) & 1);
       tc_fence_after();
       if (elect_one()) {
-        const uint32_t p = smem_u32(sP[pb]), ds = smem_u32(sS[pb]), q = smem_u32(sQ[st]), g = smem_u32(sG[st]);
+        const uint32_t p = smem_u32(sP(pb)), ds = smem_u32(sS(pb)), q = smem_u32(sQ(st)), g = smem_u32(sG(st));
 #pragma unroll
         for (int kk = 0; kk < kCols / 16; ++kk) {
+          if (dbg & 4) break;
           const uint64_t pa = umma_desc_sw128(p + kk * 32, 16, 1024), sa = umma_desc_sw128(ds + kk * 32, 16, 1024);
           umma_bf16(tm_dV, pa, umma_desc_sw128(g + kk * 2048, kCols * 128, 1024), id_a, (idx | kk) != 0);
           umma_bf16(tm_dK, sa, umma_desc_sw128(q + kk * 2048, kCols * 128, 1024), id_a, (idx | kk) != 0);
@@ -237,15 +259,29 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
     const uint32_t lane_off = static_cast<uint32_t>(quarter * 32) << 16;
     const int tid = threadIdx.x - 64;                // 0..255
     for (int idx = 0; idx < ntiles; ++idx) {
-      const int buf = idx & 1, i = i0 + idx;
-      // lse / D of this query tile into smem (threads 0..63: lse, 64..127: D)
-      if (tid < 128) {
-        const int c = tid & 63, qq = i * kCols + c;
-        const long r = static_cast<long>(b) * s + (qq < s ? qq : 0);
-        if (tid < 64) sL[buf * kCols + c] = lse[static_cast<long>(head) * Ttok + r] * LOG2E;
-        else sDv[buf * kCols + c] = Dd[static_cast<long>(head) * Ttok + r];
+      const int buf = idx & 1, i = i0 + idx, st = idx % kRingKV;
+      float* ld = sLD + st * 2 * kCols;
+      if (bulk_ld) {
+        // the slot's lse / D came with its Q/dO tile (the slot is released only after this tile's
+        // accumulate MMAs, which wait for this loop's p_full: no later phase can be pending)
+        mbar_wait(&q_full[st], (idx / kRingKV) & 1);
+      } else {
+        // lse / D of this query tile into the slot (threads 0..63: lse, 64..127: D)
+        if (tid < 128) {
+          const int c = tid & 63, qq = i * kCols + c;
+          const long r = static_cast<long>(b) * s + (qq < s ? qq : 0);
+          ld[tid] = tid < 64 ? lse[static_cast<long>(head) * Ttok + r] : Dd[static_cast<long>(head) * Ttok + r];
+        }
+        named_bar(1, 256);
       }
-      named_bar(1, 256);
+      float lv[32], dv[32];
+#pragma unroll
+      for (int c = 0; c < 32; c += 4) {
+        const float4 a = *reinterpret_cast<const float4*>(ld + half * 32 + c);
+        const float4 d = *reinterpret_cast<const float4*>(ld + kCols + half * 32 + c);
+        lv[c] = a.x * LOG2E; lv[c + 1] = a.y * LOG2E; lv[c + 2] = a.z * LOG2E; lv[c + 3] = a.w * LOG2E;
+        dv[c] = d.x; dv[c + 1] = d.y; dv[c + 2] = d.z; dv[c + 3] = d.w;
+      }
       mbar_wait(&s_full[buf], (idx >> 1) & 1);
       tc_fence_after();
       uint32_t sr[32], dr[32];
@@ -256,6 +292,12 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
       __syncwarp();
       if (lane == 0) mbar_arrive(&s_free[buf]);
       float p[32], ds[32];
+      if (dbg & 1) {
+        mbar_wait(&p_free[buf], ((idx >> 1) & 1) ^ 1);
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&p_full[buf]);
+        continue;
+      }
       // only tiles crossing the diagonal (queries < this block's last key) or the sequence end mask
       const bool edge = i * kCols < kt * kRows + kRows || i * kCols + kCols > s;
       if (edge) {
@@ -263,23 +305,22 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
         for (int c = 0; c < 32; ++c) {
           const int cc = half * 32 + c;
           const int qq = i * kCols + cc;
-          float pv = ex2(__uint_as_float(sr[c]) * sl2 - sL[buf * kCols + cc]);
+          float pv = ex2(__uint_as_float(sr[c]) * sl2 - lv[c]);
           if (qq < key || qq >= s) pv = 0.f;
           p[c] = pv;
-          ds[c] = pv * (__uint_as_float(dr[c]) - sDv[buf * kCols + cc]);
+          ds[c] = pv * (__uint_as_float(dr[c]) - dv[c]);
         }
       } else {
 #pragma unroll
         for (int c = 0; c < 32; ++c) {
-          const int cc = half * 32 + c;
-          const float pv = ex2(__uint_as_float(sr[c]) * sl2 - sL[buf * kCols + cc]);
+          const float pv = ex2(__uint_as_float(sr[c]) * sl2 - lv[c]);
           p[c] = pv;
-          ds[c] = pv * (__uint_as_float(dr[c]) - sDv[buf * kCols + cc]);
+          ds[c] = pv * (__uint_as_float(dr[c]) - dv[c]);
         }
       }
       mbar_wait(&p_free[buf], ((idx >> 1) & 1) ^ 1);   // the dV/dK MMAs of tile idx-2 consumed this buffer
-      st_half_row_sw128(sP[buf], row, 4 * half, p);
-      st_half_row_sw128(sS[buf], row, 4 * half, ds);
+      st_half_row_sw128(sP(buf), row, 4 * half, p);
+      st_half_row_sw128(sS(buf), row, 4 * half, ds);
       fence_proxy_async();
       __syncwarp();
       if (lane == 0) mbar_arrive(&p_full[buf]);
@@ -288,8 +329,13 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
     // epilogue: dV, dK rows of this thread's key
     mbar_wait(acc_done, 0);
     tc_fence_after();
-    // tcgen05.ld is warp-collective (.sync.aligned): every lane loads, only valid keys store
+    // tcgen05.ld is warp-collective (.sync.aligned): every lane loads, only valid keys store.
+    // Full 128-key blocks (s % 128 == 0): rows go to the (now idle) P/dS buffers in the SW128 layout
+    // and leave as four TMA tensor stores (coalesced); otherwise row-wise stores.
     const float scale = rsqrtf(static_cast<float>(DH));
+    const bool tma_st = (s % kRows) == 0 && !(dbg & 64);
+    auto stV = [&](int a) { return a ? sS(0) : sP(0); };
+    auto stK = [&](int a) { return a ? sS(1) : sP(1); };
     const long krow_idx = static_cast<long>(b) * s + (key < s ? key : 0);
     bf16* krow = dqkv + krow_idx * (3 * h) + h + head * DH;
     bf16* vrow = krow + h;
@@ -299,7 +345,13 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
       tmem_ld_32x32b_x32(tm_dV + c + lane_off, rv);
       tmem_ld_32x32b_x32(tm_dK + c + lane_off, rk);
       tmem_ld_wait();
-      if (key < s) {
+      if (tma_st) {
+        float fv[32], fk[32];
+#pragma unroll
+        for (int e = 0; e < 32; ++e) { fv[e] = __uint_as_float(rv[e]); fk[e] = __uint_as_float(rk[e]) * scale; }
+        st_half_row_sw128(stV(c / 64), row, (c % 64) / 8, fv);
+        st_half_row_sw128(stK(c / 64), row, (c % 64) / 8, fk);
+      } else if (key < s && !(dbg & 64)) {
 #pragma unroll
         for (int q = 0; q < 4; ++q) {
           uint4 uv, uk;
@@ -316,6 +368,19 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
         }
       }
     }
+    if (tma_st) {
+      fence_proxy_async();
+      named_bar(2, 128);
+      if (threadIdx.x == 64) {
+        const int r0 = b * s + kt * kRows;
+#pragma unroll
+        for (int a = 0; a < DH / 64; ++a) {
+          tma_store_2d(&tm_dqkv, stV(a), 2 * h + head * DH + a * 64, r0);
+          tma_store_2d(&tm_dqkv, stK(a), h + head * DH + a * 64, r0);
+        }
+        bulk_commit_wait_read();
+      }
+    }
   }
 done_dkdv:
   tc_fence_before();
@@ -327,19 +392,18 @@ done_dkdv:
 template <int DH>
 __global__ void __launch_bounds__(kThreadsB, 1)
 fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_qkv64,
-             const __grid_constant__ CUtensorMap tm_do128, const float* lse, const float* Dd, bf16* dqkv, int B, int s,
-             int nh) {
+             const __grid_constant__ CUtensorMap tm_do128, const __grid_constant__ CUtensorMap tm_dqkv,
+             const float* lse, const float* Dd, bf16* dqkv, int B, int s, int nh, int dbg) {
   using SM = Smem<DH>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sQ = smem;
   uint8_t* sG = sQ + SM::kBig;
-  uint8_t* sK[kRing];
-  uint8_t* sV[kRing];
-  for (int r = 0; r < kRing; ++r) { sK[r] = sG + SM::kBig + 2 * r * SM::kSmall; sV[r] = sK[r] + SM::kSmall; }
-  uint8_t* sS[2] = {sG + SM::kBig + 2 * kRing * SM::kSmall,               // dS [128 q][64 keys],
-                    sG + SM::kBig + 2 * kRing * SM::kSmall + SM::kP};     // double-buffered
-  uint64_t* bar = reinterpret_cast<uint64_t*>(sS[1] + SM::kP);
+  auto sK = [&](int r) { return sG + SM::kBig + 2 * r * SM::kSmall; };
+  auto sV = [&](int r) { return sG + SM::kBig + 2 * r * SM::kSmall + SM::kSmall; };
+  // dS [128 q][64 keys], double-buffered
+  auto sS = [&](int i) { return sG + SM::kBig + 2 * kRing * SM::kSmall + i * SM::kP; };
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sS(1) + SM::kP);
   uint64_t* q_fullb = bar;                // Q, dO loaded
   uint64_t* k_full = bar + 1;             // kRing
   uint64_t* k_empty = k_full + kRing;     // kRing
@@ -351,12 +415,14 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_done + 1);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-  // heaviest first: the last query tile sees every key tile
-  const int qt = gridDim.y - 1 - blockIdx.y, b = blockIdx.x / nh, head = blockIdx.x % nh;
+  // heaviest first over all (sample, head) (the last query tile sees every key tile); dbg bit 3: (sample, head)-major
+  const int nt = (s + kRows - 1) / kRows, BH = B * nh;
+  const int j = (dbg & 8) ? blockIdx.x % nt : blockIdx.x / BH, bh = (dbg & 8) ? blockIdx.x / nt : blockIdx.x % BH;
+  const int qt = nt - 1 - j, b = bh / nh, head = bh % nh;
   const int h = nh * DH;
   const long Ttok = static_cast<long>(B) * s;
   const int last_q = min(qt * kRows + kRows - 1, s - 1);
-  const int ntiles = last_q / kCols + 1;   // key tiles 0 .. last_q/64
+  const int ntiles = (dbg & 32) ? 1 : last_q / kCols + 1;   // key tiles 0 .. last_q/64
   const float sl2 = rsqrtf(static_cast<float>(DH)) * LOG2E;
 
   if (warp == 0 && lane == 0) {
@@ -380,21 +446,24 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
   if (warp == 0) {
     if (elect_one()) {
       const int row0 = b * s;
-      mbar_arrive_expect_tx(q_fullb, 2 * SM::kBig);
+      if (dbg & 128) mbar_arrive(q_fullb);
+      else mbar_arrive_expect_tx(q_fullb, 2 * SM::kBig);
 #pragma unroll
       for (int a = 0; a < DH / 64; ++a) {
+        if (dbg & 128) break;
         tma_load_2d(sQ + a * (kRows * 128), &tm_qkv128, q_fullb, head * DH + a * 64, row0 + qt * kRows);
         tma_load_2d(sG + a * (kRows * 128), &tm_do128, q_fullb, head * DH + a * 64, row0 + qt * kRows);
       }
       for (int idx = 0; idx < ntiles; ++idx) {
         const int st = idx % kRing;
         mbar_wait(&k_empty[st], ((idx / kRing) & 1) ^ 1);
+        if (dbg & 16) { mbar_arrive(&k_full[st]); continue; }
         mbar_arrive_expect_tx(&k_full[st], 2 * SM::kSmall);
         const int kr = row0 + idx * kCols;
 #pragma unroll
         for (int a = 0; a < DH / 64; ++a) {
-          tma_load_2d(sK[st] + a * (kCols * 128), &tm_qkv64, &k_full[st], h + head * DH + a * 64, kr);
-          tma_load_2d(sV[st] + a * (kCols * 128), &tm_qkv64, &k_full[st], 2 * h + head * DH + a * 64, kr);
+          tma_load_2d(sK(st) + a * (kCols * 128), &tm_qkv64, &k_full[st], h + head * DH + a * 64, kr);
+          tma_load_2d(sV(st) + a * (kCols * 128), &tm_qkv64, &k_full[st], 2 * h + head * DH + a * 64, kr);
         }
       }
     }
@@ -409,9 +478,10 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
       mbar_wait(&s_free[buf], ((idx >> 1) & 1) ^ 1);
       tc_fence_after();
       if (elect_one()) {
-        const uint32_t q = smem_u32(sQ), g = smem_u32(sG), k = smem_u32(sK[st]), v = smem_u32(sV[st]);
+        const uint32_t q = smem_u32(sQ), g = smem_u32(sG), k = smem_u32(sK(st)), v = smem_u32(sV(st));
 #pragma unroll
         for (int kk = 0; kk < DH / 16; ++kk) {
+          if (dbg & 2) break;
           const uint32_t ao = (kk >> 2) * (kRows * 128) + (kk & 3) * 32, bo = (kk >> 2) * (kCols * 128) + (kk & 3) * 32;
           umma_bf16(tm_S + buf * kCols, umma_desc_sw128(q + ao, 16, 1024), umma_desc_sw128(k + bo, 16, 1024), id_s, kk > 0);
           umma_bf16(tm_dP + buf * kCols, umma_desc_sw128(g + ao, 16, 1024), umma_desc_sw128(v + bo, 16, 1024), id_s, kk > 0);
@@ -425,11 +495,12 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
       mbar_wait(&p_full[pb], (idx >> 1) & 1);
       tc_fence_after();
       if (elect_one()) {
-        const uint32_t ds = smem_u32(sS[pb]), k = smem_u32(sK[st]);
+        const uint32_t ds = smem_u32(sS(pb)), k = smem_u32(sK(st));
 #pragma unroll
         for (int kk = 0; kk < kCols / 16; ++kk)
-          umma_bf16(tm_dQ, umma_desc_sw128(ds + kk * 32, 16, 1024), umma_desc_sw128(k + kk * 2048, kCols * 128, 1024),
-                    id_a, (idx | kk) != 0);
+          if (!(dbg & 4))
+            umma_bf16(tm_dQ, umma_desc_sw128(ds + kk * 32, 16, 1024), umma_desc_sw128(k + kk * 2048, kCols * 128, 1024),
+                      id_a, (idx | kk) != 0);
         umma_commit(&p_free[pb]);
         umma_commit(&k_empty[st]);
         if (idx == ntiles - 1) umma_commit(acc_done);
@@ -462,6 +533,12 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
       __syncwarp();
       if (lane == 0) mbar_arrive(&s_free[buf]);
       float ds[32];
+      if (dbg & 1) {
+        mbar_wait(&p_free[buf], ((idx >> 1) & 1) ^ 1);
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&p_full[buf]);
+        continue;
+      }
       if (idx * kCols + kCols - 1 > qt * kRows) {   // tile crosses the diagonal: causal mask
 #pragma unroll
         for (int c = 0; c < 32; ++c) {
@@ -478,7 +555,7 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
         }
       }
       mbar_wait(&p_free[buf], ((idx >> 1) & 1) ^ 1);
-      st_half_row_sw128(sS[buf], row, 4 * half, ds);
+      st_half_row_sw128(sS(buf), row, 4 * half, ds);
       fence_proxy_async();
       __syncwarp();
       if (lane == 0) mbar_arrive(&p_full[buf]);
@@ -487,13 +564,19 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
     mbar_wait(acc_done, 0);
     tc_fence_after();
     const float scale = rsqrtf(static_cast<float>(DH));
+    const bool tma_st = (s % kRows) == 0 && !(dbg & 64);
     bf16* qrow = dqkv + gr * (3 * h) + head * DH;
 #pragma unroll 1
     for (int c = 0; c < DH; c += 32) {
       uint32_t rq[32];
       tmem_ld_32x32b_x32(tm_dQ + c + lane_off, rq);
       tmem_ld_wait();
-      if (q < s) {
+      if (tma_st) {   // rows into the idle dS buffers (SW128), then TMA tensor stores
+        float fq[32];
+#pragma unroll
+        for (int e = 0; e < 32; ++e) fq[e] = __uint_as_float(rq[e]) * scale;
+        st_half_row_sw128(sS(c / 64), row, (c % 64) / 8, fq);
+      } else if (q < s && !(dbg & 64)) {
 #pragma unroll
         for (int e = 0; e < 4; ++e) {
           uint4 u;
@@ -503,6 +586,15 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
             hq[f] = __floats2bfloat162_rn(__uint_as_float(rq[8 * e + 2 * f]) * scale, __uint_as_float(rq[8 * e + 2 * f + 1]) * scale);
           *reinterpret_cast<uint4*>(qrow + c + 8 * e) = u;
         }
+      }
+    }
+    if (tma_st) {
+      fence_proxy_async();
+      named_bar(2, 128);
+      if (threadIdx.x == 64) {
+#pragma unroll
+        for (int a = 0; a < DH / 64; ++a) tma_store_2d(&tm_dqkv, sS(a), head * DH + a * 64, b * s + qt * kRows);
+        bulk_commit_wait_read();
       }
     }
   }
@@ -515,7 +607,7 @@ done_dq:
 // >= 116 KB so that one CTA owns the SM (each allocates all 512 TMEM columns)
 constexpr int at_least_one_sm(int b) { return b < 116 * 1024 ? 116 * 1024 : b; }
 template <int DH>
-constexpr int smem_dkdv() { return at_least_one_sm(2 * Smem<DH>::kBig + 2 * kRingKV * Smem<DH>::kSmall + 4 * Smem<DH>::kP + 4 * kCols * 4 + 256 + 1024); }
+constexpr int smem_dkdv() { return at_least_one_sm(2 * Smem<DH>::kBig + 2 * kRingKV * Smem<DH>::kSmall + 4 * Smem<DH>::kP + kRingKV * 2 * kCols * 4 + 256 + 1024); }
 template <int DH>
 constexpr int smem_dq() { return at_least_one_sm(2 * Smem<DH>::kBig + 2 * kRing * Smem<DH>::kSmall + 2 * Smem<DH>::kP + 256 + 1024); }
 
@@ -524,9 +616,10 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
             cudaStream_t st) {
   const int h = nh * DH;
   const long T = static_cast<long>(B) * s;
-  CUtensorMap m128, m64, d64, d128;
+  CUtensorMap m128, m64, d64, d128, g128;
   if (!make_tmap_bf16_2d(&m128, qkv, 3 * h, T, 3 * h, 64, 128) || !make_tmap_bf16_2d(&m64, qkv, 3 * h, T, 3 * h, 64, 64) ||
-      !make_tmap_bf16_2d(&d64, dO, h, T, h, 64, 64) || !make_tmap_bf16_2d(&d128, dO, h, T, h, 64, 128))
+      !make_tmap_bf16_2d(&d64, dO, h, T, h, 64, 64) || !make_tmap_bf16_2d(&d128, dO, h, T, h, 64, 128) ||
+      !make_tmap_bf16_2d(&g128, dqkv, 3 * h, T, 3 * h, 64, 128))
     return false;
   static bool set = false;
   if (!set) {
@@ -534,12 +627,17 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
     cudaFuncSetAttribute(fa_bwd_dq_tc<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_dq<DH>());
     set = true;
   }
-  dim3 grid(B * nh, (s + kRows - 1) / kRows);
+  dim3 grid(B * nh * ((s + kRows - 1) / kRows));
+  // experiment knob (results are wrong when bits 0-2 or 4 are set): bit 0 skips the softmax
+  // arithmetic and P/dS stores, bit 1 skips the S/dP MMAs, bit 2 skips the accumulate MMAs, bit 3
+  // orders CTAs (sample, head)-major, bit 4 skips the streamed TMA loads
+  const char* dbgs = getenv("MARIO_ATTN_DBG");
+  const int dbg = dbgs ? atoi(dbgs) : 0;
   const char* only = getenv("MARIO_ATTN_TC_ONLY");   // debugging aid: "dkdv" or "dq"
   if (!only || only[1] == 'k')
-    fa_bwd_dkdv_tc<DH><<<grid, kThreadsB, smem_dkdv<DH>(), st>>>(m128, m64, d64, lse, Dd, dqkv, B, s, nh);
+    fa_bwd_dkdv_tc<DH><<<grid, kThreadsB, smem_dkdv<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s, nh, dbg);
   if (!only || only[1] == 'q')
-    fa_bwd_dq_tc<DH><<<grid, kThreadsB, smem_dq<DH>(), st>>>(m128, m64, d128, lse, Dd, dqkv, B, s, nh);
+    fa_bwd_dq_tc<DH><<<grid, kThreadsB, smem_dq<DH>(), st>>>(m128, m64, d128, g128, lse, Dd, dqkv, B, s, nh, dbg);
   note_launch(2);
   return true;
 }
