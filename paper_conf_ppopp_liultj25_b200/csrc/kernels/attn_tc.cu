@@ -48,6 +48,12 @@ __device__ __forceinline__ float ex2(float x) {
 __device__ __forceinline__ void st_shared_f32(const void* p, float v) {
   asm volatile("st.shared.f32 [%0], %1;" :: "r"(static_cast<uint32_t>(__cvta_generic_to_shared(p))), "f"(v) : "memory");
 }
+__device__ __forceinline__ float4 ld_shared_f4(const void* p) {
+  float4 v;
+  asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];" : "=f"(v.x), "=f"(v.y), "=f"(v.z), "=f"(v.w)
+               : "r"(static_cast<uint32_t>(__cvta_generic_to_shared(p))) : "memory");
+  return v;
+}
 __device__ __forceinline__ float ld_shared_f32(const void* p) {
   float v;
   asm volatile("ld.shared.f32 %0, [%1];" : "=f"(v) : "r"(static_cast<uint32_t>(__cvta_generic_to_shared(p))) : "memory");
@@ -277,8 +283,8 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
       float lv[32], dv[32];
 #pragma unroll
       for (int c = 0; c < 32; c += 4) {
-        const float4 a = *reinterpret_cast<const float4*>(ld + half * 32 + c);
-        const float4 d = *reinterpret_cast<const float4*>(ld + kCols + half * 32 + c);
+        const float4 a = ld_shared_f4(ld + half * 32 + c);
+        const float4 d = ld_shared_f4(ld + kCols + half * 32 + c);
         lv[c] = a.x * LOG2E; lv[c + 1] = a.y * LOG2E; lv[c + 2] = a.z * LOG2E; lv[c + 3] = a.w * LOG2E;
         dv[c] = d.x; dv[c + 1] = d.y; dv[c + 2] = d.z; dv[c + 3] = d.w;
       }
