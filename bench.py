@@ -59,6 +59,19 @@ def measured_peaks():
 
 
 # ------------------------------------------------------------------ CPU oracle leg
+def gemm_traffic():
+    """DRAM bytes per GEMM launch from the committed ncu --set full capture (profiles/), or {}."""
+    p = os.path.join(ROOT, "profiles", "r01_traffic.json")
+    if not os.path.exists(p):
+        return {}
+    d = json.load(open(p)).get("gemm_bf16_tc2_kernel", {})
+    if "dram_bytes_per_launch" not in d:
+        return {}
+    return {"dram_bytes_per_launch": d["dram_bytes_per_launch"],
+            "note": f"mean dram__bytes_read+write over {d.get('launches_captured')} captured launches "
+                    f"(one layer's forward GEMMs: qkv, proj, fc1, fc2); {d.get('source', '')}"}
+
+
 def cpu_oracle_sample(cfg, layers_list=(1, 2)):
     """Time the oracle (numpy fp32, all host cores) on ONE sample (mbs=1) of the workload's
     model truncated to L in layers_list layers + embedding/head, then extrapolate linearly to the
@@ -352,6 +365,7 @@ def main():
 
     sim = plan.simulate()
     peaks, peak_kind = measured_peaks()
+    traffic = gemm_traffic()
     g = kst["gemm"]
     achieved = g["flops"] / (g["ms"] / 1e3) / 1e12 if g["ms"] > 0 else 0.0
     peak = float(peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops")))
@@ -368,7 +382,10 @@ def main():
            "roofline": {"bound": "tensor", "kernel": "gemm_bf16_tc_kernel (tcgen05, all linear layers)",
                         "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
                         "peak_source": f"{peak_kind} bf16_tflops_sustained (MEASURED_PEAKS.json)",
-                        "traffic": None, "launches_per_step": g["launches"] / kst_steps,
+                        "traffic": traffic.get("dram_bytes_per_launch"),
+                        "traffic_note": traffic.get("note"),
+                        "algorithmic_bytes_per_launch": (g["bytes"] / g["launches"]) if g["launches"] else None,
+                        "launches_per_step": g["launches"] / kst_steps,
                         "measured_in": "graph replay (latest step)" if use_graphs else "eager steps",
                         "share_of_step": (g["ms"] / kst_steps) / ms_step if ms_step > 0 else None},
            "kernels": {"note": "one extra step with every launch event-timed (not the headline region)",

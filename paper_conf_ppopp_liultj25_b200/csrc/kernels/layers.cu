@@ -1016,6 +1016,17 @@ __global__ void cast_k(const float* x, __nv_bfloat16* y, size_t n) {
   for (size_t i = blockIdx.x * static_cast<size_t>(blockDim.x) + threadIdx.x; i < n; i += static_cast<size_t>(gridDim.x) * blockDim.x)
     y[i] = __float2bfloat16_rn(x[i]);
 }
+// 8 elements per thread-iteration: two 16-byte loads, one 16-byte store
+__global__ void cast_v8_k(const float4* x, uint4* y, size_t n8) {
+  for (size_t i = blockIdx.x * static_cast<size_t>(blockDim.x) + threadIdx.x; i < n8; i += static_cast<size_t>(gridDim.x) * blockDim.x) {
+    const float4 a = x[2 * i], b = x[2 * i + 1];
+    uint4 u;
+    __nv_bfloat162* h = reinterpret_cast<__nv_bfloat162*>(&u);
+    h[0] = __floats2bfloat162_rn(a.x, a.y); h[1] = __floats2bfloat162_rn(a.z, a.w);
+    h[2] = __floats2bfloat162_rn(b.x, b.y); h[3] = __floats2bfloat162_rn(b.z, b.w);
+    y[i] = u;
+  }
+}
 __global__ void add_k(float* a, const float* b, size_t n) {
   for (size_t i = blockIdx.x * static_cast<size_t>(blockDim.x) + threadIdx.x; i < n; i += static_cast<size_t>(gridDim.x) * blockDim.x)
     a[i] += b[i];
@@ -1239,7 +1250,12 @@ void loss_reduce(const float* row_loss, int rows, double* out, cudaStream_t st) 
 }
 void cast_f32_bf16(const float* x, __nv_bfloat16* y, size_t n, cudaStream_t st) {
   KScope ks_(K_ELEMWISE, st);
-  cast_k<<<grid_for(static_cast<long>(n)), 256, 0, st>>>(x, y, n);
+  if (n % 8 == 0 && (reinterpret_cast<uintptr_t>(x) & 15) == 0 && (reinterpret_cast<uintptr_t>(y) & 15) == 0) {
+    cast_v8_k<<<grid_for(static_cast<long>(n / 8)), 256, 0, st>>>(reinterpret_cast<const float4*>(x),
+                                                                  reinterpret_cast<uint4*>(y), n / 8);
+  } else {
+    cast_k<<<grid_for(static_cast<long>(n)), 256, 0, st>>>(x, y, n);
+  }
   note_launch();
 }
 void add_f32(float* a, const float* b, size_t n, cudaStream_t st) { add_k<<<grid_for(static_cast<long>(n)), 256, 0, st>>>(a, b, n); note_launch(); }
