@@ -22,6 +22,7 @@
 #include <cuda_runtime.h>
 #include <cuda_bf16.h>
 #include <cstdio>
+#include <cstdlib>
 #include <map>
 #include <mutex>
 
@@ -141,6 +142,22 @@ __device__ __forceinline__ void epilogue_chunk(const GemmEpilogue& ep, const uin
       }
     }
   }
+}
+
+// Tile raster. raster 0: M fastest (consecutive tiles share a B panel), 1: N fastest (share an A
+// panel), G >= 2: groups of G tile-rows, M fastest inside a group, so the concurrently running tiles
+// form a compact block whose A and B panels both stay in L2 when the whole operands do not.
+__device__ __forceinline__ void tile_coords(int tile, int num_m, int num_n, int raster, int& tm, int& tn) {
+  if (raster < 2) {
+    tm = raster ? tile / num_n : tile % num_m;
+    tn = raster ? tile % num_n : tile / num_m;
+    return;
+  }
+  const int grp = tile / (raster * num_n), first_m = grp * raster;
+  const int gs = num_m - first_m < raster ? num_m - first_m : raster;
+  const int local = tile - grp * raster * num_n;
+  tm = first_m + local % gs;
+  tn = local / gs;
 }
 
 // Warp-cooperative epilogue for one 32x32 block: lane i holds row rbase + i, columns
@@ -326,7 +343,8 @@ gemm_bf16_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
     if (elect_one()) {
       int s = 0; uint32_t ph = 0;
       for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x) {
-        const int tm = n_fastest ? tile / num_n : tile % num_m, tn = n_fastest ? tile % num_n : tile / num_m;
+        int tm, tn;
+        tile_coords(tile, num_m, num_n, n_fastest, tm, tn);
         const int m0 = tm * BM, n0 = tn * BN;
         for (int kb = 0; kb < nk; ++kb) {
           mbar_wait(&empty[s], ph ^ 1);
@@ -390,7 +408,8 @@ gemm_bf16_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
     for (int tile = blockIdx.x; tile < num_tiles; tile += gridDim.x, ++t) {
       const int acc = t & 1;
       const uint32_t acc_ph = (t >> 1) & 1;
-      const int tm = n_fastest ? tile / num_n : tile % num_m, tn = n_fastest ? tile % num_n : tile / num_m;
+      int tm, tn;
+        tile_coords(tile, num_m, num_n, n_fastest, tm, tn);
       const int m0 = tm * BM, n0 = tn * BN;
       mbar_wait(&tfull[acc], acc_ph);
       tc_fence_after();
@@ -438,6 +457,7 @@ struct Cfg2 {                                             // BNP = N of the pair
 // no cycle can form even when not every pair is resident.
 struct StreamK {
   int on = 0;
+  int sleep_ns = 0;        // epilogue warps poll the accumulator barrier with this back-off (experiment)
   float* ws = nullptr;     // [npairs][2 CTAs][128 rows][256 cols] fp32
   int* flags = nullptr;    // [npairs][2], zero between launches
 };
@@ -466,6 +486,12 @@ struct SkIter {
 // first stream-K iteration of pair q
 __device__ __forceinline__ long long sk_bound(int q, long long I0, long long Isk, int P) {
   return I0 + static_cast<long long>(q) * Isk / P;
+}
+__device__ __forceinline__ bool mbar_test(uint64_t* bar, uint32_t parity) {
+  uint32_t ok;
+  asm volatile("{\n\t.reg .pred p;\n\tmbarrier.test_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+               : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+  return ok != 0;
 }
 __device__ __forceinline__ int ld_acquire(const int* p) {
   int v;
@@ -521,7 +547,8 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
       SkUnit u;
       while (itr.next(nk, u)) {
         const int tile = u.tile;
-        const int tm = n_fastest ? tile / num_n : tile % num_m, tn = n_fastest ? tile % num_n : tile / num_m;
+        int tm, tn;
+        tile_coords(tile, num_m, num_n, n_fastest, tm, tn);
         const int m0 = tm * 256 + 128 * rank, n0 = tn * BNP + (BNP / 2) * rank;
         for (int kb = u.kb0; kb < u.kb1; ++kb) {
           mbar_wait(&empty[s], ph ^ 1);
@@ -588,9 +615,11 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
       const int tile = u.tile;
       const int acc = t & 1;
       const uint32_t acc_ph = (t >> 1) & 1;
-      const int tm = n_fastest ? tile / num_n : tile % num_m, tn = n_fastest ? tile % num_n : tile / num_m;
+      int tm, tn;
+        tile_coords(tile, num_m, num_n, n_fastest, tm, tn);
       const int m0 = tm * 256 + 128 * rank, n0 = tn * BNP;
-      mbar_wait(&tfull[acc], acc_ph);
+      if (sk.sleep_ns) { while (!mbar_test(&tfull[acc], acc_ph)) __nanosleep(sk.sleep_ns); }
+      else mbar_wait(&tfull[acc], acc_ph);
       tc_fence_after();
       const int rbase = m0 + quarter * 32;
       const int lrow = quarter * 32 + lane;                     // accumulator row within this CTA
@@ -691,6 +720,15 @@ bool make_tmap(CUtensorMap* map, const void* base, uint64_t inner, uint64_t oute
   return r == CUDA_SUCCESS;
 }
 
+// Raster choice: keep the smaller operand's panel hot across the other dimension (1-D order) when one
+// whole operand fits comfortably in L2; otherwise grouped tiles (8 tile-rows) so that both operand
+// working sets of the ~74-148 concurrently running tiles stay in L2.
+int raster_for(const GemmArgs& g) {
+  const double a = 2.0 * g.M * g.K, b = 2.0 * g.N * g.K;
+  if ((a < b ? a : b) > 48e6) return 8;
+  return static_cast<long>(g.M) >= static_cast<long>(g.N) ? 1 : 0;
+}
+
 template <int BN, bool A_MN, bool B_MN>
 cudaError_t launch_bn(const GemmArgs& g, cudaStream_t st, int num_sms) {
   using C = Cfg<BN>;
@@ -717,7 +755,7 @@ cudaError_t launch_bn(const GemmArgs& g, cudaStream_t st, int num_sms) {
   const int tok = kstats_begin(K_GEMM, 2.0 * g.M * g.N * g.K,
                                2.0 * (double(g.M) * g.K + double(g.N) * g.K) + (g.ep.out_f32 ? 4.0 : 2.0) * g.M * g.N, st);
   // raster: keep the larger operand's panel hot in L2 across the other dimension's tiles
-  const int n_fastest = static_cast<long>(g.M) >= static_cast<long>(g.N) ? 1 : 0;
+  const int n_fastest = raster_for(g);
   kern<<<grid, kThreads, C::kSmem, st>>>(ta, tb, g.ep, g.M, g.N, g.K, n_fastest);
   kstats_end(tok, st);
   note_launch();
@@ -778,6 +816,8 @@ cudaError_t launch_pair(const GemmArgs& g, cudaStream_t st, int num_sms) {
   const int tiles = ((g.M + 255) / 256) * ((g.N + BNP - 1) / BNP);
   int pairs = tiles < num_sms / 2 ? tiles : num_sms / 2;
   StreamK sk;
+  static const int sleep_ns = getenv("MARIO_GEMM_SLEEP") ? atoi(getenv("MARIO_GEMM_SLEEP")) : 0;
+  sk.sleep_ns = sleep_ns;
   if (BNP == 256 && use_streamk(tiles, num_sms / 2, (g.K + BK - 1) / BK)) {
     float* ws = nullptr;
     int* flags = nullptr;
@@ -788,7 +828,7 @@ cudaError_t launch_pair(const GemmArgs& g, cudaStream_t st, int num_sms) {
   }
   const int tok = kstats_begin(K_GEMM, 2.0 * g.M * g.N * g.K,
                                2.0 * (double(g.M) * g.K + double(g.N) * g.K) + (g.ep.out_f32 ? 4.0 : 2.0) * g.M * g.N, st);
-  const int n_fastest = static_cast<long>(g.M) >= static_cast<long>(g.N) ? 1 : 0;
+  const int n_fastest = raster_for(g);
   kern<<<2 * pairs, kThreads2, C2::kSmem, st>>>(ta, tb, g.ep, g.M, g.N, g.K, n_fastest, sk);
   kstats_end(tok, st);
   note_launch();
