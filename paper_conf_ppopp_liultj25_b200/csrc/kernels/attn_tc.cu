@@ -610,12 +610,254 @@ done_dq:
   if (warp == 1) tmem_dealloc<512>(tm);
 }
 
+// ----------------------------------------------------------------- dQ, persistent
+// fa_bwd_dq_pers: the dQ kernel as a persistent grid (one CTA per SM) over work items (sample, head,
+// 128-query tile) in the same heavy-first order, CTA c taking items c, c + grid, ... The per-CTA
+// fixed cost of the one-item kernel (launch, TMEM allocation, the stationary Q/dO load, the dQ
+// epilogue: ~30% of it at the cfg-2 shape) is paid once per SM: the producer streams the next
+// item's Q/dO as soon as the last S/dP MMAs of the current one have read them, the dQ accumulator
+// is double-buffered in TMEM (dQ0 | dQ1 | S x2 | dP x2 = 512 columns), and 4 dedicated epilogue
+// warps drain dQ[n & 1] (tcgen05.ld -> scale -> bf16 -> global) while item n + 1 computes.
+// Warps: 0 TMA, 1 MMA, 2..9 softmax (one query row per thread, 32 keys of the 64-key tile each),
+// 10..13 epilogue. Counters (ring slot, S/dP buffer, dS buffer) run across items.
+constexpr int kThreadsP = 448;
+template <int DH>
+__global__ void __launch_bounds__(kThreadsP, 1)
+fa_bwd_dq_pers(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_qkv64,
+               const __grid_constant__ CUtensorMap tm_do128, const float* lse, const float* Dd, bf16* dqkv, int B,
+               int s, int nh) {
+  using SM = Smem<DH>;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sQ = smem;
+  uint8_t* sG = sQ + SM::kBig;
+  auto sK = [&](int r) { return sG + SM::kBig + 2 * r * SM::kSmall; };
+  auto sV = [&](int r) { return sG + SM::kBig + 2 * r * SM::kSmall + SM::kSmall; };
+  auto sS = [&](int i) { return sG + SM::kBig + 2 * kRing * SM::kSmall + i * SM::kP; };
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sS(1) + SM::kP);
+  uint64_t* qd_full = bar;                // 1
+  uint64_t* qd_empty = bar + 1;           // 1
+  uint64_t* k_full = bar + 2;             // kRing
+  uint64_t* k_empty = k_full + kRing;     // kRing
+  uint64_t* s_full = k_empty + kRing;     // 2
+  uint64_t* s_free = s_full + 2;          // 2
+  uint64_t* p_full = s_free + 2;          // 2
+  uint64_t* p_free = p_full + 2;          // 2
+  uint64_t* acc_full = p_free + 2;        // 2
+  uint64_t* acc_empty = acc_full + 2;     // 2
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_empty + 2);
+
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int nt = (s + kRows - 1) / kRows, BH = B * nh, W = nt * BH;
+  const int h = nh * DH;
+  const long Ttok = static_cast<long>(B) * s;
+  const float sl2 = rsqrtf(static_cast<float>(DH)) * LOG2E;
+  // item w -> (qt, b, head): heaviest query tiles first over all (sample, head)
+  auto item = [&](int w, int& qt, int& b, int& head, int& ntiles) {
+    const int j = w / BH, bh = w % BH;
+    qt = nt - 1 - j; b = bh / nh; head = bh % nh;
+    const int last_q = min(qt * kRows + kRows - 1, s - 1);
+    ntiles = last_q / kCols + 1;
+  };
+
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&tm_qkv128);
+    tma_prefetch_desc(&tm_qkv64);
+    tma_prefetch_desc(&tm_do128);
+    mbar_init(qd_full, 1); mbar_init(qd_empty, 1);
+    for (int i = 0; i < kRing; ++i) { mbar_init(&k_full[i], 1); mbar_init(&k_empty[i], 1); }
+    for (int i = 0; i < 2; ++i) {
+      mbar_init(&s_full[i], 1); mbar_init(&s_free[i], 8); mbar_init(&p_full[i], 8); mbar_init(&p_free[i], 1);
+      mbar_init(&acc_full[i], 1); mbar_init(&acc_empty[i], 4);
+    }
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc<512>(tmem_slot);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tm = *tmem_slot;
+  const uint32_t tm_dQ = tm, tm_S = tm + 2 * DH, tm_dP = tm + 2 * DH + 2 * kCols;
+
+  if (warp == 0) {
+    if (elect_one()) {
+      int kc = 0, n = 0;
+      for (int w = blockIdx.x; w < W; w += gridDim.x, ++n) {
+        int qt, b, head, ntiles;
+        item(w, qt, b, head, ntiles);
+        const int row0 = b * s;
+        mbar_wait(qd_empty, (n & 1) ^ 1);   // the previous item's S/dP MMAs are done with Q, dO
+        mbar_arrive_expect_tx(qd_full, 2 * SM::kBig);
+#pragma unroll
+        for (int a = 0; a < DH / 64; ++a) {
+          tma_load_2d(sQ + a * (kRows * 128), &tm_qkv128, qd_full, head * DH + a * 64, row0 + qt * kRows);
+          tma_load_2d(sG + a * (kRows * 128), &tm_do128, qd_full, head * DH + a * 64, row0 + qt * kRows);
+        }
+        for (int idx = 0; idx < ntiles; ++idx, ++kc) {
+          const int st = kc % kRing;
+          mbar_wait(&k_empty[st], ((kc / kRing) & 1) ^ 1);
+          mbar_arrive_expect_tx(&k_full[st], 2 * SM::kSmall);
+          const int kr = row0 + idx * kCols;
+#pragma unroll
+          for (int a = 0; a < DH / 64; ++a) {
+            tma_load_2d(sK(st) + a * (kCols * 128), &tm_qkv64, &k_full[st], h + head * DH + a * 64, kr);
+            tma_load_2d(sV(st) + a * (kCols * 128), &tm_qkv64, &k_full[st], 2 * h + head * DH + a * 64, kr);
+          }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    constexpr uint32_t id_s = umma_idesc_bf16(128, kCols, 0, 0);
+    constexpr uint32_t id_a = umma_idesc_bf16(128, DH, 0, 1);   // dQ += dS K: B = K_j read MN-major
+    int kc = 0, gc = 0, n = 0;
+    for (int w = blockIdx.x; w < W; w += gridDim.x, ++n) {
+      int qt, b, head, ntiles;
+      item(w, qt, b, head, ntiles);
+      const uint32_t dq_t = tm_dQ + (n & 1) * DH;
+      mbar_wait(qd_full, n & 1);
+      tc_fence_after();
+      auto issue_s = [&](int idx) {
+        const int st = (kc + idx) % kRing, g = gc + idx, buf = g & 1;
+        mbar_wait(&k_full[st], ((kc + idx) / kRing) & 1);
+        mbar_wait(&s_free[buf], ((g >> 1) & 1) ^ 1);
+        tc_fence_after();
+        if (elect_one()) {
+          const uint32_t q = smem_u32(sQ), gg = smem_u32(sG), k = smem_u32(sK(st)), v = smem_u32(sV(st));
+#pragma unroll
+          for (int kk = 0; kk < DH / 16; ++kk) {
+            const uint32_t ao = (kk >> 2) * (kRows * 128) + (kk & 3) * 32, bo = (kk >> 2) * (kCols * 128) + (kk & 3) * 32;
+            umma_bf16(tm_S + buf * kCols, umma_desc_sw128(q + ao, 16, 1024), umma_desc_sw128(k + bo, 16, 1024), id_s, kk > 0);
+            umma_bf16(tm_dP + buf * kCols, umma_desc_sw128(gg + ao, 16, 1024), umma_desc_sw128(v + bo, 16, 1024), id_s, kk > 0);
+          }
+          umma_commit(&s_full[buf]);
+          if (idx == ntiles - 1) umma_commit(qd_empty);   // Q/dO free once these MMAs complete
+        }
+        __syncwarp();
+      };
+      auto issue_acc = [&](int idx) {
+        const int st = (kc + idx) % kRing, g = gc + idx, pb = g & 1;
+        if (idx == 0) mbar_wait(&acc_empty[n & 1], ((n >> 1) & 1) ^ 1);   // dQ[n & 1] drained (item n - 2)
+        mbar_wait(&p_full[pb], (g >> 1) & 1);
+        tc_fence_after();
+        if (elect_one()) {
+          const uint32_t ds = smem_u32(sS(pb)), k = smem_u32(sK(st));
+#pragma unroll
+          for (int kk = 0; kk < kCols / 16; ++kk)
+            umma_bf16(dq_t, umma_desc_sw128(ds + kk * 32, 16, 1024), umma_desc_sw128(k + kk * 2048, kCols * 128, 1024),
+                      id_a, (idx | kk) != 0);
+          umma_commit(&p_free[pb]);
+          umma_commit(&k_empty[st]);
+          if (idx == ntiles - 1) umma_commit(&acc_full[n & 1]);
+        }
+        __syncwarp();
+      };
+      issue_s(0);
+      for (int idx = 1; idx < ntiles; ++idx) {
+        issue_s(idx);
+        issue_acc(idx - 1);
+      }
+      issue_acc(ntiles - 1);
+      kc += ntiles;
+      gc += ntiles;
+    }
+  } else if (warp < 10) {
+    const int quarter = warp & 3, half = (warp - 2) >> 2;
+    const int row = quarter * 32 + lane;
+    const uint32_t lane_off = static_cast<uint32_t>(quarter * 32) << 16;
+    int gc = 0;
+    for (int w = blockIdx.x; w < W; w += gridDim.x) {
+      int qt, b, head, ntiles;
+      item(w, qt, b, head, ntiles);
+      const int q = qt * kRows + row;
+      const long gr = static_cast<long>(b) * s + (q < s ? q : 0);
+      const float L = lse[static_cast<long>(head) * Ttok + gr] * LOG2E;
+      const float Dr = Dd[static_cast<long>(head) * Ttok + gr];
+      for (int idx = 0; idx < ntiles; ++idx) {
+        const int g = gc + idx, buf = g & 1;
+        mbar_wait(&s_full[buf], (g >> 1) & 1);
+        tc_fence_after();
+        uint32_t sr[32], dr[32];
+        tmem_ld_32x32b_x32(tm_S + buf * kCols + half * 32 + lane_off, sr);
+        tmem_ld_32x32b_x32(tm_dP + buf * kCols + half * 32 + lane_off, dr);
+        tmem_ld_wait();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&s_free[buf]);
+        float ds[32];
+        if (idx * kCols + kCols - 1 > qt * kRows) {   // tile crosses the diagonal: causal mask
+#pragma unroll
+          for (int c = 0; c < 32; ++c) {
+            const int key = idx * kCols + half * 32 + c;
+            float pv = ex2(__uint_as_float(sr[c]) * sl2 - L);
+            if (key > q) pv = 0.f;
+            ds[c] = pv * (__uint_as_float(dr[c]) - Dr);
+          }
+        } else {
+#pragma unroll
+          for (int c = 0; c < 32; ++c) {
+            const float pv = ex2(__uint_as_float(sr[c]) * sl2 - L);
+            ds[c] = pv * (__uint_as_float(dr[c]) - Dr);
+          }
+        }
+        mbar_wait(&p_free[buf], ((g >> 1) & 1) ^ 1);
+        st_half_row_sw128(sS(buf), row, 4 * half, ds);
+        fence_proxy_async();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&p_full[buf]);
+      }
+      gc += ntiles;
+    }
+  } else {
+    // epilogue warps 10..13: TMEM lane quarter = warp & 3
+    const int quarter = warp & 3;
+    const int row = quarter * 32 + lane;
+    const uint32_t lane_off = static_cast<uint32_t>(quarter * 32) << 16;
+    const float scale = rsqrtf(static_cast<float>(DH));
+    int n = 0;
+    for (int w = blockIdx.x; w < W; w += gridDim.x, ++n) {
+      int qt, b, head, ntiles;
+      item(w, qt, b, head, ntiles);
+      const int q = qt * kRows + row;
+      bf16* qrow = dqkv + (static_cast<long>(b) * s + (q < s ? q : 0)) * (3 * h) + head * DH;
+      mbar_wait(&acc_full[n & 1], (n >> 1) & 1);
+      tc_fence_after();
+#pragma unroll 1
+      for (int c = 0; c < DH; c += 32) {
+        uint32_t rq[32];
+        tmem_ld_32x32b_x32(tm_dQ + (n & 1) * DH + c + lane_off, rq);
+        tmem_ld_wait();
+        if (c + 32 == DH) {   // every column of dQ[n & 1] is in registers: release it to the MMA warp
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&acc_empty[n & 1]);
+        }
+        if (q < s) {
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            uint4 u;
+            __nv_bfloat162* hq = reinterpret_cast<__nv_bfloat162*>(&u);
+#pragma unroll
+            for (int f = 0; f < 4; ++f)
+              hq[f] = __floats2bfloat162_rn(__uint_as_float(rq[8 * e + 2 * f]) * scale,
+                                            __uint_as_float(rq[8 * e + 2 * f + 1]) * scale);
+            *reinterpret_cast<uint4*>(qrow + c + 8 * e) = u;
+          }
+        }
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) tmem_dealloc<512>(tm);
+}
+
 // >= 116 KB so that one CTA owns the SM (each allocates all 512 TMEM columns)
 constexpr int at_least_one_sm(int b) { return b < 116 * 1024 ? 116 * 1024 : b; }
 template <int DH>
 constexpr int smem_dkdv() { return at_least_one_sm(2 * Smem<DH>::kBig + 2 * kRingKV * Smem<DH>::kSmall + 4 * Smem<DH>::kP + kRingKV * 2 * kCols * 4 + 256 + 1024); }
 template <int DH>
 constexpr int smem_dq() { return at_least_one_sm(2 * Smem<DH>::kBig + 2 * kRing * Smem<DH>::kSmall + 2 * Smem<DH>::kP + 256 + 1024); }
+int g_attn_dq_pers = 1;   // MARIO_ATTN_DQ_PERS=0 selects the one-item-per-CTA dQ kernel
 
 template <int DH>
 bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, bf16* dqkv, int B, int s, int nh,
@@ -642,8 +884,24 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
   const char* only = getenv("MARIO_ATTN_TC_ONLY");   // debugging aid: "dkdv" or "dq"
   if (!only || only[1] == 'k')
     fa_bwd_dkdv_tc<DH><<<grid, kThreadsB, smem_dkdv<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s, nh, dbg);
-  if (!only || only[1] == 'q')
-    fa_bwd_dq_tc<DH><<<grid, kThreadsB, smem_dq<DH>(), st>>>(m128, m64, d128, g128, lse, Dd, dqkv, B, s, nh, dbg);
+  static const bool pers = getenv("MARIO_ATTN_DQ_PERS") ? atoi(getenv("MARIO_ATTN_DQ_PERS")) != 0 : g_attn_dq_pers != 0;
+  if (!only || only[1] == 'q') {
+    if (pers && dbg == 0) {
+      static bool pset = false;
+      if (!pset) {
+        cudaFuncSetAttribute(fa_bwd_dq_pers<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_dq<DH>());
+        pset = true;
+      }
+      int sms = 0, dev = 0;
+      cudaGetDevice(&dev);
+      cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+      const int items = B * nh * ((s + kRows - 1) / kRows);
+      fa_bwd_dq_pers<DH><<<items < sms ? items : sms, kThreadsP, smem_dq<DH>(), st>>>(m128, m64, d128, lse, Dd, dqkv,
+                                                                                         B, s, nh);
+    } else {
+      fa_bwd_dq_tc<DH><<<grid, kThreadsB, smem_dq<DH>(), st>>>(m128, m64, d128, g128, lse, Dd, dqkv, B, s, nh, dbg);
+    }
+  }
   note_launch(2);
   return true;
 }
