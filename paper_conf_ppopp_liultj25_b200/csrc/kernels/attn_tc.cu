@@ -117,7 +117,7 @@ template <int DH>
 __global__ void __launch_bounds__(kThreadsB, 1)
 fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_qkv64,
                const __grid_constant__ CUtensorMap tm_do64, const __grid_constant__ CUtensorMap tm_dqkv,
-               const float* lse, const float* Dd, bf16* dqkv, int B, int s, int nh, int dbg) {
+               const float* lse, const float* Dd, bf16* dqkv, int B, int s, int nh, int dbg, long long* trace) {
   const bool bulk_ld = (s % kCols) == 0;
   using SM = Smem<DH>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -215,8 +215,10 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
     constexpr uint32_t id_a = umma_idesc_bf16(128, DH, 0, 1);      // dV, dK: B = Q/dO read MN-major
     mbar_wait(kv_full, 0);
     tc_fence_after();
+    const bool tr = trace && blockIdx.x == 0 && lane == 0;
     auto issue_s = [&](int idx) {
       const int st = idx % kRingKV, buf = idx & 1;
+      if (tr) trace[0 * 64 + idx] = clock64();
       mbar_wait(&q_full[st], (idx / kRingKV) & 1);
       mbar_wait(&s_free[buf], ((idx >> 1) & 1) ^ 1);
       tc_fence_after();
@@ -232,10 +234,13 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
         umma_commit(&s_full[buf]);
       }
       __syncwarp();
+      if (tr) trace[1 * 64 + idx] = clock64();
     };
     auto issue_acc = [&](int idx) {
       const int st = idx % kRingKV, pb = idx & 1;
+      if (tr) trace[2 * 64 + idx] = clock64();
       mbar_wait(&p_full[pb], (idx >> 1) & 1);
+      if (tr) trace[3 * 64 + idx] = clock64();
       tc_fence_after();
       if (elect_one()) {
         const uint32_t p = smem_u32(sP(pb)), ds = smem_u32(sS(pb)), q = smem_u32(sQ(st)), g = smem_u32(sG(st));
@@ -288,7 +293,10 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
         lv[c] = a.x * LOG2E; lv[c + 1] = a.y * LOG2E; lv[c + 2] = a.z * LOG2E; lv[c + 3] = a.w * LOG2E;
         dv[c] = d.x; dv[c + 1] = d.y; dv[c + 2] = d.z; dv[c + 3] = d.w;
       }
+      const bool trs = trace && blockIdx.x == 0 && threadIdx.x == 64;
+      if (trs) trace[4 * 64 + idx] = clock64();
       mbar_wait(&s_full[buf], (idx >> 1) & 1);
+      if (trs) trace[5 * 64 + idx] = clock64();
       tc_fence_after();
       uint32_t sr[32], dr[32];
       tmem_ld_32x32b_x32(tm_S + buf * kCols + half * 32 + lane_off, sr);
@@ -324,12 +332,14 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
           ds[c] = pv * (__uint_as_float(dr[c]) - dv[c]);
         }
       }
+      if (trs) trace[6 * 64 + idx] = clock64();
       mbar_wait(&p_free[buf], ((idx >> 1) & 1) ^ 1);   // the dV/dK MMAs of tile idx-2 consumed this buffer
       st_half_row_sw128(sP(buf), row, 4 * half, p);
       st_half_row_sw128(sS(buf), row, 4 * half, ds);
       fence_proxy_async();
       __syncwarp();
       if (lane == 0) mbar_arrive(&p_full[buf]);
+      if (trs) trace[7 * 64 + idx] = clock64();
     }
     if (half == 1) goto done_dkdv;   // the epilogue uses one warp per lane quarter
     // epilogue: dV, dK rows of this thread's key
@@ -610,6 +620,268 @@ done_dq:
   if (warp == 1) tmem_dealloc<512>(tm);
 }
 
+// ------------------------------------------------------------------- dK / dV, "TS"
+// fa_bwd_dkdv_ts: the dK/dV kernel with P^T and dS^T kept in TMEM. The softmax threads (one key row
+// = one TMEM lane each) pack P^T / dS^T to bf16 and tcgen05.st them over the S^T / dP^T columns they
+// have just read (half h of the warps owns S columns [32h, 32h + 32) and writes its 16 packed columns
+// at [32h, 32h + 16): no cross-warp hazard), and dV += P^T dO, dK += dS^T Q read their A operand
+// from TMEM. This removes the P^T / dS^T shared-memory round trip (32 KB written + 32 KB read by the
+// tensor core per tile) and frees 64 KB of shared memory for a 4-deep Q/dO ring: a ring slot is held
+// from the S^T MMAs of its tile to the completion of its dV/dK MMAs, so the ring depth bounds how
+// far the TMA runs ahead (the 3-deep ring of fa_bwd_dkdv_tc kept ~2000 cycles per tile at the
+// cfg-2 shape, per the tools/attn_trace.py timeline). An S^T / dP^T buffer is released by the
+// commit of the dV/dK MMAs that read the P^T / dS^T written into it.
+constexpr int kRingTS = 4;
+template <int DH>
+__global__ void __launch_bounds__(kThreadsB, 1)
+fa_bwd_dkdv_ts(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_qkv64,
+               const __grid_constant__ CUtensorMap tm_do64, const __grid_constant__ CUtensorMap tm_dqkv,
+               const float* lse, const float* Dd, bf16* dqkv, int B, int s, int nh) {
+  const bool bulk_ld = (s % kCols) == 0;
+  using SM = Smem<DH>;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sK = smem;
+  uint8_t* sV = sK + SM::kBig;
+  auto sQ = [&](int r) { return sV + SM::kBig + 2 * r * SM::kSmall; };
+  auto sG = [&](int r) { return sV + SM::kBig + 2 * r * SM::kSmall + SM::kSmall; };
+  float* sLD = reinterpret_cast<float*>(sV + SM::kBig + 2 * kRingTS * SM::kSmall);   // [ring][2][64]
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sLD + kRingTS * 2 * kCols);
+  uint64_t* kv_full = bar;                 // 1
+  uint64_t* q_full = bar + 1;              // kRingTS
+  uint64_t* q_empty = q_full + kRingTS;    // kRingTS
+  uint64_t* s_full = q_empty + kRingTS;    // 2
+  uint64_t* s_free = s_full + 2;           // 2  (dV/dK MMA commit)
+  uint64_t* p_full = s_free + 2;           // 2  (8 softmax warps)
+  uint64_t* acc_done = p_full + 2;         // 1
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_done + 1);
+
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int nt = (s + kRows - 1) / kRows, BH = B * nh;
+  const int kt = blockIdx.x / BH, bh = blockIdx.x % BH, b = bh / nh, head = bh % nh;   // heaviest first
+  const int h = nh * DH;
+  const long Ttok = static_cast<long>(B) * s;
+  const int i0 = (kt * kRows) / kCols;
+  const int nq = (s + kCols - 1) / kCols;
+  const int ntiles = nq - i0;
+  const float sl2 = rsqrtf(static_cast<float>(DH)) * LOG2E;
+  (void)nt;
+
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&tm_qkv128);
+    tma_prefetch_desc(&tm_qkv64);
+    tma_prefetch_desc(&tm_do64);
+    mbar_init(kv_full, 1);
+    for (int i = 0; i < kRingTS; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); }
+    for (int i = 0; i < 2; ++i) { mbar_init(&s_full[i], 1); mbar_init(&s_free[i], 1); mbar_init(&p_full[i], 8); }
+    mbar_init(acc_done, 1);
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc<512>(tmem_slot);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tm = *tmem_slot;
+  const uint32_t tm_dV = tm, tm_dK = tm + DH, tm_S = tm + 2 * DH, tm_dP = tm + 2 * DH + 2 * kCols;
+
+  if (ntiles <= 0) {
+    __syncthreads();
+    if (warp == 1) tmem_dealloc<512>(tm);
+    return;
+  }
+
+  if (warp == 0) {
+    if (elect_one()) {
+      const int row0 = b * s;
+      mbar_arrive_expect_tx(kv_full, 2 * SM::kBig);
+#pragma unroll
+      for (int a = 0; a < DH / 64; ++a) {
+        tma_load_2d(sK + a * (kRows * 128), &tm_qkv128, kv_full, h + head * DH + a * 64, row0 + kt * kRows);
+        tma_load_2d(sV + a * (kRows * 128), &tm_qkv128, kv_full, 2 * h + head * DH + a * 64, row0 + kt * kRows);
+      }
+      for (int idx = 0; idx < ntiles; ++idx) {
+        const int st = idx % kRingTS;
+        mbar_wait(&q_empty[st], ((idx / kRingTS) & 1) ^ 1);
+        mbar_arrive_expect_tx(&q_full[st], 2 * SM::kSmall + (bulk_ld ? 2 * kCols * 4 : 0));
+        const int qr = row0 + (i0 + idx) * kCols;
+#pragma unroll
+        for (int a = 0; a < DH / 64; ++a) {
+          tma_load_2d(sQ(st) + a * (kCols * 128), &tm_qkv64, &q_full[st], head * DH + a * 64, qr);
+          tma_load_2d(sG(st) + a * (kCols * 128), &tm_do64, &q_full[st], head * DH + a * 64, qr);
+        }
+        if (bulk_ld) {
+          const long o = static_cast<long>(head) * Ttok + qr;
+          bulk_g2s(sLD + st * 2 * kCols, lse + o, kCols * 4, &q_full[st]);
+          bulk_g2s(sLD + st * 2 * kCols + kCols, Dd + o, kCols * 4, &q_full[st]);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    constexpr uint32_t id_s = umma_idesc_bf16(128, kCols, 0, 0);   // S^T, dP^T: K-major A and B
+    constexpr uint32_t id_a = umma_idesc_bf16(128, DH, 0, 1);      // dV, dK: A from TMEM, B MN-major
+    mbar_wait(kv_full, 0);
+    tc_fence_after();
+    auto issue_s = [&](int idx) {
+      const int st = idx % kRingTS, buf = idx & 1;
+      mbar_wait(&q_full[st], (idx / kRingTS) & 1);
+      mbar_wait(&s_free[buf], ((idx >> 1) & 1) ^ 1);
+      tc_fence_after();
+      if (elect_one()) {
+        const uint32_t k = smem_u32(sK), v = smem_u32(sV), q = smem_u32(sQ(st)), g = smem_u32(sG(st));
+#pragma unroll
+        for (int kk = 0; kk < DH / 16; ++kk) {
+          const uint32_t ao = (kk >> 2) * (kRows * 128) + (kk & 3) * 32, bo = (kk >> 2) * (kCols * 128) + (kk & 3) * 32;
+          umma_bf16(tm_S + buf * kCols, umma_desc_sw128(k + ao, 16, 1024), umma_desc_sw128(q + bo, 16, 1024), id_s, kk > 0);
+          umma_bf16(tm_dP + buf * kCols, umma_desc_sw128(v + ao, 16, 1024), umma_desc_sw128(g + bo, 16, 1024), id_s, kk > 0);
+        }
+        umma_commit(&s_full[buf]);
+      }
+      __syncwarp();
+    };
+    auto issue_acc = [&](int idx) {
+      const int st = idx % kRingTS, buf = idx & 1;
+      mbar_wait(&p_full[buf], (idx >> 1) & 1);
+      tc_fence_after();
+      if (elect_one()) {
+        const uint32_t q = smem_u32(sQ(st)), g = smem_u32(sG(st));
+#pragma unroll
+        for (int kk = 0; kk < kCols / 16; ++kk) {
+          // queries [16kk, 16kk + 16): packed columns (kk / 2) * 32 + (kk % 2) * 8 of the buffer
+          const uint32_t ac = buf * kCols + (kk >> 1) * 32 + (kk & 1) * 8;
+          umma_bf16_ts(tm_dV, tm_S + ac, umma_desc_sw128(g + kk * 2048, kCols * 128, 1024), id_a, (idx | kk) != 0);
+          umma_bf16_ts(tm_dK, tm_dP + ac, umma_desc_sw128(q + kk * 2048, kCols * 128, 1024), id_a, (idx | kk) != 0);
+        }
+        umma_commit(&s_free[buf]);
+        umma_commit(&q_empty[st]);
+        if (idx == ntiles - 1) umma_commit(acc_done);
+      }
+      __syncwarp();
+    };
+    issue_s(0);
+    for (int idx = 1; idx < ntiles; ++idx) {
+      issue_s(idx);
+      issue_acc(idx - 1);
+    }
+    issue_acc(ntiles - 1);
+  } else {
+    const int quarter = warp & 3, half = (warp - 2) >> 2;   // S columns [32 half, 32 half + 32)
+    const int row = quarter * 32 + lane;                     // key row within the tile
+    const int key = kt * kRows + row;
+    const uint32_t lane_off = static_cast<uint32_t>(quarter * 32) << 16;
+    const int tid = threadIdx.x - 64;
+    for (int idx = 0; idx < ntiles; ++idx) {
+      const int buf = idx & 1, i = i0 + idx, st = idx % kRingTS;
+      float* ld = sLD + st * 2 * kCols;
+      if (bulk_ld) {
+        mbar_wait(&q_full[st], (idx / kRingTS) & 1);
+      } else {
+        if (tid < 128) {
+          const int c = tid & 63, qq = i * kCols + c;
+          const long r = static_cast<long>(b) * s + (qq < s ? qq : 0);
+          ld[tid] = tid < 64 ? lse[static_cast<long>(head) * Ttok + r] : Dd[static_cast<long>(head) * Ttok + r];
+        }
+        named_bar(1, 256);
+      }
+      float lv[32], dv[32];
+#pragma unroll
+      for (int c = 0; c < 32; c += 4) {
+        const float4 a = ld_shared_f4(ld + half * 32 + c);
+        const float4 d = ld_shared_f4(ld + kCols + half * 32 + c);
+        lv[c] = a.x * LOG2E; lv[c + 1] = a.y * LOG2E; lv[c + 2] = a.z * LOG2E; lv[c + 3] = a.w * LOG2E;
+        dv[c] = d.x; dv[c + 1] = d.y; dv[c + 2] = d.z; dv[c + 3] = d.w;
+      }
+      mbar_wait(&s_full[buf], (idx >> 1) & 1);
+      tc_fence_after();
+      uint32_t sr[32], dr[32];
+      const uint32_t col = buf * kCols + half * 32 + lane_off;
+      tmem_ld_32x32b_x32(tm_S + col, sr);
+      tmem_ld_32x32b_x32(tm_dP + col, dr);
+      tmem_ld_wait();
+      uint32_t pk[16], dk[16];
+      const bool edge = i * kCols < kt * kRows + kRows || i * kCols + kCols > s;
+#pragma unroll
+      for (int c = 0; c < 32; c += 2) {
+        float p0 = ex2(__uint_as_float(sr[c]) * sl2 - lv[c]);
+        float p1 = ex2(__uint_as_float(sr[c + 1]) * sl2 - lv[c + 1]);
+        if (edge) {
+          const int qq = i * kCols + half * 32 + c;
+          if (qq < key || qq >= s) p0 = 0.f;
+          if (qq + 1 < key || qq + 1 >= s) p1 = 0.f;
+        }
+        const float d0 = p0 * (__uint_as_float(dr[c]) - dv[c]), d1 = p1 * (__uint_as_float(dr[c + 1]) - dv[c + 1]);
+        const __nv_bfloat162 pp = __floats2bfloat162_rn(p0, p1), dd = __floats2bfloat162_rn(d0, d1);
+        pk[c / 2] = *reinterpret_cast<const uint32_t*>(&pp);
+        dk[c / 2] = *reinterpret_cast<const uint32_t*>(&dd);
+      }
+      tmem_st_32x32b_x16(tm_S + col, pk);
+      tmem_st_32x32b_x16(tm_dP + col, dk);
+      tmem_st_wait();
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(&p_full[buf]);
+    }
+    if (half == 1) goto done_ts;
+    mbar_wait(acc_done, 0);
+    tc_fence_after();
+    {
+      const float scale = rsqrtf(static_cast<float>(DH));
+      const bool tma_st = (s % kRows) == 0;
+      // staging for the TMA stores: the (now idle) ring slots 0 and 1, four 128-row x 128-byte tiles
+      auto stV = [&](int a) { return a ? sG(0) : sQ(0); };
+      auto stK = [&](int a) { return a ? sG(1) : sQ(1); };
+      const long krow_idx = static_cast<long>(b) * s + (key < s ? key : 0);
+      bf16* krow = dqkv + krow_idx * (3 * h) + h + head * DH;
+      bf16* vrow = krow + h;
+#pragma unroll 1
+      for (int c = 0; c < DH; c += 32) {
+        uint32_t rv[32], rk[32];
+        tmem_ld_32x32b_x32(tm_dV + c + lane_off, rv);
+        tmem_ld_32x32b_x32(tm_dK + c + lane_off, rk);
+        tmem_ld_wait();
+        if (tma_st && kRingTS >= 2 && ntiles >= 2) {
+          float fv[32], fk[32];
+#pragma unroll
+          for (int e = 0; e < 32; ++e) { fv[e] = __uint_as_float(rv[e]); fk[e] = __uint_as_float(rk[e]) * scale; }
+          st_half_row_sw128(stV(c / 64), row, (c % 64) / 8, fv);
+          st_half_row_sw128(stK(c / 64), row, (c % 64) / 8, fk);
+        } else if (key < s) {
+#pragma unroll
+          for (int q = 0; q < 4; ++q) {
+            uint4 uv, uk;
+            __nv_bfloat162* hv = reinterpret_cast<__nv_bfloat162*>(&uv);
+            __nv_bfloat162* hk = reinterpret_cast<__nv_bfloat162*>(&uk);
+#pragma unroll
+            for (int e = 0; e < 4; ++e) {
+              hv[e] = __floats2bfloat162_rn(__uint_as_float(rv[8 * q + 2 * e]), __uint_as_float(rv[8 * q + 2 * e + 1]));
+              hk[e] = __floats2bfloat162_rn(__uint_as_float(rk[8 * q + 2 * e]) * scale,
+                                            __uint_as_float(rk[8 * q + 2 * e + 1]) * scale);
+            }
+            *reinterpret_cast<uint4*>(vrow + c + 8 * q) = uv;
+            *reinterpret_cast<uint4*>(krow + c + 8 * q) = uk;
+          }
+        }
+      }
+      if (tma_st && ntiles >= 2) {
+        fence_proxy_async();
+        named_bar(2, 128);
+        if (threadIdx.x == 64) {
+          const int r0 = b * s + kt * kRows;
+#pragma unroll
+          for (int a = 0; a < DH / 64; ++a) {
+            tma_store_2d(&tm_dqkv, stV(a), 2 * h + head * DH + a * 64, r0);
+            tma_store_2d(&tm_dqkv, stK(a), h + head * DH + a * 64, r0);
+          }
+          bulk_commit_wait_read();
+        }
+      }
+    }
+  }
+done_ts:
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) tmem_dealloc<512>(tm);
+}
+
 // ----------------------------------------------------------------- dQ, persistent
 // fa_bwd_dq_pers: the dQ kernel as a persistent grid (one CTA per SM) over work items (sample, head,
 // 128-query tile) in the same heavy-first order, CTA c taking items c, c + grid, ... The per-CTA
@@ -857,6 +1129,8 @@ template <int DH>
 constexpr int smem_dkdv() { return at_least_one_sm(2 * Smem<DH>::kBig + 2 * kRingKV * Smem<DH>::kSmall + 4 * Smem<DH>::kP + kRingKV * 2 * kCols * 4 + 256 + 1024); }
 template <int DH>
 constexpr int smem_dq() { return at_least_one_sm(2 * Smem<DH>::kBig + 2 * kRing * Smem<DH>::kSmall + 2 * Smem<DH>::kP + 256 + 1024); }
+template <int DH>
+constexpr int smem_dkdv_ts() { return at_least_one_sm(2 * Smem<DH>::kBig + 2 * kRingTS * Smem<DH>::kSmall + kRingTS * 2 * kCols * 4 + 256 + 1024); }
 int g_attn_dq_pers = 1;   // MARIO_ATTN_DQ_PERS=0 selects the one-item-per-CTA dQ kernel
 
 template <int DH>
@@ -883,7 +1157,33 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
   const int dbg = dbgs ? atoi(dbgs) : 0;
   const char* only = getenv("MARIO_ATTN_TC_ONLY");   // debugging aid: "dkdv" or "dq"
   if (!only || only[1] == 'k')
-    fa_bwd_dkdv_tc<DH><<<grid, kThreadsB, smem_dkdv<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s, nh, dbg);
+  {
+    static long long* trace = nullptr;
+    const bool want_trace = getenv("MARIO_ATTN_TRACE") != nullptr;
+    if (want_trace && !trace) { cudaMalloc(&trace, 8 * 64 * sizeof(long long)); cudaMemset(trace, 0, 8 * 64 * sizeof(long long)); }
+    static const bool ts = getenv("MARIO_ATTN_DKDV_TS") ? atoi(getenv("MARIO_ATTN_DKDV_TS")) != 0 : true;
+    if (ts && dbg == 0 && !want_trace) {
+      static bool tset = false;
+      if (!tset) {
+        cudaFuncSetAttribute(fa_bwd_dkdv_ts<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_dkdv_ts<DH>());
+        tset = true;
+      }
+      fa_bwd_dkdv_ts<DH><<<grid, kThreadsB, smem_dkdv_ts<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s, nh);
+    } else {
+      fa_bwd_dkdv_tc<DH><<<grid, kThreadsB, smem_dkdv<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s, nh, dbg,
+                                                                     want_trace ? trace : nullptr);
+    }
+    if (want_trace) {
+      long long h[8 * 64];
+      cudaStreamSynchronize(st);
+      cudaMemcpy(h, trace, sizeof(h), cudaMemcpyDeviceToHost);
+      const long long t0 = h[0];
+      fprintf(stderr, "tile  s_wait  s_issued  acc_wait  acc_go | sm_wait  sm_go  sm_math_done  sm_pfull\n");
+      for (int i = 0; i < 32; ++i)
+        fprintf(stderr, "%3d %8lld %8lld %8lld %8lld | %8lld %8lld %8lld %8lld\n", i, h[i] - t0, h[64 + i] - t0,
+                h[128 + i] - t0, h[192 + i] - t0, h[256 + i] - t0, h[320 + i] - t0, h[384 + i] - t0, h[448 + i] - t0);
+    }
+  }
   static const bool pers = getenv("MARIO_ATTN_DQ_PERS") ? atoi(getenv("MARIO_ATTN_DQ_PERS")) != 0 : g_attn_dq_pers != 0;
   if (!only || only[1] == 'q') {
     if (pers && dbg == 0) {
