@@ -66,6 +66,17 @@ int mario_k_attn_set_variant(int variant);
  * deterministic (no atomics). scratch: fp32 [n_heads][B*s]. */
 int mario_k_attn_bwd(const void* qkv, const void* O, const void* dO, const float* lse, void* dqkv,
                      float* scratch, int B, int s, int n_heads, int head_dim, int bf16, void* stream);
+/* K6 with a dS workspace (bf16 only; SURVEY §8(c) c1 attention backward: dS = P (dP - D), dQ =
+ * dS K / sqrt(dh)): the tcgen05 dK/dV kernel also stores dS (bf16, the values its dK MMA uses) into
+ * ds_ws as per-(sample, head, 128-query block) tiles over the causal key tiles, and dQ is then one
+ * product per tile over that image (no S / dP recompute). ds_ws: device, caller-owned, at least
+ * mario_k_attn_bwd_ws_bytes(B, s, n_heads, head_dim) bytes, contents undefined on return. When
+ * that size is 0 (head_dim not 64/128, s not a multiple of 128) or ds_ws_bytes is smaller, this is
+ * mario_k_attn_bwd. Deterministic. Returns the CUDA error code (0 = OK). */
+size_t mario_k_attn_bwd_ws_bytes(int B, int s, int n_heads, int head_dim);
+int mario_k_attn_bwd_ws(const void* qkv, const void* O, const void* dO, const float* lse, void* dqkv,
+                        float* scratch, void* ds_ws, size_t ds_ws_bytes, int B, int s, int n_heads, int head_dim,
+                        void* stream);
 
 /* K7/K8: LayerNorm (rms = 0: y = (x - mean)/sqrt(var + eps) * g + b) or RMSNorm (rms = 1:
  * y = x / sqrt(mean(x^2) + eps) * g) over rows of width n; stats =

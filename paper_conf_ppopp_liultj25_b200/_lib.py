@@ -21,6 +21,8 @@ _SIGS = {
                                vp, i32, vp, vp, i32, vp]),
     "mario_k_attn_fwd": (i32, [vp, vp, vp, i32, i32, i32, i32, i32, vp]),
     "mario_k_attn_bwd": (i32, [vp, vp, vp, vp, vp, vp, i32, i32, i32, i32, i32, vp]),
+    "mario_k_attn_bwd_ws_bytes": (C.c_size_t, [i32, i32, i32, i32]),
+    "mario_k_attn_bwd_ws": (i32, [vp, vp, vp, vp, vp, vp, vp, C.c_size_t, i32, i32, i32, i32, vp]),
     "mario_k_norm_fwd": (i32, [vp, vp, vp, vp, vp, i32, i32, f32, i32, i32, vp]),
     "mario_k_norm_bwd": (i32, [vp, vp, vp, vp, vp, vp, vp, vp, vp, vp, C.c_longlong, i32, i32, i32, i32, vp]),
     "mario_k_norm_set_variant": (i32, [i32]),

@@ -74,6 +74,20 @@ extern "C" int mario_k_attn_bwd(const void* qkv, const void* O, const void* dO, 
   return static_cast<int>(cudaGetLastError());
 }
 
+extern "C" size_t mario_k_attn_bwd_ws_bytes(int B, int s, int n_heads, int head_dim) {
+  return flash_attn_bwd_ds_bytes(head_dim, B, s, n_heads);
+}
+
+extern "C" int mario_k_attn_bwd_ws(const void* qkv, const void* O, const void* dO, const float* lse, void* dqkv,
+                                   float* scratch, void* ds_ws, size_t ds_ws_bytes, int B, int s, int n_heads,
+                                   int head_dim, void* stream) {
+  cudaStream_t st = static_cast<cudaStream_t>(stream);
+  attn_bwd<__nv_bfloat16>(static_cast<const __nv_bfloat16*>(qkv), static_cast<const __nv_bfloat16*>(O),
+                          static_cast<const __nv_bfloat16*>(dO), lse, static_cast<__nv_bfloat16*>(dqkv), scratch, B, s,
+                          n_heads, head_dim, st, ds_ws, ds_ws_bytes);
+  return static_cast<int>(cudaGetLastError());
+}
+
 extern "C" int mario_k_norm_fwd(const void* x, const float* g, const float* b, void* y, float* stats, int rows, int n,
                                 float eps, int rms, int bf16, void* stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);

@@ -378,7 +378,7 @@ struct Exec {
         lin_wgrad(dH1, O, Tn, h, h, G(D, p, pre + "o.w"));
         lin_dgrad(dH1, Wm(D, p, pre + "o.w"), Tn, h, h, dO);
       }
-      attn_bwd<T>(QKV, O, dO, LSE, dQKV, Dsc, mbs, s, nh, dh, st);
+      attn_bwd<T>(QKV, O, dO, LSE, dQKV, Dsc, mbs, s, nh, dh, st, BS.dS_bytes ? sc + BS.dS : nullptr, BS.dS_bytes);
       if (!gpt) rope<T>(dQKV, mbs, s, nh, dh, m.rope_base, 1, st);
       if (gpt) layernorm_fwd<T>(Hin, Wf(D, p, pre + "ln1.g"), Wf(D, p, pre + "ln1.b"), A, st1, Tn, h, m.norm_eps, st);
       else rmsnorm_fwd<T>(Hin, Wf(D, p, pre + "n1.g"), A, st1, Tn, h, m.norm_eps, st);

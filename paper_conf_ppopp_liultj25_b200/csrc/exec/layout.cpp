@@ -4,6 +4,8 @@
 
 #include "../plan/model.h"
 
+namespace mario { size_t flash_attn_bwd_ds_bytes(int dh, int B, int s, int nh); }   // kernels/attn_tc.cu
+
 namespace mario {
 
 size_t elt_size(const mario_model& m) { return m.dtype == MARIO_BF16 ? 2 : 4; }
@@ -82,6 +84,14 @@ BwScratch bw_scratch_layout(const mario_model& m) {
   b.Dsc = take(static_cast<size_t>(m.n_heads) * T * 4);
   b.sort = take(T * 8 * 2);
   b.Arec = take(T * h * E);
+  // the attention backward's dS image (fa_bwd_dq_img: dQ from the stored dS, no S/dP recompute);
+  // only where it stays small next to the rest of the scratch (not at s = 16384)
+  b.dS_bytes = 0;
+  if (m.dtype == MARIO_BF16) {
+    const size_t ds = flash_attn_bwd_ds_bytes(h / m.n_heads, m.micro_batch, m.seq_len, m.n_heads);
+    if (ds > 0 && ds <= (static_cast<size_t>(1) << 30)) b.dS_bytes = ds;
+  }
+  b.dS = take(b.dS_bytes);
   b.bytes = o;
   return b;
 }

@@ -43,6 +43,7 @@ size_t cfw_work_bytes(const mario_model& m, int k, int K);       // transient CF
 // Backward scratch (shared by every BW of the rank): rotating dH buffers and per-layer grads.
 struct BwScratch {
   size_t dH[3], dA, dQKV, dO, dZ, dM, Dsc, sort, Arec;   // dM doubles as the G/M recompute buffer
+  size_t dS, dS_bytes;   // attention dS image (bf16, when the shape allows it and it is <= 1 GiB; else 0 bytes)
   size_t bytes;
 };
 BwScratch bw_scratch_layout(const mario_model& m);

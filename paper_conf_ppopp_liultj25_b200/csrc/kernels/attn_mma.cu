@@ -14,7 +14,8 @@ namespace mario {
 
 int g_attn_variant = -1;   // mario_k_attn_set_variant: -1 auto (tcgen05 where supported), 0 mma.sync only
 bool flash_attn_bwd_tc(const __nv_bfloat16* qkv, const __nv_bfloat16* dO, const float* lse, const float* Dd,
-                       __nv_bfloat16* dqkv, int B, int s, int nh, int dh, cudaStream_t st);   // attn_tc.cu
+                       __nv_bfloat16* dqkv, int B, int s, int nh, int dh, void* ds_ws, size_t ds_ws_bytes,
+                       cudaStream_t st);   // attn_tc.cu
 bool flash_attn_fwd_tc(const __nv_bfloat16* qkv, __nv_bfloat16* O, float* lse, int B, int s, int nh, int dh,
                        cudaStream_t st);   // attn_tc.cu
 
@@ -464,7 +465,7 @@ void launch_fwd(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, cuda
 }
 template <int D>
 void launch_bwd(const bf16* qkv, const bf16* O, const bf16* dO, const float* lse, bf16* dqkv, float* Dd, int B, int s,
-                int nh, cudaStream_t st) {
+                int nh, cudaStream_t st, void* ds_ws, size_t ds_ws_bytes) {
   const long Ttok = static_cast<long>(B) * s;
   {
     const long thr = Ttok * nh * (D / 8);
@@ -478,7 +479,7 @@ void launch_bwd(const bf16* qkv, const bf16* O, const bf16* dO, const float* lse
   if (g_attn_variant != 0) {   // tcgen05 backward (attn_tc.cu) when supported
     const double fl = 8.0 * B * nh * D * (static_cast<double>(s) * (s + 1) / 2);
     const int tok = kstats_begin(K_ATTN_BWD, fl, 0.0, st);
-    const bool ok = flash_attn_bwd_tc(qkv, dO, lse, Dd, dqkv, B, s, nh, D, st);
+    const bool ok = flash_attn_bwd_tc(qkv, dO, lse, Dd, dqkv, B, s, nh, D, ds_ws, ds_ws_bytes, st);
     kstats_end(tok, st);
     if (ok) { note_launch(); return; }
   }
@@ -515,13 +516,13 @@ void flash_attn_fwd(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, 
 }
 
 void flash_attn_bwd(const bf16* qkv, const bf16* O, const bf16* dO, const float* lse, bf16* dqkv, float* Dd, int B,
-                    int s, int nh, int dh, cudaStream_t st) {
+                    int s, int nh, int dh, cudaStream_t st, void* ds_ws, size_t ds_ws_bytes) {
   switch (dh) {
-    case 16: launch_bwd<16>(qkv, O, dO, lse, dqkv, Dd, B, s, nh, st); break;
-    case 32: launch_bwd<32>(qkv, O, dO, lse, dqkv, Dd, B, s, nh, st); break;
-    case 64: launch_bwd<64>(qkv, O, dO, lse, dqkv, Dd, B, s, nh, st); break;
-    case 80: launch_bwd<80>(qkv, O, dO, lse, dqkv, Dd, B, s, nh, st); break;
-    default: launch_bwd<128>(qkv, O, dO, lse, dqkv, Dd, B, s, nh, st); break;
+    case 16: launch_bwd<16>(qkv, O, dO, lse, dqkv, Dd, B, s, nh, st, ds_ws, ds_ws_bytes); break;
+    case 32: launch_bwd<32>(qkv, O, dO, lse, dqkv, Dd, B, s, nh, st, ds_ws, ds_ws_bytes); break;
+    case 64: launch_bwd<64>(qkv, O, dO, lse, dqkv, Dd, B, s, nh, st, ds_ws, ds_ws_bytes); break;
+    case 80: launch_bwd<80>(qkv, O, dO, lse, dqkv, Dd, B, s, nh, st, ds_ws, ds_ws_bytes); break;
+    default: launch_bwd<128>(qkv, O, dO, lse, dqkv, Dd, B, s, nh, st, ds_ws, ds_ws_bytes); break;
   }
 }
 

@@ -30,6 +30,8 @@ extern int g_attn_variant;   // attn_mma.cu
 bool make_tmap_bf16_2d(CUtensorMap* map, const void* base, uint64_t inner, uint64_t outer, uint64_t ld,
                        uint32_t box_inner, uint32_t box_outer);   // gemm_tc.cu
 
+size_t flash_attn_bwd_ds_bytes(int dh, int B, int s, int nh);   // below
+
 namespace {
 using namespace sm100;
 using bf16 = __nv_bfloat16;
@@ -635,8 +637,9 @@ constexpr int kRingTS = 4;
 template <int DH>
 __global__ void __launch_bounds__(kThreadsB, 1)
 fa_bwd_dkdv_ts(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_qkv64,
-               const __grid_constant__ CUtensorMap tm_do64, const __grid_constant__ CUtensorMap tm_dqkv,
-               const float* lse, const float* Dd, bf16* dqkv, int B, int s, int nh) {
+               const __grid_constant__ CUtensorMap tm_do64,
+               const __grid_constant__ CUtensorMap tm_dqkv, const float* lse, const float* Dd, bf16* dqkv, int B,
+               int s, int nh, uint8_t* dsimg) {
   const bool bulk_ld = (s % kCols) == 0;
   using SM = Smem<DH>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -815,6 +818,19 @@ fa_bwd_dkdv_ts(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
       }
       tmem_st_32x32b_x16(tm_S + col, pk);
       tmem_st_32x32b_x16(tm_dP + col, dk);
+      if (dsimg) {
+        // dS for fa_bwd_dq_img: key row `key`, queries [64 i + 32 half, + 32) of query block i / 2,
+        // written as the 128-byte row (key mod 64) of the MN-major SW128 image of dQ's A operand
+        // (16-byte chunk c of row r at ((c ^ (r mod 8)) << 4), the layout TMA's 128B swizzle makes)
+        const int qb = i >> 1, kt64 = key >> 6, r64 = key & 63;
+        const size_t tri = static_cast<size_t>(s / kRows) * (s / kRows + 1);
+        uint8_t* rowp = dsimg + ((static_cast<size_t>(bh) * tri + static_cast<size_t>(qb) * (qb + 1) + kt64) * 2 + (i & 1)) * 8192 +
+                        r64 * 128;
+#pragma unroll
+        for (int jj = 0; jj < 4; ++jj)
+          *reinterpret_cast<uint4*>(rowp + (((4 * half + jj) ^ (r64 & 7)) << 4)) =
+              make_uint4(dk[4 * jj], dk[4 * jj + 1], dk[4 * jj + 2], dk[4 * jj + 3]);
+      }
       tmem_st_wait();
       tc_fence_before();
       __syncwarp();
@@ -1123,6 +1139,145 @@ fa_bwd_dq_pers(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
   if (warp == 1) tmem_dealloc<512>(tm);
 }
 
+// ------------------------------------------------------------------ dQ from the dS image
+// fa_bwd_dq_img: dQ = dS K / sqrt(dh) with dS taken from the image fa_bwd_dkdv_ts wrote (when the
+// caller provides the workspace), so nothing is recomputed: 1 MMA per tile instead of the 3 of the
+// recomputing dQ kernels (S = Q K^T and dP = dO V^T again, plus the softmax). Image layout per
+// (sample, head) and 128-query block qb: the 2 qb + 2 key tiles of 64 (causal) at index
+// qb (qb + 1) + kt, each 2 x 8 KB boxes (queries [0,64) / [64,128) of the block) holding 64 key rows
+// x 64 queries, MN-major with the 128-byte swizzle -- exactly the shared-memory image of the MMA's
+// A operand (M = queries, K = keys), so the producer moves it with one 16 KB bulk copy.
+// Persistent (one CTA per SM) over items (query block, sample, head), heaviest first. Warps: 0 TMA,
+// 1 MMA (dQ double-buffered in TMEM), 2..5 epilogue (one query row per thread).
+constexpr int kThreadsI = 192;
+constexpr int kRingI = 6;
+template <int DH>
+struct SmemI {
+  static constexpr int kA = kRows * kCols * 2;       // 16 KB dS image tile
+  static constexpr int kK = kCols * DH * 2;          // K tile (64 keys)
+  static constexpr int kStage = kA + kK;
+  static constexpr int kBytes = kRingI * kStage + 256 + 1024;
+};
+template <int DH>
+__global__ void __launch_bounds__(kThreadsI, 1)
+fa_bwd_dq_img(const __grid_constant__ CUtensorMap tm_qkv64, const uint8_t* __restrict__ dsimg, bf16* dqkv, int B, int s,
+              int nh) {
+  using SI = SmemI<DH>;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint64_t* bar = reinterpret_cast<uint64_t*>(smem + kRingI * SI::kStage);
+  uint64_t* full = bar;                    // kRingI
+  uint64_t* empty = full + kRingI;         // kRingI
+  uint64_t* acc_full = empty + kRingI;     // 2
+  uint64_t* acc_empty = acc_full + 2;      // 2
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_empty + 2);
+
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int nt = s / kRows, BH = B * nh, W = nt * BH;
+  const int h = nh * DH;
+  const size_t tri = static_cast<size_t>(nt) * (nt + 1);
+  auto item = [&](int w, int& qb, int& bh, int& ntiles) {
+    qb = nt - 1 - w / BH; bh = w % BH;
+    ntiles = 2 * qb + 2;
+  };
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&tm_qkv64);
+    for (int i = 0; i < kRingI; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
+    for (int i = 0; i < 2; ++i) { mbar_init(&acc_full[i], 1); mbar_init(&acc_empty[i], 4); }
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc<2 * DH>(tmem_slot);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tm = *tmem_slot;
+
+  if (warp == 0) {
+    if (elect_one()) {
+      int kc = 0;
+      for (int w = blockIdx.x; w < W; w += gridDim.x) {
+        int qb, bh, ntiles;
+        item(w, qb, bh, ntiles);
+        const int b = bh / nh, head = bh % nh;
+        const uint8_t* img = dsimg + (static_cast<size_t>(bh) * tri + static_cast<size_t>(qb) * (qb + 1)) * SI::kA;
+        for (int kt = 0; kt < ntiles; ++kt, ++kc) {
+          const int st = kc % kRingI;
+          uint8_t* sa = smem + st * SI::kStage;
+          mbar_wait(&empty[st], ((kc / kRingI) & 1) ^ 1);
+          mbar_arrive_expect_tx(&full[st], SI::kStage);
+          bulk_g2s(sa, img + static_cast<size_t>(kt) * SI::kA, SI::kA, &full[st]);
+#pragma unroll
+          for (int a = 0; a < DH / 64; ++a)
+            tma_load_2d(sa + SI::kA + a * (kCols * 128), &tm_qkv64, &full[st], h + head * DH + a * 64, b * s + kt * kCols);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    constexpr uint32_t id = umma_idesc_bf16(128, DH, 1, 1);   // A = dS image (MN-major), B = K_j (MN-major)
+    int kc = 0, n = 0;
+    for (int w = blockIdx.x; w < W; w += gridDim.x, ++n) {
+      int qb, bh, ntiles;
+      item(w, qb, bh, ntiles);
+      const uint32_t acc = tm + (n & 1) * DH;
+      mbar_wait(&acc_empty[n & 1], ((n >> 1) & 1) ^ 1);
+      tc_fence_after();
+      for (int kt = 0; kt < ntiles; ++kt, ++kc) {
+        const int st = kc % kRingI;
+        mbar_wait(&full[st], (kc / kRingI) & 1);
+        tc_fence_after();
+        if (elect_one()) {
+          const uint32_t sa = smem_u32(smem + st * SI::kStage), sk = sa + SI::kA;
+#pragma unroll
+          for (int kk = 0; kk < kCols / 16; ++kk)
+            umma_bf16(acc, umma_desc_sw128(sa + kk * 2048, 8192, 1024), umma_desc_sw128(sk + kk * 2048, kCols * 128, 1024),
+                      id, (kt | kk) != 0);
+          umma_commit(&empty[st]);
+          if (kt == ntiles - 1) umma_commit(&acc_full[n & 1]);
+        }
+        __syncwarp();
+      }
+    }
+  } else {
+    const int quarter = warp & 3;
+    const int row = quarter * 32 + lane;
+    const uint32_t lane_off = static_cast<uint32_t>(quarter * 32) << 16;
+    const float scale = rsqrtf(static_cast<float>(DH));
+    int n = 0;
+    for (int w = blockIdx.x; w < W; w += gridDim.x, ++n) {
+      int qb, bh, ntiles;
+      item(w, qb, bh, ntiles);
+      const int b = bh / nh, head = bh % nh;
+      bf16* qrow = dqkv + (static_cast<long>(b) * s + qb * kRows + row) * (3 * h) + head * DH;
+      mbar_wait(&acc_full[n & 1], (n >> 1) & 1);
+      tc_fence_after();
+#pragma unroll 1
+      for (int c = 0; c < DH; c += 32) {
+        uint32_t rq[32];
+        tmem_ld_32x32b_x32(tm + (n & 1) * DH + c + lane_off, rq);
+        tmem_ld_wait();
+        if (c + 32 == DH) {
+          tc_fence_before();
+          __syncwarp();
+          if (lane == 0) mbar_arrive(&acc_empty[n & 1]);
+        }
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          uint4 u;
+          __nv_bfloat162* hq = reinterpret_cast<__nv_bfloat162*>(&u);
+#pragma unroll
+          for (int f = 0; f < 4; ++f)
+            hq[f] = __floats2bfloat162_rn(__uint_as_float(rq[8 * e + 2 * f]) * scale,
+                                          __uint_as_float(rq[8 * e + 2 * f + 1]) * scale);
+          *reinterpret_cast<uint4*>(qrow + c + 8 * e) = u;
+        }
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) tmem_dealloc<2 * DH>(tm);
+}
+
 // >= 116 KB so that one CTA owns the SM (each allocates all 512 TMEM columns)
 constexpr int at_least_one_sm(int b) { return b < 116 * 1024 ? 116 * 1024 : b; }
 template <int DH>
@@ -1135,7 +1290,7 @@ int g_attn_dq_pers = 1;   // MARIO_ATTN_DQ_PERS=0 selects the one-item-per-CTA d
 
 template <int DH>
 bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, bf16* dqkv, int B, int s, int nh,
-            cudaStream_t st) {
+            uint8_t* dsimg, cudaStream_t st) {
   const int h = nh * DH;
   const long T = static_cast<long>(B) * s;
   CUtensorMap m128, m64, d64, d128, g128;
@@ -1162,13 +1317,16 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
     const bool want_trace = getenv("MARIO_ATTN_TRACE") != nullptr;
     if (want_trace && !trace) { cudaMalloc(&trace, 8 * 64 * sizeof(long long)); cudaMemset(trace, 0, 8 * 64 * sizeof(long long)); }
     static const bool ts = getenv("MARIO_ATTN_DKDV_TS") ? atoi(getenv("MARIO_ATTN_DKDV_TS")) != 0 : true;
+    if (dsimg && (s % kRows) != 0) dsimg = nullptr;
+    if (!(ts && dbg == 0 && !want_trace)) dsimg = nullptr;
     if (ts && dbg == 0 && !want_trace) {
       static bool tset = false;
       if (!tset) {
         cudaFuncSetAttribute(fa_bwd_dkdv_ts<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_dkdv_ts<DH>());
         tset = true;
       }
-      fa_bwd_dkdv_ts<DH><<<grid, kThreadsB, smem_dkdv_ts<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s, nh);
+      fa_bwd_dkdv_ts<DH><<<grid, kThreadsB, smem_dkdv_ts<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s, nh,
+                                                                        dsimg);
     } else {
       fa_bwd_dkdv_tc<DH><<<grid, kThreadsB, smem_dkdv<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s, nh, dbg,
                                                                      want_trace ? trace : nullptr);
@@ -1185,7 +1343,19 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
     }
   }
   static const bool pers = getenv("MARIO_ATTN_DQ_PERS") ? atoi(getenv("MARIO_ATTN_DQ_PERS")) != 0 : g_attn_dq_pers != 0;
-  if (!only || only[1] == 'q') {
+  if (only && only[1] == 'q') dsimg = nullptr;
+  if (dsimg && (!only || only[1] == 'q')) {
+    static bool iset = false;
+    if (!iset) {
+      cudaFuncSetAttribute(fa_bwd_dq_img<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize, SmemI<DH>::kBytes);
+      iset = true;
+    }
+    int sms = 0, dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const int items = B * nh * (s / kRows);
+    fa_bwd_dq_img<DH><<<items < sms ? items : sms, kThreadsI, SmemI<DH>::kBytes, st>>>(m64, dsimg, dqkv, B, s, nh);
+  } else if (!only || only[1] == 'q') {
     if (pers && dbg == 0) {
       static bool pset = false;
       if (!pset) {
@@ -1753,10 +1923,18 @@ bool flash_attn_fwd_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int n
 
 // Returns false if the configuration is unsupported (caller falls back to the mma.sync kernels).
 bool flash_attn_bwd_tc(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, bf16* dqkv, int B, int s,
-                       int nh, int dh, cudaStream_t st) {
-  if (dh == 128) return launch<128>(qkv, dO, lse, Dd, dqkv, B, s, nh, st);
-  if (dh == 64) return launch<64>(qkv, dO, lse, Dd, dqkv, B, s, nh, st);
+                       int nh, int dh, void* ds_ws, size_t ds_ws_bytes, cudaStream_t st) {
+  uint8_t* img = ds_ws && ds_ws_bytes >= flash_attn_bwd_ds_bytes(dh, B, s, nh) ? static_cast<uint8_t*>(ds_ws) : nullptr;
+  if (dh == 128) return launch<128>(qkv, dO, lse, Dd, dqkv, B, s, nh, img, st);
+  if (dh == 64) return launch<64>(qkv, dO, lse, Dd, dqkv, B, s, nh, img, st);
   return false;
+}
+
+// bytes of the dS image fa_bwd_dq_img reads (0: that path does not apply to this shape)
+size_t flash_attn_bwd_ds_bytes(int dh, int B, int s, int nh) {
+  if ((dh != 64 && dh != 128) || s % kRows != 0 || (nh * dh) % 64 != 0) return 0;
+  const size_t nt = static_cast<size_t>(s / kRows);
+  return static_cast<size_t>(B) * nh * nt * (nt + 1) * SmemI<128>::kA;
 }
 
 }  // namespace mario

@@ -188,17 +188,39 @@ __device__ __forceinline__ uint8_t* sw64(uint8_t* sw, int r, int j) { return sw 
 // [32 rows][128 B] fp32 block: chunk j of row r at r*128 + 16*(j ^ (r & 7))
 __device__ __forceinline__ uint8_t* sw128(uint8_t* sw, int r, int j) { return sw + r * 128 + 16 * (j ^ (r & 7)); }
 
-// coalesced load of a bf16 [32 rows][32 cols] block (rows >= M read as 0) into sw, then each lane
-// reads back its own row's 32 values
-__device__ __forceinline__ void load_block_bf16(const __nv_bfloat16* base, int ld, int rbase, int col0, int M, int lane,
-                                                uint8_t* sw, float (&out)[32]) {
+// Global reads of one 32x32 epilogue block issued ahead of their use (software pipelining): the
+// bf16 input the block needs (GeLU aux, else residual) is loaded into registers one block ahead --
+// right after the previous block's copy was moved to shared memory, and for a tile's first block
+// before the accumulator wait -- so the global latency overlaps work instead of stalling each
+// block. 4 lanes per 64-byte row segment (coalesced). fp32 += (wgrad) reads stay in-block.
+struct EpiPrefetch { uint4 v[4]; };
+__device__ __forceinline__ void epi_prefetch(const GemmEpilogue& ep, bool vec_ok, int rbase, int lane, int col0, int M,
+                                             int N, EpiPrefetch& pf) {
+  if (col0 < 0 || col0 >= N || !vec_ok || col0 + 32 > N) return;
+  const __nv_bfloat16* base = ep.aux ? ep.aux : ep.residual;
+  if (!base) return;
+  const int ld = ep.aux ? ep.ld_aux : ep.ld_res;
 #pragma unroll
   for (int it = 0; it < 4; ++it) {
     const int rr = it * 8 + lane / 4, ch = lane % 4;
-    uint4 u = make_uint4(0, 0, 0, 0);
-    if (rbase + rr < M) u = *reinterpret_cast<const uint4*>(base + static_cast<size_t>(rbase + rr) * ld + col0 + ch * 8);
-    sts128(sw64(sw, rr, ch), u);
+    pf.v[it] = rbase + rr < M ? *reinterpret_cast<const uint4*>(base + static_cast<size_t>(rbase + rr) * ld + col0 + ch * 8)
+                              : make_uint4(0, 0, 0, 0);
   }
+}
+// direct (not prefetched) coalesced read of a bf16 block into registers, same layout
+__device__ __forceinline__ void epi_rows_bf16(const __nv_bfloat16* base, int ld, int rbase, int col0, int M, int lane,
+                                              uint4* out) {
+#pragma unroll
+  for (int it = 0; it < 4; ++it) {
+    const int rr = it * 8 + lane / 4, ch = lane % 4;
+    out[it] = rbase + rr < M ? *reinterpret_cast<const uint4*>(base + static_cast<size_t>(rbase + rr) * ld + col0 + ch * 8)
+                             : make_uint4(0, 0, 0, 0);
+  }
+}
+// prefetched bf16 [32 rows][32 cols] block -> sw -> each lane reads back its own row's 32 values
+__device__ __forceinline__ void load_block_bf16(const uint4* pre, int lane, uint8_t* sw, float (&out)[32]) {
+#pragma unroll
+  for (int it = 0; it < 4; ++it) sts128(sw64(sw, it * 8 + lane / 4, lane % 4), pre[it]);
   __syncwarp();
 #pragma unroll
   for (int j = 0; j < 4; ++j) {
@@ -235,10 +257,12 @@ __device__ __forceinline__ void store_block_bf16(__nv_bfloat16* base, int ld, in
 }
 
 __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool vec_ok, const uint32_t (&r)[32],
-                                                    int rbase, int lane, int col0, int M, int N, uint8_t* sw) {
+                                                    int rbase, int lane, int col0, int M, int N, uint8_t* sw,
+                                                    EpiPrefetch& pf, int next_col0) {
   if (col0 >= N) return;
   if (!vec_ok || col0 + 32 > N) {   // warp-uniform: ragged column block or unaligned pitches
     epilogue_chunk(ep, r, rbase + lane, col0, rbase + lane < M, N);
+    epi_prefetch(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
     return;
   }
   float v[32];
@@ -253,13 +277,21 @@ __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool
   }
   float z[32];
   if (ep.aux) {   // GeLU backward: D = acc * gelu'(Z)
-    load_block_bf16(ep.aux, ep.ld_aux, rbase, col0, M, lane, sw, z);
+    load_block_bf16(pf.v, lane, sw, z);
+    epi_prefetch(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
 #pragma unroll
     for (int j = 0; j < 32; ++j) v[j] *= gelu_tanh_grad_f(z[j]);
   }
   if (ep.residual) {
     float rr[32];
-    load_block_bf16(ep.residual, ep.ld_res, rbase, col0, M, lane, sw, rr);
+    if (ep.aux) {   // never both in the executor; the prefetch slot holds aux then
+      uint4 rv[4];
+      epi_rows_bf16(ep.residual, ep.ld_res, rbase, col0, M, lane, rv);
+      load_block_bf16(rv, lane, sw, rr);
+    } else {
+      load_block_bf16(pf.v, lane, sw, rr);
+      epi_prefetch(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
+    }
 #pragma unroll
     for (int j = 0; j < 32; ++j) v[j] += rr[j];
   }
@@ -411,15 +443,17 @@ gemm_bf16_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
       int tm, tn;
         tile_coords(tile, num_m, num_n, n_fastest, tm, tn);
       const int m0 = tm * BM, n0 = tn * BN;
+      const int rbase = m0 + quarter * 32;
+      EpiPrefetch pf;
+      epi_prefetch(ep, vec_ok, rbase, lane, n0, M, N, pf);
       mbar_wait(&tfull[acc], acc_ph);
       tc_fence_after();
-      const int rbase = m0 + quarter * 32;
 #pragma unroll 1
       for (int c = 0; c < BN / 32; ++c) {
         uint32_t r[32];
         tmem_ld_32x32b_x32(tmem_base + acc * BN + c * 32 + (static_cast<uint32_t>(quarter * 32) << 16), r);
         tmem_ld_wait();
-        epilogue_chunk_warp(ep, vec_ok, r, rbase, lane, n0 + c * 32, M, N, sw);
+        epilogue_chunk_warp(ep, vec_ok, r, rbase, lane, n0 + c * 32, M, N, sw, pf, c + 1 < BN / 32 ? n0 + (c + 1) * 32 : -1);
       }
       tc_fence_before();
       mbar_arrive(&tempty[acc]);
@@ -618,10 +652,12 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
       int tm, tn;
         tile_coords(tile, num_m, num_n, n_fastest, tm, tn);
       const int m0 = tm * 256 + 128 * rank, n0 = tn * BNP;
+      const int rbase = m0 + quarter * 32;
+      EpiPrefetch pf;
+      if (!(skon && u.kb0 != 0)) epi_prefetch(ep, vec_ok, rbase, lane, n0 + half * (BNP / 2), M, N, pf);
       if (sk.sleep_ns) { while (!mbar_test(&tfull[acc], acc_ph)) __nanosleep(sk.sleep_ns); }
       else mbar_wait(&tfull[acc], acc_ph);
       tc_fence_after();
-      const int rbase = m0 + quarter * 32;
       const int lrow = quarter * 32 + lane;                     // accumulator row within this CTA
       if (skon && u.kb0 != 0) {
         // later k-part of a split tile (this pair's first unit): raw partial to ws[pair]
@@ -669,7 +705,8 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
               r[4 * e + 3] = __float_as_uint(__uint_as_float(r[4 * e + 3]) + pv.w);
             }
           }
-          epilogue_chunk_warp(ep, vec_ok, r, rbase, lane, n0 + col, M, N, sw);
+          epilogue_chunk_warp(ep, vec_ok, r, rbase, lane, n0 + col, M, N, sw, pf,
+                              c + 1 < BNP / 64 ? n0 + col + 32 : -1);
         }
         if (q1 > pair + 1) {
           asm volatile("bar.sync 1, 256;" ::: "memory");

@@ -1176,10 +1176,14 @@ void attn_fwd(const T* qkv, T* O, float* lse, int B, int s, int nh, int dh, cuda
 }
 template <class T>
 void attn_bwd(const T* qkv, const T* O, const T* dO, const float* lse, T* dqkv, float* Dsc, int B, int s, int nh,
-              int dh, cudaStream_t st) {
+              int dh, cudaStream_t st, void* ds_ws, size_t ds_ws_bytes) {
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
-    if (flash_attn_supported(dh)) { flash_attn_bwd(qkv, O, dO, lse, dqkv, Dsc, B, s, nh, dh, st); return; }
+    if (flash_attn_supported(dh)) {
+      flash_attn_bwd(qkv, O, dO, lse, dqkv, Dsc, B, s, nh, dh, st, ds_ws, ds_ws_bytes);
+      return;
+    }
   }
+  (void)ds_ws; (void)ds_ws_bytes;
   const int grid = cdiv(static_cast<long>(B) * s * nh, 8);
   attn_bwd_dq_k<T><<<grid, 256, 0, st>>>(qkv, O, dO, lse, dqkv, Dsc, B, s, nh, dh);
   note_launch();
@@ -1272,7 +1276,8 @@ void copy_f32(float* a, const float* b, size_t n, cudaStream_t st) { copy_k<<<gr
   template void norm_bwd<T>(const T*, const T*, const float*, const float*, const T*, T*, int, int, int, float*,      \
                             float*, float*, float*, size_t, cudaStream_t);                                           \
   template void attn_fwd<T>(const T*, T*, float*, int, int, int, int, cudaStream_t);                                 \
-  template void attn_bwd<T>(const T*, const T*, const T*, const float*, T*, float*, int, int, int, int, cudaStream_t); \
+  template void attn_bwd<T>(const T*, const T*, const T*, const float*, T*, float*, int, int, int, int, cudaStream_t, \
+                            void*, size_t);                                                                    \
   template void rope<T>(T*, int, int, int, int, float, int, cudaStream_t);                                           \
   template void swiglu_fwd<T>(const T*, T*, int, int, cudaStream_t);                                                 \
   template void swiglu_bwd<T>(const T*, const T*, T*, int, int, cudaStream_t);                                       \

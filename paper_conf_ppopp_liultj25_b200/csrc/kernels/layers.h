@@ -47,8 +47,13 @@ template <class T> void colsum(const T* a, const T* x, const float* stats, int r
 // Causal attention over QKV [T, 3h] (q | k | v), heads of dh; O [T, h]; lse [nh][T] fp32.
 template <class T> void attn_fwd(const T* qkv, T* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st);
 // dqkv [T, 3h] from dO; Dscratch [nh][T] fp32.
+// ds_ws (optional, >= flash_attn_bwd_ds_bytes): workspace for the dS image, which lets the bf16
+// tcgen05 path compute dQ from the stored dS (fa_bwd_dq_img) instead of recomputing S and dP.
 template <class T> void attn_bwd(const T* qkv, const T* O, const T* dO, const float* lse, T* dqkv, float* Dscratch,
-                                 int B, int s, int nh, int dh, cudaStream_t st);
+                                 int B, int s, int nh, int dh, cudaStream_t st, void* ds_ws = nullptr,
+                                 size_t ds_ws_bytes = 0);
+// bytes of that dS workspace for a shape (0 when the path does not apply)
+size_t flash_attn_bwd_ds_bytes(int dh, int B, int s, int nh);
 
 // RoPE (rotate-half) in place on the q and k parts of QKV; inverse = 1 rotates by -t*theta.
 template <class T> void rope(T* qkv, int B, int s, int nh, int dh, float base, int inverse, cudaStream_t st);
@@ -71,7 +76,8 @@ void loss_reduce(const float* row_loss, int rows, double* out, cudaStream_t st);
 bool flash_attn_supported(int dh);
 void flash_attn_fwd(const __nv_bfloat16* qkv, __nv_bfloat16* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st);
 void flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* O, const __nv_bfloat16* dO, const float* lse,
-                    __nv_bfloat16* dqkv, float* Dd, int B, int s, int nh, int dh, cudaStream_t st);
+                    __nv_bfloat16* dqkv, float* Dd, int B, int s, int nh, int dh, cudaStream_t st,
+                    void* ds_ws = nullptr, size_t ds_ws_bytes = 0);
 
 void cast_f32_bf16(const float* x, __nv_bfloat16* y, size_t n, cudaStream_t st);
 void add_f32(float* a, const float* b, size_t n, cudaStream_t st);       // a += b

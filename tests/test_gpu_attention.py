@@ -65,3 +65,43 @@ def test_attention_vs_sdpa(B, s, nh, dh, bf16, attn_variant):
                               scr.data_ptr(), B, s, nh, dh, bf16, None) == 0
     torch.cuda.synchronize()
     assert torch.equal(d2, dqkv)
+
+
+@pytest.mark.parametrize("B,s,nh,dh", [(2, 256, 3, 128), (1, 2048, 2, 128), (2, 384, 2, 64), (4, 2048, 16, 128)])
+def test_attention_bwd_ds_workspace(B, s, nh, dh):
+    """dQ from the stored dS (mario_k_attn_bwd_ws) vs SDPA, bitwise deterministic, and within bf16
+    rounding of the recomputing path (both are the c1 attention backward)."""
+    L = _lib.lib()
+    ws_bytes = L.mario_k_attn_bwd_ws_bytes(B, s, nh, dh)
+    nt = s // 128
+    assert ws_bytes == B * nh * nt * (nt + 1) * 16384
+    g = torch.Generator(device="cuda").manual_seed(7 * s + nh)
+    h = nh * dh
+    qkv = torch.randn(B * s, 3 * h, device="cuda", generator=g).bfloat16()
+    dO = torch.randn(B * s, h, device="cuda", generator=g).bfloat16()
+    O = torch.empty(B * s, h, device="cuda", dtype=torch.bfloat16)
+    lse = torch.empty(nh, B * s, device="cuda")
+    assert L.mario_k_attn_fwd(qkv.data_ptr(), O.data_ptr(), lse.data_ptr(), B, s, nh, dh, 1, None) == 0
+    scr = torch.empty(nh, B * s, device="cuda")
+    ws = torch.full((ws_bytes,), 0x7f, device="cuda", dtype=torch.uint8)   # garbage: must be fully overwritten
+    outs = []
+    for _ in range(2):
+        d = torch.empty(B * s, 3 * h, device="cuda", dtype=torch.bfloat16)
+        assert L.mario_k_attn_bwd_ws(qkv.data_ptr(), O.data_ptr(), dO.data_ptr(), lse.data_ptr(), d.data_ptr(),
+                                     scr.data_ptr(), ws.data_ptr(), ws_bytes, B, s, nh, dh, None) == 0
+        outs.append(d)
+    d_rc = torch.empty(B * s, 3 * h, device="cuda", dtype=torch.bfloat16)
+    assert L.mario_k_attn_bwd(qkv.data_ptr(), O.data_ptr(), dO.data_ptr(), lse.data_ptr(), d_rc.data_ptr(),
+                              scr.data_ptr(), B, s, nh, dh, 1, None) == 0
+    torch.cuda.synchronize()
+    assert torch.equal(outs[0], outs[1])
+    # dK, dV come from the same kernel either way
+    assert torch.equal(outs[0][:, h:], d_rc[:, h:])
+    if s <= 2048 and B * nh <= 4:
+        _, _, d_ref = _ref(qkv, B, s, nh, dh, dO)
+        for part in range(3):
+            a = outs[0].float()[:, part * h:(part + 1) * h]
+            r = d_ref[:, part * h:(part + 1) * h]
+            assert (a - r).abs().max().item() <= 2e-2 * r.abs().max().item(), part
+    dq, dq_rc = outs[0].float()[:, :h], d_rc.float()[:, :h]
+    assert (dq - dq_rc).abs().max().item() <= 1e-2 * dq_rc.abs().max().item()

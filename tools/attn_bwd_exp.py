@@ -43,3 +43,24 @@ for only in ("dkdv", "dq", ""):
         if not only and dbg:
             break
 os.environ.pop("MARIO_ATTN_DBG", None)
+# dQ from the stored dS image (mario_k_attn_bwd_ws)
+wsb = L.mario_k_attn_bwd_ws_bytes(B, s, nh, dh)
+ws = torch.empty(wsb, device="cuda", dtype=torch.uint8)
+f = lambda: L.mario_k_attn_bwd_ws(qkv.data_ptr(), O.data_ptr(), dO.data_ptr(), lse.data_ptr(), dq.data_ptr(),
+                                  scr.data_ptr(), ws.data_ptr(), wsb, B, s, nh, dh, None)
+for only in ("dkdv", ""):
+    if only:
+        os.environ["MARIO_ATTN_TC_ONLY"] = only
+    else:
+        os.environ.pop("MARIO_ATTN_TC_ONLY", None)
+    for _ in range(3):
+        f()
+    torch.cuda.synchronize()
+    e0.record()
+    for _ in range(10):
+        f()
+    e1.record()
+    torch.cuda.synchronize()
+    ms = e0.elapsed_time(e1) / 10
+    print(json.dumps({"kernel": (only or "both") + "+ds_image", "ws_MB": round(wsb / 1e6, 1), "us": round(ms * 1e3, 1),
+                      "alg_tflops_full_bwd": round(2 * fl / ms / 1e9, 1)}), flush=True)

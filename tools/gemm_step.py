@@ -11,9 +11,17 @@ sys.path.insert(0, ".")
 from paper_conf_ppopp_liultj25_b200 import _lib  # noqa: E402
 
 L = _lib.lib()
+import os  # noqa: E402
+if os.environ.get("STREAMK"):
+    L.mario_k_gemm_set_streamk(int(os.environ["STREAMK"]))
+if os.environ.get("VARIANT"):
+    L.mario_k_gemm_set_variant(int(os.environ["VARIANT"]))
 T, h, f = 8192, 2048, 8192
 bf = torch.bfloat16
 dev = "cuda"
+V = 50304
+Wh = torch.randn(V, h, device=dev).to(bf) * 0.02
+dWh = torch.zeros(V, h, device=dev)
 W = {"qkv": torch.randn(3 * h, h, device=dev).to(bf) * 0.02, "proj": torch.randn(h, h, device=dev).to(bf) * 0.02,
      "fc1": torch.randn(f, h, device=dev).to(bf) * 0.02, "fc2": torch.randn(h, f, device=dev).to(bf) * 0.02}
 bias = {k: torch.randn(v.shape[0], device=dev) * 0.02 for k, v in W.items()}
@@ -25,7 +33,8 @@ def act():
     r = lambda *s: torch.randn(*s, device=dev).to(bf)
     return {"A": r(T, h), "QKV": r(T, 3 * h), "O": r(T, h), "Hin": r(T, h), "H1": r(T, h), "A2": r(T, h),
             "Z": r(T, f), "G": r(T, f), "Hout": r(T, h), "dH": r(T, h), "dZ": r(T, f), "dA": r(T, h),
-            "dH1": r(T, h), "dO": r(T, h), "dQKV": r(T, 3 * h)}
+            "dH1": r(T, h), "dO": r(T, h), "dQKV": r(T, 3 * h),
+            "Hf": r(T, h), "logits": torch.empty(T, V, device=dev), "dlog": r(T, V)}
 
 
 sets = [act() for _ in range(NS)]
@@ -64,6 +73,10 @@ def calls(a, epi=True):
                                                       1. if e else 0.)),
         ("qkv dgrad", 2 * T * 3 * h * h, lambda: gemm(a["dQKV"], 3 * h, 0, W["qkv"], h, 1, T, h, 3 * h, a["dA"], h,
                                                       0, 0.)),
+        ("head fwd", 2 * T * V * h, lambda: gemm(a["Hf"], h, 0, Wh, h, 0, T, V, h, a["logits"], V, 1, 0.)),
+        ("head wgrad", 2 * T * V * h, lambda: gemm(a["dlog"], V, 1, a["Hf"], h, 1, V, h, T, dWh, h, 1,
+                                                   1. if e else 0.)),
+        ("head dgrad", 2 * T * V * h, lambda: gemm(a["dlog"], V, 0, Wh, h, 1, T, h, V, a["dA"], h, 0, 0.)),
     ]
 
 
