@@ -74,6 +74,11 @@ __device__ __forceinline__ void bulk_commit_wait_read() {
   asm volatile("cp.async.bulk.commit_group;" ::: "memory");
   asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");
 }
+// one 32-byte global store (sm_100: STG.256)
+__device__ __forceinline__ void st_global_v8(void* p, const uint32_t (&v)[8]) {
+  asm volatile("st.global.v8.b32 [%0], {%1, %2, %3, %4, %5, %6, %7, %8};" :: "l"(p), "r"(v[0]), "r"(v[1]), "r"(v[2]),
+               "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]) : "memory");
+}
 __device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;" ::: "memory"); }
 __device__ __forceinline__ void named_bar(int id, int n) { asm volatile("bar.sync %0, %1;" :: "r"(id), "r"(n) : "memory"); }
 
@@ -826,10 +831,19 @@ fa_bwd_dkdv_ts(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
         const size_t tri = static_cast<size_t>(s / kRows) * (s / kRows + 1);
         uint8_t* rowp = dsimg + ((static_cast<size_t>(bh) * tri + static_cast<size_t>(qb) * (qb + 1) + kt64) * 2 + (i & 1)) * 8192 +
                         r64 * 128;
+        // logical chunks 2p, 2p + 1 land on the aligned physical pair (4 half + 2p) ^ (r mod 8 & 6): one
+        // 32-byte store each (the lower half holds logical chunk 2p + (r & 1))
+        const bool sw = (r64 & 1) != 0;
 #pragma unroll
-        for (int jj = 0; jj < 4; ++jj)
-          *reinterpret_cast<uint4*>(rowp + (((4 * half + jj) ^ (r64 & 7)) << 4)) =
-              make_uint4(dk[4 * jj], dk[4 * jj + 1], dk[4 * jj + 2], dk[4 * jj + 3]);
+        for (int pp = 0; pp < 2; ++pp) {
+          uint32_t v[8];
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            v[e] = sw ? dk[8 * pp + 4 + e] : dk[8 * pp + e];
+            v[4 + e] = sw ? dk[8 * pp + e] : dk[8 * pp + 4 + e];
+          }
+          st_global_v8(rowp + (((4 * half + 2 * pp) ^ (r64 & 6)) << 4), v);
+        }
       }
       tmem_st_wait();
       tc_fence_before();
@@ -1150,7 +1164,10 @@ fa_bwd_dq_pers(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
 // Persistent (one CTA per SM) over items (query block, sample, head), heaviest first. Warps: 0 TMA,
 // 1 MMA (dQ double-buffered in TMEM), 2..5 epilogue (one query row per thread).
 constexpr int kThreadsI = 192;
-constexpr int kRingI = 6;
+#ifndef MARIO_DQI_RING
+#define MARIO_DQI_RING 3
+#endif
+constexpr int kRingI = MARIO_DQI_RING;   // 2 CTAs per SM (TMEM 2 x 256 columns)
 template <int DH>
 struct SmemI {
   static constexpr int kA = kRows * kCols * 2;       // 16 KB dS image tile
@@ -1354,7 +1371,9 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const int items = B * nh * (s / kRows);
-    fa_bwd_dq_img<DH><<<items < sms ? items : sms, kThreadsI, SmemI<DH>::kBytes, st>>>(m64, dsimg, dqkv, B, s, nh);
+    static const int per_sm = getenv("MARIO_DQI_CTAS") ? atoi(getenv("MARIO_DQI_CTAS")) : 2;
+    const int grid_i = items < per_sm * sms ? items : per_sm * sms;
+    fa_bwd_dq_img<DH><<<grid_i, kThreadsI, SmemI<DH>::kBytes, st>>>(m64, dsimg, dqkv, B, s, nh);
   } else if (!only || only[1] == 'q') {
     if (pers && dbg == 0) {
       static bool pset = false;
