@@ -157,7 +157,7 @@ struct Exec {
   // D[M,N] = A[M,K] . B[N,K]^T  (see kernels.h); bf16 tcgen05 or fp32 SIMT by dtype.
   void gemm(const T* A, int lda, int a_mn, const T* B, int ldb, int b_mn, int M, int N, int K, void* Dp, int ldd,
             bool out_f32, float beta, const float* bias = nullptr, const T* resid = nullptr, T* D2 = nullptr,
-            const T* aux = nullptr, bool d2_from_aux = false) {
+            const T* aux = nullptr, bool d2_from_aux = false, float* colsum_part = nullptr) {
     if constexpr (sizeof(T) == 2) {
       GemmArgs g;
       g.A = A; g.lda = lda; g.a_mn = a_mn; g.B = B; g.ldb = ldb; g.b_mn = b_mn; g.M = M; g.N = N; g.K = K;
@@ -166,6 +166,7 @@ struct Exec {
       g.ep.ldd = ldd; g.ep.beta = beta; g.ep.bias = bias;
       g.ep.residual = resid; g.ep.ld_res = ldd; g.ep.d2_bf16 = D2; g.ep.aux = aux; g.ep.ld_aux = ldd;
       g.ep.d2_from_aux = d2_from_aux ? 1 : 0;
+      g.ep.colsum_part = colsum_part;
       CU(gemm_bf16(g, st));
     } else {
       GemmF32Args g;
@@ -181,8 +182,10 @@ struct Exec {
     gemm(X, in, 0, W, in, 0, Tn, out, in, Y, out, false, 0.f, bias, resid, Y2);
   }
   // dX[T,in] = dY W (optionally * gelu'(aux); G = gelu(aux) as a second output when G != NULL)
-  void lin_dgrad(const T* dY, const T* W, int Tn, int out, int in, T* dX, const T* aux = nullptr, T* G = nullptr) {
-    gemm(dY, out, 0, W, in, 1, Tn, in, out, dX, in, false, 0.f, nullptr, nullptr, G, aux, G != nullptr);
+  // colsum_part (bf16 only): the epilogue also writes column partial sums of dX ([Tn/32][in] fp32)
+  void lin_dgrad(const T* dY, const T* W, int Tn, int out, int in, T* dX, const T* aux = nullptr, T* G = nullptr,
+                 float* colsum_part = nullptr) {
+    gemm(dY, out, 0, W, in, 1, Tn, in, out, dX, in, false, 0.f, nullptr, nullptr, G, aux, G != nullptr, colsum_part);
   }
   // dW[out,in] += dY^T X (fp32)
   void lin_wgrad(const T* dY, const T* X, int Tn, int out, int in, float* dW) {
@@ -353,13 +356,17 @@ struct Exec {
       T* dHin = (li == 0) ? (k == 0 ? dHbuf[(cur + 2) % 3] : dstage_in) : dHbuf[(cur + 2) % 3];
       if (gpt) {
         // dZ = (dH W2) * gelu'(Z); the epilogue also recomputes G = gelu(Z) for the fc2 wgrad
-        lin_dgrad(dH, Wm(D, p, pre + "fc2.w"), Tn, h, f, dZ, Z, Gt);
+        // fc1.b = column sums of dZ: fused into that epilogue (bf16), finished before `red` is reused
+        const bool fuse_b1 = sizeof(T) == 2 && Tn % 32 == 0 && f % 32 == 0 &&
+                             static_cast<size_t>(Tn / 32) * f <= red_floats;
+        lin_dgrad(dH, Wm(D, p, pre + "fc2.w"), Tn, h, f, dZ, Z, Gt, fuse_b1 ? red : nullptr);
+        if (fuse_b1) colsum_finish(red, Tn / 32, f, G(D, p, pre + "fc1.b"), st);
         lin_wgrad(dH, Gt, Tn, h, f, G(D, p, pre + "fc2.w"));
         // fc2.b: fused into the norm backward that wrote dH (this stage), else a column sum here
         if (li == lps - 1 && k != K - 1) colsum<T>(dH, nullptr, nullptr, Tn, h, h, 0, G(D, p, pre + "fc2.b"), nullptr, red, st);
         layernorm_fwd<T>(H1, Wf(D, p, pre + "ln2.g"), Wf(D, p, pre + "ln2.b"), A2, st2, Tn, h, m.norm_eps, st);
         lin_wgrad(dZ, A2, Tn, f, h, G(D, p, pre + "fc1.w"));
-        colsum<T>(dZ, nullptr, nullptr, Tn, f, f, 0, G(D, p, pre + "fc1.b"), nullptr, red, st);
+        if (!fuse_b1) colsum<T>(dZ, nullptr, nullptr, Tn, f, f, 0, G(D, p, pre + "fc1.b"), nullptr, red, st);
         lin_dgrad(dZ, Wm(D, p, pre + "fc1.w"), Tn, f, h, dA);               // dA2
         norm_bwd<T>(dA, H1, st2, Wf(D, p, pre + "ln2.g"), dH, dH1, Tn, h, 0, G(D, p, pre + "ln2.g"),
                     G(D, p, pre + "ln2.b"), G(D, p, pre + "proj.b"), red, red_floats, st);

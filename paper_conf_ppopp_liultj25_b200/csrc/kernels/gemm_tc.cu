@@ -328,6 +328,17 @@ __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool
     __syncwarp();
   } else {
     store_block_bf16(ep.d_bf16, ep.ldd, rbase, col0, M, lane, sw, v);
+    if (ep.colsum_part) {
+      // lane c: column col0 + c of the 32 bf16 rows just staged in sw, summed in row order
+      float cs = 0.f;
+#pragma unroll 8
+      for (int r = 0; r < 32; ++r) {
+        const uint8_t* p = sw64(sw, r, lane >> 3) + (lane & 7) * 2;
+        cs += __bfloat162float(*reinterpret_cast<const __nv_bfloat16*>(p));
+      }
+      ep.colsum_part[static_cast<size_t>(rbase >> 5) * N + col0 + lane] = cs;
+      __syncwarp();
+    }
     if (ep.d2_bf16) {
       const bool g_aux = ep.aux && ep.d2_from_aux;
 #pragma unroll
@@ -920,6 +931,14 @@ cudaError_t gemm_bf16(const GemmArgs& g0, cudaStream_t st) {
   if (g.M <= 0 || g.N <= 0 || g.K <= 0) return cudaSuccess;
   if ((g.lda % 8) || (g.ldb % 8)) {  // TMA: 16-byte row pitch
     fprintf(stderr, "[mario] gemm_bf16: lda=%d ldb=%d must be multiples of 8\n", g.lda, g.ldb);
+    return cudaErrorInvalidValue;
+  }
+  auto al16 = [](const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; };
+  if (g.ep.colsum_part &&
+      (g.ep.out_f32 || (g.M % 32) || (g.N % 32) || !g.ep.d_bf16 || (g.ep.ldd % 8) || !al16(g.ep.d_bf16) ||
+       (g.ep.d2_bf16 && !al16(g.ep.d2_bf16)) || (g.ep.residual && ((g.ep.ld_res % 8) || !al16(g.ep.residual))) ||
+       (g.ep.aux && ((g.ep.ld_aux % 8) || !al16(g.ep.aux))) || (g.ep.bias && !al16(g.ep.bias)))) {
+    fprintf(stderr, "[mario] gemm_bf16: fused column sums need bf16 output, M %% 32 == N %% 32 == 0, aligned D\n");
     return cudaErrorInvalidValue;
   }
   const int sms = device_sm_count();

@@ -20,6 +20,10 @@ struct GemmEpilogue {
   const __nv_bfloat16* residual = nullptr; int ld_res = 0;   // D += residual
   const __nv_bfloat16* aux = nullptr; int ld_aux = 0;        // D = acc * gelu'(aux)  (GeLU bwd)
   int d2_from_aux = 0;                    // with aux: D2 = gelu(aux) (recomputed MLP activation)
+  // optional fused column sums of the bf16 output D (a bias gradient): colsum_part[M/32][N] fp32,
+  // row block i = sum over rows [32 i, 32 i + 32) in row order. Requires bf16 output, M % 32 == 0,
+  // N % 32 == 0 and 16-byte aligned pitches (gemm_bf16 returns cudaErrorInvalidValue otherwise).
+  float* colsum_part = nullptr;
 };
 
 struct GemmArgs {

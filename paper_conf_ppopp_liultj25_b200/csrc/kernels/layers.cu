@@ -1121,6 +1121,12 @@ void norm_bwd_dx(const T* dy, const T* x, const float* stats, const float* g, co
   norm_bwd_dx_k<T><<<cdiv(rows, 8), 256, 0, st>>>(dy, x, stats, g, dres, dx, rows, n, rms);
   note_launch();
 }
+void colsum_finish(const float* partial, int nblk, int n, float* out, cudaStream_t st) {
+  KScope ks_(K_COLSUM, st);
+  colsum_final_k<<<cdiv(n, 256), 256, 0, st>>>(partial, nblk, n, 0, out, nullptr);
+  note_launch();
+}
+
 template <class T>
 void colsum(const T* a, const T* x, const float* stats, int rows, int n, int lda, int mode, float* out0, float* out1,
             float* partial, cudaStream_t st) {

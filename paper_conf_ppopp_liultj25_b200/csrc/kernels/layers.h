@@ -41,6 +41,9 @@ bool softmax_ce_fast(const float* logits, const int32_t* tok, int ld_tok, int s,
                      __nv_bfloat16* dlogits, float* row_loss, cudaStream_t st);
 // Column reductions into fp32 grads (+=): mode 0: out0 += sum_r a[r,c]
 // mode 1 (LN): out0 += sum dy*xhat, out1 += sum dy; mode 2 (RMS): out0 += sum dy*xhat.
+// out[c] += sum_b partial[b][c] over nblk row blocks (fixed order): the second pass of column sums
+// whose partials a GEMM epilogue produced (GemmEpilogue::colsum_part)
+void colsum_finish(const float* partial, int nblk, int n, float* out, cudaStream_t st);
 template <class T> void colsum(const T* a, const T* x, const float* stats, int rows, int n, int lda, int mode,
                                float* out0, float* out1, float* partial, cudaStream_t st);
 
