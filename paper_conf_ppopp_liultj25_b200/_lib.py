@@ -7,7 +7,7 @@ import ctypes as C
 import os
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libmario.so")
+LIB_PATH = os.environ.get("MARIO_LIB") or os.path.join(_PKG, "libmario.so")
 
 _lib = None
 

@@ -364,7 +364,7 @@ struct Exec {
         lin_wgrad(dH, Gt, Tn, h, f, G(D, p, pre + "fc2.w"));
         // fc2.b: fused into the norm backward that wrote dH (this stage), else a column sum here
         if (li == lps - 1 && k != K - 1) colsum<T>(dH, nullptr, nullptr, Tn, h, h, 0, G(D, p, pre + "fc2.b"), nullptr, red, st);
-        layernorm_fwd<T>(H1, Wf(D, p, pre + "ln2.g"), Wf(D, p, pre + "ln2.b"), A2, st2, Tn, h, m.norm_eps, st);
+        norm_recompute<T>(H1, Wf(D, p, pre + "ln2.g"), Wf(D, p, pre + "ln2.b"), A2, st2, Tn, h, m.norm_eps, 0, st);
         lin_wgrad(dZ, A2, Tn, f, h, G(D, p, pre + "fc1.w"));
         if (!fuse_b1) colsum<T>(dZ, nullptr, nullptr, Tn, f, f, 0, G(D, p, pre + "fc1.b"), nullptr, red, st);
         lin_dgrad(dZ, Wm(D, p, pre + "fc1.w"), Tn, f, h, dA);               // dA2
@@ -377,7 +377,7 @@ struct Exec {
         lin_wgrad(dH, Gt, Tn, h, f, G(D, p, pre + "down.w"));
         lin_dgrad(dH, Wm(D, p, pre + "down.w"), Tn, h, f, dM);              // overwrites M (consumed)
         swiglu_bwd<T>(Z, dM, dZ, Tn, f, st);
-        rmsnorm_fwd<T>(H1, Wf(D, p, pre + "n2.g"), A2, st2, Tn, h, m.norm_eps, st);
+        norm_recompute<T>(H1, Wf(D, p, pre + "n2.g"), nullptr, A2, st2, Tn, h, m.norm_eps, 1, st);
         lin_wgrad(dZ, A2, Tn, 2 * f, h, G(D, p, pre + "gu.w"));
         lin_dgrad(dZ, Wm(D, p, pre + "gu.w"), Tn, 2 * f, h, dA);
         norm_bwd<T>(dA, H1, st2, Wf(D, p, pre + "n2.g"), dH, dH1, Tn, h, 1, G(D, p, pre + "n2.g"), nullptr, nullptr,
@@ -387,8 +387,8 @@ struct Exec {
       }
       attn_bwd<T>(QKV, O, dO, LSE, dQKV, Dsc, mbs, s, nh, dh, st, BS.dS_bytes ? sc + BS.dS : nullptr, BS.dS_bytes);
       if (!gpt) rope<T>(dQKV, mbs, s, nh, dh, m.rope_base, 1, st);
-      if (gpt) layernorm_fwd<T>(Hin, Wf(D, p, pre + "ln1.g"), Wf(D, p, pre + "ln1.b"), A, st1, Tn, h, m.norm_eps, st);
-      else rmsnorm_fwd<T>(Hin, Wf(D, p, pre + "n1.g"), A, st1, Tn, h, m.norm_eps, st);
+      if (gpt) norm_recompute<T>(Hin, Wf(D, p, pre + "ln1.g"), Wf(D, p, pre + "ln1.b"), A, st1, Tn, h, m.norm_eps, 0, st);
+      else norm_recompute<T>(Hin, Wf(D, p, pre + "n1.g"), nullptr, A, st1, Tn, h, m.norm_eps, 1, st);
       lin_wgrad(dQKV, A, Tn, 3 * h, h, G(D, p, pre + "qkv.w"));
       if (gpt) colsum<T>(dQKV, nullptr, nullptr, Tn, 3 * h, 3 * h, 0, G(D, p, pre + "qkv.b"), nullptr, red, st);
       lin_dgrad(dQKV, Wm(D, p, pre + "qkv.w"), Tn, 3 * h, h, dA);

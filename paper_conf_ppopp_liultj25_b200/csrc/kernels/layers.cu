@@ -1065,6 +1065,19 @@ void embed_bwd(const int32_t* tok, int ld_tok, int B, int s, const T* dH, int h,
   if (dwpe) { embed_pos_bwd_k<T><<<grid_for(static_cast<long>(s) * h), 256, 0, st>>>(dH, B, s, h, dwpe); note_launch(); }
 }
 
+bool norm_apply(const __nv_bfloat16* x, const float* g, const float* b, const float* stats, __nv_bfloat16* y, int rows,
+                int n, cudaStream_t st);   // rowpipe.cu
+template <class T>
+void norm_recompute(const T* x, const float* g, const float* b, T* y, float* stats, int rows, int n, float eps, int rms,
+                    cudaStream_t st) {
+  if constexpr (std::is_same<T, __nv_bfloat16>::value) {
+    KScope ks_(K_NORM, st);
+    if (norm_apply(x, g, rms ? nullptr : b, stats, y, rows, n, st)) return;
+  }
+  if (rms) rmsnorm_fwd<T>(x, g, y, stats, rows, n, eps, st);
+  else layernorm_fwd<T>(x, g, b, y, stats, rows, n, eps, st);
+}
+
 template <class T>
 void layernorm_fwd(const T* x, const float* g, const float* b, T* y, float* stats, int rows, int n, float eps, cudaStream_t st) {
   KScope ks_(K_NORM, st);
@@ -1278,6 +1291,8 @@ void copy_f32(float* a, const float* b, size_t n, cudaStream_t st) { copy_k<<<gr
   template void rmsnorm_fwd<T>(const T*, const float*, T*, float*, int, int, float, cudaStream_t);                   \
   template void norm_bwd_dx<T>(const T*, const T*, const float*, const float*, const T*, T*, int, int, int,          \
                                cudaStream_t);                                                                      \
+  template void norm_recompute<T>(const T*, const float*, const float*, T*, float*, int, int, float, int,          \
+                                  cudaStream_t);                                                                 \
   template void colsum<T>(const T*, const T*, const float*, int, int, int, int, float*, float*, float*, cudaStream_t); \
   template void norm_bwd<T>(const T*, const T*, const float*, const float*, const T*, T*, int, int, int, float*,      \
                             float*, float*, float*, size_t, cudaStream_t);                                           \

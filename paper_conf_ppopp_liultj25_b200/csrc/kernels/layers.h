@@ -20,6 +20,10 @@ template <class T> void layernorm_fwd(const T* x, const float* g, const float* b
                                       int n, float eps, cudaStream_t st);
 template <class T> void rmsnorm_fwd(const T* x, const float* g, T* y, float* stats, int rows, int n, float eps,
                                     cudaStream_t st);
+// y = norm(x) from stats the forward stored (b = NULL for RMSNorm): the backward's recompute of a
+// norm output with the forward kernel's expression. Falls back to the full forward for fp32 / odd n.
+template <class T> void norm_recompute(const T* x, const float* g, const float* b, T* y, float* stats, int rows,
+                                       int n, float eps, int rms, cudaStream_t st);
 // dx = LN'(dy) (+ dres); rms = 1 selects RMSNorm.
 template <class T> void norm_bwd_dx(const T* dy, const T* x, const float* stats, const float* g, const T* dres,
                                     T* dx, int rows, int n, int rms, cudaStream_t st);

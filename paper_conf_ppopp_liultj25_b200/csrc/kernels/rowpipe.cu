@@ -461,6 +461,53 @@ inline int threads_for(int n) { return ((n / 8 + 31) / 32) * 32; }
 inline int cdivl(long a, long b) { return static_cast<int>((a + b - 1) / b); }
 }  // namespace
 
+// Backward recompute of a norm output from the forward's stored row statistics (the lean activation
+// set keeps x and (mean, rstd), not y): y = (x - mean) * rstd * g + b, the forward kernel's exact
+// expression, as one streaming pass without row reductions. Thread i owns 16-byte vectors i and
+// i + nthreads (both loads issued before any math).
+__global__ void __launch_bounds__(256) norm_apply_k(const bf16* __restrict__ x, const float* __restrict__ g,
+                                                    const float* __restrict__ b, const float* __restrict__ stats,
+                                                    bf16* __restrict__ y, long nvec, int nv_row) {
+  const long stride = static_cast<long>(gridDim.x) * blockDim.x;
+  const long i0 = static_cast<long>(blockIdx.x) * blockDim.x + threadIdx.x;
+  uint4 u[2];
+#pragma unroll
+  for (int k = 0; k < 2; ++k) {
+    const long i = i0 + k * stride;
+    if (i < nvec) u[k] = __ldg(reinterpret_cast<const uint4*>(x) + i);
+  }
+#pragma unroll
+  for (int k = 0; k < 2; ++k) {
+    const long i = i0 + k * stride;
+    if (i >= nvec) break;
+    const long r = i / nv_row;
+    const int c = static_cast<int>(i - r * nv_row) * 8;
+    const float2 ms = __ldg(reinterpret_cast<const float2*>(stats) + r);
+    float v[8], gg[8], bb[8], o[8];
+    unpack8(u[k], v);
+    load8(g + c, gg);
+    if (b) load8(b + c, bb);
+    else {
+#pragma unroll
+      for (int j = 0; j < 8; ++j) bb[j] = 0.f;
+    }
+#pragma unroll
+    for (int j = 0; j < 8; ++j) o[j] = (v[j] - ms.x) * ms.y * gg[j] + bb[j];
+    reinterpret_cast<uint4*>(y)[i] = pack8(o);
+  }
+}
+
+bool norm_apply(const bf16* x, const float* g, const float* b, const float* stats, bf16* y, int rows, int n,
+                cudaStream_t st) {
+  if (n % 8 != 0 || (reinterpret_cast<uintptr_t>(x) & 15) || (reinterpret_cast<uintptr_t>(y) & 15)) return false;
+  const long nvec = static_cast<long>(rows) * (n / 8);
+  if (nvec <= 0) return true;
+  const long thr = (nvec + 1) / 2;
+  norm_apply_k<<<cdivl(thr, 256), 256, 0, st>>>(x, g, b, stats, y, nvec, n / 8);
+  note_launch();
+  return true;
+}
+
 bool norm_pipe_supported(int n) { return n % 8 == 0 && n >= 8 && n <= 8192; }
 
 bool norm_fwd_pipe(const bf16* x, const float* g, const float* b, bf16* y, float* stats, int rows, int n, float eps,
