@@ -193,6 +193,9 @@ __device__ __forceinline__ uint8_t* sw128(uint8_t* sw, int r, int j) { return sw
 // right after the previous block's copy was moved to shared memory, and for a tile's first block
 // before the accumulator wait -- so the global latency overlaps work instead of stalling each
 // block. 4 lanes per 64-byte row segment (coalesced). fp32 += (wgrad) reads stay in-block.
+#ifndef MARIO_EPI_PREFETCH
+#define MARIO_EPI_PREFETCH 1   // 0: each block loads its own input when it starts (A/B experiments)
+#endif
 struct EpiPrefetch { uint4 v[4]; };
 __device__ __forceinline__ void epi_prefetch(const GemmEpilogue& ep, bool vec_ok, int rbase, int lane, int col0, int M,
                                              int N, EpiPrefetch& pf) {
@@ -262,9 +265,10 @@ __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool
   if (col0 >= N) return;
   if (!vec_ok || col0 + 32 > N) {   // warp-uniform: ragged column block or unaligned pitches
     epilogue_chunk(ep, r, rbase + lane, col0, rbase + lane < M, N);
-    epi_prefetch(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
+    if (MARIO_EPI_PREFETCH) epi_prefetch(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
     return;
   }
+  if (!MARIO_EPI_PREFETCH) epi_prefetch(ep, vec_ok, rbase, lane, col0, M, N, pf);
   float v[32];
 #pragma unroll
   for (int j = 0; j < 32; ++j) v[j] = __uint_as_float(r[j]);
@@ -278,7 +282,7 @@ __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool
   float z[32];
   if (ep.aux) {   // GeLU backward: D = acc * gelu'(Z)
     load_block_bf16(pf.v, lane, sw, z);
-    epi_prefetch(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
+    if (MARIO_EPI_PREFETCH) epi_prefetch(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
 #pragma unroll
     for (int j = 0; j < 32; ++j) v[j] *= gelu_tanh_grad_f(z[j]);
   }
@@ -290,7 +294,7 @@ __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool
       load_block_bf16(rv, lane, sw, rr);
     } else {
       load_block_bf16(pf.v, lane, sw, rr);
-      epi_prefetch(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
+      if (MARIO_EPI_PREFETCH) epi_prefetch(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
     }
 #pragma unroll
     for (int j = 0; j < 32; ++j) v[j] += rr[j];
@@ -456,7 +460,7 @@ gemm_bf16_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
       const int m0 = tm * BM, n0 = tn * BN;
       const int rbase = m0 + quarter * 32;
       EpiPrefetch pf;
-      epi_prefetch(ep, vec_ok, rbase, lane, n0, M, N, pf);
+      if (MARIO_EPI_PREFETCH) epi_prefetch(ep, vec_ok, rbase, lane, n0, M, N, pf);
       mbar_wait(&tfull[acc], acc_ph);
       tc_fence_after();
 #pragma unroll 1
@@ -665,7 +669,7 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
       const int m0 = tm * 256 + 128 * rank, n0 = tn * BNP;
       const int rbase = m0 + quarter * 32;
       EpiPrefetch pf;
-      if (!(skon && u.kb0 != 0)) epi_prefetch(ep, vec_ok, rbase, lane, n0 + half * (BNP / 2), M, N, pf);
+      if (MARIO_EPI_PREFETCH && !(skon && u.kb0 != 0)) epi_prefetch(ep, vec_ok, rbase, lane, n0 + half * (BNP / 2), M, N, pf);
       if (sk.sleep_ns) { while (!mbar_test(&tfull[acc], acc_ph)) __nanosleep(sk.sleep_ns); }
       else mbar_wait(&tfull[acc], acc_ph);
       tc_fence_after();
