@@ -28,6 +28,7 @@ extern "C" int mario_k_gemm_bf16(const void* A, int lda, int a_mn, const void* B
   g.ep.residual = static_cast<const __nv_bfloat16*>(residual); g.ep.ld_res = ld_res;
   g.ep.d2_bf16 = static_cast<__nv_bfloat16*>(D2);
   g.ep.aux = static_cast<const __nv_bfloat16*>(aux); g.ep.ld_aux = ld_aux;
+  g.ep.d2_from_aux = (D2 && aux) ? 1 : 0;
   return static_cast<int>(gemm_bf16(g, static_cast<cudaStream_t>(stream)));
 }
 

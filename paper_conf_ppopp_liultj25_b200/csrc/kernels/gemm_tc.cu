@@ -551,7 +551,9 @@ __device__ __forceinline__ void st_release(int* p, int v) {
   asm volatile("st.release.gpu.global.b32 [%0], %1;" :: "l"(p), "r"(v) : "memory");
 }
 
-template <int BNP, bool A_MN, bool B_MN>
+// SK: stream-K compiled in (off by default: it measured slower, and its state and code raise the
+// epilogue warps' register pressure into spills on the hot path)
+template <int BNP, bool A_MN, bool B_MN, bool SK>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads2, 1)
 gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                      GemmEpilogue ep, int M, int N, int K, int n_fastest, StreamK sk) {
@@ -572,7 +574,7 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
   const int num_m = (M + 255) / 256, num_n = (N + BNP - 1) / BNP;
   const int num_tiles = num_m * num_n;
   const int nk = (K + BK - 1) / BK;
-  const bool skon = sk.on != 0;
+  const bool skon = SK && sk.on != 0;
   const int dp_tiles = skon ? (num_tiles / npairs) * npairs : num_tiles;
   const long long I0 = static_cast<long long>(dp_tiles) * nk, Isk = static_cast<long long>(num_tiles - dp_tiles) * nk;
 
@@ -670,7 +672,7 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
       const int rbase = m0 + quarter * 32;
       EpiPrefetch pf;
       if (MARIO_EPI_PREFETCH && !(skon && u.kb0 != 0)) epi_prefetch(ep, vec_ok, rbase, lane, n0 + half * (BNP / 2), M, N, pf);
-      if (sk.sleep_ns) { while (!mbar_test(&tfull[acc], acc_ph)) __nanosleep(sk.sleep_ns); }
+      if (SK && sk.sleep_ns) { while (!mbar_test(&tfull[acc], acc_ph)) __nanosleep(sk.sleep_ns); }
       else mbar_wait(&tfull[acc], acc_ph);
       tc_fence_after();
       const int lrow = quarter * 32 + lane;                     // accumulator row within this CTA
@@ -858,10 +860,13 @@ cudaError_t launch_pair(const GemmArgs& g, cudaStream_t st, int num_sms) {
     fprintf(stderr, "[mario] gemm_bf16 (pair): tensor map failed M=%d N=%d K=%d\n", g.M, g.N, g.K);
     return cudaErrorInvalidValue;
   }
-  auto kern = gemm_bf16_tc2_kernel<BNP, A_MN, B_MN>;
   static bool attr_set = false;
   if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, C2::kSmem);
+    cudaError_t e = cudaFuncSetAttribute(gemm_bf16_tc2_kernel<BNP, A_MN, B_MN, false>,
+                                         cudaFuncAttributeMaxDynamicSharedMemorySize, C2::kSmem);
+    if (e == cudaSuccess)
+      e = cudaFuncSetAttribute(gemm_bf16_tc2_kernel<BNP, A_MN, B_MN, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                               C2::kSmem);
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
@@ -881,7 +886,12 @@ cudaError_t launch_pair(const GemmArgs& g, cudaStream_t st, int num_sms) {
   const int tok = kstats_begin(K_GEMM, 2.0 * g.M * g.N * g.K,
                                2.0 * (double(g.M) * g.K + double(g.N) * g.K) + (g.ep.out_f32 ? 4.0 : 2.0) * g.M * g.N, st);
   const int n_fastest = raster_for(g);
-  kern<<<2 * pairs, kThreads2, C2::kSmem, st>>>(ta, tb, g.ep, g.M, g.N, g.K, n_fastest, sk);
+  if (sk.on || sk.sleep_ns)
+    gemm_bf16_tc2_kernel<BNP, A_MN, B_MN, true><<<2 * pairs, kThreads2, C2::kSmem, st>>>(ta, tb, g.ep, g.M, g.N, g.K,
+                                                                                       n_fastest, sk);
+  else
+    gemm_bf16_tc2_kernel<BNP, A_MN, B_MN, false><<<2 * pairs, kThreads2, C2::kSmem, st>>>(ta, tb, g.ep, g.M, g.N, g.K,
+                                                                                        n_fastest, sk);
   kstats_end(tok, st);
   note_launch();
   return cudaGetLastError();

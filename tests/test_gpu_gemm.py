@@ -49,7 +49,7 @@ def _run(a_mn, b_mn, M, N, K, out_f32, bias=False, resid=False, gelu2=False, aux
     tol = 2e-3 if out_f32 else 1e-2
     assert (D.float() - ref).abs().max().item() <= tol * scale
     if gelu2:
-        gref = torch.nn.functional.gelu(D.float(), approximate="tanh")
+        gref = torch.nn.functional.gelu((z if aux else D).float(), approximate="tanh")
         assert (D2.float() - gref).abs().max().item() <= 2e-2 * gref.abs().max().item() + 1e-2
 
 
@@ -76,6 +76,7 @@ def test_gemm_bf16_epilogues(variant):
     _run(0, 0, 384, 640, 256, out_f32=False, bias=True, resid=True)
     _run(0, 0, 384, 640, 256, out_f32=False, bias=True, gelu2=True)
     _run(0, 1, 384, 640, 256, out_f32=False, aux=True)
+    _run(0, 1, 384, 640, 256, out_f32=False, aux=True, gelu2=True)     # D2 = gelu(aux): fc2 dgrad
 
 
 def test_gemm_bf16_deterministic():

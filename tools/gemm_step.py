@@ -62,7 +62,7 @@ def calls(a, epi=True):
         ("fc2 wgrad", 2 * T * h * f, lambda: gemm(a["dH"], h, 1, a["G"], f, 1, h, f, T, dW["fc2"], f, 1,
                                                   1. if e else 0.)),
         ("fc2 dgrad", 2 * T * h * f, lambda: gemm(a["dH"], h, 0, W["fc2"], f, 1, T, f, h, a["dZ"], f, 0, 0.,
-                                                  aux=a["Z"] if e else None)),
+                                                  d2=a["G"] if e else None, aux=a["Z"] if e else None)),
         ("fc1 wgrad", 2 * T * h * f, lambda: gemm(a["dZ"], f, 1, a["A2"], h, 1, f, h, T, dW["fc1"], h, 1,
                                                   1. if e else 0.)),
         ("fc1 dgrad", 2 * T * h * f, lambda: gemm(a["dZ"], f, 0, W["fc1"], h, 1, T, h, f, a["dA"], h, 0, 0.)),
