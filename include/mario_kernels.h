@@ -26,7 +26,8 @@ extern "C" {
  *   out_f32 = 1: D (fp32) = v + beta * D      (wgrad accumulation, beta in {0,1})
  *   out_f32 = 0: D (bf16) = v, and D2 (bf16, same pitch) = gelu_tanh(v) if D2 != NULL -- or, when
  *   aux != NULL too, D2 = gelu_tanh(aux) (the backward's recompute of the MLP activation G = gelu(Z)
- *   fused into the fc2 dgrad that reads Z anyway). */
+ *   fused into the fc2 dgrad that reads Z anyway). aux requires out_f32 = 0 and residual = NULL
+ *   (cudaErrorInvalidValue otherwise). */
 int mario_k_gemm_bf16(const void* A, int lda, int a_mn, const void* B, int ldb, int b_mn,
                       int M, int N, int K, void* D, int ldd, int out_f32, float beta,
                       const float* bias, const void* residual, int ld_res,

@@ -65,6 +65,7 @@ __device__ __forceinline__ float gelu_tanh_grad_f(float z) {
 }
 
 // Fused epilogue for 32 consecutive accumulator columns of one output row (fp32 in r[]).
+template <bool F32>
 __device__ __forceinline__ void epilogue_chunk(const GemmEpilogue& ep, const uint32_t (&r)[32], int row, int col0,
                                                bool row_ok, int N) {
   if (!row_ok || col0 >= N) return;
@@ -102,7 +103,7 @@ __device__ __forceinline__ void epilogue_chunk(const GemmEpilogue& ep, const uin
       for (int j = 0; j < 32; ++j) if (col0 + j < N) v[j] += __bfloat162float(rr[j]);
     }
   }
-  if (ep.out_f32) {
+  if constexpr (F32) {
     float* d = ep.d_f32 + static_cast<size_t>(row) * ep.ldd + col0;
     if (full_cols) {
 #pragma unroll
@@ -259,12 +260,15 @@ __device__ __forceinline__ void store_block_bf16(__nv_bfloat16* base, int ld, in
   __syncwarp();
 }
 
+// EPI (compile-time split so each path's registers stay apart: the bf16 paths spilled otherwise):
+// 0 = bf16 output without GeLU' aux, 1 = bf16 output with aux (fc2 dgrad), 2 = fp32 output (wgrad, logits)
+template <int EPI>
 __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool vec_ok, const uint32_t (&r)[32],
                                                     int rbase, int lane, int col0, int M, int N, uint8_t* sw,
                                                     EpiPrefetch& pf, int next_col0) {
   if (col0 >= N) return;
   if (!vec_ok || col0 + 32 > N) {   // warp-uniform: ragged column block or unaligned pitches
-    epilogue_chunk(ep, r, rbase + lane, col0, rbase + lane < M, N);
+    epilogue_chunk<EPI == 2>(ep, r, rbase + lane, col0, rbase + lane < M, N);
     if (MARIO_EPI_PREFETCH) epi_prefetch(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
     return;
   }
@@ -280,26 +284,22 @@ __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool
     }
   }
   float z[32];
-  if (ep.aux) {   // GeLU backward: D = acc * gelu'(Z)
+  if constexpr (EPI == 1) {   // GeLU backward: D = acc * gelu'(Z)
     load_block_bf16(pf.v, lane, sw, z);
     if (MARIO_EPI_PREFETCH) epi_prefetch(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
 #pragma unroll
     for (int j = 0; j < 32; ++j) v[j] *= gelu_tanh_grad_f(z[j]);
   }
-  if (ep.residual) {
-    float rr[32];
-    if (ep.aux) {   // never both in the executor; the prefetch slot holds aux then
-      uint4 rv[4];
-      epi_rows_bf16(ep.residual, ep.ld_res, rbase, col0, M, lane, rv);
-      load_block_bf16(rv, lane, sw, rr);
-    } else {
+  if constexpr (EPI != 1) {   // residual: not on the aux path (gemm_bf16 rejects aux + residual)
+    if (ep.residual) {
+      float rr[32];
       load_block_bf16(pf.v, lane, sw, rr);
       if (MARIO_EPI_PREFETCH) epi_prefetch(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
-    }
 #pragma unroll
-    for (int j = 0; j < 32; ++j) v[j] += rr[j];
+      for (int j = 0; j < 32; ++j) v[j] += rr[j];
+    }
   }
-  if (ep.out_f32) {
+  if constexpr (EPI == 2) {
     // issue the coalesced reads of the old D first so their latency overlaps the transposition
     float4 old[8];
     if (ep.beta != 0.f) {
@@ -344,7 +344,7 @@ __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool
       __syncwarp();
     }
     if (ep.d2_bf16) {
-      const bool g_aux = ep.aux && ep.d2_from_aux;
+      const bool g_aux = EPI == 1 && ep.d2_from_aux;
 #pragma unroll
       for (int j = 0; j < 32; ++j) v[j] = gelu_tanh_f(g_aux ? z[j] : v[j]);
       store_block_bf16(ep.d2_bf16, ep.ldd, rbase, col0, M, lane, sw, v);
@@ -468,7 +468,10 @@ gemm_bf16_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
         uint32_t r[32];
         tmem_ld_32x32b_x32(tmem_base + acc * BN + c * 32 + (static_cast<uint32_t>(quarter * 32) << 16), r);
         tmem_ld_wait();
-        epilogue_chunk_warp(ep, vec_ok, r, rbase, lane, n0 + c * 32, M, N, sw, pf, c + 1 < BN / 32 ? n0 + (c + 1) * 32 : -1);
+        const int nxt = c + 1 < BN / 32 ? n0 + (c + 1) * 32 : -1;
+        if (ep.out_f32) epilogue_chunk_warp<2>(ep, vec_ok, r, rbase, lane, n0 + c * 32, M, N, sw, pf, nxt);
+        else if (ep.aux) epilogue_chunk_warp<1>(ep, vec_ok, r, rbase, lane, n0 + c * 32, M, N, sw, pf, nxt);
+        else epilogue_chunk_warp<0>(ep, vec_ok, r, rbase, lane, n0 + c * 32, M, N, sw, pf, nxt);
       }
       tc_fence_before();
       mbar_arrive(&tempty[acc]);
@@ -553,7 +556,7 @@ __device__ __forceinline__ void st_release(int* p, int v) {
 
 // SK: stream-K compiled in (off by default: it measured slower, and its state and code raise the
 // epilogue warps' register pressure into spills on the hot path)
-template <int BNP, bool A_MN, bool B_MN, bool SK>
+template <int BNP, bool A_MN, bool B_MN, bool SK, int EPI>
 __global__ void __cluster_dims__(2, 1, 1) __launch_bounds__(kThreads2, 1)
 gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                      GemmEpilogue ep, int M, int N, int K, int n_fastest, StreamK sk) {
@@ -722,7 +725,7 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
               r[4 * e + 3] = __float_as_uint(__uint_as_float(r[4 * e + 3]) + pv.w);
             }
           }
-          epilogue_chunk_warp(ep, vec_ok, r, rbase, lane, n0 + col, M, N, sw, pf,
+          epilogue_chunk_warp<EPI>(ep, vec_ok, r, rbase, lane, n0 + col, M, N, sw, pf,
                               c + 1 < BNP / 64 ? n0 + col + 32 : -1);
         }
         if (q1 > pair + 1) {
@@ -862,11 +865,15 @@ cudaError_t launch_pair(const GemmArgs& g, cudaStream_t st, int num_sms) {
   }
   static bool attr_set = false;
   if (!attr_set) {
-    cudaError_t e = cudaFuncSetAttribute(gemm_bf16_tc2_kernel<BNP, A_MN, B_MN, false>,
-                                         cudaFuncAttributeMaxDynamicSharedMemorySize, C2::kSmem);
-    if (e == cudaSuccess)
-      e = cudaFuncSetAttribute(gemm_bf16_tc2_kernel<BNP, A_MN, B_MN, true>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                               C2::kSmem);
+    const void* ks[6] = {reinterpret_cast<const void*>(gemm_bf16_tc2_kernel<BNP, A_MN, B_MN, false, 0>),
+                         reinterpret_cast<const void*>(gemm_bf16_tc2_kernel<BNP, A_MN, B_MN, false, 1>),
+                         reinterpret_cast<const void*>(gemm_bf16_tc2_kernel<BNP, A_MN, B_MN, false, 2>),
+                         reinterpret_cast<const void*>(gemm_bf16_tc2_kernel<BNP, A_MN, B_MN, true, 0>),
+                         reinterpret_cast<const void*>(gemm_bf16_tc2_kernel<BNP, A_MN, B_MN, true, 1>),
+                         reinterpret_cast<const void*>(gemm_bf16_tc2_kernel<BNP, A_MN, B_MN, true, 2>)};
+    cudaError_t e = cudaSuccess;
+    for (int i = 0; i < 6 && e == cudaSuccess; ++i)
+      e = cudaFuncSetAttribute(ks[i], cudaFuncAttributeMaxDynamicSharedMemorySize, C2::kSmem);
     if (e != cudaSuccess) return e;
     attr_set = true;
   }
@@ -886,12 +893,17 @@ cudaError_t launch_pair(const GemmArgs& g, cudaStream_t st, int num_sms) {
   const int tok = kstats_begin(K_GEMM, 2.0 * g.M * g.N * g.K,
                                2.0 * (double(g.M) * g.K + double(g.N) * g.K) + (g.ep.out_f32 ? 4.0 : 2.0) * g.M * g.N, st);
   const int n_fastest = raster_for(g);
-  if (sk.on || sk.sleep_ns)
-    gemm_bf16_tc2_kernel<BNP, A_MN, B_MN, true><<<2 * pairs, kThreads2, C2::kSmem, st>>>(ta, tb, g.ep, g.M, g.N, g.K,
-                                                                                       n_fastest, sk);
-  else
-    gemm_bf16_tc2_kernel<BNP, A_MN, B_MN, false><<<2 * pairs, kThreads2, C2::kSmem, st>>>(ta, tb, g.ep, g.M, g.N, g.K,
-                                                                                        n_fastest, sk);
+  const dim3 grid(2 * pairs);
+  const bool skk = sk.on || sk.sleep_ns;
+  const int epi = g.ep.out_f32 ? 2 : (g.ep.aux ? 1 : 0);
+#define MARIO_PAIR_LAUNCH(SKV, EV) \
+  gemm_bf16_tc2_kernel<BNP, A_MN, B_MN, SKV, EV><<<grid, kThreads2, C2::kSmem, st>>>(ta, tb, g.ep, g.M, g.N, g.K, n_fastest, sk)
+  if (skk) {
+    if (epi == 2) MARIO_PAIR_LAUNCH(true, 2); else if (epi == 1) MARIO_PAIR_LAUNCH(true, 1); else MARIO_PAIR_LAUNCH(true, 0);
+  } else {
+    if (epi == 2) MARIO_PAIR_LAUNCH(false, 2); else if (epi == 1) MARIO_PAIR_LAUNCH(false, 1); else MARIO_PAIR_LAUNCH(false, 0);
+  }
+#undef MARIO_PAIR_LAUNCH
   kstats_end(tok, st);
   note_launch();
   return cudaGetLastError();
@@ -948,6 +960,10 @@ cudaError_t gemm_bf16(const GemmArgs& g0, cudaStream_t st) {
     return cudaErrorInvalidValue;
   }
   auto al16 = [](const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; };
+  if (g.ep.aux && (g.ep.residual || g.ep.out_f32)) {
+    fprintf(stderr, "[mario] gemm_bf16: a GeLU' aux needs bf16 output and no residual\n");
+    return cudaErrorInvalidValue;
+  }
   if (g.ep.colsum_part &&
       (g.ep.out_f32 || (g.M % 32) || (g.N % 32) || !g.ep.d_bf16 || (g.ep.ldd % 8) || !al16(g.ep.d_bf16) ||
        (g.ep.d2_bf16 && !al16(g.ep.d2_bf16)) || (g.ep.residual && ((g.ep.ld_res % 8) || !al16(g.ep.residual))) ||
