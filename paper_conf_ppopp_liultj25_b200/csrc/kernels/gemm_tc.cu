@@ -197,7 +197,15 @@ __device__ __forceinline__ uint8_t* sw128(uint8_t* sw, int r, int j) { return sw
 #ifndef MARIO_EPI_PREFETCH
 #define MARIO_EPI_PREFETCH 1   // 0: each block loads its own input when it starts (A/B experiments)
 #endif
-struct EpiPrefetch { uint4 v[4]; };
+// The block's bf16 input is copied with cp.async straight into the upper 2 KB of the warp's 4 KB
+// staging buffer (the bf16 transposition uses only the lower 2 KB), in the swizzled row layout the
+// read-back expects: no registers are held while it is in flight (a register prefetch pushed the
+// epilogue into spills). fp32 outputs (EPI 2) transpose through all 4 KB, so they load on demand.
+struct EpiPrefetch { uint8_t* buf; };   // = sw + 2048
+__device__ __forceinline__ void cp_async16(void* dst, const void* src, bool valid) {
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" :: "r"(smem_u32(dst)), "l"(src), "r"(valid ? 16 : 0)
+               : "memory");
+}
 __device__ __forceinline__ void epi_prefetch(const GemmEpilogue& ep, bool vec_ok, int rbase, int lane, int col0, int M,
                                              int N, EpiPrefetch& pf) {
   if (col0 < 0 || col0 >= N || !vec_ok || col0 + 32 > N) return;
@@ -207,28 +215,18 @@ __device__ __forceinline__ void epi_prefetch(const GemmEpilogue& ep, bool vec_ok
 #pragma unroll
   for (int it = 0; it < 4; ++it) {
     const int rr = it * 8 + lane / 4, ch = lane % 4;
-    pf.v[it] = rbase + rr < M ? *reinterpret_cast<const uint4*>(base + static_cast<size_t>(rbase + rr) * ld + col0 + ch * 8)
-                              : make_uint4(0, 0, 0, 0);
+    const bool ok = rbase + rr < M;   // rows >= M read as 0 (src-size 0)
+    cp_async16(sw64(pf.buf, rr, ch), base + static_cast<size_t>(ok ? rbase + rr : rbase) * ld + col0 + ch * 8, ok);
   }
+  asm volatile("cp.async.commit_group;" ::: "memory");
 }
-// direct (not prefetched) coalesced read of a bf16 block into registers, same layout
-__device__ __forceinline__ void epi_rows_bf16(const __nv_bfloat16* base, int ld, int rbase, int col0, int M, int lane,
-                                              uint4* out) {
-#pragma unroll
-  for (int it = 0; it < 4; ++it) {
-    const int rr = it * 8 + lane / 4, ch = lane % 4;
-    out[it] = rbase + rr < M ? *reinterpret_cast<const uint4*>(base + static_cast<size_t>(rbase + rr) * ld + col0 + ch * 8)
-                             : make_uint4(0, 0, 0, 0);
-  }
-}
-// prefetched bf16 [32 rows][32 cols] block -> sw -> each lane reads back its own row's 32 values
-__device__ __forceinline__ void load_block_bf16(const uint4* pre, int lane, uint8_t* sw, float (&out)[32]) {
-#pragma unroll
-  for (int it = 0; it < 4; ++it) sts128(sw64(sw, it * 8 + lane / 4, lane % 4), pre[it]);
+// the prefetched bf16 [32 rows][32 cols] block -> each lane's own row of 32 values
+__device__ __forceinline__ void load_block_bf16(const EpiPrefetch& pf, int lane, float (&out)[32]) {
+  asm volatile("cp.async.wait_group 0;" ::: "memory");
   __syncwarp();
 #pragma unroll
   for (int j = 0; j < 4; ++j) {
-    const uint4 u = lds128u(sw64(sw, lane, j));
+    const uint4 u = lds128u(sw64(pf.buf, lane, j));
     const __nv_bfloat162* h = reinterpret_cast<const __nv_bfloat162*>(&u);
 #pragma unroll
     for (int e = 0; e < 4; ++e) {
@@ -269,10 +267,10 @@ __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool
   if (col0 >= N) return;
   if (!vec_ok || col0 + 32 > N) {   // warp-uniform: ragged column block or unaligned pitches
     epilogue_chunk<EPI == 2>(ep, r, rbase + lane, col0, rbase + lane < M, N);
-    if (MARIO_EPI_PREFETCH) epi_prefetch(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
+    if (MARIO_EPI_PREFETCH && EPI != 2) epi_prefetch(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
     return;
   }
-  if (!MARIO_EPI_PREFETCH) epi_prefetch(ep, vec_ok, rbase, lane, col0, M, N, pf);
+  if (!MARIO_EPI_PREFETCH || EPI == 2) epi_prefetch(ep, vec_ok, rbase, lane, col0, M, N, pf);
   float v[32];
 #pragma unroll
   for (int j = 0; j < 32; ++j) v[j] = __uint_as_float(r[j]);
@@ -285,7 +283,7 @@ __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool
   }
   float z[32];
   if constexpr (EPI == 1) {   // GeLU backward: D = acc * gelu'(Z)
-    load_block_bf16(pf.v, lane, sw, z);
+    load_block_bf16(pf, lane, z);
     if (MARIO_EPI_PREFETCH) epi_prefetch(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
 #pragma unroll
     for (int j = 0; j < 32; ++j) v[j] *= gelu_tanh_grad_f(z[j]);
@@ -293,8 +291,8 @@ __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool
   if constexpr (EPI != 1) {   // residual: not on the aux path (gemm_bf16 rejects aux + residual)
     if (ep.residual) {
       float rr[32];
-      load_block_bf16(pf.v, lane, sw, rr);
-      if (MARIO_EPI_PREFETCH) epi_prefetch(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
+      load_block_bf16(pf, lane, rr);
+      if (MARIO_EPI_PREFETCH && EPI != 2) epi_prefetch(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
 #pragma unroll
       for (int j = 0; j < 32; ++j) v[j] += rr[j];
     }
@@ -459,8 +457,8 @@ gemm_bf16_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
         tile_coords(tile, num_m, num_n, n_fastest, tm, tn);
       const int m0 = tm * BM, n0 = tn * BN;
       const int rbase = m0 + quarter * 32;
-      EpiPrefetch pf;
-      if (MARIO_EPI_PREFETCH) epi_prefetch(ep, vec_ok, rbase, lane, n0, M, N, pf);
+      EpiPrefetch pf{sw + 2048};
+      if (MARIO_EPI_PREFETCH && !ep.out_f32) epi_prefetch(ep, vec_ok, rbase, lane, n0, M, N, pf);
       mbar_wait(&tfull[acc], acc_ph);
       tc_fence_after();
 #pragma unroll 1
@@ -673,8 +671,8 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
         tile_coords(tile, num_m, num_n, n_fastest, tm, tn);
       const int m0 = tm * 256 + 128 * rank, n0 = tn * BNP;
       const int rbase = m0 + quarter * 32;
-      EpiPrefetch pf;
-      if (MARIO_EPI_PREFETCH && !(skon && u.kb0 != 0)) epi_prefetch(ep, vec_ok, rbase, lane, n0 + half * (BNP / 2), M, N, pf);
+      EpiPrefetch pf{sw + 2048};
+      if (MARIO_EPI_PREFETCH && EPI != 2 && !(skon && u.kb0 != 0)) epi_prefetch(ep, vec_ok, rbase, lane, n0 + half * (BNP / 2), M, N, pf);
       if (SK && sk.sleep_ns) { while (!mbar_test(&tfull[acc], acc_ph)) __nanosleep(sk.sleep_ns); }
       else mbar_wait(&tfull[acc], acc_ph);
       tc_fence_after();
