@@ -62,6 +62,41 @@ __device__ __forceinline__ float ld_shared_f32(const void* p) {
   return v;
 }
 
+// L2 eviction priorities (MARIO_ATTN_L2HINT, default on): the tiles many CTAs re-read (K/V in the
+// forward and the dQ pass, Q/dO/lse/D in the dK/dV pass) evict_last, each CTA's own stationary
+// tiles and the once-read dS image evict_first.
+__device__ __forceinline__ uint64_t pol_first() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t pol_last() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t pol_normal() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+int attn_l2hint() {
+  // default off: A/B on whole steps was neutral (attention backward -5 ms, the following GEMMs +20-40 ms:
+  // evict_last attention tiles outlive the kernel in L2)
+  static const int v = getenv("MARIO_ATTN_L2HINT") ? atoi(getenv("MARIO_ATTN_L2HINT")) : 0;
+  return v;
+}
+__device__ __forceinline__ void tma_load_2d_h(void* dst, const void* tmap, uint64_t* bar, int c0, int c1, uint64_t pol) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint"
+      " [%0], [%1, {%3, %4}], [%2], %5;"
+      :: "r"(smem_u32(dst)), "l"(reinterpret_cast<uint64_t>(tmap)), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "l"(pol)
+      : "memory");
+}
+__device__ __forceinline__ void bulk_g2s_h(void* dst, const void* src, uint32_t bytes, uint64_t* bar, uint64_t pol) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes.L2::cache_hint [%0], [%1], %2, [%3], %4;"
+               :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)), "l"(pol) : "memory");
+}
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
                :: "r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
@@ -644,7 +679,7 @@ __global__ void __launch_bounds__(kThreadsB, 1)
 fa_bwd_dkdv_ts(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_qkv64,
                const __grid_constant__ CUtensorMap tm_do64,
                const __grid_constant__ CUtensorMap tm_dqkv, const float* lse, const float* Dd, bf16* dqkv, int B,
-               int s, int nh, uint8_t* dsimg) {
+               int s, int nh, uint8_t* dsimg, int l2hint) {
   const bool bulk_ld = (s % kCols) == 0;
   using SM = Smem<DH>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -700,12 +735,13 @@ fa_bwd_dkdv_ts(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
 
   if (warp == 0) {
     if (elect_one()) {
+      const uint64_t pf_ = l2hint ? pol_first() : pol_normal(), pl_ = l2hint ? pol_last() : pol_normal();
       const int row0 = b * s;
       mbar_arrive_expect_tx(kv_full, 2 * SM::kBig);
 #pragma unroll
       for (int a = 0; a < DH / 64; ++a) {
-        tma_load_2d(sK + a * (kRows * 128), &tm_qkv128, kv_full, h + head * DH + a * 64, row0 + kt * kRows);
-        tma_load_2d(sV + a * (kRows * 128), &tm_qkv128, kv_full, 2 * h + head * DH + a * 64, row0 + kt * kRows);
+        tma_load_2d_h(sK + a * (kRows * 128), &tm_qkv128, kv_full, h + head * DH + a * 64, row0 + kt * kRows, pf_);
+        tma_load_2d_h(sV + a * (kRows * 128), &tm_qkv128, kv_full, 2 * h + head * DH + a * 64, row0 + kt * kRows, pf_);
       }
       for (int idx = 0; idx < ntiles; ++idx) {
         const int st = idx % kRingTS;
@@ -714,13 +750,13 @@ fa_bwd_dkdv_ts(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
         const int qr = row0 + (i0 + idx) * kCols;
 #pragma unroll
         for (int a = 0; a < DH / 64; ++a) {
-          tma_load_2d(sQ(st) + a * (kCols * 128), &tm_qkv64, &q_full[st], head * DH + a * 64, qr);
-          tma_load_2d(sG(st) + a * (kCols * 128), &tm_do64, &q_full[st], head * DH + a * 64, qr);
+          tma_load_2d_h(sQ(st) + a * (kCols * 128), &tm_qkv64, &q_full[st], head * DH + a * 64, qr, pl_);
+          tma_load_2d_h(sG(st) + a * (kCols * 128), &tm_do64, &q_full[st], head * DH + a * 64, qr, pl_);
         }
         if (bulk_ld) {
           const long o = static_cast<long>(head) * Ttok + qr;
-          bulk_g2s(sLD + st * 2 * kCols, lse + o, kCols * 4, &q_full[st]);
-          bulk_g2s(sLD + st * 2 * kCols + kCols, Dd + o, kCols * 4, &q_full[st]);
+          bulk_g2s_h(sLD + st * 2 * kCols, lse + o, kCols * 4, &q_full[st], pl_);
+          bulk_g2s_h(sLD + st * 2 * kCols + kCols, Dd + o, kCols * 4, &q_full[st], pl_);
         }
       }
     }
@@ -1178,7 +1214,7 @@ struct SmemI {
 template <int DH>
 __global__ void __launch_bounds__(kThreadsI, 1)
 fa_bwd_dq_img(const __grid_constant__ CUtensorMap tm_qkv64, const uint8_t* __restrict__ dsimg, bf16* dqkv, int B, int s,
-              int nh) {
+              int nh, int l2hint) {
   using SI = SmemI<DH>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -1211,6 +1247,7 @@ fa_bwd_dq_img(const __grid_constant__ CUtensorMap tm_qkv64, const uint8_t* __res
 
   if (warp == 0) {
     if (elect_one()) {
+      const uint64_t pf_ = l2hint ? pol_first() : pol_normal(), pl_ = l2hint ? pol_last() : pol_normal();
       int kc = 0;
       for (int w = blockIdx.x; w < W; w += gridDim.x) {
         int qb, bh, ntiles;
@@ -1222,10 +1259,11 @@ fa_bwd_dq_img(const __grid_constant__ CUtensorMap tm_qkv64, const uint8_t* __res
           uint8_t* sa = smem + st * SI::kStage;
           mbar_wait(&empty[st], ((kc / kRingI) & 1) ^ 1);
           mbar_arrive_expect_tx(&full[st], SI::kStage);
-          bulk_g2s(sa, img + static_cast<size_t>(kt) * SI::kA, SI::kA, &full[st]);
+          bulk_g2s_h(sa, img + static_cast<size_t>(kt) * SI::kA, SI::kA, &full[st], pf_);
 #pragma unroll
           for (int a = 0; a < DH / 64; ++a)
-            tma_load_2d(sa + SI::kA + a * (kCols * 128), &tm_qkv64, &full[st], h + head * DH + a * 64, b * s + kt * kCols);
+            tma_load_2d_h(sa + SI::kA + a * (kCols * 128), &tm_qkv64, &full[st], h + head * DH + a * 64, b * s + kt * kCols,
+                          pl_);
         }
       }
     }
@@ -1343,7 +1381,7 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
         tset = true;
       }
       fa_bwd_dkdv_ts<DH><<<grid, kThreadsB, smem_dkdv_ts<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s, nh,
-                                                                        dsimg);
+                                                                        dsimg, attn_l2hint());
     } else {
       fa_bwd_dkdv_tc<DH><<<grid, kThreadsB, smem_dkdv<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s, nh, dbg,
                                                                      want_trace ? trace : nullptr);
@@ -1373,7 +1411,7 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
     const int items = B * nh * (s / kRows);
     static const int per_sm = getenv("MARIO_DQI_CTAS") ? atoi(getenv("MARIO_DQI_CTAS")) : 2;
     const int grid_i = items < per_sm * sms ? items : per_sm * sms;
-    fa_bwd_dq_img<DH><<<grid_i, kThreadsI, SmemI<DH>::kBytes, st>>>(m64, dsimg, dqkv, B, s, nh);
+    fa_bwd_dq_img<DH><<<grid_i, kThreadsI, SmemI<DH>::kBytes, st>>>(m64, dsimg, dqkv, B, s, nh, attn_l2hint());
   } else if (!only || only[1] == 'q') {
     if (pers && dbg == 0) {
       static bool pset = false;
@@ -1649,7 +1687,7 @@ __device__ __forceinline__ void f2_item(int i, int n, bool& is_v, int& j) {
 
 template <int DH>
 __global__ void __launch_bounds__(kF2Threads, 1)
-fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, int B, int s, int nh) {
+fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, int B, int s, int nh, int g_l2hint) {
   using SM = SmemF2<DH>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -1696,14 +1734,15 @@ fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, i
     asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");
   if (warp == 0) {
     if (elect_one()) {
+      const uint64_t pf_ = g_l2hint ? pol_first() : pol_normal(), pl_ = g_l2hint ? pol_last() : pol_normal();
       const int row0 = b * s;
       mbar_arrive_expect_tx(q_full, 2 * SM::kTile);
 #pragma unroll
       for (int t = 0; t < 2; ++t)
 #pragma unroll
         for (int a = 0; a < DH / 64; ++a)
-          tma_load_2d(sQ + t * SM::kTile + a * (kF2Q * 128), &tm_qkv128, q_full, head * DH + a * 64,
-                      row0 + q0 + t * kF2Q);
+          tma_load_2d_h(sQ + t * SM::kTile + a * (kF2Q * 128), &tm_qkv128, q_full, head * DH + a * 64,
+                        row0 + q0 + t * kF2Q, pf_);
       for (int i = 0; i < 2 * n1; ++i) {
         bool is_v;
         int j;
@@ -1714,8 +1753,8 @@ fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, i
         uint8_t* dst = sRing + st * SM::kTile;
 #pragma unroll
         for (int a = 0; a < DH / 64; ++a)
-          tma_load_2d(dst + a * (kF2N * 128), &tm_qkv128, &full[st], (is_v ? 2 * h : h) + head * DH + a * 64,
-                      row0 + j * kF2N);
+          tma_load_2d_h(dst + a * (kF2N * 128), &tm_qkv128, &full[st], (is_v ? 2 * h : h) + head * DH + a * 64,
+                        row0 + j * kF2N, pl_);
       }
     }
   } else if (warp == 1) {
@@ -1888,7 +1927,7 @@ bool launch_fwd2_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, 
     set = true;
   }
   const int nqb = (s + 2 * kF2Q - 1) / (2 * kF2Q);
-  fa_fwd2_tc<DH><<<nqb * B * nh, kF2Threads, smem, st>>>(m128, O, lse, B, s, nh);
+  fa_fwd2_tc<DH><<<nqb * B * nh, kF2Threads, smem, st>>>(m128, O, lse, B, s, nh, attn_l2hint());
   note_launch();
   return true;
 }
