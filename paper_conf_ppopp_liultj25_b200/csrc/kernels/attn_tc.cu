@@ -62,7 +62,7 @@ __device__ __forceinline__ float ld_shared_f32(const void* p) {
   return v;
 }
 
-// L2 eviction priorities (MARIO_ATTN_L2HINT, default on): the tiles many CTAs re-read (K/V in the
+// L2 eviction priorities (MARIO_ATTN_L2HINT, default off): the tiles many CTAs re-read (K/V in the
 // forward and the dQ pass, Q/dO/lse/D in the dK/dV pass) evict_last, each CTA's own stationary
 // tiles and the once-read dS image evict_first.
 __device__ __forceinline__ uint64_t pol_first() {
