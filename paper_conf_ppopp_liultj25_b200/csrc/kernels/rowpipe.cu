@@ -11,6 +11,7 @@
 // Formulas: SURVEY §8(c) c1 (LN/RMS forward, readings A1/A2; backward dx = (g - mean g - xhat
 // mean(g xhat)) / sigma, dgamma = sum dy xhat, dbeta = sum dy).
 #include <cstdint>
+#include <cstdlib>
 #include <cuda_bf16.h>
 #include <cuda_runtime.h>
 
@@ -261,7 +262,7 @@ __global__ void __launch_bounds__(1024) norm_fwd_pipe_k(const bf16* __restrict__
 // memory (row sums), phase 2 (after the barrier) re-reads dy, x, dres and writes dx, so nothing
 // but the column accumulators stays in registers; a slot is refilled at the NEXT iteration's
 // barrier, when every thread is past its phase 2. Stats of the CTA's range are staged in smem.
-template <int R>
+template <int R, int V>   // V: 16-byte chunks per thread (chunks t, t + nt, ...), amortizing the per-row work
 __global__ void __launch_bounds__(640) norm_bwd_pipe_k(const bf16* __restrict__ dy, const bf16* __restrict__ x,
                                                        const float* __restrict__ stats, const float* __restrict__ g,
                                                        const bf16* __restrict__ dres, bf16* __restrict__ dx, int rows,
@@ -274,8 +275,10 @@ __global__ void __launch_bounds__(640) norm_bwd_pipe_k(const bf16* __restrict__ 
   uint64_t* bar = reinterpret_cast<uint64_t*>(smem_raw + static_cast<size_t>(S) * sb);
   float* red = reinterpret_cast<float*>(bar + S);            // [2][32][R][2]
   float2* sstat = reinterpret_cast<float2*>(red + 2 * 32 * R * 2);
-  const int t = threadIdx.x, w = t / 32, lane = t % 32, nw = blockDim.x / 32;
-  const bool act = t * 8 < n;
+  const int t = threadIdx.x, w = t / 32, lane = t % 32, nw = blockDim.x / 32, nt = blockDim.x;
+  bool act[V];
+#pragma unroll
+  for (int k = 0; k < V; ++k) act[k] = (t + k * nt) * 8 < n;
   const int rb = static_cast<int>(static_cast<long>(rows) * blockIdx.x / nblk);
   const int re = static_cast<int>(static_cast<long>(rows) * (blockIdx.x + 1) / nblk);
   auto issue = [&](int sl, int r) {
@@ -294,10 +297,13 @@ __global__ void __launch_bounds__(640) norm_bwd_pipe_k(const bf16* __restrict__ 
     for (int i = 0; i < S && rb + i < re; ++i) issue(i, rb + i);
   for (int i = t; i < re - rb && i < max_range; i += blockDim.x)
     sstat[i] = *reinterpret_cast<const float2*>(stats + 2 * static_cast<long>(rb + i));
-  float gg[8], ag[8], ab[8], ao[8];
+  float gg[V][8], ag[V][8], ab[V][8], ao[V][8];
 #pragma unroll
-  for (int j = 0; j < 8; ++j) { gg[j] = 0.f; ag[j] = 0.f; ab[j] = 0.f; ao[j] = 0.f; }
-  if (act) load8(g + t * 8, gg);
+  for (int k = 0; k < V; ++k) {
+#pragma unroll
+    for (int j = 0; j < 8; ++j) { gg[k][j] = 0.f; ag[k][j] = 0.f; ab[k][j] = 0.f; ao[k][j] = 0.f; }
+    if (act[k]) load8(g + (t + k * nt) * 8, gg[k]);
+  }
   __syncthreads();
   const float inv_n = 1.f / n;
   for (int r0 = rb, it = 0; r0 < re; r0 += R, ++it) {
@@ -311,21 +317,25 @@ __global__ void __launch_bounds__(640) norm_bwd_pipe_k(const bf16* __restrict__ 
       const uint8_t* buf = stage0 + static_cast<size_t>(sl) * sb;
       const float2 ms = sstat[u];
       mbar_wait(&bar[sl], (u / S) & 1);
-      if (!act) continue;
-      float d[8], xh[8];
-      unpack8(lds128(buf + t * 16), d);
-      unpack8(lds128(buf + row_bytes + t * 16), xh);
       float2 a_sg = f2(0.f, 0.f), a_sgx = f2(0.f, 0.f);
 #pragma unroll
-      for (int j = 0; j < 8; j += 2) {
-        const float2 dd = f2(d[j], d[j + 1]);
-        const float2 xx = mul2(add2(f2(xh[j], xh[j + 1]), f2(-ms.x, -ms.x)), f2(ms.y, ms.y));
-        const float2 gp = mul2(dd, f2(gg[j], gg[j + 1]));
-        a_sg = add2(a_sg, gp);
-        a_sgx = fma2(gp, xx, a_sgx);
-        const float2 na = fma2(dd, xx, f2(ag[j], ag[j + 1]));
-        const float2 nb = add2(f2(ab[j], ab[j + 1]), dd);
-        ag[j] = na.x; ag[j + 1] = na.y; ab[j] = nb.x; ab[j + 1] = nb.y;
+      for (int k = 0; k < V; ++k) {
+        if (!act[k]) continue;
+        const int off = (t + k * nt) * 16;
+        float d[8], xh[8];
+        unpack8(lds128(buf + off), d);
+        unpack8(lds128(buf + row_bytes + off), xh);
+#pragma unroll
+        for (int j = 0; j < 8; j += 2) {
+          const float2 dd = f2(d[j], d[j + 1]);
+          const float2 xx = mul2(add2(f2(xh[j], xh[j + 1]), f2(-ms.x, -ms.x)), f2(ms.y, ms.y));
+          const float2 gp = mul2(dd, f2(gg[k][j], gg[k][j + 1]));
+          a_sg = add2(a_sg, gp);
+          a_sgx = fma2(gp, xx, a_sgx);
+          const float2 na = fma2(dd, xx, f2(ag[k][j], ag[k][j + 1]));
+          const float2 nb = add2(f2(ab[k][j], ab[k][j + 1]), dd);
+          ag[k][j] = na.x; ag[k][j + 1] = na.y; ab[k][j] = nb.x; ab[k][j + 1] = nb.y;
+        }
       }
       sg[q] = a_sg.x + a_sg.y;
       sgx[q] = a_sgx.x + a_sgx.y;
@@ -354,7 +364,6 @@ __global__ void __launch_bounds__(640) norm_bwd_pipe_k(const bf16* __restrict__ 
     }
     float tg[R], tgx[R];
     cross_warp_sums<R>(rp, nw, lane, tg, tgx);
-    if (!act) continue;
 #pragma unroll
     for (int q = 0; q < R; ++q) {
       const int r = r0 + q;
@@ -363,50 +372,60 @@ __global__ void __launch_bounds__(640) norm_bwd_pipe_k(const bf16* __restrict__ 
       const uint8_t* buf = stage0 + static_cast<size_t>(u % S) * sb;
       const float2 ms = sstat[u];
       const float mg = rms ? 0.f : tg[q] * inv_n, mgx = tgx[q] * inv_n;
-      float d[8], xh[8], rr[8];
-      unpack8(lds128(buf + t * 16), d);
-      unpack8(lds128(buf + row_bytes + t * 16), xh);
-      if (dres) unpack8(lds128(buf + 2 * row_bytes + t * 16), rr);
-      float o[8];
-      if (!dres) {
 #pragma unroll
-        for (int j = 0; j < 8; ++j) rr[j] = 0.f;
-      }
+      for (int k = 0; k < V; ++k) {
+        if (!act[k]) continue;
+        const int cidx = t + k * nt, off = cidx * 16;
+        float d[8], xh[8], rr[8];
+        unpack8(lds128(buf + off), d);
+        unpack8(lds128(buf + row_bytes + off), xh);
+        if (dres) {
+          unpack8(lds128(buf + 2 * row_bytes + off), rr);
+        } else {
 #pragma unroll
-      for (int j = 0; j < 8; j += 2) {
-        const float2 xhat = mul2(add2(f2(xh[j], xh[j + 1]), f2(-ms.x, -ms.x)), f2(ms.y, ms.y));
-        const float2 u = add2(mul2(f2(d[j], d[j + 1]), f2(gg[j], gg[j + 1])), f2(-mg, -mg));
-        const float2 w = fma2(xhat, f2(-mgx, -mgx), u);
-        const float2 res = fma2(w, f2(ms.y, ms.y), f2(rr[j], rr[j + 1]));
-        o[j] = res.x; o[j + 1] = res.y;
-      }
-      const uint4 pk = pack8(o);
-      *reinterpret_cast<uint4*>(dx + static_cast<long>(r) * n + t * 8) = pk;
-      if (sum_out) {
-        float qv[8];
-        unpack8(pk, qv);
+          for (int j = 0; j < 8; ++j) rr[j] = 0.f;
+        }
+        float o[8];
 #pragma unroll
         for (int j = 0; j < 8; j += 2) {
-          const float2 a = add2(f2(ao[j], ao[j + 1]), f2(qv[j], qv[j + 1]));
-          ao[j] = a.x; ao[j + 1] = a.y;
+          const float2 xhat = mul2(add2(f2(xh[j], xh[j + 1]), f2(-ms.x, -ms.x)), f2(ms.y, ms.y));
+          const float2 uu = add2(mul2(f2(d[j], d[j + 1]), f2(gg[k][j], gg[k][j + 1])), f2(-mg, -mg));
+          const float2 ww = fma2(xhat, f2(-mgx, -mgx), uu);
+          const float2 res = fma2(ww, f2(ms.y, ms.y), f2(rr[j], rr[j + 1]));
+          o[j] = res.x; o[j + 1] = res.y;
+        }
+        const uint4 pk = pack8(o);
+        *reinterpret_cast<uint4*>(dx + static_cast<long>(r) * n + cidx * 8) = pk;
+        if (sum_out) {
+          float qv[8];
+          unpack8(pk, qv);
+#pragma unroll
+          for (int j = 0; j < 8; j += 2) {
+            const float2 a = add2(f2(ao[k][j], ao[k][j + 1]), f2(qv[j], qv[j + 1]));
+            ao[k][j] = a.x; ao[k][j + 1] = a.y;
+          }
         }
       }
     }
   }
-  if (!partial || !act) return;
-  const int c = t * 8;
-  float* p0 = partial + static_cast<long>(blockIdx.x) * n + c;
-  *reinterpret_cast<float4*>(p0) = make_float4(ag[0], ag[1], ag[2], ag[3]);
-  *reinterpret_cast<float4*>(p0 + 4) = make_float4(ag[4], ag[5], ag[6], ag[7]);
-  if (!rms) {
-    float* p1 = partial + static_cast<long>(nblk + blockIdx.x) * n + c;
-    *reinterpret_cast<float4*>(p1) = make_float4(ab[0], ab[1], ab[2], ab[3]);
-    *reinterpret_cast<float4*>(p1 + 4) = make_float4(ab[4], ab[5], ab[6], ab[7]);
-  }
-  if (sum_out) {
-    float* p2 = partial + static_cast<long>(2 * nblk + blockIdx.x) * n + c;
-    *reinterpret_cast<float4*>(p2) = make_float4(ao[0], ao[1], ao[2], ao[3]);
-    *reinterpret_cast<float4*>(p2 + 4) = make_float4(ao[4], ao[5], ao[6], ao[7]);
+  if (!partial) return;
+#pragma unroll
+  for (int k = 0; k < V; ++k) {
+    if (!act[k]) continue;
+    const int c = (t + k * nt) * 8;
+    float* p0 = partial + static_cast<long>(blockIdx.x) * n + c;
+    *reinterpret_cast<float4*>(p0) = make_float4(ag[k][0], ag[k][1], ag[k][2], ag[k][3]);
+    *reinterpret_cast<float4*>(p0 + 4) = make_float4(ag[k][4], ag[k][5], ag[k][6], ag[k][7]);
+    if (!rms) {
+      float* p1 = partial + static_cast<long>(nblk + blockIdx.x) * n + c;
+      *reinterpret_cast<float4*>(p1) = make_float4(ab[k][0], ab[k][1], ab[k][2], ab[k][3]);
+      *reinterpret_cast<float4*>(p1 + 4) = make_float4(ab[k][4], ab[k][5], ab[k][6], ab[k][7]);
+    }
+    if (sum_out) {
+      float* p2 = partial + static_cast<long>(2 * nblk + blockIdx.x) * n + c;
+      *reinterpret_cast<float4*>(p2) = make_float4(ao[k][0], ao[k][1], ao[k][2], ao[k][3]);
+      *reinterpret_cast<float4*>(p2 + 4) = make_float4(ao[k][4], ao[k][5], ao[k][6], ao[k][7]);
+    }
   }
 }
 
@@ -583,8 +602,11 @@ bool norm_fwd_pipe(const bf16* x, const float* g, const float* b, bf16* y, float
   if (!norm_pipe_supported(n)) return false;
   if (rows <= 0) return true;
   const int nt = threads_for(n), sb = n * 2;
-  int S = 24576 / sb;
-  S = S < 2 * kPipeR ? 2 * kPipeR : (S > 8 ? 8 : S);
+  // ring bytes / max stages per CTA (MARIO_NORM_FWD_RING, MARIO_NORM_FWD_SMAX: tuning experiments)
+  static const int ring = getenv("MARIO_NORM_FWD_RING") ? atoi(getenv("MARIO_NORM_FWD_RING")) : 24576;
+  static const int smax = getenv("MARIO_NORM_FWD_SMAX") ? atoi(getenv("MARIO_NORM_FWD_SMAX")) : 8;
+  int S = ring / sb;
+  S = S < 2 * kPipeR ? 2 * kPipeR : (S > smax ? smax : S);
   S -= S % kPipeR;
   const size_t smem = pipe_smem_bytes(S, sb);
   static bool attr = false;
@@ -601,23 +623,25 @@ bool norm_fwd_pipe(const bf16* x, const float* g, const float* b, bf16* y, float
   return true;
 }
 
-bool norm_bwd_pipe(const bf16* dy, const bf16* x, const float* stats, const float* g, const bf16* dres, bf16* dx,
-                   int rows, int n, int rms, float* dg, float* db, float* dsum, float* partial, size_t partial_floats,
-                   cudaStream_t st) {
-  if (!norm_pipe_supported(n) || threads_for(n) > 640) return false;
-  if (rows <= 0) return true;
-  const int nt = threads_for(n), nin = dres ? 3 : 2, sb = nin * n * 2;
-  int S = 49152 / sb;
-  S = S < 2 * kPipeR ? 2 * kPipeR : (S > 6 ? 6 : S);
+template <int V>
+bool norm_bwd_pipe_v(const bf16* dy, const bf16* x, const float* stats, const float* g, const bf16* dres, bf16* dx,
+                     int rows, int n, int rms, float* dg, float* db, float* dsum, float* partial, size_t partial_floats,
+                     cudaStream_t st) {
+  const int nt = ((n / (8 * V) + 31) / 32) * 32, nin = dres ? 3 : 2, sb = nin * n * 2;
+  if (nt > 640) return false;
+  static const int ring = getenv("MARIO_NORM_BWD_RING") ? atoi(getenv("MARIO_NORM_BWD_RING")) : 49152;
+  static const int smax = getenv("MARIO_NORM_BWD_SMAX") ? atoi(getenv("MARIO_NORM_BWD_SMAX")) : 6;
+  int S = ring / sb;
+  S = S < 2 * kPipeR ? 2 * kPipeR : (S > smax ? smax : S);
   S -= S % kPipeR;
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(norm_bwd_pipe_k<kPipeR>, cudaFuncAttributeMaxDynamicSharedMemorySize, 220 * 1024);
+    cudaFuncSetAttribute(norm_bwd_pipe_k<kPipeR, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, 220 * 1024);
     attr = true;
   }
   // the stats of a CTA's range are staged in shared memory: size for the smallest grid we may use
   const size_t base = pipe_smem_bytes(S, sb);
-  int nblk = occ_grid(norm_bwd_pipe_k<kPipeR>, nt, base + 8 * static_cast<size_t>(cdivl(rows, device_sms())));
+  int nblk = occ_grid(norm_bwd_pipe_k<kPipeR, V>, nt, base + 8 * static_cast<size_t>(cdivl(rows, device_sms())));
   if (dg) {
     const long cap = static_cast<long>(partial_floats / (3 * static_cast<size_t>(n)));
     if (cap < 1) return false;
@@ -627,14 +651,26 @@ bool norm_bwd_pipe(const bf16* dy, const bf16* x, const float* stats, const floa
   const int max_range = cdivl(rows, nblk) + 1;
   const size_t smem = base + 8 * static_cast<size_t>(max_range);
   if (smem > 220 * 1024) return false;
-  norm_bwd_pipe_k<kPipeR><<<nblk, nt, smem, st>>>(dy, x, stats, g, dres, dx, rows, n, rms, dg ? partial : nullptr, nblk,
-                                          dsum ? 1 : 0, S, max_range);
+  norm_bwd_pipe_k<kPipeR, V><<<nblk, nt, smem, st>>>(dy, x, stats, g, dres, dx, rows, n, rms, dg ? partial : nullptr,
+                                                     nblk, dsum ? 1 : 0, S, max_range);
   note_launch();
   if (dg) {
     colsum_final_wide_k<<<cdivl(n, 32), 1024, 0, st>>>(partial, nblk, n, dg, rms ? nullptr : db, dsum);
     note_launch();
   }
   return true;
+}
+
+bool norm_bwd_pipe(const bf16* dy, const bf16* x, const float* stats, const float* g, const bf16* dres, bf16* dx,
+                   int rows, int n, int rms, float* dg, float* db, float* dsum, float* partial, size_t partial_floats,
+                   cudaStream_t st) {
+  if (!norm_pipe_supported(n)) return false;
+  if (rows <= 0) return true;
+  // 16-byte chunks per thread (MARIO_NORM_BWD_V)
+  static const int vsel = getenv("MARIO_NORM_BWD_V") ? atoi(getenv("MARIO_NORM_BWD_V")) : 2;
+  if (vsel == 2 && n % 2048 == 0)   // measured: h 4096 73.8 -> 63.9 us, h 2048 equal, h 5120 slower
+    return norm_bwd_pipe_v<2>(dy, x, stats, g, dres, dx, rows, n, rms, dg, db, dsum, partial, partial_floats, st);
+  return norm_bwd_pipe_v<1>(dy, x, stats, g, dres, dx, rows, n, rms, dg, db, dsum, partial, partial_floats, st);
 }
 
 bool softmax_ce_fast(const float* logits, const int32_t* tok, int ld_tok, int s, int rows, int V, float inv_ntok,
