@@ -91,6 +91,51 @@ __global__ void embed_segsum_k(const long long* keys, int Ttok, const T* dH, int
   }
 }
 
+// bf16, h % 8 == 0: one warp per segment (sorted positions sharing a token). The warp reads the
+// segment's keys 32 at a time (one division per key, ballot for the segment end), and each lane then
+// owns 8 consecutive columns per 16-byte load, adding the segment's rows in position order (the same
+// order as the scalar kernel: bitwise-identical sums for segments of up to 32 positions). The scalar
+// kernel re-divided every key for every column (179 us per micro-batch at cfg 2).
+__global__ void embed_segsum_v8_k(const long long* keys, int Ttok, const __nv_bfloat16* dH, int h, float* dwte) {
+  const int warp = (blockIdx.x * blockDim.x + threadIdx.x) / 32, lane = threadIdx.x % 32;
+  if (warp >= Ttok) return;
+  const long long v = keys[warp] / Ttok;
+  if (warp > 0 && keys[warp - 1] / Ttok == v) return;
+  float* out = dwte + v * h;
+  for (int j0 = warp; j0 < Ttok;) {
+    // this chunk of up to 32 segment members: lane i holds position of member j0 + i
+    const int j = j0 + lane;
+    const long long kj = j < Ttok ? keys[j] : LLONG_MAX;
+    const bool in = j < Ttok && kj / Ttok == v;
+    const unsigned m = __ballot_sync(0xffffffffu, in);
+    const int cnt = __popc(~m) ? __ffs(~m) - 1 : 32;   // members are a prefix of the chunk
+    const int pos = in ? static_cast<int>(kj % Ttok) : 0;
+    for (int c8 = lane; c8 < h / 8; c8 += 32) {
+      float acc[8];
+      const float4 o0 = *reinterpret_cast<const float4*>(out + c8 * 8);
+      const float4 o1 = *reinterpret_cast<const float4*>(out + c8 * 8 + 4);
+      float sum[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+      for (int i = 0; i < cnt; ++i) {
+        const int p = __shfl_sync(0xffffffffu, pos, i);
+        const uint4 u = *reinterpret_cast<const uint4*>(dH + static_cast<long>(p) * h + c8 * 8);
+        const __nv_bfloat162* hv = reinterpret_cast<const __nv_bfloat162*>(&u);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const float2 f = __bfloat1622float2(hv[e]);
+          sum[2 * e] += f.x;
+          sum[2 * e + 1] += f.y;
+        }
+      }
+      acc[0] = o0.x + sum[0]; acc[1] = o0.y + sum[1]; acc[2] = o0.z + sum[2]; acc[3] = o0.w + sum[3];
+      acc[4] = o1.x + sum[4]; acc[5] = o1.y + sum[5]; acc[6] = o1.z + sum[6]; acc[7] = o1.w + sum[7];
+      *reinterpret_cast<float4*>(out + c8 * 8) = make_float4(acc[0], acc[1], acc[2], acc[3]);
+      *reinterpret_cast<float4*>(out + c8 * 8 + 4) = make_float4(acc[4], acc[5], acc[6], acc[7]);
+    }
+    if (cnt < 32) break;
+    j0 += 32;
+  }
+}
+
 template <class T>
 __global__ void embed_pos_bwd_k(const T* dH, int B, int s, int h, float* dwpe) {
   const long n = static_cast<long>(s) * h;
@@ -1060,8 +1105,18 @@ void embed_bwd(const int32_t* tok, int ld_tok, int B, int s, const T* dH, int h,
   if (!attr) { cudaFuncSetAttribute(embed_sort_k, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024); attr = true; }
   embed_sort_k<<<1, 1024, smem, st>>>(tok, ld_tok, B, s, keys, np2);
   note_launch();
-  embed_segsum_k<T><<<cdiv(static_cast<long>(Ttok) * 32, 256), 256, 0, st>>>(keys, Ttok, dH, h, dwte);
-  note_launch();
+  if constexpr (std::is_same<T, __nv_bfloat16>::value) {
+    if (h % 8 == 0 && (reinterpret_cast<uintptr_t>(dH) & 15) == 0 && (reinterpret_cast<uintptr_t>(dwte) & 15) == 0) {
+      embed_segsum_v8_k<<<cdiv(static_cast<long>(Ttok) * 32, 256), 256, 0, st>>>(keys, Ttok, dH, h, dwte);
+      note_launch();
+    } else {
+      embed_segsum_k<T><<<cdiv(static_cast<long>(Ttok) * 32, 256), 256, 0, st>>>(keys, Ttok, dH, h, dwte);
+      note_launch();
+    }
+  } else {
+    embed_segsum_k<T><<<cdiv(static_cast<long>(Ttok) * 32, 256), 256, 0, st>>>(keys, Ttok, dH, h, dwte);
+    note_launch();
+  }
   if (dwpe) { embed_pos_bwd_k<T><<<grid_for(static_cast<long>(s) * h), 256, 0, st>>>(dH, B, s, h, dwpe); note_launch(); }
 }
 
