@@ -175,6 +175,28 @@ __global__ void embed_pos_bwd_k(const T* dH, int B, int s, int h, float* dwpe) {
   }
 }
 
+// bf16, h % 8 == 0: dwpe[t] += sum_b dH[b, t] in 16-byte chunks (same order: b ascending), 32-bit index math
+__global__ void embed_pos_bwd_v8_k(const __nv_bfloat16* dH, int B, int s, int h8, float* dwpe) {
+  const int n8 = s * h8;
+  for (int i = blockIdx.x * blockDim.x + threadIdx.x; i < n8; i += gridDim.x * blockDim.x) {
+    float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+    for (int b = 0; b < B; ++b) {
+      const uint4 u = reinterpret_cast<const uint4*>(dH)[static_cast<long>(b) * n8 + i];
+      const __nv_bfloat162* hv = reinterpret_cast<const __nv_bfloat162*>(&u);
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const float2 f = __bfloat1622float2(hv[e]);
+        acc[2 * e] += f.x;
+        acc[2 * e + 1] += f.y;
+      }
+    }
+    float4* o = reinterpret_cast<float4*>(dwpe) + 2 * static_cast<long>(i);
+    const float4 a = o[0], c = o[1];
+    o[0] = make_float4(a.x + acc[0], a.y + acc[1], a.z + acc[2], a.w + acc[3]);
+    o[1] = make_float4(c.x + acc[4], c.y + acc[5], c.z + acc[6], c.w + acc[7]);
+  }
+}
+
 // ---------------------------------------------------------------------- norms
 template <class T, bool RMS>
 __global__ void norm_fwd_k(const T* x, const float* g, const float* b, T* y, float* stats, int rows, int n, float eps) {
@@ -1153,7 +1175,17 @@ void embed_bwd(const int32_t* tok, int ld_tok, int B, int s, const T* dH, int h,
     embed_segsum_k<T><<<cdiv(static_cast<long>(Ttok) * 32, 256), 256, 0, st>>>(keys, Ttok, dH, h, dwte);
     note_launch();
   }
-  if (dwpe) { embed_pos_bwd_k<T><<<grid_for(static_cast<long>(s) * h), 256, 0, st>>>(dH, B, s, h, dwpe); note_launch(); }
+  if (dwpe) {
+    bool done = false;
+    if constexpr (std::is_same<T, __nv_bfloat16>::value) {
+      if (h % 8 == 0 && (reinterpret_cast<uintptr_t>(dH) & 15) == 0 && (reinterpret_cast<uintptr_t>(dwpe) & 15) == 0) {
+        embed_pos_bwd_v8_k<<<grid_for(static_cast<long>(s) * (h / 8)), 256, 0, st>>>(dH, B, s, h / 8, dwpe);
+        done = true;
+      }
+    }
+    if (!done) embed_pos_bwd_k<T><<<grid_for(static_cast<long>(s) * h), 256, 0, st>>>(dH, B, s, h, dwpe);
+    note_launch();
+  }
 }
 
 bool norm_apply(const __nv_bfloat16* x, const float* g, const float* b, const float* stats, __nv_bfloat16* y, int rows,
