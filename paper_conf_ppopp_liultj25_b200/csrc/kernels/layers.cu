@@ -505,15 +505,30 @@ __global__ void __launch_bounds__(256) colsum_partial_v2_k(const __nv_bfloat16* 
   const int r0 = static_cast<int>(static_cast<long>(rows) * blk / nblk);
   const int r1 = static_cast<int>(static_cast<long>(rows) * (blk + 1) / nblk);
   float s0[8] = {0, 0, 0, 0, 0, 0, 0, 0}, s1[8] = {0, 0, 0, 0, 0, 0, 0, 0};
-  if (c8 < n) {
+  if (c8 < n && mode == 0) {
+    // plain column sums (a bias gradient): 4 rows' 16-byte loads in flight per warp
+    int r = r0 + warp;
+    for (; r + 24 < r1; r += 32) {
+      uint4 u[4];
+#pragma unroll
+      for (int q = 0; q < 4; ++q) u[q] = *reinterpret_cast<const uint4*>(a + static_cast<long>(r + 8 * q) * lda + c8);
+#pragma unroll
+      for (int q = 0; q < 4; ++q) {
+        const __nv_bfloat16* hq = reinterpret_cast<const __nv_bfloat16*>(&u[q]);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) s0[j] += __bfloat162float(hq[j]);
+      }
+    }
+    for (; r < r1; r += 8) {
+      const uint4 ua = *reinterpret_cast<const uint4*>(a + static_cast<long>(r) * lda + c8);
+      const __nv_bfloat16* ha = reinterpret_cast<const __nv_bfloat16*>(&ua);
+#pragma unroll
+      for (int j = 0; j < 8; ++j) s0[j] += __bfloat162float(ha[j]);
+    }
+  } else if (c8 < n) {
     for (int r = r0 + warp; r < r1; r += 8) {
       const uint4 ua = *reinterpret_cast<const uint4*>(a + static_cast<long>(r) * lda + c8);
       const __nv_bfloat16* ha = reinterpret_cast<const __nv_bfloat16*>(&ua);
-      if (mode == 0) {
-#pragma unroll
-        for (int j = 0; j < 8; ++j) s0[j] += __bfloat162float(ha[j]);
-        continue;
-      }
       const uint4 ux = *reinterpret_cast<const uint4*>(x + static_cast<long>(r) * n + c8);
       const __nv_bfloat16* hx = reinterpret_cast<const __nv_bfloat16*>(&ux);
       const float mu = stats[2 * r], rs = stats[2 * r + 1];
@@ -539,16 +554,38 @@ __global__ void __launch_bounds__(256) colsum_partial_v2_k(const __nv_bfloat16* 
   }
 }
 
-__global__ void colsum_final_k(const float* partial, int nblk, int n, int mode, float* out0, float* out1) {
-  const int c = blockIdx.x * blockDim.x + threadIdx.x;
-  if (c >= n) return;
-  float s0 = 0.f, s1 = 0.f;
-  for (int b = 0; b < nblk; ++b) {
-    s0 += partial[static_cast<long>(b) * n + c];
-    if (mode == 1) s1 += partial[static_cast<long>(nblk + b) * n + c];
+// out_k[c] += sum_b partial[k * nblk + b][c] for k = blockIdx.y (a null out_k: nothing). Block =
+// 32 columns x 16 warps: warp w sums row blocks w, w + 16, ... with 4 loads in flight, then the
+// 16 warp sums are added in fixed order (deterministic). The grid spans n / 32 x arrays CTAs, so a
+// [256][8192] partial (fc1.b) is read by 256 CTAs instead of 32 threads-per-column chains.
+__global__ void __launch_bounds__(512) colsum_reduce_k(const float* __restrict__ partial, int nblk, int n,
+                                                       float* out0, float* out1, float* out2) {
+  __shared__ float red[16][33];
+  const int k = blockIdx.y;
+  float* o = k == 0 ? out0 : (k == 1 ? out1 : out2);
+  if (!o) return;   // uniform over the block
+  const int w = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int c = blockIdx.x * 32 + lane;
+  float a0 = 0.f, a1 = 0.f, a2 = 0.f, a3 = 0.f;
+  if (c < n) {
+    const float* p = partial + static_cast<long>(k) * nblk * n + c;
+    int b = w;
+    for (; b + 48 < nblk; b += 64) {
+      a0 += p[static_cast<long>(b) * n];
+      a1 += p[static_cast<long>(b + 16) * n];
+      a2 += p[static_cast<long>(b + 32) * n];
+      a3 += p[static_cast<long>(b + 48) * n];
+    }
+    for (; b < nblk; b += 16) a0 += p[static_cast<long>(b) * n];
   }
-  out0[c] += s0;
-  if (mode == 1) out1[c] += s1;
+  red[w][lane] = (a0 + a1) + (a2 + a3);
+  __syncthreads();
+  if (w == 0 && c < n) {
+    float t = 0.f;
+#pragma unroll
+    for (int i = 0; i < 16; ++i) t += red[i][lane];
+    o[c] += t;
+  }
 }
 
 // Block-per-row-tile norm backward (bf16, n = 8 * VPT * nthreads, nthreads % 32 == 0). Thread t owns
@@ -1257,10 +1294,14 @@ void norm_bwd_dx(const T* dy, const T* x, const float* stats, const float* g, co
   norm_bwd_dx_k<T><<<cdiv(rows, 8), 256, 0, st>>>(dy, x, stats, g, dres, dx, rows, n, rms);
   note_launch();
 }
+void colsum_reduce(const float* partial, int nblk, int n, float* out0, float* out1, float* out2, cudaStream_t st) {
+  const int arrays = out2 ? 3 : (out1 ? 2 : 1);
+  colsum_reduce_k<<<dim3(cdiv(n, 32), arrays), 512, 0, st>>>(partial, nblk, n, out0, out1, out2);
+  note_launch();
+}
 void colsum_finish(const float* partial, int nblk, int n, float* out, cudaStream_t st) {
   KScope ks_(K_COLSUM, st);
-  colsum_final_k<<<cdiv(n, 256), 256, 0, st>>>(partial, nblk, n, 0, out, nullptr);
-  note_launch();
+  colsum_reduce(partial, nblk, n, out, nullptr, nullptr, st);
 }
 
 template <class T>
@@ -1279,16 +1320,14 @@ void colsum(const T* a, const T* x, const float* stats, int rows, int n, int lda
       dim3 grid(cb, nblk);
       colsum_partial_v2_k<<<grid, 256, 0, st>>>(a, x, stats, rows, n, lda, mode == 2 ? 1 : mode, partial, nblk);
       note_launch();
-      colsum_final_k<<<cdiv(n, 256), 256, 0, st>>>(partial, nblk, n, mode == 2 ? 0 : mode, out0, out1);
-      note_launch();
+      colsum_reduce(partial, nblk, n, out0, mode == 1 ? out1 : nullptr, nullptr, st);
       return;
     }
   }
   dim3 grid(cdiv(n, 256), nblk);
   colsum_partial_k<T><<<grid, 256, 0, st>>>(a, x, stats, rows, n, lda, mode == 2 ? 1 : mode, partial, nblk);
   note_launch();
-  colsum_final_k<<<cdiv(n, 256), 256, 0, st>>>(partial, nblk, n, mode == 2 ? 0 : mode, out0, out1);
-  note_launch();
+  colsum_reduce(partial, nblk, n, out0, mode == 1 ? out1 : nullptr, nullptr, st);
 }
 
 template <class T>

@@ -48,6 +48,8 @@ bool softmax_ce_fast(const float* logits, const int32_t* tok, int ld_tok, int s,
 // out[c] += sum_b partial[b][c] over nblk row blocks (fixed order): the second pass of column sums
 // whose partials a GEMM epilogue produced (GemmEpilogue::colsum_part)
 void colsum_finish(const float* partial, int nblk, int n, float* out, cudaStream_t st);
+// out_k[c] += sum_b partial[k * nblk + b][c], k = 0..2 (null outputs skipped; no stream scope)
+void colsum_reduce(const float* partial, int nblk, int n, float* out0, float* out1, float* out2, cudaStream_t st);
 template <class T> void colsum(const T* a, const T* x, const float* stats, int rows, int n, int lda, int mode,
                                float* out0, float* out1, float* partial, cudaStream_t st);
 

@@ -429,46 +429,6 @@ __global__ void __launch_bounds__(640) norm_bwd_pipe_k(const bf16* __restrict__ 
   }
 }
 
-// out_k[c] += sum_b partial[k][b][c] (k = 0..2, null outputs skipped). Block = 32 columns x 32 warps:
-// warp w sums partial rows w, w + 32, ... (4 loads in flight per array), then the warp sums are
-// added in fixed order (deterministic).
-__global__ void __launch_bounds__(1024) colsum_final_wide_k(const float* __restrict__ partial, int nblk, int n,
-                                                            float* out0, float* out1, float* out2) {
-  __shared__ float red[3][32][33];
-  const int w = threadIdx.x / 32, lane = threadIdx.x % 32;
-  const int c = blockIdx.x * 32 + lane;
-  float s[3] = {0.f, 0.f, 0.f};
-  if (c < n) {
-    const float* p[3] = {partial, out1 ? partial + static_cast<long>(nblk) * n : nullptr,
-                         out2 ? partial + static_cast<long>(2 * nblk) * n : nullptr};
-#pragma unroll
-    for (int k = 0; k < 3; ++k) {
-      if (!p[k]) continue;
-      float a0 = 0.f, a1 = 0.f, a2 = 0.f, a3 = 0.f;
-      int bb = w;
-      for (; bb + 96 < nblk; bb += 128) {
-        a0 += p[k][static_cast<long>(bb) * n + c];
-        a1 += p[k][static_cast<long>(bb + 32) * n + c];
-        a2 += p[k][static_cast<long>(bb + 64) * n + c];
-        a3 += p[k][static_cast<long>(bb + 96) * n + c];
-      }
-      for (; bb < nblk; bb += 32) a0 += p[k][static_cast<long>(bb) * n + c];
-      s[k] = (a0 + a1) + (a2 + a3);
-    }
-  }
-#pragma unroll
-  for (int k = 0; k < 3; ++k) red[k][w][lane] = s[k];
-  __syncthreads();
-  if (w < 3 && c < n) {
-    float* o = w == 0 ? out0 : (w == 1 ? out1 : out2);
-    if (o) {
-      float tt = 0.f;
-      for (int i = 0; i < 32; ++i) tt += red[w][i][lane];
-      o[c] += tt;
-    }
-  }
-}
-
 // ---------------------------------------------------------------- softmax-CE
 // One CTA (512 threads) per row; the whole fp32 row is held in registers (thread t: float4 chunks
 // t, t + 512, ...), so the logits are read from HBM exactly once: block max, then p = 2^((z-M)log2e)
@@ -655,8 +615,7 @@ bool norm_bwd_pipe_v(const bf16* dy, const bf16* x, const float* stats, const fl
                                                      nblk, dsum ? 1 : 0, S, max_range);
   note_launch();
   if (dg) {
-    colsum_final_wide_k<<<cdivl(n, 32), 1024, 0, st>>>(partial, nblk, n, dg, rms ? nullptr : db, dsum);
-    note_launch();
+    colsum_reduce(partial, nblk, n, dg, rms ? nullptr : db, dsum, st);
   }
   return true;
 }
