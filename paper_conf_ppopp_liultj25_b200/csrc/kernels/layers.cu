@@ -506,20 +506,8 @@ __global__ void __launch_bounds__(256) colsum_partial_v2_k(const __nv_bfloat16* 
   const int r1 = static_cast<int>(static_cast<long>(rows) * (blk + 1) / nblk);
   float s0[8] = {0, 0, 0, 0, 0, 0, 0, 0}, s1[8] = {0, 0, 0, 0, 0, 0, 0, 0};
   if (c8 < n && mode == 0) {
-    // plain column sums (a bias gradient): 4 rows' 16-byte loads in flight per warp
-    int r = r0 + warp;
-    for (; r + 24 < r1; r += 32) {
-      uint4 u[4];
-#pragma unroll
-      for (int q = 0; q < 4; ++q) u[q] = *reinterpret_cast<const uint4*>(a + static_cast<long>(r + 8 * q) * lda + c8);
-#pragma unroll
-      for (int q = 0; q < 4; ++q) {
-        const __nv_bfloat16* hq = reinterpret_cast<const __nv_bfloat16*>(&u[q]);
-#pragma unroll
-        for (int j = 0; j < 8; ++j) s0[j] += __bfloat162float(hq[j]);
-      }
-    }
-    for (; r < r1; r += 8) {
+    // plain column sums (a bias gradient)
+    for (int r = r0 + warp; r < r1; r += 8) {
       const uint4 ua = *reinterpret_cast<const uint4*>(a + static_cast<long>(r) * lda + c8);
       const __nv_bfloat16* ha = reinterpret_cast<const __nv_bfloat16*>(&ua);
 #pragma unroll
@@ -1313,7 +1301,8 @@ void colsum(const T* a, const T* x, const float* stats, int rows, int n, int lda
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
     if (n % 8 == 0 && lda % 8 == 0) {
       const int cb = cdiv(n, 256);
-      int rb = (2 * 148 + cb - 1) / cb;
+      // ~8 CTAs (64 warps) per SM so enough 16-byte loads are in flight; the partial stays small
+      int rb = (8 * device_sms() + cb - 1) / cb;
       rb = rb < 1 ? 1 : (rb > 128 ? 128 : rb);
       rb = rb > rows ? rows : rb;
       nblk = rb;
