@@ -140,6 +140,14 @@ FULL = [
     ("llama2-7b-s2048", synth.with_(synth.LLAMA2_7B, n_layers=2, micro_batch=1, seq_len=2048), "1f1b", 2, 2, 1,
      4e-2, 6e-2),
     ("gpt3-2.7b-chimera", synth.with_(synth.GPT3_2P7B, n_layers=2, micro_batch=1), "chimera", 2, 2, 1, 2e-2, 5e-2),
+    # Interleave v = 2 at GPT-3 1.3B width (4 layers = 2 stages x 2 chunks; observed l2 0.93%, inf 0.86%)
+    ("gpt3-1.3b-interleave", synth.with_(synth.GPT3_1P3B, n_layers=4, micro_batch=1), "interleave", 2, 2, 2,
+     2e-2, 5e-2),
+    # LLaMA2-13B width (h 5120, 40 heads, f 13824; cfg 5's shapes at s 1024): bf16 storage alone moves
+    # the fp32 definition by 2.91% l2 (h1.n1.g) / 2.81% inf (h1.qkv.w) (tools/bf16_storage_error.py
+    # lin,norm,attn 1024 13b); GPU observed 3.42% / 3.74%; bound ~1.7x the floor (A19)
+    ("llama2-13b-s1024", synth.with_(synth.LLAMA2_13B, n_layers=2, micro_batch=1, seq_len=1024), "1f1b", 2, 2, 1,
+     5e-2, 6e-2),
 ]
 
 

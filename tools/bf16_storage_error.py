@@ -9,7 +9,9 @@ def rb(x):
     return synth.round_to_bf16(np.asarray(x, np.float32))
 
 which = set(sys.argv[1].split(",")) if len(sys.argv) > 1 else set()
-cfg = synth.with_(synth.LLAMA2_7B, n_layers=2, micro_batch=1, seq_len=256)
+seq = int(sys.argv[2]) if len(sys.argv) > 2 else 256
+base = {"7b": synth.LLAMA2_7B, "13b": synth.LLAMA2_13B}[sys.argv[3] if len(sys.argv) > 3 else "7b"]
+cfg = synth.with_(base, n_layers=2, micro_batch=1, seq_len=seq)
 P = {k: (synth.round_to_bf16(v) if v.ndim == 2 else v) for k, v in synth.make_weights(cfg).items()}
 toks = synth.make_tokens(cfg, 2)
 l0, g0 = om.step(cfg, P, toks, 2, np.float32)
@@ -29,4 +31,5 @@ if "attn" in which:
     om.attention_bwd = ab
 l1, g1 = om.step(cfg, P, toks, 2, np.float32)
 worst = max((float(np.abs(g1[k]-g0[k]).max()/np.abs(g0[k]).max()), k) for k in g0)
-print(sorted(which), "loss rel", abs(l1-l0)/l0, "worst", worst)
+worst_l2 = max((float(np.linalg.norm(g1[k]-g0[k])/np.linalg.norm(g0[k])), k) for k in g0)
+print(sorted(which), cfg.hidden, seq, "loss rel", abs(l1-l0)/l0, "worst inf", worst, "worst l2", worst_l2)
