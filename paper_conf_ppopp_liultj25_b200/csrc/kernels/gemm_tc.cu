@@ -203,10 +203,25 @@ __device__ __forceinline__ uint8_t* sw128(uint8_t* sw, int r, int j) { return sw
 // read-back expects: no registers are held while it is in flight (a register prefetch pushed the
 // epilogue into spills). fp32 outputs (EPI 2) transpose through all 4 KB, so they load on demand.
 struct EpiPrefetch { uint8_t* buf; };   // = sw + 2048
+// EF (MARIO_EPI_EF, the GeLU' epilogue only): its aux input Z and its outputs dZ and G are each
+// 134 MB at cfg 2, streamed once and larger than L2, so their lines carry evict_first and stop
+// pushing the operand panels the next waves re-read out of L2.
+// Off by default: DRAM reads of the fc2 dgrad 366 -> 284 MB per launch, but 252 -> 257 us cold and
+// whole-step A/B neutral (tools/gpu91.sh): the epilogue's issue, not the operand re-reads, paces it.
+#ifndef MARIO_EPI_EF
+#define MARIO_EPI_EF 0
+#endif
+template <bool EF = false>
 __device__ __forceinline__ void cp_async16(void* dst, const void* src, bool valid) {
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" :: "r"(smem_u32(dst)), "l"(src), "r"(valid ? 16 : 0)
-               : "memory");
+  if constexpr (EF) {
+    asm volatile("cp.async.cg.shared.global.L2::cache_hint [%0], [%1], 16, %2, %3;"
+                 :: "r"(smem_u32(dst)), "l"(src), "r"(valid ? 16 : 0), "l"(l2_policy_evict_first()) : "memory");
+  } else {
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" :: "r"(smem_u32(dst)), "l"(src), "r"(valid ? 16 : 0)
+                 : "memory");
+  }
 }
+template <bool EF = false>
 __device__ __forceinline__ void epi_prefetch(const GemmEpilogue& ep, bool vec_ok, int rbase, int lane, int col0, int M,
                                              int N, EpiPrefetch& pf) {
   if (col0 < 0 || col0 >= N || !vec_ok || col0 + 32 > N) return;
@@ -217,7 +232,7 @@ __device__ __forceinline__ void epi_prefetch(const GemmEpilogue& ep, bool vec_ok
   for (int it = 0; it < 4; ++it) {
     const int rr = it * 8 + lane / 4, ch = lane % 4;
     const bool ok = rbase + rr < M;   // rows >= M read as 0 (src-size 0)
-    cp_async16(sw64(pf.buf, rr, ch), base + static_cast<size_t>(ok ? rbase + rr : rbase) * ld + col0 + ch * 8, ok);
+    cp_async16<EF>(sw64(pf.buf, rr, ch), base + static_cast<size_t>(ok ? rbase + rr : rbase) * ld + col0 + ch * 8, ok);
   }
   asm volatile("cp.async.commit_group;" ::: "memory");
 }
@@ -239,6 +254,7 @@ __device__ __forceinline__ void load_block_bf16(const EpiPrefetch& pf, int lane,
   __syncwarp();
 }
 // each lane's row of 32 values -> bf16 -> coalesced store of the block (rows >= M skipped)
+template <bool EF = false>
 __device__ __forceinline__ void store_block_bf16(__nv_bfloat16* base, int ld, int rbase, int col0, int M, int lane,
                                                  uint8_t* sw, const float (&v)[32]) {
 #pragma unroll
@@ -254,7 +270,15 @@ __device__ __forceinline__ void store_block_bf16(__nv_bfloat16* base, int ld, in
   for (int it = 0; it < 4; ++it) {
     const int rr = it * 8 + lane / 4, ch = lane % 4;
     const uint4 u = lds128u(sw64(sw, rr, ch));
-    if (rbase + rr < M) *reinterpret_cast<uint4*>(base + static_cast<size_t>(rbase + rr) * ld + col0 + ch * 8) = u;
+    if (rbase + rr < M) {
+      __nv_bfloat16* d = base + static_cast<size_t>(rbase + rr) * ld + col0 + ch * 8;
+      if constexpr (EF) {
+        asm volatile("st.global.L2::cache_hint.v4.b32 [%0], {%1, %2, %3, %4}, %5;"
+                     :: "l"(d), "r"(u.x), "r"(u.y), "r"(u.z), "r"(u.w), "l"(l2_policy_evict_first()) : "memory");
+      } else {
+        *reinterpret_cast<uint4*>(d) = u;
+      }
+    }
   }
   __syncwarp();
 }
@@ -285,7 +309,7 @@ __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool
   float z[32];
   if constexpr (EPI == 1) {   // GeLU backward: D = acc * gelu'(Z)
     load_block_bf16(pf, lane, z);
-    if (MARIO_EPI_PREFETCH) epi_prefetch(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
+    if (MARIO_EPI_PREFETCH) epi_prefetch<MARIO_EPI_EF != 0>(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
 #pragma unroll
     for (int j = 0; j < 32; ++j) v[j] *= gelu_tanh_grad_f(z[j]);
   }
@@ -330,7 +354,7 @@ __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool
     }
     __syncwarp();
   } else {
-    store_block_bf16(ep.d_bf16, ep.ldd, rbase, col0, M, lane, sw, v);
+    store_block_bf16<EPI == 1 && MARIO_EPI_EF != 0>(ep.d_bf16, ep.ldd, rbase, col0, M, lane, sw, v);
     if (ep.colsum_part) {
       // lane c: column col0 + c of the 32 bf16 rows just staged in sw, summed in row order
       float cs = 0.f;
@@ -346,7 +370,7 @@ __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool
       const bool g_aux = EPI == 1 && ep.d2_from_aux;
 #pragma unroll
       for (int j = 0; j < 32; ++j) v[j] = gelu_tanh_f(g_aux ? z[j] : v[j]);
-      store_block_bf16(ep.d2_bf16, ep.ldd, rbase, col0, M, lane, sw, v);
+      store_block_bf16<EPI == 1 && MARIO_EPI_EF != 0>(ep.d2_bf16, ep.ldd, rbase, col0, M, lane, sw, v);
     }
   }
 }
@@ -686,7 +710,7 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
       const int m0 = tm * 256 + 128 * rank, n0 = tn * BNP;
       const int rbase = m0 + quarter * 32;
       EpiPrefetch pf{sw + 2048};
-      if (MARIO_EPI_PREFETCH && EPI != 2 && !(skon && u.kb0 != 0)) epi_prefetch(ep, vec_ok, rbase, lane, n0 + half * (BNP / 2), M, N, pf);
+      if (MARIO_EPI_PREFETCH && EPI != 2 && !(skon && u.kb0 != 0)) epi_prefetch<EPI == 1 && MARIO_EPI_EF != 0>(ep, vec_ok, rbase, lane, n0 + half * (BNP / 2), M, N, pf);
       if (SK && sk.sleep_ns) { while (!mbar_test(&tfull[acc], acc_ph)) __nanosleep(sk.sleep_ns); }
       else mbar_wait(&tfull[acc], acc_ph);
       tc_fence_after();
