@@ -286,7 +286,7 @@ class Context:
                 _check(L.mario_nccl_unique_id(uid))
             t = torch.tensor(list(uid.raw), dtype=torch.uint8)
             if dist.get_backend() == "nccl":      # NCCL process groups only move device tensors
-                t = t.to(torch.device("cuda", torch.cuda.current_device()))
+                t = t.to(torch.device("cuda", device))
             dist.broadcast(t, src=0)
             uid = C.create_string_buffer(bytes(t.cpu().tolist()), 128)
         _check(L.mario_init_dp(rank, world, device, dp, uid if world > 1 else None))

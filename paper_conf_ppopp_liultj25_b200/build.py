@@ -33,6 +33,7 @@ def _nccl_dirs():
 ARCH = ["-gencode", "arch=compute_100a,code=sm_100a"]
 COMMON = ["-O3", "-std=c++17", "-lineinfo", "-Xcompiler", "-fPIC", "--expt-relaxed-constexpr",
           "-Xptxas", "-v", "-DNDEBUG"]
+EXTRA = os.environ.get("NVCC_EXTRA", "").split()   # A/B switches, e.g. -DMARIO_EPI_EF=1
 
 
 def sources():
@@ -58,12 +59,15 @@ def build(verbose: bool = False, jobs: int = 8) -> str:
 
     def compile_one(src):
         rel = os.path.relpath(src, CSRC).replace(os.sep, "_")
-        digest = hashlib.sha1(open(src, "rb").read() + hd.encode()).hexdigest()[:12]
+        flags = [NVCC, *ARCH, *COMMON, *EXTRA, "-I", os.path.join(ROOT, "include"), "-I", CSRC, "-I", inc]
+        # the object name hashes the source, every header, the full nvcc command line and this
+        # script, so a flag or -D change (e.g. NVCC_EXTRA="-DMARIO_EPI_EF=1") never links stale objects
+        digest = hashlib.sha1(open(src, "rb").read() + hd.encode() + " ".join(flags).encode() +
+                              open(os.path.abspath(__file__), "rb").read()).hexdigest()[:12]
         obj = os.path.join(BUILD, f"{rel}.{digest}.o")
         log = obj + ".log"
         if not os.path.exists(obj):
-            cmd = [NVCC, *ARCH, *COMMON, "-I", os.path.join(ROOT, "include"), "-I", CSRC, "-I", inc,
-                   "-c", src, "-o", obj]
+            cmd = [*flags, "-c", src, "-o", obj]
             r = subprocess.run(cmd, capture_output=True, text=True)
             open(log, "w").write(r.stdout + r.stderr)
             if r.returncode != 0:

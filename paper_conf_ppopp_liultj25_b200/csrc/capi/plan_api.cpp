@@ -496,4 +496,8 @@ extern "C" int32_t mario_param_count(const struct mario_plan* P) {
   return P ? static_cast<int32_t>(P->param_names.size()) : 0;
 }
 
-extern "C" void mario_plan_destroy(struct mario_plan* P) { delete P; }
+extern "C" void mario_plan_destroy(struct mario_plan* P) {
+  if (!P) return;
+  mario::exec_forget_plan(P->serial);
+  delete P;
+}

@@ -77,9 +77,10 @@ struct Context {
   // CUDA-graph replay of whole iterations (single-process: S = 1 or loopback)
   bool graphs = false;
   cudaStream_t cap_stream = nullptr;
-  // key: (plan, weights, grads, workspace, kstats generation) — event-timed launches captured in a
-  // graph re-record their events on every replay, so a new timing set needs a new capture
-  using GKey = std::tuple<const void*, const void*, const void*, const void*, long long>;
+  // key: (plan serial, weights, grads, workspace, kstats generation) — event-timed launches captured
+  // in a graph re-record their events on every replay, so a new timing set needs a new capture.
+  // The serial is never reused (a freed plan's address can be), and mario_plan_destroy evicts.
+  using GKey = std::tuple<uint64_t, const void*, const void*, const void*, long long>;
   std::map<GKey, cudaGraphExec_t> graph_cache;
   std::map<GKey, long long> graph_kernels;
   std::set<GKey> graph_seen;
@@ -645,7 +646,7 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
   // with the same (plan, weights, grads, workspace) is captured into a CUDA graph, later calls
   // replay it (no per-kernel launch cost). Disabled while timing/kstats instrumentation is on.
   const bool graphable = g.graphs && g.world == 1 && !g.timing;
-  const auto gkey = std::make_tuple(static_cast<const void*>(&P), weights, static_cast<const void*>(grads),
+  const auto gkey = std::make_tuple(P.serial, weights, static_cast<const void*>(grads),
                                     static_cast<const void*>(workspace), kstats_generation());
   bool replayed = false, capturing = false;
   if (graphable) {
@@ -819,6 +820,18 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
 }
 
 }  // namespace
+
+void exec_forget_plan(uint64_t serial) {
+  for (auto it = g.graph_cache.begin(); it != g.graph_cache.end();) {
+    if (std::get<0>(it->first) == serial) { cudaGraphExecDestroy(it->second); it = g.graph_cache.erase(it); }
+    else ++it;
+  }
+  for (auto it = g.graph_kernels.begin(); it != g.graph_kernels.end();)
+    it = std::get<0>(it->first) == serial ? g.graph_kernels.erase(it) : std::next(it);
+  for (auto it = g.graph_seen.begin(); it != g.graph_seen.end();)
+    it = std::get<0>(*it) == serial ? g.graph_seen.erase(it) : std::next(it);
+}
+
 }  // namespace mario
 
 using namespace mario;

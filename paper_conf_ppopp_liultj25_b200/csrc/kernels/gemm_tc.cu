@@ -203,11 +203,12 @@ __device__ __forceinline__ uint8_t* sw128(uint8_t* sw, int r, int j) { return sw
 // read-back expects: no registers are held while it is in flight (a register prefetch pushed the
 // epilogue into spills). fp32 outputs (EPI 2) transpose through all 4 KB, so they load on demand.
 struct EpiPrefetch { uint8_t* buf; };   // = sw + 2048
-// EF (MARIO_EPI_EF, the GeLU' epilogue only): its aux input Z and its outputs dZ and G are each
-// 134 MB at cfg 2, streamed once and larger than L2, so their lines carry evict_first and stop
-// pushing the operand panels the next waves re-read out of L2.
-// Off by default: DRAM reads of the fc2 dgrad 366 -> 284 MB per launch, but 252 -> 257 us cold and
-// whole-step A/B neutral (tools/gpu91.sh): the epilogue's issue, not the operand re-reads, paces it.
+// EF (MARIO_EPI_EF, the GeLU' epilogue only): its aux input Z (134 MB at cfg 2, larger than L2) is
+// read exactly once, so its prefetch carries evict_first and stops pushing the operand panels the
+// next waves re-read out of L2. The outputs dZ and G are NOT streamed once (fc1 wgrad / fc1 dgrad
+// read dZ and fc2 wgrad reads G right after), so their stores keep the default policy.
+// Off by default: with the stores also evict_first, DRAM reads of the fc2 dgrad went 366 -> 284 MB
+// per launch but 252 -> 257 us cold, whole-step A/B neutral: the epilogue's issue paces it.
 #ifndef MARIO_EPI_EF
 #define MARIO_EPI_EF 0
 #endif
@@ -354,7 +355,7 @@ __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool
     }
     __syncwarp();
   } else {
-    store_block_bf16<EPI == 1 && MARIO_EPI_EF != 0>(ep.d_bf16, ep.ldd, rbase, col0, M, lane, sw, v);
+    store_block_bf16<false>(ep.d_bf16, ep.ldd, rbase, col0, M, lane, sw, v);
     if (ep.colsum_part) {
       // lane c: column col0 + c of the 32 bf16 rows just staged in sw, summed in row order
       float cs = 0.f;
@@ -370,7 +371,7 @@ __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool
       const bool g_aux = EPI == 1 && ep.d2_from_aux;
 #pragma unroll
       for (int j = 0; j < 32; ++j) v[j] = gelu_tanh_f(g_aux ? z[j] : v[j]);
-      store_block_bf16<EPI == 1 && MARIO_EPI_EF != 0>(ep.d2_bf16, ep.ldd, rbase, col0, M, lane, sw, v);
+      store_block_bf16<false>(ep.d2_bf16, ep.ldd, rbase, col0, M, lane, sw, v);
     }
   }
 }

@@ -105,6 +105,58 @@ __global__ void embed_sort_k(const int32_t* tok, int ld_tok, int B, int s, long 
   for (int i = threadIdx.x; i < T; i += blockDim.x) keys_out[i] = sk[i];
 }
 
+// Longer micro-batches (B*s > kSortChunk, e.g. s > 16384 at mbs 1): every CTA bitonic-sorts one
+// chunk of kSortChunk keys in shared memory, then merge passes double the sorted run length. Keys
+// are unique (the position is part of the key), so the order is fully determined: each element's
+// output index is its index in its own run plus the number of keys of the partner run that are
+// smaller (binary search), with no atomics.
+constexpr int kSortChunk = 16384;
+__global__ void embed_sort_chunk_k(const int32_t* tok, int ld_tok, int s, int Ttok, long long* keys_out) {
+  extern __shared__ long long sk[];
+  const int c0 = blockIdx.x * kSortChunk;
+  for (int i = threadIdx.x; i < kSortChunk; i += blockDim.x) {
+    const int g = c0 + i;
+    if (g < Ttok) {
+      const int b = g / s, t = g % s;
+      sk[i] = static_cast<long long>(tok[static_cast<long>(b) * ld_tok + t]) * Ttok + g;
+    } else {
+      sk[i] = LLONG_MAX;
+    }
+  }
+  __syncthreads();
+  for (int k = 2; k <= kSortChunk; k <<= 1) {
+    for (int j = k >> 1; j > 0; j >>= 1) {
+      for (int i = threadIdx.x; i < kSortChunk; i += blockDim.x) {
+        const int ixj = i ^ j;
+        if (ixj > i) {
+          const bool up = (i & k) == 0;
+          const long long a = sk[i], c = sk[ixj];
+          if ((a > c) == up) { sk[i] = c; sk[ixj] = a; }
+        }
+      }
+      __syncthreads();
+    }
+  }
+  for (int i = threadIdx.x; i < kSortChunk && c0 + i < Ttok; i += blockDim.x) keys_out[c0 + i] = sk[i];
+}
+
+__global__ void embed_merge_k(const long long* in, long long* out, int n, int width) {
+  const int i = blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  const int run = i / width, pair0 = (run & ~1) * width;
+  const bool left = (run & 1) == 0;
+  const int own0 = left ? pair0 : pair0 + width;
+  const int oth0 = left ? pair0 + width : pair0;
+  const int oth_n = max(0, min(width, n - oth0));
+  const long long k = in[i];
+  int lo = 0, hi = oth_n;   // number of partner keys < k
+  while (lo < hi) {
+    const int mid = (lo + hi) >> 1;
+    if (in[oth0 + mid] < k) lo = mid + 1; else hi = mid;
+  }
+  out[pair0 + (i - own0) + lo] = k;
+}
+
 template <class T>
 __global__ void embed_segsum_k(const long long* keys, int Ttok, const T* dH, int h, float* dwte) {
   const int warp = (blockIdx.x * blockDim.x + threadIdx.x) / 32, lane = threadIdx.x % 32;
@@ -1182,12 +1234,28 @@ void embed_bwd(const int32_t* tok, int ld_tok, int B, int s, const T* dH, int h,
   const int Ttok = B * s;
   int np2 = 1;
   while (np2 < Ttok) np2 <<= 1;
-  long long* keys = static_cast<long long*>(scratch);
-  const size_t smem = static_cast<size_t>(np2) * sizeof(long long);
+  long long* keys = static_cast<long long*>(scratch);   // scratch holds 2 * Ttok keys (layout.cpp)
   static bool attr = false;
-  if (!attr) { cudaFuncSetAttribute(embed_sort_k, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024); attr = true; }
-  embed_sort_k<<<1, 1024, smem, st>>>(tok, ld_tok, B, s, keys, np2);
-  note_launch();
+  if (!attr) {
+    cudaFuncSetAttribute(embed_sort_k, cudaFuncAttributeMaxDynamicSharedMemorySize, 227 * 1024);
+    cudaFuncSetAttribute(embed_sort_chunk_k, cudaFuncAttributeMaxDynamicSharedMemorySize, kSortChunk * 8);
+    attr = true;
+  }
+  if (np2 <= kSortChunk) {
+    embed_sort_k<<<1, 1024, static_cast<size_t>(np2) * sizeof(long long), st>>>(tok, ld_tok, B, s, keys, np2);
+    note_launch();
+  } else {
+    long long* buf[2] = {keys, keys + Ttok};
+    int cur = 0;
+    embed_sort_chunk_k<<<cdiv(Ttok, kSortChunk), 1024, kSortChunk * 8, st>>>(tok, ld_tok, s, Ttok, buf[0]);
+    note_launch();
+    for (int w = kSortChunk; w < Ttok; w *= 2) {
+      embed_merge_k<<<cdiv(Ttok, 256), 256, 0, st>>>(buf[cur], buf[cur ^ 1], Ttok, w);
+      note_launch();
+      cur ^= 1;
+    }
+    keys = buf[cur];
+  }
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
     if (h % 8 == 0 && (reinterpret_cast<uintptr_t>(dH) & 15) == 0 && (reinterpret_cast<uintptr_t>(dwte) & 15) == 0) {
       embed_segsum_v8_k<<<cdiv(static_cast<long>(Ttok) * 32, 256), 256, 0, st>>>(keys, Ttok, dH, h, dwte);

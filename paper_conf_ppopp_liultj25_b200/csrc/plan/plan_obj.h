@@ -1,5 +1,7 @@
 // The opaque mario_plan object (immutable after mario_plan returns).
 #pragma once
+#include <atomic>
+#include <cstdint>
 #include <string>
 #include <map>
 #include <vector>
@@ -7,7 +9,14 @@
 #include "model.h"
 #include "plan.h"
 
+inline uint64_t mario_next_plan_serial() {
+  static std::atomic<uint64_t> next{1};
+  return next.fetch_add(1);
+}
+
 struct mario_plan {
+  // never reused (unlike the object's address): keys the executor's CUDA-graph cache
+  const uint64_t serial = mario_next_plan_serial();
   mario_model model{};
   mario::plan::Pipe pp;
   int level = MARIO_LEVEL_MARIO;
@@ -46,3 +55,4 @@ struct mario_plan {
 };
 typedef struct mario_plan PlanObj;
 const std::vector<mario_commop>& comm_program_dp(const PlanObj& P, int dp, int rank);   // plan_api.cpp
+namespace mario { void exec_forget_plan(uint64_t serial); }   // executor.cu: drop cached graphs
