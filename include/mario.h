@@ -130,7 +130,8 @@ mario_status mario_plan_comm_ops_dp(const struct mario_plan* plan, int32_t dp, i
 /* Canonical text serialization (deterministic). If buf is NULL or cap too small, *needed
  * receives the size including the terminating NUL and MARIO_EINVAL is returned for cap>0. */
 mario_status mario_plan_serialize(const struct mario_plan* plan, char* buf, size_t cap, size_t* needed);
-/* Byte sizes of rank `rank`'s packed fp32 parameters (= grads) and required workspace. */
+/* Byte sizes of rank `rank`'s packed fp32 parameters (= grads) and required workspace.
+ * rank -1: loopback totals (all ranks concatenated); -2: emulated peer-transport totals. */
 mario_status mario_plan_rank_layout(const struct mario_plan* plan, int32_t rank, uint64_t* param_count,
                                     uint64_t* workspace_bytes);
 /* Packed parameter layout of `rank`: for each tensor j, its global name index (see
@@ -178,6 +179,22 @@ mario_status mario_init(int32_t rank, int32_t world, int32_t device, const void*
  * (ncclAvg) after the pipeline flush and the loss is the mean over all replicas' tokens.
  * mario_init(...) == mario_init_dp(..., dp = 1, ...). EINVAL if world % dp != 0. */
 mario_status mario_init_dp(int32_t rank, int32_t world, int32_t device, int32_t dp, const void* nccl_unique_id);
+/* Emulated pipeline over the PEER TRANSPORT: `world` pipeline ranks hosted by this process on one
+ * GPU, each with its own compute and receive streams; with sms_per_rank > 0 every rank's streams
+ * live in a green context owning a disjoint partition of that many SMs (the driver rounds to
+ * its granularity: multiples of 8 on sm_100), so the S stages run concurrently the way S GPUs do.
+ * The executor then follows the per-rank code path of the multi-process executor: each rank walks
+ * its own list; RA/RG are blocking receives implemented as a device-side wait on the
+ * sender's "ready" flag, a copy out of the sender's send slot and a "consumed" flag; SA/SG are
+ * buffered sends that raise the "ready" flag; a send slot is reused only after the
+ * receiver's "consumed" flag; tied-embedding / Chimera replica copies are summed by a
+ * reduce-scatter + all-gather over peer memory (reading A7). Buffers: mario_plan_rank_layout(-2)
+ * (all ranks' packed parameters / multi-process workspaces concatenated). Results are bitwise
+ * identical to loopback. EINVAL if the partitions do not fit or green contexts are unavailable;
+ * ESTATE if a context is already initialised. mario_run_iter then requires plan stages == world.
+ * mario_emulated_sms: SMs per rank partition (0 = unpartitioned), -1 if not emulated. */
+mario_status mario_init_emulated(int32_t world, int32_t device, int32_t sms_per_rank);
+int32_t mario_emulated_sms(void);
 /* One training iteration of `plan` on this rank (all ranks in loopback).
  *  weights : device, this rank's packed fp32 parameters (loopback: all ranks concatenated)
  *  tokens  : HOST int32 [N*mbs][s+1]; x = tokens[:, :s], y = tokens[:, 1:] (reading A4)

@@ -94,6 +94,8 @@ _lib.register("mario_tune", C.c_int32, [C.POINTER(CModel), C.c_int32, C.c_int32,
 _lib.register("mario_nccl_unique_id", C.c_int32, [C.c_void_p])
 _lib.register("mario_init", C.c_int32, [C.c_int32, C.c_int32, C.c_int32, C.c_void_p])
 _lib.register("mario_init_dp", C.c_int32, [C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_void_p])
+_lib.register("mario_init_emulated", C.c_int32, [C.c_int32, C.c_int32, C.c_int32])
+_lib.register("mario_emulated_sms", C.c_int32, [])
 _lib.register("mario_run_iter", C.c_int32, [_P, C.c_void_p, C.c_void_p, C.POINTER(C.c_float), C.c_void_p,
                                             C.c_void_p, C.c_void_p])
 _lib.register("mario_set_timing", C.c_int32, [C.c_int32])
@@ -237,10 +239,10 @@ class Plan:
 
 # ------------------------------------------------------------------------- executor
 def pack_params(plan: Plan, params: Dict[str, "object"], rank: int):
-    """Pack a {name: array} model into rank's fp32 buffer (rank=-1: loopback, all ranks
-    concatenated). Pure layout marshalling (offsets come from the library)."""
+    """Pack a {name: array} model into rank's fp32 buffer (rank=-1 loopback / -2 emulated ranks:
+    all ranks concatenated). Pure layout marshalling (offsets come from the library)."""
     import numpy as np
-    ranks = range(plan.S) if rank == -1 else [rank]
+    ranks = range(plan.S) if rank < 0 else [rank]
     bufs = []
     for r in ranks:
         total = plan.rank_layout(r)[0]
@@ -256,7 +258,7 @@ def unpack_params(plan: Plan, flat, rank: int) -> Dict[str, "object"]:
     import numpy as np
     shapes = {n: s for n, s in _shapes(plan)}
     out = {}
-    ranks = range(plan.S) if rank == -1 else [rank]
+    ranks = range(plan.S) if rank < 0 else [rank]
     base = 0
     for r in ranks:
         for name, off, cnt in plan.rank_params(r):
@@ -291,6 +293,17 @@ class Context:
             uid = C.create_string_buffer(bytes(t.cpu().tolist()), 128)
         _check(L.mario_init_dp(rank, world, device, dp, uid if world > 1 else None))
         self.rank, self.world, self.dp = rank, world, dp
+
+    @classmethod
+    def emulated(cls, world: int, device: int = 0, sms_per_rank: int = 0) -> "Context":
+        """mario_init_emulated: `world` pipeline ranks in this process on one GPU, each on its own
+        streams (and, with sms_per_rank > 0, its own green-context SM partition), exchanging
+        activations and gradients through the peer transport. Buffers: alloc_for(plan, -2)."""
+        self = cls.__new__(cls)
+        _check(_lib.lib().mario_init_emulated(world, device, sms_per_rank))
+        self.rank, self.world, self.dp = 0, world, 1
+        self.sms_per_rank = int(_lib.lib().mario_emulated_sms())
+        return self
 
     def run_iter(self, plan: Plan, weights, tokens, grads, workspace, stream=None) -> float:
         """weights/grads/workspace: device tensors (data_ptr used); tokens: host int32 array."""
@@ -337,9 +350,16 @@ def default_context(device: int = 0) -> "Context":
     return _DEFAULT_CTX[0]
 
 
+def close_default_context() -> None:
+    """Finalize the process's default context (the library holds one executor context per
+    process), e.g. before creating an emulated one."""
+    if _DEFAULT_CTX:
+        _DEFAULT_CTX.pop().close()
+
+
 def alloc_for(plan: Plan, rank: int, device="cuda"):
     """Allocate (weights, grads, workspace) device tensors sized from the plan (torch is
-    used only as the device allocator)."""
+    used only as the device allocator). rank -1: loopback, -2: emulated ranks (peer transport)."""
     import torch
     pc, ws = plan.rank_layout(rank)
     w = torch.zeros(pc, dtype=torch.float32, device=device)

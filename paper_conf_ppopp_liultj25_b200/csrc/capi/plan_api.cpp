@@ -96,16 +96,19 @@ void assign_slots_and_pools(PlanObj& P) {
     }
     P.pools_mp[d] = {ck.high, ac.high, sa.high, sg.high, rg.high};
   }
-  // loopback: send slots are held until the receiver copies them out
+  // send slots are held until the receiver copies them out (loopback) or has consumed the message
+  // (NCCL / peer transport): the slot of every message is fixed here, along the loopback order
   P.pools_lb = P.pools_mp;
+  P.sa_slot.assign(pp.S, {});
+  P.sg_slot.assign(pp.S, {});
   std::vector<SlotPool> lsa(pp.S), lsg(pp.S);
   std::map<std::tuple<int, int, int>, int> held_sa, held_sg;  // (sender dev, m, p) -> slot
   for (auto [d, i] : P.loopback_order) {
     const Instr& x = P.lists[d][i];
     const int k = pp.vstage(d, x.p);
     int sd, sp;
-    if ((x.op == FW || x.op == CFW) && k < K - 1) held_sa[{d, x.m, x.p}] = lsa[d].acquire();
-    if (x.op == BW && k > 0) held_sg[{d, x.m, x.p}] = lsg[d].acquire();
+    if ((x.op == FW || x.op == CFW) && k < K - 1) P.sa_slot[d][{x.m, x.p}] = held_sa[{d, x.m, x.p}] = lsa[d].acquire();
+    if (x.op == BW && k > 0) P.sg_slot[d][{x.m, x.p}] = held_sg[{d, x.m, x.p}] = lsg[d].acquire();
     if (x.op == RA) {
       find_inst(pp, d, x.m, x.p, FW, false, &sd, &sp);
       lsa[sd].release(held_sa[{sd, x.m, sp}]);
@@ -119,6 +122,7 @@ void assign_slots_and_pools(PlanObj& P) {
     P.pools_lb[d].send_act = lsa[d].high;
     P.pools_lb[d].send_grad = lsg[d].high;
   }
+  P.pools_mp = P.pools_lb;   // every executor uses the loopback-order slot assignment
 }
 
 void build_rank_params(PlanObj& P) {
@@ -462,9 +466,12 @@ extern "C" mario_status mario_plan_serialize(const struct mario_plan* P, char* b
 extern "C" mario_status mario_plan_rank_layout(const struct mario_plan* P, int32_t rank, uint64_t* param_count,
                                                uint64_t* workspace_bytes) {
   if (!P) return set_error(MARIO_EINVAL, "NULL plan");
-  if (rank == -1) {  // loopback: all ranks concatenated
+  if (rank == -1 || rank == -2) {  // loopback (-1) / emulated peer ranks (-2): all ranks concatenated
     uint64_t pc = 0, ws = 0;
-    for (int d = 0; d < P->pp.S; ++d) { pc += P->rank_params[d].total; ws += align_up(P->workspace_lb[d], 1 << 20); }
+    for (int d = 0; d < P->pp.S; ++d) {
+      pc += P->rank_params[d].total;
+      ws += align_up(rank == -1 ? P->workspace_lb[d] : P->workspace_mp[d], 1 << 20);
+    }
     if (param_count) *param_count = pc;
     if (workspace_bytes) *workspace_bytes = ws;
     return MARIO_OK;

@@ -13,6 +13,12 @@
 // every channel a FIFO, so any acyclic plan is deadlock-free.
 // Loopback (world == 1, multi-stage plan): every rank's list runs in this process on one GPU
 // in the simulator's round-robin order; RA/RG become device-to-device copies.
+// Peer transport (mario_init_emulated: S virtual ranks in one process, each on its own streams and,
+// optionally, its own SM partition of the GPU): the per-rank code path of the multi-process
+// executor (slot-reuse guards, blocking receives, pair gradient reductions) with the channel
+// implemented in peer memory instead of NCCL: a send is a flag the sender's stream writes after the
+// message is complete (P:222 buffered send); a receive is a stream wait on that flag, a copy out of
+// the sender's send slot and a "consumed" flag the sender's next use of the slot waits on.
 #include <cuda_runtime.h>
 #include <nccl.h>
 
@@ -20,6 +26,8 @@
 #include <cstdio>
 #include <cstring>
 #include <algorithm>
+#include <array>
+#include <initializer_list>
 #include <map>
 #include <set>
 #include <memory>
@@ -33,6 +41,7 @@
 #include "../kernels/layers.h"
 #include "../kernels/kstats.h"
 #include "arena.h"
+#include "drv.h"
 
 extern "C" long long mario_kernel_launches(void);
 
@@ -50,6 +59,12 @@ using plan::Instr;
   do {                                                                              \
     ncclResult_t r_ = (x);                                                          \
     if (r_ != ncclSuccess) throw NcclErr(std::string(#x) + ": " + ncclGetErrorString(r_)); \
+  } while (0)
+
+#define DRV(x)                                                                      \
+  do {                                                                              \
+    cudaError_t e_ = (x);                                                           \
+    if (e_ != cudaSuccess) throw CudaErr(std::string(#x) + ": stream memory operation failed"); \
   } while (0)
 
 struct CudaErr : std::runtime_error { using std::runtime_error::runtime_error; };
@@ -85,6 +100,14 @@ struct Context {
   std::map<GKey, long long> graph_kernels;
   std::set<GKey> graph_seen;
   bool sticky = false;
+  // peer transport, emulated pipeline (mario_init_emulated): `world` virtual ranks in this process
+  bool emulated = false;
+  int emu_sms = 0;                              // SMs of each rank's partition (0: unpartitioned)
+  std::vector<cudaStream_t> emu_st;             // per rank: compute stream
+  std::vector<std::array<cudaStream_t, 2>> emu_rx;   // per rank: receive streams (activation, gradient)
+  bool emu_green = false;                       // streams live in green contexts
+  uint32_t* flags = nullptr;                    // device flag block (reset every iteration)
+  size_t flags_cap = 0;
 };
 Context g;
 
@@ -106,6 +129,12 @@ struct Dev {
   std::vector<cudaEvent_t> ev_pool;
   size_t ev_next = 0;
   std::vector<std::pair<cudaEvent_t, cudaEvent_t>> timed;   // per compute instr
+  // peer transport: this rank's streams and the consumption flag guarding each send slot's reuse
+  cudaStream_t st = nullptr;
+  cudaStream_t rx[2] = {nullptr, nullptr};
+  int sms = 0;
+  std::vector<const uint32_t*> sa_guard, sg_guard;
+  std::vector<std::tuple<int, int, int>> sa_guard_key, sg_guard_key;   // the guarding message
 
   const mario_model& M() const { return P->model; }
   template <class U = uint8_t> U* at(size_t off) const { return reinterpret_cast<U*>(ws + off); }
@@ -128,9 +157,23 @@ template <class T>
 struct Exec {
   cudaStream_t st;
   bool loopback;
-  std::vector<std::unique_ptr<Dev<T>>> devs;   // loopback: all; otherwise one (this rank)
+  bool peer = false;                           // peer transport (emulated ranks, one per stream set)
+  std::vector<std::unique_ptr<Dev<T>>> devs;   // loopback / peer: all ranks; NCCL: one (this rank)
+  // peer: the flag block [ready | done][kind][receiving vstage][micro] + reduction flags, and
+  // where each message sits: (kind, receiving vstage, micro) -> (sender rank, send slot)
+  uint32_t* flags = nullptr;
+  int fK = 0, fN = 0;
+  std::map<std::tuple<int, int, int>, std::pair<int, int>> msg_slot;
+  // host walk state (peer): messages whose "ready" / "consumed" flag write is already enqueued. A
+  // flag wait is only ever enqueued after the write it waits for (like an event record before its
+  // wait): a wait enqueued first could sit in front of its own write if the driver maps the two
+  // streams onto one hardware queue, and deadlock.
+  std::set<std::tuple<int, int, int>> ready_walked, consumed_walked;
 
-  Dev<T>& dev(int d) { return loopback ? *devs[d] : *devs[0]; }
+  Dev<T>& dev(int d) { return (loopback || peer) ? *devs[d] : *devs[0]; }
+  uint32_t* flag_ready(int kind, int k, int m) { return flags + (static_cast<size_t>(kind) * fK + k) * fN + m; }
+  uint32_t* flag_done(int kind, int k, int m) { return flags + (static_cast<size_t>(2 + kind) * fK + k) * fN + m; }
+  uint32_t* flag_misc(size_t i) { return flags + static_cast<size_t>(4) * fK * fN + i; }
 
   // ---- weights --------------------------------------------------------------
   int tidx(Dev<T>& D, int p, const std::string& name) {
@@ -418,6 +461,7 @@ struct Exec {
 
   void run_instr(int d, const mario_instr& x) {
     Dev<T>& D = dev(d);
+    if (peer) { st = D.st; set_sm_budget(D.sms); }
     const mario_model& m = D.M();
     const int K = D.P->pp.K();
     const auto key = std::make_pair(x.micro, x.part);
@@ -428,9 +472,16 @@ struct Exec {
       case MARIO_OP_RC: {
         T* out = nullptr;
         if (x.op != MARIO_OP_RC && x.vstage < K - 1) {
-          int i = acquire(D.sa_used);
+          const int i = D.P->sa_slot[d].at(key);   // the plan's slot (loopback-order assignment)
+          if (D.sa_used.at(i)) throw std::runtime_error("send slot still held (planner/executor mismatch)");
+          D.sa_used[i] = true;
           D.sa_of[key] = i;
-          if (!loopback && D.sa_free_set[i]) CU(cudaStreamWaitEvent(st, D.sa_free[i], 0));
+          if (peer) {
+            if (D.sa_guard[i]) DRV(drv::wait_flag(st, D.sa_guard[i], 1));   // previous message consumed
+            msg_slot[{0, x.vstage + 1, x.micro}] = {d, i};
+          } else if (!loopback && D.sa_free_set[i]) {
+            CU(cudaStreamWaitEvent(st, D.sa_free[i], 0));
+          }
           out = send_slot(D, false, i);
         } else if (x.op == MARIO_OP_RC && x.vstage < K - 1) {
           out = D.template at<T>(D.a.cfw);   // RC's stage output is not needed: scratch
@@ -445,9 +496,16 @@ struct Exec {
         if (x.vstage < K - 1) dout = D.template at<T>(D.a.rg + static_cast<size_t>(D.rg_of[key]) * D.a.msg_stride);
         T* din = nullptr;
         if (x.vstage > 0) {
-          int i = acquire(D.sg_used);
+          const int i = D.P->sg_slot[d].at(key);
+          if (D.sg_used.at(i)) throw std::runtime_error("send slot still held (planner/executor mismatch)");
+          D.sg_used[i] = true;
           D.sg_of[key] = i;
-          if (!loopback && D.sg_free_set[i]) CU(cudaStreamWaitEvent(st, D.sg_free[i], 0));
+          if (peer) {
+            if (D.sg_guard[i]) DRV(drv::wait_flag(st, D.sg_guard[i], 1));
+            msg_slot[{1, x.vstage - 1, x.micro}] = {d, i};
+          } else if (!loopback && D.sg_free_set[i]) {
+            CU(cudaStreamWaitEvent(st, D.sg_free[i], 0));
+          }
           din = send_slot(D, true, i);
         }
         timed_begin(D);
@@ -467,6 +525,20 @@ struct Exec {
       case MARIO_OP_SG:
         // loopback: the receiver copies out of the held slot; NCCL: the send is issued by
         // issue_send() from the rank's comm program, in the receiver's order
+        if (peer) {
+          // buffered send at its list position: mark the message complete; the slot is
+          // free for this rank's next message once the receiver's "consumed" flag is up
+          const bool grad = x.op == MARIO_OP_SG;
+          auto& of = grad ? D.sg_of : D.sa_of;
+          const int i = of.at(key);
+          const int kd = grad ? x.vstage - 1 : x.vstage + 1;
+          DRV(drv::write_flag(st, flag_ready(grad, kd, x.micro), 1));
+          (grad ? D.sg_guard : D.sa_guard)[i] = flag_done(grad, kd, x.micro);
+          (grad ? D.sg_guard_key : D.sa_guard_key)[i] = std::make_tuple(grad ? 1 : 0, kd, x.micro);
+          (grad ? D.sg_used : D.sa_used)[i] = false;
+          of.erase(key);
+          ready_walked.insert(std::make_tuple(grad ? 1 : 0, kd, x.micro));
+        }
         break;
       case MARIO_OP_RA:
       case MARIO_OP_RG: {
@@ -479,7 +551,27 @@ struct Exec {
           D.rg_of[key] = i;
           dst = D.template at<T>(D.a.rg + static_cast<size_t>(i) * D.a.msg_stride);
         }
-        if (loopback) {
+        if (peer) {
+          // blocking receive: wait for the sender's flag, pull the message out of the
+          // sender's slot on this rank's receive stream, flag it consumed, then the compute stream
+          // waits for the copy at this list position
+          const int kind = grad ? 1 : 0;
+          const auto src = msg_slot.at({kind, x.vstage, x.micro});
+          Dev<T>& Sd = dev(src.first);
+          cudaStream_t rs = D.rx[kind];
+          if (!grad && D.ck_free_set[x.slot]) CU(cudaStreamWaitEvent(rs, D.ck_free[x.slot], 0));
+          if (grad) {
+            const int i = D.rg_of[key];
+            if (D.rg_free_set[i]) CU(cudaStreamWaitEvent(rs, D.rg_free[i], 0));
+          }
+          DRV(drv::wait_flag(rs, flag_ready(kind, x.vstage, x.micro), 1));
+          CU(cudaMemcpyAsync(dst, send_slot(Sd, grad, src.second), msg_bytes, cudaMemcpyDeviceToDevice, rs));
+          DRV(drv::write_flag(rs, flag_done(kind, x.vstage, x.micro), 1));
+          consumed_walked.insert(std::make_tuple(kind, x.vstage, x.micro));
+          cudaEvent_t e = D.event();
+          CU(cudaEventRecord(e, rs));
+          CU(cudaStreamWaitEvent(st, e, 0));
+        } else if (loopback) {
           Dev<T>& Sd = dev(x.peer);
           // the sender's part for this micro-batch: find via its held slots
           int sp = -1;
@@ -504,6 +596,27 @@ struct Exec {
         }
         break;
       }
+    }
+  }
+
+  // peer: may instruction x of rank d be enqueued now, i.e. is every flag it will wait on already
+  // written by enqueued work? (receives: the sender's "ready"; a send slot's reuse: the previous
+  // message's "consumed")
+  bool can_walk(int d, const mario_instr& x) {
+    Dev<T>& D = dev(d);
+    const int K = D.P->pp.K();
+    const auto key = std::make_pair(x.micro, x.part);
+    auto slot_ok = [&](int i, const std::vector<const uint32_t*>& guard,
+                       const std::vector<std::tuple<int, int, int>>& gkey) {
+      return !guard[i] || consumed_walked.count(gkey[i]) > 0;
+    };
+    switch (x.op) {
+      case MARIO_OP_RA: return ready_walked.count(std::make_tuple(0, x.vstage, x.micro)) > 0;
+      case MARIO_OP_RG: return ready_walked.count(std::make_tuple(1, x.vstage, x.micro)) > 0;
+      case MARIO_OP_FW:
+      case MARIO_OP_CFW: return x.vstage >= K - 1 || slot_ok(D.P->sa_slot[d].at(key), D.sa_guard, D.sa_guard_key);
+      case MARIO_OP_BW: return x.vstage == 0 || slot_ok(D.P->sg_slot[d].at(key), D.sg_guard, D.sg_guard_key);
+      default: return true;
     }
   }
 
@@ -595,24 +708,56 @@ void ensure_channels(const PlanObj& P) {
 template <class T>
 mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* tokens, float* loss, void* grads,
                         void* workspace, cudaStream_t st) {
-  const bool loopback = g.world == 1 && P.pp.S > 1;
-  if (!loopback && P.pp.S * g.dp != g.world) return set_error(MARIO_ESTATE, "plan stages * dp != world size");
+  const bool peer = g.emulated;
+  const bool loopback = !peer && g.world == 1 && P.pp.S > 1;
+  if (peer && P.pp.S != static_cast<int>(g.emu_st.size()))
+    return set_error(MARIO_ESTATE, "plan stages != emulated world size");
+  if (!loopback && !peer && P.pp.S * g.dp != g.world) return set_error(MARIO_ESTATE, "plan stages * dp != world size");
   const int me = g.rank % P.pp.S, off = g.rank - me;   // stage and the replica's rank offset
   const auto& prog = comm_program_dp(P, g.dp, g.rank);
   Exec<T> E;
   E.st = st;
   E.loopback = loopback;
+  E.peer = peer;
   const mario_model& m = P.model;
   const int S = P.pp.S;
   std::vector<int> my_devs;
-  if (loopback) for (int d = 0; d < S; ++d) my_devs.push_back(d);
+  if (loopback || peer) for (int d = 0; d < S; ++d) my_devs.push_back(d);
   else my_devs.push_back(me);
+  // peer: flag block = [ready | done][activation | gradient][K][N] + per-rank "backward done" + one
+  // "chunk summed" flag per (multi-copy parameter, copy)
+  std::map<int, std::vector<std::pair<int, int>>> copies;   // global param idx -> (dev, packed j)
+  for (int d = 0; d < S; ++d) {
+    const auto& rp = P.rank_params[d];
+    for (size_t j = 0; j < rp.idx.size(); ++j) copies[rp.idx[j]].push_back({d, static_cast<int>(j)});
+  }
+  size_t n_multi_flags = 0;
+  for (auto& kv : copies) if (kv.second.size() > 1) n_multi_flags += kv.second.size();
+  size_t flag_words = 0;
+  if (peer) {
+    E.fK = P.pp.K();
+    E.fN = P.pp.N;
+    flag_words = static_cast<size_t>(4) * E.fK * E.fN + S + n_multi_flags;
+    if (g.flags_cap < flag_words) {
+      if (g.flags) CU(cudaFree(g.flags));
+      g.flags = nullptr;
+      CU(cudaMalloc(&g.flags, flag_words * 4));
+      g.flags_cap = flag_words;
+    }
+    E.flags = g.flags;
+  }
   size_t wofs = 0, wsofs = 0;
   for (int d : my_devs) {
     auto D = std::make_unique<Dev<T>>();
     D->P = &P;
     D->d = d;
     const auto& pools = loopback ? P.pools_lb[d] : P.pools_mp[d];
+    if (peer) {
+      D->st = g.emu_st[d];
+      D->rx[0] = g.emu_rx[d][0];
+      D->rx[1] = g.emu_rx[d][1];
+      D->sms = g.emu_sms;
+    }
     D->a = make_arena(P, d, pools);
     D->ws = static_cast<uint8_t*>(workspace) + wsofs;
     D->w = static_cast<const float*>(weights) + wofs;
@@ -631,9 +776,16 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
     mk(D->sg_free, D->sg_free_set, D->sg_used.size());
     mk(D->rg_free, D->rg_free_set, D->rg_used.size());
     mk(D->ck_free, D->ck_free_set, std::max(1, pools.ckpt));
+    D->sa_guard.assign(D->sa_used.size(), nullptr);
+    D->sg_guard.assign(D->sg_used.size(), nullptr);
+    D->sa_guard_key.assign(D->sa_used.size(), {});
+    D->sg_guard_key.assign(D->sg_used.size(), {});
     if (loopback) {
       wofs += rp.total;
       wsofs += align_up(P.workspace_lb[d], 1 << 20);
+    } else if (peer) {
+      wofs += rp.total;
+      wsofs += align_up(P.workspace_mp[d], 1 << 20);
     }
     // tokens H2D (outside any captured graph: the host buffer changes every call)
     const size_t tok_bytes = static_cast<size_t>(P.pp.N) * m.micro_batch * (m.seq_len + 1) * 4;
@@ -669,21 +821,49 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
     }
   }
   cudaStream_t body = E.st;
+  cudaEvent_t t0_peer = nullptr;
   if (!replayed) {
+  if (peer) {
+    // reset the flags, then fork every rank's streams off the caller's (or capture) stream
+    CU(cudaMemsetAsync(E.flags, 0, flag_words * 4, body));
+    if (g.timing) {
+      CU(cudaEventCreate(&t0_peer));
+      CU(cudaEventRecord(t0_peer, body));
+    }
+    cudaEvent_t fork = E.devs[0]->event();
+    CU(cudaEventRecord(fork, body));
+    for (auto& Dp : E.devs) {
+      CU(cudaStreamWaitEvent(Dp->st, fork, 0));
+      CU(cudaStreamWaitEvent(Dp->rx[0], fork, 0));
+      CU(cudaStreamWaitEvent(Dp->rx[1], fork, 0));
+    }
+  }
   for (auto& Dp : E.devs) {
     Dev<T>& D = *Dp;
     const auto& rp = P.rank_params[D.d];
-    CU(cudaMemsetAsync(D.gr, 0, rp.total * 4, body));
-    CU(cudaMemsetAsync(D.ws + D.a.loss, 0, static_cast<size_t>(P.pp.N) * P.pp.parts() * 8, body));
+    cudaStream_t s0 = peer ? D.st : body;
+    if (peer) set_sm_budget(D.sms);
+    CU(cudaMemsetAsync(D.gr, 0, rp.total * 4, s0));
+    CU(cudaMemsetAsync(D.ws + D.a.loss, 0, static_cast<size_t>(P.pp.N) * P.pp.parts() * 8, s0));
     if (sizeof(T) == 2)
       for (size_t j = 0; j < rp.idx.size(); ++j)
         if (D.a.wcopy[j] != SIZE_MAX)
-          cast_f32_bf16(D.w + rp.off[j], reinterpret_cast<__nv_bfloat16*>(D.ws + D.a.wcopy[j]), rp.cnt[j], body);
+          cast_f32_bf16(D.w + rp.off[j], reinterpret_cast<__nv_bfloat16*>(D.ws + D.a.wcopy[j]), rp.cnt[j], s0);
   }
 
   // walk the plan
   if (loopback) {
     for (auto [d, i] : P.loopback_order) E.run_instr(d, P.instrs[d][i]);
+  } else if (peer) {
+    // every rank runs on its own streams and waits only on flags, so the device executes the
+    // plan's DAG concurrently. The host enqueues in the loopback order (a valid order of the DAG in
+    // which the send slots were assigned), so every flag wait follows the write it waits for
+    for (auto [d, i] : P.loopback_order) {
+      if (!E.can_walk(d, P.instrs[d][i])) throw std::runtime_error("peer walk: a flag wait precedes its write");
+      E.run_instr(d, P.instrs[d][i]);
+    }
+    E.st = body;
+    set_sm_budget(0);
   } else {
     const auto& L = P.instrs[me];
     std::vector<std::vector<mario_commop>> sends_after(L.size());
@@ -703,12 +883,49 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
 
   // gradient finalization (reading A7): sum every copy of each parameter (tied embeddings,
   // Chimera replicas) and write the sum back to every copy.
-  std::map<int, std::vector<std::pair<int, int>>> copies;   // global idx -> (dev, packed j)
-  for (int d = 0; d < S; ++d) {
-    const auto& rp = P.rank_params[d];
-    for (size_t j = 0; j < rp.idx.size(); ++j) copies[rp.idx[j]].push_back({d, static_cast<int>(j)});
-  }
-  if (loopback) {
+  if (peer) {
+    // Every copy of a multi-copy parameter (tied wte, Chimera replicas) is summed in copy order,
+    // one element chunk per copy, by the chunk's owner rank reading the other copies in peer memory
+    // (a reduce-scatter); the owners flag their chunks done and every other holder pulls them back
+    // (an all-gather). Flags: per-rank "all BW done" before any chunk is read, per-chunk "summed"
+    // before it is copied back, so no copy is overwritten while another rank still reads it.
+    for (auto& Dp : E.devs) DRV(drv::write_flag(Dp->st, E.flag_misc(Dp->d), 1));
+    size_t fi = static_cast<size_t>(S);
+    for (auto& kv : copies) {
+      const auto& cp = kv.second;
+      if (cp.size() < 2) continue;
+      if (cp.size() > 8) throw std::runtime_error("more than 8 copies of a parameter");
+      const size_t n = P.rank_params[cp[0].first].cnt[cp[0].second];
+      auto ptr = [&](std::pair<int, int> c) { return E.dev(c.first).gr + P.rank_params[c.first].off[c.second]; };
+      const size_t nc = cp.size(), chunk = (n + nc - 1) / nc;
+      for (size_t c = 0; c < nc; ++c) {                       // reduce-scatter: owner of chunk c = copy c
+        Dev<T>& O = E.dev(cp[c].first);
+        const size_t lo = std::min(n, c * chunk), hi = std::min(n, lo + chunk);
+        for (auto& h : cp) DRV(drv::wait_flag(O.st, E.flag_misc(h.first), 1));
+        CopySrcs src{};
+        src.n = static_cast<int>(nc);
+        for (size_t j = 0; j < nc; ++j) src.p[j] = ptr(cp[j]) + lo;
+        if (hi > lo) sum_copies_f32(ptr(cp[c]) + lo, src, hi - lo, O.st);
+        DRV(drv::write_flag(O.st, E.flag_misc(fi + c), 1));
+      }
+      for (size_t c = 0; c < nc; ++c) {                       // all-gather
+        const size_t lo = std::min(n, c * chunk), hi = std::min(n, lo + chunk);
+        for (size_t j = 0; j < nc; ++j) {
+          if (j == c) continue;
+          Dev<T>& H = E.dev(cp[j].first);
+          DRV(drv::wait_flag(H.st, E.flag_misc(fi + c), 1));
+          if (hi > lo) CU(cudaMemcpyAsync(ptr(cp[j]) + lo, ptr(cp[c]) + lo, (hi - lo) * 4, cudaMemcpyDeviceToDevice, H.st));
+        }
+      }
+      fi += nc;
+    }
+    // join every rank's stream back into the caller's (or capture) stream
+    for (auto& Dp : E.devs) {
+      cudaEvent_t e = Dp->event();
+      CU(cudaEventRecord(e, Dp->st));
+      CU(cudaStreamWaitEvent(body, e, 0));
+    }
+  } else if (loopback) {
     for (auto& kv : copies) {
       if (kv.second.size() < 2) continue;
       auto ptr = [&](std::pair<int, int> c) { return E.dev(c.first).gr + P.rank_params[c.first].off[c.second]; };
@@ -798,7 +1015,7 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
   if (g.timing) {
     g.t_start.assign(S, {});
     g.t_finish.assign(S, {});
-    cudaEvent_t t0 = nullptr;
+    cudaEvent_t t0 = t0_peer;   // peer: the fork point every rank's stream starts from
     for (auto& Dp : E.devs) if (!Dp->timed.empty() && !t0) t0 = Dp->timed[0].first;
     for (auto& Dp : E.devs) {
       for (auto& pr : Dp->timed) {
@@ -811,6 +1028,7 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
     }
     for (auto& Dp : E.devs)
       for (auto& pr : Dp->timed) { cudaEventDestroy(pr.first); cudaEventDestroy(pr.second); }
+    if (t0_peer) cudaEventDestroy(t0_peer);
   }
   for (auto& Dp : E.devs) {
     for (auto v : {&Dp->sa_free, &Dp->sg_free, &Dp->rg_free, &Dp->ck_free, &Dp->ev_pool})
@@ -868,6 +1086,46 @@ extern "C" mario_status mario_init_dp(int32_t rank, int32_t world, int32_t devic
     return set_error(MARIO_ENCCL, e.what());
   }
 }
+
+extern "C" mario_status mario_init_emulated(int32_t world, int32_t device, int32_t sms_per_rank) {
+  try {
+    if (world < 1) return set_error(MARIO_EINVAL, "world < 1");
+    if (sms_per_rank < 0) return set_error(MARIO_EINVAL, "sms_per_rank < 0");
+    if (g.inited) return set_error(MARIO_ESTATE, "already initialised");
+    CU(cudaSetDevice(device));
+    CU(cudaFree(nullptr));   // primary context up before any green context retains it
+    g.rank = 0; g.world = 1; g.device = device; g.dp = 1;
+    g.emu_st.assign(world, nullptr);
+    g.emu_rx.assign(world, {nullptr, nullptr});
+    g.emu_sms = 0;
+    g.emu_green = false;
+    if (sms_per_rank > 0) {
+      std::vector<std::vector<cudaStream_t>> ps;
+      int got = 0;
+      const std::string err = drv::make_partitions(device, world, sms_per_rank, 3, ps, &got);
+      if (!err.empty()) {
+        drv::destroy_partitions();
+        return set_error(MARIO_EINVAL, "SM partitions: " + err);
+      }
+      for (int r = 0; r < world; ++r) g.emu_st[r] = ps[r][0], g.emu_rx[r] = {ps[r][1], ps[r][2]};
+      g.emu_sms = got;
+      g.emu_green = true;
+    } else {
+      for (int r = 0; r < world; ++r) {
+        CU(cudaStreamCreateWithFlags(&g.emu_st[r], cudaStreamNonBlocking));
+        for (auto& x : g.emu_rx[r]) CU(cudaStreamCreateWithFlags(&x, cudaStreamNonBlocking));
+      }
+    }
+    g.emulated = true;
+    g.inited = true;
+    g.sticky = false;
+    return MARIO_OK;
+  } catch (const CudaErr& e) {
+    return set_error(MARIO_ECUDA, e.what());
+  }
+}
+
+extern "C" int32_t mario_emulated_sms(void) { return g.emulated ? g.emu_sms : -1; }
 
 extern "C" mario_status mario_init(int32_t rank, int32_t world, int32_t device, const void* nccl_unique_id) {
   return mario_init_dp(rank, world, device, 1, nccl_unique_id);
@@ -954,6 +1212,22 @@ extern "C" mario_status mario_finalize(void) {
   for (auto& kv : g.graph_cache) cudaGraphExecDestroy(kv.second);
   g.graph_cache.clear();
   g.graph_seen.clear();
+  if (g.emulated) {
+    cudaDeviceSynchronize();
+    for (size_t r = 0; r < g.emu_st.size(); ++r) {
+      cudaStreamDestroy(g.emu_st[r]);
+      for (auto x : g.emu_rx[r]) cudaStreamDestroy(x);
+    }
+    g.emu_st.clear();
+    g.emu_rx.clear();
+    if (g.emu_green) drv::destroy_partitions();
+    g.emu_green = false;
+    g.emulated = false;
+    g.emu_sms = 0;
+  }
+  if (g.flags) cudaFree(g.flags);
+  g.flags = nullptr;
+  g.flags_cap = 0;
   if (g.dp_comm) ncclCommDestroy(g.dp_comm);
   g.dp_comm = nullptr;
   if (g.world_comm) ncclCommDestroy(g.world_comm);

@@ -20,6 +20,7 @@
 #include <cstdio>
 #include <cstdlib>
 
+#include "kernels.h"
 #include "kstats.h"
 #include "layers.h"
 #include "sm100.cuh"
@@ -1420,9 +1421,7 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
       cudaFuncSetAttribute(fa_bwd_dq_img<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize, SmemI<DH>::kBytes);
       iset = true;
     }
-    int sms = 0, dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const int sms = device_sm_count();
     const int items = B * nh * (s / kRows);
     static const int per_sm = getenv("MARIO_DQI_CTAS") ? atoi(getenv("MARIO_DQI_CTAS")) : 2;
     const int grid_i = items < per_sm * sms ? items : per_sm * sms;
@@ -1434,9 +1433,7 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
         cudaFuncSetAttribute(fa_bwd_dq_pers<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_dq<DH>());
         pset = true;
       }
-      int sms = 0, dev = 0;
-      cudaGetDevice(&dev);
-      cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+      const int sms = device_sm_count();
       const int items = B * nh * ((s + kRows - 1) / kRows);
       fa_bwd_dq_pers<DH><<<items < sms ? items : sms, kThreadsP, smem_dq<DH>(), st>>>(m128, m64, d128, lse, Dd, dqkv,
                                                                                          B, s, nh);
@@ -1982,12 +1979,7 @@ bool flash_attn_bwd_tc_supported(int dh, int B, int s, int nh) {
 bool flash_attn_fwd_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st) {
   // g_attn_variant: -1 auto (two-Q-tile kernel unless it would launch fewer CTAs than SMs: the
   // one-Q-tile kernel has twice as many), 2 force the one-Q-tile kernel, 3 force the two-Q-tile one
-  int sms = 148;
-  {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  }
+  const int sms = device_sm_count();
   const long ctas2 = static_cast<long>((s + 2 * kF2Q - 1) / (2 * kF2Q)) * B * nh;
   if (g_attn_variant == 2 || (g_attn_variant != 3 && ctas2 < sms)) {
     if (dh == 128) return launch_fwd_tc<128>(qkv, O, lse, B, s, nh, st);

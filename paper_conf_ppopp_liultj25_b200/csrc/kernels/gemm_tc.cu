@@ -975,7 +975,13 @@ bool make_tmap_bf16_2d(CUtensorMap* map, const void* base, uint64_t inner, uint6
   return make_tmap(map, base, inner, outer, ld, box_inner, box_outer);
 }
 
-int device_sm_count() {
+// SM budget of the launching thread (set_sm_budget): the executor's emulated pipeline runs each
+// stage on an SM partition (a green context), and every persistent / SM-sized grid of a kernel
+// launched for that stage must be sized for the partition, not the device.
+static thread_local int g_sm_budget = 0;
+void set_sm_budget(int sms) { g_sm_budget = sms; }
+
+int device_sm_count_full() {
   static int n = 0;
   if (n == 0) {
     int dev = 0;
@@ -984,6 +990,11 @@ int device_sm_count() {
     if (n <= 0) n = 148;
   }
   return n;
+}
+
+int device_sm_count() {
+  const int n = device_sm_count_full();
+  return g_sm_budget > 0 && g_sm_budget < n ? g_sm_budget : n;
 }
 
 int g_gemm_variant = -1;   // mario_k_gemm_set_variant: -1 auto, 0 single-CTA, 1 pair (auto N), 2 pair N=128, 3 pair N=256

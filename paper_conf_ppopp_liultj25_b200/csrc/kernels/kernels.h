@@ -6,7 +6,9 @@
 
 namespace mario {
 
-int device_sm_count();
+int device_sm_count();          // SMs the launching thread may use (the device's, or its budget)
+void set_sm_budget(int sms);     // 0 = the whole device
+int device_sm_count_full();      // the device's SMs (reduction partitions that fix summation order)
 
 // ------------------------------------------------------------------ GEMM (K1-K4)
 struct GemmEpilogue {

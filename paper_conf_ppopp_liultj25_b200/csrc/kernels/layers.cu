@@ -8,6 +8,8 @@
 #include "layers.h"
 #include "kstats.h"
 
+#include "kernels.h"
+
 namespace mario {
 namespace {
 
@@ -784,16 +786,10 @@ inline int tile_vpt(int n) {
   return 0;
 }
 
-int device_sms() {
-  static int sms = 0;
-  if (!sms) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    if (sms <= 0) sms = 148;
-  }
-  return sms;
-}
+// the device's full SM count, NOT the launching thread's budget: the row partition of the column
+// reductions below follows it, so their fp32 partial sums (and the bits of the bias / gain
+// gradients) do not depend on the SM partition a stage runs on (emulated pipeline, set_sm_budget)
+int device_sms() { return device_sm_count_full(); }
 
 template <class K>
 int resident_grid(K kernel, int threads) {
@@ -1502,6 +1498,22 @@ void cast_f32_bf16(const float* x, __nv_bfloat16* y, size_t n, cudaStream_t st) 
 }
 void add_f32(float* a, const float* b, size_t n, cudaStream_t st) { add_k<<<grid_for(static_cast<long>(n)), 256, 0, st>>>(a, b, n); note_launch(); }
 void copy_f32(float* a, const float* b, size_t n, cudaStream_t st) { copy_k<<<grid_for(static_cast<long>(n)), 256, 0, st>>>(a, b, n); note_launch(); }
+
+// dst[i] = ((src0[i] + src1[i]) + src2[i]) + ...: the copies of one parameter summed in copy order
+// (the loopback's acc = c0; acc += c1; ... association). Every source is read before dst is
+// written, so dst may be one of the sources; sources may live in another rank's memory.
+__global__ void sum_copies_k(float* dst, CopySrcs s, size_t n) {
+  for (size_t i = blockIdx.x * static_cast<size_t>(blockDim.x) + threadIdx.x; i < n;
+       i += static_cast<size_t>(gridDim.x) * blockDim.x) {
+    float acc = s.p[0][i];
+    for (int c = 1; c < s.n; ++c) acc += s.p[c][i];
+    dst[i] = acc;
+  }
+}
+void sum_copies_f32(float* dst, const CopySrcs& srcs, size_t n, cudaStream_t st) {
+  sum_copies_k<<<grid_for(static_cast<long>(n)), 256, 0, st>>>(dst, srcs, n);
+  note_launch();
+}
 
 #define INST(T)                                                                                                     \
   template void embed_fwd<T>(const int32_t*, int, int, int, const T*, const T*, T*, int, cudaStream_t);              \

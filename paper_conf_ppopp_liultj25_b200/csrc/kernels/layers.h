@@ -91,5 +91,7 @@ void flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* O, const __nv
 void cast_f32_bf16(const float* x, __nv_bfloat16* y, size_t n, cudaStream_t st);
 void add_f32(float* a, const float* b, size_t n, cudaStream_t st);       // a += b
 void copy_f32(float* a, const float* b, size_t n, cudaStream_t st);
+struct CopySrcs { const float* p[8]; int n; };                                 // n <= 8
+void sum_copies_f32(float* dst, const CopySrcs& srcs, size_t n, cudaStream_t st);   // dst = sum in order
 
 }  // namespace mario

@@ -19,20 +19,16 @@
 #include "layers.h"
 #include "sm100.cuh"
 
+#include "kernels.h"
+
 namespace mario {
 namespace {
 using bf16 = __nv_bfloat16;
 
-int device_sms() {
-  static int sms = 0;
-  if (!sms) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    if (sms <= 0) sms = 148;
-  }
-  return sms;
-}
+// the device's full SM count, NOT the launching thread's budget: the row partition of the column
+// reductions below follows it, so their fp32 partial sums (and the bits of the bias / gain
+// gradients) do not depend on the SM partition a stage runs on (emulated pipeline, set_sm_budget)
+int device_sms() { return device_sm_count_full(); }
 using namespace sm100;
 
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {

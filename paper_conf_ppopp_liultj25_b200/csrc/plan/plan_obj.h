@@ -45,6 +45,11 @@ struct mario_plan {
   // executor pools per device (slot counts) for multi-process and loopback execution
   struct Pools { int ckpt = 0, act = 0, send_act = 0, send_grad = 0, recv_grad = 0; };
   std::vector<Pools> pools_mp, pools_lb;
+  // send slot of every message, per device: (micro, part) -> slot. Assigned once along the
+  // loopback order (a valid execution order of the plan's DAG), holding a slot from its FW/CFW (BW)
+  // until the receiver's RA (RG): every executor reuses a slot only after a message the loopback
+  // order has already consumed, so the slot-reuse waits add no cycle to the DAG.
+  std::vector<std::map<std::pair<int, int>, int>> sa_slot, sg_slot;
   std::vector<uint64_t> workspace_mp, workspace_lb;  // bytes per device
   // global execution order used by loopback (device, list index), round-robin like the simulator
   std::vector<std::pair<int, int>> loopback_order;

@@ -1,7 +1,7 @@
 # Evidence for DESIGN.md reading A19 (oracle-only experiment, not a test): how far does *storing*
 # fp32 oracle's gradients at LLaMA2-7B width?  Monkey-patch rounding into a copy of the oracle.
 import sys, numpy as np
-sys.path.insert(0, "/root/repo")
+sys.path.insert(0, __import__("os").path.dirname(__import__("os").path.dirname(__import__("os").path.dirname(__import__("os").path.abspath(__file__)))))
 import synth
 from oracle import model as om
 

@@ -1,9 +1,9 @@
 """Write tests/golden/* files that are derived values. Calls ONLY oracle/ (and synth for
-shapes) — never the CUDA/C++ product. Usage: python tools/make_goldens.py"""
+shapes) — never the CUDA/C++ product. Usage: python tests/tools/make_goldens.py"""
 import os
 import sys
 
-ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+ROOT = os.path.dirname(os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 sys.path.insert(0, ROOT)
 
 import synth  # noqa: E402

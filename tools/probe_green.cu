@@ -9,6 +9,7 @@
 #include <cstdio>
 #include <set>
 #include <vector>
+#define printf(...) (fprintf(stderr, __VA_ARGS__), fflush(stderr))
 
 #define CK(x) do { cudaError_t e = (x); if (e != cudaSuccess) { printf("FAIL %s: %s\n", #x, cudaGetErrorString(e)); return 1; } } while (0)
 #define DK(x) do { CUresult e = (x); if (e != CUDA_SUCCESS) { const char* s; cuGetErrorString_(e, &s); printf("FAIL %s: %s\n", #x, s); return 1; } } while (0)
@@ -60,6 +61,7 @@ int main() {
   CUdevResource all;
   DK(getRes(dev, &all, CU_DEV_RESOURCE_TYPE_SM));
   printf("device SMs: %u\n", all.sm.smCount);
+  printf("step: split\n");
   const int G = 8;
   for (unsigned minc : {16u, 18u}) {
     std::vector<CUdevResource> parts(G);
@@ -109,11 +111,12 @@ int main() {
   CK(cudaMalloc(&stamps, 16));
   CK(cudaMemset(flag, 0, 4));
   CK(cudaDeviceSynchronize());
-  DK(waitV(st[0], (CUdeviceptr)flag, 1, CU_STREAM_WAIT_VALUE_GEQ));
-  stamp_k<<<1, 1, 0, (cudaStream_t)st[0]>>>(stamps);
+  // the write is ENQUEUED before the wait (the executor's rule), but executes ~20 ms later
   smid_k<<<16, 32, 0, (cudaStream_t)st[1]>>>(d_sm, 40000000);
   stamp_k<<<1, 1, 0, (cudaStream_t)st[1]>>>(stamps + 1);
   DK(writeV(st[1], (CUdeviceptr)flag, 1, 0));
+  DK(waitV(st[0], (CUdeviceptr)flag, 1, CU_STREAM_WAIT_VALUE_GEQ));
+  stamp_k<<<1, 1, 0, (cudaStream_t)st[0]>>>(stamps);
   CK(cudaDeviceSynchronize());
   unsigned long long hs[2];
   CK(cudaMemcpy(hs, stamps, 16, cudaMemcpyDeviceToHost));
@@ -130,11 +133,12 @@ int main() {
   CK(cudaDeviceSynchronize());
   CK(cudaStreamBeginCapture(origin, cudaStreamCaptureModeThreadLocal));
   CK(cudaEventRecord(ef, origin));
+  for (unsigned i = 0; i < n; ++i) CK(cudaStreamWaitEvent((cudaStream_t)st[i], ef, 0));
+  smid_k<<<B, 128, 0, (cudaStream_t)st[1]>>>(d_sm + 1 * B, 20000);
+  DK(writeV(st[1], (CUdeviceptr)flag, 1, 0));
+  DK(waitV(st[0], (CUdeviceptr)flag, 1, CU_STREAM_WAIT_VALUE_GEQ));
   for (unsigned i = 0; i < n; ++i) {
-    CK(cudaStreamWaitEvent((cudaStream_t)st[i], ef, 0));
-    if (i == 0) DK(waitV(st[0], (CUdeviceptr)flag, 1, CU_STREAM_WAIT_VALUE_GEQ));
-    smid_k<<<B, 128, 0, (cudaStream_t)st[i]>>>(d_sm + i * B, 20000);
-    if (i == 1) DK(writeV(st[1], (CUdeviceptr)flag, 1, 0));
+    if (i != 1) smid_k<<<B, 128, 0, (cudaStream_t)st[i]>>>(d_sm + i * B, 20000);
     CK(cudaEventRecord(ej[i], (cudaStream_t)st[i]));
     CK(cudaStreamWaitEvent(origin, ej[i], 0));
   }
