@@ -22,6 +22,9 @@ import threading
 import time
 
 ROOT = os.path.dirname(os.path.abspath(__file__))
+# the emulated pipeline runs S ranks x (compute + 2 receive) streams concurrently: give every stream
+# its own hardware queue (the default 8 connections alias streams and serialize independent ranks)
+os.environ.setdefault("CUDA_DEVICE_MAX_CONNECTIONS", "32")
 sys.path.insert(0, ROOT)
 
 import numpy as np  # noqa: E402
@@ -45,7 +48,10 @@ def parse():
     ap.add_argument("--micro", type=int, default=32)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
-    ap.add_argument("--no-projection", action="store_true")
+    ap.add_argument("--emulate-only", action="store_true", help="only the emulated-pipeline measurement")
+    ap.add_argument("--emulate", type=int, default=8,
+                    help="N=1: also measure an S-stage pipeline of the same workload on this GPU (SM partitions, "
+                         "peer transport) at BASE / CKPT / MARIO; 0 disables")
     ap.add_argument("--graphs", type=int, default=1, help="also time CUDA-graph replay (N = 1)")
     return ap.parse_args()
 
@@ -59,17 +65,37 @@ def measured_peaks():
 
 
 # ------------------------------------------------------------------ CPU oracle leg
-def gemm_traffic():
-    """DRAM bytes per GEMM launch from the committed ncu --set full capture (profiles/), or {}."""
+def gemm_traffic(cfg):
+    """DRAM bytes per GEMM launch from the committed ncu --set full capture (profiles/), next to
+    the ALGORITHMIC bytes of the same four launches (one layer's forward GEMMs at this config:
+    operands + outputs + residual / second output, bf16), or {}."""
     p = os.path.join(ROOT, "profiles", "r01_traffic.json")
     if not os.path.exists(p):
         return {}
     d = json.load(open(p)).get("gemm_bf16_tc2_kernel", {})
     if "dram_bytes_per_launch" not in d:
         return {}
+    T, h, f = cfg.seq_len * 4, cfg.hidden, cfg.ffn_hidden      # the capture ran at mbs 4 (cfg 2)
+    alg = [2 * (T * h + 3 * h * h + T * 3 * h),                 # qkv: A, W, D
+           2 * (T * h + h * h + 2 * T * h),                     # proj: A, W, residual, D
+           2 * (T * h + f * h + 2 * T * f),                     # fc1: A, W, Z, G = gelu(Z)
+           2 * (T * f + h * f + 2 * T * h)]                     # fc2: A, W, residual, D
     return {"dram_bytes_per_launch": d["dram_bytes_per_launch"],
+            "algorithmic_bytes_per_launch": sum(alg) / len(alg),
             "note": f"mean dram__bytes_read+write over {d.get('launches_captured')} captured launches "
-                    f"(one layer's forward GEMMs: qkv, proj, fc1, fc2); {d.get('source', '')}"}
+                    f"(one layer's forward GEMMs: qkv, proj, fc1, fc2) vs the algorithmic bytes of the same four "
+                    f"launches; {d.get('source', '')}"}
+
+
+def cpu_model():
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    import platform
+    return platform.processor() or "unknown"
 
 
 def cpu_oracle_sample(cfg, layers_list=(1, 2)):
@@ -115,9 +141,13 @@ def run_reference(args, cfg, gbs):
     t = statistics.median(ts)
     v = 1.0 / t
     sample = (f"1 sample (mbs 1) of {cfg.family} L=1 and L=2 (+embedding/head, s={cfg.seq_len}) fwd+bwd "
-              f"fp32 per step, extrapolated to L={cfg.n_layers}")
+              f"fp32 per step, extrapolated to L={cfg.n_layers}; CPU: {cpu_model()}")
     out = {"impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": args.gpus,
            "steps": args.steps, "warmup": args.warmup, "ms_per_step": t * 1e3 * gbs,
+           "ms_per_step_extrapolated": True,
+           "ms_per_step_note": "EXTRAPOLATED, not timed: the measured per-sample time (value = 1 / it) times the "
+                               f"global batch {gbs}; each timed step ran one sample of the 1- and 2-layer models",
+           "ms_per_sample_measured": t * 1e3,
            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f32",
            "data": "synthetic", "config": config_dict(cfg, args, gbs),
            "cpu_baseline": {"value": v, "unit": UNIT, "cores": n_cores, "kind": "oracle", "sample": sample},
@@ -196,47 +226,107 @@ def init_weights_device(plan, rank, torch, seed=1234):
     return w
 
 
-def project_pipeline(cfg, api, torch, ctx_factory, stages=8, n_profile=8, n_micro=32):
-    """The paper's method (P:242 profile -> P:244-252 simulate): run one 8-stage Mario iteration in
-    loopback on this GPU with per-instruction CUDA events, take the mean FW/CFW, BW and RC time of
-    each virtual stage, and simulate the BASE / CKPT / MARIO plans of the 8-GPU pipeline with
-    those costs (p2p at the measured NVLink peer bandwidth, B200_PROFILING.md: 770 GB/s)."""
-    prof = api.Plan(cfg, stages, n_profile, "1f1b", "mario", dtype="bf16")
-    ctx = ctx_factory()
-    w, g, ws = api.alloc_for(prof, -1)
-    w.normal_(0.0, 0.02)
-    tok = torch.from_numpy(synth.make_tokens(cfg, n_profile)).cuda()
-    ctx.run_iter(prof, w, tok, g, ws)          # warm-up
-    ctx.set_timing(True)
-    ctx.run_iter(prof, w, tok, g, ws)
-    ctx.set_timing(False)
-    fw = [[] for _ in range(stages)]
-    bw = [[] for _ in range(stages)]
-    rc = [[] for _ in range(stages)]
-    for d in range(stages):
-        a, b = ctx.last_timeline(d)
-        comp = [x for x in prof.instrs(d) if x[0] in ("FW", "CFW", "RC", "BW")]
-        for (op, *_r), t0, t1 in zip(comp, a, b):
-            {"FW": fw, "CFW": fw, "RC": rc, "BW": bw}[op][d].append(t1 - t0)
-    mean = lambda xs: sum(xs) / len(xs) if xs else 0.0
-    costs = {"fw_ms": [mean(x) for x in fw], "bw_ms": [mean(x) for x in bw],
-             "rc_ms": [mean(x) if x else mean(fw[i]) for i, x in enumerate(rc)],
-             "p2p_alpha_ms": 0.02, "p2p_GBps": 770.0}
-    del w, g, ws
-    torch.cuda.empty_cache()
+def union_ms(iv):
+    """Length of the union of [a, b) intervals (ms)."""
+    tot, end = 0.0, None
+    for a, b in sorted(iv):
+        if end is None or a > end:
+            tot += b - a
+            end = b
+        elif b > end:
+            tot += b - end
+            end = b
+    return tot
+
+
+def emulate_pipeline(cfg, api, torch, S=8, n_micro=32, steps=2, warmup=2, levels=("base", "ckpt", "mario"),
+                     scheme="1f1b", chunks=1):
+    """Measured S-stage pipeline on ONE GPU (mario_init_emulated): every stage is a pipeline rank on
+    its own green-context SM partition (floor(148 / S) rounded down to a multiple of 8 SMs), ranks
+    exchange activations / gradients through the peer transport, and the device runs the plan's
+    DAG concurrently. Per plan (BASE / CKPT = plain 1F1B with full checkpointing / MARIO):
+    iteration time (CUDA events on the launching stream, graph replay, median of `steps`), the
+    MEASURED bubble ratio 1 - sum_d busy_d / (S * makespan) from per-rank CUDA-event timelines
+    (busy_d = union of the rank's FW/CFW/RC/BW intervals), the simulator's prediction from the same
+    run's per-virtual-stage costs (the paper's profile -> simulate loop) and the
+    per-stage memory (static arena, exact: simulated peak vs allocated bytes). The partitions share
+    HBM and L2, so absolute times are those of 1/S-th of a B200 per stage, not of S B200s."""
+    sms = (device_sms(torch) // S) // 8 * 8
     gbs = n_micro * cfg.micro_batch
-    out = {"method": "per-stage costs measured (CUDA events, 8-stage loopback on this GPU) -> planner simulator",
-           "stages": stages, "microbatches": n_micro,
-           "stage_ms": {k: [round(x, 3) for x in costs[k]] for k in ("fw_ms", "bw_ms", "rc_ms")}}
-    for level in ("base", "ckpt", "mario"):
-        p = api.Plan(cfg, stages, n_micro, "1f1b", level, dtype="bf16", costs=costs)
-        sim = p.simulate()
-        out[level] = {"makespan_ms": round(sim.makespan_ms, 2), "samples_per_s": round(gbs / (sim.makespan_ms / 1e3), 2),
-                      "bubble": round(sim.bubble_ratio, 4), "peak_gb_per_stage": [round(b / 1e9, 2) for b in sim.peak_bytes],
-                      "peak_balance_max_over_min": round(max(sim.peak_bytes) / min(sim.peak_bytes), 3)}
-    out["mario_vs_ckpt"] = round(out["ckpt"]["makespan_ms"] / out["mario"]["makespan_ms"], 4)
-    out["mario_vs_base"] = round(out["base"]["makespan_ms"] / out["mario"]["makespan_ms"], 4)
+    out = {"stages": S, "microbatches": n_micro, "scheme": scheme, "sms_per_stage": sms,
+           "method": "one process, S ranks on disjoint green-context SM partitions of this GPU, peer transport; "
+                     "iteration time = CUDA events around graph-replayed iterations (median); bubble from per-rank "
+                     "CUDA-event timelines of one extra eager iteration", "levels": {}}
+    toks = [torch.from_numpy(synth.make_tokens(cfg, n_micro, iteration=i)).cuda() for i in range(2)]
+    api.close_default_context()
+    for level in levels:
+        plan = api.Plan(cfg, S, n_micro, scheme, level, chunks=chunks, dtype="bf16")
+        ctx = api.Context.emulated(S, 0, sms)
+        try:
+            pc, wsb = plan.rank_layout(-2)
+            w = torch.empty(pc, dtype=torch.float32, device="cuda").normal_(0.0, 0.02)
+            g = torch.empty(pc, dtype=torch.float32, device="cuda")
+            ws = torch.empty(wsb, dtype=torch.uint8, device="cuda")
+            stream = torch.cuda.current_stream()
+            ctx.set_graphs(True)
+            for i in range(max(warmup, 2)):
+                ctx.run_iter(plan, w, toks[i % 2], g, ws, stream)
+            torch.cuda.synchronize()
+            ts = []
+            for i in range(steps):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(stream)
+                loss = ctx.run_iter(plan, w, toks[i % 2], g, ws, stream)
+                e1.record(stream)
+                torch.cuda.synchronize()
+                ts.append(e0.elapsed_time(e1))
+            ctx.set_graphs(False)
+            ctx.set_timing(True)
+            ctx.run_iter(plan, w, toks[0], g, ws, stream)
+            torch.cuda.synchronize()
+            ctx.set_timing(False)
+            tl = [ctx.last_timeline(d) for d in range(S)]
+            ms = statistics.median(ts)
+            span = max(max(b) for a, b in tl if b)
+            busy = [union_ms(list(zip(a, b))) for a, b in tl]
+            # per-virtual-stage costs of this run -> the simulator (P:242 profile, P:244-252 simulate)
+            K = plan.S * (chunks if scheme == "interleave" else 1)
+            fw, bw, rc = ([[] for _ in range(K)] for _ in range(3))
+            for d in range(S):
+                comp = [x for x in plan.instrs(d) if x[0] in ("FW", "CFW", "RC", "BW")]
+                for (op, m_, p_, k, *_r), t0, t1 in zip(comp, *tl[d]):
+                    {"FW": fw, "CFW": fw, "RC": rc, "BW": bw}[op][k].append(t1 - t0)
+            mean = lambda xs: sum(xs) / len(xs) if xs else 0.0
+            costs = {"fw_ms": [mean(x) for x in fw], "bw_ms": [mean(x) for x in bw],
+                     "rc_ms": [mean(x) if x else mean(fw[i]) for i, x in enumerate(rc)],
+                     "p2p_alpha_ms": 0.005, "p2p_GBps": 1500.0}
+            sim = api.Plan(cfg, S, n_micro, scheme, level, chunks=chunks, dtype="bf16", costs=costs).simulate()
+            alloc = [plan.rank_layout(d)[1] + 8 * plan.rank_layout(d)[0] for d in range(S)]
+            peaks = plan.simulate().peak_bytes
+            out["levels"][level] = {
+                "ms_per_iter": ms, "samples_per_s": gbs / (ms / 1e3), "loss": loss,
+                "bubble_measured": 1.0 - sum(busy) / (S * span),
+                "bubble_simulated": sim.bubble_ratio,
+                "makespan_measured_ms": span, "makespan_simulated_ms": sim.makespan_ms,
+                "busy_ms_per_stage": [round(b, 2) for b in busy],
+                "stage_ms": {k: [round(x, 3) for x in costs[k]] for k in ("fw_ms", "bw_ms", "rc_ms")},
+                "peak_gb_per_stage_simulated": [round(b / 1e9, 3) for b in peaks],
+                "alloc_gb_per_stage": [round(b / 1e9, 3) for b in alloc],
+                "peak_balance_max_over_min": max(peaks) / min(peaks)}
+            del w, g, ws
+        finally:
+            ctx.close()
+            torch.cuda.empty_cache()
+    lv = out["levels"]
+    if "ckpt" in lv and "mario" in lv:
+        out["mario_vs_ckpt"] = lv["ckpt"]["ms_per_iter"] / lv["mario"]["ms_per_iter"]
+    if "base" in lv and "mario" in lv:
+        out["mario_vs_base"] = lv["base"]["ms_per_iter"] / lv["mario"]["ms_per_iter"]
     return out
+
+
+def device_sms(torch):
+    return torch.cuda.get_device_properties(torch.cuda.current_device()).multi_processor_count
 
 
 def main():
@@ -250,6 +340,13 @@ def main():
     import torch
     import torch.distributed as dist
     from paper_conf_ppopp_liultj25_b200 import _lib, api
+    if args.emulate_only:
+        torch.cuda.set_device(0)
+        levels = tuple(os.environ.get("MARIO_EMU_LEVELS", "base,ckpt,mario").split(","))
+        print(json.dumps({"pipeline_emulated": emulate_pipeline(cfg, api, torch, S=args.emulate, n_micro=args.micro,
+                                                                steps=max(1, min(args.steps, 3)), warmup=2,
+                                                                levels=levels, scheme=args.scheme)}), flush=True)
+        return
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -365,26 +462,40 @@ def main():
 
     sim = plan.simulate()
     peaks, peak_kind = measured_peaks()
-    traffic = gemm_traffic()
+    traffic = gemm_traffic(cfg)
     g = kst["gemm"]
     achieved = g["flops"] / (g["ms"] / 1e3) / 1e12 if g["ms"] > 0 else 0.0
     peak = float(peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops")))
     model_flops = 3.0 * (cfg.n_layers * (2 * cfg.seq_len * (12 * cfg.hidden ** 2) + 4 * cfg.seq_len ** 2 * cfg.hidden)
                          + 2 * cfg.seq_len * cfg.hidden * cfg.vocab)
     tflops_gpu = model_flops * gbs / (ms_step / 1e3) / world / 1e12
+    # whole-step algorithmic roofline: the FLOPs the method must execute (causal
+    # attention; + Mario's recompute when stages > 1) over the step time and the dense bf16 peak
+    S_ = world // args.dp
+    layer_f = 2 * cfg.seq_len * (12 * cfg.hidden ** 2) + 2 * cfg.seq_len ** 2 * cfg.hidden
+    alg_flops = 3.0 * (cfg.n_layers * layer_f + 2 * cfg.seq_len * cfg.hidden * cfg.vocab) * gbs
+    if S_ > 1 and args.level != "base":
+        alg_flops += (S_ - 1) * (cfg.n_layers // S_) * layer_f * gbs   # RC of every checkpointed stage
+    alg_tflops = alg_flops / (ms_step / 1e3) / world / 1e12
     mem = torch.cuda.max_memory_allocated()
     out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "strong",
            "vs_baseline": None, "dtype": "bf16", "data": "synthetic (uniform tokens, random-init weights)",
            "config": config_dict(cfg, args, gbs),
            "model_tflops_per_gpu": tflops_gpu,
+           "whole_step_roofline": {"algorithmic_tflops_per_gpu": alg_tflops,
+                                   "frac_of_2250_datasheet": alg_tflops / 2250.0,
+                                   "frac_of_measured_sustained": alg_tflops / peak,
+                                   "flops_per_step": alg_flops,
+                                   "note": "causal attention FLOPs (2 s^2 h per layer-sample fwd), no RC at 1 stage"},
            "loss": losses[-1],
            "roofline": {"bound": "tensor", "kernel": "gemm_bf16_tc_kernel (tcgen05, all linear layers)",
                         "achieved": achieved, "peak": peak, "unit": "TFLOP/s", "frac": achieved / peak,
                         "peak_source": f"{peak_kind} bf16_tflops_sustained (MEASURED_PEAKS.json)",
                         "traffic": traffic.get("dram_bytes_per_launch"),
                         "traffic_note": traffic.get("note"),
-                        "algorithmic_bytes_per_launch": (g["bytes"] / g["launches"]) if g["launches"] else None,
+                        "algorithmic_bytes_per_launch": traffic.get("algorithmic_bytes_per_launch"),
+                        "algorithmic_bytes_per_launch_all_gemms": (g["bytes"] / g["launches"]) if g["launches"] else None,
                         "launches_per_step": g["launches"] / kst_steps,
                         "measured_in": "graph replay (latest step)" if use_graphs else "eager steps",
                         "share_of_step": (g["ms"] / kst_steps) / ms_step if ms_step > 0 else None},
@@ -399,18 +510,20 @@ def main():
                                   "measured_torch_max_allocated": int(mem)},
            "execution": "cuda-graph replay" if use_graphs else "eager",
            "e2e": e2e, "eager": eager}
-    if rank == 0 and world == 1 and not args.no_projection:
-        out["pipeline_projection_8gpu"] = project_pipeline(cfg, api, torch, lambda: ctx)
+    ctx.close()
+    if rank == 0 and world == 1 and args.emulate > 1:
+        out["pipeline_emulated"] = emulate_pipeline(cfg, api, torch, S=args.emulate, n_micro=args.micro,
+                                                    steps=max(1, min(args.steps, 3)), warmup=2)
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         n_cores = cores()
         os.environ.setdefault("OPENBLAS_NUM_THREADS", str(n_cores))
         t, times = cpu_oracle_sample(cfg)
         out["cpu_baseline"] = {"value": 1.0 / t, "unit": UNIT, "cores": n_cores, "kind": "oracle",
+                               "cpu_model": cpu_model(),
                                "sample": f"1 sample (mbs 1), fp32 numpy oracle, L=1 ({times[1]:.2f}s) and L=2 "
                                          f"({times[2]:.2f}s) + embedding/head at s=2048, extrapolated to 24 layers"}
     if rank == 0:
         print(json.dumps(out), flush=True)
-    ctx.close()
     if world > 1:
         dist.destroy_process_group()
 

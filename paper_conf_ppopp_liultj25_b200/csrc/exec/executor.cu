@@ -24,6 +24,7 @@
 
 #include <cmath>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <algorithm>
 #include <array>
@@ -312,20 +313,37 @@ struct Exec {
       Hin = Hout;
     }
     if (k == K - 1) {
+      // fused head (K13): final norm, then per token chunk logits -> softmax-CE -> dlogits -> the
+      // head's dgrad rows (dHf, kept for BW) and wgrad. The loss ends the graph, so the head's
+      // backward needs nothing a later instruction produces; running it here keeps only dHf [T, h]
+      // instead of dlogits [T, V] alive until BW. CFW (mode 1) records the loss only; RC (mode 2)
+      // replays the gradients without the loss; FW does both: each head contribution is added once.
+      const HeadScratch HS = head_scratch_layout(m);
+      uint8_t* hs = D.template at<uint8_t>(D.a.logits);
       T* Hl = reinterpret_cast<T*>(head_base + HA.H_last);
-      T* Hf = reinterpret_cast<T*>(head_base + HA.Hf);
       float* stf = reinterpret_cast<float*>(head_base + HA.stf);
-      T* dlog = reinterpret_cast<T*>(head_base + HA.dlogits);
+      T* dHf = reinterpret_cast<T*>(head_base + HA.dHf);
+      T* Hf = reinterpret_cast<T*>(hs + HS.Hf);
+      float* logits = reinterpret_cast<float*>(hs + HS.logits);
+      T* dlog = reinterpret_cast<T*>(hs + HS.dlog);
       const int V = m.vocab;
       if (gpt) layernorm_fwd<T>(Hl, Wf(D, p, "lnf.g"), Wf(D, p, "lnf.b"), Hf, stf, Tn, h, m.norm_eps, st);
       else rmsnorm_fwd<T>(Hl, Wf(D, p, "nf.g"), Hf, stf, Tn, h, m.norm_eps, st);
-      const T* Wh = Wm(D, p, gpt ? (m.tie_embeddings ? "wte" : "head.w") : "out.w");
-      float* logits = D.template at<float>(D.a.logits);
-      gemm(Hf, h, 0, Wh, h, 0, Tn, V, h, logits, V, true, 0.f);
+      const std::string hw = gpt ? (m.tie_embeddings ? "wte" : "head.w") : "out.w";
+      const T* Wh = Wm(D, p, hw);
       float* row_loss = reinterpret_cast<float*>(D.template at<uint8_t>(D.a.loss) +
                                                  static_cast<size_t>(D.P->pp.N) * D.P->pp.parts() * 8);
       const float inv_ntok = 1.0f / static_cast<float>(static_cast<double>(D.P->pp.N) * Tn);
-      softmax_ce<T>(logits, tok, s + 1, s, Tn, V, inv_ntok, dlog, row_loss, st);
+      for (int r0 = 0; r0 < Tn; r0 += HS.rows) {
+        const int rows = std::min(HS.rows, Tn - r0);
+        const T* Hfc = Hf + static_cast<size_t>(r0) * h;
+        gemm(Hfc, h, 0, Wh, h, 0, rows, V, h, logits, V, true, 0.f);
+        softmax_ce<T>(logits, tok, s + 1, s, rows, V, inv_ntok, dlog, row_loss + r0, st, r0);
+        if (mode != 1) {
+          lin_dgrad(dlog, Wh, rows, V, h, dHf + static_cast<size_t>(r0) * h);   // dHf rows
+          lin_wgrad(dlog, Hfc, rows, V, h, G(D, p, hw));                        // dW_head += dlog^T Hf
+        }
+      }
       if (mode != 2) loss_reduce(row_loss, Tn, D.template at<double>(D.a.loss) + x.micro, st);
     }
   }
@@ -351,27 +369,35 @@ struct Exec {
     T* dZ = reinterpret_cast<T*>(sc + BS.dZ);
     T* dM = reinterpret_cast<T*>(sc + BS.dM);
     float* Dsc = reinterpret_cast<float*>(sc + BS.Dsc);
+    // bf16 mode (reading A30): the residual-stream gradient dH is carried in fp32 between layers
+    // (dH32, two buffers: LN2 reads [0] writes [1], LN1 reads [1] writes [0]); the bf16 dH buffers
+    // are the operand copies of the GEMMs. nullptr = the bf16 dH is exact (a received message).
+    constexpr bool r32 = sizeof(T) == 2;
+    float* dH32buf[2] = {reinterpret_cast<float*>(sc + BS.dH32[0]), reinterpret_cast<float*>(sc + BS.dH32[1])};
+    const float* dH32 = nullptr;
     float* red = D.template at<float>(D.a.red);
     const size_t red_floats = D.a.red_bytes / sizeof(float);
     const int32_t* tok = D.template at<int32_t>(D.a.tokens) + static_cast<size_t>(x.micro) * mbs * (s + 1);
     int cur = 0;
     const T* dH;   // gradient of the current layer's output
     if (k == K - 1) {
-      const int V = m.vocab;
+      // the head's gradients were produced by the fused head of the FW / RC (stage_forward)
       T* Hl = reinterpret_cast<T*>(head_base + HA.H_last);
-      T* Hf = reinterpret_cast<T*>(head_base + HA.Hf);
       float* stf = reinterpret_cast<float*>(head_base + HA.stf);
-      T* dlog = reinterpret_cast<T*>(head_base + HA.dlogits);
-      const std::string hw = gpt ? (m.tie_embeddings ? "wte" : "head.w") : "out.w";
-      lin_wgrad(dlog, Hf, Tn, V, h, G(D, p, hw));
-      lin_dgrad(dlog, Wm(D, p, hw), Tn, V, h, dA);      // dHf
+      const T* dHf = reinterpret_cast<const T*>(head_base + HA.dHf);
       T* dHl = dHbuf[cur];
-      if (gpt) {
+      if constexpr (r32) {
+        norm_bwd_mixed(dHf, Hl, stf, Wf(D, p, gpt ? "lnf.g" : "nf.g"), nullptr, nullptr, dHl, dH32buf[0], Tn, h,
+                       gpt ? 0 : 1, G(D, p, gpt ? "lnf.g" : "nf.g"), gpt ? G(D, p, "lnf.b") : nullptr,
+                       gpt ? G(D, p, "h" + std::to_string(k * lps + lps - 1) + ".fc2.b") : nullptr, red, red_floats,
+                       st);
+        dH32 = dH32buf[0];
+      } else if (gpt) {
         // + the fc2 bias gradient of this stage's last layer (column sums of dHl)
-        norm_bwd<T>(dA, Hl, stf, Wf(D, p, "lnf.g"), nullptr, dHl, Tn, h, 0, G(D, p, "lnf.g"), G(D, p, "lnf.b"),
+        norm_bwd<T>(dHf, Hl, stf, Wf(D, p, "lnf.g"), nullptr, dHl, Tn, h, 0, G(D, p, "lnf.g"), G(D, p, "lnf.b"),
                     G(D, p, "h" + std::to_string(k * lps + lps - 1) + ".fc2.b"), red, red_floats, st);
       } else {
-        norm_bwd<T>(dA, Hl, stf, Wf(D, p, "nf.g"), nullptr, dHl, Tn, h, 1, G(D, p, "nf.g"), nullptr, nullptr, red,
+        norm_bwd<T>(dHf, Hl, stf, Wf(D, p, "nf.g"), nullptr, dHl, Tn, h, 1, G(D, p, "nf.g"), nullptr, nullptr, red,
                     red_floats, st);
       }
       dH = dHl;
@@ -412,8 +438,12 @@ struct Exec {
         lin_wgrad(dZ, A2, Tn, f, h, G(D, p, pre + "fc1.w"));
         if (!fuse_b1) colsum<T>(dZ, nullptr, nullptr, Tn, f, f, 0, G(D, p, pre + "fc1.b"), nullptr, red, st);
         lin_dgrad(dZ, Wm(D, p, pre + "fc1.w"), Tn, f, h, dA);               // dA2
-        norm_bwd<T>(dA, H1, st2, Wf(D, p, pre + "ln2.g"), dH, dH1, Tn, h, 0, G(D, p, pre + "ln2.g"),
-                    G(D, p, pre + "ln2.b"), G(D, p, pre + "proj.b"), red, red_floats, st);
+        if constexpr (r32)
+          norm_bwd_mixed(dA, H1, st2, Wf(D, p, pre + "ln2.g"), dH32 ? nullptr : dH, dH32, dH1, dH32buf[1], Tn, h, 0,
+                         G(D, p, pre + "ln2.g"), G(D, p, pre + "ln2.b"), G(D, p, pre + "proj.b"), red, red_floats, st);
+        else
+          norm_bwd<T>(dA, H1, st2, Wf(D, p, pre + "ln2.g"), dH, dH1, Tn, h, 0, G(D, p, pre + "ln2.g"),
+                      G(D, p, pre + "ln2.b"), G(D, p, pre + "proj.b"), red, red_floats, st);
         lin_wgrad(dH1, O, Tn, h, h, G(D, p, pre + "proj.w"));
         lin_dgrad(dH1, Wm(D, p, pre + "proj.w"), Tn, h, h, dO);
       } else {
@@ -424,8 +454,12 @@ struct Exec {
         norm_recompute<T>(H1, Wf(D, p, pre + "n2.g"), nullptr, A2, st2, Tn, h, m.norm_eps, 1, st);
         lin_wgrad(dZ, A2, Tn, 2 * f, h, G(D, p, pre + "gu.w"));
         lin_dgrad(dZ, Wm(D, p, pre + "gu.w"), Tn, 2 * f, h, dA);
-        norm_bwd<T>(dA, H1, st2, Wf(D, p, pre + "n2.g"), dH, dH1, Tn, h, 1, G(D, p, pre + "n2.g"), nullptr, nullptr,
-                    red, red_floats, st);
+        if constexpr (r32)
+          norm_bwd_mixed(dA, H1, st2, Wf(D, p, pre + "n2.g"), dH32 ? nullptr : dH, dH32, dH1, dH32buf[1], Tn, h, 1,
+                         G(D, p, pre + "n2.g"), nullptr, nullptr, red, red_floats, st);
+        else
+          norm_bwd<T>(dA, H1, st2, Wf(D, p, pre + "n2.g"), dH, dH1, Tn, h, 1, G(D, p, pre + "n2.g"), nullptr, nullptr,
+                      red, red_floats, st);
         lin_wgrad(dH1, O, Tn, h, h, G(D, p, pre + "o.w"));
         lin_dgrad(dH1, Wm(D, p, pre + "o.w"), Tn, h, h, dO);
       }
@@ -436,7 +470,15 @@ struct Exec {
       lin_wgrad(dQKV, A, Tn, 3 * h, h, G(D, p, pre + "qkv.w"));
       if (gpt) colsum<T>(dQKV, nullptr, nullptr, Tn, 3 * h, 3 * h, 0, G(D, p, pre + "qkv.b"), nullptr, red, st);
       lin_dgrad(dQKV, Wm(D, p, pre + "qkv.w"), Tn, 3 * h, h, dA);
-      if (gpt) {
+      if constexpr (r32) {
+        // the stage input's gradient leaves as a bf16 message (SG): no fp32 copy needed there
+        float* out32 = (li == 0 && k > 0) ? nullptr : dH32buf[0];
+        norm_bwd_mixed(dA, Hin, st1, Wf(D, p, pre + (gpt ? "ln1.g" : "n1.g")), nullptr, dH32buf[1], dHin, out32, Tn,
+                       h, gpt ? 0 : 1, G(D, p, pre + (gpt ? "ln1.g" : "n1.g")), gpt ? G(D, p, pre + "ln1.b") : nullptr,
+                       (gpt && li > 0) ? G(D, p, "h" + std::to_string(l - 1) + ".fc2.b") : nullptr, red, red_floats,
+                       st);
+        dH32 = out32;
+      } else if (gpt) {
         // + the previous layer's fc2 bias gradient (column sums of dHin) when it is on this stage
         norm_bwd<T>(dA, Hin, st1, Wf(D, p, pre + "ln1.g"), dH1, dHin, Tn, h, 0, G(D, p, pre + "ln1.g"),
                     G(D, p, pre + "ln1.b"), li > 0 ? G(D, p, "h" + std::to_string(l - 1) + ".fc2.b") : nullptr, red,
@@ -449,8 +491,12 @@ struct Exec {
       cur = (cur + 2) % 3;
     }
     if (k == 0) {
-      embed_bwd<T>(tok, s + 1, mbs, s, dH, h, G(D, p, gpt ? "wte" : "emb"), gpt ? G(D, p, "wpe") : nullptr,
-                   sc + BS.sort, st);
+      if (r32 && dH32)
+        embed_bwd<float>(tok, s + 1, mbs, s, dH32, h, G(D, p, gpt ? "wte" : "emb"), gpt ? G(D, p, "wpe") : nullptr,
+                         sc + BS.sort, st);
+      else
+        embed_bwd<T>(tok, s + 1, mbs, s, dH, h, G(D, p, gpt ? "wte" : "emb"), gpt ? G(D, p, "wpe") : nullptr,
+                     sc + BS.sort, st);
     }
   }
 
@@ -558,7 +604,9 @@ struct Exec {
           const int kind = grad ? 1 : 0;
           const auto src = msg_slot.at({kind, x.vstage, x.micro});
           Dev<T>& Sd = dev(src.first);
-          cudaStream_t rs = D.rx[kind];
+          // MARIO_PEER_RX=0: receive on the compute stream itself (no prefetch, fewer streams)
+          static const bool rx_streams = !getenv("MARIO_PEER_RX") || atoi(getenv("MARIO_PEER_RX")) != 0;
+          cudaStream_t rs = rx_streams ? D.rx[kind] : st;
           if (!grad && D.ck_free_set[x.slot]) CU(cudaStreamWaitEvent(rs, D.ck_free[x.slot], 0));
           if (grad) {
             const int i = D.rg_of[key];
@@ -568,9 +616,11 @@ struct Exec {
           CU(cudaMemcpyAsync(dst, send_slot(Sd, grad, src.second), msg_bytes, cudaMemcpyDeviceToDevice, rs));
           DRV(drv::write_flag(rs, flag_done(kind, x.vstage, x.micro), 1));
           consumed_walked.insert(std::make_tuple(kind, x.vstage, x.micro));
-          cudaEvent_t e = D.event();
-          CU(cudaEventRecord(e, rs));
-          CU(cudaStreamWaitEvent(st, e, 0));
+          if (rs != st) {
+            cudaEvent_t e = D.event();
+            CU(cudaEventRecord(e, rs));
+            CU(cudaStreamWaitEvent(st, e, 0));
+          }
         } else if (loopback) {
           Dev<T>& Sd = dev(x.peer);
           // the sender's part for this micro-batch: find via its held slots

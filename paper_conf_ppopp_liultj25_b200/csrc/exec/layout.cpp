@@ -46,10 +46,30 @@ HeadAct head_act_layout(const mario_model& m) {
   HeadAct H{};
   size_t o = 0;
   auto take = [&](size_t bytes) { size_t r = o; o = align_up(o + bytes); return r; };
+  (void)V;
   H.H_last = take(T * h * E);
   H.stf = take(T * 2 * 4);
+  H.dHf = take(T * h * E);
+  H.bytes = o;
+  return H;
+}
+
+HeadScratch head_scratch_layout(const mario_model& m) {
+  const size_t T = tokens_per_micro(m), E = elt_size(m), h = m.hidden, V = m.vocab;
+  const size_t budget = static_cast<size_t>(640) << 20;   // logits + dlogits of one chunk
+  size_t n = 1, rows = T;
+  while (rows * V * (4 + E) > budget && rows > 128) {
+    n *= 2;
+    rows = (T + n - 1) / n;
+    rows = (rows + 127) / 128 * 128;
+  }
+  HeadScratch H{};
+  size_t o = 0;
+  auto take = [&](size_t bytes) { size_t r = o; o = align_up(o + bytes); return r; };
+  H.rows = static_cast<int>(rows);
   H.Hf = take(T * h * E);
-  H.dlogits = take(T * V * E);
+  H.logits = take(rows * V * 4);
+  H.dlog = take(rows * V * E);
   H.bytes = o;
   return H;
 }
@@ -84,6 +104,7 @@ BwScratch bw_scratch_layout(const mario_model& m) {
   b.Dsc = take(static_cast<size_t>(m.n_heads) * T * 4);
   b.sort = take(T * 8 * 2);
   b.Arec = take(T * h * E);
+  for (int i = 0; i < 2; ++i) b.dH32[i] = take(m.dtype == MARIO_BF16 ? T * h * 4 : 0);
   // the attention backward's dS image (fa_bwd_dq_img: dQ from the stored dS, no S/dP recompute);
   // only where it stays small next to the rest of the scratch (not at s = 16384)
   b.dS_bytes = 0;
@@ -98,7 +119,7 @@ BwScratch bw_scratch_layout(const mario_model& m) {
 
 size_t bw_scratch_bytes(const mario_model& m) { return bw_scratch_layout(m).bytes; }
 
-size_t logits_bytes(const mario_model& m) { return align_up(tokens_per_micro(m) * m.vocab * 4); }
+size_t logits_bytes(const mario_model& m) { return head_scratch_layout(m).bytes; }
 
 size_t weight_copy_bytes(const mario_model& m, const std::vector<int32_t>& idx) {
   if (m.dtype != MARIO_BF16) return 0;

@@ -28,12 +28,24 @@ struct LayerTrans {
 };
 LayerTrans layer_trans_layout(const mario_model& m);
 
-// Head (last virtual stage): final-norm stats and output, dlogits.
+// Head (last virtual stage), what its BW needs: the last layer's output, the final-norm stats and
+// dHf = dloss/dHf. The logits never outlive the FW / RC that computes them (K13, fused head): the
+// head runs over token chunks (logits chunk -> softmax-CE -> dlogits chunk -> head dgrad rows of dHf
+// and head wgrad) inside the forward, since the loss ends the graph (BW needs only the
+// gradient of the stage output).
 struct HeadAct {
-  size_t H_last, stf, Hf, dlogits;
+  size_t H_last, stf, dHf;
   size_t bytes;
 };
 HeadAct head_act_layout(const mario_model& m);
+// Scratch of the fused head (per device with the last virtual stage): Hf [T, h], and a chunk of
+// `rows` tokens of fp32 logits [rows, V] and dlogits [rows, V] (compute dtype).
+struct HeadScratch {
+  size_t Hf, logits, dlog;
+  int rows;      // token rows per chunk (a power-of-2 split of T, multiple of 128 where T allows)
+  size_t bytes;
+};
+HeadScratch head_scratch_layout(const mario_model& m);
 
 size_t elt_size(const mario_model& m);
 size_t tokens_per_micro(const mario_model& m);
@@ -43,12 +55,13 @@ size_t cfw_work_bytes(const mario_model& m, int k, int K);       // transient CF
 // Backward scratch (shared by every BW of the rank): rotating dH buffers and per-layer grads.
 struct BwScratch {
   size_t dH[3], dA, dQKV, dO, dZ, dM, Dsc, sort, Arec;   // dM doubles as the G/M recompute buffer
+  size_t dH32[2];   // bf16 mode: the fp32 residual-gradient stream (reading A30); 0 bytes in fp32 mode
   size_t dS, dS_bytes;   // attention dS image (bf16, when the shape allows it and it is <= 1 GiB; else 0 bytes)
   size_t bytes;
 };
 BwScratch bw_scratch_layout(const mario_model& m);
 size_t bw_scratch_bytes(const mario_model& m);
-size_t logits_bytes(const mario_model& m);                      // fp32 [T, V]
+size_t logits_bytes(const mario_model& m);                      // head_scratch_layout(m).bytes
 size_t weight_copy_bytes(const mario_model& m, const std::vector<int32_t>& param_idx);
 
 }  // namespace mario

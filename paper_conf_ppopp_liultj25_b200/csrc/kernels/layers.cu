@@ -217,6 +217,37 @@ __global__ void embed_segsum_v8_k(const long long* keys, int Ttok, const __nv_bf
   }
 }
 
+// fp32 dH (the bf16 model's fp32 residual-gradient stream, reading A30), h % 4 == 0: the v8
+// kernel's segment walk with 4 columns per 16-byte load; same per-column summation order.
+__global__ void embed_segsum_f4_k(const long long* keys, int Ttok, const float* dH, int h, float* dwte) {
+  const int warp = (blockIdx.x * blockDim.x + threadIdx.x) / 32, lane = threadIdx.x % 32;
+  if (warp >= Ttok) return;
+  const long long v = keys[warp] / Ttok;
+  if (warp > 0 && keys[warp - 1] / Ttok == v) return;
+  float* out = dwte + v * h;
+  for (int j0 = warp; j0 < Ttok;) {
+    const int j = j0 + lane;
+    const long long kj = j < Ttok ? keys[j] : LLONG_MAX;
+    const bool in = j < Ttok && kj / Ttok == v;
+    const unsigned m = __ballot_sync(0xffffffffu, in);
+    const int cnt = __popc(~m) ? __ffs(~m) - 1 : 32;
+    const int pos = in ? static_cast<int>(kj % Ttok) : 0;
+    for (int c4 = lane; c4 < h / 4; c4 += 32) {
+      float4 acc = *reinterpret_cast<const float4*>(out + c4 * 4);
+      float4 sum = make_float4(0.f, 0.f, 0.f, 0.f);
+      for (int i = 0; i < cnt; ++i) {
+        const int p = __shfl_sync(0xffffffffu, pos, i);
+        const float4 u = *reinterpret_cast<const float4*>(dH + static_cast<long>(p) * h + c4 * 4);
+        sum.x += u.x; sum.y += u.y; sum.z += u.z; sum.w += u.w;
+      }
+      acc.x += sum.x; acc.y += sum.y; acc.z += sum.z; acc.w += sum.w;
+      *reinterpret_cast<float4*>(out + c4 * 4) = acc;
+    }
+    if (cnt < 32) break;
+    j0 += 32;
+  }
+}
+
 template <class T>
 __global__ void embed_pos_bwd_k(const T* dH, int B, int s, int h, float* dwpe) {
   const long n = static_cast<long>(s) * h;
@@ -492,6 +523,36 @@ __global__ void norm_bwd_dx_k(const T* dy, const T* x, const float* stats, const
     float d = (gp - sg - xh * sgx) * rstd;
     if (dres) d += ldf(dres + o + c);
     stf(dx + o + c, d);
+  }
+}
+
+// bf16 norm backward with the fp32 residual-gradient stream (any n; the row-pipelined kernel's
+// fallback): dx = norm'(dy) + (dres32 | dres) written as bf16 and, if dx32, as fp32.
+__global__ void norm_bwd_mixed_k(const __nv_bfloat16* dy, const __nv_bfloat16* x, const float* stats, const float* g,
+                                 const __nv_bfloat16* dres, const float* dres32, __nv_bfloat16* dx, float* dx32,
+                                 int rows, int n, int rms) {
+  const int row = blockIdx.x * (blockDim.x / 32) + threadIdx.x / 32, lane = threadIdx.x % 32;
+  if (row >= rows) return;
+  const long o = static_cast<long>(row) * n;
+  const float mean = stats[2 * row], rstd = stats[2 * row + 1];
+  float sg = 0.f, sgx = 0.f;
+  for (int c = lane; c < n; c += 32) {
+    const float gp = __bfloat162float(dy[o + c]) * g[c];
+    const float xh = (__bfloat162float(x[o + c]) - mean) * rstd;
+    sg += gp;
+    sgx += gp * xh;
+  }
+  sg = warp_sum(sg) / n;
+  sgx = warp_sum(sgx) / n;
+  if (rms) sg = 0.f;
+  for (int c = lane; c < n; c += 32) {
+    const float gp = __bfloat162float(dy[o + c]) * g[c];
+    const float xh = (__bfloat162float(x[o + c]) - mean) * rstd;
+    float d = (gp - sg - xh * sgx) * rstd;
+    if (dres32) d += dres32[o + c];
+    else if (dres) d += __bfloat162float(dres[o + c]);
+    dx[o + c] = __float2bfloat16_rn(d);
+    if (dx32) dx32[o + c] = d;
   }
 }
 
@@ -1127,7 +1188,7 @@ __global__ void swiglu_bwd_v8_k(const __nv_bfloat16* GU, const __nv_bfloat16* dM
 // ---------------------------------------------------------------- softmax-CE
 template <class T>
 __global__ void softmax_ce_k(const float* logits, const int32_t* tok, int ld_tok, int s, int V, float inv_ntok,
-                             T* dlogits, float* row_loss) {
+                             T* dlogits, float* row_loss, long row0) {
   __shared__ float sm[32], sl[32];
   const long r = blockIdx.x;
   const float* z = logits + r * V;
@@ -1157,7 +1218,7 @@ __global__ void softmax_ce_k(const float* logits, const int32_t* tok, int ld_tok
   }
   __syncthreads();
   const float lse = sm[0] + logf(sl[0]);
-  const int b = static_cast<int>(r / s), t = static_cast<int>(r % s);
+  const int b = static_cast<int>((row0 + r) / s), t = static_cast<int>((row0 + r) % s);
   const int y = tok[static_cast<long>(b) * ld_tok + t + 1];
   for (int c = threadIdx.x; c < V; c += blockDim.x) {
     const float p = __expf(z[c] - lse);
@@ -1261,7 +1322,10 @@ void embed_bwd(const int32_t* tok, int ld_tok, int B, int s, const T* dH, int h,
       note_launch();
     }
   } else {
-    embed_segsum_k<T><<<cdiv(static_cast<long>(Ttok) * 32, 256), 256, 0, st>>>(keys, Ttok, dH, h, dwte);
+    if (h % 4 == 0 && (reinterpret_cast<uintptr_t>(dH) & 15) == 0 && (reinterpret_cast<uintptr_t>(dwte) & 15) == 0)
+      embed_segsum_f4_k<<<cdiv(static_cast<long>(Ttok) * 32, 256), 256, 0, st>>>(keys, Ttok, dH, h, dwte);
+    else
+      embed_segsum_k<T><<<cdiv(static_cast<long>(Ttok) * 32, 256), 256, 0, st>>>(keys, Ttok, dH, h, dwte);
     note_launch();
   }
   if (dwpe) {
@@ -1400,6 +1464,22 @@ void norm_bwd(const T* dy, const T* x, const float* stats, const float* g, const
   if (dsum) colsum<T>(dx, nullptr, nullptr, rows, n, n, 0, dsum, nullptr, partial, st);
 }
 
+void norm_bwd_mixed(const __nv_bfloat16* dy, const __nv_bfloat16* x, const float* stats, const float* g,
+                    const __nv_bfloat16* dres, const float* dres32, __nv_bfloat16* dx, float* dx32, int rows, int n,
+                    int rms, float* dg, float* db, float* dsum, float* partial, size_t partial_floats, cudaStream_t st) {
+  KScope ks_(K_NORM, st);
+  if (norm_bwd_pipe_mixed(dy, x, stats, g, dres, dres32, dx, dx32, rows, n, rms, dg, db, dsum, partial, partial_floats,
+                          st))
+    return;
+  norm_bwd_mixed_k<<<cdiv(rows, 8), 256, 0, st>>>(dy, x, stats, g, dres, dres32, dx, dx32, rows, n, rms);
+  note_launch();
+  colsum<__nv_bfloat16>(dy, x, stats, rows, n, n, rms ? 2 : 1, dg, db, partial, st);
+  if (dsum) {
+    if (dx32) colsum<float>(dx32, nullptr, nullptr, rows, n, n, 0, dsum, nullptr, partial, st);
+    else colsum<__nv_bfloat16>(dx, nullptr, nullptr, rows, n, n, 0, dsum, nullptr, partial, st);
+  }
+}
+
 template <class T>
 void attn_fwd(const T* qkv, T* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st) {
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
@@ -1459,12 +1539,12 @@ void swiglu_bwd(const T* GU, const T* dM, T* dGU, int rows, int f, cudaStream_t 
 }
 template <class T>
 void softmax_ce(const float* logits, const int32_t* tok, int ld_tok, int s, int rows, int V, float inv_ntok,
-                T* dlogits, float* row_loss, cudaStream_t st) {
+                T* dlogits, float* row_loss, cudaStream_t st, long row0) {
   KScope ks_(K_CE, st);
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
-    if (softmax_ce_fast(logits, tok, ld_tok, s, rows, V, inv_ntok, dlogits, row_loss, st)) return;
+    if (softmax_ce_fast(logits, tok, ld_tok, s, rows, V, inv_ntok, dlogits, row_loss, st, row0)) return;
   }
-  softmax_ce_k<T><<<rows, 512, 0, st>>>(logits, tok, ld_tok, s, V, inv_ntok, dlogits, row_loss);
+  softmax_ce_k<T><<<rows, 512, 0, st>>>(logits, tok, ld_tok, s, V, inv_ntok, dlogits, row_loss, row0);
   note_launch();
 }
 template <class T>
@@ -1533,7 +1613,8 @@ void sum_copies_f32(float* dst, const CopySrcs& srcs, size_t n, cudaStream_t st)
   template void rope<T>(T*, int, int, int, int, float, int, cudaStream_t);                                           \
   template void swiglu_fwd<T>(const T*, T*, int, int, cudaStream_t);                                                 \
   template void swiglu_bwd<T>(const T*, const T*, T*, int, int, cudaStream_t);                                       \
-  template void softmax_ce<T>(const float*, const int32_t*, int, int, int, int, float, T*, float*, cudaStream_t); \
+  template void softmax_ce<T>(const float*, const int32_t*, int, int, int, int, float, T*, float*, cudaStream_t,    \
+                              long);                                                                                \
   template void gelu_fwd<T>(const T*, T*, size_t, cudaStream_t);
 INST(float)
 INST(__nv_bfloat16)

@@ -33,6 +33,17 @@ template <class T> void norm_bwd_dx(const T* dy, const T* x, const float* stats,
 template <class T> void norm_bwd(const T* dy, const T* x, const float* stats, const float* g, const T* dres, T* dx,
                                  int rows, int n, int rms, float* dg, float* db, float* dsum, float* partial,
                                  size_t partial_floats, cudaStream_t st);
+// bf16 norm backward on the fp32 residual-gradient stream (reading A30): dx = norm'(dy) + residual,
+// the residual taken from dres32 (fp32) if given, else dres (bf16), else none; dx is written as the
+// bf16 operand of the following GEMMs and, if dx32 != NULL, in fp32 for the next residual add;
+// dg / db / dsum as norm_bwd (dsum sums the fp32 dx when dx32 is given).
+void norm_bwd_mixed(const __nv_bfloat16* dy, const __nv_bfloat16* x, const float* stats, const float* g,
+                    const __nv_bfloat16* dres, const float* dres32, __nv_bfloat16* dx, float* dx32, int rows, int n,
+                    int rms, float* dg, float* db, float* dsum, float* partial, size_t partial_floats, cudaStream_t st);
+bool norm_bwd_pipe_mixed(const __nv_bfloat16* dy, const __nv_bfloat16* x, const float* stats, const float* g,
+                         const __nv_bfloat16* dres, const float* dres32, __nv_bfloat16* dx, float* dx32, int rows,
+                         int n, int rms, float* dg, float* db, float* dsum, float* partial, size_t partial_floats,
+                         cudaStream_t st);
 extern int g_norm_tile;
 // Row-pipelined bf16 kernels (rowpipe.cu); false = shape not supported (caller falls back).
 bool norm_pipe_supported(int n);
@@ -42,7 +53,7 @@ bool norm_bwd_pipe(const __nv_bfloat16* dy, const __nv_bfloat16* x, const float*
                    const __nv_bfloat16* dres, __nv_bfloat16* dx, int rows, int n, int rms, float* dg, float* db,
                    float* dsum, float* partial, size_t partial_floats, cudaStream_t st);
 bool softmax_ce_fast(const float* logits, const int32_t* tok, int ld_tok, int s, int rows, int V, float inv_ntok,
-                     __nv_bfloat16* dlogits, float* row_loss, cudaStream_t st);
+                     __nv_bfloat16* dlogits, float* row_loss, cudaStream_t st, long row0 = 0);
 // Column reductions into fp32 grads (+=): mode 0: out0 += sum_r a[r,c]
 // mode 1 (LN): out0 += sum dy*xhat, out1 += sum dy; mode 2 (RMS): out0 += sum dy*xhat.
 // out[c] += sum_b partial[b][c] over nblk row blocks (fixed order): the second pass of column sums
@@ -75,9 +86,10 @@ template <class T> void swiglu_bwd(const T* GU, const T* dM, T* dGU, int rows, i
 template <class T> void gelu_fwd(const T* Z, T* G, size_t n, cudaStream_t st);
 
 // Softmax cross-entropy over fp32 logits [rows, V]: row_loss[r] = lse - z_y;
-// dlogits (T) = (softmax - onehot) * inv_ntok. labels = tokens[:, 1:] of the micro-batch.
+// dlogits (T) = (softmax - onehot) * inv_ntok. labels = tokens[:, 1:] of the micro-batch; local row r
+// is the micro-batch's token row0 + r (a chunk of the fused head).
 template <class T> void softmax_ce(const float* logits, const int32_t* tok, int ld_tok, int s, int rows, int V,
-                                   float inv_ntok, T* dlogits, float* row_loss, cudaStream_t st);
+                                   float inv_ntok, T* dlogits, float* row_loss, cudaStream_t st, long row0 = 0);
 // out[0] (double) = sum of row_loss[0..rows) in a fixed order.
 void loss_reduce(const float* row_loss, int rows, double* out, cudaStream_t st);
 

@@ -258,15 +258,20 @@ __global__ void __launch_bounds__(1024) norm_fwd_pipe_k(const bf16* __restrict__
 // memory (row sums), phase 2 (after the barrier) re-reads dy, x, dres and writes dx, so nothing
 // but the column accumulators stays in registers; a slot is refilled at the NEXT iteration's
 // barrier, when every thread is past its phase 2. Stats of the CTA's range are staged in smem.
-template <int R, int V>   // V: 16-byte chunks per thread (chunks t, t + nt, ...), amortizing the per-row work
+// RES: residual input dres none (0) / bf16 (1) / fp32 (2); OUT32: also write dx in fp32 (dx32).
+// With the fp32 residual-gradient stream (reading A30) the layer-to-layer dH chain stays fp32 and
+// the bf16 dx is only the operand copy of the following GEMMs; the column sums of dx (a bias
+// gradient) are then taken over the fp32 values.
+template <int R, int V, int RES, bool OUT32>   // V: 16-byte chunks per thread (t, t + nt, ...)
 __global__ void __launch_bounds__(640) norm_bwd_pipe_k(const bf16* __restrict__ dy, const bf16* __restrict__ x,
                                                        const float* __restrict__ stats, const float* __restrict__ g,
-                                                       const bf16* __restrict__ dres, bf16* __restrict__ dx, int rows,
+                                                       const void* __restrict__ dres, bf16* __restrict__ dx,
+                                                       float* __restrict__ dx32, int rows,
                                                        int n, int rms, float* __restrict__ partial, int nblk,
                                                        int sum_out, int S, int max_range) {
   extern __shared__ __align__(128) uint8_t smem_raw[];
-  const int nin = dres ? 3 : 2;
-  const int row_bytes = n * 2, sb = nin * row_bytes;
+  const int row_bytes = n * 2, res_bytes = RES == 2 ? n * 4 : (RES == 1 ? n * 2 : 0);
+  const int sb = 2 * row_bytes + res_bytes;
   uint8_t* stage0 = smem_raw;
   uint64_t* bar = reinterpret_cast<uint64_t*>(smem_raw + static_cast<size_t>(S) * sb);
   float* red = reinterpret_cast<float*>(bar + S);            // [2][32][R][2]
@@ -282,7 +287,8 @@ __global__ void __launch_bounds__(640) norm_bwd_pipe_k(const bf16* __restrict__ 
     mbar_arrive_expect_tx(&bar[sl], sb);
     bulk_g2s(buf, dy + static_cast<long>(r) * n, row_bytes, &bar[sl]);
     bulk_g2s(buf + row_bytes, x + static_cast<long>(r) * n, row_bytes, &bar[sl]);
-    if (dres) bulk_g2s(buf + 2 * row_bytes, dres + static_cast<long>(r) * n, row_bytes, &bar[sl]);
+    if (RES) bulk_g2s(buf + 2 * row_bytes, static_cast<const uint8_t*>(dres) + static_cast<long>(r) * res_bytes,
+                      res_bytes, &bar[sl]);
   };
   if (t == 0) {
     for (int i = 0; i < S; ++i) mbar_init(&bar[i], 1);
@@ -375,8 +381,13 @@ __global__ void __launch_bounds__(640) norm_bwd_pipe_k(const bf16* __restrict__ 
         float d[8], xh[8], rr[8];
         unpack8(lds128(buf + off), d);
         unpack8(lds128(buf + row_bytes + off), xh);
-        if (dres) {
+        if (RES == 1) {
           unpack8(lds128(buf + 2 * row_bytes + off), rr);
+        } else if (RES == 2) {
+          const float4 r0 = *reinterpret_cast<const float4*>(buf + 2 * row_bytes + 2 * off);
+          const float4 r1 = *reinterpret_cast<const float4*>(buf + 2 * row_bytes + 2 * off + 16);
+          rr[0] = r0.x; rr[1] = r0.y; rr[2] = r0.z; rr[3] = r0.w;
+          rr[4] = r1.x; rr[5] = r1.y; rr[6] = r1.z; rr[7] = r1.w;
         } else {
 #pragma unroll
           for (int j = 0; j < 8; ++j) rr[j] = 0.f;
@@ -392,9 +403,19 @@ __global__ void __launch_bounds__(640) norm_bwd_pipe_k(const bf16* __restrict__ 
         }
         const uint4 pk = pack8(o);
         *reinterpret_cast<uint4*>(dx + static_cast<long>(r) * n + cidx * 8) = pk;
+        if (OUT32) {
+          float* d32 = dx32 + static_cast<long>(r) * n + cidx * 8;
+          *reinterpret_cast<float4*>(d32) = make_float4(o[0], o[1], o[2], o[3]);
+          *reinterpret_cast<float4*>(d32 + 4) = make_float4(o[4], o[5], o[6], o[7]);
+        }
         if (sum_out) {
           float qv[8];
-          unpack8(pk, qv);
+          if (OUT32) {
+#pragma unroll
+            for (int j = 0; j < 8; ++j) qv[j] = o[j];
+          } else {
+            unpack8(pk, qv);
+          }
 #pragma unroll
           for (int j = 0; j < 8; j += 2) {
             const float2 a = add2(f2(ao[k][j], ao[k][j + 1]), f2(qv[j], qv[j + 1]));
@@ -434,14 +455,14 @@ template <int NV>
 __global__ void __launch_bounds__(512, 1) softmax_ce_reg_k(const float* __restrict__ logits,
                                                            const int32_t* __restrict__ tok, int ld_tok, int s, int V,
                                                            float inv_ntok, bf16* __restrict__ dlogits,
-                                                           float* __restrict__ row_loss) {
+                                                           float* __restrict__ row_loss, long row0) {
   __shared__ float red[2][16];
   constexpr float LOG2E = 1.4426950408889634f;
   const long r = blockIdx.x;
   const int t = threadIdx.x, w = t / 32, lane = t % 32;
   const int nv4 = V / 4;
   const float4* z = reinterpret_cast<const float4*>(logits + r * V);
-  const int bi = static_cast<int>(r / s), ti = static_cast<int>(r % s);
+  const int bi = static_cast<int>((row0 + r) / s), ti = static_cast<int>((row0 + r) % s);
   const int y = tok[static_cast<long>(bi) * ld_tok + ti + 1];
   float zy = 0.f;
   if (t == 0) zy = logits[r * V + y];
@@ -579,11 +600,11 @@ bool norm_fwd_pipe(const bf16* x, const float* g, const float* b, bf16* y, float
   return true;
 }
 
-template <int V>
-bool norm_bwd_pipe_v(const bf16* dy, const bf16* x, const float* stats, const float* g, const bf16* dres, bf16* dx,
-                     int rows, int n, int rms, float* dg, float* db, float* dsum, float* partial, size_t partial_floats,
-                     cudaStream_t st) {
-  const int nt = ((n / (8 * V) + 31) / 32) * 32, nin = dres ? 3 : 2, sb = nin * n * 2;
+template <int V, int RES, bool OUT32>
+bool norm_bwd_pipe_v(const bf16* dy, const bf16* x, const float* stats, const float* g, const void* dres, bf16* dx,
+                     float* dx32, int rows, int n, int rms, float* dg, float* db, float* dsum, float* partial,
+                     size_t partial_floats, cudaStream_t st) {
+  const int nt = ((n / (8 * V) + 31) / 32) * 32, sb = 4 * n + (RES == 2 ? 4 * n : (RES == 1 ? 2 * n : 0));
   if (nt > 640) return false;
   static const int ring = getenv("MARIO_NORM_BWD_RING") ? atoi(getenv("MARIO_NORM_BWD_RING")) : 49152;
   static const int smax = getenv("MARIO_NORM_BWD_SMAX") ? atoi(getenv("MARIO_NORM_BWD_SMAX")) : 6;
@@ -592,12 +613,14 @@ bool norm_bwd_pipe_v(const bf16* dy, const bf16* x, const float* stats, const fl
   S -= S % kPipeR;
   static bool attr = false;
   if (!attr) {
-    cudaFuncSetAttribute(norm_bwd_pipe_k<kPipeR, V>, cudaFuncAttributeMaxDynamicSharedMemorySize, 220 * 1024);
+    cudaFuncSetAttribute(norm_bwd_pipe_k<kPipeR, V, RES, OUT32>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                         220 * 1024);
     attr = true;
   }
   // the stats of a CTA's range are staged in shared memory: size for the smallest grid we may use
   const size_t base = pipe_smem_bytes(S, sb);
-  int nblk = occ_grid(norm_bwd_pipe_k<kPipeR, V>, nt, base + 8 * static_cast<size_t>(cdivl(rows, device_sms())));
+  int nblk = occ_grid(norm_bwd_pipe_k<kPipeR, V, RES, OUT32>, nt,
+                      base + 8 * static_cast<size_t>(cdivl(rows, device_sms())));
   if (dg) {
     const long cap = static_cast<long>(partial_floats / (3 * static_cast<size_t>(n)));
     if (cap < 1) return false;
@@ -607,8 +630,9 @@ bool norm_bwd_pipe_v(const bf16* dy, const bf16* x, const float* stats, const fl
   const int max_range = cdivl(rows, nblk) + 1;
   const size_t smem = base + 8 * static_cast<size_t>(max_range);
   if (smem > 220 * 1024) return false;
-  norm_bwd_pipe_k<kPipeR, V><<<nblk, nt, smem, st>>>(dy, x, stats, g, dres, dx, rows, n, rms, dg ? partial : nullptr,
-                                                     nblk, dsum ? 1 : 0, S, max_range);
+  norm_bwd_pipe_k<kPipeR, V, RES, OUT32><<<nblk, nt, smem, st>>>(dy, x, stats, g, dres, dx, dx32, rows, n, rms,
+                                                                 dg ? partial : nullptr, nblk, dsum ? 1 : 0, S,
+                                                                 max_range);
   note_launch();
   if (dg) {
     colsum_reduce(partial, nblk, n, dg, rms ? nullptr : db, dsum, st);
@@ -624,18 +648,47 @@ bool norm_bwd_pipe(const bf16* dy, const bf16* x, const float* stats, const floa
   // 16-byte chunks per thread (MARIO_NORM_BWD_V)
   static const int vsel = getenv("MARIO_NORM_BWD_V") ? atoi(getenv("MARIO_NORM_BWD_V")) : 2;
   if (vsel == 2 && n % 2048 == 0)   // measured: h 4096 73.8 -> 63.9 us, h 2048 equal, h 5120 slower
-    return norm_bwd_pipe_v<2>(dy, x, stats, g, dres, dx, rows, n, rms, dg, db, dsum, partial, partial_floats, st);
-  return norm_bwd_pipe_v<1>(dy, x, stats, g, dres, dx, rows, n, rms, dg, db, dsum, partial, partial_floats, st);
+    return dres ? norm_bwd_pipe_v<2, 1, false>(dy, x, stats, g, dres, dx, nullptr, rows, n, rms, dg, db, dsum, partial,
+                                                partial_floats, st)
+                : norm_bwd_pipe_v<2, 0, false>(dy, x, stats, g, nullptr, dx, nullptr, rows, n, rms, dg, db, dsum,
+                                                partial, partial_floats, st);
+  return dres ? norm_bwd_pipe_v<1, 1, false>(dy, x, stats, g, dres, dx, nullptr, rows, n, rms, dg, db, dsum, partial,
+                                              partial_floats, st)
+              : norm_bwd_pipe_v<1, 0, false>(dy, x, stats, g, nullptr, dx, nullptr, rows, n, rms, dg, db, dsum, partial,
+                                              partial_floats, st);
+}
+
+bool norm_bwd_pipe_mixed(const bf16* dy, const bf16* x, const float* stats, const float* g, const bf16* dres,
+                         const float* dres32, bf16* dx, float* dx32, int rows, int n, int rms, float* dg, float* db,
+                         float* dsum, float* partial, size_t partial_floats, cudaStream_t st) {
+  if (!norm_pipe_supported(n)) return false;
+  if (rows <= 0) return true;
+  static const int vsel = getenv("MARIO_NORM_BWD_V") ? atoi(getenv("MARIO_NORM_BWD_V")) : 2;
+  const bool v2 = vsel == 2 && n % 2048 == 0;
+#define NB_CASE(VV, RR, OO, DR)                                                                                  \
+  return norm_bwd_pipe_v<VV, RR, OO>(dy, x, stats, g, DR, dx, dx32, rows, n, rms, dg, db, dsum, partial,        \
+                                     partial_floats, st)
+  if (v2) {
+    if (dres32) { if (dx32) NB_CASE(2, 2, true, dres32); NB_CASE(2, 2, false, dres32); }
+    if (dres) { if (dx32) NB_CASE(2, 1, true, dres); NB_CASE(2, 1, false, dres); }
+    if (dx32) NB_CASE(2, 0, true, nullptr);
+    NB_CASE(2, 0, false, nullptr);
+  }
+  if (dres32) { if (dx32) NB_CASE(1, 2, true, dres32); NB_CASE(1, 2, false, dres32); }
+  if (dres) { if (dx32) NB_CASE(1, 1, true, dres); NB_CASE(1, 1, false, dres); }
+  if (dx32) NB_CASE(1, 0, true, nullptr);
+  NB_CASE(1, 0, false, nullptr);
+#undef NB_CASE
 }
 
 bool softmax_ce_fast(const float* logits, const int32_t* tok, int ld_tok, int s, int rows, int V, float inv_ntok,
-                     bf16* dlogits, float* row_loss, cudaStream_t st) {
+                     bf16* dlogits, float* row_loss, cudaStream_t st, long row0) {
   if (V % 4 || V < 4) return false;
   const int need = cdivl(V / 4, 512);
   if (rows <= 0) return true;
 #define CE_CASE(NV)                                                                                            \
   if (need <= NV) {                                                                                            \
-    softmax_ce_reg_k<NV><<<rows, 512, 0, st>>>(logits, tok, ld_tok, s, V, inv_ntok, dlogits, row_loss);        \
+    softmax_ce_reg_k<NV><<<rows, 512, 0, st>>>(logits, tok, ld_tok, s, V, inv_ntok, dlogits, row_loss, row0);  \
     note_launch();                                                                                             \
     return true;                                                                                               \
   }
