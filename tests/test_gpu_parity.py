@@ -131,21 +131,37 @@ def test_deterministic_repeat():
 # ---------------------------------------------------------------------------------------------
 # Full-width parity: the BASELINE.json model widths (h, heads, f, V, s) truncated to 2 layers so
 # the fp32 CPU oracle finishes in seconds; run through the same bf16 kernels and launch shapes
-# bench.py times (tcgen05 GEMMs incl. CTA-pair tiles, tcgen05 attention backward).
-# (name, cfg, scheme, S, N, v, l2 tol, inf guard). LLaMA2-7B width: bf16 *storage* alone moves the
-# fp32 definition by 2.37% (l2) / 2.29% (inf) on h1.qkv.w at s = 2048 (tools/bf16_storage_error.py
-# lin,norm,attn 2048), so its bound is set at ~1.7x that floor (A19).
+# bench.py times (CTA-pair tcgen05 GEMMs, tcgen05 attention with the dS image, row-pipelined norms
+# with the fp32 residual-gradient stream, the fused token-chunked head).
+# GPT-3 widths are held to north_star's bound as stated: per tensor ||g-o||_inf/||o||_inf <= 2e-2
+# (reading A19; observed 0.8-1.0%). LLaMA2 widths: see LLAMA_FULL below.
+# (name, cfg, scheme, S, N, v)
+FULL_GPT = [
+    ("gpt3-1.3b", synth.with_(synth.GPT3_1P3B, n_layers=2, micro_batch=1), "1f1b", 2, 2, 1),
+    ("gpt3-2.7b-chimera", synth.with_(synth.GPT3_2P7B, n_layers=2, micro_batch=1), "chimera", 2, 2, 1),
+    ("gpt3-1.3b-interleave", synth.with_(synth.GPT3_1P3B, n_layers=4, micro_batch=1), "interleave", 2, 2, 2),
+]
+
+
+@pytest.mark.slow
+@pytest.mark.parametrize("name,cfg,scheme,S,N,v", FULL_GPT, ids=[f[0] for f in FULL_GPT])
+def test_full_width_parity_bf16_gpt(name, cfg, scheme, S, N, v):
+    params = synth.make_weights(cfg)
+    toks = synth.make_tokens(cfg, N)
+    loss, grads, _ = run_plan(cfg, S, N, scheme, "mario", "bf16", params, toks, chunks=v)
+    l_o, g_o = om.step(cfg, rounded(params), toks, N, np.float32)
+    wi, wl = check(loss, grads, l_o, g_o, 2e-2)
+    print(f"[full-width {name}] loss {loss:.6f} vs {l_o:.6f}; worst inf-rel {wi}; worst l2-rel {wl}")
+
+
+# LLaMA2 widths (h 4096 / 5120): the oracle-only storage experiment tests/tools/bf16_floor.py shows
+# that storing the tensors the GPU path stores in bf16 (each one a bf16 tensor-core operand or a
+# bf16 activation) moves the fp32 definition's worst element above 2e-2 by itself (reading A19,
+# DESIGN.md); these cases are bounded relative to that measured floor.
+# (name, cfg, scheme, S, N, v, l2 tol, inf guard)
 FULL = [
-    ("gpt3-1.3b", synth.with_(synth.GPT3_1P3B, n_layers=2, micro_batch=1), "1f1b", 2, 2, 1, 2e-2, 5e-2),
     ("llama2-7b-s2048", synth.with_(synth.LLAMA2_7B, n_layers=2, micro_batch=1, seq_len=2048), "1f1b", 2, 2, 1,
      4e-2, 6e-2),
-    ("gpt3-2.7b-chimera", synth.with_(synth.GPT3_2P7B, n_layers=2, micro_batch=1), "chimera", 2, 2, 1, 2e-2, 5e-2),
-    # Interleave v = 2 at GPT-3 1.3B width (4 layers = 2 stages x 2 chunks; observed l2 0.93%, inf 0.86%)
-    ("gpt3-1.3b-interleave", synth.with_(synth.GPT3_1P3B, n_layers=4, micro_batch=1), "interleave", 2, 2, 2,
-     2e-2, 5e-2),
-    # LLaMA2-13B width (h 5120, 40 heads, f 13824; cfg 5's shapes at s 1024): bf16 storage alone moves
-    # the fp32 definition by 2.91% l2 (h1.n1.g) / 2.81% inf (h1.qkv.w) (tools/bf16_storage_error.py
-    # lin,norm,attn 1024 13b); GPU observed 3.42% / 3.74%; bound ~1.7x the floor (A19)
     ("llama2-13b-s1024", synth.with_(synth.LLAMA2_13B, n_layers=2, micro_batch=1, seq_len=1024), "1f1b", 2, 2, 1,
      5e-2, 6e-2),
 ]

@@ -61,7 +61,7 @@ def test_s8_bf16_mario_bitwise_base(scheme, cfg, N, v):
 def test_s8_bf16_cfg2_width():
     """GPT-3 1.3B width (h 2048, 16 heads, s 2048, V 50304), L = 8 (one layer per stage), S = 8,
     N = 8, mbs 1, Mario 1F1B: the CTA-pair GEMM and the tcgen05 attention with the dS image run at
-    the shapes bench.py times; held to the A19 bound of the full-width cases."""
+    the shapes bench.py times; held to north_star's 2e-2 per-tensor inf-norm bound (A19)."""
     cfg = synth.with_(synth.GPT3_1P3B, n_layers=8, micro_batch=1)
     params = synth.make_weights(cfg)
     toks = synth.make_tokens(cfg, 8)
@@ -69,5 +69,5 @@ def test_s8_bf16_cfg2_width():
     base = run_plan(cfg, 8, 8, "1f1b", "base", "bf16", params, toks)[2]
     assert np.array_equal(flat, base)
     l_o, g_o = om.step(cfg, rounded(params), toks, 8, np.float32)
-    wi, wl = check(loss, grads, l_o, g_o, 2e-2, norm="l2", inf_guard=5e-2)
+    wi, wl = check(loss, grads, l_o, g_o, 2e-2)
     print(f"[s8 cfg2-width] loss {loss:.6f} vs {l_o:.6f}; worst inf-rel {wi}; worst l2-rel {wl}")
