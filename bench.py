@@ -34,6 +34,25 @@ import synth  # noqa: E402
 METRIC = "samples/s (GPT-3 1.3B, seq 2048, GBS 128, Mario 1F1B plan, bf16)"
 UNIT = "samples/s"
 
+# BASELINE.json configs[1..4]. The default (driver) line is cfg2; the others are
+# extra lines: at 1 GPU = 1 stage every scheme is gradient accumulation (1F1B reference point, d3),
+# and --emulate measures the config's own scheme at 8 stages on SM partitions of this GPU.
+CONFIGS = {
+    "cfg2": dict(model=lambda: synth.GPT3_1P3B, micro=32, scheme="1f1b", chunks=1, name="gpt3-1.3b",
+                 workload="cfg2: GPT-3 1.3B, seq 2048, 1F1B+Mario, bf16 (BASELINE.json configs[1])"),
+    "cfg3": dict(model=lambda: synth.LLAMA2_7B, micro=32, scheme="interleave", chunks=2, name="llama2-7b",
+                 workload="cfg3: LLaMA2 7B, seq 4096, Interleave (2 chunks/GPU) + Mario, bf16 (BASELINE.json "
+                          "configs[2])"),
+    "cfg4": dict(model=lambda: synth.GPT3_2P7B, micro=32, scheme="chimera", chunks=1, name="gpt3-2.7b",
+                 workload="cfg4: GPT-3 2.7B, seq 2048, Chimera + Mario, bf16 (BASELINE.json configs[3])"),
+    # cfg 5 does not fit one GPU even uncapped: its 1-GPU line runs 2 of the 40 layers (+ head)
+    # at s 16384 and reports the per-layer time; no 8-stage emulation (8 x up to 40 GB > one GPU's HBM)
+    "cfg5": dict(model=lambda: synth.with_(synth.LLAMA2_13B, n_layers=2), micro=2, scheme="1f1b", chunks=1,
+                 name="llama2-13b (2 of 40 layers)",
+                 workload="cfg5 per-layer: LLaMA2 13B width, seq 16384, 2 layers + head, 1 GPU (BASELINE.json "
+                          "configs[4], which needs 8 GPUs)"),
+}
+
 
 def parse():
     ap = argparse.ArgumentParser()
@@ -44,8 +63,9 @@ def parse():
     ap.add_argument("--level", default="mario", choices=["base", "ckpt", "mario"])
     ap.add_argument("--dp", type=int, default=1,
                     help="PP x DP: gpus = stages * dp; the global batch stays --micro micro-batches (strong)")
-    ap.add_argument("--scheme", default="1f1b")
-    ap.add_argument("--micro", type=int, default=32)
+    ap.add_argument("--scheme", default=None, help="default: the config's scheme (1F1B at 1 stage)")
+    ap.add_argument("--micro", type=int, default=None, help="micro-batches per iteration (default: the config's)")
+    ap.add_argument("--config", default="cfg2", choices=sorted(CONFIGS))
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--emulate-only", action="store_true", help="only the emulated-pipeline measurement")
@@ -156,8 +176,9 @@ def run_reference(args, cfg, gbs):
 
 
 def config_dict(cfg, args, gbs):
-    return {"workload": "cfg2: GPT-3 1.3B, seq 2048, 1F1B+Mario, bf16 (BASELINE.json configs[1])",
-            "model": "gpt3-1.3b", "layers": cfg.n_layers, "hidden": cfg.hidden, "heads": cfg.n_heads,
+    C = CONFIGS[args.config]
+    return {"workload": C["workload"],
+            "model": C["name"], "layers": cfg.n_layers, "hidden": cfg.hidden, "heads": cfg.n_heads,
             "global_batch": gbs, "seq_len": cfg.seq_len, "micro_batch": cfg.micro_batch,
             "microbatches": args.micro, "stages": args.gpus // args.dp, "scheme": args.scheme, "level": args.level,
             "parallelism": f"pp{args.gpus // args.dp}" + (f"xdp{args.dp}" if args.dp > 1 else ""),
@@ -331,7 +352,10 @@ def device_sms(torch):
 
 def main():
     args = parse()
-    cfg = synth.GPT3_1P3B
+    C = CONFIGS[args.config]
+    cfg = C["model"]()
+    if args.micro is None:
+        args.micro = C["micro"]
     gbs = args.micro * cfg.micro_batch
     if args.impl == "reference":
         run_reference(args, cfg, gbs)
@@ -345,7 +369,8 @@ def main():
         levels = tuple(os.environ.get("MARIO_EMU_LEVELS", "base,ckpt,mario").split(","))
         print(json.dumps({"pipeline_emulated": emulate_pipeline(cfg, api, torch, S=args.emulate, n_micro=args.micro,
                                                                 steps=max(1, min(args.steps, 3)), warmup=2,
-                                                                levels=levels, scheme=args.scheme)}), flush=True)
+                                                                levels=levels, scheme=args.scheme or C["scheme"],
+                                                                chunks=C["chunks"])}), flush=True)
         return
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -360,7 +385,10 @@ def main():
     assert world % args.dp == 0 and args.micro % args.dp == 0, "--dp must divide --gpus and --micro"
     S, rep, n_rep = world // args.dp, rank // (world // args.dp), args.micro // args.dp
     stage = rank % S
-    plan = api.Plan(cfg, S, n_rep, args.scheme, args.level, dtype="bf16")
+    scheme = args.scheme or (C["scheme"] if S > 1 else "1f1b")
+    chunks = C["chunks"] if scheme == "interleave" else 1
+    args.scheme = scheme
+    plan = api.Plan(cfg, S, n_rep, scheme, args.level, chunks=chunks, dtype="bf16")
     ctx = api.Context(rank, world, local, dp=args.dp)
     w = init_weights_device(plan, stage, torch)          # replicas of a stage hold identical weights
     pc, ws_bytes = plan.rank_layout(stage)
@@ -462,23 +490,26 @@ def main():
 
     sim = plan.simulate()
     peaks, peak_kind = measured_peaks()
-    traffic = gemm_traffic(cfg)
+    traffic = gemm_traffic(cfg) if args.config == "cfg2" else {}
     g = kst["gemm"]
     achieved = g["flops"] / (g["ms"] / 1e3) / 1e12 if g["ms"] > 0 else 0.0
     peak = float(peaks.get("bf16_tflops_sustained", peaks.get("bf16_tflops")))
-    model_flops = 3.0 * (cfg.n_layers * (2 * cfg.seq_len * (12 * cfg.hidden ** 2) + 4 * cfg.seq_len ** 2 * cfg.hidden)
+    p_lin = 12 * cfg.hidden ** 2 if cfg.family == "gpt" else 4 * cfg.hidden ** 2 + 3 * cfg.hidden * cfg.ffn_hidden
+    model_flops = 3.0 * (cfg.n_layers * (2 * cfg.seq_len * p_lin + 4 * cfg.seq_len ** 2 * cfg.hidden)
                          + 2 * cfg.seq_len * cfg.hidden * cfg.vocab)
     tflops_gpu = model_flops * gbs / (ms_step / 1e3) / world / 1e12
     # whole-step algorithmic roofline: the FLOPs the method must execute (causal
     # attention; + Mario's recompute when stages > 1) over the step time and the dense bf16 peak
     S_ = world // args.dp
-    layer_f = 2 * cfg.seq_len * (12 * cfg.hidden ** 2) + 2 * cfg.seq_len ** 2 * cfg.hidden
+    layer_f = 2 * cfg.seq_len * p_lin + 2 * cfg.seq_len ** 2 * cfg.hidden
     alg_flops = 3.0 * (cfg.n_layers * layer_f + 2 * cfg.seq_len * cfg.hidden * cfg.vocab) * gbs
     if S_ > 1 and args.level != "base":
         alg_flops += (S_ - 1) * (cfg.n_layers // S_) * layer_f * gbs   # RC of every checkpointed stage
     alg_tflops = alg_flops / (ms_step / 1e3) / world / 1e12
     mem = torch.cuda.max_memory_allocated()
-    out = {"metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+    metric = METRIC if args.config == "cfg2" else (f"samples/s ({C['name']}, seq {cfg.seq_len}, GBS {gbs}, "
+                                                   f"Mario plan, bf16)")
+    out = {"metric": metric, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "strong",
            "vs_baseline": None, "dtype": "bf16", "data": "synthetic (uniform tokens, random-init weights)",
            "config": config_dict(cfg, args, gbs),
@@ -511,8 +542,9 @@ def main():
            "execution": "cuda-graph replay" if use_graphs else "eager",
            "e2e": e2e, "eager": eager}
     ctx.close()
-    if rank == 0 and world == 1 and args.emulate > 1:
+    if rank == 0 and world == 1 and args.emulate > 1 and args.config != "cfg5":
         out["pipeline_emulated"] = emulate_pipeline(cfg, api, torch, S=args.emulate, n_micro=args.micro,
+                                                    scheme=C["scheme"], chunks=C["chunks"],
                                                     steps=max(1, min(args.steps, 3)), warmup=2)
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         n_cores = cores()

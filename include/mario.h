@@ -195,6 +195,23 @@ mario_status mario_init_dp(int32_t rank, int32_t world, int32_t device, int32_t 
  * mario_emulated_sms: SMs per rank partition (0 = unpartitioned), -1 if not emulated. */
 mario_status mario_init_emulated(int32_t world, int32_t device, int32_t sms_per_rank);
 int32_t mario_emulated_sms(void);
+/* Multi-process PEER TRANSPORT (CUDA IPC): one process per pipeline rank, on one GPU or on GPUs
+ * with peer access; the same per-rank executor path and flags as mario_init_emulated, with every
+ * other rank's workspace, grads and rank 0's flag block mapped through CUDA IPC. Flags carry the
+ * iteration number (each rank must call mario_run_iter the same number of times); an
+ * end-of-iteration barrier keeps a rank from overwriting memory another rank still reads.
+ *  mario_init_peer(rank, world, device)                     ESTATE if already initialised
+ *  mario_peer_export(workspace, grads, record)              record: 256 bytes out (IPC handles +
+ *                     offsets of this rank's caller-owned workspace / grads and its flag block);
+ *                     the buffers must come from cudaMalloc (any offset inside an allocation)
+ *  mario_peer_import(records)                               records: world x 256 bytes, rank order,
+ *                     gathered by the caller over any out-of-band channel
+ * mario_run_iter then requires exactly the exported workspace and grads (ESTATE otherwise) and
+ * plan stages == world. Tensors on a rank stay rank-local: weights/grads/workspace as
+ * mario_plan_rank_layout(rank). */
+mario_status mario_init_peer(int32_t rank, int32_t world, int32_t device);
+mario_status mario_peer_export(const void* workspace, const void* grads, void* record);
+mario_status mario_peer_import(const void* records);
 /* One training iteration of `plan` on this rank (all ranks in loopback).
  *  weights : device, this rank's packed fp32 parameters (loopback: all ranks concatenated)
  *  tokens  : HOST int32 [N*mbs][s+1]; x = tokens[:, :s], y = tokens[:, 1:] (reading A4)

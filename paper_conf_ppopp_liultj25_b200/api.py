@@ -96,6 +96,9 @@ _lib.register("mario_init", C.c_int32, [C.c_int32, C.c_int32, C.c_int32, C.c_voi
 _lib.register("mario_init_dp", C.c_int32, [C.c_int32, C.c_int32, C.c_int32, C.c_int32, C.c_void_p])
 _lib.register("mario_init_emulated", C.c_int32, [C.c_int32, C.c_int32, C.c_int32])
 _lib.register("mario_emulated_sms", C.c_int32, [])
+_lib.register("mario_init_peer", C.c_int32, [C.c_int32, C.c_int32, C.c_int32])
+_lib.register("mario_peer_export", C.c_int32, [C.c_void_p, C.c_void_p, C.c_void_p])
+_lib.register("mario_peer_import", C.c_int32, [C.c_void_p])
 _lib.register("mario_run_iter", C.c_int32, [_P, C.c_void_p, C.c_void_p, C.POINTER(C.c_float), C.c_void_p,
                                             C.c_void_p, C.c_void_p])
 _lib.register("mario_set_timing", C.c_int32, [C.c_int32])
@@ -304,6 +307,31 @@ class Context:
         self.rank, self.world, self.dp = 0, world, 1
         self.sms_per_rank = int(_lib.lib().mario_emulated_sms())
         return self
+
+    @classmethod
+    def peer(cls, rank: int, world: int, device: int = 0) -> "Context":
+        """mario_init_peer: one process per pipeline rank exchanging activations and gradients through
+        the peer transport over CUDA IPC (same GPU, or GPUs with peer access). Call bind() with the
+        rank's workspace and grads before run_iter."""
+        self = cls.__new__(cls)
+        _check(_lib.lib().mario_init_peer(rank, world, device))
+        self.rank, self.world, self.dp = rank, world, 1
+        return self
+
+    def bind(self, workspace, grads, allgather=None):
+        """Publish this rank's buffers (mario_peer_export) and map every other rank's
+        (mario_peer_import). allgather(bytes) -> [bytes per rank]; default: torch.distributed
+        all_gather_object on the current process group (argument marshalling only)."""
+        rec = C.create_string_buffer(256)
+        _check(_lib.lib().mario_peer_export(C.c_void_p(workspace.data_ptr()), C.c_void_p(grads.data_ptr()), rec))
+        if allgather is None:
+            import torch.distributed as dist
+            out = [None] * self.world
+            dist.all_gather_object(out, rec.raw)
+        else:
+            out = allgather(rec.raw)
+        buf = C.create_string_buffer(b"".join(out), 256 * self.world)
+        _check(_lib.lib().mario_peer_import(buf))
 
     def run_iter(self, plan: Plan, weights, tokens, grads, workspace, stream=None) -> float:
         """weights/grads/workspace: device tensors (data_ptr used); tokens: host int32 array."""

@@ -58,8 +58,15 @@ extern "C" int mario_k_gemm_f32(const float* A, int lda, int a_mn, const float* 
 extern "C" int mario_k_attn_fwd(const void* qkv, void* O, float* lse, int B, int s, int n_heads, int head_dim,
                                 int bf16, void* stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  if (bf16) attn_fwd<__nv_bfloat16>(static_cast<const __nv_bfloat16*>(qkv), static_cast<__nv_bfloat16*>(O), lse, B, s,
-                                    n_heads, head_dim, st);
+  if (bf16) {
+    // a padded head dim (16 / 32 / 80) takes the tcgen05 kernels through a workspace of its own here
+    void* pad = nullptr;
+    const size_t pb = flash_attn_pad_bytes(head_dim, B, s, n_heads, 0);
+    if (pb && cudaMalloc(&pad, pb) != cudaSuccess) return static_cast<int>(cudaErrorMemoryAllocation);
+    attn_fwd<__nv_bfloat16>(static_cast<const __nv_bfloat16*>(qkv), static_cast<__nv_bfloat16*>(O), lse, B, s,
+                            n_heads, head_dim, st, pad);
+    if (pad) { cudaStreamSynchronize(st); cudaFree(pad); }
+  }
   else attn_fwd<float>(static_cast<const float*>(qkv), static_cast<float*>(O), lse, B, s, n_heads, head_dim, st);
   return static_cast<int>(cudaGetLastError());
 }
@@ -67,9 +74,15 @@ extern "C" int mario_k_attn_fwd(const void* qkv, void* O, float* lse, int B, int
 extern "C" int mario_k_attn_bwd(const void* qkv, const void* O, const void* dO, const float* lse, void* dqkv,
                                 float* scratch, int B, int s, int n_heads, int head_dim, int bf16, void* stream) {
   cudaStream_t st = static_cast<cudaStream_t>(stream);
-  if (bf16) attn_bwd<__nv_bfloat16>(static_cast<const __nv_bfloat16*>(qkv), static_cast<const __nv_bfloat16*>(O),
-                                    static_cast<const __nv_bfloat16*>(dO), lse, static_cast<__nv_bfloat16*>(dqkv),
-                                    scratch, B, s, n_heads, head_dim, st);
+  if (bf16) {
+    void* pad = nullptr;
+    const size_t pb = flash_attn_pad_bytes(head_dim, B, s, n_heads, 1);
+    if (pb && cudaMalloc(&pad, pb) != cudaSuccess) return static_cast<int>(cudaErrorMemoryAllocation);
+    attn_bwd<__nv_bfloat16>(static_cast<const __nv_bfloat16*>(qkv), static_cast<const __nv_bfloat16*>(O),
+                            static_cast<const __nv_bfloat16*>(dO), lse, static_cast<__nv_bfloat16*>(dqkv), scratch, B,
+                            s, n_heads, head_dim, st, nullptr, 0, pad);
+    if (pad) { cudaStreamSynchronize(st); cudaFree(pad); }
+  }
   else attn_bwd<float>(static_cast<const float*>(qkv), static_cast<const float*>(O), static_cast<const float*>(dO), lse,
                        static_cast<float*>(dqkv), scratch, B, s, n_heads, head_dim, st);
   return static_cast<int>(cudaGetLastError());

@@ -19,6 +19,7 @@
 // implemented in peer memory instead of NCCL: a send is a flag the sender's stream writes after the
 // message is complete (P:222 buffered send); a receive is a stream wait on that flag, a copy out of
 // the sender's send slot and a "consumed" flag the sender's next use of the slot waits on.
+#include <cuda.h>
 #include <cuda_runtime.h>
 #include <nccl.h>
 
@@ -109,6 +110,19 @@ struct Context {
   bool emu_green = false;                       // streams live in green contexts
   uint32_t* flags = nullptr;                    // device flag block (reset every iteration)
   size_t flags_cap = 0;
+  // peer transport across processes (mario_init_peer: one process per rank, CUDA IPC): every rank
+  // maps the other ranks' workspace and grads and rank 0's flag block; flags carry the iteration
+  // number (epoch) instead of being reset
+  bool ipc = false;
+  uint32_t epoch = 0;
+  struct PeerPtrs { uint8_t* ws = nullptr; float* gr = nullptr; uint32_t* flags = nullptr; };
+  std::vector<PeerPtrs> peers;
+  std::vector<void*> ipc_opened;
+  uint32_t* ipc_flags_own = nullptr;            // this rank's flag block (rank 0's is the shared one)
+  size_t ipc_flag_words = 0;
+  cudaStream_t ipc_st = nullptr, ipc_rx[2] = {nullptr, nullptr};
+  const void* bound_ws = nullptr;               // the buffers the imported records describe
+  const void* bound_gr = nullptr;
 };
 Context g;
 
@@ -164,7 +178,9 @@ struct Exec {
   // where each message sits: (kind, receiving vstage, micro) -> (sender rank, send slot)
   uint32_t* flags = nullptr;
   int fK = 0, fN = 0;
-  std::map<std::tuple<int, int, int>, std::pair<int, int>> msg_slot;
+  uint32_t fv = 1;                             // value a flag is raised to: 1 (reset per call) or the epoch
+  int me = -1;                                 // multi-process peer transport: this rank (else -1: all local)
+  bool mine(int d) const { return me < 0 || d == me; }
   // host walk state (peer): messages whose "ready" / "consumed" flag write is already enqueued. A
   // flag wait is only ever enqueued after the write it waits for (like an event record before its
   // wait): a wait enqueued first could sit in front of its own write if the driver maps the two
@@ -297,7 +313,7 @@ struct Exec {
         lin_fwd(A, Wm(D, p, pre + "qkv.w"), Tn, 3 * h, h, QKV, nullptr);
         rope<T>(QKV, mbs, s, nh, dh, m.rope_base, 0, st);
       }
-      attn_fwd<T>(QKV, O, LSE, mbs, s, nh, dh, st);
+      attn_fwd<T>(QKV, O, LSE, mbs, s, nh, dh, st, LT.attn_pad ? trans + LT.attn_pad : nullptr);
       if (gpt) {
         lin_fwd(O, Wm(D, p, pre + "proj.w"), Tn, h, h, H1, Wf(D, p, pre + "proj.b"), Hin);
         layernorm_fwd<T>(H1, Wf(D, p, pre + "ln2.g"), Wf(D, p, pre + "ln2.b"), A2, st2, Tn, h, m.norm_eps, st);
@@ -463,7 +479,8 @@ struct Exec {
         lin_wgrad(dH1, O, Tn, h, h, G(D, p, pre + "o.w"));
         lin_dgrad(dH1, Wm(D, p, pre + "o.w"), Tn, h, h, dO);
       }
-      attn_bwd<T>(QKV, O, dO, LSE, dQKV, Dsc, mbs, s, nh, dh, st, BS.dS_bytes ? sc + BS.dS : nullptr, BS.dS_bytes);
+      attn_bwd<T>(QKV, O, dO, LSE, dQKV, Dsc, mbs, s, nh, dh, st, BS.dS_bytes ? sc + BS.dS : nullptr, BS.dS_bytes,
+                  BS.attn_pad ? sc + BS.attn_pad : nullptr);
       if (!gpt) rope<T>(dQKV, mbs, s, nh, dh, m.rope_base, 1, st);
       if (gpt) norm_recompute<T>(Hin, Wf(D, p, pre + "ln1.g"), Wf(D, p, pre + "ln1.b"), A, st1, Tn, h, m.norm_eps, 0, st);
       else norm_recompute<T>(Hin, Wf(D, p, pre + "n1.g"), nullptr, A, st1, Tn, h, m.norm_eps, 1, st);
@@ -523,8 +540,7 @@ struct Exec {
           D.sa_used[i] = true;
           D.sa_of[key] = i;
           if (peer) {
-            if (D.sa_guard[i]) DRV(drv::wait_flag(st, D.sa_guard[i], 1));   // previous message consumed
-            msg_slot[{0, x.vstage + 1, x.micro}] = {d, i};
+            if (D.sa_guard[i]) DRV(drv::wait_flag(st, D.sa_guard[i], fv));   // previous message consumed
           } else if (!loopback && D.sa_free_set[i]) {
             CU(cudaStreamWaitEvent(st, D.sa_free[i], 0));
           }
@@ -547,8 +563,7 @@ struct Exec {
           D.sg_used[i] = true;
           D.sg_of[key] = i;
           if (peer) {
-            if (D.sg_guard[i]) DRV(drv::wait_flag(st, D.sg_guard[i], 1));
-            msg_slot[{1, x.vstage - 1, x.micro}] = {d, i};
+            if (D.sg_guard[i]) DRV(drv::wait_flag(st, D.sg_guard[i], fv));
           } else if (!loopback && D.sg_free_set[i]) {
             CU(cudaStreamWaitEvent(st, D.sg_free[i], 0));
           }
@@ -578,7 +593,7 @@ struct Exec {
           auto& of = grad ? D.sg_of : D.sa_of;
           const int i = of.at(key);
           const int kd = grad ? x.vstage - 1 : x.vstage + 1;
-          DRV(drv::write_flag(st, flag_ready(grad, kd, x.micro), 1));
+          DRV(drv::write_flag(st, flag_ready(grad, kd, x.micro), fv));
           (grad ? D.sg_guard : D.sa_guard)[i] = flag_done(grad, kd, x.micro);
           (grad ? D.sg_guard_key : D.sa_guard_key)[i] = std::make_tuple(grad ? 1 : 0, kd, x.micro);
           (grad ? D.sg_used : D.sa_used)[i] = false;
@@ -602,7 +617,10 @@ struct Exec {
           // sender's slot on this rank's receive stream, flag it consumed, then the compute stream
           // waits for the copy at this list position
           const int kind = grad ? 1 : 0;
-          const auto src = msg_slot.at({kind, x.vstage, x.micro});
+          // the sender (Alg. 1 find_prev) and the slot the plan gave its message
+          int sd = -1, sp = -1;
+          plan::find_inst(D.P->pp, d, x.micro, x.part, grad ? MARIO_OP_BW : MARIO_OP_FW, false, &sd, &sp);
+          const std::pair<int, int> src{sd, (grad ? D.P->sg_slot : D.P->sa_slot)[sd].at({x.micro, sp})};
           Dev<T>& Sd = dev(src.first);
           // MARIO_PEER_RX=0: receive on the compute stream itself (no prefetch, fewer streams)
           static const bool rx_streams = !getenv("MARIO_PEER_RX") || atoi(getenv("MARIO_PEER_RX")) != 0;
@@ -612,9 +630,9 @@ struct Exec {
             const int i = D.rg_of[key];
             if (D.rg_free_set[i]) CU(cudaStreamWaitEvent(rs, D.rg_free[i], 0));
           }
-          DRV(drv::wait_flag(rs, flag_ready(kind, x.vstage, x.micro), 1));
+          DRV(drv::wait_flag(rs, flag_ready(kind, x.vstage, x.micro), fv));
           CU(cudaMemcpyAsync(dst, send_slot(Sd, grad, src.second), msg_bytes, cudaMemcpyDeviceToDevice, rs));
-          DRV(drv::write_flag(rs, flag_done(kind, x.vstage, x.micro), 1));
+          DRV(drv::write_flag(rs, flag_done(kind, x.vstage, x.micro), fv));
           consumed_walked.insert(std::make_tuple(kind, x.vstage, x.micro));
           if (rs != st) {
             cudaEvent_t e = D.event();
@@ -758,10 +776,15 @@ void ensure_channels(const PlanObj& P) {
 template <class T>
 mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* tokens, float* loss, void* grads,
                         void* workspace, cudaStream_t st) {
-  const bool peer = g.emulated;
+  const bool peer = g.emulated || g.ipc;
   const bool loopback = !peer && g.world == 1 && P.pp.S > 1;
-  if (peer && P.pp.S != static_cast<int>(g.emu_st.size()))
+  if (g.emulated && P.pp.S != static_cast<int>(g.emu_st.size()))
     return set_error(MARIO_ESTATE, "plan stages != emulated world size");
+  if (g.ipc) {
+    if (P.pp.S != g.world) return set_error(MARIO_ESTATE, "plan stages != peer world size");
+    if (static_cast<int>(g.peers.size()) != g.world || workspace != g.bound_ws || grads != g.bound_gr)
+      return set_error(MARIO_ESTATE, "buffers not bound: mario_peer_export / mario_peer_import first");
+  }
   if (!loopback && !peer && P.pp.S * g.dp != g.world) return set_error(MARIO_ESTATE, "plan stages * dp != world size");
   const int me = g.rank % P.pp.S, off = g.rank - me;   // stage and the replica's rank offset
   const auto& prog = comm_program_dp(P, g.dp, g.rank);
@@ -769,6 +792,10 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
   E.st = st;
   E.loopback = loopback;
   E.peer = peer;
+  if (g.ipc) {
+    E.me = g.rank;
+    E.fv = ++g.epoch;
+  }
   const mario_model& m = P.model;
   const int S = P.pp.S;
   std::vector<int> my_devs;
@@ -787,14 +814,18 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
   if (peer) {
     E.fK = P.pp.K();
     E.fN = P.pp.N;
-    flag_words = static_cast<size_t>(4) * E.fK * E.fN + S + n_multi_flags;
-    if (g.flags_cap < flag_words) {
+    // + per rank: backward done, (ipc) gathered, (ipc) loss ready
+    flag_words = static_cast<size_t>(4) * E.fK * E.fN + 3 * S + n_multi_flags;
+    if (g.ipc) {
+      if (flag_words > g.ipc_flag_words) return set_error(MARIO_EINVAL, "plan needs more peer flags than allocated");
+      E.flags = g.peers[0].flags;
+    } else if (g.flags_cap < flag_words) {
       if (g.flags) CU(cudaFree(g.flags));
       g.flags = nullptr;
       CU(cudaMalloc(&g.flags, flag_words * 4));
       g.flags_cap = flag_words;
     }
-    E.flags = g.flags;
+    if (!g.ipc) E.flags = g.flags;
   }
   size_t wofs = 0, wsofs = 0;
   for (int d : my_devs) {
@@ -802,16 +833,25 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
     D->P = &P;
     D->d = d;
     const auto& pools = loopback ? P.pools_lb[d] : P.pools_mp[d];
-    if (peer) {
+    if (g.emulated) {
       D->st = g.emu_st[d];
       D->rx[0] = g.emu_rx[d][0];
       D->rx[1] = g.emu_rx[d][1];
       D->sms = g.emu_sms;
+    } else if (g.ipc && d == E.me) {
+      D->st = g.ipc_st;
+      D->rx[0] = g.ipc_rx[0];
+      D->rx[1] = g.ipc_rx[1];
     }
     D->a = make_arena(P, d, pools);
     D->ws = static_cast<uint8_t*>(workspace) + wsofs;
     D->w = static_cast<const float*>(weights) + wofs;
     D->gr = static_cast<float*>(grads) + wofs;
+    if (g.ipc && d != E.me) {   // another process's rank: its mapped workspace and grads
+      D->ws = g.peers[d].ws;
+      D->gr = g.peers[d].gr;
+      D->w = nullptr;
+    }
     const auto& rp = P.rank_params[d];
     for (size_t j = 0; j < rp.idx.size(); ++j) D->tensor[{rp.part[j], rp.idx[j]}] = static_cast<int>(j);
     D->sa_used.assign(std::max(1, pools.send_act), false);
@@ -833,21 +873,22 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
     if (loopback) {
       wofs += rp.total;
       wsofs += align_up(P.workspace_lb[d], 1 << 20);
-    } else if (peer) {
+    } else if (g.emulated) {
       wofs += rp.total;
       wsofs += align_up(P.workspace_mp[d], 1 << 20);
     }
     // tokens H2D (outside any captured graph: the host buffer changes every call)
     const size_t tok_bytes = static_cast<size_t>(P.pp.N) * m.micro_batch * (m.seq_len + 1) * 4;
-    CU(cudaMemcpyAsync(D->ws + D->a.tokens, tokens, tok_bytes, cudaMemcpyDefault, st));   // host or device tokens
+    if (E.mine(d))
+      CU(cudaMemcpyAsync(D->ws + D->a.tokens, tokens, tok_bytes, cudaMemcpyDefault, st));   // host or device tokens
     E.devs.push_back(std::move(D));
   }
-  if (!loopback && g.world > 1) ensure_channels(P);
+  if (!loopback && !peer && g.world > 1) ensure_channels(P);
 
   // Single-process iterations are a fixed launch sequence over fixed buffers: the second call
   // with the same (plan, weights, grads, workspace) is captured into a CUDA graph, later calls
   // replay it (no per-kernel launch cost). Disabled while timing/kstats instrumentation is on.
-  const bool graphable = g.graphs && g.world == 1 && !g.timing;
+  const bool graphable = g.graphs && g.world == 1 && !g.timing && !g.ipc;
   const auto gkey = std::make_tuple(P.serial, weights, static_cast<const void*>(grads),
                                     static_cast<const void*>(workspace), kstats_generation());
   bool replayed = false, capturing = false;
@@ -874,8 +915,8 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
   cudaEvent_t t0_peer = nullptr;
   if (!replayed) {
   if (peer) {
-    // reset the flags, then fork every rank's streams off the caller's (or capture) stream
-    CU(cudaMemsetAsync(E.flags, 0, flag_words * 4, body));
+    // reset the flags (ipc: epochs instead), then fork every rank's streams off the caller's stream
+    if (!g.ipc) CU(cudaMemsetAsync(E.flags, 0, flag_words * 4, body));
     if (g.timing) {
       CU(cudaEventCreate(&t0_peer));
       CU(cudaEventRecord(t0_peer, body));
@@ -883,6 +924,7 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
     cudaEvent_t fork = E.devs[0]->event();
     CU(cudaEventRecord(fork, body));
     for (auto& Dp : E.devs) {
+      if (!E.mine(Dp->d)) continue;
       CU(cudaStreamWaitEvent(Dp->st, fork, 0));
       CU(cudaStreamWaitEvent(Dp->rx[0], fork, 0));
       CU(cudaStreamWaitEvent(Dp->rx[1], fork, 0));
@@ -890,6 +932,7 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
   }
   for (auto& Dp : E.devs) {
     Dev<T>& D = *Dp;
+    if (!E.mine(D.d)) continue;
     const auto& rp = P.rank_params[D.d];
     cudaStream_t s0 = peer ? D.st : body;
     if (peer) set_sm_budget(D.sms);
@@ -904,6 +947,11 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
   // walk the plan
   if (loopback) {
     for (auto [d, i] : P.loopback_order) E.run_instr(d, P.instrs[d][i]);
+  } else if (g.ipc) {
+    // one rank per process: walk this rank's list; every flag it waits on is raised by another
+    // process (own context, own hardware queues), so no cross-rank enqueue order is needed
+    for (const mario_instr& x : P.instrs[E.me]) E.run_instr(E.me, x);
+    E.st = body;
   } else if (peer) {
     // every rank runs on its own streams and waits only on flags, so the device executes the
     // plan's DAG concurrently. The host enqueues in the loopback order (a valid order of the DAG in
@@ -939,7 +987,8 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
     // (a reduce-scatter); the owners flag their chunks done and every other holder pulls them back
     // (an all-gather). Flags: per-rank "all BW done" before any chunk is read, per-chunk "summed"
     // before it is copied back, so no copy is overwritten while another rank still reads it.
-    for (auto& Dp : E.devs) DRV(drv::write_flag(Dp->st, E.flag_misc(Dp->d), 1));
+    const uint32_t fv = E.fv;
+    for (auto& Dp : E.devs) if (E.mine(Dp->d)) DRV(drv::write_flag(Dp->st, E.flag_misc(Dp->d), fv));
     size_t fi = static_cast<size_t>(S);
     for (auto& kv : copies) {
       const auto& cp = kv.second;
@@ -949,28 +998,40 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
       auto ptr = [&](std::pair<int, int> c) { return E.dev(c.first).gr + P.rank_params[c.first].off[c.second]; };
       const size_t nc = cp.size(), chunk = (n + nc - 1) / nc;
       for (size_t c = 0; c < nc; ++c) {                       // reduce-scatter: owner of chunk c = copy c
+        if (!E.mine(cp[c].first)) continue;
         Dev<T>& O = E.dev(cp[c].first);
         const size_t lo = std::min(n, c * chunk), hi = std::min(n, lo + chunk);
-        for (auto& h : cp) DRV(drv::wait_flag(O.st, E.flag_misc(h.first), 1));
+        for (auto& h : cp) DRV(drv::wait_flag(O.st, E.flag_misc(h.first), fv));
         CopySrcs src{};
         src.n = static_cast<int>(nc);
         for (size_t j = 0; j < nc; ++j) src.p[j] = ptr(cp[j]) + lo;
         if (hi > lo) sum_copies_f32(ptr(cp[c]) + lo, src, hi - lo, O.st);
-        DRV(drv::write_flag(O.st, E.flag_misc(fi + c), 1));
+        DRV(drv::write_flag(O.st, E.flag_misc(fi + c), fv));
       }
       for (size_t c = 0; c < nc; ++c) {                       // all-gather
         const size_t lo = std::min(n, c * chunk), hi = std::min(n, lo + chunk);
         for (size_t j = 0; j < nc; ++j) {
-          if (j == c) continue;
+          if (j == c || !E.mine(cp[j].first)) continue;
           Dev<T>& H = E.dev(cp[j].first);
-          DRV(drv::wait_flag(H.st, E.flag_misc(fi + c), 1));
+          DRV(drv::wait_flag(H.st, E.flag_misc(fi + c), fv));
           if (hi > lo) CU(cudaMemcpyAsync(ptr(cp[j]) + lo, ptr(cp[c]) + lo, (hi - lo) * 4, cudaMemcpyDeviceToDevice, H.st));
         }
       }
       fi += nc;
     }
+    if (g.ipc) {
+      // no rank may start its next iteration (zeroing grads, overwriting slots) while another still
+      // reads its memory: all-gathered barrier; then the last stage(s)' loss partials are readable
+      Dev<T>& D = E.dev(E.me);
+      const size_t gath = fi, lossf = fi + S;
+      DRV(drv::write_flag(D.st, E.flag_misc(gath + E.me), fv));
+      for (int r = 0; r < S; ++r) DRV(drv::wait_flag(D.st, E.flag_misc(gath + r), fv));
+      DRV(drv::write_flag(D.st, E.flag_misc(lossf + E.me), fv));
+      for (int r = 0; r < S; ++r) DRV(drv::wait_flag(D.st, E.flag_misc(lossf + r), fv));
+    }
     // join every rank's stream back into the caller's (or capture) stream
     for (auto& Dp : E.devs) {
+      if (!E.mine(Dp->d)) continue;
       cudaEvent_t e = Dp->event();
       CU(cudaEventRecord(e, Dp->st));
       CU(cudaStreamWaitEvent(body, e, 0));
@@ -1048,7 +1109,7 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
     CU(cudaStreamSynchronize(st));
     for (int i = 0; i < P.pp.N; ++i) sums[i] += h[i];
   }
-  if (!loopback && g.world > 1) {
+  if (!loopback && !peer && g.world > 1) {
     // share the last stage(s)' per-micro-batch sums with every rank (summed over replicas too)
     double* dbuf = reinterpret_cast<double*>(E.devs[0]->ws + E.devs[0]->a.loss);
     CU(cudaMemcpyAsync(dbuf, sums.data(), P.pp.N * 8, cudaMemcpyHostToDevice, st));
@@ -1177,6 +1238,102 @@ extern "C" mario_status mario_init_emulated(int32_t world, int32_t device, int32
 
 extern "C" int32_t mario_emulated_sms(void) { return g.emulated ? g.emu_sms : -1; }
 
+// ------------------------------------------------------------- multi-process peer transport
+namespace {
+constexpr size_t kPeerFlagWords = static_cast<size_t>(1) << 20;   // 4 MiB of flags per rank
+struct PeerRecord {            // what one rank publishes (mario_peer_export), 256 bytes
+  cudaIpcMemHandle_t ws, gr, flags;
+  uint64_t ws_off, gr_off, flags_off;
+  int32_t rank, world;
+  uint8_t pad[256 - 3 * sizeof(cudaIpcMemHandle_t) - 3 * 8 - 8];
+};
+static_assert(sizeof(PeerRecord) == 256, "peer record size");
+
+// IPC handle of the allocation containing p, and p's offset in it
+mario_status ipc_handle(const void* p, cudaIpcMemHandle_t* h, uint64_t* off) {
+  using PFN = CUresult (*)(CUdeviceptr*, size_t*, CUdeviceptr);
+  static PFN range = [] {
+    void* f = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    cudaGetDriverEntryPointByVersion("cuMemGetAddressRange", &f, 12000, cudaEnableDefault, &q);
+    return reinterpret_cast<PFN>(f);
+  }();
+  if (!range) return set_error(MARIO_ECUDA, "cuMemGetAddressRange unavailable");
+  CUdeviceptr base = 0;
+  size_t size = 0;
+  if (range(&base, &size, reinterpret_cast<CUdeviceptr>(p)) != 0) return set_error(MARIO_EINVAL, "not device memory");
+  if (cudaIpcGetMemHandle(h, reinterpret_cast<void*>(base)) != cudaSuccess)
+    return set_error(MARIO_ECUDA, "cudaIpcGetMemHandle failed (memory not from cudaMalloc?)");
+  *off = reinterpret_cast<uint64_t>(p) - static_cast<uint64_t>(base);
+  return MARIO_OK;
+}
+}  // namespace
+
+extern "C" mario_status mario_init_peer(int32_t rank, int32_t world, int32_t device) {
+  try {
+    if (world < 1 || rank < 0 || rank >= world) return set_error(MARIO_EINVAL, "bad rank/world");
+    if (g.inited) return set_error(MARIO_ESTATE, "already initialised");
+    CU(cudaSetDevice(device));
+    g.rank = rank; g.world = world; g.device = device; g.dp = 1;
+    CU(cudaMalloc(&g.ipc_flags_own, kPeerFlagWords * 4));
+    CU(cudaMemset(g.ipc_flags_own, 0, kPeerFlagWords * 4));
+    g.ipc_flag_words = kPeerFlagWords;
+    CU(cudaStreamCreateWithFlags(&g.ipc_st, cudaStreamNonBlocking));
+    for (auto& x : g.ipc_rx) CU(cudaStreamCreateWithFlags(&x, cudaStreamNonBlocking));
+    CU(cudaDeviceSynchronize());
+    g.epoch = 0;
+    g.ipc = true;
+    g.inited = true;
+    g.sticky = false;
+    return MARIO_OK;
+  } catch (const CudaErr& e) {
+    return set_error(MARIO_ECUDA, e.what());
+  }
+}
+
+extern "C" mario_status mario_peer_export(const void* workspace, const void* grads, void* record) {
+  if (!g.ipc) return set_error(MARIO_ESTATE, "mario_init_peer not called");
+  if (!workspace || !grads || !record) return set_error(MARIO_EINVAL, "NULL argument");
+  PeerRecord r{};
+  if (mario_status e = ipc_handle(workspace, &r.ws, &r.ws_off)) return e;
+  if (mario_status e = ipc_handle(grads, &r.gr, &r.gr_off)) return e;
+  if (mario_status e = ipc_handle(g.ipc_flags_own, &r.flags, &r.flags_off)) return e;
+  r.rank = g.rank;
+  r.world = g.world;
+  memcpy(record, &r, sizeof r);
+  g.bound_ws = workspace;
+  g.bound_gr = grads;
+  return MARIO_OK;
+}
+
+extern "C" mario_status mario_peer_import(const void* records) {
+  if (!g.ipc) return set_error(MARIO_ESTATE, "mario_init_peer not called");
+  if (!records || !g.bound_ws) return set_error(MARIO_EINVAL, "export this rank's buffers first");
+  for (void* p : g.ipc_opened) cudaIpcCloseMemHandle(p);
+  g.ipc_opened.clear();
+  g.peers.assign(g.world, {});
+  const PeerRecord* rec = static_cast<const PeerRecord*>(records);
+  for (int r = 0; r < g.world; ++r) {
+    if (rec[r].rank != r || rec[r].world != g.world) return set_error(MARIO_EINVAL, "records out of rank order");
+    if (r == g.rank) {
+      g.peers[r] = {static_cast<uint8_t*>(const_cast<void*>(g.bound_ws)),
+                    static_cast<float*>(const_cast<void*>(g.bound_gr)), g.ipc_flags_own};
+      continue;
+    }
+    void* base[3];
+    const cudaIpcMemHandle_t* hs[3] = {&rec[r].ws, &rec[r].gr, &rec[r].flags};
+    for (int i = 0; i < 3; ++i) {
+      if (cudaIpcOpenMemHandle(&base[i], *hs[i], cudaIpcMemLazyEnablePeerAccess) != cudaSuccess)
+        return set_error(MARIO_ECUDA, "cudaIpcOpenMemHandle failed for rank " + std::to_string(r));
+      g.ipc_opened.push_back(base[i]);
+    }
+    g.peers[r] = {static_cast<uint8_t*>(base[0]) + rec[r].ws_off,
+                  reinterpret_cast<float*>(static_cast<uint8_t*>(base[1]) + rec[r].gr_off),
+                  reinterpret_cast<uint32_t*>(static_cast<uint8_t*>(base[2]) + rec[r].flags_off)};
+  }
+  return MARIO_OK;
+}
+
 extern "C" mario_status mario_init(int32_t rank, int32_t world, int32_t device, const void* nccl_unique_id) {
   return mario_init_dp(rank, world, device, 1, nccl_unique_id);
 }
@@ -1278,6 +1435,20 @@ extern "C" mario_status mario_finalize(void) {
   if (g.flags) cudaFree(g.flags);
   g.flags = nullptr;
   g.flags_cap = 0;
+  if (g.ipc) {
+    cudaDeviceSynchronize();
+    for (void* p : g.ipc_opened) cudaIpcCloseMemHandle(p);
+    g.ipc_opened.clear();
+    g.peers.clear();
+    if (g.ipc_flags_own) cudaFree(g.ipc_flags_own);
+    g.ipc_flags_own = nullptr;
+    if (g.ipc_st) cudaStreamDestroy(g.ipc_st);
+    for (auto& x : g.ipc_rx) { if (x) cudaStreamDestroy(x); x = nullptr; }
+    g.ipc_st = nullptr;
+    g.ipc = false;
+    g.bound_ws = g.bound_gr = nullptr;
+    g.world = 1;
+  }
   if (g.dp_comm) ncclCommDestroy(g.dp_comm);
   g.dp_comm = nullptr;
   if (g.world_comm) ncclCommDestroy(g.world_comm);

@@ -4,7 +4,10 @@
 
 #include "../plan/model.h"
 
-namespace mario { size_t flash_attn_bwd_ds_bytes(int dh, int B, int s, int nh); }   // kernels/attn_tc.cu
+namespace mario {
+size_t flash_attn_bwd_ds_bytes(int dh, int B, int s, int nh);           // kernels/attn_tc.cu
+size_t flash_attn_pad_bytes(int dh, int B, int s, int nh, int bwd);      // kernels/attn_mma.cu
+}
 
 namespace mario {
 
@@ -37,6 +40,8 @@ LayerTrans layer_trans_layout(const mario_model& m) {
   L.A = take(T * h * E);
   L.A2 = take(T * h * E);
   L.G = take(T * f * E);
+  L.attn_pad = take(m.dtype == MARIO_BF16
+                        ? flash_attn_pad_bytes(h / m.n_heads, m.micro_batch, m.seq_len, m.n_heads, 0) : 0);
   L.bytes = o;
   return L;
 }
@@ -105,6 +110,8 @@ BwScratch bw_scratch_layout(const mario_model& m) {
   b.sort = take(T * 8 * 2);
   b.Arec = take(T * h * E);
   for (int i = 0; i < 2; ++i) b.dH32[i] = take(m.dtype == MARIO_BF16 ? T * h * 4 : 0);
+  b.attn_pad = take(m.dtype == MARIO_BF16
+                        ? flash_attn_pad_bytes(h / m.n_heads, m.micro_batch, m.seq_len, m.n_heads, 1) : 0);
   // the attention backward's dS image (fa_bwd_dq_img: dQ from the stored dS, no S/dP recompute);
   // only where it stays small next to the rest of the scratch (not at s = 16384)
   b.dS_bytes = 0;

@@ -24,6 +24,7 @@ LayerAct layer_act_layout(const mario_model& m);
 // Per-layer transients of the forward (reused layer after layer): A, A2 [T,h], G|M [T,f].
 struct LayerTrans {
   size_t A, A2, G;
+  size_t attn_pad;   // padded-head-dim attention workspace (bf16, dh not 64 / 128), else 0 bytes
   size_t bytes;
 };
 LayerTrans layer_trans_layout(const mario_model& m);
@@ -56,6 +57,7 @@ size_t cfw_work_bytes(const mario_model& m, int k, int K);       // transient CF
 struct BwScratch {
   size_t dH[3], dA, dQKV, dO, dZ, dM, Dsc, sort, Arec;   // dM doubles as the G/M recompute buffer
   size_t dH32[2];   // bf16 mode: the fp32 residual-gradient stream (reading A30); 0 bytes in fp32 mode
+  size_t attn_pad;  // padded-head-dim attention backward workspace (bf16, dh not 64 / 128), else 0 bytes
   size_t dS, dS_bytes;   // attention dS image (bf16, when the shape allows it and it is <= 1 GiB; else 0 bytes)
   size_t bytes;
 };

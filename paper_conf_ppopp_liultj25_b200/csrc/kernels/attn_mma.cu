@@ -505,7 +505,111 @@ void launch_bwd(const bf16* qkv, const bf16* O, const bf16* dO, const float* lse
 
 bool flash_attn_supported(int dh) { return dh == 16 || dh == 32 || dh == 64 || dh == 80 || dh == 128; }
 
-void flash_attn_fwd(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st) {
+// ------------------------------------------------------------------ padded head dims on tcgen05
+// Head dims the tcgen05 kernels do not tile (16, 32, 80: GPT-3 2.7B's dh 80 in cfg 4) run on the
+// dh_p = 64 / 128 kernels over zero-padded copies: QKV [T][3][nh][dh] -> [T][3][nh][dh_p] with the
+// q part scaled by c = sqrt(dh_p / dh), so the kernels' 1/sqrt(dh_p) softmax scale gives
+// q.k / sqrt(dh) exactly up to the one bf16 rounding of c q (none when c is a power of 2); the
+// zero columns add nothing to q.k, and O / dK / dV padding columns are zero and dropped. dQ of the
+// unscaled q is c dQ'. Row sums D = rowsum(dO O) come from the unpadded tensors.
+namespace {
+int padded_dh(int dh) { return dh < 64 ? 64 : 128; }
+bool needs_pad(int dh) { return dh != 64 && dh != 128 && dh % 8 == 0 && dh < 128; }
+
+// out[t][p][h][0..Dp) = in[t][p][h][0..dh) (x scale for p == 0), zero-padded; 16-byte chunks
+__global__ void attn_pad_k(const bf16* __restrict__ in, bf16* __restrict__ out, long T, int parts, int nh, int dh,
+                           int Dp, float scale0) {
+  const int cpr = Dp / 8;
+  const long total = T * parts * nh * cpr;
+  for (long i = blockIdx.x * static_cast<long>(blockDim.x) + threadIdx.x; i < total;
+       i += static_cast<long>(gridDim.x) * blockDim.x) {
+    const int j = static_cast<int>(i % cpr);
+    long r = i / cpr;
+    const int hh = static_cast<int>(r % nh);
+    r /= nh;
+    const int p = static_cast<int>(r % parts);
+    const long t = r / parts;
+    uint4 v = make_uint4(0, 0, 0, 0);
+    if (j * 8 < dh) {
+      v = *reinterpret_cast<const uint4*>(in + (t * parts + p) * nh * static_cast<long>(dh) + hh * dh + j * 8);
+      if (p == 0 && scale0 != 1.f) {
+        __nv_bfloat162* h2 = reinterpret_cast<__nv_bfloat162*>(&v);
+#pragma unroll
+        for (int e = 0; e < 4; ++e) {
+          const float2 f = __bfloat1622float2(h2[e]);
+          h2[e] = __floats2bfloat162_rn(f.x * scale0, f.y * scale0);
+        }
+      }
+    }
+    *reinterpret_cast<uint4*>(out + (t * parts + p) * nh * static_cast<long>(Dp) + hh * Dp + j * 8) = v;
+  }
+}
+// out[t][p][h][0..dh) = in[t][p][h][0..dh) of the padded layout (x scale for p == 0)
+__global__ void attn_unpad_k(const bf16* __restrict__ in, bf16* __restrict__ out, long T, int parts, int nh, int dh,
+                             int Dp, float scale0) {
+  const int cpr = dh / 8;
+  const long total = T * parts * nh * cpr;
+  for (long i = blockIdx.x * static_cast<long>(blockDim.x) + threadIdx.x; i < total;
+       i += static_cast<long>(gridDim.x) * blockDim.x) {
+    const int j = static_cast<int>(i % cpr);
+    long r = i / cpr;
+    const int hh = static_cast<int>(r % nh);
+    r /= nh;
+    const int p = static_cast<int>(r % parts);
+    const long t = r / parts;
+    uint4 v = *reinterpret_cast<const uint4*>(in + (t * parts + p) * nh * static_cast<long>(Dp) + hh * Dp + j * 8);
+    if (p == 0 && scale0 != 1.f) {
+      __nv_bfloat162* h2 = reinterpret_cast<__nv_bfloat162*>(&v);
+#pragma unroll
+      for (int e = 0; e < 4; ++e) {
+        const float2 f = __bfloat1622float2(h2[e]);
+        h2[e] = __floats2bfloat162_rn(f.x * scale0, f.y * scale0);
+      }
+    }
+    *reinterpret_cast<uint4*>(out + (t * parts + p) * nh * static_cast<long>(dh) + hh * dh + j * 8) = v;
+  }
+}
+void pad(const bf16* in, bf16* out, long T, int parts, int nh, int dh, int Dp, float sc, cudaStream_t st) {
+  const long total = T * parts * nh * (Dp / 8);
+  const long g = (total + 255) / 256;
+  attn_pad_k<<<static_cast<int>(g < 148 * 16 ? g : 148 * 16), 256, 0, st>>>(in, out, T, parts, nh, dh, Dp, sc);
+  note_launch();
+}
+void unpad(const bf16* in, bf16* out, long T, int parts, int nh, int dh, int Dp, float sc, cudaStream_t st) {
+  const long total = T * parts * nh * (dh / 8);
+  const long g = (total + 255) / 256;
+  attn_unpad_k<<<static_cast<int>(g < 148 * 16 ? g : 148 * 16), 256, 0, st>>>(in, out, T, parts, nh, dh, Dp, sc);
+  note_launch();
+}
+}  // namespace
+
+size_t flash_attn_pad_bytes(int dh, int B, int s, int nh, int bwd) {
+  if (!needs_pad(dh)) return 0;
+  const int Dp = padded_dh(dh);
+  if (!flash_attn_bwd_tc_supported(Dp, B, s, nh)) return 0;
+  const size_t T = static_cast<size_t>(B) * s, row = static_cast<size_t>(nh) * Dp * 2;
+  const size_t al = 256;
+  auto up = [&](size_t x) { return (x + al - 1) / al * al; };
+  // fwd: qkv' [T, 3 nh Dp], O' [T, nh Dp]; bwd: qkv', dO', dqkv' (+ the dS image for dh_p)
+  if (!bwd) return up(T * 3 * row) + up(T * row);
+  return up(T * 3 * row) + up(T * row) + up(T * 3 * row) + up(flash_attn_bwd_ds_bytes(Dp, B, s, nh));
+}
+
+void flash_attn_fwd(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st,
+                    void* pad_ws) {
+  if (pad_ws && needs_pad(dh) && g_attn_variant != 0 && flash_attn_pad_bytes(dh, B, s, nh, 0)) {
+    const int Dp = padded_dh(dh);
+    const long T = static_cast<long>(B) * s;
+    bf16* qkvp = static_cast<bf16*>(pad_ws);
+    bf16* Op = qkvp + ((T * 3 * nh * Dp * 2 + 255) / 256 * 256) / 2;
+    const double fl = 4.0 * B * nh * dh * (static_cast<double>(s) * (s + 1) / 2);
+    const int tok = kstats_begin(K_ATTN_FWD, fl, 0.0, st);
+    pad(qkv, qkvp, T, 3, nh, dh, Dp, sqrtf(static_cast<float>(Dp) / dh), st);
+    const bool ok = flash_attn_fwd_tc(qkvp, Op, lse, B, s, nh, Dp, st);
+    if (ok) unpad(Op, O, T, 1, nh, dh, Dp, 1.f, st);
+    kstats_end(tok, st);
+    if (ok) return;
+  }
   switch (dh) {
     case 16: launch_fwd<16>(qkv, O, lse, B, s, nh, st); break;
     case 32: launch_fwd<32>(qkv, O, lse, B, s, nh, st); break;
@@ -516,7 +620,34 @@ void flash_attn_fwd(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, 
 }
 
 void flash_attn_bwd(const bf16* qkv, const bf16* O, const bf16* dO, const float* lse, bf16* dqkv, float* Dd, int B,
-                    int s, int nh, int dh, cudaStream_t st, void* ds_ws, size_t ds_ws_bytes) {
+                    int s, int nh, int dh, cudaStream_t st, void* ds_ws, size_t ds_ws_bytes, void* pad_ws) {
+  (void)ds_ws; (void)ds_ws_bytes;
+  if (pad_ws && needs_pad(dh) && g_attn_variant != 0 && flash_attn_pad_bytes(dh, B, s, nh, 1)) {
+    const int Dp = padded_dh(dh);
+    const long T = static_cast<long>(B) * s;
+    auto up = [](long x) { return (x + 255) / 256 * 256; };
+    uint8_t* w = static_cast<uint8_t*>(pad_ws);
+    bf16* qkvp = reinterpret_cast<bf16*>(w);
+    bf16* dOp = reinterpret_cast<bf16*>(w + up(T * 3 * nh * Dp * 2));
+    bf16* dqkvp = reinterpret_cast<bf16*>(w + up(T * 3 * nh * Dp * 2) + up(T * nh * Dp * 2));
+    uint8_t* img = w + up(T * 3 * nh * Dp * 2) + up(T * nh * Dp * 2) + up(T * 3 * nh * Dp * 2);
+    const size_t img_bytes = flash_attn_bwd_ds_bytes(Dp, B, s, nh);
+    {   // D = rowsum(dO * O) of the unpadded head (padding columns are zero)
+      const long thr = T * nh * 32;
+      fa_bwd_dot_k<<<static_cast<int>((thr + 255) / 256), 256, 0, st>>>(O, dO, Dd, T, nh, dh);
+      note_launch();
+    }
+    const float c = sqrtf(static_cast<float>(Dp) / dh);
+    const double fl = 8.0 * B * nh * dh * (static_cast<double>(s) * (s + 1) / 2);
+    const int tok = kstats_begin(K_ATTN_BWD, fl, 0.0, st);
+    pad(qkv, qkvp, T, 3, nh, dh, Dp, c, st);
+    pad(dO, dOp, T, 1, nh, dh, Dp, 1.f, st);
+    const bool ok = flash_attn_bwd_tc(qkvp, dOp, lse, Dd, dqkvp, B, s, nh, Dp, img_bytes ? img : nullptr, img_bytes,
+                                      st);
+    if (ok) unpad(dqkvp, dqkv, T, 3, nh, dh, Dp, c, st);
+    kstats_end(tok, st);
+    if (ok) { note_launch(); return; }
+  }
   switch (dh) {
     case 16: launch_bwd<16>(qkv, O, dO, lse, dqkv, Dd, B, s, nh, st, ds_ws, ds_ws_bytes); break;
     case 32: launch_bwd<32>(qkv, O, dO, lse, dqkv, Dd, B, s, nh, st, ds_ws, ds_ws_bytes); break;

@@ -1481,23 +1481,24 @@ void norm_bwd_mixed(const __nv_bfloat16* dy, const __nv_bfloat16* x, const float
 }
 
 template <class T>
-void attn_fwd(const T* qkv, T* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st) {
+void attn_fwd(const T* qkv, T* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st, void* pad_ws) {
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
-    if (flash_attn_supported(dh)) { flash_attn_fwd(qkv, O, lse, B, s, nh, dh, st); return; }
+    if (flash_attn_supported(dh)) { flash_attn_fwd(qkv, O, lse, B, s, nh, dh, st, pad_ws); return; }
   }
+  (void)pad_ws;
   attn_fwd_k<T><<<cdiv(static_cast<long>(B) * s * nh, 8), 256, 0, st>>>(qkv, O, lse, B, s, nh, dh);
   note_launch();
 }
 template <class T>
 void attn_bwd(const T* qkv, const T* O, const T* dO, const float* lse, T* dqkv, float* Dsc, int B, int s, int nh,
-              int dh, cudaStream_t st, void* ds_ws, size_t ds_ws_bytes) {
+              int dh, cudaStream_t st, void* ds_ws, size_t ds_ws_bytes, void* pad_ws) {
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
     if (flash_attn_supported(dh)) {
-      flash_attn_bwd(qkv, O, dO, lse, dqkv, Dsc, B, s, nh, dh, st, ds_ws, ds_ws_bytes);
+      flash_attn_bwd(qkv, O, dO, lse, dqkv, Dsc, B, s, nh, dh, st, ds_ws, ds_ws_bytes, pad_ws);
       return;
     }
   }
-  (void)ds_ws; (void)ds_ws_bytes;
+  (void)ds_ws; (void)ds_ws_bytes; (void)pad_ws;
   const int grid = cdiv(static_cast<long>(B) * s * nh, 8);
   attn_bwd_dq_k<T><<<grid, 256, 0, st>>>(qkv, O, dO, lse, dqkv, Dsc, B, s, nh, dh);
   note_launch();
@@ -1607,9 +1608,9 @@ void sum_copies_f32(float* dst, const CopySrcs& srcs, size_t n, cudaStream_t st)
   template void colsum<T>(const T*, const T*, const float*, int, int, int, int, float*, float*, float*, cudaStream_t); \
   template void norm_bwd<T>(const T*, const T*, const float*, const float*, const T*, T*, int, int, int, float*,      \
                             float*, float*, float*, size_t, cudaStream_t);                                           \
-  template void attn_fwd<T>(const T*, T*, float*, int, int, int, int, cudaStream_t);                                 \
+  template void attn_fwd<T>(const T*, T*, float*, int, int, int, int, cudaStream_t, void*);                                 \
   template void attn_bwd<T>(const T*, const T*, const T*, const float*, T*, float*, int, int, int, int, cudaStream_t, \
-                            void*, size_t);                                                                    \
+                            void*, size_t, void*);                                                                 \
   template void rope<T>(T*, int, int, int, int, float, int, cudaStream_t);                                           \
   template void swiglu_fwd<T>(const T*, T*, int, int, cudaStream_t);                                                 \
   template void swiglu_bwd<T>(const T*, const T*, T*, int, int, cudaStream_t);                                       \

@@ -65,13 +65,14 @@ template <class T> void colsum(const T* a, const T* x, const float* stats, int r
                                float* out0, float* out1, float* partial, cudaStream_t st);
 
 // Causal attention over QKV [T, 3h] (q | k | v), heads of dh; O [T, h]; lse [nh][T] fp32.
-template <class T> void attn_fwd(const T* qkv, T* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st);
+template <class T> void attn_fwd(const T* qkv, T* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st,
+                                 void* pad_ws = nullptr);
 // dqkv [T, 3h] from dO; Dscratch [nh][T] fp32.
 // ds_ws (optional, >= flash_attn_bwd_ds_bytes): workspace for the dS image, which lets the bf16
 // tcgen05 path compute dQ from the stored dS (fa_bwd_dq_img) instead of recomputing S and dP.
 template <class T> void attn_bwd(const T* qkv, const T* O, const T* dO, const float* lse, T* dqkv, float* Dscratch,
                                  int B, int s, int nh, int dh, cudaStream_t st, void* ds_ws = nullptr,
-                                 size_t ds_ws_bytes = 0);
+                                 size_t ds_ws_bytes = 0, void* pad_ws = nullptr);
 // bytes of that dS workspace for a shape (0 when the path does not apply)
 size_t flash_attn_bwd_ds_bytes(int dh, int B, int s, int nh);
 
@@ -95,10 +96,21 @@ void loss_reduce(const float* row_loss, int rows, double* out, cudaStream_t st);
 
 // Tensor-core flash attention (bf16, mma.sync), used by attn_fwd/attn_bwd<bf16>.
 bool flash_attn_supported(int dh);
-void flash_attn_fwd(const __nv_bfloat16* qkv, __nv_bfloat16* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st);
+// pad_ws (>= flash_attn_pad_bytes): a head dim the tcgen05 kernels do not tile (16, 32, 80) runs
+// on them over zero-padded copies (attn_mma.cu); without it such head dims take mma.sync.
+void flash_attn_fwd(const __nv_bfloat16* qkv, __nv_bfloat16* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st,
+                    void* pad_ws = nullptr);
 void flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* O, const __nv_bfloat16* dO, const float* lse,
                     __nv_bfloat16* dqkv, float* Dd, int B, int s, int nh, int dh, cudaStream_t st,
-                    void* ds_ws = nullptr, size_t ds_ws_bytes = 0);
+                    void* ds_ws = nullptr, size_t ds_ws_bytes = 0, void* pad_ws = nullptr);
+// bytes of the padded-head workspace (bwd = 0 forward, 1 backward incl. its dS image); 0: no padding
+size_t flash_attn_pad_bytes(int dh, int B, int s, int nh, int bwd);
+bool flash_attn_bwd_tc_supported(int dh, int B, int s, int nh);
+bool flash_attn_fwd_tc(const __nv_bfloat16* qkv, __nv_bfloat16* O, float* lse, int B, int s, int nh, int dh,
+                       cudaStream_t st);
+bool flash_attn_bwd_tc(const __nv_bfloat16* qkv, const __nv_bfloat16* dO, const float* lse, const float* Dd,
+                       __nv_bfloat16* dqkv, int B, int s, int nh, int dh, void* ds_ws, size_t ds_ws_bytes,
+                       cudaStream_t st);
 
 void cast_f32_bf16(const float* x, __nv_bfloat16* y, size_t n, cudaStream_t st);
 void add_f32(float* a, const float* b, size_t n, cudaStream_t st);       // a += b
