@@ -352,10 +352,10 @@ def device_sms(torch):
 
 def main():
     args = parse()
-    C = CONFIGS[args.config]
-    cfg = C["model"]()
+    CE = CONFIGS[args.config]
+    cfg = CE["model"]()
     if args.micro is None:
-        args.micro = C["micro"]
+        args.micro = CE["micro"]
     gbs = args.micro * cfg.micro_batch
     if args.impl == "reference":
         run_reference(args, cfg, gbs)
@@ -369,8 +369,8 @@ def main():
         levels = tuple(os.environ.get("MARIO_EMU_LEVELS", "base,ckpt,mario").split(","))
         print(json.dumps({"pipeline_emulated": emulate_pipeline(cfg, api, torch, S=args.emulate, n_micro=args.micro,
                                                                 steps=max(1, min(args.steps, 3)), warmup=2,
-                                                                levels=levels, scheme=args.scheme or C["scheme"],
-                                                                chunks=C["chunks"])}), flush=True)
+                                                                levels=levels, scheme=args.scheme or CE["scheme"],
+                                                                chunks=CE["chunks"])}), flush=True)
         return
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -385,8 +385,8 @@ def main():
     assert world % args.dp == 0 and args.micro % args.dp == 0, "--dp must divide --gpus and --micro"
     S, rep, n_rep = world // args.dp, rank // (world // args.dp), args.micro // args.dp
     stage = rank % S
-    scheme = args.scheme or (C["scheme"] if S > 1 else "1f1b")
-    chunks = C["chunks"] if scheme == "interleave" else 1
+    scheme = args.scheme or (CE["scheme"] if S > 1 else "1f1b")
+    chunks = CE["chunks"] if scheme == "interleave" else 1
     args.scheme = scheme
     plan = api.Plan(cfg, S, n_rep, scheme, args.level, chunks=chunks, dtype="bf16")
     ctx = api.Context(rank, world, local, dp=args.dp)
@@ -507,7 +507,7 @@ def main():
         alg_flops += (S_ - 1) * (cfg.n_layers // S_) * layer_f * gbs   # RC of every checkpointed stage
     alg_tflops = alg_flops / (ms_step / 1e3) / world / 1e12
     mem = torch.cuda.max_memory_allocated()
-    metric = METRIC if args.config == "cfg2" else (f"samples/s ({C['name']}, seq {cfg.seq_len}, GBS {gbs}, "
+    metric = METRIC if args.config == "cfg2" else (f"samples/s ({CE['name']}, seq {cfg.seq_len}, GBS {gbs}, "
                                                    f"Mario plan, bf16)")
     out = {"metric": metric, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
            "warmup": args.warmup, "ms_per_step": ms_step, "higher_is_better": True, "scaling": "strong",
@@ -544,7 +544,7 @@ def main():
     ctx.close()
     if rank == 0 and world == 1 and args.emulate > 1 and args.config != "cfg5":
         out["pipeline_emulated"] = emulate_pipeline(cfg, api, torch, S=args.emulate, n_micro=args.micro,
-                                                    scheme=C["scheme"], chunks=C["chunks"],
+                                                    scheme=CE["scheme"], chunks=CE["chunks"],
                                                     steps=max(1, min(args.steps, 3)), warmup=2)
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         n_cores = cores()

@@ -13,11 +13,6 @@
 namespace mario {
 
 int g_attn_variant = -1;   // mario_k_attn_set_variant: -1 auto (tcgen05 where supported), 0 mma.sync only
-bool flash_attn_bwd_tc(const __nv_bfloat16* qkv, const __nv_bfloat16* dO, const float* lse, const float* Dd,
-                       __nv_bfloat16* dqkv, int B, int s, int nh, int dh, void* ds_ws, size_t ds_ws_bytes,
-                       cudaStream_t st);   // attn_tc.cu
-bool flash_attn_fwd_tc(const __nv_bfloat16* qkv, __nv_bfloat16* O, float* lse, int B, int s, int nh, int dh,
-                       cudaStream_t st);   // attn_tc.cu
 
 namespace {
 
@@ -507,11 +502,10 @@ bool flash_attn_supported(int dh) { return dh == 16 || dh == 32 || dh == 64 || d
 
 // ------------------------------------------------------------------ padded head dims on tcgen05
 // Head dims the tcgen05 kernels do not tile (16, 32, 80: GPT-3 2.7B's dh 80 in cfg 4) run on the
-// dh_p = 64 / 128 kernels over zero-padded copies: QKV [T][3][nh][dh] -> [T][3][nh][dh_p] with the
-// q part scaled by c = sqrt(dh_p / dh), so the kernels' 1/sqrt(dh_p) softmax scale gives
-// q.k / sqrt(dh) exactly up to the one bf16 rounding of c q (none when c is a power of 2); the
-// zero columns add nothing to q.k, and O / dK / dV padding columns are zero and dropped. dQ of the
-// unscaled q is c dQ'. Row sums D = rowsum(dO O) come from the unpadded tensors.
+// dh_p = 64 / 128 kernels over zero-padded copies: QKV [T][3][nh][dh] -> [T][3][nh][dh_p], the
+// kernels told the true softmax scale 1/sqrt(dh); the zero columns add nothing to q.k, and the
+// O / dQ / dK / dV padding columns are zero and dropped. Row sums D = rowsum(dO O) come from the
+// unpadded tensors. Same values as an unpadded kernel: only zeros are added to each dot product.
 namespace {
 int padded_dh(int dh) { return dh < 64 ? 64 : 128; }
 bool needs_pad(int dh) { return dh != 64 && dh != 128 && dh % 8 == 0 && dh < 128; }
@@ -604,8 +598,8 @@ void flash_attn_fwd(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, 
     bf16* Op = qkvp + ((T * 3 * nh * Dp * 2 + 255) / 256 * 256) / 2;
     const double fl = 4.0 * B * nh * dh * (static_cast<double>(s) * (s + 1) / 2);
     const int tok = kstats_begin(K_ATTN_FWD, fl, 0.0, st);
-    pad(qkv, qkvp, T, 3, nh, dh, Dp, sqrtf(static_cast<float>(Dp) / dh), st);
-    const bool ok = flash_attn_fwd_tc(qkvp, Op, lse, B, s, nh, Dp, st);
+    pad(qkv, qkvp, T, 3, nh, dh, Dp, 1.f, st);
+    const bool ok = flash_attn_fwd_tc(qkvp, Op, lse, B, s, nh, Dp, st, rsqrtf(static_cast<float>(dh)));
     if (ok) unpad(Op, O, T, 1, nh, dh, Dp, 1.f, st);
     kstats_end(tok, st);
     if (ok) return;
@@ -637,14 +631,13 @@ void flash_attn_bwd(const bf16* qkv, const bf16* O, const bf16* dO, const float*
       fa_bwd_dot_k<<<static_cast<int>((thr + 255) / 256), 256, 0, st>>>(O, dO, Dd, T, nh, dh);
       note_launch();
     }
-    const float c = sqrtf(static_cast<float>(Dp) / dh);
     const double fl = 8.0 * B * nh * dh * (static_cast<double>(s) * (s + 1) / 2);
     const int tok = kstats_begin(K_ATTN_BWD, fl, 0.0, st);
-    pad(qkv, qkvp, T, 3, nh, dh, Dp, c, st);
+    pad(qkv, qkvp, T, 3, nh, dh, Dp, 1.f, st);
     pad(dO, dOp, T, 1, nh, dh, Dp, 1.f, st);
     const bool ok = flash_attn_bwd_tc(qkvp, dOp, lse, Dd, dqkvp, B, s, nh, Dp, img_bytes ? img : nullptr, img_bytes,
-                                      st);
-    if (ok) unpad(dqkvp, dqkv, T, 3, nh, dh, Dp, c, st);
+                                      st, rsqrtf(static_cast<float>(dh)));
+    if (ok) unpad(dqkvp, dqkv, T, 3, nh, dh, Dp, 1.f, st);
     kstats_end(tok, st);
     if (ok) { note_launch(); return; }
   }

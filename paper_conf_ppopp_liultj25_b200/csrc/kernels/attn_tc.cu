@@ -175,7 +175,8 @@ template <int DH>
 __global__ void __launch_bounds__(kThreadsB, 1)
 fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_qkv64,
                const __grid_constant__ CUtensorMap tm_do64, const __grid_constant__ CUtensorMap tm_dqkv,
-               const float* lse, const float* Dd, bf16* dqkv, int B, int s, int nh, int dbg, long long* trace) {
+               const float* lse, const float* Dd, bf16* dqkv, int B, int s, int nh, int dbg, long long* trace,
+               float qk_scale) {
   const bool bulk_ld = (s % kCols) == 0;
   using SM = Smem<DH>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -212,7 +213,7 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
   const int i0 = (kt * kRows) / kCols;
   const int nq = (s + kCols - 1) / kCols;
   const int ntiles = (dbg & 32) ? min(nq - i0, 1) : nq - i0;
-  const float sl2 = rsqrtf(static_cast<float>(DH)) * LOG2E;
+  const float sl2 = qk_scale * LOG2E;
 
   if (warp == 0 && lane == 0) {
     tma_prefetch_desc(&tm_qkv128);
@@ -406,7 +407,7 @@ fa_bwd_dkdv_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
     // tcgen05.ld is warp-collective (.sync.aligned): every lane loads, only valid keys store.
     // Full 128-key blocks (s % 128 == 0): rows go to the (now idle) P/dS buffers in the SW128 layout
     // and leave as four TMA tensor stores (coalesced); otherwise row-wise stores.
-    const float scale = rsqrtf(static_cast<float>(DH));
+    const float scale = qk_scale;
     const bool tma_st = (s % kRows) == 0 && !(dbg & 64);
     auto stV = [&](int a) { return a ? sS(0) : sP(0); };
     auto stK = [&](int a) { return a ? sS(1) : sP(1); };
@@ -467,7 +468,7 @@ template <int DH>
 __global__ void __launch_bounds__(kThreadsB, 1)
 fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_qkv64,
              const __grid_constant__ CUtensorMap tm_do128, const __grid_constant__ CUtensorMap tm_dqkv,
-             const float* lse, const float* Dd, bf16* dqkv, int B, int s, int nh, int dbg) {
+             const float* lse, const float* Dd, bf16* dqkv, int B, int s, int nh, int dbg, float qk_scale) {
   using SM = Smem<DH>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -497,7 +498,7 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
   const long Ttok = static_cast<long>(B) * s;
   const int last_q = min(qt * kRows + kRows - 1, s - 1);
   const int ntiles = (dbg & 32) ? 1 : last_q / kCols + 1;   // key tiles 0 .. last_q/64
-  const float sl2 = rsqrtf(static_cast<float>(DH)) * LOG2E;
+  const float sl2 = qk_scale * LOG2E;
 
   if (warp == 0 && lane == 0) {
     tma_prefetch_desc(&tm_qkv128);
@@ -637,7 +638,7 @@ fa_bwd_dq_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constan
     if (half == 1) goto done_dq;
     mbar_wait(acc_done, 0);
     tc_fence_after();
-    const float scale = rsqrtf(static_cast<float>(DH));
+    const float scale = qk_scale;
     const bool tma_st = (s % kRows) == 0 && !(dbg & 64);
     bf16* qrow = dqkv + gr * (3 * h) + head * DH;
 #pragma unroll 1
@@ -695,7 +696,7 @@ __global__ void __launch_bounds__(kThreadsB, 1)
 fa_bwd_dkdv_ts(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_qkv64,
                const __grid_constant__ CUtensorMap tm_do64,
                const __grid_constant__ CUtensorMap tm_dqkv, const float* lse, const float* Dd, bf16* dqkv, int B,
-               int s, int nh, uint8_t* dsimg, int l2hint) {
+               int s, int nh, uint8_t* dsimg, int l2hint, float qk_scale) {
   const bool bulk_ld = (s % kCols) == 0;
   using SM = Smem<DH>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -723,7 +724,7 @@ fa_bwd_dkdv_ts(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
   const int i0 = (kt * kRows) / kCols;
   const int nq = (s + kCols - 1) / kCols;
   const int ntiles = nq - i0;
-  const float sl2 = rsqrtf(static_cast<float>(DH)) * LOG2E;
+  const float sl2 = qk_scale * LOG2E;
   (void)nt;
 
   if (warp == 0 && lane == 0) {
@@ -906,7 +907,7 @@ fa_bwd_dkdv_ts(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
     mbar_wait(acc_done, 0);
     tc_fence_after();
     {
-      const float scale = rsqrtf(static_cast<float>(DH));
+      const float scale = qk_scale;
       const bool tma_st = (s % kRows) == 0;
       // staging for the TMA stores: the (now idle) ring slots 0 and 1, four 128-row x 128-byte tiles
       auto stV = [&](int a) { return a ? sG(0) : sQ(0); };
@@ -979,7 +980,7 @@ template <int DH>
 __global__ void __launch_bounds__(kThreadsP, 1)
 fa_bwd_dq_pers(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_qkv64,
                const __grid_constant__ CUtensorMap tm_do128, const float* lse, const float* Dd, bf16* dqkv, int B,
-               int s, int nh) {
+               int s, int nh, float qk_scale) {
   using SM = Smem<DH>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -1005,7 +1006,7 @@ fa_bwd_dq_pers(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
   const int nt = (s + kRows - 1) / kRows, BH = B * nh, W = nt * BH;
   const int h = nh * DH;
   const long Ttok = static_cast<long>(B) * s;
-  const float sl2 = rsqrtf(static_cast<float>(DH)) * LOG2E;
+  const float sl2 = qk_scale * LOG2E;
   // item w -> (qt, b, head): heaviest query tiles first over all (sample, head)
   auto item = [&](int w, int& qt, int& b, int& head, int& ntiles) {
     const int j = w / BH, bh = w % BH;
@@ -1166,7 +1167,7 @@ fa_bwd_dq_pers(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
     const int quarter = warp & 3;
     const int row = quarter * 32 + lane;
     const uint32_t lane_off = static_cast<uint32_t>(quarter * 32) << 16;
-    const float scale = rsqrtf(static_cast<float>(DH));
+    const float scale = qk_scale;
     int n = 0;
     for (int w = blockIdx.x; w < W; w += gridDim.x, ++n) {
       int qt, b, head, ntiles;
@@ -1230,7 +1231,7 @@ struct SmemI {
 template <int DH>
 __global__ void __launch_bounds__(kThreadsI, 1)
 fa_bwd_dq_img(const __grid_constant__ CUtensorMap tm_qkv64, const uint8_t* __restrict__ dsimg, bf16* dqkv, int B, int s,
-              int nh, int l2hint) {
+              int nh, int l2hint, float qk_scale) {
   using SI = SmemI<DH>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -1312,7 +1313,7 @@ fa_bwd_dq_img(const __grid_constant__ CUtensorMap tm_qkv64, const uint8_t* __res
     const int quarter = warp & 3;
     const int row = quarter * 32 + lane;
     const uint32_t lane_off = static_cast<uint32_t>(quarter * 32) << 16;
-    const float scale = rsqrtf(static_cast<float>(DH));
+    const float scale = qk_scale;
     int n = 0;
     for (int w = blockIdx.x; w < W; w += gridDim.x, ++n) {
       int qb, bh, ntiles;
@@ -1361,7 +1362,7 @@ int g_attn_dq_pers = 1;   // MARIO_ATTN_DQ_PERS=0 selects the one-item-per-CTA d
 
 template <int DH>
 bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, bf16* dqkv, int B, int s, int nh,
-            uint8_t* dsimg, cudaStream_t st) {
+            uint8_t* dsimg, cudaStream_t st, float qk_scale) {
   const int h = nh * DH;
   const long T = static_cast<long>(B) * s;
   CUtensorMap m128, m64, d64, d128, g128;
@@ -1397,10 +1398,10 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
         tset = true;
       }
       fa_bwd_dkdv_ts<DH><<<grid, kThreadsB, smem_dkdv_ts<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s, nh,
-                                                                        dsimg, attn_l2hint());
+                                                                        dsimg, attn_l2hint(), qk_scale);
     } else {
       fa_bwd_dkdv_tc<DH><<<grid, kThreadsB, smem_dkdv<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s, nh, dbg,
-                                                                     want_trace ? trace : nullptr);
+                                                                     want_trace ? trace : nullptr, qk_scale);
     }
     if (want_trace) {
       long long h[8 * 64];
@@ -1425,7 +1426,8 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
     const int items = B * nh * (s / kRows);
     static const int per_sm = getenv("MARIO_DQI_CTAS") ? atoi(getenv("MARIO_DQI_CTAS")) : 2;
     const int grid_i = items < per_sm * sms ? items : per_sm * sms;
-    fa_bwd_dq_img<DH><<<grid_i, kThreadsI, SmemI<DH>::kBytes, st>>>(m64, dsimg, dqkv, B, s, nh, attn_l2hint());
+    fa_bwd_dq_img<DH><<<grid_i, kThreadsI, SmemI<DH>::kBytes, st>>>(m64, dsimg, dqkv, B, s, nh, attn_l2hint(),
+                                                                     qk_scale);
   } else if (!only || only[1] == 'q') {
     if (pers && dbg == 0) {
       static bool pset = false;
@@ -1436,9 +1438,10 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
       const int sms = device_sm_count();
       const int items = B * nh * ((s + kRows - 1) / kRows);
       fa_bwd_dq_pers<DH><<<items < sms ? items : sms, kThreadsP, smem_dq<DH>(), st>>>(m128, m64, d128, lse, Dd, dqkv,
-                                                                                         B, s, nh);
+                                                                                         B, s, nh, qk_scale);
     } else {
-      fa_bwd_dq_tc<DH><<<grid, kThreadsB, smem_dq<DH>(), st>>>(m128, m64, d128, g128, lse, Dd, dqkv, B, s, nh, dbg);
+      fa_bwd_dq_tc<DH><<<grid, kThreadsB, smem_dq<DH>(), st>>>(m128, m64, d128, g128, lse, Dd, dqkv, B, s, nh, dbg,
+                                                               qk_scale);
     }
   }
   note_launch(2);
@@ -1456,7 +1459,7 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
 template <int DH>
 __global__ void __launch_bounds__(kThreadsB, 1)
 fa_fwd_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_qkv64, bf16* O,
-          float* lse, int B, int s, int nh) {
+          float* lse, int B, int s, int nh, float qk_scale) {
   using SM = Smem<DH>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -1483,7 +1486,7 @@ fa_fwd_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__
   const long Ttok = static_cast<long>(B) * s;
   const int last_q = min(qt * kRows + kRows - 1, s - 1);
   const int ntiles = last_q / kCols + 1;
-  const float sl2 = rsqrtf(static_cast<float>(DH)) * LOG2E;
+  const float sl2 = qk_scale * LOG2E;
 
   if (warp == 0 && lane == 0) {
     tma_prefetch_desc(&tm_qkv128);
@@ -1703,7 +1706,8 @@ __device__ __forceinline__ void f2_item(int i, int n, bool& is_v, int& j) {
 
 template <int DH>
 __global__ void __launch_bounds__(kF2Threads, 1)
-fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, int B, int s, int nh, int g_l2hint) {
+fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, int B, int s, int nh, int g_l2hint,
+           float qk_scale) {
   using SM = SmemF2<DH>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -1728,7 +1732,7 @@ fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, i
   const long Ttok = static_cast<long>(B) * s;
   const int q0 = qb * 2 * kF2Q;
   const int n0 = 2 * qb + 1, n1 = 2 * qb + 2;      // key tiles seen by Q tile 0 / 1
-  const float sl2 = rsqrtf(static_cast<float>(DH)) * LOG2E;
+  const float sl2 = qk_scale * LOG2E;
 
   if (warp == 0 && lane == 0) {
     tma_prefetch_desc(&tm_qkv128);
@@ -1932,7 +1936,7 @@ fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, i
 }
 
 template <int DH>
-bool launch_fwd2_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, cudaStream_t st) {
+bool launch_fwd2_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, cudaStream_t st, float qk_scale) {
   const int h = nh * DH;
   const long T = static_cast<long>(B) * s;
   CUtensorMap m128;
@@ -1944,7 +1948,7 @@ bool launch_fwd2_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, 
     set = true;
   }
   const int nqb = (s + 2 * kF2Q - 1) / (2 * kF2Q);
-  fa_fwd2_tc<DH><<<nqb * B * nh, kF2Threads, smem, st>>>(m128, O, lse, B, s, nh, attn_l2hint());
+  fa_fwd2_tc<DH><<<nqb * B * nh, kF2Threads, smem, st>>>(m128, O, lse, B, s, nh, attn_l2hint(), qk_scale);
   note_launch();
   return true;
 }
@@ -1953,7 +1957,7 @@ template <int DH>
 constexpr int smem_fwd() { return at_least_one_sm(Smem<DH>::kBig + 2 * kRing * Smem<DH>::kSmall + 2 * Smem<DH>::kP + 2 * kRows * 4 + 256 + 1024); }
 
 template <int DH>
-bool launch_fwd_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, cudaStream_t st) {
+bool launch_fwd_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, cudaStream_t st, float qk_scale) {
   const int h = nh * DH;
   const long T = static_cast<long>(B) * s;
   CUtensorMap m128, m64;
@@ -1965,7 +1969,7 @@ bool launch_fwd_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, c
     set = true;
   }
   dim3 grid((s + kRows - 1) / kRows, B * nh);
-  fa_fwd_tc<DH><<<grid, kThreadsB, smem_fwd<DH>(), st>>>(m128, m64, O, lse, B, s, nh);
+  fa_fwd_tc<DH><<<grid, kThreadsB, smem_fwd<DH>(), st>>>(m128, m64, O, lse, B, s, nh, qk_scale);
   note_launch();
   return true;
 }
@@ -1976,27 +1980,30 @@ bool flash_attn_bwd_tc_supported(int dh, int B, int s, int nh) {
   return (dh == 64 || dh == 128) && ((nh * dh) % 64 == 0);
 }
 
-bool flash_attn_fwd_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st) {
+bool flash_attn_fwd_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st,
+                       float qk_scale) {
+  if (qk_scale <= 0.f) qk_scale = rsqrtf(static_cast<float>(dh));
   // g_attn_variant: -1 auto (two-Q-tile kernel unless it would launch fewer CTAs than SMs: the
   // one-Q-tile kernel has twice as many), 2 force the one-Q-tile kernel, 3 force the two-Q-tile one
   const int sms = device_sm_count();
   const long ctas2 = static_cast<long>((s + 2 * kF2Q - 1) / (2 * kF2Q)) * B * nh;
   if (g_attn_variant == 2 || (g_attn_variant != 3 && ctas2 < sms)) {
-    if (dh == 128) return launch_fwd_tc<128>(qkv, O, lse, B, s, nh, st);
-    if (dh == 64) return launch_fwd_tc<64>(qkv, O, lse, B, s, nh, st);
+    if (dh == 128) return launch_fwd_tc<128>(qkv, O, lse, B, s, nh, st, qk_scale);
+    if (dh == 64) return launch_fwd_tc<64>(qkv, O, lse, B, s, nh, st, qk_scale);
     return false;
   }
-  if (dh == 128) return launch_fwd2_tc<128>(qkv, O, lse, B, s, nh, st);
-  if (dh == 64) return launch_fwd2_tc<64>(qkv, O, lse, B, s, nh, st);
+  if (dh == 128) return launch_fwd2_tc<128>(qkv, O, lse, B, s, nh, st, qk_scale);
+  if (dh == 64) return launch_fwd2_tc<64>(qkv, O, lse, B, s, nh, st, qk_scale);
   return false;
 }
 
 // Returns false if the configuration is unsupported (caller falls back to the mma.sync kernels).
 bool flash_attn_bwd_tc(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, bf16* dqkv, int B, int s,
-                       int nh, int dh, void* ds_ws, size_t ds_ws_bytes, cudaStream_t st) {
+                       int nh, int dh, void* ds_ws, size_t ds_ws_bytes, cudaStream_t st, float qk_scale) {
+  if (qk_scale <= 0.f) qk_scale = rsqrtf(static_cast<float>(dh));
   uint8_t* img = ds_ws && ds_ws_bytes >= flash_attn_bwd_ds_bytes(dh, B, s, nh) ? static_cast<uint8_t*>(ds_ws) : nullptr;
-  if (dh == 128) return launch<128>(qkv, dO, lse, Dd, dqkv, B, s, nh, img, st);
-  if (dh == 64) return launch<64>(qkv, dO, lse, Dd, dqkv, B, s, nh, img, st);
+  if (dh == 128) return launch<128>(qkv, dO, lse, Dd, dqkv, B, s, nh, img, st, qk_scale);
+  if (dh == 64) return launch<64>(qkv, dO, lse, Dd, dqkv, B, s, nh, img, st, qk_scale);
   return false;
 }
 

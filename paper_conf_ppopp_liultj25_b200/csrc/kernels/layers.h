@@ -106,11 +106,12 @@ void flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* O, const __nv
 // bytes of the padded-head workspace (bwd = 0 forward, 1 backward incl. its dS image); 0: no padding
 size_t flash_attn_pad_bytes(int dh, int B, int s, int nh, int bwd);
 bool flash_attn_bwd_tc_supported(int dh, int B, int s, int nh);
+// qk_scale: the softmax scale of q.k (<= 0: 1/sqrt(dh); the padded path passes 1/sqrt of the true dh)
 bool flash_attn_fwd_tc(const __nv_bfloat16* qkv, __nv_bfloat16* O, float* lse, int B, int s, int nh, int dh,
-                       cudaStream_t st);
+                       cudaStream_t st, float qk_scale = 0.f);
 bool flash_attn_bwd_tc(const __nv_bfloat16* qkv, const __nv_bfloat16* dO, const float* lse, const float* Dd,
                        __nv_bfloat16* dqkv, int B, int s, int nh, int dh, void* ds_ws, size_t ds_ws_bytes,
-                       cudaStream_t st);
+                       cudaStream_t st, float qk_scale = 0.f);
 
 void cast_f32_bf16(const float* x, __nv_bfloat16* y, size_t n, cudaStream_t st);
 void add_f32(float* a, const float* b, size_t n, cudaStream_t st);       // a += b

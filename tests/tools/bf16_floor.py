@@ -207,6 +207,9 @@ def main():
     if not os.environ.get("FP32DH_ONLY"):
         variants += [(f"all-{p}", set(POINTS) - {p}) for p in pts]
         variants += [(f"only-{p}", {p}) for p in pts]
+    keep = os.environ.get("VARIANTS")
+    if keep:
+        variants = [v for v in variants if v[0] in keep.split(",")]
     for tag, on in variants:
         l1, g1 = step_rounded(cfg, params, toks, N, on)
         (ei, ki), (el, kl) = errors(g1, g_o)
