@@ -141,6 +141,9 @@ mario_status mario_plan_rank_params(const struct mario_plan* plan, int32_t rank,
 /* Name of the global parameter `idx` (canonical order), e.g. "h3.qkv.w". */
 const char* mario_param_name(const struct mario_plan* plan, int32_t idx);
 int32_t mario_param_count(const struct mario_plan* plan);
+/* Shape of global parameter `idx`: *ndim (1 or 2) dims written to dims[4] (row-major, e.g.
+ * qkv.w = [3h, h]). EINVAL on a bad index or NULL pointers. */
+mario_status mario_param_shape(const struct mario_plan* plan, int32_t idx, int64_t* dims, int32_t* ndim);
 /* k of MARIO_LEVEL_BUDGET (0 for the other levels); -1 on NULL. */
 int32_t mario_plan_unckpt_tail(const struct mario_plan* plan);
 void mario_plan_destroy(struct mario_plan* plan);

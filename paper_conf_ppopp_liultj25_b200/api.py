@@ -86,6 +86,7 @@ _lib.register("mario_plan_rank_params", C.c_int32, [_P, C.c_int32, C.POINTER(C.P
                                                     C.POINTER(C.POINTER(C.c_uint64)), C.POINTER(C.c_int32)])
 _lib.register("mario_param_name", C.c_char_p, [_P, C.c_int32])
 _lib.register("mario_param_count", C.c_int32, [_P])
+_lib.register("mario_param_shape", C.c_int32, [_P, C.c_int32, C.POINTER(C.c_int64), C.POINTER(C.c_int32)])
 _lib.register("mario_plan_destroy", None, [_P])
 _lib.register("mario_plan_unckpt_tail", C.c_int32, [_P])
 _lib.register("mario_last_error", C.c_char_p, [])
@@ -272,8 +273,14 @@ def unpack_params(plan: Plan, flat, rank: int) -> Dict[str, "object"]:
 
 
 def _shapes(plan: Plan):
-    import synth
-    return synth.param_shapes(plan.cfg)
+    """(name, shape) of every global parameter, from the library (mario_param_shape)."""
+    L = _lib.lib()
+    out = []
+    dims, nd = (C.c_int64 * 4)(), C.c_int32()
+    for i, name in enumerate(plan.param_names()):
+        _check(L.mario_param_shape(plan.handle, i, dims, C.byref(nd)))
+        out.append((name, tuple(int(dims[j]) for j in range(nd.value))))
+    return out
 
 
 class Context:

@@ -60,6 +60,66 @@ struct SlotPool {
   void release(int i) { if (i >= 0) used[i] = false; }
 };
 
+// Every instruction in order of its time on the simulator's timeline (A12: compute at its start, a
+// send when posted, a receive when its data is in), merged over the devices so each device's list
+// order is kept and a receive never precedes its send. Empty if the lists do not simulate.
+std::vector<std::pair<int, int>> timed_order(const Pipe& pp, const Lists& L, const SimCosts& c) {
+  const int S = pp.S, P = pp.parts();
+  std::vector<std::vector<double>> t(S);
+  std::vector<double> post(static_cast<size_t>(S) * pp.N * P * 2, -1.0);
+  auto key = [&](int d, int m, int p, bool grad) { return ((static_cast<size_t>(d) * pp.N + m) * P + p) * 2 + (grad ? 1 : 0); };
+  std::vector<size_t> ptr(S, 0);
+  std::vector<double> dev_t(S, 0.0);
+  size_t total = 0, done = 0;
+  for (const List& l : L) total += l.size();
+  for (int d = 0; d < S; ++d) t[d].assign(L[d].size(), 0.0);
+  while (done < total) {
+    bool progressed = false;
+    for (int d = 0; d < S; ++d) {
+      while (ptr[d] < L[d].size()) {
+        const Instr& x = L[d][ptr[d]];
+        const int k = pp.vstage(d, x.p);
+        if (is_send(x.op)) {
+          post[key(d, x.m, x.p, x.op == SG)] = dev_t[d];
+        } else if (is_recv(x.op)) {
+          int sd, sp;
+          if (!find_inst(pp, d, x.m, x.p, x.op == RA ? FW : BW, false, &sd, &sp)) return {};
+          const double pt = post[key(sd, x.m, sp, x.op == RG)];
+          if (pt < 0) break;
+          dev_t[d] = std::max(dev_t[d], pt + (x.op == RA ? c.comm_act : c.comm_grad));
+        }
+        t[d][ptr[d]] = dev_t[d];
+        if (is_compute(x.op)) dev_t[d] += (x.op == FW || x.op == CFW) ? c.fw[k] : x.op == RC ? c.rc[k] : c.bw[k];
+        ++ptr[d];
+        ++done;
+        progressed = true;
+      }
+    }
+    if (!progressed) return {};
+  }
+  std::vector<std::pair<int, int>> order;
+  std::set<std::tuple<int, int, int, int>> sent;   // (sender device, op, m, p)
+  std::fill(ptr.begin(), ptr.end(), 0);
+  while (order.size() < total) {
+    int best = -1;
+    for (int d = 0; d < S; ++d) {
+      if (ptr[d] >= L[d].size()) continue;
+      const Instr& x = L[d][ptr[d]];
+      if (is_recv(x.op)) {
+        int sd, sp;
+        find_inst(pp, d, x.m, x.p, x.op == RA ? FW : BW, false, &sd, &sp);
+        if (!sent.count({sd, x.op == RA ? SA : SG, x.m, sp})) continue;
+      }
+      if (best < 0 || t[d][ptr[d]] < t[best][ptr[best]]) best = d;
+    }
+    if (best < 0) return {};
+    const Instr& x = L[best][ptr[best]];
+    if (is_send(x.op)) sent.insert({best, x.op, x.m, x.p});
+    order.push_back({best, static_cast<int>(ptr[best]++)});
+  }
+  return order;
+}
+
 void assign_slots_and_pools(PlanObj& P) {
   const Pipe& pp = P.pp;
   const int K = pp.K();
@@ -96,38 +156,48 @@ void assign_slots_and_pools(PlanObj& P) {
     }
     P.pools_mp[d] = {ck.high, ac.high, sa.high, sg.high, rg.high};
   }
-  // send slots are held until the receiver copies them out (loopback) or has consumed the message
-  // (NCCL / peer transport): the slot of every message is fixed here, along the loopback order
+  // send slots are held from the producing FW/CFW (BW) until the receiver copies them out (loopback)
+  // or has consumed the message (NCCL / peer transport): the slot of every message is fixed here,
+  // along a valid execution order of the DAG (see plan_obj.h)
+  auto assign = [&](const std::vector<std::pair<int, int>>& order, std::vector<std::map<std::pair<int, int>, int>>& sa,
+                    std::vector<std::map<std::pair<int, int>, int>>& sg, std::vector<PlanObj::Pools>& pools) {
+    sa.assign(pp.S, {});
+    sg.assign(pp.S, {});
+    std::vector<SlotPool> lsa(pp.S), lsg(pp.S);
+    std::map<std::tuple<int, int, int>, int> held_sa, held_sg;  // (sender dev, m, p) -> slot
+    for (auto [d, i] : order) {
+      const Instr& x = P.lists[d][i];
+      const int k = pp.vstage(d, x.p);
+      int sd, sp;
+      if ((x.op == FW || x.op == CFW) && k < K - 1) sa[d][{x.m, x.p}] = held_sa[{d, x.m, x.p}] = lsa[d].acquire();
+      if (x.op == BW && k > 0) sg[d][{x.m, x.p}] = held_sg[{d, x.m, x.p}] = lsg[d].acquire();
+      if (x.op == RA) {
+        find_inst(pp, d, x.m, x.p, FW, false, &sd, &sp);
+        lsa[sd].release(held_sa[{sd, x.m, sp}]);
+      }
+      if (x.op == RG) {
+        find_inst(pp, d, x.m, x.p, BW, false, &sd, &sp);
+        lsg[sd].release(held_sg[{sd, x.m, sp}]);
+      }
+    }
+    for (int d = 0; d < pp.S; ++d) {
+      pools[d].send_act = lsa[d].high;
+      pools[d].send_grad = lsg[d].high;
+    }
+  };
   P.pools_lb = P.pools_mp;
-  P.sa_slot.assign(pp.S, {});
-  P.sg_slot.assign(pp.S, {});
-  std::vector<SlotPool> lsa(pp.S), lsg(pp.S);
-  std::map<std::tuple<int, int, int>, int> held_sa, held_sg;  // (sender dev, m, p) -> slot
-  for (auto [d, i] : P.loopback_order) {
-    const Instr& x = P.lists[d][i];
-    const int k = pp.vstage(d, x.p);
-    int sd, sp;
-    if ((x.op == FW || x.op == CFW) && k < K - 1) P.sa_slot[d][{x.m, x.p}] = held_sa[{d, x.m, x.p}] = lsa[d].acquire();
-    if (x.op == BW && k > 0) P.sg_slot[d][{x.m, x.p}] = held_sg[{d, x.m, x.p}] = lsg[d].acquire();
-    if (x.op == RA) {
-      find_inst(pp, d, x.m, x.p, FW, false, &sd, &sp);
-      lsa[sd].release(held_sa[{sd, x.m, sp}]);
-    }
-    if (x.op == RG) {
-      find_inst(pp, d, x.m, x.p, BW, false, &sd, &sp);
-      lsg[sd].release(held_sg[{sd, x.m, sp}]);
-    }
-  }
-  for (int d = 0; d < pp.S; ++d) {
-    P.pools_lb[d].send_act = lsa[d].high;
-    P.pools_lb[d].send_grad = lsg[d].high;
-  }
-  P.pools_mp = P.pools_lb;   // every executor uses the loopback-order slot assignment
+  assign(P.loopback_order, P.sa_slot_lb, P.sg_slot_lb, P.pools_lb);
+  P.peer_order = timed_order(pp, P.lists, P.costs);
+  if (P.peer_order.empty()) P.peer_order = P.loopback_order;
+  assign(P.peer_order, P.sa_slot, P.sg_slot, P.pools_mp);
 }
 
 void build_rank_params(PlanObj& P) {
   P.params = model_params(P.model);
-  for (auto& ps : P.params) P.param_names.push_back(ps.name);
+  for (auto& ps : P.params) {
+    P.param_index[ps.name] = static_cast<int>(P.param_names.size());
+    P.param_names.push_back(ps.name);
+  }
   const int K = P.pp.K();
   P.rank_params.assign(P.pp.S, {});
   for (int d = 0; d < P.pp.S; ++d) {
@@ -349,11 +419,25 @@ extern "C" mario_status mario_plan(const mario_model* model, int32_t stages, int
       assign_slots_and_pools(*P);
       fill_static(*P, costs);
       if (lvl == MARIO_LEVEL_MARIO) {
-        P->lists = pass4_prepose_forward(pp, P->lists, P->costs, static_cast<double>(mem_budget_bytes));
-        P->loopback_order.clear();
-        if (!walk_order(pp, P->lists, P->loopback_order)) return set_error(MARIO_EDEADLOCK, "plan deadlocks");
-        assign_slots_and_pools(*P);
-        fill_static(*P, costs);
+        // Pass 4's budget test (P:272 via reading A17) walks the lists with the static bytes of the
+        // un-preposed plan, but a preposed CFW's output stays buffered until the receiver consumes it
+        // (P:222), so the plan's send slots -- part of the static bytes -- can grow. If the finished
+        // plan exceeds the budget, pass 4 is re-run against the budget minus the excess (at most a
+        // few times; the last resort preposes nothing, which never needs more than CKPT).
+        const Lists before = P->lists;
+        double eff = static_cast<double>(mem_budget_bytes);
+        for (int attempt = 0;; ++attempt) {
+          P->lists = (mem_budget_bytes > 0 && eff <= 0) ? before : pass4_prepose_forward(pp, before, P->costs, eff);
+          P->loopback_order.clear();
+          if (!walk_order(pp, P->lists, P->loopback_order)) return set_error(MARIO_EDEADLOCK, "plan deadlocks");
+          assign_slots_and_pools(*P);
+          fill_static(*P, costs);
+          if (mem_budget_bytes == 0 || eff <= 0) break;
+          const MemResult mr = memory_walk(pp, P->lists, P->costs);
+          const double worst = *std::max_element(mr.peak.begin(), mr.peak.end());
+          if (worst <= static_cast<double>(mem_budget_bytes)) break;
+          eff = attempt < 4 ? eff - (worst - static_cast<double>(mem_budget_bytes)) * 1.05 - 1.0 : 0.0;
+        }
       }
       return MARIO_OK;
     };
@@ -497,6 +581,15 @@ extern "C" mario_status mario_plan_rank_params(const struct mario_plan* P, int32
 extern "C" const char* mario_param_name(const struct mario_plan* P, int32_t idx) {
   if (!P || idx < 0 || idx >= static_cast<int32_t>(P->param_names.size())) return nullptr;
   return P->param_names[idx].c_str();
+}
+
+extern "C" mario_status mario_param_shape(const struct mario_plan* P, int32_t idx, int64_t* dims, int32_t* ndim) {
+  if (!P || idx < 0 || idx >= static_cast<int32_t>(P->params.size()) || !dims || !ndim)
+    return set_error(MARIO_EINVAL, "bad argument");
+  const auto& sh = P->params[idx].shape;
+  *ndim = static_cast<int32_t>(sh.size());
+  for (size_t i = 0; i < sh.size() && i < 4; ++i) dims[i] = sh[i];
+  return MARIO_OK;
 }
 
 extern "C" int32_t mario_param_count(const struct mario_plan* P) {

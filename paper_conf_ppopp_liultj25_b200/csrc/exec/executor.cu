@@ -194,12 +194,11 @@ struct Exec {
 
   // ---- weights --------------------------------------------------------------
   int tidx(Dev<T>& D, int p, const std::string& name) {
-    const auto& names = D.P->param_names;
-    for (size_t i = 0; i < names.size(); ++i)
-      if (names[i] == name) {
-        auto it = D.tensor.find({p, static_cast<int>(i)});
-        if (it != D.tensor.end()) return it->second;
-      }
+    const auto g = D.P->param_index.find(name);
+    if (g != D.P->param_index.end()) {
+      auto it = D.tensor.find({p, g->second});
+      if (it != D.tensor.end()) return it->second;
+    }
     throw std::runtime_error("parameter " + name + " not held by part " + std::to_string(p));
   }
   const T* Wm(Dev<T>& D, int p, const std::string& name) {   // compute-dtype matrix
@@ -535,7 +534,7 @@ struct Exec {
       case MARIO_OP_RC: {
         T* out = nullptr;
         if (x.op != MARIO_OP_RC && x.vstage < K - 1) {
-          const int i = D.P->sa_slot[d].at(key);   // the plan's slot (loopback-order assignment)
+          const int i = (loopback ? D.P->sa_slot_lb : D.P->sa_slot)[d].at(key);   // the plan's slot
           if (D.sa_used.at(i)) throw std::runtime_error("send slot still held (planner/executor mismatch)");
           D.sa_used[i] = true;
           D.sa_of[key] = i;
@@ -558,7 +557,7 @@ struct Exec {
         if (x.vstage < K - 1) dout = D.template at<T>(D.a.rg + static_cast<size_t>(D.rg_of[key]) * D.a.msg_stride);
         T* din = nullptr;
         if (x.vstage > 0) {
-          const int i = D.P->sg_slot[d].at(key);
+          const int i = (loopback ? D.P->sg_slot_lb : D.P->sg_slot)[d].at(key);
           if (D.sg_used.at(i)) throw std::runtime_error("send slot still held (planner/executor mismatch)");
           D.sg_used[i] = true;
           D.sg_of[key] = i;
@@ -954,9 +953,9 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
     E.st = body;
   } else if (peer) {
     // every rank runs on its own streams and waits only on flags, so the device executes the
-    // plan's DAG concurrently. The host enqueues in the loopback order (a valid order of the DAG in
+    // plan's DAG concurrently. The host enqueues in peer_order (the simulated timeline, the order in
     // which the send slots were assigned), so every flag wait follows the write it waits for
-    for (auto [d, i] : P.loopback_order) {
+    for (auto [d, i] : P.peer_order) {
       if (!E.can_walk(d, P.instrs[d][i])) throw std::runtime_error("peer walk: a flag wait precedes its write");
       E.run_instr(d, P.instrs[d][i]);
     }

@@ -129,9 +129,16 @@ __device__ __forceinline__ void cross_warp_sums(const float* rp, int nw, int lan
 }
 
 // shared memory: S slots of `stage_bytes` (16-byte multiples), S mbarriers, the reduction buffers
-constexpr int kPipeR = 2;   // rows per iteration of the norm kernels
-inline size_t pipe_smem_bytes(int S, int stage_bytes) {
-  return static_cast<size_t>(S) * stage_bytes + S * sizeof(uint64_t) + 2 * 32 * kPipeR * 2 * sizeof(float);
+// rows per iteration of the norm kernels (R; their reductions interleave, one barrier per R rows):
+// MARIO_NORM_FWD_R / MARIO_NORM_BWD_R select 2, 4 or 8
+inline size_t pipe_smem_bytes(int S, int stage_bytes, int R) {
+  return static_cast<size_t>(S) * stage_bytes + S * sizeof(uint64_t) + 2 * 32 * R * 2 * sizeof(float);
+}
+int norm_rows_per_iter(bool fwd) {
+  static const int f = getenv("MARIO_NORM_FWD_R") ? atoi(getenv("MARIO_NORM_FWD_R")) : 2;
+  static const int b = getenv("MARIO_NORM_BWD_R") ? atoi(getenv("MARIO_NORM_BWD_R")) : 2;
+  const int r = fwd ? f : b;
+  return r == 8 ? 8 : (r == 4 ? 4 : 2);
 }
 
 // ------------------------------------------------------------------------- forward
@@ -574,10 +581,9 @@ bool norm_apply(const bf16* x, const float* g, const float* b, const float* stat
 
 bool norm_pipe_supported(int n) { return n % 8 == 0 && n >= 8 && n <= 8192; }
 
-bool norm_fwd_pipe(const bf16* x, const float* g, const float* b, bf16* y, float* stats, int rows, int n, float eps,
-                   int rms, cudaStream_t st) {
-  if (!norm_pipe_supported(n)) return false;
-  if (rows <= 0) return true;
+template <int kPipeR>
+bool norm_fwd_pipe_r(const bf16* x, const float* g, const float* b, bf16* y, float* stats, int rows, int n, float eps,
+                     int rms, cudaStream_t st) {
   const int nt = threads_for(n), sb = n * 2;
   // ring bytes / max stages per CTA (MARIO_NORM_FWD_RING, MARIO_NORM_FWD_SMAX: tuning experiments)
   static const int ring = getenv("MARIO_NORM_FWD_RING") ? atoi(getenv("MARIO_NORM_FWD_RING")) : 24576;
@@ -585,7 +591,7 @@ bool norm_fwd_pipe(const bf16* x, const float* g, const float* b, bf16* y, float
   int S = ring / sb;
   S = S < 2 * kPipeR ? 2 * kPipeR : (S > smax ? smax : S);
   S -= S % kPipeR;
-  const size_t smem = pipe_smem_bytes(S, sb);
+  const size_t smem = pipe_smem_bytes(S, sb, kPipeR);
   static bool attr = false;
   if (!attr) {
     cudaFuncSetAttribute(norm_fwd_pipe_k<false, kPipeR>, cudaFuncAttributeMaxDynamicSharedMemorySize, 200 * 1024);
@@ -600,8 +606,19 @@ bool norm_fwd_pipe(const bf16* x, const float* g, const float* b, bf16* y, float
   return true;
 }
 
-template <int V, int RES, bool OUT32>
-bool norm_bwd_pipe_v(const bf16* dy, const bf16* x, const float* stats, const float* g, const void* dres, bf16* dx,
+bool norm_fwd_pipe(const bf16* x, const float* g, const float* b, bf16* y, float* stats, int rows, int n, float eps,
+                   int rms, cudaStream_t st) {
+  if (!norm_pipe_supported(n)) return false;
+  if (rows <= 0) return true;
+  switch (norm_rows_per_iter(true)) {
+    case 8: return norm_fwd_pipe_r<8>(x, g, b, y, stats, rows, n, eps, rms, st);
+    case 4: return norm_fwd_pipe_r<4>(x, g, b, y, stats, rows, n, eps, rms, st);
+    default: return norm_fwd_pipe_r<2>(x, g, b, y, stats, rows, n, eps, rms, st);
+  }
+}
+
+template <int V, int RES, bool OUT32, int kPipeR>
+bool norm_bwd_pipe_vr(const bf16* dy, const bf16* x, const float* stats, const float* g, const void* dres, bf16* dx,
                      float* dx32, int rows, int n, int rms, float* dg, float* db, float* dsum, float* partial,
                      size_t partial_floats, cudaStream_t st) {
   const int nt = ((n / (8 * V) + 31) / 32) * 32, sb = 4 * n + (RES == 2 ? 4 * n : (RES == 1 ? 2 * n : 0));
@@ -618,7 +635,7 @@ bool norm_bwd_pipe_v(const bf16* dy, const bf16* x, const float* stats, const fl
     attr = true;
   }
   // the stats of a CTA's range are staged in shared memory: size for the smallest grid we may use
-  const size_t base = pipe_smem_bytes(S, sb);
+  const size_t base = pipe_smem_bytes(S, sb, kPipeR);
   int nblk = occ_grid(norm_bwd_pipe_k<kPipeR, V, RES, OUT32>, nt,
                       base + 8 * static_cast<size_t>(cdivl(rows, device_sms())));
   if (dg) {
@@ -638,6 +655,17 @@ bool norm_bwd_pipe_v(const bf16* dy, const bf16* x, const float* stats, const fl
     colsum_reduce(partial, nblk, n, dg, rms ? nullptr : db, dsum, st);
   }
   return true;
+}
+
+template <int V, int RES, bool OUT32>
+bool norm_bwd_pipe_v(const bf16* dy, const bf16* x, const float* stats, const float* g, const void* dres, bf16* dx,
+                     float* dx32, int rows, int n, int rms, float* dg, float* db, float* dsum, float* partial,
+                     size_t partial_floats, cudaStream_t st) {
+  if (norm_rows_per_iter(false) == 4)
+    return norm_bwd_pipe_vr<V, RES, OUT32, 4>(dy, x, stats, g, dres, dx, dx32, rows, n, rms, dg, db, dsum, partial,
+                                              partial_floats, st);
+  return norm_bwd_pipe_vr<V, RES, OUT32, 2>(dy, x, stats, g, dres, dx, dx32, rows, n, rms, dg, db, dsum, partial,
+                                            partial_floats, st);
 }
 
 bool norm_bwd_pipe(const bf16* dy, const bf16* x, const float* stats, const float* g, const bf16* dres, bf16* dx,

@@ -35,6 +35,7 @@ struct mario_plan {
   // parameters
   std::vector<mario::ParamSpec> params;
   std::vector<std::string> param_names;
+  std::map<std::string, int> param_index;   // name -> global index (executor weight lookups)
   struct RankParams {
     std::vector<int32_t> idx;        // global param index per packed tensor
     std::vector<uint64_t> off, cnt;  // element offset / count in the packed buffer
@@ -45,11 +46,15 @@ struct mario_plan {
   // executor pools per device (slot counts) for multi-process and loopback execution
   struct Pools { int ckpt = 0, act = 0, send_act = 0, send_grad = 0, recv_grad = 0; };
   std::vector<Pools> pools_mp, pools_lb;
-  // send slot of every message, per device: (micro, part) -> slot. Assigned once along the
-  // loopback order (a valid execution order of the plan's DAG), holding a slot from its FW/CFW (BW)
-  // until the receiver's RA (RG): every executor reuses a slot only after a message the loopback
-  // order has already consumed, so the slot-reuse waits add no cycle to the DAG.
-  std::vector<std::map<std::pair<int, int>, int>> sa_slot, sg_slot;
+  // send slot of every message, per device: (micro, part) -> slot, held from its FW/CFW (BW) until
+  // the receiver's RA (RG). Assigned once along a valid execution order of the plan's DAG, so an
+  // executor that reuses a slot only after its previous message was consumed adds no cycle:
+  //  - sa_slot / sg_slot (pools_mp): along peer_order, the simulator's timeline (instructions in
+  //    order of their simulated times), used by the per-rank executors (peer transport, NCCL);
+  //  - sa_slot_lb / sg_slot_lb (pools_lb): along loopback_order, used by the loopback executor,
+  //    which copies a message out at the receiver's RA in that order.
+  std::vector<std::map<std::pair<int, int>, int>> sa_slot, sg_slot, sa_slot_lb, sg_slot_lb;
+  std::vector<std::pair<int, int>> peer_order;   // (device, list index) in simulated-time order
   std::vector<uint64_t> workspace_mp, workspace_lb;  // bytes per device
   // global execution order used by loopback (device, list index), round-robin like the simulator
   std::vector<std::pair<int, int>> loopback_order;

@@ -98,13 +98,38 @@ def run(epi, iters=6):
     return {k: (sum(x[0] for x in v) / sum(x[1] for x in v) / 1e9, sum(x[1] for x in v) / len(v)) for k, v in out.items()}
 
 
+def cublas(iters=6):
+    """The same (M, N, K) as plain cuBLAS bf16 GEMMs (torch.mm, bf16 out), for context."""
+    shapes = {"qkv fwd": (T, 3 * h, h), "proj fwd": (T, h, h), "fc1 fwd": (T, f, h), "fc2 fwd": (T, h, f),
+              "fc2 wgrad": (h, f, T), "fc2 dgrad": (T, f, h), "fc1 wgrad": (f, h, T), "fc1 dgrad": (T, h, f),
+              "proj wgrad": (h, h, T), "proj dgrad": (T, h, h), "qkv wgrad": (3 * h, h, T), "qkv dgrad": (T, h, 3 * h),
+              "head fwd": (T, V, h), "head wgrad": (V, h, T), "head dgrad": (T, h, V)}
+    out = {}
+    for name, (M, N, K) in shapes.items():
+        a = [torch.randn(M, K, device=dev).to(bf) for _ in range(NS)]
+        b = [torch.randn(K, N, device=dev).to(bf) for _ in range(NS)]
+        ts = []
+        for it in range(iters):
+            e0, e1 = torch.cuda.Event(True), torch.cuda.Event(True)
+            e0.record()
+            torch.mm(a[it % NS], b[it % NS])
+            e1.record()
+            ts.append((e0, e1))
+        torch.cuda.synchronize()
+        ms = sum(e0.elapsed_time(e1) for e0, e1 in ts[2:]) / (iters - 2)
+        out[name] = 2.0 * M * N * K / ms / 1e9
+        del a, b
+    return out
+
+
 with_epi = run(True)
 no_epi = run(False)
+cub = cublas()
 tot_fl = tot_ms = 0.0
 for name, fl, _ in calls(sets[0]):
     tf, ms = with_epi[name]
     tot_fl += fl
     tot_ms += ms
     print(json.dumps({"gemm": name, "tflops_epi": round(tf, 1), "us_epi": round(ms * 1e3, 1),
-                      "tflops_noepi": round(no_epi[name][0], 1)}))
+                      "tflops_noepi": round(no_epi[name][0], 1), "tflops_cublas": round(cub[name], 1)}))
 print(json.dumps({"layer_total_tflops": round(tot_fl / tot_ms / 1e9, 1), "layer_ms": round(tot_ms, 3)}))
