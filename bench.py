@@ -69,6 +69,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--emulate-only", action="store_true", help="only the emulated-pipeline measurement")
+    ap.add_argument("--emulate-levels", default="base,ckpt,mario",
+                    help="plans the emulated pipeline measures (BASE of cfg3 needs more than one GPU's HBM)")
     ap.add_argument("--emulate", type=int, default=8,
                     help="N=1: also measure an S-stage pipeline of the same workload on this GPU (SM partitions, "
                          "peer transport) at BASE / CKPT / MARIO; 0 disables")
@@ -366,7 +368,7 @@ def main():
     from paper_conf_ppopp_liultj25_b200 import _lib, api
     if args.emulate_only:
         torch.cuda.set_device(0)
-        levels = tuple(os.environ.get("MARIO_EMU_LEVELS", "base,ckpt,mario").split(","))
+        levels = tuple(args.emulate_levels.split(","))
         print(json.dumps({"pipeline_emulated": emulate_pipeline(cfg, api, torch, S=args.emulate, n_micro=args.micro,
                                                                 steps=max(1, min(args.steps, 3)), warmup=2,
                                                                 levels=levels, scheme=args.scheme or CE["scheme"],
@@ -545,6 +547,7 @@ def main():
     if rank == 0 and world == 1 and args.emulate > 1 and args.config != "cfg5":
         out["pipeline_emulated"] = emulate_pipeline(cfg, api, torch, S=args.emulate, n_micro=args.micro,
                                                     scheme=CE["scheme"], chunks=CE["chunks"],
+                                                    levels=tuple(args.emulate_levels.split(",")),
                                                     steps=max(1, min(args.steps, 3)), warmup=2)
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         n_cores = cores()
