@@ -69,6 +69,9 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--emulate-only", action="store_true", help="only the emulated-pipeline measurement")
+    ap.add_argument("--emulate-lmbs", type=int, default=0,
+                    help="also measure the emulated Mario plan with this larger micro-batch at the same global "
+                         "batch (the paper's lmbs configuration, P:286)")
     ap.add_argument("--emulate-levels", default="base,ckpt,mario",
                     help="plans the emulated pipeline measures (BASE of cfg3 needs more than one GPU's HBM)")
     ap.add_argument("--emulate", type=int, default=8,
@@ -369,10 +372,18 @@ def main():
     if args.emulate_only:
         torch.cuda.set_device(0)
         levels = tuple(args.emulate_levels.split(","))
-        print(json.dumps({"pipeline_emulated": emulate_pipeline(cfg, api, torch, S=args.emulate, n_micro=args.micro,
-                                                                steps=max(1, min(args.steps, 3)), warmup=2,
-                                                                levels=levels, scheme=args.scheme or CE["scheme"],
-                                                                chunks=CE["chunks"])}), flush=True)
+        res = {"pipeline_emulated": emulate_pipeline(cfg, api, torch, S=args.emulate, n_micro=args.micro,
+                                                     steps=max(1, min(args.steps, 3)), warmup=2,
+                                                     levels=levels, scheme=args.scheme or CE["scheme"],
+                                                     chunks=CE["chunks"])}
+        if args.emulate_lmbs:
+            lm = args.emulate_lmbs
+            res["pipeline_emulated_lmbs"] = emulate_pipeline(
+                synth.with_(cfg, micro_batch=lm), api, torch, S=args.emulate, n_micro=gbs // lm,
+                steps=max(1, min(args.steps, 3)), warmup=2, levels=("mario",), scheme=args.scheme or CE["scheme"],
+                chunks=CE["chunks"])
+            res["pipeline_emulated_lmbs"]["micro_batch"] = lm
+        print(json.dumps(res), flush=True)
         return
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -544,6 +555,12 @@ def main():
            "execution": "cuda-graph replay" if use_graphs else "eager",
            "e2e": e2e, "eager": eager}
     ctx.close()
+    if rank == 0 and world == 1 and args.emulate > 1 and args.config != "cfg5" and args.emulate_lmbs:
+        lm = args.emulate_lmbs
+        out["pipeline_emulated_lmbs"] = emulate_pipeline(
+            synth.with_(cfg, micro_batch=lm), api, torch, S=args.emulate, n_micro=gbs // lm,
+            steps=max(1, min(args.steps, 3)), warmup=2, levels=("mario",), scheme=CE["scheme"], chunks=CE["chunks"])
+        out["pipeline_emulated_lmbs"]["micro_batch"] = lm
     if rank == 0 and world == 1 and args.emulate > 1 and args.config != "cfg5":
         out["pipeline_emulated"] = emulate_pipeline(cfg, api, torch, S=args.emulate, n_micro=args.micro,
                                                     scheme=CE["scheme"], chunks=CE["chunks"],

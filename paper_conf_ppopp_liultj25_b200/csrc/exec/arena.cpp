@@ -47,6 +47,8 @@ Arena make_arena(const PlanObj& P, int dev, const PlanObj::Pools& pools) {
   a.loss = take(static_cast<size_t>(P.pp.N) * P.pp.parts() * 8 + tokens_per_micro(m) * 4);
   a.red_bytes = static_cast<size_t>(kRedBlocks) * red_width(m) * 4 * 2;
   a.red = take(a.red_bytes);
+  if (m.family == MARIO_LLAMA && m.dtype == MARIO_BF16)
+    a.rope = take(static_cast<size_t>(m.seq_len) * (m.hidden / m.n_heads / 2) * 8);
   a.total = o;
   return a;
 }

@@ -17,6 +17,7 @@ struct Arena {
   size_t cfw = 0, bw = 0, logits = SIZE_MAX;
   size_t sa = 0, sg = 0, rg = 0, msg_stride = 0; int n_sa = 0, n_sg = 0, n_rg = 0;
   size_t tokens = 0, loss = 0, red = 0, red_bytes = 0;
+  size_t rope = SIZE_MAX;         // LLaMA bf16: RoPE (cos, sin) table [s][dh/2], rebuilt each iteration
   size_t total = 0;
 };
 

@@ -213,6 +213,10 @@ struct Exec {
     return D.gr + D.P->rank_params[D.d].off[tidx(D, p, name)];
   }
 
+  const float2* rope_tab(Dev<T>& D) const {
+    return D.a.rope == SIZE_MAX ? nullptr : reinterpret_cast<const float2*>(D.ws + D.a.rope);
+  }
+
   // ---- GEMM dispatch --------------------------------------------------------
   // D[M,N] = A[M,K] . B[N,K]^T  (see kernels.h); bf16 tcgen05 or fp32 SIMT by dtype.
   void gemm(const T* A, int lda, int a_mn, const T* B, int ldb, int b_mn, int M, int N, int K, void* Dp, int ldd,
@@ -310,7 +314,7 @@ struct Exec {
       } else {
         rmsnorm_fwd<T>(Hin, Wf(D, p, pre + "n1.g"), A, st1, Tn, h, m.norm_eps, st);
         lin_fwd(A, Wm(D, p, pre + "qkv.w"), Tn, 3 * h, h, QKV, nullptr);
-        rope<T>(QKV, mbs, s, nh, dh, m.rope_base, 0, st);
+        rope<T>(QKV, mbs, s, nh, dh, m.rope_base, 0, st, rope_tab(D));
       }
       attn_fwd<T>(QKV, O, LSE, mbs, s, nh, dh, st, LT.attn_pad ? trans + LT.attn_pad : nullptr);
       if (gpt) {
@@ -480,7 +484,7 @@ struct Exec {
       }
       attn_bwd<T>(QKV, O, dO, LSE, dQKV, Dsc, mbs, s, nh, dh, st, BS.dS_bytes ? sc + BS.dS : nullptr, BS.dS_bytes,
                   BS.attn_pad ? sc + BS.attn_pad : nullptr);
-      if (!gpt) rope<T>(dQKV, mbs, s, nh, dh, m.rope_base, 1, st);
+      if (!gpt) rope<T>(dQKV, mbs, s, nh, dh, m.rope_base, 1, st, rope_tab(D));
       if (gpt) norm_recompute<T>(Hin, Wf(D, p, pre + "ln1.g"), Wf(D, p, pre + "ln1.b"), A, st1, Tn, h, m.norm_eps, 0, st);
       else norm_recompute<T>(Hin, Wf(D, p, pre + "n1.g"), nullptr, A, st1, Tn, h, m.norm_eps, 1, st);
       lin_wgrad(dQKV, A, Tn, 3 * h, h, G(D, p, pre + "qkv.w"));
@@ -941,6 +945,8 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
       for (size_t j = 0; j < rp.idx.size(); ++j)
         if (D.a.wcopy[j] != SIZE_MAX)
           cast_f32_bf16(D.w + rp.off[j], reinterpret_cast<__nv_bfloat16*>(D.ws + D.a.wcopy[j]), rp.cnt[j], s0);
+    if (D.a.rope != SIZE_MAX)
+      rope_table(reinterpret_cast<float2*>(D.ws + D.a.rope), m.seq_len, m.hidden / m.n_heads, m.rope_base, s0);
   }
 
   // walk the plan

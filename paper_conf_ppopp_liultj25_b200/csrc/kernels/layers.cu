@@ -1080,6 +1080,57 @@ __global__ void rope_k(T* qkv, int B, int s, int nh, int dh, float base, int inv
   }
 }
 
+// RoPE angle table (c, s)[t][j] = (cos, sin)(t * base^(-2j/dh)), the angles in double precision and
+// rounded to fp32 exactly as rope_k computes them per element (so the two paths agree bitwise).
+__global__ void rope_table_k(float2* tab, int s, int dh, float base) {
+  const int half = dh / 2;
+  const long n = static_cast<long>(s) * half;
+  for (long i = blockIdx.x * static_cast<long>(blockDim.x) + threadIdx.x; i < n; i += static_cast<long>(gridDim.x) * blockDim.x) {
+    const int j = static_cast<int>(i % half), t = static_cast<int>(i / half);
+    const double theta = pow(static_cast<double>(base), -2.0 * j / dh);
+    double sn, cs;
+    sincos(t * theta, &sn, &cs);
+    tab[i] = make_float2(static_cast<float>(cs), static_cast<float>(sn));
+  }
+}
+// bf16 RoPE from the table: one CTA per token row (blockIdx.y), thread = (head, 8 consecutive j):
+// q and k halves as 16-byte vectors, no per-element division or double-precision math.
+__global__ void rope_v8_k(__nv_bfloat16* qkv, const float2* __restrict__ tab, int s, int nh, int dh, int inverse) {
+  const int half = dh / 2, h8 = half / 8;
+  const int tid = blockIdx.x * blockDim.x + threadIdx.x;
+  if (tid >= nh * h8) return;
+  const int head = tid / h8, j0 = (tid - head * h8) * 8;
+  const long r = blockIdx.y;
+  const int t = static_cast<int>(r % s);
+  const int h = nh * dh;
+  const float sgn = inverse ? -1.f : 1.f;
+  float c[8], sn[8];
+  const float4* tp = reinterpret_cast<const float4*>(tab + static_cast<long>(t) * half + j0);
+#pragma unroll
+  for (int e = 0; e < 4; ++e) {
+    const float4 v = tp[e];
+    c[2 * e] = v.x; sn[2 * e] = sgn * v.y; c[2 * e + 1] = v.z; sn[2 * e + 1] = sgn * v.w;
+  }
+#pragma unroll
+  for (int part = 0; part < 2; ++part) {   // q, then k
+    __nv_bfloat16* p = qkv + r * 3 * h + part * h + head * dh;
+    uint4 u1 = *reinterpret_cast<const uint4*>(p + j0), u2 = *reinterpret_cast<const uint4*>(p + j0 + half);
+    const __nv_bfloat16* x1 = reinterpret_cast<const __nv_bfloat16*>(&u1);
+    const __nv_bfloat16* x2 = reinterpret_cast<const __nv_bfloat16*>(&u2);
+    uint4 o1, o2;
+    __nv_bfloat16* y1 = reinterpret_cast<__nv_bfloat16*>(&o1);
+    __nv_bfloat16* y2 = reinterpret_cast<__nv_bfloat16*>(&o2);
+#pragma unroll
+    for (int e = 0; e < 8; ++e) {
+      const float a = __bfloat162float(x1[e]), b = __bfloat162float(x2[e]);
+      y1[e] = __float2bfloat16_rn(a * c[e] - b * sn[e]);
+      y2[e] = __float2bfloat16_rn(a * sn[e] + b * c[e]);
+    }
+    *reinterpret_cast<uint4*>(p + j0) = o1;
+    *reinterpret_cast<uint4*>(p + j0 + half) = o2;
+  }
+}
+
 // --------------------------------------------------------------------- SwiGLU
 template <class T>
 __global__ void swiglu_fwd_k(const T* GU, T* M, int rows, int f) {
@@ -1138,12 +1189,15 @@ __global__ void gelu_fwd_v8_k(const uint4* Z, uint4* G, size_t n8) {
   }
 }
 // GU row = [gate (f) | up (f)]; M = silu(gate) * up
+// 2-D grid (x: 16-byte column vectors, y: rows): no per-vector row division
 __global__ void swiglu_fwd_v8_k(const __nv_bfloat16* GU, __nv_bfloat16* M, int rows, int f) {
   const int f8 = f / 8;
-  const long n8 = static_cast<long>(rows) * f8;
-  for (long i = blockIdx.x * static_cast<long>(blockDim.x) + threadIdx.x; i < n8; i += static_cast<long>(gridDim.x) * blockDim.x) {
-    const long r = i / f8;
-    const int j8 = static_cast<int>(i - r * f8) * 8;
+  {
+    const long r = blockIdx.y;
+    const int jv = blockIdx.x * blockDim.x + threadIdx.x;
+    if (jv >= f8 || r >= rows) return;
+    const long i = r * f8 + jv;
+    const int j8 = jv * 8;
     const uint4 ug = *reinterpret_cast<const uint4*>(GU + r * 2 * f + j8);
     const uint4 uu = *reinterpret_cast<const uint4*>(GU + r * 2 * f + f + j8);
     const __nv_bfloat16* hg = reinterpret_cast<const __nv_bfloat16*>(&ug);
@@ -1160,10 +1214,12 @@ __global__ void swiglu_fwd_v8_k(const __nv_bfloat16* GU, __nv_bfloat16* M, int r
 }
 __global__ void swiglu_bwd_v8_k(const __nv_bfloat16* GU, const __nv_bfloat16* dM, __nv_bfloat16* dGU, int rows, int f) {
   const int f8 = f / 8;
-  const long n8 = static_cast<long>(rows) * f8;
-  for (long i = blockIdx.x * static_cast<long>(blockDim.x) + threadIdx.x; i < n8; i += static_cast<long>(gridDim.x) * blockDim.x) {
-    const long r = i / f8;
-    const int j8 = static_cast<int>(i - r * f8) * 8;
+  {
+    const long r = blockIdx.y;
+    const int jv = blockIdx.x * blockDim.x + threadIdx.x;
+    if (jv >= f8 || r >= rows) return;
+    const long i = r * f8 + jv;
+    const int j8 = jv * 8;
     const uint4 ug = *reinterpret_cast<const uint4*>(GU + r * 2 * f + j8);
     const uint4 uu = *reinterpret_cast<const uint4*>(GU + r * 2 * f + f + j8);
     const uint4 ud = *reinterpret_cast<const uint4*>(dM + i * 8);
@@ -1506,9 +1562,26 @@ void attn_bwd(const T* qkv, const T* O, const T* dO, const float* lse, T* dqkv, 
   note_launch();
 }
 
-template <class T>
-void rope(T* qkv, int B, int s, int nh, int dh, float base, int inverse, cudaStream_t st) {
+void rope_table(float2* tab, int s, int dh, float base, cudaStream_t st) {
   KScope ks_(K_ELEMWISE, st);
+  rope_table_k<<<grid_for(static_cast<long>(s) * (dh / 2)), 256, 0, st>>>(tab, s, dh, base);
+  note_launch();
+}
+template <class T>
+void rope(T* qkv, int B, int s, int nh, int dh, float base, int inverse, cudaStream_t st, const float2* tab) {
+  KScope ks_(K_ELEMWISE, st);
+  if constexpr (std::is_same<T, __nv_bfloat16>::value) {
+    const int h8 = dh / 16;
+    if (tab && dh % 16 == 0 && static_cast<long>(B) * s <= 65535 &&
+        (reinterpret_cast<uintptr_t>(qkv) & 15) == 0) {
+      const int nthr = nh * h8, bx = nthr < 256 ? ((nthr + 31) / 32) * 32 : 256;
+      dim3 grid((nthr + bx - 1) / bx, static_cast<unsigned>(static_cast<long>(B) * s));
+      rope_v8_k<<<grid, bx, 0, st>>>(qkv, tab, s, nh, dh, inverse);
+      note_launch();
+      return;
+    }
+  }
+  (void)tab;
   rope_k<T><<<grid_for(static_cast<long>(B) * s * nh * (dh / 2)), 256, 0, st>>>(qkv, B, s, nh, dh, base, inverse);
   note_launch();
 }
@@ -1517,7 +1590,7 @@ void swiglu_fwd(const T* GU, T* M, int rows, int f, cudaStream_t st) {
   KScope ks_(K_ELEMWISE, st);
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
     if (f % 8 == 0) {
-      swiglu_fwd_v8_k<<<grid_for(static_cast<long>(rows) * f / 8), 256, 0, st>>>(GU, M, rows, f);
+      swiglu_fwd_v8_k<<<dim3(cdiv(f / 8, 256), rows), 256, 0, st>>>(GU, M, rows, f);
       note_launch();
       return;
     }
@@ -1530,7 +1603,7 @@ void swiglu_bwd(const T* GU, const T* dM, T* dGU, int rows, int f, cudaStream_t 
   KScope ks_(K_ELEMWISE, st);
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
     if (f % 8 == 0) {
-      swiglu_bwd_v8_k<<<grid_for(static_cast<long>(rows) * f / 8), 256, 0, st>>>(GU, dM, dGU, rows, f);
+      swiglu_bwd_v8_k<<<dim3(cdiv(f / 8, 256), rows), 256, 0, st>>>(GU, dM, dGU, rows, f);
       note_launch();
       return;
     }
@@ -1611,7 +1684,7 @@ void sum_copies_f32(float* dst, const CopySrcs& srcs, size_t n, cudaStream_t st)
   template void attn_fwd<T>(const T*, T*, float*, int, int, int, int, cudaStream_t, void*);                                 \
   template void attn_bwd<T>(const T*, const T*, const T*, const float*, T*, float*, int, int, int, int, cudaStream_t, \
                             void*, size_t, void*);                                                                 \
-  template void rope<T>(T*, int, int, int, int, float, int, cudaStream_t);                                           \
+  template void rope<T>(T*, int, int, int, int, float, int, cudaStream_t, const float2*);                             \
   template void swiglu_fwd<T>(const T*, T*, int, int, cudaStream_t);                                                 \
   template void swiglu_bwd<T>(const T*, const T*, T*, int, int, cudaStream_t);                                       \
   template void softmax_ce<T>(const float*, const int32_t*, int, int, int, int, float, T*, float*, cudaStream_t,    \

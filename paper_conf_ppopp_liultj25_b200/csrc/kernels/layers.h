@@ -77,7 +77,10 @@ template <class T> void attn_bwd(const T* qkv, const T* O, const T* dO, const fl
 size_t flash_attn_bwd_ds_bytes(int dh, int B, int s, int nh);
 
 // RoPE (rotate-half) in place on the q and k parts of QKV; inverse = 1 rotates by -t*theta.
-template <class T> void rope(T* qkv, int B, int s, int nh, int dh, float base, int inverse, cudaStream_t st);
+// tab (optional, bf16 path): the (cos, sin) table rope_table wrote for this (s, dh, base).
+template <class T> void rope(T* qkv, int B, int s, int nh, int dh, float base, int inverse, cudaStream_t st,
+                             const float2* tab = nullptr);
+void rope_table(float2* tab, int s, int dh, float base, cudaStream_t st);   // [s][dh/2] (cos, sin)
 
 // SwiGLU: M = silu(GU[:, :f]) * GU[:, f:];  backward dGU from dM.
 template <class T> void swiglu_fwd(const T* GU, T* M, int rows, int f, cudaStream_t st);
