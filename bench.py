@@ -316,16 +316,7 @@ def emulate_pipeline(cfg, api, torch, S=8, n_micro=32, steps=2, warmup=2, levels
             span = max(max(b) for a, b in tl if b)
             busy = [union_ms(list(zip(a, b))) for a, b in tl]
             # per-virtual-stage costs of this run -> the simulator (P:242 profile, P:244-252 simulate)
-            K = plan.S * (chunks if scheme == "interleave" else 1)
-            fw, bw, rc = ([[] for _ in range(K)] for _ in range(3))
-            for d in range(S):
-                comp = [x for x in plan.instrs(d) if x[0] in ("FW", "CFW", "RC", "BW")]
-                for (op, m_, p_, k, *_r), t0, t1 in zip(comp, *tl[d]):
-                    {"FW": fw, "CFW": fw, "RC": rc, "BW": bw}[op][k].append(t1 - t0)
-            mean = lambda xs: sum(xs) / len(xs) if xs else 0.0
-            costs = {"fw_ms": [mean(x) for x in fw], "bw_ms": [mean(x) for x in bw],
-                     "rc_ms": [mean(x) if x else mean(fw[i]) for i, x in enumerate(rc)],
-                     "p2p_alpha_ms": 0.005, "p2p_GBps": 1500.0}
+            costs = ctx.last_costs(plan)
             sim = api.Plan(cfg, S, n_micro, scheme, level, chunks=chunks, dtype="bf16", costs=costs).simulate()
             alloc = [plan.rank_layout(d)[1] + 8 * plan.rank_layout(d)[0] for d in range(S)]
             peaks = plan.simulate().peak_bytes

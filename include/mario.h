@@ -234,6 +234,11 @@ mario_status mario_set_graphs(int32_t enable);
  * iteration start, CUDA events) when timing was enabled with mario_set_timing(1). */
 mario_status mario_set_timing(int32_t enable);
 mario_status mario_last_timeline(int32_t device, const double** start_ms, const double** finish_ms, int32_t* n);
+/* The paper's profile step: per-virtual-stage mean FW/CFW, BW and RC durations (ms) of the
+ * last timed mario_run_iter of `plan` (timing on), written to three caller arrays of K = stages x
+ * chunks entries -- the mario_costs arrays, so mario_plan can re-plan and simulate with measured costs.
+ * A stage without RC reports its forward time. ESTATE if no timed iteration is recorded. */
+mario_status mario_last_costs(const struct mario_plan* plan, double* fw_ms, double* bw_ms, double* rc_ms);
 /* OS (Table 3): AdamW (reading A27: decoupled weight decay, bias correction; step >= 1)
  * applied in place to n packed fp32 parameters with fp32 moments m, v (device pointers, caller
  * owned, zero-initialised before step 1); grads as returned by mario_run_iter. Asynchronous on

@@ -107,6 +107,8 @@ _lib.register("mario_set_graphs", C.c_int32, [C.c_int32])
 _lib.register("mario_last_timeline", C.c_int32, [C.c_int32, C.POINTER(C.POINTER(C.c_double)),
                                                  C.POINTER(C.POINTER(C.c_double)), C.POINTER(C.c_int32)])
 _lib.register("mario_finalize", C.c_int32, [])
+_lib.register("mario_last_costs", C.c_int32, [_P, C.POINTER(C.c_double), C.POINTER(C.c_double),
+                                              C.POINTER(C.c_double)])
 _lib.register("mario_adamw_step", C.c_int32, [C.c_void_p, C.c_void_p, C.c_void_p, C.c_void_p, C.c_uint64, C.c_float,
                                               C.c_float, C.c_float, C.c_float, C.c_float, C.c_int32, C.c_void_p])
 
@@ -367,6 +369,15 @@ class Context:
         a, b, n = C.POINTER(C.c_double)(), C.POINTER(C.c_double)(), C.c_int32()
         _check(_lib.lib().mario_last_timeline(d, C.byref(a), C.byref(b), C.byref(n)))
         return [a[i] for i in range(n.value)], [b[i] for i in range(n.value)]
+
+    def last_costs(self, plan: Plan, p2p_alpha_ms: float = 0.005, p2p_GBps: float = 1500.0) -> dict:
+        """mario_last_costs: the measured per-virtual-stage costs of the last timed iteration, as the
+        `costs` dict Plan() takes (the paper's profile -> simulate loop)."""
+        K = plan.S * (plan.chunks if plan.scheme == "interleave" else 1)
+        fw, bw, rc = (C.c_double * K)(), (C.c_double * K)(), (C.c_double * K)()
+        _check(_lib.lib().mario_last_costs(plan.handle, fw, bw, rc))
+        return {"fw_ms": list(fw), "bw_ms": list(bw), "rc_ms": list(rc), "p2p_alpha_ms": p2p_alpha_ms,
+                "p2p_GBps": p2p_GBps}
 
     def close(self):
         _lib.lib().mario_finalize()

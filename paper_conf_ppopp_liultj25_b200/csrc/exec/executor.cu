@@ -1411,6 +1411,37 @@ extern "C" mario_status mario_last_timeline(int32_t device, const double** start
   return MARIO_OK;
 }
 
+// The paper's profiled estimators: per-virtual-stage mean durations of FW/CFW, BW and RC
+// in the last timed iteration of `plan` on this rank (every rank's in loopback / emulated mode),
+// in the layout mario_costs expects ([K] arrays). A stage with no RC gets its forward time.
+extern "C" mario_status mario_last_costs(const struct mario_plan* plan, double* fw_ms, double* bw_ms, double* rc_ms) {
+  if (!plan || !fw_ms || !bw_ms || !rc_ms) return set_error(MARIO_EINVAL, "NULL argument");
+  const int K = plan->pp.K();
+  std::vector<double> sum[3];
+  std::vector<int> cnt[3];
+  for (int c = 0; c < 3; ++c) { sum[c].assign(K, 0.0); cnt[c].assign(K, 0); }
+  bool any = false;
+  for (int d = 0; d < plan->pp.S && d < static_cast<int>(g.t_start.size()); ++d) {
+    size_t j = 0;
+    for (const mario_instr& x : plan->instrs[d]) {
+      if (x.op != MARIO_OP_FW && x.op != MARIO_OP_CFW && x.op != MARIO_OP_RC && x.op != MARIO_OP_BW) continue;
+      if (j >= g.t_start[d].size()) break;
+      const int c = (x.op == MARIO_OP_BW) ? 1 : (x.op == MARIO_OP_RC ? 2 : 0);
+      sum[c][x.vstage] += g.t_finish[d][j] - g.t_start[d][j];
+      ++cnt[c][x.vstage];
+      ++j;
+      any = true;
+    }
+  }
+  if (!any) return set_error(MARIO_ESTATE, "no timed iteration of this plan (mario_set_timing(1) first)");
+  for (int k = 0; k < K; ++k) {
+    fw_ms[k] = cnt[0][k] ? sum[0][k] / cnt[0][k] : 0.0;
+    bw_ms[k] = cnt[1][k] ? sum[1][k] / cnt[1][k] : 0.0;
+    rc_ms[k] = cnt[2][k] ? sum[2][k] / cnt[2][k] : fw_ms[k];
+  }
+  return MARIO_OK;
+}
+
 extern "C" mario_status mario_finalize(void) {
   for (auto& kv : g.channels) {
     if (kv.second.comm) ncclCommDestroy(kv.second.comm);

@@ -143,3 +143,24 @@ def test_peer_ranks_run_concurrently():
                 overlap += max(0.0, min(b0, b1) - max(a0, a1))
     busy = sum(b - a for a, b, _ in iv)
     assert overlap > 0.2 * busy, (overlap, busy)
+
+
+def test_profile_then_simulate_matches_measured():
+    """P:242-252 in the library: time an emulated 4-stage iteration, read the per-virtual-stage costs
+    back (mario_last_costs), re-plan with them and compare the simulator's makespan and bubble with
+    the measured per-rank timelines (the emulated pipeline: real concurrency, real p2p)."""
+    cfg = synth.with_(synth.GPT3_1P3B, n_layers=4, micro_batch=1, seq_len=1024, hidden=1024, n_heads=8,
+                      ffn_hidden=4096, vocab=8192)
+    params = synth.make_weights(cfg, parity=False)
+    toks = synth.make_tokens(cfg, 8)
+    with Emu(4, 32) as ctx:
+        plan, _ = run_peer(ctx, cfg, 4, 8, "1f1b", "mario", "bf16", params, toks)
+        ctx.set_timing(True)
+        run_peer(ctx, cfg, 4, 8, "1f1b", "mario", "bf16", params, toks)
+        ctx.set_timing(False)
+        tl = [ctx.last_timeline(d) for d in range(4)]
+        costs = ctx.last_costs(plan)
+    assert all(x > 0 for x in costs["fw_ms"] + costs["bw_ms"])
+    measured = max(max(b) for _, b in tl)
+    sim = api.Plan(cfg, 4, 8, "1f1b", "mario", dtype="bf16", costs=costs).simulate()
+    assert abs(sim.makespan_ms - measured) <= 0.15 * measured, (sim.makespan_ms, measured)
