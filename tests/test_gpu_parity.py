@@ -36,7 +36,8 @@ def check(loss, grads, l_o, g_o, tol, norm="inf", inf_guard=None):
     cases); norm="l2": ||g-o||_2/||o||_2 <= tol plus ||.||_inf-relative <= inf_guard (full-width
     bf16 cases, where bf16 activation storage alone moves the fp32 definition by ~2% in the
     worst element at h = 4096; tools/bf16_storage_error.py, A19)."""
-    assert abs(loss - l_o) <= tol * abs(l_o), (loss, l_o)
+    # the loss is held to north_star's bound as stated (2e-2 bf16 / 1e-4 fp32) in every case
+    assert abs(loss - l_o) <= min(tol, 2e-2) * abs(l_o), (loss, l_o)
     worst_inf, worst_l2 = (None, 0.0), (None, 0.0)
     for k, v in g_o.items():
         d = grads[k].astype(np.float64) - v
