@@ -546,17 +546,25 @@ def main():
            "execution": "cuda-graph replay" if use_graphs else "eager",
            "e2e": e2e, "eager": eager}
     ctx.close()
+    # the extra measurements never cost the headline line: a failure is recorded, not raised
     if rank == 0 and world == 1 and args.emulate > 1 and args.config != "cfg5" and args.emulate_lmbs:
         lm = args.emulate_lmbs
-        out["pipeline_emulated_lmbs"] = emulate_pipeline(
-            synth.with_(cfg, micro_batch=lm), api, torch, S=args.emulate, n_micro=gbs // lm,
-            steps=max(1, min(args.steps, 3)), warmup=2, levels=("mario",), scheme=CE["scheme"], chunks=CE["chunks"])
-        out["pipeline_emulated_lmbs"]["micro_batch"] = lm
+        try:
+            out["pipeline_emulated_lmbs"] = emulate_pipeline(
+                synth.with_(cfg, micro_batch=lm), api, torch, S=args.emulate, n_micro=gbs // lm,
+                steps=max(1, min(args.steps, 3)), warmup=2, levels=("mario",), scheme=CE["scheme"],
+                chunks=CE["chunks"])
+            out["pipeline_emulated_lmbs"]["micro_batch"] = lm
+        except Exception as e:   # noqa: BLE001
+            out["pipeline_emulated_lmbs"] = {"error": repr(e)[:300]}
     if rank == 0 and world == 1 and args.emulate > 1 and args.config != "cfg5":
-        out["pipeline_emulated"] = emulate_pipeline(cfg, api, torch, S=args.emulate, n_micro=args.micro,
-                                                    scheme=CE["scheme"], chunks=CE["chunks"],
-                                                    levels=tuple(args.emulate_levels.split(",")),
-                                                    steps=max(1, min(args.steps, 3)), warmup=2)
+        try:
+            out["pipeline_emulated"] = emulate_pipeline(cfg, api, torch, S=args.emulate, n_micro=args.micro,
+                                                        scheme=CE["scheme"], chunks=CE["chunks"],
+                                                        levels=tuple(args.emulate_levels.split(",")),
+                                                        steps=max(1, min(args.steps, 3)), warmup=2)
+        except Exception as e:   # noqa: BLE001
+            out["pipeline_emulated"] = {"error": repr(e)[:300]}
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         n_cores = cores()
         os.environ.setdefault("OPENBLAS_NUM_THREADS", str(n_cores))

@@ -106,6 +106,8 @@ struct Context {
   bool emulated = false;
   int emu_sms = 0;                              // SMs of each rank's partition (0: unpartitioned)
   std::vector<cudaStream_t> emu_st;             // per rank: compute stream
+  std::vector<cudaStream_t> emu_side;           // per rank: side stream (independent wgrads)
+  cudaStream_t side_st = nullptr;               // loopback / NCCL: side stream of the caller's work
   std::vector<std::array<cudaStream_t, 2>> emu_rx;   // per rank: receive streams (activation, gradient)
   bool emu_green = false;                       // streams live in green contexts
   uint32_t* flags = nullptr;                    // device flag block (reset every iteration)
@@ -120,7 +122,7 @@ struct Context {
   std::vector<void*> ipc_opened;
   uint32_t* ipc_flags_own = nullptr;            // this rank's flag block (rank 0's is the shared one)
   size_t ipc_flag_words = 0;
-  cudaStream_t ipc_st = nullptr, ipc_rx[2] = {nullptr, nullptr};
+  cudaStream_t ipc_st = nullptr, ipc_rx[2] = {nullptr, nullptr}, ipc_side = nullptr;
   const void* bound_ws = nullptr;               // the buffers the imported records describe
   const void* bound_gr = nullptr;
 };
@@ -147,6 +149,7 @@ struct Dev {
   // peer transport: this rank's streams and the consumption flag guarding each send slot's reuse
   cudaStream_t st = nullptr;
   cudaStream_t rx[2] = {nullptr, nullptr};
+  cudaStream_t side = nullptr;   // independent backward GEMMs (MARIO_GEMM_OVERLAP)
   int sms = 0;
   std::vector<const uint32_t*> sa_guard, sg_guard;
   std::vector<std::tuple<int, int, int>> sa_guard_key, sg_guard_key;   // the guarding message
@@ -171,6 +174,7 @@ int acquire(std::vector<bool>& used) {
 template <class T>
 struct Exec {
   cudaStream_t st;
+  int gemm_persistent = 1;   // the next GEMMs' grid mode (see GemmArgs::persistent)
   bool loopback;
   bool peer = false;                           // peer transport (emulated ranks, one per stream set)
   std::vector<std::unique_ptr<Dev<T>>> devs;   // loopback / peer: all ranks; NCCL: one (this rank)
@@ -231,6 +235,7 @@ struct Exec {
       g.ep.residual = resid; g.ep.ld_res = ldd; g.ep.d2_bf16 = D2; g.ep.aux = aux; g.ep.ld_aux = ldd;
       g.ep.d2_from_aux = d2_from_aux ? 1 : 0;
       g.ep.colsum_part = colsum_part;
+      g.persistent = gemm_persistent;
       CU(gemm_bf16(g, st));
     } else {
       GemmF32Args g;
@@ -254,6 +259,38 @@ struct Exec {
   // dW[out,in] += dY^T X (fp32)
   void lin_wgrad(const T* dY, const T* X, int Tn, int out, int in, float* dW) {
     gemm(dY, out, 1, X, in, 1, out, in, Tn, dW, in, true, 1.f);
+  }
+
+  // ---- overlap of independent backward GEMMs (MARIO_GEMM_OVERLAP=1) ------------------------
+  // A wgrad that does not depend on the dgrad next to it runs on the rank's side stream as a
+  // non-persistent grid, launched after the persistent dgrad: its CTA pairs take the SMs the
+  // dgrad's last, partly empty wave frees (256 pair tiles on 74 pairs = 3.46 waves at cfg 2). Tiles
+  // are still computed whole by one pair each, so the results are bitwise unchanged.
+  static bool overlap_on() {
+    static const bool on = getenv("MARIO_GEMM_OVERLAP") && atoi(getenv("MARIO_GEMM_OVERLAP")) != 0;
+    return on;
+  }
+  bool side_open = false;
+  template <class F>
+  void on_side(Dev<T>& D, F&& f) {
+    if (!(sizeof(T) == 2 && overlap_on() && D.side)) { f(); return; }
+    cudaEvent_t e = D.event();
+    CU(cudaEventRecord(e, st));
+    CU(cudaStreamWaitEvent(D.side, e, 0));
+    cudaStream_t keep = st;
+    st = D.side;
+    gemm_persistent = 0;
+    f();
+    gemm_persistent = 1;
+    st = keep;
+    side_open = true;
+  }
+  void join_side(Dev<T>& D) {
+    if (!side_open) return;
+    cudaEvent_t e = D.event();
+    CU(cudaEventRecord(e, D.side));
+    CU(cudaStreamWaitEvent(st, e, 0));
+    side_open = false;
   }
 
   // ---- forward of one virtual stage -------------------------------------------
@@ -454,42 +491,43 @@ struct Exec {
         // fc2.b: fused into the norm backward that wrote dH (this stage), else a column sum here
         if (li == lps - 1 && k != K - 1) colsum<T>(dH, nullptr, nullptr, Tn, h, h, 0, G(D, p, pre + "fc2.b"), nullptr, red, st);
         norm_recompute<T>(H1, Wf(D, p, pre + "ln2.g"), Wf(D, p, pre + "ln2.b"), A2, st2, Tn, h, m.norm_eps, 0, st);
-        lin_wgrad(dZ, A2, Tn, f, h, G(D, p, pre + "fc1.w"));
         if (!fuse_b1) colsum<T>(dZ, nullptr, nullptr, Tn, f, f, 0, G(D, p, pre + "fc1.b"), nullptr, red, st);
         lin_dgrad(dZ, Wm(D, p, pre + "fc1.w"), Tn, f, h, dA);               // dA2
+        on_side(D, [&] { lin_wgrad(dZ, A2, Tn, f, h, G(D, p, pre + "fc1.w")); });
         if constexpr (r32)
           norm_bwd_mixed(dA, H1, st2, Wf(D, p, pre + "ln2.g"), dH32 ? nullptr : dH, dH32, dH1, dH32buf[1], Tn, h, 0,
                          G(D, p, pre + "ln2.g"), G(D, p, pre + "ln2.b"), G(D, p, pre + "proj.b"), red, red_floats, st);
         else
           norm_bwd<T>(dA, H1, st2, Wf(D, p, pre + "ln2.g"), dH, dH1, Tn, h, 0, G(D, p, pre + "ln2.g"),
                       G(D, p, pre + "ln2.b"), G(D, p, pre + "proj.b"), red, red_floats, st);
-        lin_wgrad(dH1, O, Tn, h, h, G(D, p, pre + "proj.w"));
         lin_dgrad(dH1, Wm(D, p, pre + "proj.w"), Tn, h, h, dO);
+        on_side(D, [&] { lin_wgrad(dH1, O, Tn, h, h, G(D, p, pre + "proj.w")); });
       } else {
         swiglu_fwd<T>(Z, Gt, Tn, f, st);                                      // recompute M (into dM)
         lin_wgrad(dH, Gt, Tn, h, f, G(D, p, pre + "down.w"));
         lin_dgrad(dH, Wm(D, p, pre + "down.w"), Tn, h, f, dM);              // overwrites M (consumed)
         swiglu_bwd<T>(Z, dM, dZ, Tn, f, st);
         norm_recompute<T>(H1, Wf(D, p, pre + "n2.g"), nullptr, A2, st2, Tn, h, m.norm_eps, 1, st);
-        lin_wgrad(dZ, A2, Tn, 2 * f, h, G(D, p, pre + "gu.w"));
         lin_dgrad(dZ, Wm(D, p, pre + "gu.w"), Tn, 2 * f, h, dA);
+        on_side(D, [&] { lin_wgrad(dZ, A2, Tn, 2 * f, h, G(D, p, pre + "gu.w")); });
         if constexpr (r32)
           norm_bwd_mixed(dA, H1, st2, Wf(D, p, pre + "n2.g"), dH32 ? nullptr : dH, dH32, dH1, dH32buf[1], Tn, h, 1,
                          G(D, p, pre + "n2.g"), nullptr, nullptr, red, red_floats, st);
         else
           norm_bwd<T>(dA, H1, st2, Wf(D, p, pre + "n2.g"), dH, dH1, Tn, h, 1, G(D, p, pre + "n2.g"), nullptr, nullptr,
                       red, red_floats, st);
-        lin_wgrad(dH1, O, Tn, h, h, G(D, p, pre + "o.w"));
         lin_dgrad(dH1, Wm(D, p, pre + "o.w"), Tn, h, h, dO);
+        on_side(D, [&] { lin_wgrad(dH1, O, Tn, h, h, G(D, p, pre + "o.w")); });
       }
       attn_bwd<T>(QKV, O, dO, LSE, dQKV, Dsc, mbs, s, nh, dh, st, BS.dS_bytes ? sc + BS.dS : nullptr, BS.dS_bytes,
                   BS.attn_pad ? sc + BS.attn_pad : nullptr);
       if (!gpt) rope<T>(dQKV, mbs, s, nh, dh, m.rope_base, 1, st, rope_tab(D));
+      join_side(D);   // the fc1 / MLP-input wgrad read A2 (Arec), which the recompute below overwrites
       if (gpt) norm_recompute<T>(Hin, Wf(D, p, pre + "ln1.g"), Wf(D, p, pre + "ln1.b"), A, st1, Tn, h, m.norm_eps, 0, st);
       else norm_recompute<T>(Hin, Wf(D, p, pre + "n1.g"), nullptr, A, st1, Tn, h, m.norm_eps, 1, st);
-      lin_wgrad(dQKV, A, Tn, 3 * h, h, G(D, p, pre + "qkv.w"));
       if (gpt) colsum<T>(dQKV, nullptr, nullptr, Tn, 3 * h, 3 * h, 0, G(D, p, pre + "qkv.b"), nullptr, red, st);
       lin_dgrad(dQKV, Wm(D, p, pre + "qkv.w"), Tn, 3 * h, h, dA);
+      on_side(D, [&] { lin_wgrad(dQKV, A, Tn, 3 * h, h, G(D, p, pre + "qkv.w")); });
       if constexpr (r32) {
         // the stage input's gradient leaves as a bf16 message (SG): no fp32 copy needed there
         float* out32 = (li == 0 && k > 0) ? nullptr : dH32buf[0];
@@ -507,6 +545,7 @@ struct Exec {
         norm_bwd<T>(dA, Hin, st1, Wf(D, p, pre + "n1.g"), dH1, dHin, Tn, h, 1, G(D, p, pre + "n1.g"), nullptr, nullptr,
                     red, red_floats, st);
       }
+      join_side(D);   // this layer's wgrads read buffers the next layer overwrites
       dH = dHin;
       cur = (cur + 2) % 3;
     }
@@ -840,11 +879,16 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
       D->st = g.emu_st[d];
       D->rx[0] = g.emu_rx[d][0];
       D->rx[1] = g.emu_rx[d][1];
+      D->side = g.emu_side[d];
       D->sms = g.emu_sms;
     } else if (g.ipc && d == E.me) {
       D->st = g.ipc_st;
       D->rx[0] = g.ipc_rx[0];
       D->rx[1] = g.ipc_rx[1];
+      D->side = g.ipc_side;
+    } else {
+      if (!g.side_st) CU(cudaStreamCreateWithFlags(&g.side_st, cudaStreamNonBlocking));
+      D->side = g.side_st;
     }
     D->a = make_arena(P, d, pools);
     D->ws = static_cast<uint8_t*>(workspace) + wsofs;
@@ -1213,23 +1257,25 @@ extern "C" mario_status mario_init_emulated(int32_t world, int32_t device, int32
     g.rank = 0; g.world = 1; g.device = device; g.dp = 1;
     g.emu_st.assign(world, nullptr);
     g.emu_rx.assign(world, {nullptr, nullptr});
+    g.emu_side.assign(world, nullptr);
     g.emu_sms = 0;
     g.emu_green = false;
     if (sms_per_rank > 0) {
       std::vector<std::vector<cudaStream_t>> ps;
       int got = 0;
-      const std::string err = drv::make_partitions(device, world, sms_per_rank, 3, ps, &got);
+      const std::string err = drv::make_partitions(device, world, sms_per_rank, 4, ps, &got);
       if (!err.empty()) {
         drv::destroy_partitions();
         return set_error(MARIO_EINVAL, "SM partitions: " + err);
       }
-      for (int r = 0; r < world; ++r) g.emu_st[r] = ps[r][0], g.emu_rx[r] = {ps[r][1], ps[r][2]};
+      for (int r = 0; r < world; ++r) g.emu_st[r] = ps[r][0], g.emu_rx[r] = {ps[r][1], ps[r][2]}, g.emu_side[r] = ps[r][3];
       g.emu_sms = got;
       g.emu_green = true;
     } else {
       for (int r = 0; r < world; ++r) {
         CU(cudaStreamCreateWithFlags(&g.emu_st[r], cudaStreamNonBlocking));
         for (auto& x : g.emu_rx[r]) CU(cudaStreamCreateWithFlags(&x, cudaStreamNonBlocking));
+        CU(cudaStreamCreateWithFlags(&g.emu_side[r], cudaStreamNonBlocking));
       }
     }
     g.emulated = true;
@@ -1285,6 +1331,7 @@ extern "C" mario_status mario_init_peer(int32_t rank, int32_t world, int32_t dev
     g.ipc_flag_words = kPeerFlagWords;
     CU(cudaStreamCreateWithFlags(&g.ipc_st, cudaStreamNonBlocking));
     for (auto& x : g.ipc_rx) CU(cudaStreamCreateWithFlags(&x, cudaStreamNonBlocking));
+    CU(cudaStreamCreateWithFlags(&g.ipc_side, cudaStreamNonBlocking));
     CU(cudaDeviceSynchronize());
     g.epoch = 0;
     g.ipc = true;
@@ -1460,9 +1507,11 @@ extern "C" mario_status mario_finalize(void) {
     for (size_t r = 0; r < g.emu_st.size(); ++r) {
       cudaStreamDestroy(g.emu_st[r]);
       for (auto x : g.emu_rx[r]) cudaStreamDestroy(x);
+      if (r < g.emu_side.size()) cudaStreamDestroy(g.emu_side[r]);
     }
     g.emu_st.clear();
     g.emu_rx.clear();
+    g.emu_side.clear();
     if (g.emu_green) drv::destroy_partitions();
     g.emu_green = false;
     g.emulated = false;
@@ -1480,7 +1529,9 @@ extern "C" mario_status mario_finalize(void) {
     g.ipc_flags_own = nullptr;
     if (g.ipc_st) cudaStreamDestroy(g.ipc_st);
     for (auto& x : g.ipc_rx) { if (x) cudaStreamDestroy(x); x = nullptr; }
+    if (g.ipc_side) cudaStreamDestroy(g.ipc_side);
     g.ipc_st = nullptr;
+    g.ipc_side = nullptr;
     g.ipc = false;
     g.bound_ws = g.bound_gr = nullptr;
     g.world = 1;

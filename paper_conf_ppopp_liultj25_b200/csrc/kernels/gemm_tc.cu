@@ -915,11 +915,11 @@ cudaError_t launch_pair(const GemmArgs& g, cudaStream_t st, int num_sms) {
     attr_set = true;
   }
   const int tiles = ((g.M + 255) / 256) * ((g.N + BNP - 1) / BNP);
-  int pairs = tiles < num_sms / 2 ? tiles : num_sms / 2;
+  int pairs = (tiles < num_sms / 2 || !g.persistent) ? tiles : num_sms / 2;
   StreamK sk;
   static const int sleep_ns = getenv("MARIO_GEMM_SLEEP") ? atoi(getenv("MARIO_GEMM_SLEEP")) : 0;
   sk.sleep_ns = sleep_ns;
-  if (BNP == 256 && use_streamk(tiles, num_sms / 2, (g.K + BK - 1) / BK)) {
+  if (BNP == 256 && g.persistent && use_streamk(tiles, num_sms / 2, (g.K + BK - 1) / BK)) {
     float* ws = nullptr;
     int* flags = nullptr;
     if (streamk_workspace(num_sms / 2, st, &ws, &flags)) {

@@ -35,6 +35,9 @@ struct GemmArgs {
   int M = 0, N = 0, K = 0;
   GemmEpilogue ep;
   int use_pair = -1;   // -1: auto, 0: never use the CTA-pair kernel, 1: always (if M, N >= 256)
+  // 0: one CTA pair per tile instead of a persistent grid: when an independent GEMM runs on another
+  // stream, its pairs are dispatched as the other kernel's last wave frees SMs (fills the wave tail)
+  int persistent = 1;
 };
 
 cudaError_t gemm_bf16(const GemmArgs& g, cudaStream_t st);   // tcgen05 + TMA + TMEM
