@@ -69,6 +69,12 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--emulate-only", action="store_true", help="only the emulated-pipeline measurement")
+    ap.add_argument("--transport", default="nccl", choices=["nccl", "peer"],
+                    help="N > 1: channel transport between the rank processes (peer: CUDA IPC peer memory, "
+                         "ranks may share a GPU)")
+    ap.add_argument("--levels", default="",
+                    help="N > 1: also time these plans (e.g. base,ckpt,mario) in the same invocation, each with "
+                         "its measured bubble ratio and per-stage memory")
     ap.add_argument("--emulate-lmbs", type=int, default=0,
                     help="also measure the emulated Mario plan with this larger micro-batch at the same global "
                          "batch (the paper's lmbs configuration, P:286)")
@@ -187,6 +193,7 @@ def config_dict(cfg, args, gbs):
             "global_batch": gbs, "seq_len": cfg.seq_len, "micro_batch": cfg.micro_batch,
             "microbatches": args.micro, "stages": args.gpus // args.dp, "scheme": args.scheme, "level": args.level,
             "parallelism": f"pp{args.gpus // args.dp}" + (f"xdp{args.dp}" if args.dp > 1 else ""),
+            "transport": args.transport if args.gpus > 1 else "none (1 stage)",
             "l2": "no flush: every iteration streams >100 GB of weights/activations through HBM (>> 126 MB L2)"}
 
 
@@ -342,6 +349,84 @@ def emulate_pipeline(cfg, api, torch, S=8, n_micro=32, steps=2, warmup=2, levels
     return out
 
 
+def allmax(x, cpu_group, torch, dist):
+    """Max over ranks (gloo process groups reduce host tensors, NCCL device tensors)."""
+    t = torch.tensor([float(x)], device="cpu" if cpu_group else "cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def multi_level(args, cfg, api, torch, dist, S, n_rep, scheme, chunks, rank, world, local, peer, stage, gbs):
+    """N > 1: BASE / CKPT / MARIO (--levels) timed in one invocation on the real multi-process
+    pipeline: per plan the iteration time (CUDA events, max over ranks), the measured bubble ratio
+    1 - sum_d busy_d / (S * t_iter) (busy_d = union of rank d's FW/CFW/RC/BW event intervals, SURVEY
+    §8(d) d3), the simulator's bubble from the ranks' own measured stage costs, and the
+    per-stage memory (static arena = simulated peak)."""
+    out = {}
+    for level in [x for x in args.levels.split(",") if x]:
+        plan = api.Plan(cfg, S, n_rep, scheme, level, chunks=chunks, dtype="bf16")
+        ctx = api.Context.peer(rank, world, local) if peer else api.Context(rank, world, local, dp=args.dp)
+        try:
+            w = init_weights_device(plan, stage, torch)
+            pc, wsb = plan.rank_layout(stage)
+            g = torch.zeros(pc, dtype=torch.float32, device="cuda")
+            ws = torch.empty(wsb, dtype=torch.uint8, device="cuda")
+            if peer:
+                ctx.bind(ws, g)
+            toks = [torch.from_numpy(synth.make_tokens(cfg, n_rep, iteration=i)).cuda() for i in range(2)]
+            stream = torch.cuda.current_stream()
+            for i in range(max(2, args.warmup)):
+                ctx.run_iter(plan, w, toks[i % 2], g, ws, stream)
+            torch.cuda.synchronize()
+            dist.barrier()
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            for i in range(args.steps):
+                ctx.run_iter(plan, w, toks[i % 2], g, ws, stream)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            ms = allmax(e0.elapsed_time(e1) / args.steps, peer, torch, dist)
+            ctx.set_timing(True)
+            dist.barrier()
+            e0.record(stream)
+            ctx.run_iter(plan, w, toks[0], g, ws, stream)
+            e1.record(stream)
+            torch.cuda.synchronize()
+            ctx.set_timing(False)
+            t_it = allmax(e0.elapsed_time(e1), peer, torch, dist)
+            a, b = ctx.last_timeline(stage)
+            busy = union_ms(list(zip(a, b)))
+            c = ctx.last_costs(plan)
+            rows = [None] * world
+            dist.all_gather_object(rows, (stage, busy, c))
+            if rank == 0:
+                K = len(c["fw_ms"])
+                merged = {k: [0.0] * K for k in ("fw_ms", "bw_ms", "rc_ms")}
+                for _st, _b, cc in rows:
+                    for k in merged:
+                        for i, v in enumerate(cc[k]):
+                            merged[k][i] = max(merged[k][i], v)
+                merged.update(p2p_alpha_ms=0.005, p2p_GBps=770.0)
+                sim = api.Plan(cfg, S, n_rep, scheme, level, chunks=chunks, dtype="bf16", costs=merged).simulate()
+                busy_all = [r[1] for r in sorted(rows)]
+                peaks = plan.simulate().peak_bytes
+                out[level] = {"ms_per_iter": ms, "samples_per_s": gbs / (ms / 1e3),
+                              "bubble_measured": 1.0 - sum(busy_all) / (S * t_it),
+                              "bubble_simulated": sim.bubble_ratio, "makespan_simulated_ms": sim.makespan_ms,
+                              "timed_iteration_ms": t_it, "busy_ms_per_stage": [round(x, 2) for x in busy_all],
+                              "peak_gb_per_stage_simulated": [round(x / 1e9, 3) for x in peaks],
+                              "peak_balance_max_over_min": max(peaks) / min(peaks)}
+            del w, g, ws
+        finally:
+            torch.cuda.synchronize()
+            dist.barrier()
+            ctx.close()
+            torch.cuda.empty_cache()
+    if rank == 0 and "ckpt" in out and "mario" in out:
+        out["mario_vs_ckpt"] = out["ckpt"]["ms_per_iter"] / out["mario"]["ms_per_iter"]
+    return out
+
+
 def device_sms(torch):
     return torch.cuda.get_device_properties(torch.cuda.current_device()).multi_processor_count
 
@@ -381,10 +466,16 @@ def main():
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     assert world == args.gpus, f"--gpus {args.gpus} but WORLD_SIZE {world}"
+    peer = world > 1 and args.transport == "peer"
+    if peer:
+        local = local % torch.cuda.device_count()   # ranks may share a GPU (CUDA IPC)
     torch.cuda.set_device(local)
     if world > 1:
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        if peer:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
     L = _lib.lib()
     assert world % args.dp == 0 and args.micro % args.dp == 0, "--dp must divide --gpus and --micro"
     S, rep, n_rep = world // args.dp, rank // (world // args.dp), args.micro // args.dp
@@ -393,11 +484,14 @@ def main():
     chunks = CE["chunks"] if scheme == "interleave" else 1
     args.scheme = scheme
     plan = api.Plan(cfg, S, n_rep, scheme, args.level, chunks=chunks, dtype="bf16")
-    ctx = api.Context(rank, world, local, dp=args.dp)
+    assert not peer or args.dp == 1, "--transport peer runs pure pipeline parallelism"
+    ctx = api.Context.peer(rank, world, local) if peer else api.Context(rank, world, local, dp=args.dp)
     w = init_weights_device(plan, stage, torch)          # replicas of a stage hold identical weights
     pc, ws_bytes = plan.rank_layout(stage)
     grads = torch.zeros(pc, dtype=torch.float32, device="cuda")
     ws = torch.empty(ws_bytes, dtype=torch.uint8, device="cuda")
+    if peer:
+        ctx.bind(ws, grads)
     stream = torch.cuda.current_stream()
     tok_host = [synth.make_tokens(cfg, n_rep, iteration=i * args.dp + rep) for i in range(args.warmup + args.steps)]
     tok_dev = [torch.from_numpy(t).cuda() for t in tok_host]
@@ -445,9 +539,7 @@ def main():
     kst_steps = 1 if use_graphs else args.steps      # graph records hold the latest replay only
     L.mario_kstats_enable(0)
     if world > 1:
-        t = torch.tensor([ms_total], device="cuda")
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        ms_total = float(t.item())
+        ms_total = allmax(ms_total, peer, torch, dist)
     ms_step = ms_total / args.steps
     value = gbs / (ms_step / 1e3)
 
@@ -462,9 +554,7 @@ def main():
         torch.cuda.synchronize()
         dt = (time.perf_counter() - t0) / args.steps
         if world > 1:
-            t = torch.tensor([dt], device="cuda")
-            dist.all_reduce(t, op=dist.ReduceOp.MAX)
-            dt = float(t.item())
+            dt = allmax(dt, peer, torch, dist)
         e2e = {"value": gbs / dt, "unit": UNIT, "h2d_bytes_per_step": int(tok_host[0].nbytes),
                "d2h_bytes_per_step": 4 + 8 * n_rep, "graphs": bool(use_graphs)}
 
@@ -546,6 +636,12 @@ def main():
            "execution": "cuda-graph replay" if use_graphs else "eager",
            "e2e": e2e, "eager": eager}
     ctx.close()
+    if world > 1 and args.levels:
+        del w, grads, ws
+        torch.cuda.empty_cache()
+        lv = multi_level(args, cfg, api, torch, dist, S, n_rep, scheme, chunks, rank, world, local, peer, stage, gbs)
+        if rank == 0:
+            out["levels"] = lv
     # the extra measurements never cost the headline line: a failure is recorded, not raised
     if rank == 0 and world == 1 and args.emulate > 1 and args.config != "cfg5" and args.emulate_lmbs:
         lm = args.emulate_lmbs
