@@ -164,3 +164,19 @@ def test_profile_then_simulate_matches_measured():
     measured = max(max(b) for _, b in tl)
     sim = api.Plan(cfg, 4, 8, "1f1b", "mario", dtype="bf16", costs=costs).simulate()
     assert abs(sim.makespan_ms - measured) <= 0.15 * measured, (sim.makespan_ms, measured)
+
+
+@pytest.mark.slow
+def test_peer_cfg2_width_bitwise_equals_loopback():
+    """Real message sizes and the production kernels on SM partitions: GPT-3 1.3B width (h 2048,
+    s 2048, V 50304), 4 layers over 4 ranks of 32 SMs, N = 8, Mario 1F1B, bf16: bitwise the
+    loopback result (8 MB activation / gradient messages through the peer transport)."""
+    cfg = synth.with_(synth.GPT3_1P3B, n_layers=4, micro_batch=1)
+    params = synth.make_weights(cfg)
+    toks = synth.make_tokens(cfg, 8)
+    ref = run_loopback(cfg, 4, 8, "1f1b", "mario", "bf16", params, toks)
+    with Emu(4, 32) as ctx:
+        _, outs = run_peer(ctx, cfg, 4, 8, "1f1b", "mario", "bf16", params, toks, repeat=2)
+    for loss, g in outs:
+        assert loss == ref[0]
+        assert np.array_equal(g, ref[1])
