@@ -286,6 +286,8 @@ def emulate_pipeline(cfg, api, torch, S=8, n_micro=32, steps=2, warmup=2, levels
     HBM and L2, so absolute times are those of 1/S-th of a B200 per stage, not of S B200s."""
     sms = (device_sms(torch) // S) // 8 * 8
     gbs = n_micro * cfg.micro_batch
+    pk, _ = measured_peaks()
+    peak_sustained = float(pk.get("bf16_tflops_sustained", pk.get("bf16_tflops", 1400.0)))
     out = {"stages": S, "microbatches": n_micro, "scheme": scheme, "sms_per_stage": sms,
            "method": "one process, S ranks on disjoint green-context SM partitions of this GPU, peer transport; "
                      "iteration time = CUDA events around graph-replayed iterations (median); bubble from per-rank "
@@ -327,8 +329,15 @@ def emulate_pipeline(cfg, api, torch, S=8, n_micro=32, steps=2, warmup=2, levels
             sim = api.Plan(cfg, S, n_micro, scheme, level, chunks=chunks, dtype="bf16", costs=costs).simulate()
             alloc = [plan.rank_layout(d)[1] + 8 * plan.rank_layout(d)[0] for d in range(S)]
             peaks = plan.simulate().peak_bytes
+            p_lin = (12 * cfg.hidden ** 2 if cfg.family == "gpt"
+                     else 4 * cfg.hidden ** 2 + 3 * cfg.hidden * cfg.ffn_hidden)
+            mflops = 3.0 * (cfg.n_layers * (2 * cfg.seq_len * p_lin + 4 * cfg.seq_len ** 2 * cfg.hidden)
+                            + 2 * cfg.seq_len * cfg.hidden * cfg.vocab) * gbs
+            tf_stage = mflops / (ms / 1e3) / S / 1e12
             out["levels"][level] = {
                 "ms_per_iter": ms, "samples_per_s": gbs / (ms / 1e3), "loss": loss,
+                "model_tflops_per_stage": tf_stage,
+                "model_tflops_per_stage_frac_of_partition_peak": tf_stage / (peak_sustained * sms / device_sms(torch)),
                 "bubble_measured": 1.0 - sum(busy) / (S * span),
                 "bubble_simulated": sim.bubble_ratio,
                 "makespan_measured_ms": span, "makespan_simulated_ms": sim.makespan_ms,
