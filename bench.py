@@ -620,6 +620,12 @@ def main():
            "whole_step_roofline": {"algorithmic_tflops_per_gpu": alg_tflops,
                                    "frac_of_2250_datasheet": alg_tflops / 2250.0,
                                    "frac_of_measured_sustained": alg_tflops / peak,
+                                   # the peak at the SM clock the run saw (148 SMs x 8192 dense
+                                   # bf16 FLOP/clk x f_SM, NVML median under load)
+                                   "clock_limited_peak_tflops": (device_sms(torch) * 8192 * clk["sm_mhz"] * 1e6 / 1e12
+                                                                 if clk.get("sm_mhz") else None),
+                                   "frac_of_clock_limited_peak": (alg_tflops / (device_sms(torch) * 8192 * clk["sm_mhz"] * 1e6 / 1e12)
+                                                                  if clk.get("sm_mhz") else None),
                                    "flops_per_step": alg_flops,
                                    "note": "causal attention FLOPs (2 s^2 h per layer-sample fwd), no RC at 1 stage"},
            "loss": losses[-1],

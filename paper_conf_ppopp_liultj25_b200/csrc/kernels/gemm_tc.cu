@@ -1023,14 +1023,6 @@ cudaError_t gemm_bf16(const GemmArgs& g0, cudaStream_t st) {
   // CTA-pair tiles (256x256, or 256x128 when it quantizes the last wave better; a 256x128 tile
   // costs ~4% more operand traffic per FLOP) when they fill the machine, else single-CTA tiles.
   const long tiles_pair = static_cast<long>((g.M + 255) / 256) * ((g.N + 255) / 256);
-  // few-wave shapes (cfg 4 at mbs 1: M = 2048 tokens -> 80 pair tiles on 74 pairs, 1.08 waves, 54% of
-  // the pair slots busy): single-CTA 128 x 128 tiles quantize better (320 tiles on 148 SMs: 72%)
-  static const bool small_ok = !getenv("MARIO_GEMM_FEWWAVE") || atoi(getenv("MARIO_GEMM_FEWWAVE")) != 0;
-  if (small_ok && g.use_pair == -1 && g.persistent && tiles_pair >= sms / 4) {
-    const long t128 = static_cast<long>((g.M + BM - 1) / BM) * ((g.N + 127) / 128);
-    const double e_pair = wave_eff(tiles_pair, sms / 2), e_128 = wave_eff(t128, sms);
-    if (e_pair < 0.7 && e_128 > e_pair + 0.15) return launch_major<128>(g, st, sms);
-  }
   if (g.use_pair != 0 && g.M >= 256 && g.N >= 256 && (tiles_pair >= sms / 4 || g.use_pair > 0)) {
     const long t256 = tiles_pair, t128 = static_cast<long>((g.M + 255) / 256) * ((g.N + 127) / 128);
     (void)t256; (void)t128;
