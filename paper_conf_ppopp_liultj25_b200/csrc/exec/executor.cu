@@ -1520,6 +1520,8 @@ extern "C" mario_status mario_finalize(void) {
   if (g.flags) cudaFree(g.flags);
   g.flags = nullptr;
   g.flags_cap = 0;
+  if (g.side_st) cudaStreamDestroy(g.side_st);
+  g.side_st = nullptr;
   if (g.ipc) {
     cudaDeviceSynchronize();
     for (void* p : g.ipc_opened) cudaIpcCloseMemHandle(p);

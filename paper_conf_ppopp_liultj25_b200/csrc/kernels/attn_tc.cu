@@ -1984,8 +1984,10 @@ bool flash_attn_fwd_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int n
                        float qk_scale) {
   if (qk_scale <= 0.f) qk_scale = rsqrtf(static_cast<float>(dh));
   // g_attn_variant: -1 auto (two-Q-tile kernel unless it would launch fewer CTAs than SMs: the
-  // one-Q-tile kernel has twice as many), 2 force the one-Q-tile kernel, 3 force the two-Q-tile one
-  const int sms = device_sm_count();
+  // one-Q-tile kernel has twice as many), 2 force the one-Q-tile kernel, 3 force the two-Q-tile one.
+  // The choice uses the whole GPU's SM count, not the thread's SM budget: the two kernels round
+  // differently, and a stage must compute the same bits on an SM partition as in loopback.
+  const int sms = device_sm_count_full();
   const long ctas2 = static_cast<long>((s + 2 * kF2Q - 1) / (2 * kF2Q)) * B * nh;
   if (g_attn_variant == 2 || (g_attn_variant != 3 && ctas2 < sms)) {
     if (dh == 128) return launch_fwd_tc<128>(qkv, O, lse, B, s, nh, st, qk_scale);
