@@ -19,6 +19,7 @@
 #include <cuda_bf16.h>
 #include <cstdio>
 #include <cstdlib>
+#include <vector>
 
 #include "kernels.h"
 #include "kstats.h"
@@ -696,8 +697,15 @@ __global__ void __launch_bounds__(kThreadsB, 1)
 fa_bwd_dkdv_ts(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_qkv64,
                const __grid_constant__ CUtensorMap tm_do64,
                const __grid_constant__ CUtensorMap tm_dqkv, const float* lse, const float* Dd, bf16* dqkv, int B,
-               int s, int nh, uint8_t* dsimg, int l2hint, float qk_scale) {
+               int s, int nh, uint8_t* dsimg, int l2hint, float qk_scale, long long* trace) {
   const bool bulk_ld = (s % kCols) == 0;
+  if (trace && threadIdx.x == 0 && blockIdx.x < 8192) {   // per-CTA (SM, start ns) for the trace tool
+    uint64_t gt; uint32_t sm;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt));
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
+    trace[512 + 3 * blockIdx.x] = sm;
+    trace[512 + 3 * blockIdx.x + 1] = static_cast<long long>(gt);
+  }
   using SM = Smem<DH>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -782,10 +790,13 @@ fa_bwd_dkdv_ts(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
     constexpr uint32_t id_a = umma_idesc_bf16(128, DH, 0, 1);      // dV, dK: A from TMEM, B MN-major
     mbar_wait(kv_full, 0);
     tc_fence_after();
+    const bool tr = trace && blockIdx.x == 0 && lane == 0;
     auto issue_s = [&](int idx) {
       const int st = idx % kRingTS, buf = idx & 1;
+      if (tr) trace[0 * 64 + idx] = clock64();
       mbar_wait(&q_full[st], (idx / kRingTS) & 1);
       mbar_wait(&s_free[buf], ((idx >> 1) & 1) ^ 1);
+      if (tr) trace[1 * 64 + idx] = clock64();
       tc_fence_after();
       if (elect_one()) {
         const uint32_t k = smem_u32(sK), v = smem_u32(sV), q = smem_u32(sQ(st)), g = smem_u32(sG(st));
@@ -801,7 +812,9 @@ fa_bwd_dkdv_ts(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
     };
     auto issue_acc = [&](int idx) {
       const int st = idx % kRingTS, buf = idx & 1;
+      if (tr) trace[2 * 64 + idx] = clock64();
       mbar_wait(&p_full[buf], (idx >> 1) & 1);
+      if (tr) trace[3 * 64 + idx] = clock64();
       tc_fence_after();
       if (elect_one()) {
         const uint32_t q = smem_u32(sQ(st)), g = smem_u32(sG(st));
@@ -830,8 +843,10 @@ fa_bwd_dkdv_ts(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
     const int key = kt * kRows + row;
     const uint32_t lane_off = static_cast<uint32_t>(quarter * 32) << 16;
     const int tid = threadIdx.x - 64;
-    for (int idx = 0; idx < ntiles; ++idx) {
-      const int buf = idx & 1, i = i0 + idx, st = idx % kRingTS;
+    float lv[32], dv[32];
+    // lse (pre-scaled by log2 e) and D of the tile's 32 queries of this half, from the ring slot
+    auto load_ld = [&](int idx) {
+      const int i = i0 + idx, st = idx % kRingTS;
       float* ld = sLD + st * 2 * kCols;
       if (bulk_ld) {
         mbar_wait(&q_full[st], (idx / kRingTS) & 1);
@@ -843,7 +858,6 @@ fa_bwd_dkdv_ts(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
         }
         named_bar(1, 256);
       }
-      float lv[32], dv[32];
 #pragma unroll
       for (int c = 0; c < 32; c += 4) {
         const float4 a = ld_shared_f4(ld + half * 32 + c);
@@ -851,24 +865,35 @@ fa_bwd_dkdv_ts(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
         lv[c] = a.x * LOG2E; lv[c + 1] = a.y * LOG2E; lv[c + 2] = a.z * LOG2E; lv[c + 3] = a.w * LOG2E;
         dv[c] = d.x; dv[c + 1] = d.y; dv[c + 2] = d.z; dv[c + 3] = d.w;
       }
+    };
+    load_ld(0);
+    for (int idx = 0; idx < ntiles; ++idx) {
+      const int buf = idx & 1, i = i0 + idx;
+      const bool trs = trace && blockIdx.x == 0 && threadIdx.x == 64;
+      if (trs) trace[4 * 64 + idx] = clock64();
       mbar_wait(&s_full[buf], (idx >> 1) & 1);
+      if (trs) trace[5 * 64 + idx] = clock64();
       tc_fence_after();
       uint32_t sr[32], dr[32];
       const uint32_t col = buf * kCols + half * 32 + lane_off;
       tmem_ld_32x32b_x32(tm_S + col, sr);
       tmem_ld_32x32b_x32(tm_dP + col, dr);
       tmem_ld_wait();
+      if (trs) trace[6 * 64 + idx] = clock64();
       uint32_t pk[16], dk[16];
-      const bool edge = i * kCols < kt * kRows + kRows || i * kCols + kCols > s;
+      float pv[32];
+#pragma unroll
+      for (int c = 0; c < 32; ++c) pv[c] = ex2(__uint_as_float(sr[c]) * sl2 - lv[c]);
+      // causal / ragged mask only on the diagonal and last tiles, as one branch-free pass (a
+      // per-element branch inside the loop above cost 16 branch regions on every tile)
+      if (i * kCols < kt * kRows + kRows || i * kCols + kCols > s) {
+        const int lo = key - (i * kCols + half * 32), hi = s - (i * kCols + half * 32);
+#pragma unroll
+        for (int c = 0; c < 32; ++c) pv[c] = (c < lo || c >= hi) ? 0.f : pv[c];
+      }
 #pragma unroll
       for (int c = 0; c < 32; c += 2) {
-        float p0 = ex2(__uint_as_float(sr[c]) * sl2 - lv[c]);
-        float p1 = ex2(__uint_as_float(sr[c + 1]) * sl2 - lv[c + 1]);
-        if (edge) {
-          const int qq = i * kCols + half * 32 + c;
-          if (qq < key || qq >= s) p0 = 0.f;
-          if (qq + 1 < key || qq + 1 >= s) p1 = 0.f;
-        }
+        const float p0 = pv[c], p1 = pv[c + 1];
         const float d0 = p0 * (__uint_as_float(dr[c]) - dv[c]), d1 = p1 * (__uint_as_float(dr[c + 1]) - dv[c + 1]);
         const __nv_bfloat162 pp = __floats2bfloat162_rn(p0, p1), dd = __floats2bfloat162_rn(d0, d1);
         pk[c / 2] = *reinterpret_cast<const uint32_t*>(&pp);
@@ -876,6 +901,14 @@ fa_bwd_dkdv_ts(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
       }
       tmem_st_32x32b_x16(tm_S + col, pk);
       tmem_st_32x32b_x16(tm_dP + col, dk);
+      tmem_st_wait();
+      tc_fence_before();
+      __syncwarp();
+      if (trs) trace[7 * 64 + idx] = clock64();
+      if (lane == 0) mbar_arrive(&p_full[buf]);
+      // the next tile's lse / D before this tile's dS-image stores: behind ~16 KB of global stores
+      // per CTA in the LSU queue, these shared loads delayed the next tile's softmax by 400-800 clk
+      if (idx + 1 < ntiles) load_ld(idx + 1);
       if (dsimg) {
         // dS for fa_bwd_dq_img: key row `key`, queries [64 i + 32 half, + 32) of query block i / 2,
         // written as the 128-byte row (key mod 64) of the MN-major SW128 image of dQ's A operand
@@ -898,10 +931,6 @@ fa_bwd_dkdv_ts(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
           st_global_v8(rowp + (((4 * half + 2 * pp) ^ (r64 & 6)) << 4), v);
         }
       }
-      tmem_st_wait();
-      tc_fence_before();
-      __syncwarp();
-      if (lane == 0) mbar_arrive(&p_full[buf]);
     }
     if (half == 1) goto done_ts;
     mbar_wait(acc_done, 0);
@@ -963,6 +992,11 @@ done_ts:
   tc_fence_before();
   __syncthreads();
   if (warp == 1) tmem_dealloc<512>(tm);
+  if (trace && threadIdx.x == 0 && blockIdx.x < 8192) {
+    uint64_t gt;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt));
+    trace[512 + 3 * blockIdx.x + 2] = static_cast<long long>(gt);
+  }
 }
 
 // ----------------------------------------------------------------- dQ, persistent
@@ -1387,18 +1421,20 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
   {
     static long long* trace = nullptr;
     const bool want_trace = getenv("MARIO_ATTN_TRACE") != nullptr;
-    if (want_trace && !trace) { cudaMalloc(&trace, 8 * 64 * sizeof(long long)); cudaMemset(trace, 0, 8 * 64 * sizeof(long long)); }
+    constexpr size_t kTraceWords = 8 * 64 + 3 * 8192;
+    if (want_trace && !trace) { cudaMalloc(&trace, kTraceWords * sizeof(long long)); cudaMemset(trace, 0, kTraceWords * sizeof(long long)); }
     static const bool ts = getenv("MARIO_ATTN_DKDV_TS") ? atoi(getenv("MARIO_ATTN_DKDV_TS")) != 0 : true;
     if (dsimg && (s % kRows) != 0) dsimg = nullptr;
-    if (!(ts && dbg == 0 && !want_trace)) dsimg = nullptr;
-    if (ts && dbg == 0 && !want_trace) {
+    if (!(ts && dbg == 0)) dsimg = nullptr;
+    if (ts && dbg == 0) {
       static bool tset = false;
       if (!tset) {
         cudaFuncSetAttribute(fa_bwd_dkdv_ts<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_dkdv_ts<DH>());
         tset = true;
       }
       fa_bwd_dkdv_ts<DH><<<grid, kThreadsB, smem_dkdv_ts<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s, nh,
-                                                                        dsimg, attn_l2hint(), qk_scale);
+                                                                        dsimg, attn_l2hint(), qk_scale,
+                                                                        want_trace ? trace : nullptr);
     } else {
       fa_bwd_dkdv_tc<DH><<<grid, kThreadsB, smem_dkdv<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s, nh, dbg,
                                                                      want_trace ? trace : nullptr, qk_scale);
@@ -1408,10 +1444,19 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
       cudaStreamSynchronize(st);
       cudaMemcpy(h, trace, sizeof(h), cudaMemcpyDeviceToHost);
       const long long t0 = h[0];
-      fprintf(stderr, "tile  s_wait  s_issued  acc_wait  acc_go | sm_wait  sm_go  sm_math_done  sm_pfull\n");
+      fprintf(stderr, "tile   s_req    s_go  acc_req  acc_go | sm_req   sm_go   sm_ld  sm_done\n");
       for (int i = 0; i < 32; ++i)
         fprintf(stderr, "%3d %8lld %8lld %8lld %8lld | %8lld %8lld %8lld %8lld\n", i, h[i] - t0, h[64 + i] - t0,
                 h[128 + i] - t0, h[192 + i] - t0, h[256 + i] - t0, h[320 + i] - t0, h[384 + i] - t0, h[448 + i] - t0);
+      const char* dump = getenv("MARIO_ATTN_TRACE_CTAS");   // file for the per-CTA (sm, start, end) records
+      if (dump && grid.x <= 8192) {
+        std::vector<long long> c(3 * grid.x);
+        cudaMemcpy(c.data(), trace + 512, c.size() * sizeof(long long), cudaMemcpyDeviceToHost);
+        if (FILE* f = fopen(dump, "w")) {
+          for (unsigned j = 0; j < grid.x; ++j) fprintf(f, "%u %lld %lld %lld\n", j, c[3 * j], c[3 * j + 1], c[3 * j + 2]);
+          fclose(f);
+        }
+      }
     }
   }
   static const bool pers = getenv("MARIO_ATTN_DQ_PERS") ? atoi(getenv("MARIO_ATTN_DQ_PERS")) != 0 : g_attn_dq_pers != 0;
