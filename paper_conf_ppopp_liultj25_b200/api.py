@@ -445,6 +445,46 @@ def tune(cfg, devices: int, global_batch: int, mem_budget: int = 0, costs: Optio
     return rows, best.value
 
 
+def profile_costs(cfg, mbs_list=(1, 2, 4, 8), ctx: Optional["Context"] = None, dtype: str = "bf16",
+                  p2p_alpha_ms: float = 0.01, p2p_GBps: float = 770.0, dp_efficiency: float = 0.95,
+                  seed: int = 0) -> dict:
+    """The paper's profiling step ("we profile the execution time of each layer ... under
+    different micro-batch sizes") as the measured estimators mario_tune takes (Eq. 1):
+    for every micro-batch size, a 2-layer slice of `cfg` runs as a 2-stage BASE 1F1B plan with 2
+    micro-batches in loopback, timed per instruction (mario_set_timing); stage 0's FW / BW give
+    the per-layer forward / backward time, the last stage's excess over it the embedding + head
+    (+ loss) time. Weights N(0, 0.02) and uniform tokens on the device (the dense model's speed
+    does not depend on their values). Returns the `costs` dict tune() takes."""
+    import torch
+    ctx = ctx or default_context()
+    gen = torch.Generator(device="cuda").manual_seed(seed)
+    out = {"mbs": [], "layer_fw_ms": [], "layer_bw_ms": [], "head_fw_ms": [], "head_bw_ms": [],
+           "p2p_alpha_ms": p2p_alpha_ms, "p2p_GBps": p2p_GBps, "dp_efficiency": dp_efficiency}
+    for mbs in mbs_list:
+        sl = replace(cfg, n_layers=2, micro_batch=mbs)
+        plan = Plan(sl, 2, 2, "1f1b", "base", dtype=dtype)
+        w, g, ws = alloc_for(plan, -1)
+        w.normal_(0.0, 0.02, generator=gen)
+        toks = torch.randint(0, cfg.vocab, (2 * mbs, cfg.seq_len + 1), dtype=torch.int32, device="cuda",
+                             generator=gen)
+        for _ in range(2):   # warm-up (first-call setup, graph capture)
+            ctx.run_iter(plan, w, toks, g, ws)
+        ctx.set_timing(True)
+        try:
+            ctx.run_iter(plan, w, toks, g, ws)
+        finally:
+            ctx.set_timing(False)
+        c = ctx.last_costs(plan)
+        out["mbs"].append(mbs)
+        out["layer_fw_ms"].append(c["fw_ms"][0])
+        out["layer_bw_ms"].append(c["bw_ms"][0])
+        out["head_fw_ms"].append(max(0.0, c["fw_ms"][1] - c["fw_ms"][0]))
+        out["head_bw_ms"].append(max(0.0, c["bw_ms"][1] - c["bw_ms"][0]))
+        del w, g, ws, toks
+        torch.cuda.empty_cache()
+    return out
+
+
 def max_seq_len(cfg, stages: int, microbatches: int, level: str, mem_budget: int, scheme: str = "1f1b",
                 chunks: int = 1, start: int = 1024, step: int = 64, limit: int = 1 << 20) -> int:
     """Sequence-length scaling (§6.5): the largest s = start + i*step

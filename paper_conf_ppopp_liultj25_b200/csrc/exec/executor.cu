@@ -33,6 +33,7 @@
 #include <map>
 #include <set>
 #include <memory>
+#include <mutex>
 #include <stdexcept>
 #include <string>
 #include <tuple>
@@ -129,6 +130,35 @@ struct Context {
 Context g;
 
 // ------------------------------------------------------------- per-device state
+// Ordering events outlive one mario_run_iter call in a per-device cache: a call takes what it
+// needs and hands them back at the end instead of creating and destroying every slot / dependency
+// event per iteration (re-recording an event whose earlier record is still pending is legal; the
+// waits enqueued before already refer to that earlier record).
+std::mutex g_ev_mu;
+std::map<int, std::vector<cudaEvent_t>> g_ev_cache;
+cudaEvent_t ev_get() {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  {
+    std::lock_guard<std::mutex> lk(g_ev_mu);
+    auto& v = g_ev_cache[dev];
+    if (!v.empty()) {
+      cudaEvent_t e = v.back();
+      v.pop_back();
+      return e;
+    }
+  }
+  cudaEvent_t e;
+  CU(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+  return e;
+}
+void ev_put(cudaEvent_t e) {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  std::lock_guard<std::mutex> lk(g_ev_mu);
+  g_ev_cache[dev].push_back(e);
+}
+
 template <class T>
 struct Dev {
   const PlanObj* P = nullptr;
@@ -157,11 +187,7 @@ struct Dev {
   const mario_model& M() const { return P->model; }
   template <class U = uint8_t> U* at(size_t off) const { return reinterpret_cast<U*>(ws + off); }
   cudaEvent_t event() {
-    if (ev_next == ev_pool.size()) {
-      cudaEvent_t e;
-      CU(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
-      ev_pool.push_back(e);
-    }
+    if (ev_next == ev_pool.size()) ev_pool.push_back(ev_get());
     return ev_pool[ev_next++];
   }
 };
@@ -907,7 +933,7 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
     auto mk = [&](std::vector<cudaEvent_t>& v, std::vector<bool>& set, size_t n) {
       v.resize(n);
       set.assign(n, false);
-      for (auto& e : v) CU(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+      for (auto& e : v) e = ev_get();
     };
     mk(D->sa_free, D->sa_free_set, D->sa_used.size());
     mk(D->sg_free, D->sg_free_set, D->sg_used.size());
@@ -1192,7 +1218,7 @@ mario_status run_iter_t(const PlanObj& P, const void* weights, const int32_t* to
   }
   for (auto& Dp : E.devs) {
     for (auto v : {&Dp->sa_free, &Dp->sg_free, &Dp->rg_free, &Dp->ck_free, &Dp->ev_pool})
-      for (auto e : *v) cudaEventDestroy(e);
+      for (auto e : *v) ev_put(e);
   }
   return MARIO_OK;
 }
@@ -1502,6 +1528,17 @@ extern "C" mario_status mario_finalize(void) {
   for (auto& kv : g.graph_cache) cudaGraphExecDestroy(kv.second);
   g.graph_cache.clear();
   g.graph_seen.clear();
+  {
+    std::lock_guard<std::mutex> lk(g_ev_mu);
+    int cur = 0;
+    cudaGetDevice(&cur);
+    for (auto& kv : g_ev_cache) {
+      cudaSetDevice(kv.first);
+      for (auto e : kv.second) cudaEventDestroy(e);
+    }
+    g_ev_cache.clear();
+    cudaSetDevice(cur);
+  }
   if (g.emulated) {
     cudaDeviceSynchronize();
     for (size_t r = 0; r < g.emu_st.size(); ++r) {

@@ -85,6 +85,31 @@ def test_bf16_parity(cfg):
     check(loss, grads, l_o, g_o, 2e-2)
 
 
+UNTIED_GPT = synth.with_(synth.TINY_GPT, tie_embeddings=False)
+
+
+@pytest.mark.parametrize("scheme,S,N,v", [("1f1b", 1, 4, 1), ("1f1b", 4, 4, 1), ("interleave", 2, 4, 2),
+                                          ("chimera", 2, 4, 1)], ids=["s1", "1f1b-s4", "interleave", "chimera"])
+def test_fp32_parity_untied_gpt_head(scheme, S, N, v):
+    """GPT with its own head matrix (tie_embeddings = False, A1 without the tie): the head gradient
+    lands in a separate parameter on the last stage and wte's gradient comes from the embedding
+    backward alone; Chimera holds two replicas of both."""
+    params = synth.make_weights(UNTIED_GPT)
+    assert "head" in params or any(k.startswith("head") for k in params)
+    toks = synth.make_tokens(UNTIED_GPT, N)
+    loss, grads, _ = run_plan(UNTIED_GPT, S, N, scheme, "mario", "f32", params, toks, chunks=v)
+    l_o, g_o = om.step(UNTIED_GPT, params, toks, N, np.float32)
+    check(loss, grads, l_o, g_o, 1e-4)
+
+
+def test_bf16_parity_untied_gpt_head():
+    params = synth.make_weights(UNTIED_GPT)
+    toks = synth.make_tokens(UNTIED_GPT, 4)
+    loss, grads, _ = run_plan(UNTIED_GPT, 2, 4, "1f1b", "mario", "bf16", params, toks)
+    l_o, g_o = om.step(UNTIED_GPT, rounded(params), toks, 4, np.float32)
+    check(loss, grads, l_o, g_o, 2e-2)
+
+
 @pytest.mark.parametrize("dtype", ["f32", "bf16"])
 def test_mario_bitwise_equals_base(dtype):
     """Rescheduling + checkpointing must not change a single bit."""

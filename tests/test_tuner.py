@@ -81,3 +81,19 @@ def test_budget_level_in_grid_never_worse_than_mario():
     assert n > 0
     _, b0 = api.tune(synth.GPT3_1P3B, 8, 128)
     assert all(r["level"] != "mario_budget" for r in api.tune(synth.GPT3_1P3B, 8, 128)[0])
+
+
+@pytest.mark.gpu
+def test_profile_costs_measured_estimators_drive_the_tuner():
+    """P:242 profile step inside the library (api.profile_costs): measured per-layer / head costs per
+    micro-batch size, then mario_tune (Eq. 1) on them. Costs are positive, a micro-batch 4x larger
+    costs more per layer, and the tuner finds a feasible configuration under 40 GB."""
+    cfg = synth.with_(synth.GPT3_1P3B, seq_len=1024)
+    costs = api.profile_costs(cfg, (1, 4))
+    assert costs["mbs"] == [1, 4]
+    for k in ("layer_fw_ms", "layer_bw_ms"):
+        assert all(v > 0 for v in costs[k]), costs
+        assert costs[k][1] > costs[k][0], costs
+    assert all(v >= 0 for v in costs["head_fw_ms"] + costs["head_bw_ms"])
+    rows, best = api.tune(cfg, 8, 64, mem_budget=40 * 10 ** 9, costs=costs)
+    assert best >= 0 and rows[best]["feasible"] and rows[best]["micro_batch"] in (1, 4)

@@ -1,7 +1,7 @@
 """The paper's schedule tuner with MEASURED estimators (§5.3 Eq. 1; profile step P:242):
-per micro-batch size, one profiled loopback iteration of a 2-layer, 2-stage slice of the model gives
-the per-layer forward / backward time and the head's extra time (mario_last_costs); mario_tune then
-grid-searches scheme x PP x DP x mbs x level for the full model on 8 GPUs under a memory budget and
+api.profile_costs times, per micro-batch size, one loopback iteration of a 2-layer, 2-stage slice of
+the model (per-layer forward / backward time and the head's extra time, mario_last_costs); mario_tune
+then grid-searches scheme x PP x DP x mbs x level for the full model on 8 GPUs under a memory budget and
 names the "Auto" configuration.
 
     python tools/tune_measured.py [cfg2|cfg3|cfg4] [budget_GB]
@@ -10,7 +10,6 @@ import json
 import os
 import sys
 
-import torch
 
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import synth  # noqa: E402
@@ -21,29 +20,7 @@ name = sys.argv[1] if len(sys.argv) > 1 else "cfg2"
 budget = int(float(sys.argv[2]) * 1e9) if len(sys.argv) > 2 else 40 * 10 ** 9
 gbs = {"cfg2": 128, "cfg3": 32, "cfg4": 32}[name]
 full = CFG[name]
-ctx = api.default_context()
-mbs_list, lf, lb, hf, hb = [], [], [], [], []
-for mbs in (1, 2, 4, 8):
-    cfg = synth.with_(full, n_layers=2, micro_batch=mbs)
-    plan = api.Plan(cfg, 2, 2, "1f1b", "base", dtype="bf16")
-    w, g, ws = api.alloc_for(plan, -1)
-    w.normal_(0.0, 0.02)
-    toks = synth.make_tokens(cfg, 2)
-    for _ in range(2):
-        ctx.run_iter(plan, w, toks, g, ws)
-    ctx.set_timing(True)
-    ctx.run_iter(plan, w, toks, g, ws)
-    ctx.set_timing(False)
-    c = ctx.last_costs(plan)
-    mbs_list.append(mbs)
-    lf.append(c["fw_ms"][0])
-    lb.append(c["bw_ms"][0])
-    hf.append(max(0.0, c["fw_ms"][1] - c["fw_ms"][0]))
-    hb.append(max(0.0, c["bw_ms"][1] - c["bw_ms"][0]))
-    del w, g, ws
-    torch.cuda.empty_cache()
-costs = {"mbs": mbs_list, "layer_fw_ms": lf, "layer_bw_ms": lb, "head_fw_ms": hf, "head_bw_ms": hb,
-         "p2p_alpha_ms": 0.01, "p2p_GBps": 770.0, "dp_efficiency": 0.95}
+costs = api.profile_costs(full, (1, 2, 4, 8))
 rows, best = api.tune(full, 8, gbs, mem_budget=budget, costs=costs)
 feas = sorted([r for r in rows if r["feasible"]], key=lambda r: -r["samples_per_s"])
 out = {"config": name, "devices": 8, "global_batch": gbs, "mem_budget_GB": budget / 1e9,
