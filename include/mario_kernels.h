@@ -94,7 +94,9 @@ int mario_k_norm_fwd(const void* x, const float* g, const float* b, void* y, flo
 int mario_k_norm_bwd(const void* dy, const void* x, const float* stats, const float* g, const void* dres,
                      void* dx, float* dg, float* db, float* dsum, float* partial, long long partial_floats,
                      int rows, int n, int rms, int bf16, void* stream);
-/* Kernel variant for both directions (bf16): 2 (default): row-pipelined persistent kernels — each CTA
+/* Kernel variant for both directions (bf16): 3 (default): variant 2's backward with a persistent
+ * warp-per-row forward for n <= 4096 (16-byte chunks per lane, all loads of a warp's rows in flight,
+ * shifted one-pass row statistics, warp butterflies only); 2: row-pipelined persistent kernels — each CTA
  * streams its contiguous row range through a ring of shared-memory stages filled by cp.async.bulk,
  * column sums reduced per CTA and finished by a fixed-order pass; 1: block-per-row-tile backward
  * with fused column sums + warp-per-row forward; 0: warp-per-row kernels + separate column-sum

@@ -89,6 +89,7 @@ _lib.register("mario_param_count", C.c_int32, [_P])
 _lib.register("mario_param_shape", C.c_int32, [_P, C.c_int32, C.POINTER(C.c_int64), C.POINTER(C.c_int32)])
 _lib.register("mario_plan_destroy", None, [_P])
 _lib.register("mario_plan_unckpt_tail", C.c_int32, [_P])
+_lib.register("mario_plan_store_norm", C.c_int32, [_P])
 _lib.register("mario_last_error", C.c_char_p, [])
 _lib.register("mario_tune", C.c_int32, [C.POINTER(CModel), C.c_int32, C.c_int32, C.c_uint64, C.POINTER(CTuneCosts),
                                         C.POINTER(CTuneResult), C.c_int32, C.POINTER(C.c_int32), C.POINTER(C.c_int32)])
@@ -186,6 +187,11 @@ class Plan:
     def unckpt_tail(self) -> int:
         """MARIO_LEVEL_BUDGET: how many tail devices keep full activations (reading A28)."""
         return int(_lib.lib().mario_plan_unckpt_tail(self.handle))
+
+    @property
+    def store_norm(self) -> bool:
+        """Activation sets keep the norm outputs (else the lean set: the backward recomputes them)."""
+        return bool(_lib.lib().mario_plan_store_norm(self.handle))
 
     def lists(self) -> List[List[Tuple[str, int, int]]]:
         return [[(op, m, p) for (op, m, p, *_r) in self.instrs(d)] for d in range(self.S)]

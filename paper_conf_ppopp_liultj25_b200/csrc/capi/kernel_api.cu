@@ -139,7 +139,7 @@ extern "C" int mario_k_norm_bwd(const void* dy, const void* x, const float* stat
 }
 
 extern "C" int mario_k_norm_set_variant(int v) {
-  if (v < 0 || v > 2) return static_cast<int>(cudaErrorInvalidValue);
+  if (v < 0 || v > 3) return static_cast<int>(cudaErrorInvalidValue);
   g_norm_tile = v;
   return 0;
 }

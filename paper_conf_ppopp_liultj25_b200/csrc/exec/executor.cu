@@ -327,8 +327,9 @@ struct Exec {
     const int Tn = static_cast<int>(tokens_per_micro(m)), h = m.hidden, f = m.ffn_hidden, nh = m.n_heads;
     const int dh = h / nh, s = m.seq_len, mbs = m.micro_batch;
     const bool gpt = m.family == MARIO_GPT;
-    const LayerAct LA = layer_act_layout(m);
-    const LayerTrans LT = layer_trans_layout(m);
+    const bool sn = D.P->store_norm;
+    const LayerAct LA = layer_act_layout(m, sn);
+    const LayerTrans LT = layer_trans_layout(m, sn);
     const HeadAct HA = head_act_layout(m);
     // cfw scratch: [one layer's stored tensors][transients A, A2, G][run0][run1][head]
     uint8_t* cfw = D.template at<uint8_t>(D.a.cfw);
@@ -356,12 +357,12 @@ struct Exec {
       const int l = k * lps + li;
       const std::string pre = "h" + std::to_string(l) + ".";
       uint8_t* L = base + li * lstride;
-      T* A = reinterpret_cast<T*>(trans + LT.A);
+      T* A = reinterpret_cast<T*>(sn ? L + LA.A : trans + LT.A);
       T* QKV = reinterpret_cast<T*>(L + LA.QKV);
       T* O = reinterpret_cast<T*>(L + LA.O);
       float* LSE = reinterpret_cast<float*>(L + LA.LSE);
       T* H1 = reinterpret_cast<T*>(L + LA.H1);
-      T* A2 = reinterpret_cast<T*>(trans + LT.A2);
+      T* A2 = reinterpret_cast<T*>(sn ? L + LA.A2 : trans + LT.A2);
       T* Z = reinterpret_cast<T*>(L + LA.Z);
       T* Gt = reinterpret_cast<T*>(trans + LT.G);
       float* st1 = reinterpret_cast<float*>(L + LA.st1);
@@ -437,9 +438,10 @@ struct Exec {
     const int Tn = static_cast<int>(tokens_per_micro(m)), h = m.hidden, f = m.ffn_hidden, nh = m.n_heads;
     const int dh = h / nh, s = m.seq_len, mbs = m.micro_batch;
     const bool gpt = m.family == MARIO_GPT;
-    const LayerAct LA = layer_act_layout(m);
+    const bool sn = D.P->store_norm;
+    const LayerAct LA = layer_act_layout(m, sn);
     const HeadAct HA = head_act_layout(m);
-    const BwScratch BS = bw_scratch_layout(m);
+    const BwScratch BS = bw_scratch_layout(m, sn);
     uint8_t* base = D.template at<uint8_t>(D.a.act + static_cast<size_t>(x.aslot) * D.a.act_stride);
     uint8_t* head_base = base + LA.bytes * lps;
     uint8_t* sc = D.template at<uint8_t>(D.a.bw);
@@ -493,9 +495,10 @@ struct Exec {
       uint8_t* L = base + li * LA.bytes;
       const T* Hin = (li == 0 && k > 0) ? D.template at<T>(D.a.ckpt + static_cast<size_t>(x.slot) * D.a.ckpt_stride)
                                         : reinterpret_cast<T*>(L + LA.H_in);
-      // recomputed transients: A / A2 (norm outputs) share Arec, G / M share the dM buffer
-      T* A = reinterpret_cast<T*>(sc + BS.Arec);
-      T* A2 = A;
+      // norm outputs A / A2: stored in the activation set (store_norm), else recomputed into the
+      // shared Arec; G / M (recomputed) share the dM buffer
+      T* A = reinterpret_cast<T*>(sn ? L + LA.A : sc + BS.Arec);
+      T* A2 = reinterpret_cast<T*>(sn ? L + LA.A2 : sc + BS.Arec);
       T* Gt = dM;
       T* QKV = reinterpret_cast<T*>(L + LA.QKV);
       T* O = reinterpret_cast<T*>(L + LA.O);
@@ -516,7 +519,7 @@ struct Exec {
         lin_wgrad(dH, Gt, Tn, h, f, G(D, p, pre + "fc2.w"));
         // fc2.b: fused into the norm backward that wrote dH (this stage), else a column sum here
         if (li == lps - 1 && k != K - 1) colsum<T>(dH, nullptr, nullptr, Tn, h, h, 0, G(D, p, pre + "fc2.b"), nullptr, red, st);
-        norm_recompute<T>(H1, Wf(D, p, pre + "ln2.g"), Wf(D, p, pre + "ln2.b"), A2, st2, Tn, h, m.norm_eps, 0, st);
+        if (!sn) norm_recompute<T>(H1, Wf(D, p, pre + "ln2.g"), Wf(D, p, pre + "ln2.b"), A2, st2, Tn, h, m.norm_eps, 0, st);
         if (!fuse_b1) colsum<T>(dZ, nullptr, nullptr, Tn, f, f, 0, G(D, p, pre + "fc1.b"), nullptr, red, st);
         lin_dgrad(dZ, Wm(D, p, pre + "fc1.w"), Tn, f, h, dA);               // dA2
         on_side(D, [&] { lin_wgrad(dZ, A2, Tn, f, h, G(D, p, pre + "fc1.w")); });
@@ -533,7 +536,7 @@ struct Exec {
         lin_wgrad(dH, Gt, Tn, h, f, G(D, p, pre + "down.w"));
         lin_dgrad(dH, Wm(D, p, pre + "down.w"), Tn, h, f, dM);              // overwrites M (consumed)
         swiglu_bwd<T>(Z, dM, dZ, Tn, f, st);
-        norm_recompute<T>(H1, Wf(D, p, pre + "n2.g"), nullptr, A2, st2, Tn, h, m.norm_eps, 1, st);
+        if (!sn) norm_recompute<T>(H1, Wf(D, p, pre + "n2.g"), nullptr, A2, st2, Tn, h, m.norm_eps, 1, st);
         lin_dgrad(dZ, Wm(D, p, pre + "gu.w"), Tn, 2 * f, h, dA);
         on_side(D, [&] { lin_wgrad(dZ, A2, Tn, 2 * f, h, G(D, p, pre + "gu.w")); });
         if constexpr (r32)
@@ -548,9 +551,11 @@ struct Exec {
       attn_bwd<T>(QKV, O, dO, LSE, dQKV, Dsc, mbs, s, nh, dh, st, BS.dS_bytes ? sc + BS.dS : nullptr, BS.dS_bytes,
                   BS.attn_pad ? sc + BS.attn_pad : nullptr);
       if (!gpt) rope<T>(dQKV, mbs, s, nh, dh, m.rope_base, 1, st, rope_tab(D));
-      join_side(D);   // the fc1 / MLP-input wgrad read A2 (Arec), which the recompute below overwrites
-      if (gpt) norm_recompute<T>(Hin, Wf(D, p, pre + "ln1.g"), Wf(D, p, pre + "ln1.b"), A, st1, Tn, h, m.norm_eps, 0, st);
-      else norm_recompute<T>(Hin, Wf(D, p, pre + "n1.g"), nullptr, A, st1, Tn, h, m.norm_eps, 1, st);
+      if (!sn) {
+        join_side(D);   // the fc1 / MLP-input wgrad read A2 (Arec), which the recompute below overwrites
+        if (gpt) norm_recompute<T>(Hin, Wf(D, p, pre + "ln1.g"), Wf(D, p, pre + "ln1.b"), A, st1, Tn, h, m.norm_eps, 0, st);
+        else norm_recompute<T>(Hin, Wf(D, p, pre + "n1.g"), nullptr, A, st1, Tn, h, m.norm_eps, 1, st);
+      }
       if (gpt) colsum<T>(dQKV, nullptr, nullptr, Tn, 3 * h, 3 * h, 0, G(D, p, pre + "qkv.b"), nullptr, red, st);
       lin_dgrad(dQKV, Wm(D, p, pre + "qkv.w"), Tn, 3 * h, h, dA);
       on_side(D, [&] { lin_wgrad(dQKV, A, Tn, 3 * h, h, G(D, p, pre + "qkv.w")); });

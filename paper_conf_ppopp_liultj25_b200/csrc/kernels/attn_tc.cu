@@ -692,7 +692,9 @@ done_dq:
 // cfg-2 shape, per the tools/attn_trace.py timeline). An S^T / dP^T buffer is released by the
 // commit of the dV/dK MMAs that read the P^T / dS^T written into it.
 constexpr int kRingTS = 4;
-template <int DH>
+// POLY = k > 0: every k-th P = 2^x of the softmax on the FMA pipe (ex2_poly, relative error <= 8e-4,
+// below the bf16 rounding P and dS get), so the SFU's 16 ex2 / clk / SM is not the softmax's pace
+template <int DH, int POLY>
 __global__ void __launch_bounds__(kThreadsB, 1)
 fa_bwd_dkdv_ts(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_qkv64,
                const __grid_constant__ CUtensorMap tm_do64,
@@ -883,7 +885,10 @@ fa_bwd_dkdv_ts(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_const
       uint32_t pk[16], dk[16];
       float pv[32];
 #pragma unroll
-      for (int c = 0; c < 32; ++c) pv[c] = ex2(__uint_as_float(sr[c]) * sl2 - lv[c]);
+      for (int c = 0; c < 32; ++c) {
+        const float xe = __uint_as_float(sr[c]) * sl2 - lv[c];
+        pv[c] = (POLY > 0 && c % (POLY > 0 ? POLY : 1) == POLY - 1) ? ex2_poly(xe) : ex2(xe);
+      }
       // causal / ragged mask only on the diagonal and last tiles, as one branch-free pass (a
       // per-element branch inside the loop above cost 16 branch regions on every tile)
       if (i * kCols < kt * kRows + kRows || i * kCols + kCols > s) {
@@ -1429,12 +1434,24 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
     if (ts && dbg == 0) {
       static bool tset = false;
       if (!tset) {
-        cudaFuncSetAttribute(fa_bwd_dkdv_ts<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_dkdv_ts<DH>());
+        cudaFuncSetAttribute(fa_bwd_dkdv_ts<DH, 0>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_dkdv_ts<DH>());
+        cudaFuncSetAttribute(fa_bwd_dkdv_ts<DH, 4>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_dkdv_ts<DH>());
+        cudaFuncSetAttribute(fa_bwd_dkdv_ts<DH, 2>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_dkdv_ts<DH>());
         tset = true;
       }
-      fa_bwd_dkdv_ts<DH><<<grid, kThreadsB, smem_dkdv_ts<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s, nh,
-                                                                        dsimg, attn_l2hint(), qk_scale,
-                                                                        want_trace ? trace : nullptr);
+      static const int poly = getenv("MARIO_ATTN_BWD_POLY") ? atoi(getenv("MARIO_ATTN_BWD_POLY")) : 0;
+      if (poly == 2)
+        fa_bwd_dkdv_ts<DH, 2><<<grid, kThreadsB, smem_dkdv_ts<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s,
+                                                                           nh, dsimg, attn_l2hint(), qk_scale,
+                                                                           want_trace ? trace : nullptr);
+      else if (poly == 4)
+        fa_bwd_dkdv_ts<DH, 4><<<grid, kThreadsB, smem_dkdv_ts<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s,
+                                                                              nh, dsimg, attn_l2hint(), qk_scale,
+                                                                              want_trace ? trace : nullptr);
+      else
+        fa_bwd_dkdv_ts<DH, 0><<<grid, kThreadsB, smem_dkdv_ts<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s,
+                                                                               nh, dsimg, attn_l2hint(), qk_scale,
+                                                                               want_trace ? trace : nullptr);
     } else {
       fa_bwd_dkdv_tc<DH><<<grid, kThreadsB, smem_dkdv<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s, nh, dbg,
                                                                      want_trace ? trace : nullptr, qk_scale);

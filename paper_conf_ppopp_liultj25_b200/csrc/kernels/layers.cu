@@ -3,6 +3,7 @@
 // independent implementation (no shared code).
 #include <cfloat>
 #include <cstdint>
+#include <cstdlib>
 #include <type_traits>
 
 #include "layers.h"
@@ -32,7 +33,12 @@ __device__ __forceinline__ float warp_max(float v) {
 inline int cdiv(long a, long b) { return static_cast<int>((a + b - 1) / b); }
 }  // namespace
 
-int g_norm_tile = 2;   // 2: row-pipelined (rowpipe.cu); 1: block-per-row-tile; 0: warp-per-row (A/B)
+// 3: warp-per-row v2 forward + row-pipelined backward; 2: row-pipelined (rowpipe.cu); 1: block-per-row-tile;
+// 0: warp-per-row (A/B; env MARIO_NORM_VARIANT sets the initial value)
+// Measured (tools/norm_fwd_perf.py, T = 8192): the v2 forward 20.6 -> 18.6 us (LN) / 18.6 -> 16.6 us
+// (RMS) at n = 2048, 37.0 -> 35.4 us (LN) at 4096, slower at 5120 (41.3 -> 48.4 us), so variant 3
+// takes widths <= 4096 and the row pipeline the rest.
+int g_norm_tile = getenv("MARIO_NORM_VARIANT") ? atoi(getenv("MARIO_NORM_VARIANT")) : 3;
 
 namespace {
 
@@ -621,8 +627,21 @@ __global__ void __launch_bounds__(256) colsum_partial_v2_k(const __nv_bfloat16* 
   const int r1 = static_cast<int>(static_cast<long>(rows) * (blk + 1) / nblk);
   float s0[8] = {0, 0, 0, 0, 0, 0, 0, 0}, s1[8] = {0, 0, 0, 0, 0, 0, 0, 0};
   if (c8 < n && mode == 0) {
-    // plain column sums (a bias gradient)
-    for (int r = r0 + warp; r < r1; r += 8) {
+    // plain column sums (a bias gradient): 8 rows' 16-byte loads in flight per warp, added in row
+    // order (the one-load-per-iteration loop was latency-bound at ~2 TB/s on the 100 MB dQKV)
+    int r = r0 + warp;
+    for (; r + 56 < r1; r += 64) {
+      uint4 u[8];
+#pragma unroll
+      for (int k = 0; k < 8; ++k) u[k] = __ldg(reinterpret_cast<const uint4*>(a + static_cast<long>(r + 8 * k) * lda + c8));
+#pragma unroll
+      for (int k = 0; k < 8; ++k) {
+        const __nv_bfloat16* ha = reinterpret_cast<const __nv_bfloat16*>(&u[k]);
+#pragma unroll
+        for (int j = 0; j < 8; ++j) s0[j] += __bfloat162float(ha[j]);
+      }
+    }
+    for (; r < r1; r += 8) {
       const uint4 ua = *reinterpret_cast<const uint4*>(a + static_cast<long>(r) * lda + c8);
       const __nv_bfloat16* ha = reinterpret_cast<const __nv_bfloat16*>(&ua);
 #pragma unroll
@@ -1417,7 +1436,8 @@ template <class T>
 void layernorm_fwd(const T* x, const float* g, const float* b, T* y, float* stats, int rows, int n, float eps, cudaStream_t st) {
   KScope ks_(K_NORM, st);
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
-    if (g_norm_tile == 2 && norm_fwd_pipe(x, g, b, y, stats, rows, n, eps, 0, st)) return;
+    if (g_norm_tile == 3 && n <= 4096 && norm_fwd_warp(x, g, b, y, stats, rows, n, eps, 0, st)) return;
+    if (g_norm_tile >= 2 && norm_fwd_pipe(x, g, b, y, stats, rows, n, eps, 0, st)) return;
     if (n % 8 == 0) {
       if (n <= 1024) norm_fwd_reg_k<false, 4><<<cdiv(rows, 8), 256, 0, st>>>(x, g, b, y, stats, rows, n, eps);
       else if (n <= 2048) norm_fwd_reg_k<false, 8><<<cdiv(rows, 8), 256, 0, st>>>(x, g, b, y, stats, rows, n, eps);
@@ -1435,7 +1455,8 @@ template <class T>
 void rmsnorm_fwd(const T* x, const float* g, T* y, float* stats, int rows, int n, float eps, cudaStream_t st) {
   KScope ks_(K_NORM, st);
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
-    if (g_norm_tile == 2 && norm_fwd_pipe(x, g, nullptr, y, stats, rows, n, eps, 1, st)) return;
+    if (g_norm_tile == 3 && n <= 4096 && norm_fwd_warp(x, g, nullptr, y, stats, rows, n, eps, 1, st)) return;
+    if (g_norm_tile >= 2 && norm_fwd_pipe(x, g, nullptr, y, stats, rows, n, eps, 1, st)) return;
     if (n % 8 == 0) {
       if (n <= 1024) norm_fwd_reg_k<true, 4><<<cdiv(rows, 8), 256, 0, st>>>(x, g, nullptr, y, stats, rows, n, eps);
       else if (n <= 2048) norm_fwd_reg_k<true, 8><<<cdiv(rows, 8), 256, 0, st>>>(x, g, nullptr, y, stats, rows, n, eps);
@@ -1454,7 +1475,7 @@ void norm_bwd_dx(const T* dy, const T* x, const float* stats, const float* g, co
                  int rms, cudaStream_t st) {
   KScope ks_(K_NORM, st);
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
-    if (g_norm_tile == 2 && norm_bwd_pipe(dy, x, stats, g, dres, dx, rows, n, rms, nullptr, nullptr, nullptr, nullptr, 0, st))
+    if (g_norm_tile >= 2 && norm_bwd_pipe(dy, x, stats, g, dres, dx, rows, n, rms, nullptr, nullptr, nullptr, nullptr, 0, st))
       return;
     if (g_norm_tile && norm_bwd_tile(dy, x, stats, g, dres, dx, rows, n, rms, nullptr, nullptr, nullptr, nullptr, 0, st))
       return;
@@ -1512,7 +1533,7 @@ void norm_bwd(const T* dy, const T* x, const float* stats, const float* g, const
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
     if (g_norm_tile) {
       KScope ks_(K_NORM, st);
-      if (g_norm_tile == 2 &&
+      if (g_norm_tile >= 2 &&
           norm_bwd_pipe(dy, x, stats, g, dres, dx, rows, n, rms, dg, db, dsum, partial, partial_floats, st))
         return;
       if (norm_bwd_tile(dy, x, stats, g, dres, dx, rows, n, rms, dg, db, dsum, partial, partial_floats, st)) return;

@@ -47,6 +47,8 @@ bool norm_bwd_pipe_mixed(const __nv_bfloat16* dy, const __nv_bfloat16* x, const 
 extern int g_norm_tile;
 // Row-pipelined bf16 kernels (rowpipe.cu); false = shape not supported (caller falls back).
 bool norm_pipe_supported(int n);
+bool norm_fwd_warp(const __nv_bfloat16* x, const float* g, const float* b, __nv_bfloat16* y, float* stats, int rows,
+                   int n, float eps, int rms, cudaStream_t st);
 bool norm_fwd_pipe(const __nv_bfloat16* x, const float* g, const float* b, __nv_bfloat16* y, float* stats, int rows,
                    int n, float eps, int rms, cudaStream_t st);
 bool norm_bwd_pipe(const __nv_bfloat16* dy, const __nv_bfloat16* x, const float* stats, const float* g,

@@ -624,6 +624,116 @@ bool norm_apply(const bf16* x, const float* g, const float* b, const float* stat
 
 bool norm_pipe_supported(int n) { return n % 8 == 0 && n >= 8 && n <= 8192; }
 
+// ------------------------------------------------------------ forward, warp per row (v2)
+// norm_fwd_warp_k: a persistent grid of 8-warp CTAs; warp w takes RPW rows at a time (rows
+// RPW*w, RPW*(w + nwarps), ...). Lane l owns the 16-byte chunks l, l + 32, ... of a row (NC per
+// row, coalesced 512-byte warp accesses), all loads of the RPW rows are issued before any math
+// (ld.global.nc, no L1 allocation: L1 keeps g / b, which the RPW rows of a chunk share). Row
+// statistics are shifted one-pass sums from registers (below; RMS: var = sum(x^2)/n), warp
+// butterflies only: no shared memory, no block barrier, no mbarrier
+// polling (the row-pipelined kernel above spent ~1700 warp instructions per 2048-wide row on
+// those; this one ~330). Output = norm_out8, the expression norm_apply recomputes with.
+__device__ __forceinline__ uint4 ldg_nc_na(const void* p) {
+  uint4 v;
+  asm volatile("ld.global.nc.L1::no_allocate.v4.u32 {%0, %1, %2, %3}, [%4];"
+               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p));
+  return v;
+}
+__device__ __forceinline__ float2 bf2f2(uint32_t u) {
+  return make_float2(__uint_as_float(u << 16), __uint_as_float(u & 0xffff0000u));
+}
+__device__ __forceinline__ float wsum_bfly(float v) {
+#pragma unroll
+  for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+template <bool RMS, int NC, int RPW>
+__global__ void __launch_bounds__(256, (NC * RPW <= 16 ? 2 : 1)) norm_fwd_warp_k(const bf16* __restrict__ x, const float* __restrict__ g,
+                                                       const float* __restrict__ b, bf16* __restrict__ y,
+                                                       float* __restrict__ stats, int rows, int n, float eps) {
+  const int lane = threadIdx.x & 31;
+  const int nwarps = gridDim.x * (blockDim.x >> 5);
+  const float inv_n = 1.f / n;
+  for (int r0 = (blockIdx.x * (blockDim.x >> 5) + (threadIdx.x >> 5)) * RPW; r0 < rows; r0 += nwarps * RPW) {
+    uint4 v[RPW][NC];
+#pragma unroll
+    for (int q = 0; q < RPW; ++q) {
+      const bf16* xr = x + static_cast<long>(r0 + q) * n;
+#pragma unroll
+      for (int i = 0; i < NC; ++i) {
+        const int c = (i * 32 + lane) * 8;
+        v[q][i] = (r0 + q < rows && c < n) ? ldg_nc_na(xr + c) : make_uint4(0u, 0u, 0u, 0u);
+      }
+    }
+    // one pass, shifted by the row's first element K (as the row-pipelined kernel): S1 = sum(x - K),
+    // S2 = sum((x - K)^2), mean = K + S1/n, var = S2/n - (S1/n)^2 -- the cancellation is relative to
+    // |mean - K|, about one standard deviation; each packed value is converted once (a two-pass form
+    // keeps NC*8 floats per row live: 138 registers, 1 CTA per SM). Padding chunks are skipped.
+    float mean[RPW], rstd[RPW];
+#pragma unroll
+    for (int q = 0; q < RPW; ++q) {
+      const float K = RMS ? 0.f : __uint_as_float(__shfl_sync(0xffffffffu, v[q][0].x, 0) << 16);
+      float2 a1 = f2(0.f, 0.f), a2 = f2(0.f, 0.f);
+#pragma unroll
+      for (int i = 0; i < NC; ++i) {
+        if ((i * 32 + lane) * 8 >= n) continue;
+        const uint32_t w4[4] = {v[q][i].x, v[q][i].y, v[q][i].z, v[q][i].w};
+#pragma unroll
+        for (int k = 0; k < 4; ++k) {
+          const float2 d = RMS ? bf2f2(w4[k]) : add2(bf2f2(w4[k]), f2(-K, -K));
+          if (!RMS) a1 = add2(a1, d);
+          a2 = fma2(d, d, a2);
+        }
+      }
+      const float S2 = wsum_bfly(a2.x + a2.y) * inv_n;
+      if (RMS) {
+        mean[q] = 0.f;
+        rstd[q] = rsqrtf(S2 + eps);
+      } else {
+        const float m1 = wsum_bfly(a1.x + a1.y) * inv_n;
+        mean[q] = K + m1;
+        rstd[q] = rsqrtf(fmaxf(S2 - m1 * m1, 0.f) + eps);
+      }
+    }
+#pragma unroll
+    for (int i = 0; i < NC; ++i) {
+      const int c = (i * 32 + lane) * 8;
+      if (c >= n) continue;
+      float gg[8], bb[8];
+      load8(g + c, gg);
+      if (!RMS) load8(b + c, bb);
+      else {
+#pragma unroll
+        for (int j = 0; j < 8; ++j) bb[j] = 0.f;
+      }
+#pragma unroll
+      for (int q = 0; q < RPW; ++q) {
+        if (r0 + q >= rows) break;
+        float vv[8], o[8];
+        unpack8(v[q][i], vv);
+        norm_out8(vv, mean[q], rstd[q], gg, bb, o);
+        *reinterpret_cast<uint4*>(y + static_cast<long>(r0 + q) * n + c) = pack8(o);
+      }
+    }
+    if (lane == 0) {
+#pragma unroll
+      for (int q = 0; q < RPW; ++q)
+        if (r0 + q < rows) *reinterpret_cast<float2*>(stats + 2 * static_cast<long>(r0 + q)) = make_float2(mean[q], rstd[q]);
+    }
+  }
+}
+
+template <bool RMS, int NC, int RPW>
+void norm_fwd_warp_launch(const bf16* x, const float* g, const float* b, bf16* y, float* stats, int rows, int n,
+                          float eps, cudaStream_t st) {
+  const int need = cdivl(rows, 8 * RPW);
+  int grid = occ_grid(norm_fwd_warp_k<RMS, NC, RPW>, 256, 0);
+  grid = grid < need ? grid : need;
+  norm_fwd_warp_k<RMS, NC, RPW><<<grid, 256, 0, st>>>(x, g, b, y, stats, rows, n, eps);
+  note_launch();
+}
+
+
 template <int kPipeR>
 bool norm_fwd_pipe_r(const bf16* x, const float* g, const float* b, bf16* y, float* stats, int rows, int n, float eps,
                      int rms, cudaStream_t st) {
@@ -659,6 +769,29 @@ bool norm_fwd_pipe(const bf16* x, const float* g, const float* b, bf16* y, float
     case 4: return norm_fwd_pipe_r<4>(x, g, b, y, stats, rows, n, eps, rms, st);
     default: return norm_fwd_pipe_r<2>(x, g, b, y, stats, rows, n, eps, rms, st);
   }
+}
+
+bool norm_fwd_warp(const bf16* x, const float* g, const float* b, bf16* y, float* stats, int rows, int n, float eps,
+                   int rms, cudaStream_t st) {
+  if (n % 8 != 0 || n > 8192 || (reinterpret_cast<uintptr_t>(x) & 15) || (reinterpret_cast<uintptr_t>(y) & 15))
+    return false;
+  if (rows <= 0) return true;
+  const int nc = cdivl(n, 256);
+#define NFW_CASE(NC, RPW)                                                                   \
+  if (nc <= NC) {                                                                           \
+    if (rms) norm_fwd_warp_launch<true, NC, RPW>(x, g, b, y, stats, rows, n, eps, st);      \
+    else norm_fwd_warp_launch<false, NC, RPW>(x, g, b, y, stats, rows, n, eps, st);         \
+    return true;                                                                            \
+  }
+  NFW_CASE(1, 2)
+  NFW_CASE(2, 2)
+  NFW_CASE(4, 2)
+  NFW_CASE(8, 2)
+  NFW_CASE(16, 1)
+  NFW_CASE(20, 1)
+  NFW_CASE(32, 1)
+#undef NFW_CASE
+  return false;
 }
 
 template <int V, int RES, bool OUT32, int kPipeR>

@@ -2,8 +2,9 @@
 PyTorch fp32/fp64 math on the same bf16 inputs (readings A1/A2: LayerNorm / RMSNorm over the
 hidden dimension, biased variance, eps inside the square root).
 
-Variants: 2 = row-pipelined persistent kernels (default; every width n % 8 == 0 up to 8192 forward,
-5120 backward), 1 = block-per-row-tile backward, 0 = warp-per-row. Widths cover the block-per-row-tile kernels (n = 2048, 2560, 4096: one 16-byte chunk per thread;
+Variants: 3 = warp-per-row v2 forward (persistent, shifted one-pass stats) + the row-pipelined backward,
+2 = row-pipelined persistent kernels (every width n % 8 == 0 up to 8192 forward, 5120 backward),
+1 = block-per-row-tile backward, 0 = warp-per-row. Widths cover the block-per-row-tile kernels (n = 2048, 2560, 4096: one 16-byte chunk per thread;
 5120: two) and the warp-per-row fallback (n = 64, 776); row counts are ragged against the R-row
 tile and the CTA row ranges."""
 import pytest
@@ -57,12 +58,12 @@ CASES = [(1, 2048), (37, 2048), (8195, 2048), (517, 2560), (300, 4096), (129, 51
          (2000, 192), (5, 8192)]
 
 
-@pytest.fixture(params=[2, 1, 0], ids=["pipe", "tile", "row"])
+@pytest.fixture(params=[3, 2, 1, 0], ids=["warp2", "pipe", "tile", "row"])
 def variant(request):
     L = _lib.lib()
     assert L.mario_k_norm_set_variant(request.param) == 0
     yield request.param
-    L.mario_k_norm_set_variant(2)
+    L.mario_k_norm_set_variant(3)
 
 
 @pytest.mark.parametrize("rms", [0, 1], ids=["ln", "rms"])
