@@ -51,5 +51,7 @@ for (B, s, nh, dh) in [(4, 2048, 16, 128), (1, 4096, 32, 128), (2, 2048, 32, 128
         for j, t in enumerate((q, k, v)):
             got = dq[:s, j * h + hd * dh: j * h + (hd + 1) * dh].double()
             errs.append(float((got - t.grad).abs().max() / t.grad.abs().max()))
+    if os.environ.get("ATTN_AB_SAVE"):
+        torch.save(dq.cpu(), f"{os.environ['ATTN_AB_SAVE']}_{B}_{s}_{nh}.pt")
     print(json.dumps({"shape": [B, s, nh, dh], "env": tag, "bwd_us": round(ms * 1e3, 1),
                       "tflops": round(fl / ms / 1e9, 1), "max_rel_err_dq_dk_dv": round(max(errs), 5)}), flush=True)
