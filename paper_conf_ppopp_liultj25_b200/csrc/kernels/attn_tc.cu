@@ -1399,7 +1399,12 @@ fa_bwd_dq_img(const __grid_constant__ CUtensorMap tm_qkv64, const uint8_t* __res
 // in issue order, so S(i + 1) cannot overwrite the P^T(i) columns before dV(i) has read them (the
 // same reliance as MARIO_ATTN_BWD_INORDER of fa_bwd_dkdv_ts, measured bitwise equal). The softmax
 // (8 warps: TMEM lane quarter = warp & 3, query half = 64 columns) computes P(i) while dP(i) runs and
-// dS(i) while dV(i) runs. Same arithmetic in the same order as fa_bwd_dkdv_ts: dQKV bitwise equal
+// dS(i) while dV(i) runs. One CTA per item: a persistent form (snake item order, which balances the
+// causal item weights like dynamic dispatch; next item's S/dP MMAs overlapping the dV/dK epilogue) is
+// bitwise equal but measured slower, 256.6 -> 260.8 us, because its epilogue must store dV/dK from
+// registers (ring slot 0, the TMA-store staging here, is then in use): 16-byte stores across 32 rows
+// per warp instruction cost 13 us over the TMA store (profiles/r02/attn_bwd_pers_ab.jsonl).
+// Same arithmetic in the same order as fa_bwd_dkdv_ts: dQKV bitwise equal
 // (tools/ab_n128.sh); attention backward 267.4 -> 256.6 us at the cfg-2 shape, 433.8 -> 417.7 us at
 // B 1, s 4096, 32 heads. Polynomial exponentials for a share of P (as the forward) measured neutral or
 // slower here, so the SFU is not this kernel's pace. Writes the same dS image as fa_bwd_dkdv_ts (one
@@ -1411,20 +1416,11 @@ struct SmemN {
   static constexpr int kLD = 2 * kRows * 4;                    // lse, D of a 128-query tile
   static constexpr int kBytes = 2 * kTile + kRingN * 2 * kTile + kRingN * kLD + 256 + 1024;
 };
-// Persistent form: with a grid smaller than the B*nh*(s/128) work items, CTA c takes items in snake
-// order (round r: item r*G + c, or r*G + G-1-c on odd rounds, items heaviest first), which balances the
-// causal item weights like the hardware's dynamic dispatch (round-robin did not: the persistent
-// 64-query attempt lost 282 -> 291 us to it). Across items the barrier phases run on (global tile
-// counter g, item counter n); item n+1's K/V load waits for acc_done(n) (every MMA of n complete),
-// its S/dP MMAs overlap the dV/dK epilogue of n (direct 16-byte stores from the TMEM rows), and its
-// first dV MMA waits for acc_free(n) (the epilogue has read dV/dK out of TMEM). A grid of one CTA per
-// item runs the same code with one round. Each item's arithmetic does not depend on its CTA, so the
-// two forms give bitwise the same dQKV.
 template <int DH>
 __global__ void __launch_bounds__(kThreadsB, 1)
 fa_bwd_dkdv_n128(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_do128,
-                 const float* lse, const float* Dd, bf16* dqkv, int B, int s, int nh, uint8_t* dsimg,
-                 float qk_scale) {
+                 const __grid_constant__ CUtensorMap tm_dqkv, const float* lse, const float* Dd, bf16* dqkv, int B,
+                 int s, int nh, uint8_t* dsimg, float qk_scale) {
   using SN = SmemN<DH>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -1441,19 +1437,17 @@ fa_bwd_dkdv_n128(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_con
   uint64_t* dp_full = s_full + 1;          // 1  dP^T(i) in TMEM
   uint64_t* p_full = dp_full + 1;          // 1  P^T(i) packed (8 softmax warps)
   uint64_t* ds_full = p_full + 1;          // 1  dS^T(i) packed (8 softmax warps)
-  uint64_t* acc_done = ds_full + 1;        // 1  every MMA of the item complete
-  uint64_t* acc_free = acc_done + 1;       // 1  dV / dK read out of TMEM (8 softmax warps)
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_free + 1);
+  uint64_t* acc_done = ds_full + 1;        // 1
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_done + 1);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const int BH = B * nh;
+  const int kt = blockIdx.x / BH, bh = blockIdx.x % BH, b = bh / nh, head = bh % nh;   // heaviest first
   const int h = nh * DH;
   const long Ttok = static_cast<long>(B) * s;
   const int nq = s / kRows;
-  const int W = nq * BH, G = gridDim.x, c = blockIdx.x;
+  const int ntiles = nq - kt;              // query tiles kt .. nq - 1 (tile kt is the diagonal)
   const float sl2 = qk_scale * LOG2E;
-  // item of round r for this CTA (-1 past the end); item w: key block w / BH (heaviest first), (b, head)
-  auto item_of = [&](int r) { const int w = r * G + ((r & 1) ? G - 1 - c : c); return w < W ? w : -1; };
 
   if (warp == 0 && lane == 0) {
     tma_prefetch_desc(&tm_qkv128);
@@ -1461,7 +1455,6 @@ fa_bwd_dkdv_n128(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_con
     mbar_init(kv_full, 1);
     for (int i = 0; i < kRingN; ++i) { mbar_init(&q_full[i], 1); mbar_init(&q_empty[i], 1); }
     mbar_init(s_full, 1); mbar_init(dp_full, 1); mbar_init(p_full, 8); mbar_init(ds_full, 8); mbar_init(acc_done, 1);
-    mbar_init(acc_free, 8);
     fence_barrier_init();
   }
   if (warp == 1) tmem_alloc<512>(tmem_slot);
@@ -1473,222 +1466,202 @@ fa_bwd_dkdv_n128(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_con
 
   if (warp == 0) {
     if (elect_one()) {
-      int g = 0;
-      for (int n = 0;; ++n) {
-        const int w = item_of(n);
-        if (w < 0) break;
-        const int kt = w / BH, bh = w % BH, b = bh / nh, head = bh % nh, ntiles = nq - kt;
-        const int row0 = b * s;
-        if (n > 0) mbar_wait(acc_done, (n - 1) & 1);   // the previous item's MMAs are done with K / V
-        mbar_arrive_expect_tx(kv_full, 2 * SN::kTile);
+      const int row0 = b * s;
+      mbar_arrive_expect_tx(kv_full, 2 * SN::kTile);
+#pragma unroll
+      for (int a = 0; a < DH / 64; ++a) {
+        tma_load_2d(sK + a * (kRows * 128), &tm_qkv128, kv_full, h + head * DH + a * 64, row0 + kt * kRows);
+        tma_load_2d(sV + a * (kRows * 128), &tm_qkv128, kv_full, 2 * h + head * DH + a * 64, row0 + kt * kRows);
+      }
+      for (int idx = 0; idx < ntiles; ++idx) {
+        const int st = idx % kRingN;
+        mbar_wait(&q_empty[st], ((idx / kRingN) & 1) ^ 1);
+        mbar_arrive_expect_tx(&q_full[st], 2 * SN::kTile + SN::kLD);
+        const int qr = row0 + (kt + idx) * kRows;
 #pragma unroll
         for (int a = 0; a < DH / 64; ++a) {
-          tma_load_2d(sK + a * (kRows * 128), &tm_qkv128, kv_full, h + head * DH + a * 64, row0 + kt * kRows);
-          tma_load_2d(sV + a * (kRows * 128), &tm_qkv128, kv_full, 2 * h + head * DH + a * 64, row0 + kt * kRows);
+          tma_load_2d(sQ(st) + a * (kRows * 128), &tm_qkv128, &q_full[st], head * DH + a * 64, qr);
+          tma_load_2d(sG(st) + a * (kRows * 128), &tm_do128, &q_full[st], head * DH + a * 64, qr);
         }
-        for (int idx = 0; idx < ntiles; ++idx, ++g) {
-          const int st = g % kRingN;
-          mbar_wait(&q_empty[st], ((g / kRingN) & 1) ^ 1);
-          mbar_arrive_expect_tx(&q_full[st], 2 * SN::kTile + SN::kLD);
-          const int qr = row0 + (kt + idx) * kRows;
-#pragma unroll
-          for (int a = 0; a < DH / 64; ++a) {
-            tma_load_2d(sQ(st) + a * (kRows * 128), &tm_qkv128, &q_full[st], head * DH + a * 64, qr);
-            tma_load_2d(sG(st) + a * (kRows * 128), &tm_do128, &q_full[st], head * DH + a * 64, qr);
-          }
-          const long o = static_cast<long>(head) * Ttok + qr;
-          bulk_g2s(sLD + st * 2 * kRows, lse + o, kRows * 4, &q_full[st]);
-          bulk_g2s(sLD + st * 2 * kRows + kRows, Dd + o, kRows * 4, &q_full[st]);
-        }
+        const long o = static_cast<long>(head) * Ttok + qr;
+        bulk_g2s(sLD + st * 2 * kRows, lse + o, kRows * 4, &q_full[st]);
+        bulk_g2s(sLD + st * 2 * kRows + kRows, Dd + o, kRows * 4, &q_full[st]);
       }
     }
   } else if (warp == 1) {
     constexpr uint32_t id_s = umma_idesc_bf16(128, kRows, 0, 0);   // S^T, dP^T: K-major A and B, N = 128
     constexpr uint32_t id_a = umma_idesc_bf16(128, DH, 0, 1);      // dV, dK: A from TMEM, B MN-major
-    int g = 0;
-    for (int n = 0;; ++n) {
-      const int w = item_of(n);
-      if (w < 0) break;
-      const int ntiles = nq - w / BH;
-      mbar_wait(kv_full, n & 1);
+    mbar_wait(kv_full, 0);
+    tc_fence_after();
+    for (int idx = 0; idx < ntiles; ++idx) {
+      const int st = idx % kRingN, par = idx & 1;
+      mbar_wait(&q_full[st], (idx / kRingN) & 1);
       tc_fence_after();
-      for (int idx = 0; idx < ntiles; ++idx, ++g) {
-        const int st = g % kRingN, par = g & 1;
-        mbar_wait(&q_full[st], (g / kRingN) & 1);
-        tc_fence_after();
-        const uint32_t k = smem_u32(sK), v = smem_u32(sV), q = smem_u32(sQ(st)), gg = smem_u32(sG(st));
-        if (elect_one()) {
+      const uint32_t k = smem_u32(sK), v = smem_u32(sV), q = smem_u32(sQ(st)), g = smem_u32(sG(st));
+      if (elect_one()) {
 #pragma unroll
-          for (int kk = 0; kk < DH / 16; ++kk) {
-            const uint32_t o = (kk >> 2) * (kRows * 128) + (kk & 3) * 32;
-            umma_bf16(tm_S, umma_desc_sw128(k + o, 16, 1024), umma_desc_sw128(q + o, 16, 1024), id_s, kk > 0);
-          }
-          umma_commit(s_full);
-#pragma unroll
-          for (int kk = 0; kk < DH / 16; ++kk) {
-            const uint32_t o = (kk >> 2) * (kRows * 128) + (kk & 3) * 32;
-            umma_bf16(tm_dP, umma_desc_sw128(v + o, 16, 1024), umma_desc_sw128(gg + o, 16, 1024), id_s, kk > 0);
-          }
-          umma_commit(dp_full);
+        for (int kk = 0; kk < DH / 16; ++kk) {
+          const uint32_t o = (kk >> 2) * (kRows * 128) + (kk & 3) * 32;
+          umma_bf16(tm_S, umma_desc_sw128(k + o, 16, 1024), umma_desc_sw128(q + o, 16, 1024), id_s, kk > 0);
         }
-        __syncwarp();
-        if (idx == 0 && n > 0) mbar_wait(acc_free, (n - 1) & 1);   // dV / dK of the previous item read out
-        mbar_wait(p_full, par);
-        tc_fence_after();
-        if (elect_one()) {
+        umma_commit(s_full);
 #pragma unroll
-          for (int kk = 0; kk < kRows / 16; ++kk) {
-            // queries [16kk, 16kk + 16): half kk / 4 packed them at columns 64 (kk / 4) + 8 (kk % 4)
-            const uint32_t ac = (kk >> 2) * 64 + (kk & 3) * 8;
-            umma_bf16_ts(tm_dV, tm_S + ac, umma_desc_sw128(gg + kk * 2048, kRows * 128, 1024), id_a, (idx | kk) != 0);
-          }
+        for (int kk = 0; kk < DH / 16; ++kk) {
+          const uint32_t o = (kk >> 2) * (kRows * 128) + (kk & 3) * 32;
+          umma_bf16(tm_dP, umma_desc_sw128(v + o, 16, 1024), umma_desc_sw128(g + o, 16, 1024), id_s, kk > 0);
         }
-        __syncwarp();
-        mbar_wait(ds_full, par);
-        tc_fence_after();
-        if (elect_one()) {
-#pragma unroll
-          for (int kk = 0; kk < kRows / 16; ++kk) {
-            const uint32_t ac = (kk >> 2) * 64 + (kk & 3) * 8;
-            umma_bf16_ts(tm_dK, tm_dP + ac, umma_desc_sw128(q + kk * 2048, kRows * 128, 1024), id_a, (idx | kk) != 0);
-          }
-          umma_commit(&q_empty[st]);
-          if (idx == ntiles - 1) umma_commit(acc_done);
-        }
-        __syncwarp();
+        umma_commit(dp_full);
       }
+      __syncwarp();
+      mbar_wait(p_full, par);
+      tc_fence_after();
+      if (elect_one()) {
+#pragma unroll
+        for (int kk = 0; kk < kRows / 16; ++kk) {
+          // queries [16kk, 16kk + 16): half kk / 4 packed them at columns 64 (kk / 4) + 8 (kk % 4)
+          const uint32_t ac = (kk >> 2) * 64 + (kk & 3) * 8;
+          umma_bf16_ts(tm_dV, tm_S + ac, umma_desc_sw128(g + kk * 2048, kRows * 128, 1024), id_a, (idx | kk) != 0);
+        }
+      }
+      __syncwarp();
+      mbar_wait(ds_full, par);
+      tc_fence_after();
+      if (elect_one()) {
+#pragma unroll
+        for (int kk = 0; kk < kRows / 16; ++kk) {
+          const uint32_t ac = (kk >> 2) * 64 + (kk & 3) * 8;
+          umma_bf16_ts(tm_dK, tm_dP + ac, umma_desc_sw128(q + kk * 2048, kRows * 128, 1024), id_a, (idx | kk) != 0);
+        }
+        umma_commit(&q_empty[st]);
+        if (idx == ntiles - 1) umma_commit(acc_done);
+      }
+      __syncwarp();
     }
   } else {
     const int quarter = warp & 3, half = (warp - 2) >> 2;   // S^T columns (queries) [64 half, 64 half + 64)
     const int row = quarter * 32 + lane;                     // key row within the block
+    const int key = kt * kRows + row;
     const uint32_t lane_off = static_cast<uint32_t>(quarter * 32) << 16;
     const uint32_t col = half * 64 + lane_off;
-    int g = 0;
-    for (int n = 0;; ++n) {
-      const int w = item_of(n);
-      if (w < 0) break;
-      const int kt = w / BH, bh = w % BH, b = bh / nh, head = bh % nh, ntiles = nq - kt;
-      const int key = kt * kRows + row;
-      for (int idx = 0; idx < ntiles; ++idx, ++g) {
-        const int i = kt + idx, st = g % kRingN, par = g & 1;
-        const float* ld = sLD + st * 2 * kRows + half * 64;
-        mbar_wait(&q_full[st], (g / kRingN) & 1);   // lse / D of this tile
-        mbar_wait(s_full, par);
-        tc_fence_after();
-        float p[64];
-        {
-          uint32_t sr[32];
+    for (int idx = 0; idx < ntiles; ++idx) {
+      const int i = kt + idx, st = idx % kRingN, par = idx & 1;
+      const float* ld = sLD + st * 2 * kRows + half * 64;
+      mbar_wait(&q_full[st], (idx / kRingN) & 1);   // lse / D of this tile (the MMA thread saw it complete)
+      mbar_wait(s_full, par);
+      tc_fence_after();
+      float p[64];
+      {
+        uint32_t sr[32];
 #pragma unroll
-          for (int hh = 0; hh < 2; ++hh) {
-            tmem_ld_32x32b_x32(tm_S + col + hh * 32, sr);
-            tmem_ld_wait();
+        for (int hh = 0; hh < 2; ++hh) {
+          tmem_ld_32x32b_x32(tm_S + col + hh * 32, sr);
+          tmem_ld_wait();
 #pragma unroll
-            for (int c4 = 0; c4 < 32; c4 += 4) {
-              const float4 l4 = ld_shared_f4(ld + hh * 32 + c4);
-              const float lv[4] = {l4.x * LOG2E, l4.y * LOG2E, l4.z * LOG2E, l4.w * LOG2E};
-#pragma unroll
-              for (int e = 0; e < 4; ++e) p[hh * 32 + c4 + e] = ex2(__uint_as_float(sr[c4 + e]) * sl2 - lv[e]);
-            }
-          }
-        }
-        if (i == kt) {   // diagonal tile: P^T[key][q] = 0 for q < key
-          const int lo = row - half * 64;
-#pragma unroll
-          for (int cc = 0; cc < 64; ++cc) p[cc] = cc < lo ? 0.f : p[cc];
-        }
-        {
-          uint32_t pk[32];
-#pragma unroll
-          for (int cc = 0; cc < 64; cc += 2) {
-            const __nv_bfloat162 pp = __floats2bfloat162_rn(p[cc], p[cc + 1]);
-            pk[cc / 2] = *reinterpret_cast<const uint32_t*>(&pp);
-          }
-          tmem_st_32x32b_x32(tm_S + col, pk);
-          tmem_st_wait();
-        }
-        tc_fence_before();
-        __syncwarp();
-        if (lane == 0) mbar_arrive(p_full);
-        mbar_wait(dp_full, par);
-        tc_fence_after();
-        uint32_t dk[32];
-        {
-          uint32_t dr[32];
-#pragma unroll
-          for (int hh = 0; hh < 2; ++hh) {
-            tmem_ld_32x32b_x32(tm_dP + col + hh * 32, dr);
-            tmem_ld_wait();
-#pragma unroll
-            for (int c4 = 0; c4 < 32; c4 += 4) {
-              const float4 d4 = ld_shared_f4(ld + kRows + hh * 32 + c4);
-              const int cc = hh * 32 + c4;
-              const float d0 = p[cc] * (__uint_as_float(dr[c4]) - d4.x), d1 = p[cc + 1] * (__uint_as_float(dr[c4 + 1]) - d4.y);
-              const float d2 = p[cc + 2] * (__uint_as_float(dr[c4 + 2]) - d4.z), d3 = p[cc + 3] * (__uint_as_float(dr[c4 + 3]) - d4.w);
-              const __nv_bfloat162 a0 = __floats2bfloat162_rn(d0, d1), a1 = __floats2bfloat162_rn(d2, d3);
-              dk[cc / 2] = *reinterpret_cast<const uint32_t*>(&a0);
-              dk[cc / 2 + 1] = *reinterpret_cast<const uint32_t*>(&a1);
-            }
-          }
-        }
-        tmem_st_32x32b_x32(tm_dP + col, dk);
-        tmem_st_wait();
-        tc_fence_before();
-        __syncwarp();
-        if (lane == 0) mbar_arrive(ds_full);
-        if (dsimg) {
-          // dS image (fa_bwd_dq_img's A operand): query block i, 64-key tile key / 64, box = query half;
-          // key row (key mod 64) as the 128-byte row of an MN-major SW128 tile (16-byte chunk c of row r
-          // at ((c ^ (r mod 8)) << 4)); chunks 2p, 2p + 1 land on the aligned pair (2p ^ (r & 6)), swapped
-          // when r is odd: one 32-byte store per pair
-          const int kt64 = key >> 6, r64 = key & 63;
-          const size_t tri = static_cast<size_t>(nq) * (nq + 1);
-          uint8_t* rowp = dsimg + ((static_cast<size_t>(bh) * tri + static_cast<size_t>(i) * (i + 1) + kt64) * 2 + half) *
-                                      8192 + r64 * 128;
-          const bool sw = (r64 & 1) != 0;
-#pragma unroll
-          for (int pp = 0; pp < 4; ++pp) {
-            uint32_t v8[8];
+          for (int c = 0; c < 32; c += 4) {
+            const float4 l4 = ld_shared_f4(ld + hh * 32 + c);
+            const float lv[4] = {l4.x * LOG2E, l4.y * LOG2E, l4.z * LOG2E, l4.w * LOG2E};
 #pragma unroll
             for (int e = 0; e < 4; ++e) {
-              v8[e] = sw ? dk[8 * pp + 4 + e] : dk[8 * pp + e];
-              v8[4 + e] = sw ? dk[8 * pp + e] : dk[8 * pp + 4 + e];
+              const int cc = hh * 32 + c + e;
+              p[cc] = ex2(__uint_as_float(sr[c + e]) * sl2 - lv[e]);
             }
-            st_global_v8(rowp + (((2 * pp) ^ (r64 & 6)) << 4), v8);
           }
         }
       }
-      // epilogue: the two query halves take half of dV's and dK's columns each, TMEM -> registers ->
-      // 16-byte global stores of the key row (dK scaled by 1/sqrt(dh)); TMEM released as soon as read
-      mbar_wait(acc_done, n & 1);
-      tc_fence_after();
-      bf16* krow = dqkv + (static_cast<long>(b) * s + key) * (3 * h) + h + head * DH;
-      bf16* vrow = krow + h;
-#pragma unroll 1
-      for (int c0 = half * (DH / 2); c0 < (half + 1) * (DH / 2); c0 += 32) {
-        uint32_t rv[32], rk[32];
-        tmem_ld_32x32b_x32(tm_dV + c0 + lane_off, rv);
-        tmem_ld_32x32b_x32(tm_dK + c0 + lane_off, rk);
-        tmem_ld_wait();
-        if (c0 + 32 == (half + 1) * (DH / 2)) {
-          tc_fence_before();
-          __syncwarp();
-          if (lane == 0) mbar_arrive(acc_free);
-        }
+      if (i == kt) {   // diagonal tile: P^T[key][q] = 0 for q < key
+        const int lo = row - half * 64;
 #pragma unroll
-        for (int q4 = 0; q4 < 4; ++q4) {
-          uint4 uv, uk;
-          __nv_bfloat162* hv = reinterpret_cast<__nv_bfloat162*>(&uv);
-          __nv_bfloat162* hk = reinterpret_cast<__nv_bfloat162*>(&uk);
+        for (int c = 0; c < 64; ++c) p[c] = c < lo ? 0.f : p[c];
+      }
+      {
+        uint32_t pk[32];
+#pragma unroll
+        for (int c = 0; c < 64; c += 2) {
+          const __nv_bfloat162 pp = __floats2bfloat162_rn(p[c], p[c + 1]);
+          pk[c / 2] = *reinterpret_cast<const uint32_t*>(&pp);
+        }
+        tmem_st_32x32b_x32(tm_S + col, pk);
+        tmem_st_wait();
+      }
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(p_full);
+      mbar_wait(dp_full, par);
+      tc_fence_after();
+      uint32_t dk[32];
+      {
+        uint32_t dr[32];
+#pragma unroll
+        for (int hh = 0; hh < 2; ++hh) {
+          tmem_ld_32x32b_x32(tm_dP + col + hh * 32, dr);
+          tmem_ld_wait();
+#pragma unroll
+          for (int c = 0; c < 32; c += 4) {
+            const float4 d4 = ld_shared_f4(ld + kRows + hh * 32 + c);
+            const int cc = hh * 32 + c;
+            const float d0 = p[cc] * (__uint_as_float(dr[c]) - d4.x), d1 = p[cc + 1] * (__uint_as_float(dr[c + 1]) - d4.y);
+            const float d2 = p[cc + 2] * (__uint_as_float(dr[c + 2]) - d4.z), d3 = p[cc + 3] * (__uint_as_float(dr[c + 3]) - d4.w);
+            const __nv_bfloat162 a0 = __floats2bfloat162_rn(d0, d1), a1 = __floats2bfloat162_rn(d2, d3);
+            dk[cc / 2] = *reinterpret_cast<const uint32_t*>(&a0);
+            dk[cc / 2 + 1] = *reinterpret_cast<const uint32_t*>(&a1);
+          }
+        }
+      }
+      tmem_st_32x32b_x32(tm_dP + col, dk);
+      tmem_st_wait();
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(ds_full);
+      if (dsimg) {
+        // dS image (fa_bwd_dq_img's A operand): query block i, 64-key tile key / 64, box = query half;
+        // key row (key mod 64) as the 128-byte row of an MN-major SW128 tile (16-byte chunk c of row r
+        // at ((c ^ (r mod 8)) << 4)); chunks 2p, 2p + 1 land on the aligned pair (2p ^ (r & 6)), swapped
+        // when r is odd: one 32-byte store per pair
+        const int kt64 = key >> 6, r64 = key & 63;
+        const size_t tri = static_cast<size_t>(nq) * (nq + 1);
+        uint8_t* rowp = dsimg + ((static_cast<size_t>(bh) * tri + static_cast<size_t>(i) * (i + 1) + kt64) * 2 + half) * 8192 +
+                        r64 * 128;
+        const bool sw = (r64 & 1) != 0;
+#pragma unroll
+        for (int pp = 0; pp < 4; ++pp) {
+          uint32_t v8[8];
 #pragma unroll
           for (int e = 0; e < 4; ++e) {
-            hv[e] = __floats2bfloat162_rn(__uint_as_float(rv[8 * q4 + 2 * e]), __uint_as_float(rv[8 * q4 + 2 * e + 1]));
-            hk[e] = __floats2bfloat162_rn(__uint_as_float(rk[8 * q4 + 2 * e]) * qk_scale,
-                                          __uint_as_float(rk[8 * q4 + 2 * e + 1]) * qk_scale);
+            v8[e] = sw ? dk[8 * pp + 4 + e] : dk[8 * pp + e];
+            v8[4 + e] = sw ? dk[8 * pp + e] : dk[8 * pp + 4 + e];
           }
-          *reinterpret_cast<uint4*>(vrow + c0 + 8 * q4) = uv;
-          *reinterpret_cast<uint4*>(krow + c0 + 8 * q4) = uk;
+          st_global_v8(rowp + (((2 * pp) ^ (r64 & 6)) << 4), v8);
         }
       }
+    }
+    // epilogue: dV and dK (scaled by 1/sqrt(dh)) through the idle ring slot 0 as SW128 K-major tiles
+    // of 128 rows x 64 columns, TMA-stored; the two query halves take half of the columns each
+    mbar_wait(acc_done, 0);
+    tc_fence_after();
+    auto stV = [&](int a) { return sQ(0) + a * (kRows * 128); };
+    auto stK = [&](int a) { return sG(0) + a * (kRows * 128); };
+#pragma unroll 1
+    for (int c = half * (DH / 2); c < (half + 1) * (DH / 2); c += 32) {
+      uint32_t rv[32], rk[32];
+      tmem_ld_32x32b_x32(tm_dV + c + lane_off, rv);
+      tmem_ld_32x32b_x32(tm_dK + c + lane_off, rk);
+      tmem_ld_wait();
+      float fv[32], fk[32];
+#pragma unroll
+      for (int e = 0; e < 32; ++e) { fv[e] = __uint_as_float(rv[e]); fk[e] = __uint_as_float(rk[e]) * qk_scale; }
+      st_half_row_sw128(stV(c / 64), row, (c % 64) / 8, fv);
+      st_half_row_sw128(stK(c / 64), row, (c % 64) / 8, fk);
+    }
+    fence_proxy_async();
+    named_bar(1, 256);
+    if (threadIdx.x == 64) {
+      const int r0 = b * s + kt * kRows;
+#pragma unroll
+      for (int a = 0; a < DH / 64; ++a) {
+        tma_store_2d(&tm_dqkv, stV(a), 2 * h + head * DH + a * 64, r0);
+        tma_store_2d(&tm_dqkv, stK(a), h + head * DH + a * 64, r0);
+      }
+      bulk_commit_wait_read();
     }
   }
   tc_fence_before();
@@ -1754,14 +1727,8 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
           cudaFuncSetAttribute(fa_bwd_dkdv_n128<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize, SmemN<DH>::kBytes);
           nset = true;
         }
-        // persistent (MARIO_ATTN_DKDV_PERS=1): one CTA per SM of the full device (the item -> CTA map
-        // does not change any item's arithmetic, so the launching thread's SM budget is irrelevant)
-        static const int pers = getenv("MARIO_ATTN_DKDV_PERS") ? atoi(getenv("MARIO_ATTN_DKDV_PERS")) : 0;
-        const int items = static_cast<int>(grid.x);
-        const int sms = device_sm_count();
-        const int g = (pers && items > sms) ? sms : items;
-        fa_bwd_dkdv_n128<DH><<<g, kThreadsB, SmemN<DH>::kBytes, st>>>(m128, d128, lse, Dd, dqkv, B, s, nh, dsimg,
-                                                                        qk_scale);
+        fa_bwd_dkdv_n128<DH><<<grid, kThreadsB, SmemN<DH>::kBytes, st>>>(m128, d128, g128, lse, Dd, dqkv, B, s, nh,
+                                                                           dsimg, qk_scale);
       } else
       fa_bwd_dkdv_ts<DH><<<grid, kThreadsB, smem_dkdv_ts<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s, nh,
                                                                         dsimg, attn_l2hint(), qk_scale,
