@@ -1669,6 +1669,228 @@ fa_bwd_dkdv_n128(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_con
   if (warp == 1) tmem_dealloc<512>(tm);
 }
 
+// ------------------------------------------------------------------- dQ, 128-key tiles
+// fa_bwd_dq_n128: the recomputing dQ kernel (no dS image: cfg 5's s = 16384, whose image would be
+// 10.8 GB, and callers without a workspace) on 128-key tiles, the mirror of fa_bwd_dkdv_n128: one CTA
+// per 128 queries (TMEM lanes), heaviest query blocks first; S = Q K_j^T and dP = dO V_j^T as M128 N128
+// K16 MMAs (the N = 64 tiles of fa_bwd_dq_pers run at 43% of the tensor rate), dS = P (dP - D) packed
+// to bf16 in place over dP by 8 softmax warps (lane quarter x 64-key half; lse and D are row constants
+// in registers), dQ += dS K_j with A from TMEM. TMEM dQ | S | dP. The MMA thread issues S(j+1) as soon
+// as the softmax has S(j) in registers (s_free), dQ(j) once dS(j) is in TMEM, then dP(j+1): dP(j+1)
+// overwrites the dS(j) columns only after dQ(j) read them (tcgen05.mma executes in issue order).
+// K/V tiles stream through a 2-deep ring; the dQ tile goes out through the idle Q/dO staging by TMA.
+// Same arithmetic in the same order as fa_bwd_dq_pers (dQ bitwise equal). s % 128 == 0 only.
+template <int DH>
+struct SmemQN {
+  static constexpr int kTile = kRows * DH * 2;                 // 128-row Q, dO, K or V tile
+  static constexpr int kBytes = 2 * kTile + kRingN * 2 * kTile + 256 + 1024;
+};
+template <int DH>
+__global__ void __launch_bounds__(kThreadsB, 1)
+fa_bwd_dq_n128(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_do128,
+               const __grid_constant__ CUtensorMap tm_dqkv, const float* lse, const float* Dd, int B, int s, int nh,
+               float qk_scale) {
+  using SQ = SmemQN<DH>;
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+  uint8_t* sQ = smem;
+  uint8_t* sG = sQ + SQ::kTile;
+  auto sK = [&](int r) { return sG + SQ::kTile + r * 2 * SQ::kTile; };
+  auto sV = [&](int r) { return sG + SQ::kTile + r * 2 * SQ::kTile + SQ::kTile; };
+  uint64_t* bar = reinterpret_cast<uint64_t*>(sG + SQ::kTile + kRingN * 2 * SQ::kTile);
+  uint64_t* qd_full = bar;                 // 1
+  uint64_t* kv_full = bar + 1;             // kRingN
+  uint64_t* kv_empty = kv_full + kRingN;   // kRingN
+  uint64_t* s_full = kv_empty + kRingN;    // 1  S(j) in TMEM
+  uint64_t* s_free = s_full + 1;           // 1  S(j) read by the softmax (8 warps)
+  uint64_t* dp_full = s_free + 1;          // 1  dP(j) in TMEM
+  uint64_t* ds_full = dp_full + 1;         // 1  dS(j) packed (8 warps)
+  uint64_t* acc_done = ds_full + 1;        // 1
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(acc_done + 1);
+
+  const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+  const int BH = B * nh, nt = s / kRows;
+  const int qb = nt - 1 - static_cast<int>(blockIdx.x) / BH, bh = blockIdx.x % BH, b = bh / nh, head = bh % nh;
+  const int h = nh * DH;
+  const long Ttok = static_cast<long>(B) * s;
+  const int ntiles = qb + 1;               // key tiles 0 .. qb (tile qb is the diagonal)
+  const float sl2 = qk_scale * LOG2E;
+
+  if (warp == 0 && lane == 0) {
+    tma_prefetch_desc(&tm_qkv128);
+    tma_prefetch_desc(&tm_do128);
+    mbar_init(qd_full, 1);
+    for (int i = 0; i < kRingN; ++i) { mbar_init(&kv_full[i], 1); mbar_init(&kv_empty[i], 1); }
+    mbar_init(s_full, 1); mbar_init(s_free, 8); mbar_init(dp_full, 1); mbar_init(ds_full, 8); mbar_init(acc_done, 1);
+    fence_barrier_init();
+  }
+  if (warp == 1) tmem_alloc<512>(tmem_slot);
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tm = *tmem_slot;
+  const uint32_t tm_dQ = tm, tm_S = tm + DH, tm_dP = tm + DH + kRows;
+
+  if (warp == 0) {
+    if (elect_one()) {
+      const int row0 = b * s;
+      mbar_arrive_expect_tx(qd_full, 2 * SQ::kTile);
+#pragma unroll
+      for (int a = 0; a < DH / 64; ++a) {
+        tma_load_2d(sQ + a * (kRows * 128), &tm_qkv128, qd_full, head * DH + a * 64, row0 + qb * kRows);
+        tma_load_2d(sG + a * (kRows * 128), &tm_do128, qd_full, head * DH + a * 64, row0 + qb * kRows);
+      }
+      for (int j = 0; j < ntiles; ++j) {
+        const int st = j % kRingN;
+        mbar_wait(&kv_empty[st], ((j / kRingN) & 1) ^ 1);
+        mbar_arrive_expect_tx(&kv_full[st], 2 * SQ::kTile);
+#pragma unroll
+        for (int a = 0; a < DH / 64; ++a) {
+          tma_load_2d(sK(st) + a * (kRows * 128), &tm_qkv128, &kv_full[st], h + head * DH + a * 64, row0 + j * kRows);
+          tma_load_2d(sV(st) + a * (kRows * 128), &tm_qkv128, &kv_full[st], 2 * h + head * DH + a * 64, row0 + j * kRows);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    constexpr uint32_t id_s = umma_idesc_bf16(128, kRows, 0, 0);   // S, dP: K-major A and B, N = 128
+    constexpr uint32_t id_a = umma_idesc_bf16(128, DH, 0, 1);      // dQ: A = dS from TMEM, B = K MN-major
+    mbar_wait(qd_full, 0);
+    tc_fence_after();
+    const uint32_t q = smem_u32(sQ), gg = smem_u32(sG);
+    auto issue_s = [&](int j) {   // S(j) = Q K_j^T
+      const int st = j % kRingN;
+      mbar_wait(&kv_full[st], (j / kRingN) & 1);
+      tc_fence_after();
+      if (elect_one()) {
+        const uint32_t k = smem_u32(sK(st));
+#pragma unroll
+        for (int kk = 0; kk < DH / 16; ++kk) {
+          const uint32_t o = (kk >> 2) * (kRows * 128) + (kk & 3) * 32;
+          umma_bf16(tm_S, umma_desc_sw128(q + o, 16, 1024), umma_desc_sw128(k + o, 16, 1024), id_s, kk > 0);
+        }
+        umma_commit(s_full);
+      }
+      __syncwarp();
+    };
+    auto issue_dp = [&](int j) {   // dP(j) = dO V_j^T (K/V of tile j already waited for by issue_s)
+      const int st = j % kRingN;
+      if (elect_one()) {
+        const uint32_t v = smem_u32(sV(st));
+#pragma unroll
+        for (int kk = 0; kk < DH / 16; ++kk) {
+          const uint32_t o = (kk >> 2) * (kRows * 128) + (kk & 3) * 32;
+          umma_bf16(tm_dP, umma_desc_sw128(gg + o, 16, 1024), umma_desc_sw128(v + o, 16, 1024), id_s, kk > 0);
+        }
+        umma_commit(dp_full);
+      }
+      __syncwarp();
+    };
+    issue_s(0);
+    issue_dp(0);
+    for (int j = 0; j < ntiles; ++j) {
+      const int st = j % kRingN;
+      if (j + 1 < ntiles) {
+        mbar_wait(s_free, j & 1);   // the softmax holds S(j) in registers
+        issue_s(j + 1);
+      }
+      mbar_wait(ds_full, j & 1);
+      tc_fence_after();
+      if (elect_one()) {
+        const uint32_t k = smem_u32(sK(st));
+#pragma unroll
+        for (int kk = 0; kk < kRows / 16; ++kk) {
+          // keys [16kk, 16kk + 16): half kk / 4 packed them at columns 64 (kk / 4) + 8 (kk % 4)
+          const uint32_t ac = (kk >> 2) * 64 + (kk & 3) * 8;
+          umma_bf16_ts(tm_dQ, tm_dP + ac, umma_desc_sw128(k + kk * 2048, kRows * 128, 1024), id_a, (j | kk) != 0);
+        }
+        umma_commit(&kv_empty[st]);
+        if (j == ntiles - 1) umma_commit(acc_done);
+      }
+      __syncwarp();
+      if (j + 1 < ntiles) issue_dp(j + 1);
+    }
+  } else {
+    const int quarter = warp & 3, half = (warp - 2) >> 2;   // S columns (keys) [64 half, 64 half + 64)
+    const int row = quarter * 32 + lane;                     // query row within the block
+    const uint32_t lane_off = static_cast<uint32_t>(quarter * 32) << 16;
+    const uint32_t col = half * 64 + lane_off;
+    const long gr = static_cast<long>(b) * s + qb * kRows + row;
+    const float L = lse[static_cast<long>(head) * Ttok + gr] * LOG2E;
+    const float Dr = Dd[static_cast<long>(head) * Ttok + gr];
+    for (int j = 0; j < ntiles; ++j) {
+      const int par = j & 1;
+      mbar_wait(s_full, par);
+      tc_fence_after();
+      float p[64];
+      {
+        uint32_t sr[64];
+        tmem_ld_32x32b_x32(tm_S + col, *reinterpret_cast<uint32_t(*)[32]>(&sr[0]));
+        tmem_ld_32x32b_x32(tm_S + col + 32, *reinterpret_cast<uint32_t(*)[32]>(&sr[32]));
+        tmem_ld_wait();
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(s_free);
+#pragma unroll
+        for (int c = 0; c < 64; ++c) p[c] = ex2(__uint_as_float(sr[c]) * sl2 - L);
+      }
+      if (j == qb) {   // diagonal tile: P[q][key] = 0 for key > q
+        const int hi = row - half * 64;
+#pragma unroll
+        for (int c = 0; c < 64; ++c) p[c] = c > hi ? 0.f : p[c];
+      }
+      mbar_wait(dp_full, par);
+      tc_fence_after();
+      uint32_t dk[32];
+      {
+        uint32_t dr[32];
+#pragma unroll
+        for (int hh = 0; hh < 2; ++hh) {
+          tmem_ld_32x32b_x32(tm_dP + col + hh * 32, dr);
+          tmem_ld_wait();
+#pragma unroll
+          for (int c = 0; c < 32; c += 2) {
+            const int cc = hh * 32 + c;
+            const __nv_bfloat162 d2 = __floats2bfloat162_rn(p[cc] * (__uint_as_float(dr[c]) - Dr),
+                                                            p[cc + 1] * (__uint_as_float(dr[c + 1]) - Dr));
+            dk[cc / 2] = *reinterpret_cast<const uint32_t*>(&d2);
+          }
+        }
+      }
+      tmem_st_32x32b_x32(tm_dP + col, dk);
+      tmem_st_wait();
+      tc_fence_before();
+      __syncwarp();
+      if (lane == 0) mbar_arrive(ds_full);
+    }
+    // epilogue: dQ (scaled by 1/sqrt(dh)) through the idle Q / dO tiles as SW128 K-major 128 x 64 tiles,
+    // TMA-stored; the two halves take half of the columns each
+    mbar_wait(acc_done, 0);
+    tc_fence_after();
+    auto stQ = [&](int a) { return a < 2 ? sQ + a * (kRows * 128) : sG + (a - 2) * (kRows * 128); };
+#pragma unroll 1
+    for (int c0 = half * (DH / 2); c0 < (half + 1) * (DH / 2); c0 += 32) {
+      uint32_t rq[32];
+      tmem_ld_32x32b_x32(tm_dQ + c0 + lane_off, rq);
+      tmem_ld_wait();
+      float fq[32];
+#pragma unroll
+      for (int e = 0; e < 32; ++e) fq[e] = __uint_as_float(rq[e]) * qk_scale;
+      st_half_row_sw128(stQ(c0 / 64), row, (c0 % 64) / 8, fq);
+    }
+    fence_proxy_async();
+    named_bar(1, 256);
+    if (threadIdx.x == 64) {
+      const int r0 = b * s + qb * kRows;
+#pragma unroll
+      for (int a = 0; a < DH / 64; ++a) tma_store_2d(&tm_dqkv, stQ(a), head * DH + a * 64, r0);
+      bulk_commit_wait_read();
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 1) tmem_dealloc<512>(tm);
+}
+
 // >= 116 KB so that one CTA owns the SM (each allocates all 512 TMEM columns)
 constexpr int at_least_one_sm(int b) { return b < 116 * 1024 ? 116 * 1024 : b; }
 template <int DH>
@@ -1772,7 +1994,18 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
     fa_bwd_dq_img<DH><<<grid_i, kThreadsI, SmemI<DH>::kBytes, st>>>(m64, dsimg, dqkv, B, s, nh, attn_l2hint(),
                                                                      qk_scale);
   } else if (!only || only[1] == 'q') {
-    if (pers && dbg == 0) {
+    // 128-key tiles (fa_bwd_dq_n128) where s % 128 == 0: 1835 -> 1601 us for the whole backward at B 1,
+    // s 16384, 8 heads; 532 -> 489 us at s 4096 (dQ bitwise equal); MARIO_ATTN_DQ_N128=0: fa_bwd_dq_pers
+    static const int qn128 = getenv("MARIO_ATTN_DQ_N128") ? atoi(getenv("MARIO_ATTN_DQ_N128")) : 1;
+    if (qn128 && dbg == 0 && (s % kRows) == 0) {
+      static bool qset = false;
+      if (!qset) {
+        cudaFuncSetAttribute(fa_bwd_dq_n128<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize, SmemQN<DH>::kBytes);
+        qset = true;
+      }
+      fa_bwd_dq_n128<DH><<<B * nh * (s / kRows), kThreadsB, SmemQN<DH>::kBytes, st>>>(m128, d128, g128, lse, Dd, B, s,
+                                                                                      nh, qk_scale);
+    } else if (pers && dbg == 0) {
       static bool pset = false;
       if (!pset) {
         cudaFuncSetAttribute(fa_bwd_dq_pers<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem_dq<DH>());

@@ -14,7 +14,7 @@
 #include "sm100.cuh"
 using namespace mario::sm100;
 
-template <int MODE>
+template <int MODE, bool BG = false>
 __global__ void __launch_bounds__(128, 1) k(long long* cyc, int iters) {
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* sm = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -22,6 +22,8 @@ __global__ void __launch_bounds__(128, 1) k(long long* cyc, int iters) {
   __shared__ __align__(8) uint64_t bar;
   const int warp = threadIdx.x / 32;
   for (int i = threadIdx.x; i < 96 * 1024 / 4; i += blockDim.x) reinterpret_cast<uint32_t*>(sm)[i] = 0x3c003c00u;
+  __syncthreads();
+  if (threadIdx.x == 0) reinterpret_cast<uint32_t*>(sm)[96 * 1024 / 4 - 1] = 0u;   // background stop flag
   if (warp == 0) tmem_alloc<512>(&slot);
   if (threadIdx.x == 32) { mbar_init(&bar, 1); fence_barrier_init(); }
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -51,21 +53,32 @@ __global__ void __launch_bounds__(128, 1) k(long long* cyc, int iters) {
     mbar_wait(&bar, 0);
     long long t1 = clock64();
     cyc[blockIdx.x] = t1 - t0;
+    if (BG) reinterpret_cast<volatile uint32_t*>(sm)[96 * 1024 / 4 - 1] = 1u;   // stop flag
+  } else if (BG && threadIdx.x >= 32) {
+    // background: warps 1-3 store 16 bytes per lane into a 16 KB region (no overlap with A / B) as
+    // fast as they can, like softmax warps writing P tiles, until the MMA thread is done
+    volatile uint32_t* stop = reinterpret_cast<volatile uint32_t*>(sm) + 96 * 1024 / 4 - 1;
+    uint4* dst = reinterpret_cast<uint4*>(sm + 64 * 1024);
+    uint4 v = make_uint4(threadIdx.x, 1, 2, 3);
+    for (int i = 0; *stop == 0u; ++i) {
+#pragma unroll
+      for (int j = 0; j < 8; ++j) dst[((i * 8 + j) * 96 + threadIdx.x - 32) & 1023] = v;
+    }
   }
   tc_fence_before();
   __syncthreads();
   if (warp == 0) tmem_dealloc<512>(tm);
 }
 
-template <int MODE>
+template <int MODE, bool BG = false>
 void run(const char* name, int sms) {
   long long* d;
   cudaMalloc(&d, sms * sizeof(long long));
   const int smem = 100 * 1024;
-  cudaFuncSetAttribute(k<MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  cudaFuncSetAttribute(k<MODE, BG>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
   for (int iters : {64, 4096}) {
-    k<MODE><<<sms, 128, smem>>>(d, iters);
-    k<MODE><<<sms, 128, smem>>>(d, iters);
+    k<MODE, BG><<<sms, 128, smem>>>(d, iters);
+    k<MODE, BG><<<sms, 128, smem>>>(d, iters);
     cudaError_t e = cudaDeviceSynchronize();
     if (e) { printf("%s: %s\n", name, cudaGetErrorString(e)); return; }
     long long h[1024];
@@ -85,5 +98,8 @@ int main() {
   run<1>("SS N128", sms);
   run<2>("SS N256", sms);
   run<3>("TS N128", sms);
+  run<1, true>("SS N128+st", sms);
+  run<3, true>("TS N128+st", sms);
+  run<2, true>("SS N256+st", sms);
   return 0;
 }
