@@ -815,6 +815,9 @@ bool norm_bwd_pipe_vr(const bf16* dy, const bf16* x, const float* stats, const f
   const size_t base = pipe_smem_bytes(S, sb, kPipeR);
   int nblk = occ_grid(norm_bwd_pipe_k<kPipeR, V, RES, OUT32>, nt,
                       base + 8 * static_cast<size_t>(cdivl(rows, device_sms())));
+  // CTAs per SM cap (MARIO_NORM_BWD_CPS, A/B: fewer CTAs = fewer column-sum partials to reduce)
+  static const int cps = getenv("MARIO_NORM_BWD_CPS") ? atoi(getenv("MARIO_NORM_BWD_CPS")) : 0;
+  if (cps > 0 && nblk > cps * device_sms()) nblk = cps * device_sms();
   if (dg) {
     const long cap = static_cast<long>(partial_floats / (3 * static_cast<size_t>(n)));
     if (cap < 1) return false;
