@@ -148,8 +148,8 @@ mario_status mario_param_shape(const struct mario_plan* plan, int32_t idx, int64
 int32_t mario_plan_unckpt_tail(const struct mario_plan* plan);
 /* 1 if the plan's activation sets keep the layers' norm outputs (the backward reads them instead
  * of recomputing them; chosen unless it would exceed mem_budget_bytes, where the lean set is
- * planned instead; env MARIO_STORE_NORM=0/1 forces either), 0 for the lean set, -1 on NULL. */
-int32_t mario_plan_store_norm(const struct mario_plan* plan);
+ * planned instead; env MARIO_STORE_ACT=0/1 forces either), 0 for the lean set, -1 on NULL. */
+int32_t mario_plan_store_act(const struct mario_plan* plan);
 void mario_plan_destroy(struct mario_plan* plan);
 
 /* Schedule tuner (§5.3, Eq. 1): grid search

@@ -89,7 +89,7 @@ _lib.register("mario_param_count", C.c_int32, [_P])
 _lib.register("mario_param_shape", C.c_int32, [_P, C.c_int32, C.POINTER(C.c_int64), C.POINTER(C.c_int32)])
 _lib.register("mario_plan_destroy", None, [_P])
 _lib.register("mario_plan_unckpt_tail", C.c_int32, [_P])
-_lib.register("mario_plan_store_norm", C.c_int32, [_P])
+_lib.register("mario_plan_store_act", C.c_int32, [_P])
 _lib.register("mario_last_error", C.c_char_p, [])
 _lib.register("mario_tune", C.c_int32, [C.POINTER(CModel), C.c_int32, C.c_int32, C.c_uint64, C.POINTER(CTuneCosts),
                                         C.POINTER(CTuneResult), C.c_int32, C.POINTER(C.c_int32), C.POINTER(C.c_int32)])
@@ -189,9 +189,9 @@ class Plan:
         return int(_lib.lib().mario_plan_unckpt_tail(self.handle))
 
     @property
-    def store_norm(self) -> bool:
+    def store_act(self) -> bool:
         """Activation sets keep the norm outputs (else the lean set: the backward recomputes them)."""
-        return bool(_lib.lib().mario_plan_store_norm(self.handle))
+        return bool(_lib.lib().mario_plan_store_act(self.handle))
 
     def lists(self) -> List[List[Tuple[str, int, int]]]:
         return [[(op, m, p) for (op, m, p, *_r) in self.instrs(d)] for d in range(self.S)]

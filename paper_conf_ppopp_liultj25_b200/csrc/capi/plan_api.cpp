@@ -225,9 +225,9 @@ void fill_costs(PlanObj& P, const mario_costs* c) {
     s.fw[k] = (c && c->fw_ms) ? c->fw_ms[k] : fl / 1e12;   // analytic: 1 PFLOP/s effective
     s.bw[k] = (c && c->bw_ms) ? c->bw_ms[k] : 2.0 * fl / 1e12;
     s.rc[k] = (c && c->rc_ms) ? c->rc_ms[k] : s.fw[k];
-    s.act[k] = (c && c->act_bytes) ? c->act_bytes[k] : static_cast<double>(act_set_bytes(P.model, k, K, P.store_norm));
+    s.act[k] = (c && c->act_bytes) ? c->act_bytes[k] : static_cast<double>(act_set_bytes(P.model, k, K, P.store_act));
     s.ckpt[k] = (c && c->ckpt_bytes) ? c->ckpt_bytes[k] : (k == 0 ? 0.0 : static_cast<double>(stage_input_bytes(P.model)));
-    s.work[k] = (c && c->work_bytes) ? c->work_bytes[k] : static_cast<double>(cfw_work_bytes(P.model, k, K, P.store_norm));
+    s.work[k] = (c && c->work_bytes) ? c->work_bytes[k] : static_cast<double>(cfw_work_bytes(P.model, k, K, P.store_act));
   }
   const double msg = static_cast<double>(tokens_per_micro(P.model)) * P.model.hidden * elt_size(P.model);
   double alpha = 0.01, gbps = 700.0;
@@ -395,14 +395,14 @@ extern "C" mario_status mario_plan(const mario_model* model, int32_t stages, int
     if (scheme == MARIO_CHIMERA && (stages % 2 || microbatches % stages))
       return set_error(MARIO_EINVAL, "Chimera needs even stages and microbatches % stages == 0");
     // activation sets keep the norm outputs (exec/layout.h) unless the budget needs the lean set;
-    // MARIO_STORE_NORM=0/1 forces either (A/B measurements, lean-path tests)
+    // MARIO_STORE_ACT=0/1 forces either (A/B measurements, lean-path tests)
     bool sn = true, sn_forced = false;
-    if (const char* e = getenv("MARIO_STORE_NORM")) { sn = atoi(e) != 0; sn_forced = true; }
+    if (const char* e = getenv("MARIO_STORE_ACT")) { sn = atoi(e) != 0; sn_forced = true; }
     // one candidate plan: `lvl` in {BASE, CKPT, MARIO}; `keep_tail` devices un-checkpointed (A28)
     auto build = [&](int lvl, int keep_tail, std::unique_ptr<PlanObj>& P) -> mario_status {
       P = std::make_unique<PlanObj>();
       P->model = *model;
-      P->store_norm = sn;
+      P->store_act = sn;
       P->pp = pp;
       P->level = level;
       P->budget = mem_budget_bytes;
@@ -496,7 +496,7 @@ extern "C" mario_status mario_plan(const mario_model* model, int32_t stages, int
   });
 }
 
-extern "C" int32_t mario_plan_store_norm(const struct mario_plan* P) { return P ? (P->store_norm ? 1 : 0) : -1; }
+extern "C" int32_t mario_plan_store_act(const struct mario_plan* P) { return P ? (P->store_act ? 1 : 0) : -1; }
 
 extern "C" int32_t mario_plan_unckpt_tail(const struct mario_plan* P) { return P ? P->unckpt_tail : -1; }
 

@@ -25,8 +25,8 @@ Arena make_arena(const PlanObj& P, int dev, const PlanObj::Pools& pools) {
   bool has_last = false;
   for (int p = 0; p < P.pp.parts(); ++p) {
     int k = P.pp.vstage(dev, p);
-    act_max = std::max(act_max, act_set_bytes(m, k, K, P.store_norm));
-    cfw_max = std::max(cfw_max, cfw_work_bytes(m, k, K, P.store_norm));
+    act_max = std::max(act_max, act_set_bytes(m, k, K, P.store_act));
+    cfw_max = std::max(cfw_max, cfw_work_bytes(m, k, K, P.store_act));
     has_last = has_last || k == K - 1;
   }
   a.ckpt_stride = stage_input_bytes(m);
@@ -36,7 +36,7 @@ Arena make_arena(const PlanObj& P, int dev, const PlanObj::Pools& pools) {
   a.n_act = pools.act;
   a.act = take(a.act_stride * std::max(1, a.n_act));
   a.cfw = take(cfw_max);
-  a.bw = take(bw_scratch_bytes(m, P.store_norm));
+  a.bw = take(bw_scratch_bytes(m, P.store_act));
   if (has_last) a.logits = take(logits_bytes(m));
   a.msg_stride = stage_input_bytes(m);
   a.n_sa = pools.send_act; a.n_sg = pools.send_grad; a.n_rg = pools.recv_grad;

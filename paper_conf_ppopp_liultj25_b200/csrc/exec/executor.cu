@@ -327,7 +327,7 @@ struct Exec {
     const int Tn = static_cast<int>(tokens_per_micro(m)), h = m.hidden, f = m.ffn_hidden, nh = m.n_heads;
     const int dh = h / nh, s = m.seq_len, mbs = m.micro_batch;
     const bool gpt = m.family == MARIO_GPT;
-    const bool sn = D.P->store_norm;
+    const bool sn = D.P->store_act;
     const LayerAct LA = layer_act_layout(m, sn);
     const LayerTrans LT = layer_trans_layout(m, sn);
     const HeadAct HA = head_act_layout(m);
@@ -364,7 +364,7 @@ struct Exec {
       T* H1 = reinterpret_cast<T*>(L + LA.H1);
       T* A2 = reinterpret_cast<T*>(sn ? L + LA.A2 : trans + LT.A2);
       T* Z = reinterpret_cast<T*>(L + LA.Z);
-      T* Gt = reinterpret_cast<T*>(trans + LT.G);
+      T* Gt = reinterpret_cast<T*>(sn ? L + LA.G : trans + LT.G);
       float* st1 = reinterpret_cast<float*>(L + LA.st1);
       float* st2 = reinterpret_cast<float*>(L + LA.st2);
       // output of this layer
@@ -438,7 +438,7 @@ struct Exec {
     const int Tn = static_cast<int>(tokens_per_micro(m)), h = m.hidden, f = m.ffn_hidden, nh = m.n_heads;
     const int dh = h / nh, s = m.seq_len, mbs = m.micro_batch;
     const bool gpt = m.family == MARIO_GPT;
-    const bool sn = D.P->store_norm;
+    const bool sn = D.P->store_act;
     const LayerAct LA = layer_act_layout(m, sn);
     const HeadAct HA = head_act_layout(m);
     const BwScratch BS = bw_scratch_layout(m, sn);
@@ -495,11 +495,11 @@ struct Exec {
       uint8_t* L = base + li * LA.bytes;
       const T* Hin = (li == 0 && k > 0) ? D.template at<T>(D.a.ckpt + static_cast<size_t>(x.slot) * D.a.ckpt_stride)
                                         : reinterpret_cast<T*>(L + LA.H_in);
-      // norm outputs A / A2: stored in the activation set (store_norm), else recomputed into the
-      // shared Arec; G / M (recomputed) share the dM buffer
+      // norm outputs A / A2 and the MLP activation G / M: stored in the activation set (store_act),
+      // else recomputed (A / A2 into the shared Arec, G / M into the dM buffer)
       T* A = reinterpret_cast<T*>(sn ? L + LA.A : sc + BS.Arec);
       T* A2 = reinterpret_cast<T*>(sn ? L + LA.A2 : sc + BS.Arec);
-      T* Gt = dM;
+      T* Gt = sn ? reinterpret_cast<T*>(L + LA.G) : dM;
       T* QKV = reinterpret_cast<T*>(L + LA.QKV);
       T* O = reinterpret_cast<T*>(L + LA.O);
       float* LSE = reinterpret_cast<float*>(L + LA.LSE);
@@ -510,11 +510,11 @@ struct Exec {
       T* dH1 = dHbuf[(cur + 1) % 3];
       T* dHin = (li == 0) ? (k == 0 ? dHbuf[(cur + 2) % 3] : dstage_in) : dHbuf[(cur + 2) % 3];
       if (gpt) {
-        // dZ = (dH W2) * gelu'(Z); the epilogue also recomputes G = gelu(Z) for the fc2 wgrad
-        // fc1.b = column sums of dZ: fused into that epilogue (bf16), finished before `red` is reused
+        // dZ = (dH W2) * gelu'(Z); in the lean set the epilogue also recomputes G = gelu(Z) for the fc2
+        // wgrad; fc1.b = column sums of dZ: fused into that epilogue (bf16), finished before `red` is reused
         const bool fuse_b1 = sizeof(T) == 2 && Tn % 32 == 0 && f % 32 == 0 &&
                              static_cast<size_t>(Tn / 32) * f <= red_floats;
-        lin_dgrad(dH, Wm(D, p, pre + "fc2.w"), Tn, h, f, dZ, Z, Gt, fuse_b1 ? red : nullptr);
+        lin_dgrad(dH, Wm(D, p, pre + "fc2.w"), Tn, h, f, dZ, Z, sn ? nullptr : Gt, fuse_b1 ? red : nullptr);
         if (fuse_b1) colsum_finish(red, Tn / 32, f, G(D, p, pre + "fc1.b"), st);
         lin_wgrad(dH, Gt, Tn, h, f, G(D, p, pre + "fc2.w"));
         // fc2.b: fused into the norm backward that wrote dH (this stage), else a column sum here
@@ -532,7 +532,7 @@ struct Exec {
         lin_dgrad(dH1, Wm(D, p, pre + "proj.w"), Tn, h, h, dO);
         on_side(D, [&] { lin_wgrad(dH1, O, Tn, h, h, G(D, p, pre + "proj.w")); });
       } else {
-        swiglu_fwd<T>(Z, Gt, Tn, f, st);                                      // recompute M (into dM)
+        if (!sn) swiglu_fwd<T>(Z, Gt, Tn, f, st);                             // recompute M (into dM)
         lin_wgrad(dH, Gt, Tn, h, f, G(D, p, pre + "down.w"));
         lin_dgrad(dH, Wm(D, p, pre + "down.w"), Tn, h, f, dM);              // overwrites M (consumed)
         swiglu_bwd<T>(Z, dM, dZ, Tn, f, st);

@@ -14,7 +14,7 @@ namespace mario {
 size_t elt_size(const mario_model& m) { return m.dtype == MARIO_BF16 ? 2 : 4; }
 size_t tokens_per_micro(const mario_model& m) { return static_cast<size_t>(m.micro_batch) * m.seq_len; }
 
-LayerAct layer_act_layout(const mario_model& m, bool store_norm) {
+LayerAct layer_act_layout(const mario_model& m, bool store_act) {
   const size_t T = tokens_per_micro(m), E = elt_size(m), h = m.hidden, f = m.ffn_hidden;
   const size_t nh = m.n_heads;
   LayerAct L{};
@@ -28,20 +28,21 @@ LayerAct layer_act_layout(const mario_model& m, bool store_norm) {
   L.H1 = take(T * h * E);
   L.st2 = take(T * 2 * 4);
   L.Z = take(T * (m.family == MARIO_GPT ? f : 2 * f) * E);   // GPT: Z; LLaMA: GU = [gate | up]
-  L.A = take(store_norm ? T * h * E : 0);
-  L.A2 = take(store_norm ? T * h * E : 0);
+  L.A = take(store_act ? T * h * E : 0);
+  L.A2 = take(store_act ? T * h * E : 0);
+  L.G = take(store_act ? T * f * E : 0);
   L.bytes = o;
   return L;
 }
 
-LayerTrans layer_trans_layout(const mario_model& m, bool store_norm) {
+LayerTrans layer_trans_layout(const mario_model& m, bool store_act) {
   const size_t T = tokens_per_micro(m), E = elt_size(m), h = m.hidden, f = m.ffn_hidden;
   LayerTrans L{};
   size_t o = 0;
   auto take = [&](size_t bytes) { size_t r = o; o = align_up(o + bytes); return r; };
-  L.A = take(store_norm ? 0 : T * h * E);
-  L.A2 = take(store_norm ? 0 : T * h * E);
-  L.G = take(T * f * E);
+  L.A = take(store_act ? 0 : T * h * E);
+  L.A2 = take(store_act ? 0 : T * h * E);
+  L.G = take(store_act ? 0 : T * f * E);
   L.attn_pad = take(m.dtype == MARIO_BF16
                         ? flash_attn_pad_bytes(h / m.n_heads, m.micro_batch, m.seq_len, m.n_heads, 0) : 0);
   L.bytes = o;
@@ -83,21 +84,21 @@ HeadScratch head_scratch_layout(const mario_model& m) {
 
 size_t stage_input_bytes(const mario_model& m) { return align_up(tokens_per_micro(m) * m.hidden * elt_size(m)); }
 
-size_t act_set_bytes(const mario_model& m, int k, int K, bool store_norm) {
+size_t act_set_bytes(const mario_model& m, int k, int K, bool store_act) {
   const int lps = m.n_layers / K;
-  size_t b = layer_act_layout(m, store_norm).bytes * lps;
+  size_t b = layer_act_layout(m, store_act).bytes * lps;
   if (k == K - 1) b += head_act_layout(m).bytes;
   return b;
 }
 
-size_t cfw_work_bytes(const mario_model& m, int k, int K, bool store_norm) {
+size_t cfw_work_bytes(const mario_model& m, int k, int K, bool store_act) {
   // one layer's stored + transient tensors + the two running residual buffers (+ head)
-  size_t b = layer_act_layout(m, store_norm).bytes + layer_trans_layout(m, store_norm).bytes + 2 * stage_input_bytes(m);
+  size_t b = layer_act_layout(m, store_act).bytes + layer_trans_layout(m, store_act).bytes + 2 * stage_input_bytes(m);
   if (k == K - 1) b += head_act_layout(m).bytes;
   return b;
 }
 
-BwScratch bw_scratch_layout(const mario_model& m, bool store_norm) {
+BwScratch bw_scratch_layout(const mario_model& m, bool store_act) {
   const size_t T = tokens_per_micro(m), E = elt_size(m), h = m.hidden, f = m.ffn_hidden;
   BwScratch b{};
   size_t o = 0;
@@ -110,7 +111,7 @@ BwScratch bw_scratch_layout(const mario_model& m, bool store_norm) {
   b.dM = take(T * f * E);
   b.Dsc = take(static_cast<size_t>(m.n_heads) * T * 4);
   b.sort = take(T * 8 * 2);
-  b.Arec = take(store_norm ? 0 : T * h * E);
+  b.Arec = take(store_act ? 0 : T * h * E);
   for (int i = 0; i < 2; ++i) b.dH32[i] = take(m.dtype == MARIO_BF16 ? T * h * 4 : 0);
   b.attn_pad = take(m.dtype == MARIO_BF16
                         ? flash_attn_pad_bytes(h / m.n_heads, m.micro_batch, m.seq_len, m.n_heads, 1) : 0);
@@ -126,7 +127,7 @@ BwScratch bw_scratch_layout(const mario_model& m, bool store_norm) {
   return b;
 }
 
-size_t bw_scratch_bytes(const mario_model& m, bool store_norm) { return bw_scratch_layout(m, store_norm).bytes; }
+size_t bw_scratch_bytes(const mario_model& m, bool store_act) { return bw_scratch_layout(m, store_act).bytes; }
 
 size_t logits_bytes(const mario_model& m) { return head_scratch_layout(m).bytes; }
 

@@ -22,7 +22,7 @@ struct mario_plan {
   int level = MARIO_LEVEL_MARIO;
   uint64_t budget = 0;
   int unckpt_tail = 0;   // MARIO_LEVEL_BUDGET: devices S-k .. S-1 left un-checkpointed (A28)
-  bool store_norm = true;   // activation sets keep the norm outputs A, A2 (exec/layout.h); lean if the budget needs it
+  bool store_act = true;   // activation sets keep the norm outputs A, A2 (exec/layout.h); lean if the budget needs it
   int lps = 1;                       // layers per virtual stage
   mario::plan::Lists lists;
   std::vector<std::vector<mario_instr>> instrs;   // per device, exported IR

@@ -88,22 +88,29 @@ def test_bf16_parity(cfg):
 @pytest.mark.parametrize("cfg", [synth.TINY_GPT, TINY_L, synth.with_(synth.GPT3_1P3B, n_layers=2, micro_batch=1)],
                          ids=["gpt", "llama", "gpt-1.3b-width"])
 @pytest.mark.parametrize("dtype", ["f32", "bf16"])
-def test_lean_activation_set_bitwise(cfg, dtype, monkeypatch):
-    """The lean activation set (MARIO_STORE_NORM=0: the backward recomputes the norm outputs A, A2
-    from the stored (mean, rstd) with the forward's expression) gives bitwise the gradients of the
-    default set that stores them, and meets the oracle."""
+def test_lean_activation_set(cfg, dtype, monkeypatch):
+    """The lean activation set (MARIO_STORE_ACT=0: the backward recomputes the norm outputs A, A2 from
+    the stored (mean, rstd) with the forward's expression, and the MLP activation from Z / GU) meets
+    the oracle like the default set that stores them, and gives bitwise its gradients wherever the
+    recompute reads what the forward read: everywhere in fp32, and for LLaMA in bf16 (swiglu of the
+    bf16 GU both times). GPT in bf16 differs by design: the stored G = gelu(.) is the forward's, taken
+    from the fp32 pre-activation, the lean recompute takes it from the bf16 Z."""
     if dtype == "f32" and cfg.hidden > 64:
         pytest.skip("fp32 SIMT GEMMs at full width: slow and covered by the tiny cases")
     params = synth.make_weights(cfg)
     toks = synth.make_tokens(cfg, 4)
     stored = run_plan(cfg, 2, 4, "1f1b", "mario", dtype, params, toks)
-    monkeypatch.setenv("MARIO_STORE_NORM", "0")
-    assert not api.Plan(cfg, 2, 4, "1f1b", "mario", dtype=dtype).store_norm
+    monkeypatch.setenv("MARIO_STORE_ACT", "0")
+    assert not api.Plan(cfg, 2, 4, "1f1b", "mario", dtype=dtype).store_act
     lean = run_plan(cfg, 2, 4, "1f1b", "mario", dtype, params, toks)
-    assert stored[0] == lean[0] and np.array_equal(stored[2], lean[2])
+    if dtype == "f32" or cfg.family == "llama":
+        assert stored[0] == lean[0] and np.array_equal(stored[2], lean[2])
     if cfg.hidden <= 64:
         l_o, g_o = om.step(cfg, params if dtype == "f32" else rounded(params), toks, 4, np.float32)
-        check(lean[0], lean[1], l_o, g_o, 1e-4 if dtype == "f32" else 2e-2)
+        for loss, grads in (stored[:2], lean[:2]):
+            check(loss, grads, l_o, g_o, 1e-4 if dtype == "f32" else 2e-2)
+    else:   # full width: the oracle takes minutes here; the two sets agree within the bf16 bound
+        check(lean[0], lean[1], stored[0], {k: v.astype(np.float64) for k, v in stored[1].items()}, 2e-2)
 
 
 UNTIED_GPT = synth.with_(synth.TINY_GPT, tie_embeddings=False)

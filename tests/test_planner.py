@@ -218,21 +218,21 @@ def test_max_seq_len_boundary_and_order():
     assert api.max_seq_len(cfg, 8, 16, "base", 10 ** 6) == 0
 
 
-def test_store_norm_default_and_lean_fallback(monkeypatch):
+def test_store_act_default_and_lean_fallback(monkeypatch):
     """Activation sets keep the norm outputs A, A2 (+2 [T, h] per layer) unless the budget needs
     the lean set: a budget between the lean and the stored peak plans the lean set instead of
-    failing; MARIO_STORE_NORM forces either."""
+    failing; MARIO_STORE_ACT forces either."""
     cfg = synth.with_(synth.GPT3_1P3B, n_layers=8, micro_batch=1)
     full = Plan(cfg, 4, 8, "1f1b", "mario")
-    assert full.store_norm
-    monkeypatch.setenv("MARIO_STORE_NORM", "0")
+    assert full.store_act
+    monkeypatch.setenv("MARIO_STORE_ACT", "0")
     lean = Plan(cfg, 4, 8, "1f1b", "mario")
-    assert not lean.store_norm
-    monkeypatch.delenv("MARIO_STORE_NORM")
+    assert not lean.store_act
+    monkeypatch.delenv("MARIO_STORE_ACT")
     p_full, p_lean = max(full.simulate().peak_bytes), max(lean.simulate().peak_bytes)
     assert p_full > p_lean   # + A, A2 per stored layer, - the lean transients (Arec, CFW A/A2)
     mid = Plan(cfg, 4, 8, "1f1b", "mario", mem_budget=(p_full + p_lean) // 2)
-    assert not mid.store_norm and max(mid.simulate().peak_bytes) <= (p_full + p_lean) // 2
+    assert not mid.store_act and max(mid.simulate().peak_bytes) <= (p_full + p_lean) // 2
     assert mid.lists() == lean.lists()
     with pytest.raises(MarioError) as e:
         Plan(cfg, 4, 8, "1f1b", "mario", mem_budget=p_lean // 2)
