@@ -713,45 +713,6 @@ __global__ void __launch_bounds__(512) colsum_reduce_k(const float* __restrict__
   }
 }
 
-// The same reduction with 32 warps per CTA and every row load of a thread issued before any add:
-// warp w takes rows w, w + 32, ... (up to 32 * MAXR rows per batch), so a norm backward's 444 partial
-// rows are two round trips of 8 loads per thread (2 CTAs / SM: <= 32 registers) instead of the 16-warp
-// kernel's ~7 dependent ones
-// (7.9 us for its 3 x 444 x 2048 partials: latency, not bandwidth). Fixed order: per-thread row order,
-// then the 32 warp totals in order (deterministic; other bits than colsum_reduce_k's 8-way split).
-template <int MAXR>
-__global__ void __launch_bounds__(1024, 2) colsum_reduce32_k(const float* __restrict__ partial, int nblk, int n,
-                                                          float* out0, float* out1, float* out2) {
-  __shared__ float red[32][33];
-  const int k = blockIdx.y;
-  float* o = k == 0 ? out0 : (k == 1 ? out1 : out2);
-  if (!o) return;   // uniform over the block
-  const int w = threadIdx.x / 32, lane = threadIdx.x % 32;
-  const int c = blockIdx.x * 32 + lane;
-  float acc = 0.f;
-  if (c < n) {
-    const float* p = partial + static_cast<long>(k) * nblk * n + c;
-    for (int b0 = w; b0 < nblk; b0 += 32 * MAXR) {
-      float v[MAXR];
-#pragma unroll
-      for (int j = 0; j < MAXR; ++j) {
-        const int b = b0 + 32 * j;
-        v[j] = b < nblk ? __ldg(p + static_cast<long>(b) * n) : 0.f;
-      }
-#pragma unroll
-      for (int j = 0; j < MAXR; ++j) acc += v[j];
-    }
-  }
-  red[w][lane] = acc;
-  __syncthreads();
-  if (w == 0 && c < n) {
-    float t = 0.f;
-#pragma unroll
-    for (int i = 0; i < 32; ++i) t += red[i][lane];
-    o[c] += t;
-  }
-}
-
 // Block-per-row-tile norm backward (bf16, n = 8 * VPT * nthreads, nthreads % 32 == 0). Thread t owns
 // the 16-byte chunks t, t + nthreads, ... of every row (coalesced), R rows are in flight per
 // iteration, row sums are reduced warp -> shared memory -> block, and each thread keeps its
@@ -1531,9 +1492,9 @@ void norm_bwd_dx(const T* dy, const T* x, const float* stats, const float* g, co
 }
 void colsum_reduce(const float* partial, int nblk, int n, float* out0, float* out1, float* out2, cudaStream_t st) {
   const int arrays = out2 ? 3 : (out1 ? 2 : 1);
-  static const int v32 = getenv("MARIO_COLSUM_REDUCE") ? atoi(getenv("MARIO_COLSUM_REDUCE")) : 32;
-  if (v32 == 32) colsum_reduce32_k<8><<<dim3(cdiv(n, 32), arrays), 1024, 0, st>>>(partial, nblk, n, out0, out1, out2);
-  else colsum_reduce_k<<<dim3(cdiv(n, 32), arrays), 512, 0, st>>>(partial, nblk, n, out0, out1, out2);
+  // (a 32-warp variant with every row load issued first measured no faster in whole steps:
+  // profiles/r02/colsum_reduce_ab.txt)
+  colsum_reduce_k<<<dim3(cdiv(n, 32), arrays), 512, 0, st>>>(partial, nblk, n, out0, out1, out2);
   note_launch();
 }
 void colsum_finish(const float* partial, int nblk, int n, float* out, cudaStream_t st) {
