@@ -380,7 +380,7 @@ struct Exec {
         lin_fwd(A, Wm(D, p, pre + "qkv.w"), Tn, 3 * h, h, QKV, nullptr);
         rope<T>(QKV, mbs, s, nh, dh, m.rope_base, 0, st, rope_tab(D));
       }
-      attn_fwd<T>(QKV, O, LSE, mbs, s, nh, dh, st, LT.attn_pad ? trans + LT.attn_pad : nullptr);
+      attn_fwd<T>(QKV, O, LSE, mbs, s, nh, dh, st, LT.attn_pad_bytes ? trans + LT.attn_pad : nullptr);
       if (gpt) {
         lin_fwd(O, Wm(D, p, pre + "proj.w"), Tn, h, h, H1, Wf(D, p, pre + "proj.b"), Hin);
         layernorm_fwd<T>(H1, Wf(D, p, pre + "ln2.g"), Wf(D, p, pre + "ln2.b"), A2, st2, Tn, h, m.norm_eps, st);
@@ -549,7 +549,7 @@ struct Exec {
         on_side(D, [&] { lin_wgrad(dH1, O, Tn, h, h, G(D, p, pre + "o.w")); });
       }
       attn_bwd<T>(QKV, O, dO, LSE, dQKV, Dsc, mbs, s, nh, dh, st, BS.dS_bytes ? sc + BS.dS : nullptr, BS.dS_bytes,
-                  BS.attn_pad ? sc + BS.attn_pad : nullptr);
+                  BS.attn_pad_bytes ? sc + BS.attn_pad : nullptr);
       if (!gpt) rope<T>(dQKV, mbs, s, nh, dh, m.rope_base, 1, st, rope_tab(D));
       if (!sn) {
         join_side(D);   // the fc1 / MLP-input wgrad read A2 (Arec), which the recompute below overwrites

@@ -43,8 +43,8 @@ LayerTrans layer_trans_layout(const mario_model& m, bool store_act) {
   L.A = take(store_act ? 0 : T * h * E);
   L.A2 = take(store_act ? 0 : T * h * E);
   L.G = take(store_act ? 0 : T * f * E);
-  L.attn_pad = take(m.dtype == MARIO_BF16
-                        ? flash_attn_pad_bytes(h / m.n_heads, m.micro_batch, m.seq_len, m.n_heads, 0) : 0);
+  L.attn_pad_bytes = m.dtype == MARIO_BF16 ? flash_attn_pad_bytes(h / m.n_heads, m.micro_batch, m.seq_len, m.n_heads, 0) : 0;
+  L.attn_pad = take(L.attn_pad_bytes);
   L.bytes = o;
   return L;
 }
@@ -113,8 +113,8 @@ BwScratch bw_scratch_layout(const mario_model& m, bool store_act) {
   b.sort = take(T * 8 * 2);
   b.Arec = take(store_act ? 0 : T * h * E);
   for (int i = 0; i < 2; ++i) b.dH32[i] = take(m.dtype == MARIO_BF16 ? T * h * 4 : 0);
-  b.attn_pad = take(m.dtype == MARIO_BF16
-                        ? flash_attn_pad_bytes(h / m.n_heads, m.micro_batch, m.seq_len, m.n_heads, 1) : 0);
+  b.attn_pad_bytes = m.dtype == MARIO_BF16 ? flash_attn_pad_bytes(h / m.n_heads, m.micro_batch, m.seq_len, m.n_heads, 1) : 0;
+  b.attn_pad = take(b.attn_pad_bytes);
   // the attention backward's dS image (fa_bwd_dq_img: dQ from the stored dS, no S/dP recompute);
   // only where it stays small next to the rest of the scratch (not at s = 16384)
   b.dS_bytes = 0;

@@ -31,7 +31,8 @@ LayerAct layer_act_layout(const mario_model& m, bool store_act);
 // only).
 struct LayerTrans {
   size_t A, A2, G;
-  size_t attn_pad;   // padded-head-dim attention workspace (bf16, dh not 64 / 128), else 0 bytes
+  size_t attn_pad, attn_pad_bytes;   // padded-head-dim attention workspace (bf16, dh not 64 / 128), else 0 bytes
+                                     // (test the size: with store_act the offset itself can be 0)
   size_t bytes;
 };
 LayerTrans layer_trans_layout(const mario_model& m, bool store_act);
@@ -65,7 +66,7 @@ struct BwScratch {
   size_t dH[3], dA, dQKV, dO, dZ, dM, Dsc, sort;   // dM doubles as the G/M recompute buffer
   size_t Arec;      // lean set: the recomputed norm output (0 bytes with store_act)
   size_t dH32[2];   // bf16 mode: the fp32 residual-gradient stream (reading A30); 0 bytes in fp32 mode
-  size_t attn_pad;  // padded-head-dim attention backward workspace (bf16, dh not 64 / 128), else 0 bytes
+  size_t attn_pad, attn_pad_bytes;  // padded-head-dim attention backward workspace (bf16, dh not 64 / 128), else 0 bytes
   size_t dS, dS_bytes;   // attention dS image (bf16, when the shape allows it and it is <= 1 GiB; else 0 bytes)
   size_t bytes;
 };
