@@ -251,7 +251,8 @@ struct Exec {
   // D[M,N] = A[M,K] . B[N,K]^T  (see kernels.h); bf16 tcgen05 or fp32 SIMT by dtype.
   void gemm(const T* A, int lda, int a_mn, const T* B, int ldb, int b_mn, int M, int N, int K, void* Dp, int ldd,
             bool out_f32, float beta, const float* bias = nullptr, const T* resid = nullptr, T* D2 = nullptr,
-            const T* aux = nullptr, bool d2_from_aux = false, float* colsum_part = nullptr) {
+            const T* aux = nullptr, bool d2_from_aux = false, float* colsum_part = nullptr, const T* dot = nullptr,
+            float* dot_out = nullptr, int dot_seg = 0) {
     if constexpr (sizeof(T) == 2) {
       GemmArgs g;
       g.A = A; g.lda = lda; g.a_mn = a_mn; g.B = B; g.ldb = ldb; g.b_mn = b_mn; g.M = M; g.N = N; g.K = K;
@@ -261,6 +262,7 @@ struct Exec {
       g.ep.residual = resid; g.ep.ld_res = ldd; g.ep.d2_bf16 = D2; g.ep.aux = aux; g.ep.ld_aux = ldd;
       g.ep.d2_from_aux = d2_from_aux ? 1 : 0;
       g.ep.colsum_part = colsum_part;
+      g.ep.dot = dot; g.ep.ld_dot = ldd; g.ep.dot_out = dot_out; g.ep.dot_seg = dot_seg; g.ep.dot_stride = M;
       g.persistent = gemm_persistent;
       CU(gemm_bf16(g, st));
     } else {
@@ -270,6 +272,12 @@ struct Exec {
       g.ld_res = ldd; g.D2 = D2; g.aux = aux; g.ld_aux = ldd; g.d2_from_aux = d2_from_aux ? 1 : 0;
       CU(gemm_f32(g, st));
     }
+  }
+  // dX[T,in] = dY W with, per head of `seg` columns, Dd[head][t] = sum bf16(dX[t, head]) * X[t, head]
+  // fused into the epilogue (bf16: the attention backward's D = rowsum(dO o O))
+  void lin_dgrad_dot(const T* dY, const T* W, int Tn, int out, int in, T* dX, const T* X, float* Dd, int seg) {
+    gemm(dY, out, 0, W, in, 1, Tn, in, out, dX, in, false, 0.f, nullptr, nullptr, nullptr, nullptr, false, nullptr, X,
+         Dd, seg);
   }
   // Y[T,out] = X W^T (+bias, +resid, D2 = gelu)
   void lin_fwd(const T* X, const T* W, int Tn, int out, int in, T* Y, const float* bias, const T* resid = nullptr,
@@ -453,6 +461,10 @@ struct Exec {
     T* dZ = reinterpret_cast<T*>(sc + BS.dZ);
     T* dM = reinterpret_cast<T*>(sc + BS.dM);
     float* Dsc = reinterpret_cast<float*>(sc + BS.Dsc);
+    // the attention backward's D = rowsum(dO o O) per head from the dO GEMM's epilogue (bf16, head dims
+    // the unpadded tcgen05 backward takes: the padded path computes D on the unpadded heads itself)
+    static const bool fuse_D_env = getenv("MARIO_FUSE_D") ? atoi(getenv("MARIO_FUSE_D")) != 0 : true;
+    const bool fuse_D = fuse_D_env && sizeof(T) == 2 && (dh == 64 || dh == 128);
     // bf16 mode (reading A30): the residual-stream gradient dH is carried in fp32 between layers
     // (dH32, two buffers: LN2 reads [0] writes [1], LN1 reads [1] writes [0]); the bf16 dH buffers
     // are the operand copies of the GEMMs. nullptr = the bf16 dH is exact (a received message).
@@ -529,7 +541,8 @@ struct Exec {
         else
           norm_bwd<T>(dA, H1, st2, Wf(D, p, pre + "ln2.g"), dH, dH1, Tn, h, 0, G(D, p, pre + "ln2.g"),
                       G(D, p, pre + "ln2.b"), G(D, p, pre + "proj.b"), red, red_floats, st);
-        lin_dgrad(dH1, Wm(D, p, pre + "proj.w"), Tn, h, h, dO);
+        if (fuse_D) lin_dgrad_dot(dH1, Wm(D, p, pre + "proj.w"), Tn, h, h, dO, O, Dsc, dh);
+        else lin_dgrad(dH1, Wm(D, p, pre + "proj.w"), Tn, h, h, dO);
         on_side(D, [&] { lin_wgrad(dH1, O, Tn, h, h, G(D, p, pre + "proj.w")); });
       } else {
         if (!sn) swiglu_fwd<T>(Z, Gt, Tn, f, st);                             // recompute M (into dM)
@@ -545,10 +558,12 @@ struct Exec {
         else
           norm_bwd<T>(dA, H1, st2, Wf(D, p, pre + "n2.g"), dH, dH1, Tn, h, 1, G(D, p, pre + "n2.g"), nullptr, nullptr,
                       red, red_floats, st);
-        lin_dgrad(dH1, Wm(D, p, pre + "o.w"), Tn, h, h, dO);
+        if (fuse_D) lin_dgrad_dot(dH1, Wm(D, p, pre + "o.w"), Tn, h, h, dO, O, Dsc, dh);
+        else lin_dgrad(dH1, Wm(D, p, pre + "o.w"), Tn, h, h, dO);
         on_side(D, [&] { lin_wgrad(dH1, O, Tn, h, h, G(D, p, pre + "o.w")); });
       }
-      attn_bwd<T>(QKV, O, dO, LSE, dQKV, Dsc, mbs, s, nh, dh, st, BS.dS_bytes ? sc + BS.dS : nullptr, BS.dS_bytes,
+      // O = nullptr: D = rowsum(dO o O) is already in Dsc (fused into the dO GEMM above)
+      attn_bwd<T>(QKV, fuse_D ? nullptr : O, dO, LSE, dQKV, Dsc, mbs, s, nh, dh, st, BS.dS_bytes ? sc + BS.dS : nullptr, BS.dS_bytes,
                   BS.attn_pad_bytes ? sc + BS.attn_pad : nullptr);
       if (!gpt) rope<T>(dQKV, mbs, s, nh, dh, m.rope_base, 1, st, rope_tab(D));
       if (!sn) {

@@ -462,7 +462,7 @@ template <int D>
 void launch_bwd(const bf16* qkv, const bf16* O, const bf16* dO, const float* lse, bf16* dqkv, float* Dd, int B, int s,
                 int nh, cudaStream_t st, void* ds_ws, size_t ds_ws_bytes) {
   const long Ttok = static_cast<long>(B) * s;
-  {
+  if (O) {   // O == nullptr: the caller already wrote D = rowsum(dO o O) into Dd
     const long thr = Ttok * nh * (D / 8);
     const int grid = static_cast<int>((thr + 255) / 256);
     if (D == 128) fa_bwd_dot_v8_k<16><<<grid, 256, 0, st>>>(O, dO, Dd, Ttok, nh);

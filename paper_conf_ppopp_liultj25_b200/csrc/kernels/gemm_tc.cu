@@ -173,7 +173,8 @@ __device__ __forceinline__ bool epilogue_vec_ok(const GemmEpilogue& ep) {
   auto al = [](const void* p) { return (reinterpret_cast<uintptr_t>(p) & 15) == 0; };
   return (ep.ldd % 8) == 0 && (ep.out_f32 ? al(ep.d_f32) : al(ep.d_bf16)) && (!ep.d2_bf16 || al(ep.d2_bf16)) &&
          (!ep.residual || ((ep.ld_res % 8) == 0 && al(ep.residual))) &&
-         (!ep.aux || ((ep.ld_aux % 8) == 0 && al(ep.aux))) && (!ep.bias || al(ep.bias));
+         (!ep.aux || ((ep.ld_aux % 8) == 0 && al(ep.aux))) && (!ep.bias || al(ep.bias)) &&
+         (!ep.dot || ((ep.ld_dot % 8) == 0 && al(ep.dot)));
 }
 __device__ __forceinline__ void sts128(uint8_t* p, const uint4& v) {
   asm volatile("st.shared.v4.u32 [%0], {%1, %2, %3, %4};" :: "r"(smem_u32(p)), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w)
@@ -222,13 +223,15 @@ __device__ __forceinline__ void cp_async16(void* dst, const void* src, bool vali
                  : "memory");
   }
 }
-template <bool EF = false>
+// DOT: the block of the fused row dot's input (ep.dot) instead of the aux / residual input (a separate
+// instantiation: a three-way pick in the shared one made the register-tight GeLU' epilogue spill)
+template <bool EF = false, bool DOT = false>
 __device__ __forceinline__ void epi_prefetch(const GemmEpilogue& ep, bool vec_ok, int rbase, int lane, int col0, int M,
                                              int N, EpiPrefetch& pf) {
   if (col0 < 0 || col0 >= N || !vec_ok || col0 + 32 > N) return;
-  const __nv_bfloat16* base = ep.aux ? ep.aux : ep.residual;
+  const __nv_bfloat16* base = DOT ? ep.dot : (ep.aux ? ep.aux : ep.residual);
   if (!base) return;
-  const int ld = ep.aux ? ep.ld_aux : ep.ld_res;
+  const int ld = DOT ? ep.ld_dot : (ep.aux ? ep.ld_aux : ep.ld_res);
 #pragma unroll
   for (int it = 0; it < 4; ++it) {
     const int rr = it * 8 + lane / 4, ch = lane % 4;
@@ -289,7 +292,7 @@ __device__ __forceinline__ void store_block_bf16(__nv_bfloat16* base, int ld, in
 template <int EPI>
 __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool vec_ok, const uint32_t (&r)[32],
                                                     int rbase, int lane, int col0, int M, int N, uint8_t* sw,
-                                                    EpiPrefetch& pf, int next_col0) {
+                                                    EpiPrefetch& pf, int next_col0, float& dacc) {
   if (col0 >= N) return;
   if (!vec_ok || col0 + 32 > N) {   // warp-uniform: ragged column block or unaligned pitches
     epilogue_chunk<EPI == 2>(ep, r, rbase + lane, col0, rbase + lane < M, N);
@@ -321,6 +324,15 @@ __device__ __forceinline__ void epilogue_chunk_warp(const GemmEpilogue& ep, bool
       if (MARIO_EPI_PREFETCH && EPI != 2) epi_prefetch(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
 #pragma unroll
       for (int j = 0; j < 32; ++j) v[j] += rr[j];
+    }
+  }
+  if constexpr (EPI == 0) {   // row dot of the bf16-rounded output with ep.dot (no residual / aux here)
+    if (ep.dot_out) {
+      float xx[32];
+      load_block_bf16(pf, lane, xx);
+      if (MARIO_EPI_PREFETCH) epi_prefetch<false, true>(ep, vec_ok, rbase, lane, next_col0, M, N, pf);
+#pragma unroll
+      for (int j = 0; j < 32; ++j) dacc = fmaf(__bfloat162float(__float2bfloat16_rn(v[j])), xx[j], dacc);
     }
   }
   if constexpr (EPI == 2) {
@@ -484,18 +496,29 @@ gemm_bf16_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_consta
       const int m0 = tm * BM, n0 = tn * BN;
       const int rbase = m0 + quarter * 32;
       EpiPrefetch pf{sw + 2048};
-      if (MARIO_EPI_PREFETCH && !ep.out_f32) epi_prefetch(ep, vec_ok, rbase, lane, n0, M, N, pf);
+      if (MARIO_EPI_PREFETCH && !ep.out_f32) {
+        if (ep.dot_out && !ep.aux) epi_prefetch<false, true>(ep, vec_ok, rbase, lane, n0, M, N, pf);
+        else epi_prefetch(ep, vec_ok, rbase, lane, n0, M, N, pf);
+      }
       mbar_wait(&tfull[acc], acc_ph);
       tc_fence_after();
+      float dacc = 0.f;   // fused row dot (ep.dot_out) over the current segment
 #pragma unroll 1
       for (int c = 0; c < BN / 32; ++c) {
         uint32_t r[32];
         tmem_ld_32x32b_x32(tmem_base + acc * BN + c * 32 + (static_cast<uint32_t>(quarter * 32) << 16), r);
         tmem_ld_wait();
         const int nxt = c + 1 < BN / 32 ? n0 + (c + 1) * 32 : -1;
-        if (ep.out_f32) epilogue_chunk_warp<2>(ep, vec_ok, r, rbase, lane, n0 + c * 32, M, N, sw, pf, nxt);
-        else if (ep.aux) epilogue_chunk_warp<1>(ep, vec_ok, r, rbase, lane, n0 + c * 32, M, N, sw, pf, nxt);
-        else epilogue_chunk_warp<0>(ep, vec_ok, r, rbase, lane, n0 + c * 32, M, N, sw, pf, nxt);
+        if (ep.out_f32) epilogue_chunk_warp<2>(ep, vec_ok, r, rbase, lane, n0 + c * 32, M, N, sw, pf, nxt, dacc);
+        else if (ep.aux) epilogue_chunk_warp<1>(ep, vec_ok, r, rbase, lane, n0 + c * 32, M, N, sw, pf, nxt, dacc);
+        else {
+          epilogue_chunk_warp<0>(ep, vec_ok, r, rbase, lane, n0 + c * 32, M, N, sw, pf, nxt, dacc);
+          if (ep.dot_out && (n0 + c * 32 + 32) % ep.dot_seg == 0) {
+            if (rbase + lane < M)
+              ep.dot_out[static_cast<long>((n0 + c * 32) / ep.dot_seg) * ep.dot_stride + rbase + lane] = dacc;
+            dacc = 0.f;
+          }
+        }
       }
       tc_fence_before();
       mbar_arrive(&tempty[acc]);
@@ -711,7 +734,10 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
       const int m0 = tm * 256 + 128 * rank, n0 = tn * BNP;
       const int rbase = m0 + quarter * 32;
       EpiPrefetch pf{sw + 2048};
-      if (MARIO_EPI_PREFETCH && EPI != 2 && !(skon && u.kb0 != 0)) epi_prefetch<EPI == 1 && MARIO_EPI_EF != 0>(ep, vec_ok, rbase, lane, n0 + half * (BNP / 2), M, N, pf);
+      if (MARIO_EPI_PREFETCH && EPI != 2 && !(skon && u.kb0 != 0)) {
+        if (EPI == 0 && ep.dot_out) epi_prefetch<false, true>(ep, vec_ok, rbase, lane, n0 + half * (BNP / 2), M, N, pf);
+        else epi_prefetch<EPI == 1 && MARIO_EPI_EF != 0>(ep, vec_ok, rbase, lane, n0 + half * (BNP / 2), M, N, pf);
+      }
       if (SK && sk.sleep_ns) { while (!mbar_test(&tfull[acc], acc_ph)) __nanosleep(sk.sleep_ns); }
       else mbar_wait(&tfull[acc], acc_ph);
       tc_fence_after();
@@ -744,6 +770,7 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
                 while (ld_acquire(&sk.flags[q * 2 + rank]) == 0) __nanosleep(64);
           asm volatile("bar.sync 1, 256;" ::: "memory");
         }
+        float dacc = 0.f;   // fused row dot (ep.dot_out) over the current segment
 #pragma unroll 1
         for (int c = 0; c < BNP / 64; ++c) {
           uint32_t r[32];
@@ -763,7 +790,12 @@ gemm_bf16_tc2_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_const
             }
           }
           epilogue_chunk_warp<EPI>(ep, vec_ok, r, rbase, lane, n0 + col, M, N, sw, pf,
-                              c + 1 < BNP / 64 ? n0 + col + 32 : -1);
+                              c + 1 < BNP / 64 ? n0 + col + 32 : -1, dacc);
+          if (EPI == 0 && ep.dot_out && (n0 + col + 32) % ep.dot_seg == 0) {   // a segment (head) complete
+            if (rbase + lane < M)
+              ep.dot_out[static_cast<long>((n0 + col) / ep.dot_seg) * ep.dot_stride + rbase + lane] = dacc;
+            dacc = 0.f;
+          }
         }
         if (q1 > pair + 1) {
           asm volatile("bar.sync 1, 256;" ::: "memory");
@@ -1017,6 +1049,13 @@ cudaError_t gemm_bf16(const GemmArgs& g0, cudaStream_t st) {
        (g.ep.d2_bf16 && !al16(g.ep.d2_bf16)) || (g.ep.residual && ((g.ep.ld_res % 8) || !al16(g.ep.residual))) ||
        (g.ep.aux && ((g.ep.ld_aux % 8) || !al16(g.ep.aux))) || (g.ep.bias && !al16(g.ep.bias)))) {
     fprintf(stderr, "[mario] gemm_bf16: fused column sums need bf16 output, M %% 32 == N %% 32 == 0, aligned D\n");
+    return cudaErrorInvalidValue;
+  }
+  if (g.ep.dot_out &&
+      (g.ep.out_f32 || g.ep.aux || g.ep.residual || !g.ep.dot || g.ep.dot_seg <= 0 || (g.ep.dot_seg % 32) ||
+       (g.N % g.ep.dot_seg) || (g.N % 32) || !g.ep.d_bf16 || (g.ep.ldd % 8) || (g.ep.ld_dot % 8) ||
+       !al16(g.ep.d_bf16) || !al16(g.ep.dot) || (g.ep.bias && !al16(g.ep.bias)))) {
+    fprintf(stderr, "[mario] gemm_bf16: fused row dots need bf16 output without aux / residual, 32 | seg | N\n");
     return cudaErrorInvalidValue;
   }
   const int sms = device_sm_count();

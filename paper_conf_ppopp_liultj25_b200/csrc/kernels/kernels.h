@@ -26,6 +26,13 @@ struct GemmEpilogue {
   // row block i = sum over rows [32 i, 32 i + 32) in row order. Requires bf16 output, M % 32 == 0,
   // N % 32 == 0 and 16-byte aligned pitches (gemm_bf16 returns cudaErrorInvalidValue otherwise).
   float* colsum_part = nullptr;
+  // optional fused per-segment row dots of the bf16 output D with a bf16 input X (the attention
+  // backward's D = rowsum(dO o O) per head, taken in the dO-producing GEMM): for every row r and
+  // segment j of dot_seg columns, dot_out[j * dot_stride + r] = sum over the segment of bf16(D) * X.
+  // Requires bf16 output without aux / residual, dot_seg % 32 == 0, N % dot_seg == 0, N % 32 == 0,
+  // 16-byte aligned pitches (gemm_bf16 returns cudaErrorInvalidValue otherwise).
+  const __nv_bfloat16* dot = nullptr; int ld_dot = 0;
+  float* dot_out = nullptr; int dot_seg = 0; long dot_stride = 0;
 };
 
 struct GemmArgs {

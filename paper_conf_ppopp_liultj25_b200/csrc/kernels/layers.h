@@ -105,6 +105,7 @@ bool flash_attn_supported(int dh);
 // on them over zero-padded copies (attn_mma.cu); without it such head dims take mma.sync.
 void flash_attn_fwd(const __nv_bfloat16* qkv, __nv_bfloat16* O, float* lse, int B, int s, int nh, int dh, cudaStream_t st,
                     void* pad_ws = nullptr);
+// O == nullptr (head dims 16/32/64/128, no padding): Dd already holds D = rowsum(dO o O) per head
 void flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* O, const __nv_bfloat16* dO, const float* lse,
                     __nv_bfloat16* dqkv, float* Dd, int B, int s, int nh, int dh, cudaStream_t st,
                     void* ds_ws = nullptr, size_t ds_ws_bytes = 0, void* pad_ws = nullptr);
