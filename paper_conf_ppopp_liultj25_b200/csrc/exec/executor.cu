@@ -562,16 +562,21 @@ struct Exec {
         else lin_dgrad(dH1, Wm(D, p, pre + "o.w"), Tn, h, h, dO);
         on_side(D, [&] { lin_wgrad(dH1, O, Tn, h, h, G(D, p, pre + "o.w")); });
       }
-      // O = nullptr: D = rowsum(dO o O) is already in Dsc (fused into the dO GEMM above)
-      attn_bwd<T>(QKV, fuse_D ? nullptr : O, dO, LSE, dQKV, Dsc, mbs, s, nh, dh, st, BS.dS_bytes ? sc + BS.dS : nullptr, BS.dS_bytes,
-                  BS.attn_pad_bytes ? sc + BS.attn_pad : nullptr);
+      // O = nullptr: D = rowsum(dO o O) is already in Dsc (fused into the dO GEMM above). GPT: the
+      // attention kernels may also leave the qkv-bias column partials per 32 tokens in `red`
+      static const bool fuse_qkvb = getenv("MARIO_FUSE_QKVB") ? atoi(getenv("MARIO_FUSE_QKVB")) != 0 : true;
+      const bool bp_fit = fuse_qkvb && gpt && Tn % 32 == 0 && static_cast<size_t>(Tn / 32) * 3 * h <= red_floats;
+      bool qkvb_part = false;
+      attn_bwd<T>(QKV, fuse_D ? nullptr : O, dO, LSE, dQKV, Dsc, mbs, s, nh, dh, st, BS.dS_bytes ? sc + BS.dS : nullptr,
+                  BS.dS_bytes, BS.attn_pad_bytes ? sc + BS.attn_pad : nullptr, bp_fit ? red : nullptr, &qkvb_part);
       if (!gpt) rope<T>(dQKV, mbs, s, nh, dh, m.rope_base, 1, st, rope_tab(D));
       if (!sn) {
         join_side(D);   // the fc1 / MLP-input wgrad read A2 (Arec), which the recompute below overwrites
         if (gpt) norm_recompute<T>(Hin, Wf(D, p, pre + "ln1.g"), Wf(D, p, pre + "ln1.b"), A, st1, Tn, h, m.norm_eps, 0, st);
         else norm_recompute<T>(Hin, Wf(D, p, pre + "n1.g"), nullptr, A, st1, Tn, h, m.norm_eps, 1, st);
       }
-      if (gpt) colsum<T>(dQKV, nullptr, nullptr, Tn, 3 * h, 3 * h, 0, G(D, p, pre + "qkv.b"), nullptr, red, st);
+      if (gpt && qkvb_part) colsum_finish(red, Tn / 32, 3 * h, G(D, p, pre + "qkv.b"), st);
+      else if (gpt) colsum<T>(dQKV, nullptr, nullptr, Tn, 3 * h, 3 * h, 0, G(D, p, pre + "qkv.b"), nullptr, red, st);
       lin_dgrad(dQKV, Wm(D, p, pre + "qkv.w"), Tn, 3 * h, h, dA);
       on_side(D, [&] { lin_wgrad(dQKV, A, Tn, 3 * h, h, G(D, p, pre + "qkv.w")); });
       if constexpr (r32) {

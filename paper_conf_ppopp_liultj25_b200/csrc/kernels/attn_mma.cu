@@ -460,7 +460,8 @@ void launch_fwd(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, cuda
 }
 template <int D>
 void launch_bwd(const bf16* qkv, const bf16* O, const bf16* dO, const float* lse, bf16* dqkv, float* Dd, int B, int s,
-                int nh, cudaStream_t st, void* ds_ws, size_t ds_ws_bytes) {
+                int nh, cudaStream_t st, void* ds_ws, size_t ds_ws_bytes, float* bpart = nullptr,
+                bool* bpart_done = nullptr) {
   const long Ttok = static_cast<long>(B) * s;
   if (O) {   // O == nullptr: the caller already wrote D = rowsum(dO o O) into Dd
     const long thr = Ttok * nh * (D / 8);
@@ -474,7 +475,8 @@ void launch_bwd(const bf16* qkv, const bf16* O, const bf16* dO, const float* lse
   if (g_attn_variant != 0) {   // tcgen05 backward (attn_tc.cu) when supported
     const double fl = 8.0 * B * nh * D * (static_cast<double>(s) * (s + 1) / 2);
     const int tok = kstats_begin(K_ATTN_BWD, fl, 0.0, st);
-    const bool ok = flash_attn_bwd_tc(qkv, dO, lse, Dd, dqkv, B, s, nh, D, ds_ws, ds_ws_bytes, st);
+    const bool ok = flash_attn_bwd_tc(qkv, dO, lse, Dd, dqkv, B, s, nh, D, ds_ws, ds_ws_bytes, st, 0.f, bpart,
+                                      bpart_done);
     kstats_end(tok, st);
     if (ok) { note_launch(); return; }
   }
@@ -614,8 +616,10 @@ void flash_attn_fwd(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, 
 }
 
 void flash_attn_bwd(const bf16* qkv, const bf16* O, const bf16* dO, const float* lse, bf16* dqkv, float* Dd, int B,
-                    int s, int nh, int dh, cudaStream_t st, void* ds_ws, size_t ds_ws_bytes, void* pad_ws) {
+                    int s, int nh, int dh, cudaStream_t st, void* ds_ws, size_t ds_ws_bytes, void* pad_ws, float* bpart,
+                    bool* bpart_done) {
   (void)ds_ws; (void)ds_ws_bytes;
+  if (bpart_done) *bpart_done = false;
   if (pad_ws && needs_pad(dh) && g_attn_variant != 0 && flash_attn_pad_bytes(dh, B, s, nh, 1)) {
     const int Dp = padded_dh(dh);
     const long T = static_cast<long>(B) * s;
@@ -644,9 +648,9 @@ void flash_attn_bwd(const bf16* qkv, const bf16* O, const bf16* dO, const float*
   switch (dh) {
     case 16: launch_bwd<16>(qkv, O, dO, lse, dqkv, Dd, B, s, nh, st, ds_ws, ds_ws_bytes); break;
     case 32: launch_bwd<32>(qkv, O, dO, lse, dqkv, Dd, B, s, nh, st, ds_ws, ds_ws_bytes); break;
-    case 64: launch_bwd<64>(qkv, O, dO, lse, dqkv, Dd, B, s, nh, st, ds_ws, ds_ws_bytes); break;
+    case 64: launch_bwd<64>(qkv, O, dO, lse, dqkv, Dd, B, s, nh, st, ds_ws, ds_ws_bytes, bpart, bpart_done); break;
     case 80: launch_bwd<80>(qkv, O, dO, lse, dqkv, Dd, B, s, nh, st, ds_ws, ds_ws_bytes); break;
-    default: launch_bwd<128>(qkv, O, dO, lse, dqkv, Dd, B, s, nh, st, ds_ws, ds_ws_bytes); break;
+    default: launch_bwd<128>(qkv, O, dO, lse, dqkv, Dd, B, s, nh, st, ds_ws, ds_ws_bytes, bpart, bpart_done); break;
   }
 }
 

@@ -1268,7 +1268,7 @@ struct SmemI {
 template <int DH>
 __global__ void __launch_bounds__(kThreadsI, 1)
 fa_bwd_dq_img(const __grid_constant__ CUtensorMap tm_qkv64, const uint8_t* __restrict__ dsimg, bf16* dqkv, int B, int s,
-              int nh, int l2hint, float qk_scale) {
+              int nh, int l2hint, float qk_scale, float* bpart) {
   using SI = SmemI<DH>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -1369,15 +1369,38 @@ fa_bwd_dq_img(const __grid_constant__ CUtensorMap tm_qkv64, const uint8_t* __res
           __syncwarp();
           if (lane == 0) mbar_arrive(&acc_empty[n & 1]);
         }
+        float cs[32];
 #pragma unroll
         for (int e = 0; e < 4; ++e) {
           uint4 u;
           __nv_bfloat162* hq = reinterpret_cast<__nv_bfloat162*>(&u);
 #pragma unroll
-          for (int f = 0; f < 4; ++f)
+          for (int f = 0; f < 4; ++f) {
             hq[f] = __floats2bfloat162_rn(__uint_as_float(rq[8 * e + 2 * f]) * scale,
                                           __uint_as_float(rq[8 * e + 2 * f + 1]) * scale);
+            const float2 back = __bfloat1622float2(hq[f]);
+            cs[8 * e + 2 * f] = back.x;
+            cs[8 * e + 2 * f + 1] = back.y;
+          }
           *reinterpret_cast<uint4*>(qrow + c + 8 * e) = u;
+        }
+        if (bpart) {
+          // column sums of this warp's 32 stored rows x 32 columns (the q-bias gradient partial of its
+          // 32-row block): a transposing butterfly, 16 + 8 + 4 + 2 + 1 shuffles; at each step a lane
+          // keeps the half of its columns its lane bit selects and adds the partner's copy of that half,
+          // so lane l ends with column l (fixed order: deterministic). The kernel is DRAM-bound on the
+          // image, so these shuffles run in its shadow.
+#pragma unroll
+          for (int o = 16; o >= 1; o >>= 1) {
+            const bool up = (lane & o) != 0;
+#pragma unroll
+            for (int j = 0; j < o; ++j) {
+              const float send = up ? cs[j] : cs[j + o];
+              const float keep = up ? cs[j + o] : cs[j];
+              cs[j] = keep + __shfl_xor_sync(0xffffffffu, send, o);
+            }
+          }
+          bpart[((static_cast<long>(b) * s + qb * kRows) / 32 + quarter) * (3 * h) + head * DH + c + lane] = cs[0];
         }
       }
     }
@@ -1420,7 +1443,7 @@ template <int DH>
 __global__ void __launch_bounds__(kThreadsB, 1)
 fa_bwd_dkdv_n128(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__ CUtensorMap tm_do128,
                  const __grid_constant__ CUtensorMap tm_dqkv, const float* lse, const float* Dd, bf16* dqkv, int B,
-                 int s, int nh, uint8_t* dsimg, float qk_scale) {
+                 int s, int nh, uint8_t* dsimg, float qk_scale, float* bpart) {
   using SN = SmemN<DH>;
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -1663,6 +1686,26 @@ fa_bwd_dkdv_n128(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_con
       }
       bulk_commit_wait_read();
     }
+    if (bpart) {
+      // column sums of the staged bf16 dV / dK tiles (exactly what is stored), per 32-row block in
+      // row order: bpart[(token / 32)][3h] gets the qkv-bias gradient partials of the k and v columns
+      // (read alongside the TMA store: both only read the staging tiles)
+      const int t = threadIdx.x - 64;
+      if (t < 2 * DH) {
+        const bool isK = t >= DH;
+        const int c = isK ? t - DH : t, ch = (c % 64) / 8, e = c % 8;
+        const uint8_t* tile = isK ? stK(c / 64) : stV(c / 64);
+        float* dst = bpart + ((static_cast<long>(b) * s + kt * kRows) / 32) * (3 * h) + (isK ? h : 2 * h) + head * DH + c;
+#pragma unroll 1
+        for (int q = 0; q < kRows / 32; ++q) {
+          float acc = 0.f;
+#pragma unroll 8
+          for (int r = 32 * q; r < 32 * q + 32; ++r)
+            acc += __bfloat162float(*reinterpret_cast<const bf16*>(tile + r * 128 + ((ch ^ (r & 7)) << 4) + e * 2));
+          dst[static_cast<long>(q) * (3 * h)] = acc;
+        }
+      }
+    }
   }
   tc_fence_before();
   __syncthreads();
@@ -1903,7 +1946,8 @@ int g_attn_dq_pers = 1;   // MARIO_ATTN_DQ_PERS=0 selects the one-item-per-CTA d
 
 template <int DH>
 bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, bf16* dqkv, int B, int s, int nh,
-            uint8_t* dsimg, cudaStream_t st, float qk_scale) {
+            uint8_t* dsimg, cudaStream_t st, float qk_scale, float* bpart, bool* bpart_done) {
+  if (bpart_done) *bpart_done = false;
   const int h = nh * DH;
   const long T = static_cast<long>(B) * s;
   CUtensorMap m128, m64, d64, d128, g128;
@@ -1949,8 +1993,11 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
           cudaFuncSetAttribute(fa_bwd_dkdv_n128<DH>, cudaFuncAttributeMaxDynamicSharedMemorySize, SmemN<DH>::kBytes);
           nset = true;
         }
+        // the qkv-bias column partials come from this kernel (k, v) and fa_bwd_dq_img (q): both or none
+        const bool bp = bpart && dsimg && (!only || only[1] == 'k');
         fa_bwd_dkdv_n128<DH><<<grid, kThreadsB, SmemN<DH>::kBytes, st>>>(m128, d128, g128, lse, Dd, dqkv, B, s, nh,
-                                                                           dsimg, qk_scale);
+                                                                           dsimg, qk_scale, bp ? bpart : nullptr);
+        if (bp && bpart_done) *bpart_done = true;
       } else
       fa_bwd_dkdv_ts<DH><<<grid, kThreadsB, smem_dkdv_ts<DH>(), st>>>(m128, m64, d64, g128, lse, Dd, dqkv, B, s, nh,
                                                                         dsimg, attn_l2hint(), qk_scale,
@@ -1992,7 +2039,7 @@ bool launch(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, 
     static const int per_sm = getenv("MARIO_DQI_CTAS") ? atoi(getenv("MARIO_DQI_CTAS")) : 2;
     const int grid_i = items < per_sm * sms ? items : per_sm * sms;
     fa_bwd_dq_img<DH><<<grid_i, kThreadsI, SmemI<DH>::kBytes, st>>>(m64, dsimg, dqkv, B, s, nh, attn_l2hint(),
-                                                                     qk_scale);
+                                                                     qk_scale, (bpart_done && *bpart_done) ? bpart : nullptr);
   } else if (!only || only[1] == 'q') {
     // 128-key tiles (fa_bwd_dq_n128) where s % 128 == 0: 1835 -> 1601 us for the whole backward at B 1,
     // s 16384, 8 heads; 532 -> 489 us at s 4096 (dQ bitwise equal); MARIO_ATTN_DQ_N128=0: fa_bwd_dq_pers
@@ -2577,11 +2624,13 @@ bool flash_attn_fwd_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int n
 
 // Returns false if the configuration is unsupported (caller falls back to the mma.sync kernels).
 bool flash_attn_bwd_tc(const bf16* qkv, const bf16* dO, const float* lse, const float* Dd, bf16* dqkv, int B, int s,
-                       int nh, int dh, void* ds_ws, size_t ds_ws_bytes, cudaStream_t st, float qk_scale) {
+                       int nh, int dh, void* ds_ws, size_t ds_ws_bytes, cudaStream_t st, float qk_scale, float* bpart,
+                       bool* bpart_done) {
+  if (bpart_done) *bpart_done = false;
   if (qk_scale <= 0.f) qk_scale = rsqrtf(static_cast<float>(dh));
   uint8_t* img = ds_ws && ds_ws_bytes >= flash_attn_bwd_ds_bytes(dh, B, s, nh) ? static_cast<uint8_t*>(ds_ws) : nullptr;
-  if (dh == 128) return launch<128>(qkv, dO, lse, Dd, dqkv, B, s, nh, img, st, qk_scale);
-  if (dh == 64) return launch<64>(qkv, dO, lse, Dd, dqkv, B, s, nh, img, st, qk_scale);
+  if (dh == 128) return launch<128>(qkv, dO, lse, Dd, dqkv, B, s, nh, img, st, qk_scale, bpart, bpart_done);
+  if (dh == 64) return launch<64>(qkv, dO, lse, Dd, dqkv, B, s, nh, img, st, qk_scale, bpart, bpart_done);
   return false;
 }
 

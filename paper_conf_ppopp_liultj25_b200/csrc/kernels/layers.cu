@@ -1573,13 +1573,15 @@ void attn_fwd(const T* qkv, T* O, float* lse, int B, int s, int nh, int dh, cuda
 }
 template <class T>
 void attn_bwd(const T* qkv, const T* O, const T* dO, const float* lse, T* dqkv, float* Dsc, int B, int s, int nh,
-              int dh, cudaStream_t st, void* ds_ws, size_t ds_ws_bytes, void* pad_ws) {
+              int dh, cudaStream_t st, void* ds_ws, size_t ds_ws_bytes, void* pad_ws, float* bpart, bool* bpart_done) {
+  if (bpart_done) *bpart_done = false;
   if constexpr (std::is_same<T, __nv_bfloat16>::value) {
     if (flash_attn_supported(dh)) {
-      flash_attn_bwd(qkv, O, dO, lse, dqkv, Dsc, B, s, nh, dh, st, ds_ws, ds_ws_bytes, pad_ws);
+      flash_attn_bwd(qkv, O, dO, lse, dqkv, Dsc, B, s, nh, dh, st, ds_ws, ds_ws_bytes, pad_ws, bpart, bpart_done);
       return;
     }
   }
+  (void)bpart;
   (void)ds_ws; (void)ds_ws_bytes; (void)pad_ws;
   const int grid = cdiv(static_cast<long>(B) * s * nh, 8);
   attn_bwd_dq_k<T><<<grid, 256, 0, st>>>(qkv, O, dO, lse, dqkv, Dsc, B, s, nh, dh);
@@ -1709,7 +1711,7 @@ void sum_copies_f32(float* dst, const CopySrcs& srcs, size_t n, cudaStream_t st)
                             float*, float*, float*, size_t, cudaStream_t);                                           \
   template void attn_fwd<T>(const T*, T*, float*, int, int, int, int, cudaStream_t, void*);                                 \
   template void attn_bwd<T>(const T*, const T*, const T*, const float*, T*, float*, int, int, int, int, cudaStream_t, \
-                            void*, size_t, void*);                                                                 \
+                            void*, size_t, void*, float*, bool*);                                                  \
   template void rope<T>(T*, int, int, int, int, float, int, cudaStream_t, const float2*);                             \
   template void swiglu_fwd<T>(const T*, T*, int, int, cudaStream_t);                                                 \
   template void swiglu_bwd<T>(const T*, const T*, T*, int, int, cudaStream_t);                                       \

@@ -72,9 +72,11 @@ template <class T> void attn_fwd(const T* qkv, T* O, float* lse, int B, int s, i
 // dqkv [T, 3h] from dO; Dscratch [nh][T] fp32.
 // ds_ws (optional, >= flash_attn_bwd_ds_bytes): workspace for the dS image, which lets the bf16
 // tcgen05 path compute dQ from the stored dS (fa_bwd_dq_img) instead of recomputing S and dP.
+// bpart / bpart_done: see flash_attn_bwd_tc (bf16 only; *bpart_done = false otherwise)
 template <class T> void attn_bwd(const T* qkv, const T* O, const T* dO, const float* lse, T* dqkv, float* Dscratch,
                                  int B, int s, int nh, int dh, cudaStream_t st, void* ds_ws = nullptr,
-                                 size_t ds_ws_bytes = 0, void* pad_ws = nullptr);
+                                 size_t ds_ws_bytes = 0, void* pad_ws = nullptr, float* bpart = nullptr,
+                                 bool* bpart_done = nullptr);
 // bytes of that dS workspace for a shape (0 when the path does not apply)
 size_t flash_attn_bwd_ds_bytes(int dh, int B, int s, int nh);
 
@@ -108,16 +110,20 @@ void flash_attn_fwd(const __nv_bfloat16* qkv, __nv_bfloat16* O, float* lse, int 
 // O == nullptr (head dims 16/32/64/128, no padding): Dd already holds D = rowsum(dO o O) per head
 void flash_attn_bwd(const __nv_bfloat16* qkv, const __nv_bfloat16* O, const __nv_bfloat16* dO, const float* lse,
                     __nv_bfloat16* dqkv, float* Dd, int B, int s, int nh, int dh, cudaStream_t st,
-                    void* ds_ws = nullptr, size_t ds_ws_bytes = 0, void* pad_ws = nullptr);
+                    void* ds_ws = nullptr, size_t ds_ws_bytes = 0, void* pad_ws = nullptr, float* bpart = nullptr,
+                    bool* bpart_done = nullptr);
 // bytes of the padded-head workspace (bwd = 0 forward, 1 backward incl. its dS image); 0: no padding
 size_t flash_attn_pad_bytes(int dh, int B, int s, int nh, int bwd);
 bool flash_attn_bwd_tc_supported(int dh, int B, int s, int nh);
 // qk_scale: the softmax scale of q.k (<= 0: 1/sqrt(dh); the padded path passes 1/sqrt of the true dh)
 bool flash_attn_fwd_tc(const __nv_bfloat16* qkv, __nv_bfloat16* O, float* lse, int B, int s, int nh, int dh,
                        cudaStream_t st, float qk_scale = 0.f);
+// bpart (optional): fp32 [B*s/32][3*nh*dh] column partial sums of the written dQKV per 32-row block (the
+// qkv-bias gradient's), filled only when the dK/dV kernel with the dS image and fa_bwd_dq_img run
+// (*bpart_done = true); otherwise untouched and the caller sums dQKV itself.
 bool flash_attn_bwd_tc(const __nv_bfloat16* qkv, const __nv_bfloat16* dO, const float* lse, const float* Dd,
                        __nv_bfloat16* dqkv, int B, int s, int nh, int dh, void* ds_ws, size_t ds_ws_bytes,
-                       cudaStream_t st, float qk_scale = 0.f);
+                       cudaStream_t st, float qk_scale = 0.f, float* bpart = nullptr, bool* bpart_done = nullptr);
 
 void cast_f32_bf16(const float* x, __nv_bfloat16* y, size_t n, cudaStream_t st);
 void add_f32(float* a, const float* b, size_t n, cudaStream_t st);       // a += b

@@ -113,6 +113,34 @@ def test_lean_activation_set(cfg, dtype, monkeypatch):
         check(lean[0], lean[1], stored[0], {k: v.astype(np.float64) for k, v in stored[1].items()}, 2e-2)
 
 
+def test_fused_qkv_bias_sums_match_column_sum_pass():
+    """GPT at cfg-2 width (s 2048: the dS-image attention backward): the qkv-bias gradient taken from
+    the attention kernels' column partials (dK / dV from the dK/dV kernel's staged tiles, dQ from the
+    dQ kernel's registers) equals the separate column-sum pass over the stored dQKV up to fp32
+    summation order, and every other gradient is bitwise the same."""
+    import subprocess, sys, os, json
+    cfg = synth.with_(synth.GPT3_1P3B, n_layers=2, micro_batch=1)
+    params = synth.make_weights(cfg)
+    toks = synth.make_tokens(cfg, 2)
+    fused = run_plan(cfg, 1, 2, "1f1b", "mario", "bf16", params, toks)
+    # the knob is read once per process: the unfused run goes through a child process
+    code = ("import numpy as np, synth, sys; sys.path.insert(0, 'tests'); from test_gpu_parity import run_plan; "
+            "cfg = synth.with_(synth.GPT3_1P3B, n_layers=2, micro_batch=1); "
+            "r = run_plan(cfg, 1, 2, '1f1b', 'mario', 'bf16', synth.make_weights(cfg), synth.make_tokens(cfg, 2)); "
+            "np.save(sys.argv[1], r[2])")
+    out = os.path.join(os.environ.get("TMPDIR", "/tmp"), "mario_qkvb_unfused.npy")
+    env = dict(os.environ, MARIO_FUSE_QKVB="0")
+    subprocess.run([sys.executable, "-c", code, out], check=True, env=env, cwd=os.path.dirname(os.path.dirname(__file__)))
+    ref = np.load(out)
+    plan = api.Plan(cfg, 1, 2, "1f1b", "mario", dtype="bf16")
+    a, b = api.unpack_params(plan, fused[2], 0), api.unpack_params(plan, ref, 0)
+    for k in a:
+        if k.endswith("qkv.b"):
+            assert np.abs(a[k] - b[k]).max() <= 1e-4 * np.abs(b[k]).max(), k
+        else:
+            assert np.array_equal(a[k], b[k]), k
+
+
 UNTIED_GPT = synth.with_(synth.TINY_GPT, tie_embeddings=False)
 
 

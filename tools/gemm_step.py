@@ -12,6 +12,9 @@ from paper_conf_ppopp_liultj25_b200 import _lib  # noqa: E402
 
 L = _lib.lib()
 import os  # noqa: E402
+# the default stored activation set keeps G = gelu(Z) from the forward, so the fc2 dgrad epilogue has
+# no G output; MARIO_STORE_ACT=0 (lean set) times it with the recomputed G as a second output
+LEAN = os.environ.get("MARIO_STORE_ACT", "1") == "0"
 if os.environ.get("STREAMK"):
     L.mario_k_gemm_set_streamk(int(os.environ["STREAMK"]))
 if os.environ.get("VARIANT"):
@@ -62,7 +65,7 @@ def calls(a, epi=True):
         ("fc2 wgrad", 2 * T * h * f, lambda: gemm(a["dH"], h, 1, a["G"], f, 1, h, f, T, dW["fc2"], f, 1,
                                                   1. if e else 0.)),
         ("fc2 dgrad", 2 * T * h * f, lambda: gemm(a["dH"], h, 0, W["fc2"], f, 1, T, f, h, a["dZ"], f, 0, 0.,
-                                                  d2=a["G"] if e else None, aux=a["Z"] if e else None)),
+                                                  d2=a["G"] if (e and LEAN) else None, aux=a["Z"] if e else None)),
         ("fc1 wgrad", 2 * T * h * f, lambda: gemm(a["dZ"], f, 1, a["A2"], h, 1, f, h, T, dW["fc1"], h, 1,
                                                   1. if e else 0.)),
         ("fc1 dgrad", 2 * T * h * f, lambda: gemm(a["dZ"], f, 0, W["fc1"], h, 1, T, h, f, a["dA"], h, 0, 0.)),
