@@ -1688,22 +1688,32 @@ fa_bwd_dkdv_n128(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_con
     }
     if (bpart) {
       // column sums of the staged bf16 dV / dK tiles (exactly what is stored), per 32-row block in
-      // row order: bpart[(token / 32)][3h] gets the qkv-bias gradient partials of the k and v columns
-      // (read alongside the TMA store: both only read the staging tiles)
-      const int t = threadIdx.x - 64;
-      if (t < 2 * DH) {
-        const bool isK = t >= DH;
-        const int c = isK ? t - DH : t, ch = (c % 64) / 8, e = c % 8;
-        const uint8_t* tile = isK ? stK(c / 64) : stV(c / 64);
-        float* dst = bpart + ((static_cast<long>(b) * s + kt * kRows) / 32) * (3 * h) + (isK ? h : 2 * h) + head * DH + c;
-#pragma unroll 1
-        for (int q = 0; q < kRows / 32; ++q) {
-          float acc = 0.f;
-#pragma unroll 8
-          for (int r = 32 * q; r < 32 * q + 32; ++r)
-            acc += __bfloat162float(*reinterpret_cast<const bf16*>(tile + r * 128 + ((ch ^ (r & 7)) << 4) + e * 2));
-          dst[static_cast<long>(q) * (3 * h)] = acc;
+      // row order: bpart[(token / 32)][3h] gets the qkv-bias gradient partials of the k and v columns.
+      // Thread t: 16-byte chunk column j = t % 32 (8 columns of dV, then dK) over the 32 rows of row
+      // block t / 32 -- a warp reads whole 128-byte swizzled rows (4 wavefronts per instruction).
+      // Read alongside the TMA store: both only read the staging tiles.
+      const int t = threadIdx.x - 64, j = t % 32, q = t / 32;
+      constexpr int kChunks = 2 * DH / 8;
+      if (j < kChunks && q < kRows / 32) {
+        const bool isK = j >= DH / 8;
+        const int cc = isK ? j - DH / 8 : j;            // chunk within the tile's row (8 columns)
+        const uint8_t* tile = isK ? stK(cc / 8) : stV(cc / 8);
+        float acc[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+#pragma unroll 4
+        for (int r = 32 * q; r < 32 * q + 32; ++r) {
+          const uint4 u = *reinterpret_cast<const uint4*>(tile + r * 128 + (((cc % 8) ^ (r & 7)) << 4));
+          const __nv_bfloat162* hh = reinterpret_cast<const __nv_bfloat162*>(&u);
+#pragma unroll
+          for (int e = 0; e < 4; ++e) {
+            const float2 f = __bfloat1622float2(hh[e]);
+            acc[2 * e] += f.x;
+            acc[2 * e + 1] += f.y;
+          }
         }
+        float* dst = bpart + ((static_cast<long>(b) * s + kt * kRows) / 32 + q) * (3 * h) + (isK ? h : 2 * h) +
+                     head * DH + cc * 8;
+        *reinterpret_cast<float4*>(dst) = make_float4(acc[0], acc[1], acc[2], acc[3]);
+        *reinterpret_cast<float4*>(dst + 4) = make_float4(acc[4], acc[5], acc[6], acc[7]);
       }
     }
   }

@@ -113,22 +113,29 @@ def test_lean_activation_set(cfg, dtype, monkeypatch):
         check(lean[0], lean[1], stored[0], {k: v.astype(np.float64) for k, v in stored[1].items()}, 2e-2)
 
 
-def test_fused_qkv_bias_sums_match_column_sum_pass():
-    """GPT at cfg-2 width (s 2048: the dS-image attention backward): the qkv-bias gradient taken from
-    the attention kernels' column partials (dK / dV from the dK/dV kernel's staged tiles, dQ from the
-    dQ kernel's registers) equals the separate column-sum pass over the stored dQKV up to fp32
-    summation order, and every other gradient is bitwise the same."""
-    import subprocess, sys, os, json
-    cfg = synth.with_(synth.GPT3_1P3B, n_layers=2, micro_batch=1)
+QKVB_CASES = {"gpt-1.3b-width": "synth.with_(synth.GPT3_1P3B, n_layers=2, micro_batch=1)",
+              "dh64-s256-mbs2": "synth.with_(synth.GPT3_1P3B, n_layers=2, hidden=1024, n_heads=16, ffn_hidden=4096, "
+                                "seq_len=256, micro_batch=2)"}
+
+
+@pytest.mark.parametrize("case", sorted(QKVB_CASES))
+def test_fused_qkv_bias_sums_match_column_sum_pass(case):
+    """GPT with s % 128 == 0 (the dS-image attention backward; dh 128 and dh 64, one and two samples
+    per micro-batch): the qkv-bias gradient taken from the attention kernels' column partials (dK / dV
+    from the dK/dV kernel's staged tiles, dQ from the dQ kernel's registers) equals the separate
+    column-sum pass over the stored dQKV up to fp32 summation order, and every other gradient is
+    bitwise the same (the fused attention D is on in both runs)."""
+    import subprocess, sys, os
+    cfg = eval(QKVB_CASES[case])
     params = synth.make_weights(cfg)
     toks = synth.make_tokens(cfg, 2)
     fused = run_plan(cfg, 1, 2, "1f1b", "mario", "bf16", params, toks)
     # the knob is read once per process: the unfused run goes through a child process
     code = ("import numpy as np, synth, sys; sys.path.insert(0, 'tests'); from test_gpu_parity import run_plan; "
-            "cfg = synth.with_(synth.GPT3_1P3B, n_layers=2, micro_batch=1); "
+            f"cfg = {QKVB_CASES[case]}; "
             "r = run_plan(cfg, 1, 2, '1f1b', 'mario', 'bf16', synth.make_weights(cfg), synth.make_tokens(cfg, 2)); "
             "np.save(sys.argv[1], r[2])")
-    out = os.path.join(os.environ.get("TMPDIR", "/tmp"), "mario_qkvb_unfused.npy")
+    out = os.path.join(os.environ.get("TMPDIR", "/tmp"), f"mario_qkvb_unfused_{case}.npy")
     env = dict(os.environ, MARIO_FUSE_QKVB="0")
     subprocess.run([sys.executable, "-c", code, out], check=True, env=env, cwd=os.path.dirname(os.path.dirname(__file__)))
     ref = np.load(out)
