@@ -2316,7 +2316,10 @@ fa_fwd_tc(const __grid_constant__ CUtensorMap tm_qkv128, const __grid_constant__
 constexpr int kF2Q = 128;        // rows per Q tile
 constexpr int kF2N = 128;        // keys per tile
 constexpr int kF2Threads = 384;
-constexpr int kF2Stages = 3;
+#ifndef MARIO_F2_STAGES
+#define MARIO_F2_STAGES 3   // K/V ring depth of the two-Q-tile forward (A/B: NVCC_EXTRA=-DMARIO_F2_STAGES=n)
+#endif
+constexpr int kF2Stages = MARIO_F2_STAGES;
 #ifndef MARIO_POLY_EX2
 #define MARIO_POLY_EX2 1
 #endif
