@@ -2320,6 +2320,9 @@ constexpr int kF2Threads = 384;
 #define MARIO_F2_STAGES 3   // K/V ring depth of the two-Q-tile forward (A/B: NVCC_EXTRA=-DMARIO_F2_STAGES=n)
 #endif
 constexpr int kF2Stages = MARIO_F2_STAGES;
+#ifndef MARIO_F2_DBG
+#define MARIO_F2_DBG 0   // 1: softmax exponentials replaced by an FMA (timing experiment only, wrong results)
+#endif
 #ifndef MARIO_POLY_EX2
 #define MARIO_POLY_EX2 1
 #endif
@@ -2528,7 +2531,11 @@ fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, i
 #pragma unroll
       for (int c = 0; c < kF2N; ++c) {
         const float arg = fmaf(x[c], sl2, -m_used);
+#if MARIO_F2_DBG   // experiment: exponentials replaced by an FMA (wrong results) to time the softmax share
+        x[c] = arg * 0.0009765625f + 1.f;
+#else
         x[c] = (kPolyEx2 && (c & 3) == 3) ? ex2_poly(arg) : ex2(arg);
+#endif
         ls += x[c];
       }
       l += ls;
