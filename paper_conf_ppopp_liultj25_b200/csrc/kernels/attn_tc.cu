@@ -2346,8 +2346,16 @@ __device__ __forceinline__ void f2_item(int i, int n, bool& is_v, int& j) {
 template <int DH>
 __global__ void __launch_bounds__(kF2Threads, 1)
 fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, int B, int s, int nh, int g_l2hint,
-           float qk_scale) {
+           float qk_scale, long long* trace) {
   using SM = SmemF2<DH>;
+  // trace (MARIO_ATTN_FWD_TRACE): per CTA (sm, start, end) globaltimer ns, for tools/attn_fwd_trace.py
+  if (trace && threadIdx.x == 0) {
+    uint64_t gt; uint32_t smid;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt));
+    asm volatile("mov.u32 %0, %%smid;" : "=r"(smid));
+    trace[3 * blockIdx.x] = smid;
+    trace[3 * blockIdx.x + 1] = static_cast<long long>(gt);
+  }
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
   uint8_t* sQ = smem;                                   // [2][kTile]
@@ -2576,6 +2584,11 @@ fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, i
   tc_fence_before();
   __syncthreads();
   if (warp == 1) tmem_dealloc<512>(tm);
+  if (trace && threadIdx.x == 0) {
+    uint64_t gt;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(gt));
+    trace[3 * blockIdx.x + 2] = static_cast<long long>(gt);
+  }
 }
 
 template <int DH>
@@ -2591,7 +2604,21 @@ bool launch_fwd2_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, 
     set = true;
   }
   const int nqb = (s + 2 * kF2Q - 1) / (2 * kF2Q);
-  fa_fwd2_tc<DH><<<nqb * B * nh, kF2Threads, smem, st>>>(m128, O, lse, B, s, nh, attn_l2hint(), qk_scale);
+  const int grid = nqb * B * nh;
+  static const char* tfile = getenv("MARIO_ATTN_FWD_TRACE");
+  static long long* trace = nullptr;
+  if (tfile && !trace) cudaMalloc(&trace, 3 * 65536 * sizeof(long long));
+  fa_fwd2_tc<DH><<<grid, kF2Threads, smem, st>>>(m128, O, lse, B, s, nh, attn_l2hint(), qk_scale,
+                                                 (tfile && grid <= 65536) ? trace : nullptr);
+  if (tfile && grid <= 65536) {
+    std::vector<long long> c(3 * grid);
+    cudaStreamSynchronize(st);
+    cudaMemcpy(c.data(), trace, c.size() * sizeof(long long), cudaMemcpyDeviceToHost);
+    if (FILE* f = fopen(tfile, "w")) {
+      for (int j = 0; j < grid; ++j) fprintf(f, "%d %lld %lld %lld\n", j, c[3 * j], c[3 * j + 1], c[3 * j + 2]);
+      fclose(f);
+    }
+  }
   note_launch();
   return true;
 }
