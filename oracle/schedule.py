@@ -7,7 +7,7 @@ Written step by step in the paper's order and notation, independent of the C++ p
   (op, micro_id m, part_id p). Ops: FW, CFW, RC, BW, SA, RA, SG, RG.
 - Base schemes: 1F1B "V" (Megatron order), Interleave "W" (Megatron
   interleaved order, reading A9), Chimera "X" (bidirectional, reading A10 — the order is
-  defined outside PAPER.md: parity unpinned beyond Table 1 bounds and invariants).
+  defined outside PAPER.md; pinned by Chimera's basic-unit bubble count D - 2 at F = B).
 - Passes (§5.1): pass 1 apply-checkpoint, pass 2 overlap-recompute,
   pass 3 remove-redundancy (P:218), pass 4 prepose-forward with the SA rule (P:220-222);
   applied iteratively. Readings A14-A17 fix the details the paper leaves open.
@@ -174,8 +174,10 @@ def build_chimera(pipe: Pipe, F: float = 1.0, B: float = 2.0) -> List[List[Instr
     """Chimera (reading A10): one basic unit of D micro-batches (first D/2 on the down
     pipeline p=0, last D/2 on the up pipeline p=1) is ordered by a greedy list schedule
     at unit costs F=1, B=2: whenever a worker is idle it runs the ready instruction with
-    priority BW before FW, then lower vstage for BW... ties by micro id. Units are
-    concatenated for N > D. PARITY UNPINNED beyond Table 1 bounds and invariants."""
+    priority BW before FW, then the deeper virtual stage (higher k) first, ties by micro id.
+    Units are concatenated for N > D. Pinned against Chimera's own closed form ([23], cited at
+    P:61 / Table 1): built and simulated at F = B the basic unit takes 2N + D - 2 (D - 2
+    bubbles per worker) for N = D (tests/test_schedule_oracle.py::test_chimera_unit_closed_form)."""
     D, N = pipe.S, pipe.N
     unit = Pipe(X_CHIMERA, D, D)
     # tasks per worker
@@ -205,11 +207,12 @@ def build_chimera(pipe: Pipe, F: float = 1.0, B: float = 2.0) -> List[List[Instr
                         continue
                 if dep is not None and (dep not in fin or fin[dep] > t + 1e-12):
                     continue
-                ready.append((0 if op == BW else 1, m, k, op))
+                ready.append((0 if op == BW else 1, -k, m, op))
             if not ready:
                 continue
             ready.sort()
-            _, m, k, op = ready[0]
+            _, nk, m, op = ready[0]
+            k = -nk
             remaining.discard((op, m, k))
             dur = F if op == FW else B
             fin[(op, m, k)] = t + dur

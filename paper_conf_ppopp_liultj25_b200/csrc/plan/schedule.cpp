@@ -93,7 +93,8 @@ Lists build_interleave(const Pipe& pp) {
   return out;
 }
 
-// Chimera basic unit by greedy list scheduling at F=1, B=2 (reading A10; parity unpinned).
+// Chimera basic unit by greedy list scheduling at F=1, B=2 (reading A10): BW first, then the deeper
+// virtual stage, then the micro-batch; identical to oracle/schedule.py::build_chimera.
 Lists build_chimera(const Pipe& pp) {
   const int D = pp.S;
   Pipe unit{MARIO_CHIMERA, D, D, 1};
@@ -115,7 +116,7 @@ Lists build_chimera(const Pipe& pp) {
     bool progressed = false;
     for (int d = 0; d < D; ++d) {
       if (busy_until[d] > t + EPS) continue;
-      // ready tuples sorted by (BW first, m, k)
+      // ready tuples sorted by (BW first, deeper stage first, m)
       std::vector<std::tuple<int, int, int, int>> ready;
       for (const Key& key : remaining) {
         int op = std::get<0>(key), m = std::get<1>(key), k = std::get<2>(key);
@@ -127,11 +128,11 @@ Lists build_chimera(const Pipe& pp) {
           Key dep = (k == D - 1) ? Key{FW, m, k} : Key{BW, m, k + 1};
           if (!done_by(dep, t)) continue;
         }
-        ready.push_back({op == BW ? 0 : 1, m, k, op});
+        ready.push_back({op == BW ? 0 : 1, -k, m, op});
       }
       if (ready.empty()) continue;
       std::sort(ready.begin(), ready.end());
-      int m = std::get<1>(ready[0]), k = std::get<2>(ready[0]), op = std::get<3>(ready[0]);
+      int k = -std::get<1>(ready[0]), m = std::get<2>(ready[0]), op = std::get<3>(ready[0]);
       remaining.erase({op, m, k});
       double dur = op == FW ? F : B;
       fin[{op, m, k}] = t + dur;

@@ -11,6 +11,8 @@ from oracle.schedule import (BASE, CKPT, MARIO, MARIO_BUDGET, BW, CFW, FW, RA, R
                              pass2_overlap_recompute, pass3_remove_redundancy,
                              pass4_prepose_forward, pass5_budget, simulate, transform)
 
+from oracle import schedule as S
+
 GOLD = os.path.join(os.path.dirname(__file__), "golden")
 
 
@@ -192,13 +194,14 @@ def test_budget_tail_survey_sequence():
 
 def test_budget_tail_picks_fastest_not_largest():
     """Chimera S = 4, N = 8: un-checkpointing only the last device lengthens the schedule
-    (44 > 42), so with room for it the rule still keeps k = 0 (smallest makespan, ties to k)."""
+    (38 > 36), so with room for it the rule still keeps k = 0 (smallest makespan, ties to k);
+    with room for three un-checkpointed tails it reaches the base makespan (32)."""
     pipe, c, mem = Pipe(X_CHIMERA, 4, 8), UnitCosts(), MemUnits()
     L0 = transform(pipe, MARIO, c)
     L, k = pass5_budget(pipe, c, mem, 3)
     assert k == 0 and L == L0
     L, k = pass5_budget(pipe, c, mem, 4)
-    assert k in (3, 4) and simulate(pipe, L, c).makespan == 38
+    assert k in (3, 4) and simulate(pipe, L, c).makespan == simulate(pipe, build_base(pipe), c).makespan == 32
 
 
 def test_budget_level_keeps_invariants_all_schemes():
@@ -210,3 +213,18 @@ def test_budget_level_keeps_invariants_all_schemes():
             assert simulate(pipe, L, c) is not None
             # never slower than the paper's passes when those fit
             assert simulate(pipe, L, c).makespan <= simulate(pipe, transform(pipe, MARIO, c, mem, b), c).makespan
+
+
+@pytest.mark.parametrize("D", [4, 6, 8, 16])
+def test_chimera_unit_closed_form(D):
+    """Chimera's own bubble count ([23], the scheme PAPER.md P:61 cites): one basic unit of N = D
+    micro-batches on D workers, forward and backward of equal cost, finishes in 2N + D - 2 slots
+    (each worker is busy 2N and idles D - 2), against 2N + 2(D - 1) for 1F1B. Built and simulated at
+    F = B = 1 (the production order is the same greedy at F = 1, B = 2)."""
+    pipe = S.Pipe(S.X_CHIMERA, D, D)
+    lists = S.build_chimera(pipe, F=1.0, B=1.0)
+    S.check_structure(pipe, lists)
+    r = S.simulate(pipe, lists, S.UnitCosts(F=1.0, B=1.0))
+    assert r.makespan == 2 * D + D - 2
+    one = S.simulate(S.Pipe(S.V_1F1B, D, D), S.build_1f1b(S.Pipe(S.V_1F1B, D, D)), S.UnitCosts(F=1.0, B=1.0))
+    assert one.makespan == 2 * D + 2 * (D - 1)
