@@ -146,9 +146,9 @@ int32_t mario_param_count(const struct mario_plan* plan);
 mario_status mario_param_shape(const struct mario_plan* plan, int32_t idx, int64_t* dims, int32_t* ndim);
 /* k of MARIO_LEVEL_BUDGET (0 for the other levels); -1 on NULL. */
 int32_t mario_plan_unckpt_tail(const struct mario_plan* plan);
-/* 1 if the plan's activation sets keep the layers' norm outputs (the backward reads them instead
- * of recomputing them; chosen unless it would exceed mem_budget_bytes, where the lean set is
- * planned instead; env MARIO_STORE_ACT=0/1 forces either), 0 for the lean set, -1 on NULL. */
+/* 1 if the plan's activation sets keep the layers' norm outputs and MLP activation (the backward
+ * reads them instead of recomputing them; chosen unless it would exceed mem_budget_bytes, where the
+ * lean set is planned instead; env MARIO_STORE_ACT=0/1 forces either), 0 for the lean set, -1 on NULL. */
 int32_t mario_plan_store_act(const struct mario_plan* plan);
 void mario_plan_destroy(struct mario_plan* plan);
 

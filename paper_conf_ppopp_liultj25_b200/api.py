@@ -190,7 +190,8 @@ class Plan:
 
     @property
     def store_act(self) -> bool:
-        """Activation sets keep the norm outputs (else the lean set: the backward recomputes them)."""
+        """Activation sets keep the norm outputs and the MLP activation (else the lean set: the backward
+        recomputes them)."""
         return bool(_lib.lib().mario_plan_store_act(self.handle))
 
     def lists(self) -> List[List[Tuple[str, int, int]]]:
