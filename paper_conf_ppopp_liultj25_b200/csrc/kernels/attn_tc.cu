@@ -2320,6 +2320,12 @@ constexpr int kF2Threads = 384;
 #define MARIO_F2_STAGES 3   // K/V ring depth of the two-Q-tile forward (A/B: NVCC_EXTRA=-DMARIO_F2_STAGES=n)
 #endif
 constexpr int kF2Stages = MARIO_F2_STAGES;
+// per-thread register split after setmaxnreg: TMA / MMA warps vs the two softmax warpgroups
+// (4 x 32 x CTRL + 8 x 32 x SMAX <= 65536)
+#ifndef MARIO_F2_CTRL_REGS
+#define MARIO_F2_CTRL_REGS "88"
+#define MARIO_F2_SMAX_REGS "208"
+#endif
 #ifndef MARIO_F2_DBG
 #define MARIO_F2_DBG 0   // 1: softmax exponentials replaced by an FMA (timing experiment only, wrong results)
 #endif
@@ -2369,17 +2375,22 @@ fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, i
   uint64_t* s_free = s_full + 2;                   // 2
   uint64_t* p_full = s_free + 2;                   // 2
   uint64_t* o_done = p_full + 2;                   // 2
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(o_done + 2);
+  uint64_t* q_empty = o_done + 2;                  // 1  (persistent: the item's S MMAs are done with Q)
+  uint64_t* o_free = q_empty + 1;                  // 2  (persistent: the epilogue has read O_t)
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(o_free + 2);
 
   const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
   const int BH = B * nh, nqb = (s + 2 * kF2Q - 1) / (2 * kF2Q);
-  const int qb = nqb - 1 - static_cast<int>(blockIdx.x) / BH;   // heaviest query blocks first
-  const int bh = static_cast<int>(blockIdx.x) % BH, b = bh / nh, head = bh % nh;
   const int h = nh * DH;
   const long Ttok = static_cast<long>(B) * s;
-  const int q0 = qb * 2 * kF2Q;
-  const int n0 = 2 * qb + 1, n1 = 2 * qb + 2;      // key tiles seen by Q tile 0 / 1
   const float sl2 = qk_scale * LOG2E;
+  // work items w = (query block, sample, head), heaviest query blocks first; a grid smaller than the
+  // item count runs persistently, CTA c taking items in snake order (round r: r*G + c, or
+  // r*G + G-1-c on odd rounds), which balances the causal item weights like dynamic dispatch. Item
+  // n+1's Q load, K/V loads and S MMAs overlap item n's last PV and epilogue; barrier phases run on
+  // across items (per-tile step bases). One CTA per item runs the same code for one round.
+  const int W = nqb * BH, G = gridDim.x, cta = blockIdx.x;
+  auto item_of = [=](int r) { const int w = r * G + ((r & 1) ? G - 1 - cta : cta); return w < W ? w : -1; };
 
   if (warp == 0 && lane == 0) {
     tma_prefetch_desc(&tm_qkv128);
@@ -2387,7 +2398,9 @@ fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, i
     for (int i = 0; i < kF2Stages; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 1); }
     for (int t = 0; t < 2; ++t) {
       mbar_init(&s_full[t], 1); mbar_init(&s_free[t], 4); mbar_init(&p_full[t], 4); mbar_init(&o_done[t], 1);
+      mbar_init(&o_free[t], 4);
     }
+    mbar_init(q_empty, 1);
     fence_barrier_init();
   }
   if (warp == 1) tmem_alloc<512>(tmem_slot);
@@ -2398,44 +2411,57 @@ fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, i
   const uint32_t tm_S0 = tm, tm_O0 = tm + 2 * kF2N;
 
   if (warp < 4) {
-    asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");
+    asm volatile("setmaxnreg.dec.sync.aligned.u32 " MARIO_F2_CTRL_REGS ";");
   if (warp == 0) {
     if (elect_one()) {
       const uint64_t pf_ = g_l2hint ? pol_first() : pol_normal(), pl_ = g_l2hint ? pol_last() : pol_normal();
-      const int row0 = b * s;
-      mbar_arrive_expect_tx(q_full, 2 * SM::kTile);
+      int gi = 0;   // ring items across work items
+      for (int n = 0;; ++n) {
+        const int w = item_of(n);
+        if (w < 0) break;
+        const int qb = nqb - 1 - w / BH, bh = w % BH, b = bh / nh, head = bh % nh;
+        const int q0 = qb * 2 * kF2Q, n1 = 2 * qb + 2, row0 = b * s;
+        if (n > 0) mbar_wait(q_empty, (n - 1) & 1);   // the previous item's S MMAs have read Q
+        mbar_arrive_expect_tx(q_full, 2 * SM::kTile);
 #pragma unroll
-      for (int t = 0; t < 2; ++t)
+        for (int t = 0; t < 2; ++t)
 #pragma unroll
-        for (int a = 0; a < DH / 64; ++a)
-          tma_load_2d_h(sQ + t * SM::kTile + a * (kF2Q * 128), &tm_qkv128, q_full, head * DH + a * 64,
-                        row0 + q0 + t * kF2Q, pf_);
-      for (int i = 0; i < 2 * n1; ++i) {
-        bool is_v;
-        int j;
-        f2_item(i, n1, is_v, j);
-        const int st = i % kF2Stages;
-        mbar_wait(&empty[st], ((i / kF2Stages) & 1) ^ 1);
-        mbar_arrive_expect_tx(&full[st], SM::kTile);
-        uint8_t* dst = sRing + st * SM::kTile;
+          for (int a = 0; a < DH / 64; ++a)
+            tma_load_2d_h(sQ + t * SM::kTile + a * (kF2Q * 128), &tm_qkv128, q_full, head * DH + a * 64,
+                          row0 + q0 + t * kF2Q, pf_);
+        for (int i = 0; i < 2 * n1; ++i, ++gi) {
+          bool is_v;
+          int j;
+          f2_item(i, n1, is_v, j);
+          const int st = gi % kF2Stages;
+          mbar_wait(&empty[st], ((gi / kF2Stages) & 1) ^ 1);
+          mbar_arrive_expect_tx(&full[st], SM::kTile);
+          uint8_t* dst = sRing + st * SM::kTile;
 #pragma unroll
-        for (int a = 0; a < DH / 64; ++a)
-          tma_load_2d_h(dst + a * (kF2N * 128), &tm_qkv128, &full[st], (is_v ? 2 * h : h) + head * DH + a * 64,
-                        row0 + j * kF2N, pl_);
+          for (int a = 0; a < DH / 64; ++a)
+            tma_load_2d_h(dst + a * (kF2N * 128), &tm_qkv128, &full[st], (is_v ? 2 * h : h) + head * DH + a * 64,
+                          row0 + j * kF2N, pl_);
+        }
       }
     }
   } else if (warp == 1) {
     constexpr uint32_t id_s = umma_idesc_bf16(kF2Q, kF2N, 0, 0);
     constexpr uint32_t id_o = umma_idesc_bf16(kF2Q, DH, 0, 1);   // B = V read MN-major
-    mbar_wait(q_full, 0);
+    int item = 0;                 // ring items across work items
+    int base0 = 0, base1 = 0;     // per-tile S / PV count of the previous work items (barrier phases)
+    for (int n = 0;; ++n) {
+    const int w = item_of(n);
+    if (w < 0) break;
+    const int qb = nqb - 1 - w / BH;
+    const int n0 = 2 * qb + 1, n1 = 2 * qb + 2;
+    mbar_wait(q_full, n & 1);
     tc_fence_after();
-    int item = 0;
     auto issue_s = [&](int j) {
       const int st = item % kF2Stages;
       mbar_wait(&full[st], (item / kF2Stages) & 1);
       for (int t = 0; t < 2; ++t) {
         if (t == 0 && j >= n0) continue;
-        mbar_wait(&s_free[t], (j & 1) ^ 1);
+        mbar_wait(&s_free[t], (((t ? base1 : base0) + j) & 1) ^ 1);
         tc_fence_after();
         if (elect_one()) {
           const uint32_t q = smem_u32(sQ + t * SM::kTile), k = smem_u32(sRing + st * SM::kTile);
@@ -2458,7 +2484,8 @@ fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, i
       mbar_wait(&full[st], (item / kF2Stages) & 1);
       for (int t = 0; t < 2; ++t) {
         if (t == 0 && j >= n0) continue;
-        mbar_wait(&p_full[t], j & 1);
+        if (j == 0 && n > 0) mbar_wait(&o_free[t], (n - 1) & 1);   // the previous item's O_t read out
+        mbar_wait(&p_full[t], ((t ? base1 : base0) + j) & 1);
         tc_fence_after();
         if (elect_one()) {
           const uint32_t p = smem_u32(sP + t * SM::kP), v = smem_u32(sRing + st * SM::kTile);
@@ -2479,21 +2506,33 @@ fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, i
     issue_s(0);
     for (int j = 0; j < n1; ++j) {
       if (j + 1 < n1) issue_s(j + 1);
+      if (j + 1 == n1 - 1 || (j == 0 && n1 == 1)) {   // every S MMA of the item issued: Q free when done
+        if (elect_one()) umma_commit(q_empty);
+        __syncwarp();
+      }
       issue_pv(j);
+    }
+    base0 += n0;
+    base1 += n1;
     }
   }
   } else {
-    asm volatile("setmaxnreg.inc.sync.aligned.u32 224;");
+    asm volatile("setmaxnreg.inc.sync.aligned.u32 " MARIO_F2_SMAX_REGS ";");
     const int t = (warp - 4) >> 2, quarter = warp & 3;
     const int row = quarter * 32 + lane;
-    const int q = q0 + t * kF2Q + row;
-    const int nt = t == 0 ? n0 : n1;
     const uint32_t lane_off = static_cast<uint32_t>(quarter * 32) << 16;
     const uint32_t tS = tm_S0 + t * kF2N + lane_off, tO = tm_O0 + t * DH + lane_off;
     uint8_t* myP = sP + t * SM::kP;
+    int bs = 0;   // this tile's S / PV count of the previous work items
+    for (int n = 0;; ++n) {
+    const int w = item_of(n);
+    if (w < 0) break;
+    const int qb = nqb - 1 - w / BH;
+    const int q = qb * 2 * kF2Q + t * kF2Q + row;
+    const int nt = t == 0 ? 2 * qb + 1 : 2 * qb + 2;
     float m_used = -INFINITY, l = 0.f;
     for (int j = 0; j < nt; ++j) {
-      mbar_wait(&s_full[t], j & 1);
+      mbar_wait(&s_full[t], (bs + j) & 1);
       tc_fence_after();
       uint32_t xr[kF2N];
 #pragma unroll
@@ -2517,7 +2556,7 @@ fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, i
         m_used = m_cand;                          // finite: key 0 <= q
       } else if (__any_sync(0xffffffffu, m_cand > m_used + 8.f)) {
         // raise the running max: O_t (after PV_t(j-1)) and l rescaled by 2^(m_old - m_new)
-        mbar_wait(&o_done[t], (j - 1) & 1);
+        mbar_wait(&o_done[t], (bs + j - 1) & 1);
         tc_fence_after();
         waited = true;
         const float m_new = fmaxf(m_used, m_cand);
@@ -2548,7 +2587,7 @@ fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, i
       }
       l += ls;
       if (j > 0 && !waited) {                     // P_t smem is free once PV_t(j-1) completed
-        mbar_wait(&o_done[t], (j - 1) & 1);
+        mbar_wait(&o_done[t], (bs + j - 1) & 1);
       }
 #pragma unroll
       for (int c0 = 0; c0 < kF2N; c0 += 32)
@@ -2558,15 +2597,21 @@ fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, i
       __syncwarp();
       if (lane == 0) mbar_arrive(&p_full[t]);
     }
-    mbar_wait(&o_done[t], (nt - 1) & 1);
+    mbar_wait(&o_done[t], (bs + nt - 1) & 1);
     tc_fence_after();
     const float inv = 1.f / l;
+    const int bh = w % BH, b = bh / nh, head = bh % nh;
     bf16* orow = O + (static_cast<long>(b) * s + (q < s ? q : 0)) * h + head * DH;
 #pragma unroll 1
     for (int c0 = 0; c0 < DH; c0 += 32) {
       uint32_t r[32];
       tmem_ld_32x32b_x32(tO + c0, r);
       tmem_ld_wait();
+      if (c0 + 32 == DH) {   // every column of O_t in registers: the next item's PV_t may overwrite it
+        tc_fence_before();
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&o_free[t]);
+      }
       if (q < s) {
 #pragma unroll
         for (int d = 0; d < 32; d += 8) {
@@ -2580,6 +2625,8 @@ fa_fwd2_tc(const __grid_constant__ CUtensorMap tm_qkv128, bf16* O, float* lse, i
       }
     }
     if (q < s) lse[static_cast<long>(head) * Ttok + static_cast<long>(b) * s + q] = (m_used + log2f(l)) / LOG2E;
+    bs += nt;
+    }
   }
   tc_fence_before();
   __syncthreads();
@@ -2604,7 +2651,14 @@ bool launch_fwd2_tc(const bf16* qkv, bf16* O, float* lse, int B, int s, int nh, 
     set = true;
   }
   const int nqb = (s + 2 * kF2Q - 1) / (2 * kF2Q);
-  const int grid = nqb * B * nh;
+  const int items = nqb * B * nh;
+  // persistent (default; MARIO_ATTN_FWD_PERS=0: one CTA per item): one CTA per SM the launching thread
+  // may use (its green-context partition in the emulated pipeline). The item -> CTA map does not change
+  // any item's arithmetic: O and lse are bitwise those of the one-CTA-per-item launch. Measured 85.5 ->
+  // 81.1 us at the cfg-2 shape (profiles/r02/attn_fwd_pers_ab.jsonl).
+  static const int pers = getenv("MARIO_ATTN_FWD_PERS") ? atoi(getenv("MARIO_ATTN_FWD_PERS")) : 1;
+  const int sms = device_sm_count();
+  const int grid = (pers && items > sms) ? sms : items;
   static const char* tfile = getenv("MARIO_ATTN_FWD_TRACE");
   static long long* trace = nullptr;
   if (tfile && !trace) cudaMalloc(&trace, 3 * 65536 * sizeof(long long));
